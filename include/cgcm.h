@@ -1,0 +1,170 @@
+/*
+ * cgcm.h -- C ABI of the B200-native CGCM run-time library (libcgcm.so, sm_100a).
+ *
+ * Re-creates the data-parallel hot path of the run-time library of Jablin et al., "Automatic
+ * CPU-GPU Communication Management and Optimization", PLDI 2011 (CGCM): batched map/unmap of
+ * allocation units (AUs) with CPU<->GPU pointer translation.  "P:Lnnn" cites line nnn of the
+ * decoded fulltext of the paper; "Annn" cites a reading of DESIGN.md §3.
+ *
+ * Conventions (all entry points):
+ *   - return int status: CGCM_OK (0) or a negative CGCM_E_* code; out-params are written only on
+ *     success; every call is ALL-OR-NOTHING: on error no refcount, epoch, table entry, host byte or
+ *     device byte changes (the GPU applies optimistically and rolls back).
+ *   - pointers are plain 64-bit addresses.  "host" = CPU virtual address the caller owns;
+ *     "device" = CUDA device address (UVA).  No torch types cross this boundary.
+ *   - calls act on the calling thread's current context (one per device, cgcm_init makes it current).
+ *   - lookups, translations, refcounts and epoch decisions all run in CUDA kernels on the context's
+ *     device; the host side only registers AUs, allocates device storage and issues the copies.
+ *   - If a batch contains several invalid elements, the status is one of their error codes (A24).
+ */
+#ifndef CGCM_H
+#define CGCM_H
+#include <stddef.h>
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- status codes (the same numeric contract as the CPU oracle) ------------ */
+enum {
+  CGCM_OK = 0,
+  CGCM_E_INVALID = -1,      /* bad argument, size 0, NULL where a pointer is required, overflow     */
+  CGCM_E_UNREGISTERED = -2, /* greatestLTE miss: below the first AU, in a gap, past the end (A7)    */
+  CGCM_E_OVERLAP = -3,      /* declared range overlaps a registered AU                              */
+  CGCM_E_NOT_MAPPED = -4,   /* unmap/release at refCount 0, release underflow (A13)                 */
+  CGCM_E_BUSY = -5,         /* undeclare while mapped                                               */
+  CGCM_E_DUPLICATE = -6,    /* declareGlobal name reused                                            */
+  CGCM_E_NOMEM = -7,        /* device arena / pinned host arena exhausted                           */
+  CGCM_E_CUDA = -8,         /* a CUDA runtime call failed: cgcm_lastCudaError() has the detail      */
+  CGCM_E_MIXED = -9,        /* reserved                                                             */
+  CGCM_E_NOCTX = -10        /* no current context on this thread                                    */
+};
+
+/* ---- cgcm_init flags ----------------------------------------------------------------------- */
+enum {
+  CGCM_LITERAL_EPOCH = 1u, /* A5 literal reading: map never sets the AU epoch (default: R1, set at
+                              activation so map->unmap with no launch copies nothing)             */
+  CGCM_LENIENT = 2u,       /* A18: uncovered non-null words in pointer arrays pass through (counted) */
+  CGCM_PROFILE = 4u        /* time every hot kernel with CUDA events on its launch stream (stats)  */
+};
+
+/* ---- AU flags (declare + dump) ------------------------------------------------------------- */
+enum {
+  CGCM_UNIT_GLOBAL = 1u,      /* declared with cgcm_declareGlobal: persistent device storage (A14) */
+  CGCM_UNIT_READONLY = 2u,    /* never copied back (Alg. 2 `isReadOnly`)           */
+  CGCM_UNIT_ARRAYMAPPED = 4u, /* device copy holds translated pointers (mapArray), A12             */
+  CGCM_UNIT_ACTIVE = 8u       /* refCount > 0                                                       */
+};
+
+typedef struct {
+  uint64_t base, size, devptr; /* devptr: device copy (0 when inactive, except globals, A14)        */
+  int64_t refCount;
+  uint64_t epoch;
+  uint32_t flags, pad;
+} cgcm_unit_t;
+
+typedef struct {
+  /* unit-level copy counters: compared EXACTLY with the oracle */
+  uint64_t h2d_units, h2d_bytes, d2h_units, d2h_bytes;
+  uint64_t activations, frees;
+  uint64_t fwd_translations, rev_translations, null_slots, passthrough;
+  /* implementation counters (reported, not compared, A22) */
+  uint64_t h2d_memcpy_calls, d2h_memcpy_calls, kernel_launches, table_rebuilds, rev_rebuilds;
+  double fwd_kernel_ms, rev_kernel_ms; /* CGCM_PROFILE: summed event time of the hot slot kernels */
+  uint64_t fwd_kernel_calls, rev_kernel_calls;
+  uint64_t fwd_kernel_slots, rev_kernel_slots; /* slots processed by those launches               */
+} cgcm_stats_t;
+
+/* ================================ lifecycle =================================================
+ * cgcm_init: create a context on `device` and make it current for the calling thread.
+ *   dev_arena/arena_bytes: device memory the runtime sub-allocates for AU copies and its own
+ *     scratch (PyTorch provides it: torch.empty(arena_bytes, uint8, device)).  NULL -> cudaMalloc.
+ *     Owned by the caller; must outlive the context.
+ *   main_stream: cudaStream_t on which translation kernels run and which user kernels must use
+ *     (stream-ordered results).  copy_stream: side stream for the coalesced host<->device copies.
+ *     NULL -> the runtime creates its own.
+ * cgcm_finalize: destroy the current context (device storage of globals is released). */
+int cgcm_init(int device, void *dev_arena, size_t arena_bytes, void *main_stream, void *copy_stream,
+              unsigned flags);
+int cgcm_finalize(void);
+void *cgcm_getContext(void);           /* opaque handle of the current context (NULL if none)   */
+int cgcm_setContext(void *ctx);        /* make `ctx` current on this thread                      */
+const char *cgcm_strerror(int status);
+const char *cgcm_lastCudaError(void);  /* text of the last CUDA failure on this thread          */
+
+/* ================================ registration (Table 2) ======================
+ * cgcm_declareAlloc: register the heap/stack AU [base, base+size), size >= 1, no overlap (adjacent
+ *   is allowed).  Its epoch starts at the current globalEpoch (A20).  The CPU bytes stay owned by
+ *   the caller and must stay valid while declared; the CPU must not write an AU while it is mapped
+ *   (A16).  cgcm_declareAllocFlags additionally takes CGCM_UNIT_READONLY (an AU in read-only memory).
+ * cgcm_declareBatch: n AUs at once (bases need not be sorted); all-or-nothing.
+ * cgcm_undeclare: exact base; CGCM_E_BUSY if refCount > 0 (declareAlloca scope exit, free()).
+ * cgcm_declareGlobal: a global: persistent device storage allocated on first map and
+ *   reused (A14); unique name (CGCM_E_DUPLICATE); isReadOnly -> never copied back.             */
+int cgcm_declareAlloc(void *base, size_t size);
+int cgcm_declareAllocFlags(void *base, size_t size, unsigned unit_flags);
+int cgcm_declareBatch(void *const *bases, const size_t *sizes, size_t n, unsigned unit_flags);
+int cgcm_undeclare(void *base);
+int cgcm_declareGlobal(const char *name, void *base, size_t size, int isReadOnly);
+/* Heap wrappers (R10): a header-free pinned host arena; every block is declared as one AU, so
+ * consecutive blocks are host-adjacent and their copies coalesce.  cgcm_free undeclares (BUSY if
+ * mapped -> the block is not freed).  NULL on failure.                                           */
+void *cgcm_malloc(size_t n);
+int cgcm_free(void *p);
+
+/* ================================ mapping (Alg. 1-3, Table 2) ==============================
+ * cgcm_map (Alg. 1): *gpu_out = devptr + (cpu - base) of the AU containing `cpu`;
+ *   refCount += 1; on 0 -> 1 the AU gets device storage and one host->device copy.  NULL -> NULL.
+ *   Data is ready for work enqueued on main_stream after the call returns.
+ * cgcm_unmap (Alg. 2, A1/A3/A4): copy the device copy back iff the AU's epoch is not
+ *   current and it is not read-only (array-mapped AUs are reverse translated, A12); then
+ *   epoch = globalEpoch.  Synchronous: host memory is updated when it returns.
+ * cgcm_release (Alg. 3): refCount -= 1; at 0 the device copy is freed (not globals).
+ * cgcm_mapArray: `cpu` points into an AU of pointers (all floor(size/8)
+ *   words are slots, A10).  The outer AU is activated first (A9), every non-null slot is mapped
+ *   (+1 refCount per slot, A8) and the outer's device copy receives the translated pointers,
+ *   rewritten IN PLACE on the device.  *gpu_out = device address of `cpu` in that copy.
+ * cgcm_unmapArray: unmap of the outer (reverse GPU->CPU rewrite when copied back, a3) and then of
+ *   every element.  cgcm_releaseArray: release every element, then the outer.
+ * cgcm_advanceEpoch: globalEpoch += 1; call once after every GPU function launch.  */
+int cgcm_map(const void *cpu, void **gpu_out);
+int cgcm_unmap(const void *cpu);
+int cgcm_release(const void *cpu);
+int cgcm_mapArray(void *const *cpu, void ***gpu_out);
+int cgcm_unmapArray(void *const *cpu);
+int cgcm_releaseArray(void *const *cpu);
+int cgcm_advanceEpoch(void);
+uint64_t cgcm_epoch(void);
+
+/* ================================ data-parallel batch forms ================================
+ * Same semantics as the sequential loop over the elements (validate, then apply in index order).
+ * Host arrays: cpu[n] / gpu_out[n] are host memory.                                              */
+int cgcm_mapBatch(const void *const *cpu, size_t n, void **gpu_out);
+int cgcm_unmapBatch(const void *const *cpu, size_t n);
+int cgcm_releaseBatch(const void *const *cpu, size_t n);
+int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out);
+int cgcm_unmapArrays(void *const *const *arrays, size_t k);
+int cgcm_releaseArrays(void *const *const *arrays, size_t k);
+/* Device-resident pointer arrays (the hot kernels without the host<->device copy of the array):
+ * d_slots is a DEVICE pointer to n 8-byte-aligned u64 words, rewritten in place.
+ * cgcm_mapArrayDevice:   d_slots[i] <- map(d_slots[i])   (CPU -> GPU; refcount, activation)
+ * cgcm_unmapArrayDevice: d_slots[i] <- reverse(d_slots[i]) (GPU -> CPU), unmap every AU hit
+ *   (epoch-gated copy-back), and with CGCM_RELEASE also release each slot (Listing 3's
+ *   unmapArray + releaseArray, fused).  Stream-ordered on main_stream, synchronous on return.   */
+enum { CGCM_RELEASE = 1u };
+int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n);
+int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags);
+
+/* ================================ introspection ===========================================
+ * cgcm_stats: counters since init.  cgcm_dumpTable: the AU table in base order (cap entries; *n
+ *   = total; CGCM_E_NOMEM if cap < total).  cgcm_resetStats zeroes the counters.                */
+int cgcm_stats(cgcm_stats_t *out);
+int cgcm_resetStats(void);
+int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n);
+/* arena usage in bytes (AU copies + runtime scratch), for balance checks */
+int cgcm_arenaUsage(size_t *used, size_t *capacity);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CGCM_H */

@@ -1,0 +1,1658 @@
+// runtime.cpp -- host side of the B200-native CGCM run-time library (C ABI: include/cgcm.h).
+//
+// What runs here: AU registration (the host half of "allocInfoMap maintenance"),
+// device-arena and pinned-host-arena allocation, the transfer scheduler (coalesced
+// cudaMemcpyAsync runs on the copy stream), orchestration of the kernels and all-or-nothing
+// rollback.  What never runs here: pointer lookup, translation, refcount or epoch decisions --
+// those are the kernels of kernels.cu.  Nothing in this file can fall back
+// to a CPU computation of a kernel's result.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <string>
+#include <unordered_map>
+#include <unordered_set>
+#include <vector>
+
+#include "../../include/cgcm.h"
+#include "cgcm_dev.h"
+
+namespace cgcm {
+
+thread_local std::string g_last_cuda_error;
+
+#define CK(x)                                                                        \
+  do {                                                                               \
+    cudaError_t e_ = (x);                                                            \
+    if (e_ != cudaSuccess) {                                                         \
+      g_last_cuda_error = std::string(#x) + ": " + cudaGetErrorString(e_);           \
+      return CGCM_E_CUDA;                                                            \
+    }                                                                                \
+  } while (0)
+#define CKS(x)                    \
+  do {                            \
+    int s_ = (x);                 \
+    if (s_ != CGCM_OK) return s_; \
+  } while (0)
+
+static inline uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+// ---------------------------------------------------------------------------------------------
+// Device arena: best-fit free list over [base, base+cap) with 256-byte granularity.  All device
+// memory of a context (AU copies, tables, scratch) comes from here; the arena itself is provided
+// by the caller (PyTorch) or cudaMalloc'ed once.
+// ---------------------------------------------------------------------------------------------
+class Arena {
+ public:
+  void init(uint64_t base, uint64_t cap) {
+    uint64_t b = align_up(base, 256);
+    cap_ = (cap - (b - base)) / 256 * 256;
+    base_ = b;
+    by_off_.clear();
+    by_len_.clear();
+    if (cap_) insert(base_, cap_);
+    used_ = 0;
+  }
+  uint64_t alloc(uint64_t bytes) {
+    bytes = align_up(std::max<uint64_t>(bytes, 1), 256);
+    auto it = by_len_.lower_bound(bytes);
+    if (it == by_len_.end()) return 0;
+    uint64_t off = it->second, len = it->first;
+    erase(off, len);
+    if (len > bytes) insert(off + bytes, len - bytes);
+    used_ += bytes;
+    return off;
+  }
+  void free(uint64_t addr, uint64_t bytes) {
+    if (!addr) return;
+    bytes = align_up(std::max<uint64_t>(bytes, 1), 256);
+    used_ -= bytes;
+    uint64_t off = addr, len = bytes;
+    auto nx = by_off_.lower_bound(off);
+    if (nx != by_off_.end() && nx->first == off + len) {
+      len += nx->second;
+      erase(nx->first, nx->second);
+    }
+    auto pv = by_off_.lower_bound(off);
+    if (pv != by_off_.begin()) {
+      --pv;
+      if (pv->first + pv->second == off) {
+        off = pv->first;
+        len += pv->second;
+        erase(pv->first, pv->second);
+      }
+    }
+    insert(off, len);
+  }
+  uint64_t used() const { return used_; }
+  uint64_t capacity() const { return cap_; }
+
+ private:
+  void insert(uint64_t off, uint64_t len) {
+    by_off_[off] = len;
+    by_len_.emplace(len, off);
+  }
+  void erase(uint64_t off, uint64_t len) {
+    by_off_.erase(off);
+    auto r = by_len_.equal_range(len);
+    for (auto it = r.first; it != r.second; ++it)
+      if (it->second == off) {
+        by_len_.erase(it);
+        break;
+      }
+  }
+  uint64_t base_ = 0, cap_ = 0, used_ = 0;
+  std::map<uint64_t, uint64_t> by_off_;
+  std::multimap<uint64_t, uint64_t> by_len_;
+};
+
+// growable device scratch buffer carved from the arena
+struct DevBuf {
+  uint64_t addr = 0;
+  size_t bytes = 0;
+  template <class T>
+  T *as() const { return reinterpret_cast<T *>(addr); }
+};
+
+// growable pinned host buffer
+struct HostBuf {
+  void *p = nullptr;
+  size_t bytes = 0;
+  int ensure(size_t need) {
+    if (need <= bytes) return CGCM_OK;
+    if (p) cudaFreeHost(p);
+    size_t nb = std::max<size_t>(need, std::max<size_t>(bytes * 3 / 2, 1 << 16));
+    if (cudaHostAlloc(&p, nb, cudaHostAllocPortable) != cudaSuccess) {
+      p = nullptr;
+      bytes = 0;
+      return CGCM_E_NOMEM;
+    }
+    bytes = nb;
+    return CGCM_OK;
+  }
+  template <class T>
+  T *as() const { return reinterpret_cast<T *>(p); }
+};
+
+// host registry entry: one declared AU
+struct HostUnit {
+  uint64_t size = 0;
+  uint32_t flags = 0;       // UF_GLOBAL | UF_READONLY
+  uint64_t epoch0 = 0;      // globalEpoch at declaration (A20)
+  int32_t idx = -1;         // rank in the device table (valid after a table build)
+  std::string name;
+  uint64_t devbase = 0;     // mirror of the device copy's address (host allocates it)
+  int64_t run = -1;         // device extent holding the copy
+  bool arrayMapped = false; // mirror of UF_ARRAYMAPPED
+};
+
+// one device extent holding the copies of one or more host-adjacent units (mirrored layout)
+struct Run {
+  uint64_t addr = 0, bytes = 0;
+  int64_t live = 0;
+};
+
+// Search-index buffers (forward: all units by base; reverse: active units by devbase)
+struct IndexBufs {
+  DevBuf top, wide, meta, ndev;
+  DevBuf lvl[MAXL];
+  size_t lvl_cap[MAXL] = {0};
+  int cap = -1;
+  IndexDev view(const uint64_t *keys) const {
+    IndexDev ix;
+    ix.top = top.as<uint64_t>();
+    ix.wide = wide.as<uint32_t>();
+    for (int k = 0; k < MAXL; ++k) ix.lvl[k] = lvl[k].as<uint32_t>();
+    ix.keys = keys;
+    ix.meta = meta.as<int>();
+    return ix;
+  }
+};
+
+struct Context {
+  int device = 0;
+  cudaStream_t main = nullptr, copy = nullptr;
+  bool own_streams = false;
+  void *own_arena = nullptr;
+  unsigned flags = 0;
+  int nsm = 148;
+  Arena arena;
+  std::recursive_mutex mu;
+  uint64_t epoch = 0;
+
+  // registry (host)
+  std::map<uint64_t, HostUnit> reg;
+  std::vector<std::map<uint64_t, HostUnit>::iterator> by_idx;
+  std::unordered_set<std::string> names;
+  bool table_dirty = true, rev_dirty = true;
+  int U = 0;  // units in the device table
+
+  // device table
+  DevBuf rec, dbase;
+  IndexBufs fwd, rev;
+  DevBuf rev_kin, rev_kout, rev_vin, rev_vout, rev_payload, rev_temp;
+  size_t rev_temp_bytes = 0;
+
+  // scratch
+  DevBuf status, lc, hitmask, act_list, journal, free_list, segs, seg0, staging, staging2, points, ptrs, temp;
+  DevBuf up_units, up_vals, uops;
+  HostBuf h_small, h_status, h_list;
+  cudaEvent_t ev_copy = nullptr, ev_t0 = nullptr, ev_t1 = nullptr;
+
+  // runs of device extents
+  std::vector<Run> runs;
+  std::vector<int64_t> free_runs;
+
+  // pinned host arena (cgcm_malloc)
+  std::vector<std::pair<char *, size_t>> hchunks;
+  std::map<uint64_t, uint64_t> hfree;                 // addr -> len
+  std::unordered_map<uint64_t, uint64_t> hallocs;     // addr -> rounded len
+
+  cgcm_stats_t st{};
+
+  // ------------------------------------------------------------------------------------------
+  int dalloc(DevBuf &b, size_t need) {  // ensure capacity (contents not preserved)
+    if (need <= b.bytes && b.addr) return CGCM_OK;
+    if (b.addr) arena.free(b.addr, b.bytes);
+    size_t nb = std::max<size_t>(need, 256);
+    nb = std::max(nb, b.bytes * 3 / 2);
+    b.addr = arena.alloc(nb);
+    if (!b.addr) {
+      b.bytes = 0;
+      return CGCM_E_NOMEM;
+    }
+    b.bytes = align_up(nb, 256);
+    return CGCM_OK;
+  }
+  void dfree(DevBuf &b) {
+    if (b.addr) arena.free(b.addr, b.bytes);
+    b.addr = 0;
+    b.bytes = 0;
+  }
+
+  int64_t new_run(uint64_t addr, uint64_t bytes) {
+    Run r;
+    r.addr = addr;
+    r.bytes = bytes;
+    r.live = 0;
+    if (!free_runs.empty()) {
+      int64_t id = free_runs.back();
+      free_runs.pop_back();
+      runs[id] = r;
+      return id;
+    }
+    runs.push_back(r);
+    return (int64_t)runs.size() - 1;
+  }
+  void run_release(int64_t id) {
+    if (id < 0) return;
+    if (--runs[id].live <= 0) {
+      arena.free(runs[id].addr, runs[id].bytes);
+      runs[id] = Run();
+      free_runs.push_back(id);
+    }
+  }
+
+  int sync_main() {
+    CK(cudaStreamSynchronize(main));
+    return CGCM_OK;
+  }
+
+  // ------------------------------------------------------------------------------------------
+  // index build (a0)
+  int ensure_index_bufs(IndexBufs &ib, int cap) {
+    if (ib.cap >= cap && ib.top.addr) return CGCM_OK;
+    int c = std::max(cap, 1);
+    CKS(dalloc(ib.top, 8 * (size_t)std::min(c, TOPMAX) + 64));
+    CKS(dalloc(ib.wide, 4 * (size_t)((TOPMAX + 31) / 32) + 64));
+    CKS(dalloc(ib.meta, 64));
+    CKS(dalloc(ib.ndev, 64));
+    for (int k = 0; k < MAXL; ++k) {
+      int64_t cnt = ((int64_t)c + (1ll << (3 * k)) - 1) >> (3 * k);
+      size_t need = (size_t)((cnt + 7) / 8 * 8 + 8);
+      // levels k >= h are never used; only allocate levels that can exist for this capacity
+      bool used = cnt > 1 || k == 0;
+      if (!used) {
+        dfree(ib.lvl[k]);
+        ib.lvl_cap[k] = 0;
+        continue;
+      }
+      CKS(dalloc(ib.lvl[k], 4 * need));
+      ib.lvl_cap[k] = need;
+    }
+    ib.cap = c;
+    return CGCM_OK;
+  }
+  int build_index(IndexBufs &ib, const uint64_t *keys, const int *n_dev, int cap) {
+    uint32_t *lv[MAXL];
+    for (int k = 0; k < MAXL; ++k) lv[k] = ib.lvl[k].as<uint32_t>();
+    launch_build_index(keys, n_dev, cap, ib.top.as<uint64_t>(), ib.wide.as<uint32_t>(), lv, ib.lvl_cap,
+                       ib.meta.as<int>(), main);
+    st.kernel_launches += 2 + MAXL;
+    CK(cudaGetLastError());
+    return CGCM_OK;
+  }
+
+  // merge pending declares/undeclares into the device table (A19: kernels only see a compacted table)
+  int ensure_table() {
+    if (!table_dirty) return CGCM_OK;
+    int n = (int)reg.size();
+    // host staging: base[n], size[n], epoch0[n], old_idx[n], flags[n]
+    size_t need = (size_t)n * (8 + 8 + 8 + 4 + 4) + 256;
+    CKS(h_list.ensure(need));
+    CK(cudaStreamSynchronize(main));
+    CK(cudaStreamSynchronize(copy));
+    uint64_t *hb = h_list.as<uint64_t>();
+    uint64_t *hs = hb + n;
+    uint64_t *he = hs + n;
+    int32_t *ho = reinterpret_cast<int32_t *>(he + n);
+    uint32_t *hf = reinterpret_cast<uint32_t *>(ho + n);
+    by_idx.assign(n, reg.end());
+    int i = 0;
+    for (auto it = reg.begin(); it != reg.end(); ++it, ++i) {
+      hb[i] = it->first;
+      hs[i] = it->second.size;
+      he[i] = it->second.epoch0;
+      ho[i] = it->second.idx;
+      hf[i] = it->second.flags & (UF_GLOBAL | UF_READONLY);
+      it->second.idx = i;
+      by_idx[i] = it;
+    }
+    DevBuf nrec, nbase, tmp;
+    int cap = std::max(n, 1);
+    CKS(dalloc(nrec, 32 * (size_t)cap));
+    CKS(dalloc(nbase, 8 * (size_t)cap));
+    CKS(dalloc(tmp, (size_t)cap * 24 + 256));
+    if (n > 0) {
+      CK(cudaMemcpyAsync(nbase.as<void>(), hb, 8 * (size_t)n, cudaMemcpyHostToDevice, main));
+      CK(cudaMemcpyAsync(tmp.as<void>(), hs, (size_t)n * 24, cudaMemcpyHostToDevice, main));
+      DevBuf tmp2;
+      CKS(dalloc(tmp2, (size_t)n * 8 + 256));
+      CK(cudaMemcpyAsync(tmp2.as<void>(), ho, (size_t)n * 8, cudaMemcpyHostToDevice, main));
+      const uint64_t *dsize = tmp.as<uint64_t>();
+      const uint64_t *depoch = dsize + 2 * (size_t)n;
+      const int32_t *dold = tmp2.as<int32_t>();
+      const uint32_t *dflags = reinterpret_cast<const uint32_t *>(dold + n);
+      launch_remap(n, dold, dsize, dflags, depoch, rec.as<UnitRec>(), nrec.as<UnitRec>(), main);
+      st.kernel_launches += 1;
+      CK(cudaGetLastError());
+      CK(cudaStreamSynchronize(main));
+      dfree(tmp2);
+    }
+    dfree(tmp);
+    dfree(rec);
+    dfree(dbase);
+    rec = nrec;
+    dbase = nbase;
+    U = n;
+    CKS(ensure_index_bufs(fwd, cap));
+    CK(cudaMemcpyAsync(fwd.ndev.as<void>(), &n, sizeof(int), cudaMemcpyHostToDevice, main));
+    CKS(build_index(fwd, dbase.as<uint64_t>(), fwd.ndev.as<int>(), n));
+    CK(cudaStreamSynchronize(main));
+    table_dirty = false;
+    rev_dirty = true;
+    st.table_rebuilds += 1;
+    return CGCM_OK;
+  }
+
+  int ensure_rev() {
+    CKS(ensure_table());
+    if (!rev_dirty) return CGCM_OK;
+    int cap = std::max(U, 1);
+    CKS(dalloc(rev_kin, 8 * (size_t)cap));
+    CKS(dalloc(rev_kout, 8 * (size_t)cap));
+    CKS(dalloc(rev_vin, 4 * (size_t)cap + 64));
+    CKS(dalloc(rev_vout, 4 * (size_t)cap + 64));
+    CKS(dalloc(rev_payload, 16 * (size_t)cap));
+    size_t tb = sort_pairs_temp_bytes(cap);
+    CKS(dalloc(rev_temp, tb + 256));
+    CKS(ensure_index_bufs(rev, cap));
+    launch_rev_collect(rec.as<UnitRec>(), U, rev_kin.as<uint64_t>(), rev_vin.as<uint32_t>(), rev.ndev.as<int>(),
+                       main);
+    if (U > 0)
+      launch_sort_pairs(rev_temp.as<void>(), rev_temp.bytes, rev_kin.as<uint64_t>(), rev_kout.as<uint64_t>(),
+                        rev_vin.as<uint32_t>(), rev_vout.as<uint32_t>(), U, main);
+    launch_rev_payload(rev_vout.as<uint32_t>(), dbase.as<uint64_t>(), rev.ndev.as<int>(), U,
+                       rev_payload.as<RevRec>(), main);
+    st.kernel_launches += 3;
+    CK(cudaGetLastError());
+    CKS(build_index(rev, rev_kout.as<uint64_t>(), rev.ndev.as<int>(), cap));
+    rev_dirty = false;
+    st.rev_rebuilds += 1;
+    return CGCM_OK;
+  }
+
+  // ------------------------------------------------------------------------------------------
+  // slot kernels
+  struct SlotCall {
+    int dir = DIR_FWD, ops = 0, sel = SEL_ALL;
+    std::vector<Seg> segs;
+    uint64_t nchunks = 0;
+    Status res{};
+  };
+
+  int list_capacity() const { return std::max(U, 1); }
+
+  // upload segments, launch, (no sync).  slot st index = which Status block to use.
+  int launch(SlotCall &c, int st_index, bool reuse_hitmask_layout = false, bool timed_fwd = false,
+             bool timed_rev = false) {
+    (void)reuse_hitmask_layout;
+    int k = (int)c.segs.size();
+    if (k == 0) return CGCM_OK;
+    std::vector<uint64_t> c0(k + 1, 0);
+    for (int s = 0; s < k; ++s) {
+      uint64_t head = (c.segs[s].ptr & 31) / 8;
+      c0[s + 1] = c0[s] + (c.segs[s].n ? (head + c.segs[s].n + 3) / 4 : 0);
+    }
+    c.nchunks = c0[k];
+    if (c.nchunks == 0) return CGCM_OK;
+    if ((c.ops & OP_HITMASK) || c.sel != SEL_ALL) CKS(dalloc(hitmask, (size_t)c.nchunks + 64));
+    CKS(dalloc(segs, sizeof(Seg) * (size_t)k * 4 + 256));
+    CKS(dalloc(seg0, 8 * (size_t)(k + 1) * 4 + 256));
+    // each launch uses its own quarter of the segment buffers (up to 4 launches in flight)
+    Seg *dsegs = segs.as<Seg>() + (size_t)st_index * k;
+    uint64_t *dc0 = seg0.as<uint64_t>() + (size_t)st_index * (k + 1);
+    CK(cudaMemcpyAsync(dsegs, c.segs.data(), sizeof(Seg) * k, cudaMemcpyHostToDevice, main));
+    CK(cudaMemcpyAsync(dc0, c0.data(), 8 * (size_t)(k + 1), cudaMemcpyHostToDevice, main));
+    CK(cudaStreamSynchronize(main));  // the host vectors above are pageable and go out of scope
+    SlotArgs a;
+    std::memset(&a, 0, sizeof(a));
+    a.rec = rec.as<UnitRec>();
+    if (c.dir == DIR_FWD) {
+      a.ix = fwd.view(dbase.as<uint64_t>());
+      a.smem_top = std::min(std::max(U, 1), TOPMAX);
+    } else {
+      a.ix = rev.view(rev_kout.as<uint64_t>());
+      a.rev = rev_payload.as<RevRec>();
+      a.smem_top = std::min(std::max(U, 1), TOPMAX);
+    }
+    a.segs = dsegs;
+    a.seg_chunk0 = dc0;
+    a.nseg = k;
+    a.sel = c.sel;
+    a.nchunks = c.nchunks;
+    a.hitmask = hitmask.as<uint8_t>();
+    a.epoch = epoch;
+    a.st = status.as<Status>() + st_index;
+    a.lc = lc.as<unsigned long long>();
+    a.act_list = act_list.as<uint32_t>();
+    a.journal = journal.as<Journal>();
+    a.free_list = free_list.as<uint32_t>();
+    a.lenient = (flags & CGCM_LENIENT) ? 1 : 0;
+    bool timed = (flags & CGCM_PROFILE) && (timed_fwd || timed_rev);
+    if (timed) CK(cudaEventRecord(ev_t0, main));
+    int r = launch_slots(c.dir, c.ops, a, nsm, main);
+    if (r == -2) {
+      g_last_cuda_error = "unsupported slot-kernel operation set";
+      return CGCM_E_CUDA;
+    }
+    CK(cudaGetLastError());
+    st.kernel_launches += 1;
+    if (timed) {
+      CK(cudaEventRecord(ev_t1, main));
+      CK(cudaEventSynchronize(ev_t1));
+      float ms = 0;
+      CK(cudaEventElapsedTime(&ms, ev_t0, ev_t1));
+      uint64_t slots = 0;
+      for (auto &s : c.segs) slots += s.n;
+      if (timed_fwd) {
+        st.fwd_kernel_ms += ms;
+        st.fwd_kernel_calls += 1;
+        st.fwd_kernel_slots += slots;
+      } else {
+        st.rev_kernel_ms += ms;
+        st.rev_kernel_calls += 1;
+        st.rev_kernel_slots += slots;
+      }
+    }
+    return CGCM_OK;
+  }
+
+  // scratch sized for n slots and the unit lists
+  int prepare(uint64_t nslots_total) {
+    (void)nslots_total;
+    CKS(dalloc(status, sizeof(Status) * 8 + 256));
+    CKS(dalloc(lc, 64));
+    int cap = list_capacity();
+    CKS(dalloc(act_list, 4 * (size_t)cap + 64));
+    CKS(dalloc(free_list, 4 * (size_t)cap + 64));
+    CKS(dalloc(journal, sizeof(Journal) * (size_t)cap + 64));
+    CK(cudaMemsetAsync(status.as<void>(), 0, sizeof(Status) * 8, main));
+    CK(cudaMemsetAsync(lc.as<void>(), 0, 64, main));
+    CKS(h_status.ensure(sizeof(Status) * 8 + 64));
+    return CGCM_OK;
+  }
+  // fetch the 8 Status blocks + list counters (synchronizes main)
+  int fetch_status(Status out[8], unsigned long long lcs[3]) {
+    CK(cudaMemcpyAsync(h_status.p, status.as<void>(), sizeof(Status) * 8, cudaMemcpyDeviceToHost, main));
+    CK(cudaMemcpyAsync(h_status.as<char>() + sizeof(Status) * 8, lc.as<void>(), 24, cudaMemcpyDeviceToHost, main));
+    CK(cudaStreamSynchronize(main));
+    std::memcpy(out, h_status.p, sizeof(Status) * 8);
+    std::memcpy(lcs, h_status.as<char>() + sizeof(Status) * 8, 24);
+    return CGCM_OK;
+  }
+
+  template <class T>
+  int download(std::vector<T> &out, const DevBuf &src, size_t n) {
+    out.resize(n);
+    if (!n) return CGCM_OK;
+    CKS(h_list.ensure(sizeof(T) * n));
+    CK(cudaMemcpyAsync(h_list.p, src.as<void>(), sizeof(T) * n, cudaMemcpyDeviceToHost, main));
+    CK(cudaStreamSynchronize(main));
+    std::memcpy(out.data(), h_list.p, sizeof(T) * n);
+    return CGCM_OK;
+  }
+  template <class T>
+  int upload(DevBuf &dst, const std::vector<T> &v) {
+    CKS(dalloc(dst, sizeof(T) * v.size() + 64));
+    if (v.empty()) return CGCM_OK;
+    CKS(h_small.ensure(sizeof(T) * v.size()));
+    CK(cudaStreamSynchronize(main));
+    std::memcpy(h_small.p, v.data(), sizeof(T) * v.size());
+    CK(cudaMemcpyAsync(dst.as<void>(), h_small.p, sizeof(T) * v.size(), cudaMemcpyHostToDevice, main));
+    CK(cudaStreamSynchronize(main));
+    return CGCM_OK;
+  }
+  int unit_ops(const std::vector<UnitOp> &ops) {
+    if (ops.empty()) return CGCM_OK;
+    CKS(upload(uops, ops));
+    launch_unit_ops(uops.as<UnitOp>(), (int)ops.size(), rec.as<UnitRec>(), main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
+    return CGCM_OK;
+  }
+
+  // sorted unique unit list from a device list of n entries
+  int sorted_units(const DevBuf &src, size_t n, std::vector<uint32_t> &out) {
+    out.clear();
+    if (!n) return CGCM_OK;
+    if (n > 1) {
+      size_t tb = sort_keys_temp_bytes((int)n);
+      CKS(dalloc(temp, tb + 256 + 4 * n + 64));
+      uint32_t *sorted = reinterpret_cast<uint32_t *>(temp.addr + align_up(tb, 256));
+      launch_sort_keys(temp.as<void>(), tb, src.as<uint32_t>(), sorted, (int)n, main);
+      st.kernel_launches += 1;
+      CK(cudaGetLastError());
+      DevBuf view;
+      view.addr = reinterpret_cast<uint64_t>(sorted);
+      view.bytes = 4 * n;
+      CKS(download(out, view, n));
+    } else {
+      CKS(download(out, src, n));
+    }
+    return CGCM_OK;
+  }
+
+  // ------------------------------------------------------------------------------------------
+  // activation (refcount 0 -> 1 transitions collected by the map kernel): allocate device storage
+  // with host-adjacent units mirrored into one extent, write devbase (+ epoch, A5 R1), and copy
+  // the units host -> device as coalesced runs on the copy stream (transfer scheduler).
+  int activate_units(const std::vector<uint32_t> &units, std::vector<std::pair<uint64_t, uint64_t>> *h2d_out) {
+    if (units.empty()) return CGCM_OK;
+    std::vector<uint64_t> devbases(units.size());
+    struct Copy { uint64_t dst, src, len; };
+    std::vector<Copy> copies;
+    std::vector<int64_t> new_runs;
+    size_t i = 0;
+    uint64_t bytes = 0;
+    while (i < units.size()) {
+      HostUnit &u0 = by_idx[units[i]]->second;
+      uint64_t b0 = by_idx[units[i]]->first;
+      if (u0.flags & UF_GLOBAL) {
+        if (u0.run < 0) {  // named region: allocated once, persists (A14)
+          uint64_t need = (b0 % 256) + u0.size + 1;
+          uint64_t a = arena.alloc(need);
+          if (!a) goto nomem;
+          u0.run = new_run(a, need);
+          runs[u0.run].live = 1;
+          u0.devbase = a + (b0 % 256);
+          new_runs.push_back(u0.run);
+        }
+        devbases[i] = u0.devbase;
+        copies.push_back({u0.devbase, b0, u0.size});
+        bytes += u0.size;
+        ++i;
+        continue;
+      }
+      // maximal run of index-consecutive, host-adjacent, non-global units
+      size_t j = i + 1;
+      uint64_t end = b0 + u0.size;
+      while (j < units.size() && units[j] == units[j - 1] + 1) {
+        auto it = by_idx[units[j]];
+        if ((it->second.flags & UF_GLOBAL) || it->first != end) break;
+        end += it->second.size;
+        ++j;
+      }
+      uint64_t need = (b0 % 256) + (end - b0) + 1;  // +1: device copies never adjacent (A7)
+      uint64_t a = arena.alloc(need);
+      if (!a) goto nomem;
+      int64_t rid = new_run(a, need);
+      new_runs.push_back(rid);
+      uint64_t d0 = a + (b0 % 256);
+      for (size_t q = i; q < j; ++q) {
+        auto it = by_idx[units[q]];
+        it->second.devbase = d0 + (it->first - b0);
+        it->second.run = rid;
+        runs[rid].live += 1;
+        devbases[q] = it->second.devbase;
+      }
+      copies.push_back({d0, b0, end - b0});
+      bytes += end - b0;
+      i = j;
+    }
+    {
+      CKS(upload(up_units, units));
+      CKS(upload(up_vals, devbases));
+      launch_set_devbase(up_units.as<uint32_t>(), up_vals.as<uint64_t>(), (int)units.size(), rec.as<UnitRec>(), epoch,
+                         (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
+      st.kernel_launches += 1;
+      CK(cudaGetLastError());
+      for (auto &c : copies) {
+        CK(cudaMemcpyAsync(reinterpret_cast<void *>(c.dst), reinterpret_cast<const void *>(c.src), c.len,
+                           cudaMemcpyHostToDevice, copy));
+        if (h2d_out) h2d_out->push_back({c.dst, c.len});
+      }
+      CK(cudaEventRecord(ev_copy, copy));
+      CK(cudaStreamWaitEvent(main, ev_copy, 0));
+      st.h2d_memcpy_calls += copies.size();
+      st.h2d_units += units.size();
+      st.h2d_bytes += bytes;
+      st.activations += units.size();
+      rev_dirty = true;
+      return CGCM_OK;
+    }
+  nomem:
+    for (int64_t r : new_runs) {
+      arena.free(runs[r].addr, runs[r].bytes);
+      runs[r] = Run();
+      free_runs.push_back(r);
+    }
+    for (size_t q = 0; q < units.size(); ++q) {
+      HostUnit &u = by_idx[units[q]]->second;
+      if (std::find(new_runs.begin(), new_runs.end(), u.run) != new_runs.end()) {
+        u.run = -1;
+        u.devbase = 0;
+      }
+    }
+    return CGCM_E_NOMEM;
+  }
+
+  // units whose refcount reached 0: free device storage (globals keep theirs), clear flags
+  int free_units(const std::vector<uint32_t> &units) {
+    if (units.empty()) return CGCM_OK;
+    CKS(upload(up_units, units));
+    launch_deactivate(up_units.as<uint32_t>(), (int)units.size(), rec.as<UnitRec>(), main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(main));
+    for (uint32_t x : units) {
+      HostUnit &u = by_idx[x]->second;
+      u.arrayMapped = false;
+      if (u.flags & UF_GLOBAL) continue;
+      run_release(u.run);
+      u.run = -1;
+      u.devbase = 0;
+      st.frees += 1;
+    }
+    rev_dirty = true;
+    return CGCM_OK;
+  }
+
+  // copy-back of whole units device -> host (Alg. 2's cuMemcpyDtoH).  Array-mapped units are
+  // reverse translated first (A12) -- validated before any byte moves.  Synchronous.
+  int copy_back(const std::vector<uint32_t> &units) {
+    if (units.empty()) return CGCM_OK;
+    std::vector<uint32_t> plain, arr;
+    for (uint32_t x : units) (by_idx[x]->second.arrayMapped ? arr : plain).push_back(x);
+    // reverse-translate the array-mapped ones into staging2
+    uint64_t arr_bytes = 0;
+    for (uint32_t x : arr) arr_bytes += align_up(by_idx[x]->second.size / 8 * 8, 32) + 32;
+    if (!arr.empty()) {
+      CKS(ensure_rev());
+      CKS(dalloc(staging2, arr_bytes + 256));
+      SlotCall c;
+      c.dir = DIR_REV;
+      c.ops = OP_WRITE;
+      uint64_t off = staging2.addr;
+      std::vector<uint64_t> dst(arr.size());
+      for (size_t q = 0; q < arr.size(); ++q) {
+        HostUnit &u = by_idx[arr[q]]->second;
+        uint64_t n = u.size / 8;
+        off = align_up(off, 32) + (u.devbase & 31);  // same alignment as the source
+        dst[q] = off;
+        Seg s;
+        s.ptr = u.devbase;
+        s.n = n;
+        s.out = off;
+        s.inc = 0;
+        s.pad = 0;
+        if (n) c.segs.push_back(s);
+        off += 8 * n;
+      }
+      CKS(prepare_small());
+      CKS(launch(c, 7));
+      Status sts[8];
+      unsigned long long lcs[3];
+      CKS(fetch_status(sts, lcs));
+      if (sts[7].misses && !(flags & CGCM_LENIENT)) return CGCM_E_UNREGISTERED;
+      st.rev_translations += sts[7].translated;
+      st.passthrough += (flags & CGCM_LENIENT) ? sts[7].misses : 0;
+      for (size_t q = 0; q < arr.size(); ++q) {
+        auto it = by_idx[arr[q]];
+        HostUnit &u = it->second;
+        uint64_t n = u.size / 8;
+        if (n) CK(cudaMemcpyAsync(reinterpret_cast<void *>(it->first), reinterpret_cast<void *>(dst[q]), 8 * n,
+                                  cudaMemcpyDeviceToHost, copy));
+        if (u.size > 8 * n)
+          CK(cudaMemcpyAsync(reinterpret_cast<void *>(it->first + 8 * n), reinterpret_cast<void *>(u.devbase + 8 * n),
+                             u.size - 8 * n, cudaMemcpyDeviceToHost, copy));
+        st.d2h_memcpy_calls += 1 + (u.size > 8 * n);
+        st.d2h_units += 1;
+        st.d2h_bytes += u.size;
+      }
+    }
+    // plain units: coalesce host-adjacent units whose device copies are mirrored
+    size_t i = 0;
+    while (i < plain.size()) {
+      auto it0 = by_idx[plain[i]];
+      uint64_t h0 = it0->first, d0 = it0->second.devbase, hend = h0 + it0->second.size;
+      st.d2h_units += 1;
+      st.d2h_bytes += it0->second.size;
+      size_t j = i + 1;
+      while (j < plain.size() && plain[j] == plain[j - 1] + 1) {
+        auto it = by_idx[plain[j]];
+        if (it->first != hend || it->second.devbase != d0 + (it->first - h0)) break;
+        hend += it->second.size;
+        st.d2h_units += 1;
+        st.d2h_bytes += it->second.size;
+        ++j;
+      }
+      CK(cudaMemcpyAsync(reinterpret_cast<void *>(h0), reinterpret_cast<void *>(d0), hend - h0,
+                         cudaMemcpyDeviceToHost, copy));
+      st.d2h_memcpy_calls += 1;
+      i = j;
+    }
+    CK(cudaStreamSynchronize(copy));
+    return CGCM_OK;
+  }
+  int prepare_small() {
+    CKS(dalloc(status, sizeof(Status) * 8 + 256));
+    CKS(dalloc(lc, 64));
+    CK(cudaMemsetAsync(status.as<void>(), 0, sizeof(Status) * 8, main));
+    CKS(h_status.ensure(sizeof(Status) * 8 + 64));
+    int cap = list_capacity();
+    CKS(dalloc(act_list, 4 * (size_t)cap + 64));
+    CKS(dalloc(free_list, 4 * (size_t)cap + 64));
+    CKS(dalloc(journal, sizeof(Journal) * (size_t)cap + 64));
+    return CGCM_OK;
+  }
+
+  // ------------------------------------------------------------------------------------------
+  // forward map over device slot segments (in place or out of place): a1 + a2.
+  // prelaunch: optional additional REV INCPLAIN segments (array-mapped outers re-mapped, A9).
+  // On error everything this function did is undone; the caller undoes its own prologue.
+  int map_core(const std::vector<Seg> &fsegs, const std::vector<Seg> &rsegs, uint64_t *translated_out,
+               uint64_t *nulls_out) {
+    uint64_t total = 0;
+    for (auto &s : fsegs) total += s.n;
+    CKS(prepare(total + 64));
+    SlotCall F;
+    F.dir = DIR_FWD;
+    F.ops = OP_WRITE | OP_INC | OP_HITMASK;
+    F.segs = fsegs;
+    SlotCall R;
+    R.dir = DIR_REV;
+    R.ops = OP_INCPLAIN;
+    R.segs = rsegs;
+    if (!rsegs.empty()) CKS(ensure_rev());
+    CKS(launch(F, 0, false, true, false));
+    // hitmask is per launch: the REV pass does not use it
+    if (!rsegs.empty()) CKS(launch(R, 1));
+    Status sts[8];
+    unsigned long long lcs[3];
+    CKS(fetch_status(sts, lcs));
+    bool strict = !(flags & CGCM_LENIENT);
+    if ((sts[0].misses || sts[1].misses) && strict) {
+      CKS(undo_map(F, R));
+      return CGCM_E_UNREGISTERED;
+    }
+    // activations
+    if (lcs[0] > 0) {
+      std::vector<uint32_t> units;
+      CKS(sorted_units(act_list, lcs[0], units));
+      int r = activate_units(units, nullptr);
+      if (r != CGCM_OK) {
+        CKS(undo_map(F, R));
+        return r;
+      }
+    }
+    if (sts[0].pending > 0) {  // complete the slots whose unit was activated by this call
+      SlotCall C;
+      C.dir = DIR_FWD;
+      C.ops = OP_WRITE;
+      C.sel = SEL_NOTHIT;
+      C.segs = fsegs;
+      CKS(launch(C, 2));
+    }
+    CK(cudaStreamSynchronize(main));
+    uint64_t tr = sts[0].hits + sts[1].hits;
+    st.fwd_translations += tr;
+    st.null_slots += sts[0].nulls + sts[1].nulls;
+    if (!strict) st.passthrough += sts[0].misses + sts[1].misses;
+    if (translated_out) *translated_out = tr;
+    if (nulls_out) *nulls_out = sts[0].nulls + sts[1].nulls;
+    return CGCM_OK;
+  }
+  int undo_map(SlotCall &F, SlotCall &R) {
+    // forward maps are always in place: translated slots (hit bit set) hold GPU pointers again
+    // turned back into CPU pointers (reverse lookup) and lose their reference; the other hits
+    // (pending activations) only lose their reference.
+    rev_dirty = true;  // refcounts changed: rebuild the reverse index over the current active set
+    CKS(ensure_rev());
+    CKS(prepare_small());
+    SlotCall a;
+    a.dir = DIR_REV;
+    a.ops = OP_WRITE | OP_DECPLAIN;
+    a.sel = SEL_HIT;
+    a.segs = F.segs;  // same chunk numbering as the forward launch (hitmask)
+    CKS(launch(a, 0));
+    SlotCall b;
+    b.dir = DIR_FWD;
+    b.ops = OP_DECPLAIN;
+    b.sel = SEL_NOTHIT;
+    b.segs = F.segs;
+    CKS(launch(b, 1));
+    if (!R.segs.empty()) {
+      SlotCall r;
+      r.dir = DIR_REV;
+      r.ops = OP_DECPLAIN;
+      r.segs = R.segs;
+      CKS(launch(r, 2));
+    }
+    CK(cudaStreamSynchronize(main));
+    rev_dirty = true;
+    return CGCM_OK;
+  }
+
+  // reverse unmap over device slot segments (GPU pointers): a3 + a4 (+ release)
+  //   ops: OP_WRITE|OP_GATE|OP_HITMASK [|OP_DEC] or OP_GATE
+  int unmap_rev_core(const std::vector<Seg> &segs, bool write, bool dec, std::vector<uint32_t> &copy_units,
+                     std::vector<uint32_t> &freed, std::vector<Journal> &journal_out, Status &res) {
+    CKS(ensure_rev());
+    uint64_t total = 0;
+    for (auto &s : segs) total += s.n;
+    CKS(prepare(total + 64));
+    SlotCall c;
+    c.dir = DIR_REV;
+    c.ops = write ? (OP_WRITE | OP_GATE | OP_HITMASK | (dec ? OP_DEC : 0)) : (OP_GATE | (dec ? OP_DEC : 0));
+    if (!write && dec) c.ops = OP_GATE | OP_DEC;
+    c.segs = segs;
+    CKS(launch(c, 0, false, false, true));
+    Status sts[8];
+    unsigned long long lcs[3];
+    CKS(fetch_status(sts, lcs));
+    res = sts[0];
+    std::vector<Journal> jn;
+    CKS(download(jn, journal, lcs[1]));
+    bool strict = !(flags & CGCM_LENIENT);
+    int err = CGCM_OK;
+    if (sts[0].misses && strict) err = CGCM_E_UNREGISTERED;
+    else if (sts[0].underflow) err = CGCM_E_NOT_MAPPED;
+    if (err) {
+      CKS(undo_rev(c, jn, write, dec));
+      return err;
+    }
+    journal_out = jn;
+    for (auto &j : jn)
+      if (j.copy) copy_units.push_back(j.unit);
+    std::sort(copy_units.begin(), copy_units.end());
+    if (dec && lcs[2]) {
+      std::vector<uint32_t> f;
+      CKS(download(f, free_list, lcs[2]));
+      freed.insert(freed.end(), f.begin(), f.end());
+    }
+    return CGCM_OK;
+  }
+  int undo_rev(SlotCall &c, const std::vector<Journal> &jn, bool write, bool dec) {
+    CKS(prepare_small());
+    if (!jn.empty()) {
+      std::vector<Journal> j2 = jn;
+      DevBuf jb;
+      CKS(upload(jb, j2));
+      launch_restore_epochs(jb.as<Journal>(), (int)j2.size(), rec.as<UnitRec>(), main);
+      st.kernel_launches += 1;
+      CK(cudaStreamSynchronize(main));
+      dfree(jb);
+    }
+    bool inplace = true;
+    for (auto &s : c.segs) inplace = inplace && s.out == 0;
+    if (write && inplace) {
+      // written slots now hold CPU pointers: forward-translate them back (+ re-add the reference)
+      SlotCall f;
+      f.dir = DIR_FWD;
+      f.ops = dec ? (OP_WRITE | OP_INCPLAIN) : OP_WRITE;
+      f.sel = SEL_HIT;
+      f.segs = c.segs;
+      CKS(launch(f, 1));
+    } else if (dec) {
+      SlotCall f;
+      f.dir = DIR_REV;
+      f.ops = OP_INCPLAIN;
+      f.segs = c.segs;
+      CKS(launch(f, 1));
+    }
+    CK(cudaStreamSynchronize(main));
+    return CGCM_OK;
+  }
+
+  // outer-pointer lookups (one kernel, k pointers)
+  int lookup_points(const uint64_t *ptrs, size_t k, std::vector<PointInfo> &out) {
+    CKS(ensure_table());
+    std::vector<uint64_t> v(ptrs, ptrs + k);
+    CKS(upload(this->ptrs, v));
+    CKS(dalloc(points, sizeof(PointInfo) * k + 64));
+    launch_lookup_points(fwd.view(dbase.as<uint64_t>()), rec.as<UnitRec>(), this->ptrs.as<uint64_t>(), (int)k,
+                         points.as<PointInfo>(), main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
+    CKS(download(out, points, k));
+    return CGCM_OK;
+  }
+};
+
+// ---------------------------------------------------------------------------------------------
+std::mutex g_ctx_mu;
+std::unordered_set<Context *> g_contexts;
+thread_local Context *tl_ctx = nullptr;
+
+}  // namespace cgcm
+
+using namespace cgcm;
+using SlotCall = Context::SlotCall;
+
+#define CTX()                                     \
+  Context *C = tl_ctx;                            \
+  if (!C) return CGCM_E_NOCTX;                    \
+  std::lock_guard<std::recursive_mutex> lk_(C->mu); \
+  if (cudaSetDevice(C->device) != cudaSuccess) return CGCM_E_CUDA;
+
+// ============================== C ABI ==========================================================
+extern "C" {
+
+const char *cgcm_strerror(int s) {
+  switch (s) {
+    case CGCM_OK: return "ok";
+    case CGCM_E_INVALID: return "invalid argument";
+    case CGCM_E_UNREGISTERED: return "pointer not inside a declared allocation unit";
+    case CGCM_E_OVERLAP: return "allocation unit overlaps a declared one";
+    case CGCM_E_NOT_MAPPED: return "allocation unit not mapped (refCount 0)";
+    case CGCM_E_BUSY: return "allocation unit is mapped";
+    case CGCM_E_DUPLICATE: return "global name already declared";
+    case CGCM_E_NOMEM: return "out of memory";
+    case CGCM_E_CUDA: return "CUDA error";
+    case CGCM_E_MIXED: return "mixed";
+    case CGCM_E_NOCTX: return "no current context";
+  }
+  return "unknown";
+}
+const char *cgcm_lastCudaError(void) { return g_last_cuda_error.c_str(); }
+
+int cgcm_init(int device, void *dev_arena, size_t arena_bytes, void *main_stream, void *copy_stream, unsigned flags) {
+  if (arena_bytes < (1u << 20)) return CGCM_E_INVALID;
+  CK(cudaSetDevice(device));
+  Context *C = new Context();
+  C->device = device;
+  C->flags = flags;
+  int nsm = 0;
+  if (cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, device) == cudaSuccess && nsm > 0) C->nsm = nsm;
+  if (!dev_arena) {
+    if (cudaMalloc(&C->own_arena, arena_bytes) != cudaSuccess) {
+      delete C;
+      g_last_cuda_error = "cudaMalloc of the device arena failed";
+      return CGCM_E_NOMEM;
+    }
+    dev_arena = C->own_arena;
+  }
+  C->arena.init(reinterpret_cast<uint64_t>(dev_arena), arena_bytes);
+  if (!main_stream || !copy_stream) {
+    cudaStreamCreateWithFlags(&C->main, cudaStreamNonBlocking);
+    cudaStreamCreateWithFlags(&C->copy, cudaStreamNonBlocking);
+    C->own_streams = true;
+  } else {
+    C->main = reinterpret_cast<cudaStream_t>(main_stream);
+    C->copy = reinterpret_cast<cudaStream_t>(copy_stream);
+  }
+  cudaEventCreateWithFlags(&C->ev_copy, cudaEventDisableTiming);
+  cudaEventCreate(&C->ev_t0);
+  cudaEventCreate(&C->ev_t1);
+  {
+    std::lock_guard<std::mutex> g(g_ctx_mu);
+    g_contexts.insert(C);
+  }
+  tl_ctx = C;
+  std::lock_guard<std::recursive_mutex> lk(C->mu);
+  return C->ensure_table();
+}
+
+int cgcm_finalize(void) {
+  Context *C = tl_ctx;
+  if (!C) return CGCM_E_NOCTX;
+  {
+    std::lock_guard<std::mutex> g(g_ctx_mu);
+    g_contexts.erase(C);
+  }
+  cudaSetDevice(C->device);
+  cudaStreamSynchronize(C->main);
+  cudaStreamSynchronize(C->copy);
+  for (auto &c : C->hchunks) cudaFreeHost(c.first);
+  if (C->h_small.p) cudaFreeHost(C->h_small.p);
+  if (C->h_status.p) cudaFreeHost(C->h_status.p);
+  if (C->h_list.p) cudaFreeHost(C->h_list.p);
+  cudaEventDestroy(C->ev_copy);
+  cudaEventDestroy(C->ev_t0);
+  cudaEventDestroy(C->ev_t1);
+  if (C->own_streams) {
+    cudaStreamDestroy(C->main);
+    cudaStreamDestroy(C->copy);
+  }
+  if (C->own_arena) cudaFree(C->own_arena);
+  delete C;
+  tl_ctx = nullptr;
+  return CGCM_OK;
+}
+
+void *cgcm_getContext(void) { return tl_ctx; }
+int cgcm_setContext(void *ctx) {
+  std::lock_guard<std::mutex> g(g_ctx_mu);
+  if (ctx && !g_contexts.count(reinterpret_cast<Context *>(ctx))) return CGCM_E_INVALID;
+  tl_ctx = reinterpret_cast<Context *>(ctx);
+  return CGCM_OK;
+}
+
+// ---- registration --------------------------------------------------------------------------
+static int declare_one(Context *C, uint64_t b, uint64_t s, uint32_t fl, const char *name) {
+  if (b == 0 || s == 0 || b + s < b) return CGCM_E_INVALID;
+  auto succ = C->reg.lower_bound(b);
+  if (succ != C->reg.end() && succ->first < b + s) return CGCM_E_OVERLAP;
+  if (succ != C->reg.begin()) {
+    auto pred = std::prev(succ);
+    if (pred->first + pred->second.size > b) return CGCM_E_OVERLAP;
+  }
+  HostUnit u;
+  u.size = s;
+  u.flags = fl;
+  u.epoch0 = C->epoch;
+  if (name) u.name = name;
+  C->reg.emplace_hint(succ, b, u);
+  C->table_dirty = true;
+  return CGCM_OK;
+}
+
+int cgcm_declareAlloc(void *base, size_t size) {
+  CTX();
+  return declare_one(C, reinterpret_cast<uint64_t>(base), size, 0, nullptr);
+}
+int cgcm_declareAllocFlags(void *base, size_t size, unsigned unit_flags) {
+  CTX();
+  return declare_one(C, reinterpret_cast<uint64_t>(base), size, (unit_flags & CGCM_UNIT_READONLY) ? UF_READONLY : 0,
+                     nullptr);
+}
+int cgcm_declareBatch(void *const *bases, const size_t *sizes, size_t n, unsigned unit_flags) {
+  CTX();
+  if (n && (!bases || !sizes)) return CGCM_E_INVALID;
+  std::vector<size_t> ord(n);
+  for (size_t i = 0; i < n; ++i) ord[i] = i;
+  auto B = [&](size_t i) { return reinterpret_cast<uint64_t>(bases[i]); };
+  std::sort(ord.begin(), ord.end(), [&](size_t a, size_t b) { return B(a) < B(b); });
+  for (size_t q = 0; q < n; ++q) {  // validate everything first (all-or-nothing)
+    uint64_t b = B(ord[q]), s = sizes[ord[q]];
+    if (b == 0 || s == 0 || b + s < b) return CGCM_E_INVALID;
+    if (q + 1 < n && b + s > B(ord[q + 1])) return CGCM_E_OVERLAP;
+    auto succ = C->reg.lower_bound(b);
+    if (succ != C->reg.end() && succ->first < b + s) return CGCM_E_OVERLAP;
+    if (succ != C->reg.begin()) {
+      auto pred = std::prev(succ);
+      if (pred->first + pred->second.size > b) return CGCM_E_OVERLAP;
+    }
+  }
+  uint32_t fl = (unit_flags & CGCM_UNIT_READONLY) ? UF_READONLY : 0;
+  auto hint = C->reg.begin();
+  for (size_t q = 0; q < n; ++q) {
+    HostUnit u;
+    u.size = sizes[ord[q]];
+    u.flags = fl;
+    u.epoch0 = C->epoch;
+    hint = C->reg.lower_bound(B(ord[q]));
+    hint = C->reg.emplace_hint(hint, B(ord[q]), u);
+  }
+  if (n) C->table_dirty = true;
+  return CGCM_OK;
+}
+int cgcm_declareGlobal(const char *name, void *base, size_t size, int isReadOnly) {
+  CTX();
+  if (!name || !*name) return CGCM_E_INVALID;
+  if (C->names.count(name)) return CGCM_E_DUPLICATE;
+  int s = declare_one(C, reinterpret_cast<uint64_t>(base), size, UF_GLOBAL | (isReadOnly ? UF_READONLY : 0), name);
+  if (s == CGCM_OK) C->names.insert(name);
+  return s;
+}
+int cgcm_undeclare(void *base) {
+  CTX();
+  uint64_t b = reinterpret_cast<uint64_t>(base);
+  auto it = C->reg.find(b);
+  if (it == C->reg.end()) return CGCM_E_UNREGISTERED;
+  HostUnit &u = it->second;
+  if (u.idx >= 0) {  // idx refers to the current device table until the next ensure_table()
+    int32_t rc = 0;
+    CK(cudaMemcpyAsync(&rc, &C->rec.as<UnitRec>()[u.idx].refcount, 4, cudaMemcpyDeviceToHost, C->main));
+    CK(cudaStreamSynchronize(C->main));
+    if (rc > 0) return CGCM_E_BUSY;
+  }
+  if (u.flags & UF_GLOBAL) {
+    C->names.erase(u.name);
+    if (u.run >= 0) C->run_release(u.run);
+  }
+  C->reg.erase(it);
+  C->table_dirty = true;
+  return CGCM_OK;
+}
+
+// ---- pinned host arena (R10 heap wrappers) ---------------------------------------------------
+void *cgcm_malloc(size_t n) {
+  Context *C = tl_ctx;
+  if (!C || n == 0) return nullptr;
+  std::lock_guard<std::recursive_mutex> lk(C->mu);
+  uint64_t len = align_up(n, 16);
+  auto pick = C->hfree.end();
+  for (auto it = C->hfree.begin(); it != C->hfree.end(); ++it)
+    if (it->second >= len) {
+      pick = it;
+      break;
+    }
+  if (pick == C->hfree.end()) {
+    size_t chunk = std::max<size_t>(align_up(len, 1 << 21), (size_t)256 << 20);
+    void *p = nullptr;
+    cudaSetDevice(C->device);
+    if (cudaHostAlloc(&p, chunk, cudaHostAllocPortable) != cudaSuccess) return nullptr;
+    C->hchunks.push_back({static_cast<char *>(p), chunk});
+    pick = C->hfree.emplace(reinterpret_cast<uint64_t>(p), chunk).first;
+  }
+  uint64_t a = pick->first, l = pick->second;
+  C->hfree.erase(pick);
+  if (l > len) C->hfree.emplace(a + len, l - len);
+  if (declare_one(C, a, n, 0, nullptr) != CGCM_OK) {
+    C->hfree.emplace(a, len);
+    return nullptr;
+  }
+  C->hallocs[a] = len;
+  return reinterpret_cast<void *>(a);
+}
+int cgcm_free(void *p) {
+  Context *C = tl_ctx;
+  if (!C) return CGCM_E_NOCTX;
+  if (!p) return CGCM_OK;
+  std::lock_guard<std::recursive_mutex> lk(C->mu);
+  uint64_t a = reinterpret_cast<uint64_t>(p);
+  auto it = C->hallocs.find(a);
+  if (it == C->hallocs.end()) return CGCM_E_INVALID;
+  int s = cgcm_undeclare(p);
+  if (s != CGCM_OK) return s;
+  uint64_t len = it->second;
+  C->hallocs.erase(it);
+  // coalesce with neighbours
+  auto nx = C->hfree.lower_bound(a);
+  if (nx != C->hfree.end() && nx->first == a + len) {
+    len += nx->second;
+    C->hfree.erase(nx);
+  }
+  auto pv = C->hfree.lower_bound(a);
+  if (pv != C->hfree.begin()) {
+    --pv;
+    if (pv->first + pv->second == a) {
+      a = pv->first;
+      len += pv->second;
+      C->hfree.erase(pv);
+    }
+  }
+  C->hfree.emplace(a, len);
+  return CGCM_OK;
+}
+
+// ---- device-resident arrays -------------------------------------------------------------------
+int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n) {
+  CTX();
+  if (n == 0) return CGCM_OK;
+  if (!d_slots || (reinterpret_cast<uint64_t>(d_slots) & 7)) return CGCM_E_INVALID;
+  CKS(C->ensure_table());
+  Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
+  return C->map_core({s}, {}, nullptr, nullptr);
+}
+
+int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
+  CTX();
+  if (n == 0) return CGCM_OK;
+  if (!d_slots || (reinterpret_cast<uint64_t>(d_slots) & 7)) return CGCM_E_INVALID;
+  Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
+  std::vector<uint32_t> copy_units, freed;
+  std::vector<Journal> jn;
+  Status res{};
+  bool rel = (flags & CGCM_RELEASE) != 0;
+  CKS(C->unmap_rev_core({s}, true, rel, copy_units, freed, jn, res));
+  int r = C->copy_back(copy_units);
+  if (r != CGCM_OK) {
+    // reverse translation of an array-mapped element failed: undo the whole call
+    SlotCall c;
+    c.dir = DIR_REV;
+    c.ops = OP_WRITE | OP_GATE | OP_HITMASK | (rel ? OP_DEC : 0);
+    c.segs = {s};
+    C->undo_rev(c, jn, true, rel);
+    return r;
+  }
+  C->st.rev_translations += res.translated;
+  if (C->flags & CGCM_LENIENT) C->st.passthrough += res.misses;
+  CKS(C->free_units(freed));
+  return CGCM_OK;
+}
+
+// ---- host-array batch forms ---------------------------------------------------------------------
+static int stage_in(Context *C, const void *const *cpu, size_t n, uint64_t &dptr) {
+  CKS(C->dalloc(C->staging, 8 * n + 64));
+  CKS(C->h_small.ensure(8 * n));
+  CK(cudaStreamSynchronize(C->main));
+  std::memcpy(C->h_small.p, cpu, 8 * n);
+  CK(cudaMemcpyAsync(C->staging.as<void>(), C->h_small.p, 8 * n, cudaMemcpyHostToDevice, C->main));
+  dptr = C->staging.addr;
+  return CGCM_OK;
+}
+
+int cgcm_mapBatch(const void *const *cpu, size_t n, void **gpu_out) {
+  CTX();
+  if (n == 0) return CGCM_OK;
+  if (!cpu || !gpu_out) return CGCM_E_INVALID;
+  CKS(C->ensure_table());
+  uint64_t d = 0;
+  CKS(stage_in(C, cpu, n, d));
+  Seg s{d, n, 0, 1, 0};
+  CKS(C->map_core({s}, {}, nullptr, nullptr));
+  CK(cudaMemcpyAsync(C->h_small.p, C->staging.as<void>(), 8 * n, cudaMemcpyDeviceToHost, C->main));
+  CK(cudaStreamSynchronize(C->main));
+  std::memcpy(gpu_out, C->h_small.p, 8 * n);
+  return CGCM_OK;
+}
+
+int cgcm_unmapBatch(const void *const *cpu, size_t n) {
+  CTX();
+  if (n == 0) return CGCM_OK;
+  if (!cpu) return CGCM_E_INVALID;
+  CKS(C->ensure_table());
+  uint64_t d = 0;
+  CKS(stage_in(C, cpu, n, d));
+  CKS(C->prepare(n + 64));
+  SlotCall c;
+  c.dir = DIR_FWD;
+  c.ops = OP_GATE | OP_CHECKMAPPED;
+  c.segs = {Seg{d, n, 0, 1, 0}};
+  CKS(C->launch(c, 0));
+  Status sts[8];
+  unsigned long long lcs[3];
+  CKS(C->fetch_status(sts, lcs));
+  std::vector<Journal> jn;
+  CKS(C->download(jn, C->journal, lcs[1]));
+  int err = CGCM_OK;
+  if (sts[0].misses && !(C->flags & CGCM_LENIENT)) err = CGCM_E_UNREGISTERED;
+  else if (sts[0].notmapped) err = CGCM_E_NOT_MAPPED;
+  std::vector<uint32_t> cu;
+  for (auto &j : jn)
+    if (j.copy) cu.push_back(j.unit);
+  std::sort(cu.begin(), cu.end());
+  if (!err) err = C->copy_back(cu);
+  if (err) {
+    SlotCall u;
+    CKS(C->undo_rev(u, jn, false, false));
+    return err;
+  }
+  return CGCM_OK;
+}
+
+int cgcm_releaseBatch(const void *const *cpu, size_t n) {
+  CTX();
+  if (n == 0) return CGCM_OK;
+  if (!cpu) return CGCM_E_INVALID;
+  CKS(C->ensure_table());
+  uint64_t d = 0;
+  CKS(stage_in(C, cpu, n, d));
+  CKS(C->prepare(n + 64));
+  SlotCall c;
+  c.dir = DIR_FWD;
+  c.ops = OP_DEC;
+  c.segs = {Seg{d, n, 0, 1, 0}};
+  CKS(C->launch(c, 0));
+  Status sts[8];
+  unsigned long long lcs[3];
+  CKS(C->fetch_status(sts, lcs));
+  int err = CGCM_OK;
+  if (sts[0].misses && !(C->flags & CGCM_LENIENT)) err = CGCM_E_UNREGISTERED;
+  else if (sts[0].underflow) err = CGCM_E_NOT_MAPPED;
+  if (err) {
+    SlotCall u;
+    u.dir = DIR_FWD;
+    u.ops = OP_INCPLAIN;
+    u.segs = c.segs;
+    CKS(C->prepare_small());
+    CKS(C->launch(u, 0));
+    CK(cudaStreamSynchronize(C->main));
+    return err;
+  }
+  std::vector<uint32_t> f;
+  CKS(C->download(f, C->free_list, lcs[2]));
+  return C->free_units(f);
+}
+
+int cgcm_map(const void *cpu, void **gpu_out) {
+  if (!gpu_out) return CGCM_E_INVALID;
+  void *out = nullptr;
+  int s = cgcm_mapBatch(&cpu, 1, &out);
+  if (s == CGCM_OK) *gpu_out = out;
+  return s;
+}
+int cgcm_unmap(const void *cpu) { return cgcm_unmapBatch(&cpu, 1); }
+int cgcm_release(const void *cpu) { return cgcm_releaseBatch(&cpu, 1); }
+
+// ---- array variants ---------------------------------------------------
+namespace {
+struct Outer {
+  int unit;
+  PointInfo info;
+  int mult;
+  int first;  // index of first appearance
+};
+int distinct_outers(const std::vector<PointInfo> &infos, std::vector<Outer> &out, std::vector<int> &which) {
+  std::unordered_map<int, int> pos;
+  which.resize(infos.size());
+  for (size_t j = 0; j < infos.size(); ++j) {
+    if (infos[j].unit < 0) return CGCM_E_UNREGISTERED;
+    auto it = pos.find(infos[j].unit);
+    if (it == pos.end()) {
+      pos[infos[j].unit] = (int)out.size();
+      which[j] = (int)out.size();
+      out.push_back({infos[j].unit, infos[j], 1, (int)j});
+    } else {
+      out[it->second].mult += 1;
+      which[j] = it->second;
+    }
+  }
+  return CGCM_OK;
+}
+}  // namespace
+
+int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
+  CTX();
+  if (k == 0) return CGCM_OK;
+  if (!arrays || !gpu_out) return CGCM_E_INVALID;
+  std::vector<PointInfo> infos;
+  CKS(C->lookup_points(reinterpret_cast<const uint64_t *>(arrays), k, infos));
+  std::vector<Outer> outs;
+  std::vector<int> which;
+  CKS(distinct_outers(infos, outs, which));
+  // prologue: activate inactive outers (raw copy of the CPU pointer array, rewritten in place),
+  // then refcount/flags of every outer -- the outer AU first (A9)
+  std::vector<uint32_t> act;
+  for (auto &o : outs)
+    if (o.info.refcount == 0) act.push_back((uint32_t)o.unit);
+  std::sort(act.begin(), act.end());
+  std::vector<std::pair<uint64_t, uint64_t>> copies;
+  CKS(C->activate_units(act, &copies));
+  std::vector<UnitOp> ops;
+  std::vector<Seg> fsegs, rsegs;
+  for (auto &o : outs) {
+    HostUnit &hu = C->by_idx[o.unit]->second;
+    ops.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)o.mult});
+    ops.push_back({(uint32_t)o.unit, UOP_OR_FLAGS, UF_ARRAYMAPPED});
+    uint64_t n = o.info.size / 8;
+    if (!n) continue;
+    Seg s{hu.devbase, n, 0, o.mult, 0};
+    if (o.info.refcount > 0 && (o.info.flags & UF_ARRAYMAPPED)) rsegs.push_back(s);  // A9: refcounts only
+    else fsegs.push_back(s);
+  }
+  // unit ops must not run before the outers' set_devbase: same stream, issued after
+  CKS(C->unit_ops(ops));
+  uint64_t tr = 0, nl = 0;
+  int r = C->map_core(fsegs, rsegs, &tr, &nl);
+  if (r != CGCM_OK) {
+    // undo the prologue
+    std::vector<UnitOp> undo;
+    for (auto &o : outs) {
+      undo.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)(-o.mult)});
+      if (!(o.info.flags & UF_ARRAYMAPPED)) undo.push_back({(uint32_t)o.unit, UOP_AND_FLAGS, ~(uint64_t)UF_ARRAYMAPPED});
+      if (o.info.refcount == 0) undo.push_back({(uint32_t)o.unit, UOP_SET_EPOCH, o.info.epoch});
+    }
+    C->unit_ops(undo);
+    cudaStreamSynchronize(C->main);
+    std::vector<uint32_t> deact;
+    for (auto &o : outs)
+      if (o.info.refcount == 0) deact.push_back((uint32_t)o.unit);
+    // free_units counts frees: compensate (these were never reported as activations)
+    uint64_t frees0 = C->st.frees;
+    C->st.activations -= act.size();
+    C->st.h2d_units -= act.size();
+    for (uint32_t x : act) C->st.h2d_bytes -= C->by_idx[x]->second.size;
+    C->free_units(deact);
+    C->st.frees = frees0;
+    return r;
+  }
+  for (auto &o : outs) C->by_idx[o.unit]->second.arrayMapped = true;
+  for (size_t j = 0; j < k; ++j) {
+    const Outer &o = outs[which[j]];
+    uint64_t dev = C->by_idx[o.unit]->second.devbase;
+    gpu_out[j] = reinterpret_cast<void **>(dev + (reinterpret_cast<uint64_t>(arrays[j]) - o.info.base));
+  }
+  return CGCM_OK;
+}
+
+int cgcm_unmapArrays(void *const *const *arrays, size_t k) {
+  CTX();
+  if (k == 0) return CGCM_OK;
+  if (!arrays) return CGCM_E_INVALID;
+  std::vector<PointInfo> infos;
+  CKS(C->lookup_points(reinterpret_cast<const uint64_t *>(arrays), k, infos));
+  std::vector<Outer> outs;
+  std::vector<int> which;
+  CKS(distinct_outers(infos, outs, which));
+  for (auto &o : outs)
+    if (o.info.refcount <= 0) return CGCM_E_NOT_MAPPED;
+  CKS(C->ensure_rev());
+  // prologue: every outer's epoch becomes current first, so that self-references and outers that
+  // are elements of other outers are not copied twice (A12)
+  std::vector<UnitOp> ops;
+  std::vector<Journal> outer_jn;
+  struct OC { int unit; uint64_t stage; };
+  std::vector<OC> outer_copies;
+  std::vector<Seg> rsegs_copy, rsegs_gate, fsegs_gate;
+  uint64_t stage_bytes = 0;
+  for (auto &o : outs) {
+    bool copy_o = o.info.epoch != C->epoch && !(o.info.flags & UF_READONLY);
+    if (o.info.epoch != C->epoch) {
+      ops.push_back({(uint32_t)o.unit, UOP_SET_EPOCH, C->epoch});
+      outer_jn.push_back({o.info.epoch, (uint32_t)o.unit, 0});
+    }
+    uint64_t n = o.info.size / 8;
+    if (copy_o) {
+      outer_copies.push_back({o.unit, 0});
+      if (o.info.flags & UF_ARRAYMAPPED) stage_bytes += align_up(8 * n, 32) + 64;
+    }
+  }
+  CKS(C->dalloc(C->staging2, stage_bytes + 256));
+  uint64_t off = C->staging2.addr;
+  for (auto &oc : outer_copies) {
+    auto &o = *std::find_if(outs.begin(), outs.end(), [&](const Outer &x) { return x.unit == oc.unit; });
+    uint64_t n = o.info.size / 8;
+    if (o.info.flags & UF_ARRAYMAPPED) {
+      off = align_up(off, 32) + (o.info.devbase & 31);
+      oc.stage = off;
+      off += 8 * n;
+    }
+  }
+  for (auto &o : outs) {
+    uint64_t n = o.info.size / 8;
+    if (!n) continue;
+    auto oc = std::find_if(outer_copies.begin(), outer_copies.end(), [&](const OC &x) { return x.unit == o.unit; });
+    if (o.info.flags & UF_ARRAYMAPPED) {
+      if (oc != outer_copies.end()) rsegs_copy.push_back(Seg{o.info.devbase, n, oc->stage, 1, 0});
+      else rsegs_gate.push_back(Seg{o.info.devbase, n, 0, 1, 0});
+    } else {
+      fsegs_gate.push_back(Seg{o.info.devbase, n, 0, 1, 0});  // raw CPU pointers (scalar-mapped outer)
+    }
+  }
+  CKS(C->unit_ops(ops));
+  uint64_t total = 0;
+  for (auto &o : outs) total += o.info.size / 8;
+  CKS(C->prepare(total + 64));
+  SlotCall A, B, F;
+  A.dir = DIR_REV; A.ops = OP_WRITE | OP_GATE | OP_HITMASK; A.segs = rsegs_copy;
+  B.dir = DIR_REV; B.ops = OP_GATE; B.segs = rsegs_gate;
+  F.dir = DIR_FWD; F.ops = OP_GATE | OP_CHECKMAPPED; F.segs = fsegs_gate;
+  CKS(C->launch(A, 0, false, false, true));
+  CKS(C->launch(B, 1));
+  CKS(C->launch(F, 2));
+  Status sts[8];
+  unsigned long long lcs[3];
+  CKS(C->fetch_status(sts, lcs));
+  std::vector<Journal> jn;
+  CKS(C->download(jn, C->journal, lcs[1]));
+  bool strict = !(C->flags & CGCM_LENIENT);
+  int err = CGCM_OK;
+  if ((sts[0].misses || sts[1].misses || sts[2].misses) && strict) err = CGCM_E_UNREGISTERED;
+  else if (sts[2].notmapped) err = CGCM_E_NOT_MAPPED;
+  std::vector<uint32_t> cu;
+  for (auto &j : jn)
+    if (j.copy) cu.push_back(j.unit);
+  std::sort(cu.begin(), cu.end());
+  if (!err) {
+    // outers first: their reverse-translated slots (staged) + trailing bytes, or raw bytes
+    err = C->copy_back(cu);  // validates array-mapped elements before moving bytes
+  }
+  if (err) {
+    std::vector<Journal> all = jn;
+    all.insert(all.end(), outer_jn.begin(), outer_jn.end());
+    SlotCall none;
+    C->undo_rev(none, all, false, false);
+    return err;
+  }
+  for (auto &oc : outer_copies) {
+    auto &o = *std::find_if(outs.begin(), outs.end(), [&](const Outer &x) { return x.unit == oc.unit; });
+    uint64_t n = o.info.size / 8;
+    if (o.info.flags & UF_ARRAYMAPPED) {
+      if (n) CK(cudaMemcpyAsync(reinterpret_cast<void *>(o.info.base), reinterpret_cast<void *>(oc.stage), 8 * n,
+                                cudaMemcpyDeviceToHost, C->main));
+      if (o.info.size > 8 * n)
+        CK(cudaMemcpyAsync(reinterpret_cast<void *>(o.info.base + 8 * n),
+                           reinterpret_cast<void *>(o.info.devbase + 8 * n), o.info.size - 8 * n,
+                           cudaMemcpyDeviceToHost, C->main));
+      C->st.d2h_memcpy_calls += 1 + (o.info.size > 8 * n);
+    } else {
+      CK(cudaMemcpyAsync(reinterpret_cast<void *>(o.info.base), reinterpret_cast<void *>(o.info.devbase), o.info.size,
+                         cudaMemcpyDeviceToHost, C->main));
+      C->st.d2h_memcpy_calls += 1;
+    }
+    C->st.d2h_units += 1;
+    C->st.d2h_bytes += o.info.size;
+  }
+  CK(cudaStreamSynchronize(C->main));
+  C->st.rev_translations += sts[0].translated;
+  if (!strict) C->st.passthrough += sts[0].misses;
+  return CGCM_OK;
+}
+
+int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
+  CTX();
+  if (k == 0) return CGCM_OK;
+  if (!arrays) return CGCM_E_INVALID;
+  std::vector<PointInfo> infos;
+  CKS(C->lookup_points(reinterpret_cast<const uint64_t *>(arrays), k, infos));
+  std::vector<Outer> outs;
+  std::vector<int> which;
+  CKS(distinct_outers(infos, outs, which));
+  for (auto &o : outs)
+    if (o.info.refcount < o.mult) return CGCM_E_NOT_MAPPED;
+  std::vector<Seg> rsegs, fsegs;
+  for (auto &o : outs) {
+    uint64_t n = o.info.size / 8;
+    if (!n) continue;
+    Seg s{o.info.devbase, n, 0, o.mult, 0};
+    ((o.info.flags & UF_ARRAYMAPPED) ? rsegs : fsegs).push_back(s);
+  }
+  if (!rsegs.empty()) CKS(C->ensure_rev());
+  // the outers' own references go first (plain decrement); slot decrements detect underflow / zero
+  std::vector<UnitOp> ops;
+  std::vector<uint32_t> outer_zero;
+  for (auto &o : outs) {
+    ops.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)(-o.mult)});
+    if (o.info.refcount == o.mult) outer_zero.push_back((uint32_t)o.unit);
+  }
+  CKS(C->unit_ops(ops));
+  uint64_t total = 0;
+  for (auto &o : outs) total += o.info.size / 8;
+  CKS(C->prepare(total + 64));
+  SlotCall R, F;
+  R.dir = DIR_REV; R.ops = OP_DEC; R.segs = rsegs;
+  F.dir = DIR_FWD; F.ops = OP_DEC; F.segs = fsegs;
+  CKS(C->launch(R, 0));
+  CKS(C->launch(F, 1));
+  Status sts[8];
+  unsigned long long lcs[3];
+  CKS(C->fetch_status(sts, lcs));
+  bool strict = !(C->flags & CGCM_LENIENT);
+  int err = CGCM_OK;
+  if ((sts[0].misses || sts[1].misses) && strict) err = CGCM_E_UNREGISTERED;
+  else if (sts[0].underflow || sts[1].underflow) err = CGCM_E_NOT_MAPPED;
+  if (err) {
+    CKS(C->prepare_small());
+    SlotCall r2, f2;
+    r2.dir = DIR_REV; r2.ops = OP_INCPLAIN; r2.segs = rsegs;
+    f2.dir = DIR_FWD; f2.ops = OP_INCPLAIN; f2.segs = fsegs;
+    CKS(C->launch(r2, 0));
+    CKS(C->launch(f2, 1));
+    std::vector<UnitOp> undo;
+    for (auto &o : outs) undo.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)o.mult});
+    CKS(C->unit_ops(undo));
+    CK(cudaStreamSynchronize(C->main));
+    return err;
+  }
+  std::vector<uint32_t> f;
+  CKS(C->download(f, C->free_list, lcs[2]));
+  // an outer reaches 0 through its own decrement only if no slot pointed into it
+  for (uint32_t x : outer_zero) f.push_back(x);
+  std::sort(f.begin(), f.end());
+  f.erase(std::unique(f.begin(), f.end()), f.end());
+  // outers whose zero came from a slot decrement are already in f; outers with remaining slot refs
+  // into them (self-reference) cannot be in outer_zero (their refcount exceeded mult)
+  return C->free_units(f);
+}
+
+int cgcm_mapArray(void *const *cpu, void ***gpu_out) {
+  if (!gpu_out) return CGCM_E_INVALID;
+  void **out = nullptr;
+  int s = cgcm_mapArrays(&cpu, 1, &out);
+  if (s == CGCM_OK) *gpu_out = out;
+  return s;
+}
+int cgcm_unmapArray(void *const *cpu) { return cgcm_unmapArrays(&cpu, 1); }
+int cgcm_releaseArray(void *const *cpu) { return cgcm_releaseArrays(&cpu, 1); }
+
+int cgcm_advanceEpoch(void) {
+  CTX();
+  C->epoch += 1;  // "increases every time the program launches a GPU function"
+  return CGCM_OK;
+}
+uint64_t cgcm_epoch(void) {
+  Context *C = tl_ctx;
+  return C ? C->epoch : 0;
+}
+
+// ---- introspection ------------------------------------------------------------------------------
+int cgcm_stats(cgcm_stats_t *out) {
+  CTX();
+  if (!out) return CGCM_E_INVALID;
+  *out = C->st;
+  return CGCM_OK;
+}
+int cgcm_resetStats(void) {
+  CTX();
+  std::memset(&C->st, 0, sizeof(C->st));
+  return CGCM_OK;
+}
+int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
+  CTX();
+  CKS(C->ensure_table());
+  if (n) *n = (size_t)C->U;
+  if (!out || cap == 0) return (size_t)C->U <= cap ? CGCM_OK : CGCM_E_NOMEM;
+  std::vector<UnitRec> recs;
+  CKS(C->download(recs, C->rec, (size_t)C->U));
+  size_t m = std::min(cap, (size_t)C->U);
+  for (size_t i = 0; i < m; ++i) {
+    const UnitRec &r = recs[i];
+    cgcm_unit_t &u = out[i];
+    u.base = C->by_idx[i]->first;
+    u.size = r.size;
+    bool act = r.refcount > 0;
+    u.devptr = (act || ((r.flags & UF_GLOBAL) && (r.flags & UF_STORAGE))) ? r.devbase : 0;
+    u.refCount = r.refcount;
+    u.epoch = r.epoch;
+    u.flags = ((r.flags & UF_GLOBAL) ? CGCM_UNIT_GLOBAL : 0) | ((r.flags & UF_READONLY) ? CGCM_UNIT_READONLY : 0) |
+              ((r.flags & UF_ARRAYMAPPED) ? CGCM_UNIT_ARRAYMAPPED : 0) | (act ? CGCM_UNIT_ACTIVE : 0);
+    u.pad = 0;
+  }
+  return (size_t)C->U <= cap ? CGCM_OK : CGCM_E_NOMEM;
+}
+int cgcm_arenaUsage(size_t *used, size_t *capacity) {
+  CTX();
+  if (used) *used = C->arena.used();
+  if (capacity) *capacity = C->arena.capacity();
+  return CGCM_OK;
+}
+
+}  // extern "C"

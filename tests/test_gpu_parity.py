@@ -1,0 +1,384 @@
+"""GPU parity tests: the CUDA path (libcgcm.so through the C ABI) against the CPU oracle, element by
+element, on seeded inputs.  Needs a B200 (run via gpurun); marked `gpu`.
+"""
+import numpy as np
+import pytest
+
+import workloads as W
+from tests.harness import Pair, HostBuf, host_read, host_write
+
+pytestmark = pytest.mark.gpu
+
+ALPHA = 0.999
+
+
+@pytest.fixture(scope="module")
+def cgcm_mod():
+    import paper_conf_pldi_jablinpjjba11_b200 as cg
+    return cg
+
+
+@pytest.fixture
+def pair(cgcm_mod):
+    from oracle import Oracle
+    ctx = cgcm_mod.Context(0, arena_bytes=1 << 30)
+    o = Oracle()
+    p = Pair(ctx, o)
+    yield p
+    ctx.close()
+    o.close()
+
+
+def test_native_library_is_loaded(cgcm_mod):
+    import os
+    maps = open("/proc/self/maps").read()
+    cgcm_mod.lib()
+    maps = open("/proc/self/maps").read()
+    assert os.path.realpath(cgcm_mod.LIB_PATH) in maps
+
+
+def test_scalar_map_unmap_release(pair):
+    P = pair
+    buf = HostBuf(1 << 16)
+    bases = [buf.addr + 0x1000 * k + 8 * k for k in range(8)]
+    for k, b in enumerate(bases):
+        assert P.declare(b, 64 + 40 * k, np.full(64 + 40 * k, k + 1, dtype=np.uint8)) == 0
+    P.check("declared")
+    for k, b in enumerate(bases):
+        for off in (0, 1, (64 + 40 * k) // 2, 64 + 40 * k):
+            P.run("map", b + off)
+    P.check("mapped")
+    P.check_device_units()
+    # GPU function writes (raw device write), launch, unmap copies once per epoch
+    for u in P.g.dump():
+        P.g.dev_write(u["devptr"], np.full(u["size"], 0xAB, dtype=np.uint8))
+        P.o.dev_write(u["devptr"], np.full(u["size"], 0xAB, dtype=np.uint8))
+    P.run("unmap", bases[0])           # no launch since map: no copy (A5 R1)
+    P.advance()
+    for b in bases:
+        P.run("unmap", b)
+        P.run("unmap", b + 3)          # same epoch: no second copy
+    P.check("unmapped")
+    for b in bases:
+        for _ in range(4):
+            P.run("release", b)
+    P.check("released")
+    P.run("release", bases[0])         # underflow -> NOT_MAPPED
+    P.run("map", 0)                    # NULL
+    P.check("end")
+    assert P.g.arenaUsage()[0] == P.g.arenaUsage()[0]
+
+
+def test_mapArray_roundtrip_permutation(pair):
+    P = pair
+    buf = HostBuf(1 << 20)
+    rows = [buf.addr + 0x800 * k for k in range(16)]
+    for k, r in enumerate(rows):
+        P.declare(r, 256, np.full(32, k + 0.5))
+    pp = buf.addr + 0x80000
+    targets = [r + 8 * (k % 5) for k, r in enumerate(rows)] + [0, rows[3]]
+    P.declare(pp, 8 * len(targets), np.asarray(targets, dtype=np.uint64))
+    st, d = P.run("mapArray", pp)
+    assert st == 0
+    P.check("mapArray")
+    P.check_device_units()
+    dev = P.g.dev_read(d, 8 * len(targets)).view(np.uint64).copy()
+    perm = np.array([5, 2, 9, 0, 1, 3, 4, 6, 7, 8, 10, 11, 12, 13, 14, 15, 16, 17])
+    P.g.dev_write(d, dev[perm])
+    P.o.dev_write(d, dev[perm])
+    P.advance()
+    P.run("unmapArray", pp)
+    P.check("unmapArray permuted")
+    got = np.frombuffer(host_read(pp, 8 * len(targets)), dtype=np.uint64)
+    assert (got == np.asarray(targets, dtype=np.uint64)[perm]).all()
+    P.g.dev_write(d, dev)
+    P.o.dev_write(d, dev)
+    P.advance()
+    P.run("unmapArray", pp)
+    P.run("releaseArray", pp)
+    P.check("released")
+    assert all(u["refCount"] == 0 for u in P.g.dump())
+
+
+def setup_A(P, nrows, ncols, seed=1):
+    """double **rows: nrows row AUs + the row-pointer AU from the pinned header-free heap."""
+    vals = W.config_A_values(nrows, ncols, seed)
+    rows = [P.malloc(8 * ncols, vals[r]) for r in range(nrows)]
+    pp = P.malloc(8 * nrows, np.asarray(rows, dtype=np.uint64))
+    return rows, pp, vals
+
+
+@pytest.mark.parametrize("promoted", [False, True])
+def test_config_A_naive_vs_promoted(pair, promoted):
+    P = pair
+    nrows = ncols = 256
+    iters = 100
+    rows, pp, vals = setup_A(P, nrows, ncols)
+    P.check("setup")
+
+    def step(d):
+        assert P.g.sample_scale(d, nrows, ncols, ALPHA) == 0
+        P.g.synchronize()
+        P.o.kernel_scale(d, nrows, ncols, ALPHA)
+        P.advance()
+
+    if not promoted:
+        for it in range(iters):
+            st, d = P.run("mapArray", pp)
+            step(d)
+            P.run("unmapArray", pp)
+            P.run("releaseArray", pp)
+            if it % 25 == 0:
+                P.check(f"iter {it}")
+    else:
+        st, d0 = P.run("mapArray", pp)
+        for it in range(iters):
+            st, d = P.run("mapArray", pp)
+            assert d == d0
+            step(d)
+            P.run("releaseArray", pp)
+            if it % 25 == 0:
+                P.check(f"iter {it}")
+        P.run("unmapArray", pp)
+        P.run("releaseArray", pp)
+    P.check("end")
+    s = P.g.stats()
+    if promoted:
+        assert (s["h2d_units"], s["h2d_bytes"], s["d2h_units"], s["d2h_bytes"]) == (257, 526336, 257, 526336)
+    else:
+        assert (s["h2d_units"], s["h2d_bytes"]) == (25700, 52633600)
+        assert (s["d2h_units"], s["d2h_bytes"]) == (25700, 52633600)
+    x = vals.copy()
+    for _ in range(iters):
+        x = x * np.float64(ALPHA)
+    got = np.stack([np.frombuffer(host_read(a, 8 * ncols), dtype=np.float64) for a in rows])
+    assert got.tobytes() == x.tobytes()
+
+
+def test_errors_leave_state_unchanged(pair):
+    P = pair
+    buf = HostBuf(1 << 16)
+    a, b = buf.addr + 0x1000, buf.addr + 0x2000
+    P.declare(a, 64, np.arange(8, dtype=np.uint64))
+    P.declare(b, 64)
+    pp = buf.addr + 0x8000
+    P.declare(pp, 24, np.array([a, b + 8, buf.addr + 0x3000], dtype=np.uint64))
+    P.run("mapArray", pp)                          # last slot unregistered
+    P.run("mapBatch", [a, a + 64, a + 65])         # past the end
+    P.run("mapBatch", [a, a + 0x800])              # gap
+    P.run("unmap", a)
+    P.run("release", a)
+    P.check("after errors")
+    P.run("map", a)
+    P.run("releaseBatch", [a, a + 8])              # second release underflows
+    P.check("after release underflow")
+    assert P.g.undeclare(a) == P.o.undeclare(a) == -5
+    assert P.g.declareAlloc(a + 0x30, 8) == -3
+    P.run("release", a)
+    host_write(pp, np.array([a, b + 8, 0], dtype=np.uint64))
+    P.sync_host_to_oracle(pp, 24)
+    P.run("mapArray", pp)
+    P.run("release", b)                            # steal the element's reference
+    P.run("releaseArray", pp)                      # underflow on b -> rolled back
+    P.check("after releaseArray underflow")
+
+
+def test_self_referential_pool(pair):
+    P = pair
+    buf = HostBuf(4096)
+    pool, n = buf.addr, 8
+    P.declare(pool, 8 * n, np.array([pool + 8 * ((k + 1) % n) for k in range(n)], dtype=np.uint64))
+    P.run("mapArray", pool)
+    P.check("mapped")
+    P.check_device_units()
+    P.advance()
+    P.run("unmapArray", pool)
+    P.check("unmapped")
+    P.run("releaseArray", pool)
+    P.check("released")
+
+
+def test_globals(pair):
+    P = pair
+    buf = HostBuf(4096)
+    P.declare_global("g_ro", buf.addr, 48, ro=True)
+    P.declare_global("g_rw", buf.addr + 256, 48)
+    for _ in range(2):
+        P.run("map", buf.addr)
+        P.run("map", buf.addr + 256)
+        P.advance()
+        P.run("unmap", buf.addr)
+        P.run("unmap", buf.addr + 256)
+        P.run("release", buf.addr)
+        P.run("release", buf.addr + 256)
+        P.check("globals cycle")
+    assert P.g.declareGlobal("g_ro", buf.addr + 1024, 8) == -6
+
+
+def config_C_setup(P, U, seed=3):
+    offs, sizes, span = W.table_layout(U, seed)
+    R = W.reserve_readonly(span)
+    bases = offs + np.uint64(R)
+    assert P.g.declareBatch(bases, sizes, readonly=True) == 0
+    for b, s in zip(bases, sizes):
+        assert P.o.declareAlloc(int(b), int(s), readonly=True) == 0
+    return offs, sizes, R, span
+
+
+@pytest.mark.parametrize("U,Q", [(1 << 12, (1 << 16) + 13), (50000, 300001)])
+def test_config_C_device_arrays(pair, U, Q):
+    """mapArrayDevice / unmapArrayDevice (+release) vs the oracle's mapSlots / unmapSlots."""
+    import torch
+    P = pair
+    offs, sizes, R, span = config_C_setup(P, U)
+    q, u = W.queries(offs, sizes, Q, 3)
+    slots = (q + np.uint64(R)).astype(np.uint64)
+    slots[::97] = 0                                        # NULL slots
+    d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+    assert P.g.mapArrayDevice(d.data_ptr(), Q) == 0
+    P.feed_replay()
+    ref = slots.copy()
+    assert P.o.mapSlots(ref) == 0
+    got = d.cpu().numpy().view(np.uint64)
+    assert (got == ref).all()
+    P.check("mapped")
+    P.advance()
+    assert P.g.unmapArrayDevice(d.data_ptr(), Q, release=True) == 0
+    assert P.o.unmapSlots(ref, release=True) == 0
+    got = d.cpu().numpy().view(np.uint64)
+    assert (got == ref).all() and (got == slots).all()
+    P.check("unmapped")
+    W.release_reservation(R, span)
+
+
+def test_config_C_device_array_errors(pair):
+    import torch
+    P = pair
+    offs, sizes, R, span = config_C_setup(P, 1000)
+    q, u = W.queries(offs, sizes, 5000, 3)
+    slots = (q + np.uint64(R)).astype(np.uint64)
+    slots[1234] = np.uint64(R) + offs[10] + sizes[10] + np.uint64(1) if offs[11] - offs[10] > sizes[10] + 1 \
+        else np.uint64(R + span + 100)
+    d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+    before = P.g.dump()
+    assert P.g.mapArrayDevice(d.data_ptr(), len(slots)) == -2
+    assert (d.cpu().numpy().view(np.uint64) == slots).all()      # in-place rewrite rolled back
+    assert P.g.dump() == before
+    W.release_reservation(R, span)
+
+
+def tree_sums(vals, N):
+    out = np.zeros(N)
+    for i in range(N - 1, -1, -1):
+        s = vals[i]
+        if 2 * i + 1 < N:
+            s = s + out[2 * i + 1]
+        if 2 * i + 2 < N:
+            s = s + out[2 * i + 2]
+        out[i] = s
+    return out
+
+
+@pytest.mark.parametrize("N", [1, 7, 1000, 1 << 14])
+def test_config_D_tree(pair, N):
+    P = pair
+    import math
+    vals = W.tree_values(N)
+    order = W.tree_alloc_order(N)
+    nodes = P.g.malloc(32 * N)
+    P.g.undeclare(nodes)
+    pos = np.empty(N, dtype=np.int64)
+    pos[order] = np.arange(N)
+    addr = np.uint64(nodes) + np.uint64(32) * pos.astype(np.uint64)
+    arena = np.zeros((N, 4), dtype=np.float64)
+    arena[:, 1] = vals[order]
+    arena.view(np.int64)[:, 0] = order
+    host_write(nodes, arena)
+    bases = [nodes + 32 * k for k in range(N)]
+    assert P.g.declareBatch(bases, [32] * N) == 0
+    for b in bases:
+        P.o.declareAlloc(b, 32)
+    P.units.update({b: 32 for b in bases})
+    P.o.host_write(nodes, arena)
+    child = W.tree_children(N)
+    table = np.where(child >= 0, addr[np.maximum(child, 0)], 0).astype(np.uint64)
+    CB = P.g.malloc(16 * N)
+    P.g.undeclare(CB)
+    P.declare(CB, 16 * N, table)
+    st, cdev = P.run("mapArray", CB)
+    st, rdev = P.run("map", int(addr[0]))
+    depth = int(math.floor(math.log2(N))) if N > 1 else 0
+    for dlev in range(depth, -1, -1):
+        lo, hi = (1 << dlev) - 1, min((1 << (dlev + 1)) - 1, N)
+        assert P.g.sample_treesum_level(cdev, rdev, N, lo, hi) == 0
+        P.g.synchronize()
+        P.o.kernel_treesum_level(cdev, rdev, N, lo, hi)
+        P.advance()
+    P.run("unmapArray", CB)
+    P.run("unmap", int(addr[0]))
+    P.run("releaseArray", CB)
+    P.run("release", int(addr[0]))
+    P.check("tree done")
+    exp = tree_sums(vals, N)
+    got = np.frombuffer(host_read(nodes, 32 * N), dtype=np.float64).reshape(N, 4)[pos, 2]
+    assert got.tobytes() == exp.tobytes()
+
+
+def test_random_stress(pair):
+    """Seeded random interleavings of declare/map/mapArray/advance/unmap/release (SURVEY §4 tier 3)."""
+    P = pair
+    rng = np.random.default_rng(7)
+    buf = HostBuf(1 << 20)
+    units = []
+    cur = buf.addr
+    for k in range(300):
+        cur += int(rng.integers(0, 3)) * 16
+        size = int(rng.integers(1, 40)) * 8
+        units.append((cur, size))
+        cur += size
+    for b, s in units:
+        P.declare(b, s, rng.integers(0, 255, s, dtype=np.uint8))
+    arrays = []
+    for j in range(6):  # pointer arrays into random units (interior, one-past-end, NULL, aliases)
+        n = int(rng.integers(1, 40))
+        tg = []
+        for _ in range(n):
+            b, s = units[int(rng.integers(0, len(units)))]
+            r = rng.random()
+            tg.append(0 if r < 0.1 else b + int(rng.integers(0, s + 1)))
+        cur = (cur + 64) // 32 * 32
+        pa = cur
+        cur += 8 * n + int(rng.integers(1, 5)) * 8
+        P.declare(pa, 8 * n, np.asarray(tg, dtype=np.uint64))
+        arrays.append(pa)
+    mapped_arrays = []
+    for step in range(400):
+        r = rng.random()
+        if r < 0.25:
+            b, s = units[int(rng.integers(0, len(units)))]
+            P.run("map", b + int(rng.integers(0, s + 1)))
+        elif r < 0.35:
+            b, s = units[int(rng.integers(0, len(units)))]
+            P.run("unmap", b)
+        elif r < 0.45:
+            b, s = units[int(rng.integers(0, len(units)))]
+            P.run("release", b)
+        elif r < 0.6:
+            pa = arrays[int(rng.integers(0, len(arrays)))]
+            st, _ = P.run("mapArray", pa)
+            if st == 0:
+                mapped_arrays.append(pa)
+        elif r < 0.7 and mapped_arrays:
+            pa = mapped_arrays[int(rng.integers(0, len(mapped_arrays)))]
+            P.run("unmapArray", pa)
+        elif r < 0.8 and mapped_arrays:
+            pa = mapped_arrays.pop(int(rng.integers(0, len(mapped_arrays))))
+            P.run("releaseArray", pa)
+        elif r < 0.9:
+            P.advance()
+        else:
+            ps = [units[int(rng.integers(0, len(units)))][0] for _ in range(int(rng.integers(1, 20)))]
+            P.run("mapBatch", ps)
+        if step % 20 == 0:
+            P.check(f"step {step}")
+    P.check("end")
