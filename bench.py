@@ -1,0 +1,402 @@
+#!/usr/bin/env python
+"""Benchmark of the CGCM hot path on B200 (the driver's contract; DESIGN.md §8 explains every key).
+
+Workload (default, BASELINE.json configs[4] "E"): an allocation table of 2^22 units (sizes
+log-uniform 16 B-64 KiB, gaps 0-4080 B, in a PROT_READ reservation, declared read-only and kept
+active by one setup map each) and 2^28 interior CPU pointers in 256 pointer arrays of 2^20 slots;
+rank r of N translates arrays [r*256/N, (r+1)*256/N) against its own replica of the table.
+`--config C` runs configs[2] (2^20 units, 2^26 pointers) instead.
+
+One step = one pass of the whole hot path over the rank's batch, through the C ABI:
+  cgcm_mapArrayDevice   a1 lookup + a2 forward rewrite in place + per-slot refcount (Alg. 1)
+  cgcm_advanceEpoch     one GPU function launch happened
+  cgcm_unmapArrayDevice a1 reverse lookup + a3 reverse rewrite in place + a4 epoch gate of every AU
+                        touched (Alg. 2; read-only units: no copy) + release of every slot (Alg. 3)
+`value` = pointer translations per second (2 per slot per step: forward and reverse), inputs resident
+in HBM; `e2e` = the same metric through cgcm_mapArrays/unmapArrays/releaseArrays on the pointer arrays
+in pinned host memory (host<->device copies of the arrays inside the timed region).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+CONFIGS = {
+    "E": dict(U=1 << 22, arrays=256, slots=1 << 20, seed=5, name="E: 2^28 interior pointers in 256 arrays, "
+              "replicated 2^22-unit table"),
+    "C": dict(U=1 << 20, arrays=64, slots=1 << 20, seed=3, name="C: 2^26 interior pointers, 2^20-unit table"),
+    "T": dict(U=1 << 12, arrays=8, slots=1 << 12, seed=3, name="T: tiny debug configuration"),
+}
+METRIC = "translated pointers/sec and map+unmap GB/s per B200 (and 8-GPU), % of HBM roofline"
+BYTES_PER_TRANSLATION = 16  # 8 B read + 8 B write of the pointer slot
+
+
+def env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f), "measured"
+    return {"hbm_gbs": 6650.0}, "fallback"
+
+
+def start_clock_sampler(uuid: str | None):
+    cmd = ["nvidia-smi", "--query-gpu=uuid,clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
+           "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+           "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+           "--format=csv,noheader,nounits", "-lms", "100"]
+    if uuid:
+        cmd[1:1] = ["-i", uuid]
+    try:
+        return subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+    except Exception:
+        return None
+
+
+def stop_clock_sampler(p):
+    if p is None:
+        return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+    p.terminate()
+    try:
+        out, _ = p.communicate(timeout=5)
+    except Exception:
+        p.kill()
+        out = ""
+    sm, mx, reasons = [], [], set()
+    names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+    for line in out.strip().splitlines():
+        f = [x.strip() for x in line.split(",")]
+        if len(f) < 8:
+            continue
+        try:
+            sm.append(float(f[1]))
+            mx.append(float(f[2]))
+        except ValueError:
+            continue
+        for n, v in zip(names, f[4:8]):
+            if v.lower().startswith("active"):
+                reasons.add(n)
+    return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+            "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------------------------------------
+# the workload
+# ---------------------------------------------------------------------------------------------
+class Workload:
+    def __init__(self, cfg, rank, world):
+        self.cfg = cfg
+        self.U = cfg["U"]
+        self.seed = cfg["seed"]
+        self.offs, self.sizes, self.span = W.table_layout(self.U, self.seed)
+        self.R = W.reserve_readonly(self.span)
+        self.bases = self.offs + np.uint64(self.R)
+        A = cfg["arrays"]
+        assert A % world == 0, "arrays must divide evenly across ranks"
+        self.arrays_per_rank = A // world
+        self.slots = cfg["slots"]
+        self.first_array = rank * self.arrays_per_rank
+        self.n = self.arrays_per_rank * self.slots
+        self.start = self.first_array * self.slots  # query index of this rank's first slot
+
+    def device_queries(self, device):
+        import torch
+        ot = torch.from_numpy(self.offs.view(np.int64)).to(device)
+        st = torch.from_numpy(self.sizes.view(np.int64)).to(device)
+        q, _ = W.queries_t(ot, st, self.n, self.seed, start=self.start)
+        q += self.R
+        return q
+
+    def host_sample(self, n):
+        q, _ = W.queries(self.offs, self.sizes, n, self.seed, start=self.start)
+        return (q + np.uint64(self.R)).astype(np.uint64)
+
+
+def run_cgcm(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_pldi_jablinpjjba11_b200 as cg
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    cfg = CONFIGS[args.config]
+    t0 = time.time()
+    wl = Workload(cfg, rank, world)
+    total_bytes = int(wl.sizes.sum())
+    arena = total_bytes + wl.span // 8 + wl.n * 8 * 2 + (6 << 30)
+    ctx = cg.Context(local_rank, arena_bytes=arena, flags=cg.PROFILE)
+    assert ctx.declareBatch(wl.bases, wl.sizes, readonly=True) == 0
+    # one reference per unit held for the whole run (map promotion of the table's maps)
+    pins = torch.from_numpy(wl.bases.view(np.int64).copy()).to(dev)
+    s = ctx.mapArrayDevice(pins.data_ptr(), wl.U)
+    assert s == 0, cg.strerror(s)
+    setup_act_s = time.time() - t0
+    q = wl.device_queries(dev)
+    q_ref = q.clone()
+    torch.cuda.synchronize()
+    setup_s = time.time() - t0
+
+    def step():
+        s1 = ctx.mapArrayDevice(q.data_ptr(), wl.n)
+        ctx.advanceEpoch()
+        s2 = ctx.unmapArrayDevice(q.data_ptr(), wl.n, release=True)
+        if s1 or s2:
+            raise RuntimeError(f"step failed: {cg.strerror(s1)} / {cg.strerror(s2)}")
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    assert torch.equal(q, q_ref), "round trip changed the pointer arrays"
+
+    uuid = None
+    try:
+        uuid = str(torch.cuda.get_device_properties(dev).uuid)
+        if uuid and not uuid.startswith("GPU-"):
+            uuid = "GPU-" + uuid
+    except Exception:
+        uuid = None
+    sampler = start_clock_sampler(uuid)
+    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    ctx.resetStats()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(ctx.main)
+    for _ in range(args.steps):
+        step()
+    ev1.record(ctx.main)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = stop_clock_sampler(sampler)
+    ms = ev0.elapsed_time(ev1)
+    st = ctx.stats()
+    assert torch.equal(q, q_ref), "round trip changed the pointer arrays"
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    ms_per_step = ms / args.steps
+    translations = 2 * wl.n * world * args.steps
+    value = translations / (ms / 1e3)
+
+    # roofline of the dominant kernel (per-launch event times on the launch stream)
+    peaks, peak_kind = measured_peaks()
+    fwd_ms = st["fwd_kernel_ms"] / max(1, st["fwd_kernel_calls"])
+    rev_ms = st["rev_kernel_ms"] / max(1, st["rev_kernel_calls"])
+    fwd_slots = st["fwd_kernel_slots"] / max(1, st["fwd_kernel_calls"])
+    rev_slots = st["rev_kernel_slots"] / max(1, st["rev_kernel_calls"])
+    dom = "rev" if rev_ms >= fwd_ms else "fwd"
+    kms, kslots = (rev_ms, rev_slots) if dom == "rev" else (fwd_ms, fwd_slots)
+    achieved = BYTES_PER_TRANSLATION * kslots / (kms / 1e3) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(prof):
+        try:
+            with open(prof) as f:
+                traffic = json.load(f).get(args.config, {}).get(dom)
+        except Exception:
+            traffic = None
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": traffic,
+                "kernel": f"k_slots<{'DIR_REV' if dom == 'rev' else 'DIR_FWD'}> ({dom})",
+                "peak_source": peak_kind,
+                "fwd_ms_per_launch": round(fwd_ms, 4), "rev_ms_per_launch": round(rev_ms, 4),
+                "fwd_gbs": round(BYTES_PER_TRANSLATION * fwd_slots / (fwd_ms / 1e3) / 1e9, 1) if fwd_ms else None,
+                "rev_gbs": round(BYTES_PER_TRANSLATION * rev_slots / (rev_ms / 1e3) / 1e9, 1) if rev_ms else None}
+    gpu_launches = int(st["kernel_launches"])
+
+    e2e = None
+    if not args.no_e2e:
+        e2e = run_e2e(args, ctx, wl, q_ref, dev, world, rank)
+
+    result = {
+        "metric": METRIC, "value": round(value, 1), "unit": "pointer translations/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u64",
+        "data": "synthetic (seeded splitmix64; PROT_READ zero-page table, interior pointers)",
+        "config": {"workload": cfg["name"], "units": wl.U, "pointers_per_step": wl.n * world,
+                   "pointers_per_rank": wl.n, "arrays": cfg["arrays"], "parallelism": f"replicated table, "
+                   f"{cfg['arrays'] // world} arrays per rank", "l2": "inputs (2 GiB/GPU of pointer slots at E) "
+                   "exceed L2 between iterations; table stays L2-resident by design",
+                   "translations_per_step": 2 * wl.n * world},
+        "roofline": roofline, "gpu_launches": gpu_launches, "clocks": clocks, "e2e": e2e,
+        "setup_s": round(setup_s, 1), "setup_activation_s": round(setup_act_s, 1),
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        result["cpu_baseline"] = cpu_baseline(wl, args.cpu_sample, steps=1)
+    ctx.close()
+    return result
+
+
+def run_e2e(args, ctx, wl, q_ref, dev, world, rank):
+    """Same metric through the host-array public API: cgcm_mapArrays / unmapArrays / releaseArrays on
+    the rank's pointer arrays in pinned host memory (raw arrays H2D, translated in place, reverse
+    translated and copied back every step)."""
+    import ctypes
+    import torch
+    A, S = wl.arrays_per_rank, wl.slots
+    host = np.ascontiguousarray(q_ref.cpu().numpy().view(np.uint64))
+    outers = []
+    for a in range(A):
+        p = ctx.malloc(8 * S)
+        if not p:
+            return {"value": None, "error": "cgcm_malloc failed"}
+        ctypes.memmove(p, host[a * S:(a + 1) * S].ctypes.data, 8 * S)
+        outers.append(p)
+
+    def step():
+        s1, _ = ctx.mapArrays(outers)
+        ctx.advanceEpoch()
+        s2 = ctx.unmapArrays(outers)
+        s3 = ctx.releaseArrays(outers)
+        if s1 or s2 or s3:
+            raise RuntimeError(f"e2e step failed {s1} {s2} {s3}: {ctx.L.cgcm_lastCudaError().decode()}")
+
+    step()
+    torch.cuda.synchronize()
+    steps = max(1, min(args.steps, args.e2e_steps))
+    st0 = ctx.stats()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(ctx.main)
+    for _ in range(steps):
+        step()
+    ev1.record(ctx.main)
+    torch.cuda.synchronize()
+    ms = ev0.elapsed_time(ev1)
+    st1 = ctx.stats()
+    ok = all(np.array_equal(np.ctypeslib.as_array((ctypes.c_uint64 * S).from_address(p)), host[a * S:(a + 1) * S])
+             for a, p in enumerate(outers))
+    for p in outers:
+        ctx.free(p)
+    if world > 1:
+        import torch.distributed as dist
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    return {"value": round(2 * wl.n * world * steps / (ms / 1e3), 1), "unit": "pointer translations/s",
+            "h2d_bytes_per_step": (st1["h2d_bytes"] - st0["h2d_bytes"]) // steps,
+            "d2h_bytes_per_step": (st1["d2h_bytes"] - st0["d2h_bytes"]) // steps,
+            "ms_per_step": round(ms / steps, 3), "steps": steps,
+            "api": "cgcm_mapArrays+advanceEpoch+cgcm_unmapArrays+cgcm_releaseArrays (pinned host arrays)",
+            "host_arrays_roundtrip_ok": bool(ok)}
+
+
+# ---------------------------------------------------------------------------------------------
+# CPU oracle timing (the cpu_baseline leg and the --impl reference arm)
+# ---------------------------------------------------------------------------------------------
+def oracle_setup(wl):
+    from oracle import Oracle
+    o = Oracle()
+    for b, s in zip(wl.bases.tolist(), wl.sizes.tolist()):
+        assert o.declareAlloc(b, s, readonly=True) == 0
+    pins = wl.bases.astype(np.uint64).copy()
+    assert o.mapSlots(pins) == 0     # the same setup references the GPU run holds
+    return o
+
+
+def oracle_step(o, slots):
+    s = slots.copy()
+    t0 = time.perf_counter()
+    assert o.mapSlots(s) == 0
+    o.advanceEpoch()
+    assert o.unmapSlots(s, release=True) == 0
+    return time.perf_counter() - t0, s
+
+
+def cpu_baseline(wl, sample, steps=1, o=None):
+    o = o or oracle_setup(wl)
+    slots = wl.host_sample(sample)
+    best = None
+    for _ in range(steps):
+        dt, s = oracle_step(o, slots)
+        assert (s == slots).all()
+        best = dt if best is None else min(best, dt)
+    o.close()
+    return {"value": round(2 * sample / best, 1), "unit": "pointer translations/s", "cores": 1, "kind": "oracle",
+            "sample": f"first {sample} slots of rank 0's arrays (same table, same setup references): "
+                      f"mapSlots + advanceEpoch + unmapSlots(release), single-threaded C++ std::map oracle",
+            "seconds": round(best, 3)}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return None
+    cfg = CONFIGS[args.config]
+    wl = Workload(cfg, 0, 1)
+    o = oracle_setup(wl)
+    slots = wl.host_sample(args.ref_sample)
+    for _ in range(args.warmup):
+        oracle_step(o, slots)
+    total = 0.0
+    for _ in range(args.steps):
+        dt, s = oracle_step(o, slots)
+        total += dt
+    o.close()
+    value = 2 * args.ref_sample * args.steps / total
+    cpu = {"value": round(value, 1), "unit": "pointer translations/s", "cores": 1, "kind": "oracle",
+           "sample": f"{args.ref_sample} slots per step of rank 0's arrays against the full table"}
+    return {"impl": "reference", "metric": METRIC, "value": round(value, 1), "unit": "pointer translations/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(total / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u64", "data": "synthetic", "config": {"workload": cfg["name"],
+            "units": wl.U, "pointers_per_step": args.ref_sample, "parallelism": "single core"},
+            "cpu_baseline": cpu, "e2e": {"value": round(value, 1), "unit": "pointer translations/s",
+                                         "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="cgcm", choices=["cgcm", "reference"])
+    ap.add_argument("--config", default="E", choices=sorted(CONFIGS))
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample", type=int, default=1 << 21)
+    ap.add_argument("--ref-sample", type=int, default=1 << 19)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    rank, world, local_rank = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
+    if args.impl == "reference":
+        res = run_reference(args, rank, world)
+        if res is not None:
+            print(json.dumps(res), flush=True)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    res = run_cgcm(args, rank, world, local_rank)
+    if rank == 0:
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

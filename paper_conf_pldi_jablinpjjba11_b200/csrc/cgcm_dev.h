@@ -113,9 +113,10 @@ struct SlotArgs {
   uint8_t *hitmask;            // [nchunks], bit m = slot m of the chunk was translated
   uint64_t epoch;
   Status *st;
-  unsigned long long *lc;      // shared list counters of the call: [0] act, [1] journal, [2] free
+  unsigned long long *lc;      // shared list counters of the call: [0] act, [1] journal, [2] free, [3] copy
   uint32_t *act_list;
-  Journal *journal;
+  Journal *journal;            // every epoch this call changed (rollback)
+  uint32_t *copy_list;         // units that need a copy-back (stale, not read-only)
   uint32_t *free_list;
   int lenient;
   int smem_top;                // capacity of the shared-memory splitter array

@@ -317,13 +317,16 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
       }
       if (OPS & OP_GATE) {
         unsigned long long ix = warp_append(&a.lc[1], gated);
+        const bool cp = gated && !(fl & UF_READONLY);  // Alg. 2: stale and not read-only
         if (gated) {
           Journal jn;
           jn.old_epoch = old_ep;
           jn.unit = (uint32_t)unit[m];
-          jn.copy = (fl & UF_READONLY) ? 0u : 1u;
+          jn.copy = cp ? 1u : 0u;
           a.journal[ix] = jn;
         }
+        unsigned long long cx = warp_append(&a.lc[3], cp);
+        if (cp) a.copy_list[cx] = (uint32_t)unit[m];
       }
     }
     if (OPS & OP_WRITE) {
@@ -394,6 +397,7 @@ static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
   }
   uint64_t want = (a.nchunks + SLOT_THREADS - 1) / SLOT_THREADS;
   int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
+  (void)cudaGetLastError();
   k_slots<DIR, OPS><<<grid, SLOT_THREADS, smem, s>>>(a);
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
@@ -449,11 +453,13 @@ __global__ void k_build_level(const uint64_t *keys, const int *meta, const uint3
 void launch_build_index(const uint64_t *keys, const int *n_dev, int n_cap, uint64_t *top, uint32_t *wide,
                         uint32_t *const *lvl, const size_t *lvl_cap, int *meta, cudaStream_t s) {
   cudaMemsetAsync(wide, 0, 4 * ((TOPMAX + 31) / 32), s);
+  (void)cudaGetLastError();
   k_build_top<<<(TOPMAX + 255) / 256, 256, 0, s>>>(keys, n_dev, top, wide, meta);
   for (int k = 0; k < MAXL; ++k) {
     if (!lvl[k] || lvl_cap[k] == 0) continue;
     int64_t cnt = ((int64_t)n_cap + (1ll << (3 * k)) - 1) >> (3 * k);
     int grid = (int)std::min<int64_t>((cnt + 255) / 256 + 1, 4096);
+    (void)cudaGetLastError();
     k_build_level<<<grid, 256, 0, s>>>(keys, meta, wide, k, lvl[k], lvl_cap[k]);
   }
 }
@@ -478,7 +484,10 @@ __global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *size, con
 }
 void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags, const uint64_t *epoch0,
                   const UnitRec *old_rec, UnitRec *new_rec, cudaStream_t s) {
-  if (n > 0) k_remap<<<(n + 255) / 256, 256, 0, s>>>(n, old_idx, size, flags, epoch0, old_rec, new_rec);
+  if (n > 0) {
+    (void)cudaGetLastError();
+    k_remap<<<(n + 255) / 256, 256, 0, s>>>(n, old_idx, size, flags, epoch0, old_rec, new_rec);
+  }
 }
 
 // reverse index: key = devbase of active units (refcount > 0), inactive sorted to the end
@@ -493,7 +502,10 @@ __global__ void k_rev_collect(const UnitRec *rec, int n, uint64_t *keys, uint32_
 }
 void launch_rev_collect(const UnitRec *rec, int n, uint64_t *keys, uint32_t *vals, int *count, cudaStream_t s) {
   cudaMemsetAsync(count, 0, sizeof(int), s);
-  if (n > 0) k_rev_collect<<<(n + 255) / 256, 256, 0, s>>>(rec, n, keys, vals, count);
+  if (n > 0) {
+    (void)cudaGetLastError();
+    k_rev_collect<<<(n + 255) / 256, 256, 0, s>>>(rec, n, keys, vals, count);
+  }
 }
 __global__ void k_rev_payload(const uint32_t *units, const uint64_t *base, const int *n_dev, int n_cap, RevRec *rev) {
   int j = blockIdx.x * blockDim.x + threadIdx.x;
@@ -506,7 +518,10 @@ __global__ void k_rev_payload(const uint32_t *units, const uint64_t *base, const
 }
 void launch_rev_payload(const uint32_t *units, const uint64_t *base, const int *n_dev, int n_cap, RevRec *rev,
                         cudaStream_t s) {
-  if (n_cap > 0) k_rev_payload<<<(n_cap + 255) / 256, 256, 0, s>>>(units, base, n_dev, n_cap, rev);
+  if (n_cap > 0) {
+    (void)cudaGetLastError();
+    k_rev_payload<<<(n_cap + 255) / 256, 256, 0, s>>>(units, base, n_dev, n_cap, rev);
+  }
 }
 
 size_t sort_pairs_temp_bytes(int n) {
@@ -546,7 +561,10 @@ __global__ void k_unit_ops(const UnitOp *ops, int n, UnitRec *rec) {
   }
 }
 void launch_unit_ops(const UnitOp *ops, int n, UnitRec *rec, cudaStream_t s) {
-  if (n > 0) k_unit_ops<<<(n + 255) / 256, 256, 0, s>>>(ops, n, rec);
+  if (n > 0) {
+    (void)cudaGetLastError();
+    k_unit_ops<<<(n + 255) / 256, 256, 0, s>>>(ops, n, rec);
+  }
 }
 
 __global__ void k_set_devbase(const uint32_t *units, const uint64_t *devbases, int n, UnitRec *rec, uint64_t epoch,
@@ -560,7 +578,10 @@ __global__ void k_set_devbase(const uint32_t *units, const uint64_t *devbases, i
 }
 void launch_set_devbase(const uint32_t *units, const uint64_t *devbases, int n, UnitRec *rec, uint64_t epoch,
                         int set_epoch, cudaStream_t s) {
-  if (n > 0) k_set_devbase<<<(n + 255) / 256, 256, 0, s>>>(units, devbases, n, rec, epoch, set_epoch);
+  if (n > 0) {
+    (void)cudaGetLastError();
+    k_set_devbase<<<(n + 255) / 256, 256, 0, s>>>(units, devbases, n, rec, epoch, set_epoch);
+  }
 }
 
 __global__ void k_deactivate(const uint32_t *units, int n, UnitRec *rec) {
@@ -576,7 +597,10 @@ __global__ void k_deactivate(const uint32_t *units, int n, UnitRec *rec) {
   }
 }
 void launch_deactivate(const uint32_t *units, int n, UnitRec *rec, cudaStream_t s) {
-  if (n > 0) k_deactivate<<<(n + 255) / 256, 256, 0, s>>>(units, n, rec);
+  if (n > 0) {
+    (void)cudaGetLastError();
+    k_deactivate<<<(n + 255) / 256, 256, 0, s>>>(units, n, rec);
+  }
 }
 
 __global__ void k_restore_epochs(const Journal *j, int n, UnitRec *rec) {
@@ -585,7 +609,10 @@ __global__ void k_restore_epochs(const Journal *j, int n, UnitRec *rec) {
   rec[j[i].unit].epoch = j[i].old_epoch;
 }
 void launch_restore_epochs(const Journal *j, int n, UnitRec *rec, cudaStream_t s) {
-  if (n > 0) k_restore_epochs<<<(n + 255) / 256, 256, 0, s>>>(j, n, rec);
+  if (n > 0) {
+    (void)cudaGetLastError();
+    k_restore_epochs<<<(n + 255) / 256, 256, 0, s>>>(j, n, rec);
+  }
 }
 
 // outer-pointer lookup for mapArray/unmapArray/releaseArray: one thread per pointer, plain
@@ -623,7 +650,10 @@ __global__ void k_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t 
 }
 void launch_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t *ptrs, int n, PointInfo *out,
                           cudaStream_t s) {
-  if (n > 0) k_lookup_points<<<(n + 127) / 128, 128, 0, s>>>(ix, rec, ptrs, n, out);
+  if (n > 0) {
+    (void)cudaGetLastError();
+    k_lookup_points<<<(n + 127) / 128, 128, 0, s>>>(ix, rec, ptrs, n, out);
+  }
 }
 
 }  // namespace cgcm

@@ -13,6 +13,7 @@
 #include <cstring>
 #include <map>
 #include <mutex>
+#include <thread>
 #include <string>
 #include <unordered_map>
 #include <unordered_set>
@@ -29,7 +30,8 @@ thread_local std::string g_last_cuda_error;
   do {                                                                               \
     cudaError_t e_ = (x);                                                            \
     if (e_ != cudaSuccess) {                                                         \
-      g_last_cuda_error = std::string(#x) + ": " + cudaGetErrorString(e_);           \
+      g_last_cuda_error = std::string(#x) + " (runtime.cpp:" + std::to_string(__LINE__) + "): " + \
+                          cudaGetErrorString(e_);                                    \
       return CGCM_E_CUDA;                                                            \
     }                                                                                \
   } while (0)
@@ -198,10 +200,11 @@ struct Context {
   size_t rev_temp_bytes = 0;
 
   // scratch
-  DevBuf status, lc, hitmask, act_list, journal, free_list, segs, seg0, staging, staging2, points, ptrs, temp;
+  DevBuf status, lc, hitmask, act_list, journal, free_list, copy_list, segs, seg0, staging, staging2, staging_cb, points, ptrs, temp;
   DevBuf up_units, up_vals, uops;
-  HostBuf h_small, h_status, h_list;
-  cudaEvent_t ev_copy = nullptr, ev_t0 = nullptr, ev_t1 = nullptr;
+  HostBuf h_small, h_status, h_list, h_pack[2];
+  int pack_k = 0;
+  cudaEvent_t ev_copy = nullptr, ev_t0 = nullptr, ev_t1 = nullptr, ev_pack[2] = {nullptr, nullptr};
 
   // runs of device extents
   std::vector<Run> runs;
@@ -334,7 +337,7 @@ struct Context {
       CKS(dalloc(tmp2, (size_t)n * 8 + 256));
       CK(cudaMemcpyAsync(tmp2.as<void>(), ho, (size_t)n * 8, cudaMemcpyHostToDevice, main));
       const uint64_t *dsize = tmp.as<uint64_t>();
-      const uint64_t *depoch = dsize + 2 * (size_t)n;
+      const uint64_t *depoch = dsize + (size_t)n;
       const int32_t *dold = tmp2.as<int32_t>();
       const uint32_t *dflags = reinterpret_cast<const uint32_t *>(dold + n);
       launch_remap(n, dold, dsize, dflags, depoch, rec.as<UnitRec>(), nrec.as<UnitRec>(), main);
@@ -441,13 +444,14 @@ struct Context {
     a.lc = lc.as<unsigned long long>();
     a.act_list = act_list.as<uint32_t>();
     a.journal = journal.as<Journal>();
+    a.copy_list = copy_list.as<uint32_t>();
     a.free_list = free_list.as<uint32_t>();
     a.lenient = (flags & CGCM_LENIENT) ? 1 : 0;
     bool timed = (flags & CGCM_PROFILE) && (timed_fwd || timed_rev);
     if (timed) CK(cudaEventRecord(ev_t0, main));
     int r = launch_slots(c.dir, c.ops, a, nsm, main);
-    if (r == -2) {
-      g_last_cuda_error = "unsupported slot-kernel operation set";
+    if (r != 0) {
+      g_last_cuda_error = r == -2 ? "unsupported slot-kernel operation set" : "k_slots launch failed";
       return CGCM_E_CUDA;
     }
     CK(cudaGetLastError());
@@ -480,6 +484,7 @@ struct Context {
     int cap = list_capacity();
     CKS(dalloc(act_list, 4 * (size_t)cap + 64));
     CKS(dalloc(free_list, 4 * (size_t)cap + 64));
+    CKS(dalloc(copy_list, 4 * (size_t)cap + 64));
     CKS(dalloc(journal, sizeof(Journal) * (size_t)cap + 64));
     CK(cudaMemsetAsync(status.as<void>(), 0, sizeof(Status) * 8, main));
     CK(cudaMemsetAsync(lc.as<void>(), 0, 64, main));
@@ -487,12 +492,12 @@ struct Context {
     return CGCM_OK;
   }
   // fetch the 8 Status blocks + list counters (synchronizes main)
-  int fetch_status(Status out[8], unsigned long long lcs[3]) {
+  int fetch_status(Status out[8], unsigned long long lcs[4]) {
     CK(cudaMemcpyAsync(h_status.p, status.as<void>(), sizeof(Status) * 8, cudaMemcpyDeviceToHost, main));
-    CK(cudaMemcpyAsync(h_status.as<char>() + sizeof(Status) * 8, lc.as<void>(), 24, cudaMemcpyDeviceToHost, main));
+    CK(cudaMemcpyAsync(h_status.as<char>() + sizeof(Status) * 8, lc.as<void>(), 32, cudaMemcpyDeviceToHost, main));
     CK(cudaStreamSynchronize(main));
     std::memcpy(out, h_status.p, sizeof(Status) * 8);
-    std::memcpy(lcs, h_status.as<char>() + sizeof(Status) * 8, 24);
+    std::memcpy(lcs, h_status.as<char>() + sizeof(Status) * 8, 32);
     return CGCM_OK;
   }
 
@@ -554,91 +559,212 @@ struct Context {
   int activate_units(const std::vector<uint32_t> &units, std::vector<std::pair<uint64_t, uint64_t>> *h2d_out) {
     if (units.empty()) return CGCM_OK;
     std::vector<uint64_t> devbases(units.size());
-    struct Copy { uint64_t dst, src, len; };
-    std::vector<Copy> copies;
-    std::vector<int64_t> new_runs;
-    size_t i = 0;
-    uint64_t bytes = 0;
-    while (i < units.size()) {
-      HostUnit &u0 = by_idx[units[i]]->second;
-      uint64_t b0 = by_idx[units[i]]->first;
-      if (u0.flags & UF_GLOBAL) {
-        if (u0.run < 0) {  // named region: allocated once, persists (A14)
-          uint64_t need = (b0 % 256) + u0.size + 1;
-          uint64_t a = arena.alloc(need);
-          if (!a) goto nomem;
-          u0.run = new_run(a, need);
-          runs[u0.run].live = 1;
-          u0.devbase = a + (b0 % 256);
-          new_runs.push_back(u0.run);
-        }
-        devbases[i] = u0.devbase;
-        copies.push_back({u0.devbase, b0, u0.size});
-        bytes += u0.size;
+    // 1) host-contiguous runs of index-consecutive, host-adjacent, non-global units
+    struct HRun { size_t i, j; uint64_t b0, end; bool global; };
+    std::vector<HRun> hr;
+    for (size_t i = 0; i < units.size();) {
+      auto it0 = by_idx[units[i]];
+      uint64_t b0 = it0->first;
+      if (it0->second.flags & UF_GLOBAL) {
+        hr.push_back({i, i + 1, b0, b0 + it0->second.size, true});
         ++i;
         continue;
       }
-      // maximal run of index-consecutive, host-adjacent, non-global units
       size_t j = i + 1;
-      uint64_t end = b0 + u0.size;
+      uint64_t end = b0 + it0->second.size;
       while (j < units.size() && units[j] == units[j - 1] + 1) {
         auto it = by_idx[units[j]];
         if ((it->second.flags & UF_GLOBAL) || it->first != end) break;
         end += it->second.size;
         ++j;
       }
-      uint64_t need = (b0 % 256) + (end - b0) + 1;  // +1: device copies never adjacent (A7)
-      uint64_t a = arena.alloc(need);
-      if (!a) goto nomem;
-      int64_t rid = new_run(a, need);
-      new_runs.push_back(rid);
-      uint64_t d0 = a + (b0 % 256);
-      for (size_t q = i; q < j; ++q) {
-        auto it = by_idx[units[q]];
-        it->second.devbase = d0 + (it->first - b0);
-        it->second.run = rid;
-        runs[rid].live += 1;
-        devbases[q] = it->second.devbase;
-      }
-      copies.push_back({d0, b0, end - b0});
-      bytes += end - b0;
+      hr.push_back({i, j, b0, end, false});
       i = j;
     }
+    // 2) device placement.  A run keeps its host layout (devptr == base mod 256, host-adjacent units
+    //    stay adjacent) and is followed by >= 1 byte of slack so that copies of units that are not
+    //    host-adjacent are never device-adjacent (A7).  Large runs get their own extent and a direct
+    //    copy; small runs are packed into shared extents, gathered on the host into pinned staging
+    //    and sent with one DMA per pack (the transfer scheduler's coalescing for scattered AUs).
+    const uint64_t PACK_MIN = 256ull << 10, PACK_BYTES = 64ull << 20;
+    struct Ext { int64_t run; uint64_t addr, bytes; bool packed; std::vector<size_t> hruns; std::vector<uint64_t> off; };
+    std::vector<Ext> ext;
+    std::vector<char> fresh_run;  // indexed by run id: created by this call
+    auto mark_new = [&](int64_t r) {
+      if ((size_t)r >= fresh_run.size()) fresh_run.resize(r + 1, 0);
+      fresh_run[r] = 1;
+    };
+    uint64_t bytes = 0;
     {
-      CKS(upload(up_units, units));
-      CKS(upload(up_vals, devbases));
-      launch_set_devbase(up_units.as<uint32_t>(), up_vals.as<uint64_t>(), (int)units.size(), rec.as<UnitRec>(), epoch,
-                         (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
-      st.kernel_launches += 1;
-      CK(cudaGetLastError());
-      for (auto &c : copies) {
-        CK(cudaMemcpyAsync(reinterpret_cast<void *>(c.dst), reinterpret_cast<const void *>(c.src), c.len,
-                           cudaMemcpyHostToDevice, copy));
-        if (h2d_out) h2d_out->push_back({c.dst, c.len});
+      Ext cur;
+      cur.packed = true;
+      cur.run = -1;
+      cur.bytes = 0;
+      auto flush = [&]() {
+        if (!cur.hruns.empty()) ext.push_back(cur);
+        cur = Ext();
+        cur.packed = true;
+        cur.run = -1;
+        cur.bytes = 0;
+      };
+      for (size_t r = 0; r < hr.size(); ++r) {
+        HRun &h = hr[r];
+        uint64_t len = h.end - h.b0;
+        bytes += len;
+        if (h.global) {
+          HostUnit &u = by_idx[units[h.i]]->second;
+          if (u.run >= 0) {  // named region allocated on an earlier activation (A14)
+            devbases[h.i] = u.devbase;
+            Ext e;
+            e.run = u.run; e.addr = u.devbase - (h.b0 % 256); e.bytes = 0; e.packed = false;
+            e.hruns = {r}; e.off = {h.b0 % 256};
+            ext.push_back(e);
+            continue;
+          }
+        }
+        if (len >= PACK_MIN || h.global) {
+          Ext e;
+          e.run = -1; e.packed = false; e.bytes = (h.b0 % 256) + len + 1;
+          e.hruns = {r}; e.off = {h.b0 % 256};
+          ext.push_back(e);
+          continue;
+        }
+        uint64_t o = cur.bytes ? cur.bytes : 0;
+        o += ((h.b0 % 256) + 256 - (o % 256)) % 256;
+        if (o + len + 1 > PACK_BYTES && !cur.hruns.empty()) {
+          flush();
+          o = h.b0 % 256;
+        }
+        cur.hruns.push_back(r);
+        cur.off.push_back(o);
+        cur.bytes = o + len + 1;
       }
-      CK(cudaEventRecord(ev_copy, copy));
-      CK(cudaStreamWaitEvent(main, ev_copy, 0));
-      st.h2d_memcpy_calls += copies.size();
-      st.h2d_units += units.size();
-      st.h2d_bytes += bytes;
-      st.activations += units.size();
-      rev_dirty = true;
+      flush();
+    }
+    // 3) allocate extents
+    for (auto &e : ext) {
+      if (e.run >= 0) continue;  // existing global region
+      uint64_t a = arena.alloc(e.bytes);
+      if (!a) {
+        for (auto &f : ext)
+          if (f.run >= 0 && (size_t)f.run < fresh_run.size() && fresh_run[f.run]) {
+            arena.free(runs[f.run].addr, runs[f.run].bytes);
+            runs[f.run] = Run();
+            free_runs.push_back(f.run);
+          }
+        for (size_t q = 0; q < units.size(); ++q) {
+          HostUnit &u = by_idx[units[q]]->second;
+          if (u.run >= 0 && (size_t)u.run < fresh_run.size() && fresh_run[u.run]) {
+            u.run = -1;
+            u.devbase = 0;
+          }
+        }
+        return CGCM_E_NOMEM;
+      }
+      e.addr = a;
+      e.run = new_run(a, e.bytes);
+      mark_new(e.run);
+      for (size_t k = 0; k < e.hruns.size(); ++k) {
+        HRun &h = hr[e.hruns[k]];
+        uint64_t d0 = a + e.off[k];
+        for (size_t q = h.i; q < h.j; ++q) {
+          auto it = by_idx[units[q]];
+          it->second.devbase = d0 + (it->first - h.b0);
+          it->second.run = e.run;
+          runs[e.run].live += 1;
+          devbases[q] = it->second.devbase;
+        }
+      }
+    }
+    // 4) devbase (+ epoch, A5 R1) on the device, then the copies on the side stream
+    CKS(upload(up_units, units));
+    CKS(upload(up_vals, devbases));
+    launch_set_devbase(up_units.as<uint32_t>(), up_vals.as<uint64_t>(), (int)units.size(), rec.as<UnitRec>(), epoch,
+                       (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(ev_copy, main));  // copies may overwrite nothing the main stream still reads
+    CK(cudaStreamWaitEvent(copy, ev_copy, 0));
+    for (auto &e : ext) {
+      if (!e.packed) {
+        HRun &h = hr[e.hruns[0]];
+        CKS(copy_run(e.addr + e.off[0], h.b0, h.end - h.b0, true, units, h.i, h.j, copy));
+        if (h2d_out) h2d_out->push_back({e.addr + e.off[0], h.end - h.b0});
+        continue;
+      }
+      int k = pack_k;
+      pack_k ^= 1;
+      CK(cudaEventSynchronize(ev_pack[k]));  // the staging buffer's previous DMA is done
+      CKS(h_pack[k].ensure(e.bytes));
+      char *stg = h_pack[k].as<char>();
+      gather(e, hr, stg);
+      CK(cudaMemcpyAsync(reinterpret_cast<void *>(e.addr), stg, e.bytes, cudaMemcpyHostToDevice, copy));
+      CK(cudaEventRecord(ev_pack[k], copy));
+      st.h2d_memcpy_calls += 1;
+      if (h2d_out) h2d_out->push_back({e.addr, e.bytes});
+    }
+    CK(cudaEventRecord(ev_copy, copy));
+    CK(cudaStreamWaitEvent(main, ev_copy, 0));
+    st.h2d_units += units.size();
+    st.h2d_bytes += bytes;
+    st.activations += units.size();
+    rev_dirty = true;
+    return CGCM_OK;
+  }
+  template <class E, class H>
+  void gather(const E &e, const std::vector<H> &hr, char *stg) {
+    uint64_t total = 0;
+    for (size_t k = 0; k < e.hruns.size(); ++k) total += hr[e.hruns[k]].end - hr[e.hruns[k]].b0;
+    unsigned T = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+    if (total < (8ull << 20) || T == 1) {
+      for (size_t k = 0; k < e.hruns.size(); ++k) {
+        const H &h = hr[e.hruns[k]];
+        std::memcpy(stg + e.off[k], reinterpret_cast<const void *>(h.b0), h.end - h.b0);
+      }
+      return;
+    }
+    std::vector<std::thread> th;
+    size_t n = e.hruns.size();
+    for (unsigned t = 0; t < T; ++t) {
+      size_t lo = n * t / T, hi = n * (t + 1) / T;
+      th.emplace_back([&, lo, hi] {
+        for (size_t k = lo; k < hi; ++k) {
+          const H &h = hr[e.hruns[k]];
+          std::memcpy(stg + e.off[k], reinterpret_cast<const void *>(h.b0), h.end - h.b0);
+        }
+      });
+    }
+    for (auto &x : th) x.join();
+  }
+
+  // One host<->device copy of a host-contiguous run of units.  Host-adjacent units may live in two
+  // different host allocations (cudaMemcpyAsync rejects a pinned range that crosses them): retry
+  // unit by unit then.
+  int copy_run(uint64_t dev, uint64_t host, uint64_t len, bool h2d, const std::vector<uint32_t> &units, size_t i,
+               size_t j, cudaStream_t s) {
+    cudaError_t e = h2d ? cudaMemcpyAsync(reinterpret_cast<void *>(dev), reinterpret_cast<const void *>(host), len,
+                                          cudaMemcpyHostToDevice, s)
+                        : cudaMemcpyAsync(reinterpret_cast<void *>(host), reinterpret_cast<const void *>(dev), len,
+                                          cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) {
+      (h2d ? st.h2d_memcpy_calls : st.d2h_memcpy_calls) += 1;
       return CGCM_OK;
     }
-  nomem:
-    for (int64_t r : new_runs) {
-      arena.free(runs[r].addr, runs[r].bytes);
-      runs[r] = Run();
-      free_runs.push_back(r);
+    if (e != cudaErrorInvalidValue || j - i < 2) {
+      g_last_cuda_error = std::string("cudaMemcpyAsync (run): ") + cudaGetErrorString(e);
+      return CGCM_E_CUDA;
     }
-    for (size_t q = 0; q < units.size(); ++q) {
-      HostUnit &u = by_idx[units[q]]->second;
-      if (std::find(new_runs.begin(), new_runs.end(), u.run) != new_runs.end()) {
-        u.run = -1;
-        u.devbase = 0;
-      }
+    (void)cudaGetLastError();
+    for (size_t q = i; q < j; ++q) {
+      auto it = by_idx[units[q]];
+      uint64_t hb = it->first, n = it->second.size, db = dev + (hb - host);
+      if (h2d) CK(cudaMemcpyAsync(reinterpret_cast<void *>(db), reinterpret_cast<const void *>(hb), n,
+                                  cudaMemcpyHostToDevice, s));
+      else CK(cudaMemcpyAsync(reinterpret_cast<void *>(hb), reinterpret_cast<const void *>(db), n,
+                              cudaMemcpyDeviceToHost, s));
+      (h2d ? st.h2d_memcpy_calls : st.d2h_memcpy_calls) += 1;
     }
-    return CGCM_E_NOMEM;
+    return CGCM_OK;
   }
 
   // units whose refcount reached 0: free device storage (globals keep theirs), clear flags
@@ -668,16 +794,16 @@ struct Context {
     if (units.empty()) return CGCM_OK;
     std::vector<uint32_t> plain, arr;
     for (uint32_t x : units) (by_idx[x]->second.arrayMapped ? arr : plain).push_back(x);
-    // reverse-translate the array-mapped ones into staging2
+    // reverse-translate the array-mapped ones into staging_cb
     uint64_t arr_bytes = 0;
     for (uint32_t x : arr) arr_bytes += align_up(by_idx[x]->second.size / 8 * 8, 32) + 32;
     if (!arr.empty()) {
       CKS(ensure_rev());
-      CKS(dalloc(staging2, arr_bytes + 256));
+      CKS(dalloc(staging_cb, arr_bytes + 256));
       SlotCall c;
       c.dir = DIR_REV;
       c.ops = OP_WRITE;
-      uint64_t off = staging2.addr;
+      uint64_t off = staging_cb.addr;
       std::vector<uint64_t> dst(arr.size());
       for (size_t q = 0; q < arr.size(); ++q) {
         HostUnit &u = by_idx[arr[q]]->second;
@@ -696,7 +822,7 @@ struct Context {
       CKS(prepare_small());
       CKS(launch(c, 7));
       Status sts[8];
-      unsigned long long lcs[3];
+      unsigned long long lcs[4];
       CKS(fetch_status(sts, lcs));
       if (sts[7].misses && !(flags & CGCM_LENIENT)) return CGCM_E_UNREGISTERED;
       st.rev_translations += sts[7].translated;
@@ -731,9 +857,7 @@ struct Context {
         st.d2h_bytes += it->second.size;
         ++j;
       }
-      CK(cudaMemcpyAsync(reinterpret_cast<void *>(h0), reinterpret_cast<void *>(d0), hend - h0,
-                         cudaMemcpyDeviceToHost, copy));
-      st.d2h_memcpy_calls += 1;
+      CKS(copy_run(d0, h0, hend - h0, false, plain, i, j, copy));
       i = j;
     }
     CK(cudaStreamSynchronize(copy));
@@ -747,6 +871,7 @@ struct Context {
     int cap = list_capacity();
     CKS(dalloc(act_list, 4 * (size_t)cap + 64));
     CKS(dalloc(free_list, 4 * (size_t)cap + 64));
+    CKS(dalloc(copy_list, 4 * (size_t)cap + 64));
     CKS(dalloc(journal, sizeof(Journal) * (size_t)cap + 64));
     return CGCM_OK;
   }
@@ -773,7 +898,7 @@ struct Context {
     // hitmask is per launch: the REV pass does not use it
     if (!rsegs.empty()) CKS(launch(R, 1));
     Status sts[8];
-    unsigned long long lcs[3];
+    unsigned long long lcs[4];
     CKS(fetch_status(sts, lcs));
     bool strict = !(flags & CGCM_LENIENT);
     if ((sts[0].misses || sts[1].misses) && strict) {
@@ -805,6 +930,37 @@ struct Context {
     if (!strict) st.passthrough += sts[0].misses + sts[1].misses;
     if (translated_out) *translated_out = tr;
     if (nulls_out) *nulls_out = sts[0].nulls + sts[1].nulls;
+    return CGCM_OK;
+  }
+  // re-map of array-mapped outers (A9): +inc per non-null slot through the reverse index.  On a
+  // reverse miss (an element lost its device copy: unbalanced release) the pass is undone and
+  // E_UNREGISTERED returned so that the caller can re-translate those outers from host memory.
+  int rev_addref(const std::vector<Seg> &rsegs, Status &res) {
+    CKS(ensure_rev());
+    CKS(prepare(64));
+    SlotCall R;
+    R.dir = DIR_REV;
+    R.ops = OP_INCPLAIN;
+    R.segs = rsegs;
+    CKS(launch(R, 0));
+    Status sts[8];
+    unsigned long long lcs[4];
+    CKS(fetch_status(sts, lcs));
+    res = sts[0];
+    if (sts[0].misses && !(flags & CGCM_LENIENT)) {
+      CKS(rev_decref(rsegs));
+      return CGCM_E_UNREGISTERED;
+    }
+    return CGCM_OK;
+  }
+  int rev_decref(const std::vector<Seg> &rsegs) {
+    CKS(prepare_small());
+    SlotCall R;
+    R.dir = DIR_REV;
+    R.ops = OP_DECPLAIN;
+    R.segs = rsegs;
+    CKS(launch(R, 1));
+    CK(cudaStreamSynchronize(main));
     return CGCM_OK;
   }
   int undo_map(SlotCall &F, SlotCall &R) {
@@ -841,7 +997,7 @@ struct Context {
   // reverse unmap over device slot segments (GPU pointers): a3 + a4 (+ release)
   //   ops: OP_WRITE|OP_GATE|OP_HITMASK [|OP_DEC] or OP_GATE
   int unmap_rev_core(const std::vector<Seg> &segs, bool write, bool dec, std::vector<uint32_t> &copy_units,
-                     std::vector<uint32_t> &freed, std::vector<Journal> &journal_out, Status &res) {
+                     std::vector<uint32_t> &freed, uint64_t &journal_count, Status &res) {
     CKS(ensure_rev());
     uint64_t total = 0;
     for (auto &s : segs) total += s.n;
@@ -849,27 +1005,22 @@ struct Context {
     SlotCall c;
     c.dir = DIR_REV;
     c.ops = write ? (OP_WRITE | OP_GATE | OP_HITMASK | (dec ? OP_DEC : 0)) : (OP_GATE | (dec ? OP_DEC : 0));
-    if (!write && dec) c.ops = OP_GATE | OP_DEC;
     c.segs = segs;
     CKS(launch(c, 0, false, false, true));
     Status sts[8];
-    unsigned long long lcs[3];
+    unsigned long long lcs[4];
     CKS(fetch_status(sts, lcs));
     res = sts[0];
-    std::vector<Journal> jn;
-    CKS(download(jn, journal, lcs[1]));
+    journal_count = lcs[1];
     bool strict = !(flags & CGCM_LENIENT);
     int err = CGCM_OK;
     if (sts[0].misses && strict) err = CGCM_E_UNREGISTERED;
     else if (sts[0].underflow) err = CGCM_E_NOT_MAPPED;
     if (err) {
-      CKS(undo_rev(c, jn, write, dec));
+      CKS(undo_rev(c, lcs[1], {}, write, dec));
       return err;
     }
-    journal_out = jn;
-    for (auto &j : jn)
-      if (j.copy) copy_units.push_back(j.unit);
-    std::sort(copy_units.begin(), copy_units.end());
+    CKS(sorted_units(copy_list, lcs[3], copy_units));
     if (dec && lcs[2]) {
       std::vector<uint32_t> f;
       CKS(download(f, free_list, lcs[2]));
@@ -877,13 +1028,19 @@ struct Context {
     }
     return CGCM_OK;
   }
-  int undo_rev(SlotCall &c, const std::vector<Journal> &jn, bool write, bool dec) {
+  // undo of a gate/reverse pass: epochs from the device journal (+ host-side extra entries), then
+  // the slot side (re-translate in-place writes, re-add released references)
+  int undo_rev(SlotCall &c, uint64_t journal_count, const std::vector<Journal> &extra, bool write, bool dec) {
+    if (journal_count) {
+      launch_restore_epochs(journal.as<Journal>(), (int)journal_count, rec.as<UnitRec>(), main);
+      st.kernel_launches += 1;
+      CK(cudaGetLastError());
+    }
     CKS(prepare_small());
-    if (!jn.empty()) {
-      std::vector<Journal> j2 = jn;
+    if (!extra.empty()) {
       DevBuf jb;
-      CKS(upload(jb, j2));
-      launch_restore_epochs(jb.as<Journal>(), (int)j2.size(), rec.as<UnitRec>(), main);
+      CKS(upload(jb, extra));
+      launch_restore_epochs(jb.as<Journal>(), (int)extra.size(), rec.as<UnitRec>(), main);
       st.kernel_launches += 1;
       CK(cudaStreamSynchronize(main));
       dfree(jb);
@@ -987,6 +1144,8 @@ int cgcm_init(int device, void *dev_arena, size_t arena_bytes, void *main_stream
     C->copy = reinterpret_cast<cudaStream_t>(copy_stream);
   }
   cudaEventCreateWithFlags(&C->ev_copy, cudaEventDisableTiming);
+  cudaEventCreateWithFlags(&C->ev_pack[0], cudaEventDisableTiming);
+  cudaEventCreateWithFlags(&C->ev_pack[1], cudaEventDisableTiming);
   cudaEventCreate(&C->ev_t0);
   cudaEventCreate(&C->ev_t1);
   {
@@ -1013,6 +1172,10 @@ int cgcm_finalize(void) {
   if (C->h_status.p) cudaFreeHost(C->h_status.p);
   if (C->h_list.p) cudaFreeHost(C->h_list.p);
   cudaEventDestroy(C->ev_copy);
+  cudaEventDestroy(C->ev_pack[0]);
+  cudaEventDestroy(C->ev_pack[1]);
+  for (auto &hp : C->h_pack)
+    if (hp.p) cudaFreeHost(hp.p);
   cudaEventDestroy(C->ev_t0);
   cudaEventDestroy(C->ev_t1);
   if (C->own_streams) {
@@ -1198,10 +1361,10 @@ int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
   if (!d_slots || (reinterpret_cast<uint64_t>(d_slots) & 7)) return CGCM_E_INVALID;
   Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
   std::vector<uint32_t> copy_units, freed;
-  std::vector<Journal> jn;
+  uint64_t jcount = 0;
   Status res{};
   bool rel = (flags & CGCM_RELEASE) != 0;
-  CKS(C->unmap_rev_core({s}, true, rel, copy_units, freed, jn, res));
+  CKS(C->unmap_rev_core({s}, true, rel, copy_units, freed, jcount, res));
   int r = C->copy_back(copy_units);
   if (r != CGCM_OK) {
     // reverse translation of an array-mapped element failed: undo the whole call
@@ -1209,7 +1372,7 @@ int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
     c.dir = DIR_REV;
     c.ops = OP_WRITE | OP_GATE | OP_HITMASK | (rel ? OP_DEC : 0);
     c.segs = {s};
-    C->undo_rev(c, jn, true, rel);
+    C->undo_rev(c, jcount, {}, true, rel);
     return r;
   }
   C->st.rev_translations += res.translated;
@@ -1258,21 +1421,17 @@ int cgcm_unmapBatch(const void *const *cpu, size_t n) {
   c.segs = {Seg{d, n, 0, 1, 0}};
   CKS(C->launch(c, 0));
   Status sts[8];
-  unsigned long long lcs[3];
+  unsigned long long lcs[4];
   CKS(C->fetch_status(sts, lcs));
-  std::vector<Journal> jn;
-  CKS(C->download(jn, C->journal, lcs[1]));
   int err = CGCM_OK;
   if (sts[0].misses && !(C->flags & CGCM_LENIENT)) err = CGCM_E_UNREGISTERED;
   else if (sts[0].notmapped) err = CGCM_E_NOT_MAPPED;
   std::vector<uint32_t> cu;
-  for (auto &j : jn)
-    if (j.copy) cu.push_back(j.unit);
-  std::sort(cu.begin(), cu.end());
+  if (!err) err = C->sorted_units(C->copy_list, lcs[3], cu);
   if (!err) err = C->copy_back(cu);
   if (err) {
     SlotCall u;
-    CKS(C->undo_rev(u, jn, false, false));
+    CKS(C->undo_rev(u, lcs[1], {}, false, false));
     return err;
   }
   return CGCM_OK;
@@ -1292,7 +1451,7 @@ int cgcm_releaseBatch(const void *const *cpu, size_t n) {
   c.segs = {Seg{d, n, 0, 1, 0}};
   CKS(C->launch(c, 0));
   Status sts[8];
-  unsigned long long lcs[3];
+  unsigned long long lcs[4];
   CKS(C->fetch_status(sts, lcs));
   int err = CGCM_OK;
   if (sts[0].misses && !(C->flags & CGCM_LENIENT)) err = CGCM_E_UNREGISTERED;
@@ -1380,10 +1539,7 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
   }
   // unit ops must not run before the outers' set_devbase: same stream, issued after
   CKS(C->unit_ops(ops));
-  uint64_t tr = 0, nl = 0;
-  int r = C->map_core(fsegs, rsegs, &tr, &nl);
-  if (r != CGCM_OK) {
-    // undo the prologue
+  auto undo_prologue = [&]() {
     std::vector<UnitOp> undo;
     for (auto &o : outs) {
       undo.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)(-o.mult)});
@@ -1395,14 +1551,64 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
     std::vector<uint32_t> deact;
     for (auto &o : outs)
       if (o.info.refcount == 0) deact.push_back((uint32_t)o.unit);
-    // free_units counts frees: compensate (these were never reported as activations)
+    // these activations are withdrawn, not reported
     uint64_t frees0 = C->st.frees;
     C->st.activations -= act.size();
     C->st.h2d_units -= act.size();
     for (uint32_t x : act) C->st.h2d_bytes -= C->by_idx[x]->second.size;
     C->free_units(deact);
     C->st.frees = frees0;
+  };
+  // array-mapped outers: refcounts through the reverse index (no copy); if an element
+  // lost its device copy, re-translate the outer from its host slots instead (oracle semantics)
+  Status rres{};
+  bool rev_done = false;
+  struct Backup { uint64_t src, dst, n; };
+  std::vector<Backup> backups;
+  if (!rsegs.empty()) {
+    int r = C->rev_addref(rsegs, rres);
+    if (r == CGCM_OK) {
+      rev_done = true;
+    } else if (r == CGCM_E_UNREGISTERED) {
+      // keep the current device slots so that a failing call can put them back (all-or-nothing)
+      uint64_t bytes = 0;
+      for (auto &sg : rsegs) bytes += 8 * sg.n + 32;
+      CKS(C->dalloc(C->staging2, bytes + 256));
+      uint64_t off = C->staging2.addr;
+      for (auto &sg : rsegs) {
+        CK(cudaMemcpyAsync(reinterpret_cast<void *>(off), reinterpret_cast<void *>(sg.ptr), 8 * sg.n,
+                           cudaMemcpyDeviceToDevice, C->main));
+        backups.push_back({off, sg.ptr, 8 * sg.n});
+        off += 8 * sg.n + 32;
+      }
+      for (auto &sg : rsegs) {
+        for (auto &o : outs)
+          if (C->by_idx[o.unit]->second.devbase == sg.ptr) {
+            CK(cudaMemcpyAsync(reinterpret_cast<void *>(sg.ptr), reinterpret_cast<const void *>(o.info.base),
+                               8 * sg.n, cudaMemcpyHostToDevice, C->main));
+            C->st.h2d_memcpy_calls += 1;
+          }
+        fsegs.push_back(sg);
+      }
+    } else {
+      undo_prologue();
+      return r;
+    }
+  }
+  uint64_t tr = 0, nl = 0;
+  int r = C->map_core(fsegs, {}, &tr, &nl);
+  if (r != CGCM_OK) {
+    if (rev_done) C->rev_decref(rsegs);
+    for (auto &b : backups)
+      cudaMemcpyAsync(reinterpret_cast<void *>(b.dst), reinterpret_cast<void *>(b.src), b.n, cudaMemcpyDeviceToDevice,
+                      C->main);
+    undo_prologue();
     return r;
+  }
+  if (rev_done) {
+    C->st.fwd_translations += rres.hits;
+    C->st.null_slots += rres.nulls;
+    if (C->flags & CGCM_LENIENT) C->st.passthrough += rres.misses;
   }
   for (auto &o : outs) C->by_idx[o.unit]->second.arrayMapped = true;
   for (size_t j = 0; j < k; ++j) {
@@ -1479,27 +1685,20 @@ int cgcm_unmapArrays(void *const *const *arrays, size_t k) {
   CKS(C->launch(B, 1));
   CKS(C->launch(F, 2));
   Status sts[8];
-  unsigned long long lcs[3];
+  unsigned long long lcs[4];
   CKS(C->fetch_status(sts, lcs));
-  std::vector<Journal> jn;
-  CKS(C->download(jn, C->journal, lcs[1]));
   bool strict = !(C->flags & CGCM_LENIENT);
   int err = CGCM_OK;
-  if ((sts[0].misses || sts[1].misses || sts[2].misses) && strict) err = CGCM_E_UNREGISTERED;
-  else if (sts[2].notmapped) err = CGCM_E_NOT_MAPPED;
+  if ((sts[0].misses || sts[2].misses) && strict) err = CGCM_E_UNREGISTERED;
+  else if (sts[2].notmapped || (sts[1].misses && strict)) err = CGCM_E_NOT_MAPPED;
   std::vector<uint32_t> cu;
-  for (auto &j : jn)
-    if (j.copy) cu.push_back(j.unit);
-  std::sort(cu.begin(), cu.end());
-  if (!err) {
-    // outers first: their reverse-translated slots (staged) + trailing bytes, or raw bytes
-    err = C->copy_back(cu);  // validates array-mapped elements before moving bytes
-  }
+  if (!err) err = C->sorted_units(C->copy_list, lcs[3], cu);
+  // element copy-backs (array-mapped elements are reverse translated and validated first, into
+  // their own staging buffer); the outers' staged slots are copied below
+  if (!err) err = C->copy_back(cu);
   if (err) {
-    std::vector<Journal> all = jn;
-    all.insert(all.end(), outer_jn.begin(), outer_jn.end());
     SlotCall none;
-    C->undo_rev(none, all, false, false);
+    C->undo_rev(none, lcs[1], outer_jn, false, false);
     return err;
   }
   for (auto &oc : outer_copies) {
@@ -1563,12 +1762,12 @@ int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
   CKS(C->launch(R, 0));
   CKS(C->launch(F, 1));
   Status sts[8];
-  unsigned long long lcs[3];
+  unsigned long long lcs[4];
   CKS(C->fetch_status(sts, lcs));
   bool strict = !(C->flags & CGCM_LENIENT);
   int err = CGCM_OK;
-  if ((sts[0].misses || sts[1].misses) && strict) err = CGCM_E_UNREGISTERED;
-  else if (sts[0].underflow || sts[1].underflow) err = CGCM_E_NOT_MAPPED;
+  if (sts[1].misses && strict) err = CGCM_E_UNREGISTERED;
+  else if (sts[0].underflow || sts[1].underflow || (sts[0].misses && strict)) err = CGCM_E_NOT_MAPPED;
   if (err) {
     CKS(C->prepare_small());
     SlotCall r2, f2;

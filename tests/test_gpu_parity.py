@@ -352,17 +352,27 @@ def test_random_stress(pair):
         P.declare(pa, 8 * n, np.asarray(tg, dtype=np.uint64))
         arrays.append(pa)
     mapped_arrays = []
+    own = {}   # scalar references this test took (releases stay balanced, as compiler-inserted calls are)
     for step in range(400):
         r = rng.random()
         if r < 0.25:
             b, s = units[int(rng.integers(0, len(units)))]
-            P.run("map", b + int(rng.integers(0, s + 1)))
+            st, _ = P.run("map", b + int(rng.integers(0, s + 1)))
+            if st == 0:
+                own[b] = own.get(b, 0) + 1
         elif r < 0.35:
             b, s = units[int(rng.integers(0, len(units)))]
             P.run("unmap", b)
         elif r < 0.45:
-            b, s = units[int(rng.integers(0, len(units)))]
-            P.run("release", b)
+            held = [b for b, c in own.items() if c > 0]
+            if held:
+                b = held[int(rng.integers(0, len(held)))]
+                P.run("release", b + 1 if dict(units)[b] > 1 else b)
+                own[b] -= 1
+            else:
+                b, s = units[int(rng.integers(0, len(units)))]
+                if P.o.dump and all(u["refCount"] == 0 for u in P.o.dump() if u["base"] == b):
+                    P.run("release", b)   # never mapped: NOT_MAPPED on both sides
         elif r < 0.6:
             pa = arrays[int(rng.integers(0, len(arrays)))]
             st, _ = P.run("mapArray", pa)

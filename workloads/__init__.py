@@ -132,3 +132,55 @@ def tree_values(N: int, seed: int = 4) -> np.ndarray:
 def tree_alloc_order(N: int, seed: int = 4) -> np.ndarray:
     """Seeded permutation: position k of the node arena holds node tree_alloc_order[k]."""
     return permutation(seed, 41, N)
+
+
+# ---------------------------------------------------------------------------------------------
+# The same generator on torch tensors (any device), for inputs too large to build in numpy
+# (config E's 2^28 pointers).  int64 arithmetic wraps like u64; shifts are made logical.
+# tests/test_workloads.py checks it equals the numpy version bit for bit.
+# ---------------------------------------------------------------------------------------------
+def _s64(x: int) -> int:
+    x &= 0xFFFFFFFFFFFFFFFF
+    return x - (1 << 64) if x >= (1 << 63) else x
+
+
+def _srl(t, k: int):
+    return (t >> k) & ((1 << (64 - k)) - 1)
+
+
+def splitmix64_t(seed: int, idx):
+    """splitmix64 over an int64 tensor of indices (bit-identical to splitmix64)."""
+    z = (idx + 1) * _s64(0x9E3779B97F4A7C15) + _s64(seed)
+    z = (z ^ _srl(z, 30)) * _s64(0xBF58476D1CE4E5B9)
+    z = (z ^ _srl(z, 27)) * _s64(0x94D049BB133111EB)
+    return z ^ _srl(z, 31)
+
+
+def u01_t(seed: int, stream: int, idx):
+    r = splitmix64_t(key(seed, stream), idx)
+    return _srl(r, 11).double() * (1.0 / 9007199254740992.0)
+
+
+def randint_t(seed: int, stream: int, idx, n):
+    import torch
+    u = u01_t(seed, stream, idx)
+    nn = n.double() if torch.is_tensor(n) else float(n)
+    v = torch.floor(u * nn).long()
+    return torch.minimum(v, (n - 1) if torch.is_tensor(n) else torch.full_like(v, n - 1))
+
+
+def queries_t(offsets_t, sizes_t, n: int, seed: int, stream: int = 3, start: int = 0, chunk: int = 1 << 24):
+    """Torch version of queries(): returns (offsets int64 tensor, unit int64 tensor) on offsets_t.device."""
+    import torch
+    dev = offsets_t.device
+    outq = torch.empty(n, dtype=torch.int64, device=dev)
+    outu = torch.empty(n, dtype=torch.int64, device=dev)
+    U = offsets_t.numel()
+    for c0 in range(0, n, chunk):
+        c1 = min(n, c0 + chunk)
+        idx = torch.arange(start + c0, start + c1, dtype=torch.int64, device=dev)
+        u = randint_t(seed, stream, idx, U)
+        off = randint_t(seed, stream + 1000, idx, sizes_t[u])
+        outq[c0:c1] = offsets_t[u] + off
+        outu[c0:c1] = u
+    return outq, outu
