@@ -8,47 +8,58 @@
 namespace cgcm {
 
 // Allocation-unit record (D3): one 32-byte sector per unit, indexed by the unit's rank
-// in base order.  size/devbase drive translation, epoch the copy-back gate (Alg. 2), refcount
-// Alg. 1/3.  devbase != 0 <=> the unit has device storage (active, or a global's named region).
+// in base order.  The first 16 bytes are everything a forward translation needs (one 16-byte
+// gather): size, the unit's flags in the size word's top byte, and the device base.
+//   szf     = size (bits 0..55) | flags (bits 56..63)
+//   devbase = device copy (valid iff UF_STORAGE)
+//   epoch   = Alg. 2's per-unit epoch
+//   refcount (Alg. 1/3)
 struct __align__(32) UnitRec {
-  uint64_t size;
+  uint64_t szf;
   uint64_t devbase;
   uint64_t epoch;
   int32_t refcount;
-  uint32_t flags;
+  uint32_t pad;
 };
 static_assert(sizeof(UnitRec) == 32, "UnitRec must be one sector");
 
 enum : uint32_t {
-  UF_GLOBAL = 1u,
-  UF_READONLY = 2u,
-  UF_ARRAYMAPPED = 4u,
-  UF_ACTIVE = 8u,   // only in dumps
-  UF_STORAGE = 16u  // devbase valid
+  UF_GLOBAL = 1u,       // declareGlobal: named region persists (A14)
+  UF_READONLY = 2u,     // never copied back (Alg. 2)
+  UF_ARRAYMAPPED = 4u,  // device copy holds translated pointers (A12)
+  UF_ACTIVE = 8u,       // refcount > 0 at the start of the current call (stable during a call)
+  UF_STORAGE = 16u      // devbase valid
 };
+constexpr int FSHIFT = 56;
+constexpr uint64_t SIZE_MASK = (1ull << FSHIFT) - 1;
+constexpr uint64_t MAX_UNIT_SIZE = SIZE_MASK;
+__host__ __device__ __forceinline__ uint64_t rec_size(uint64_t szf) { return szf & SIZE_MASK; }
+__host__ __device__ __forceinline__ uint32_t rec_flags(uint64_t szf) { return (uint32_t)(szf >> FSHIFT); }
 
-// Sorted-key search index ("device-resident sorted interval array with a shared-memory-staged
-// top-level search index", north_star).  Keys are sorted u64 (AU bases for the forward index,
-// device bases of active AUs for the reverse index).
-//   top[t]  = keys[t * 8^h]                      (u64, staged in shared memory by every CTA)
-//   lvl[k][j] = keys[j * 8^k] - top[bucket]      (u32, groups of 8 = one 32-byte sector)
-//   wide bit t: bucket t spans >= 2^32-1 bytes -> binary search over keys[] instead
-// A lookup costs the shared-memory search + h sector loads (+ the record sector).
+// Sorted-key search index, built by the host (top level, directory) and the device (levels):
+//   keys      n sorted u64 (AU bases for the forward index, extent device starts for the reverse)
+//   top[t]    keys[t * 8^h], t < ntop <= TOPMAX        -- staged in shared memory by every CTA
+//   dir/seg   radix directory over top[]: the keys are split into segments at gaps >= 2^32;
+//             segment s covers top[t0_s, tend_s) and has nb_s buckets of width 2^shift_s;
+//             dir[off_s + d] = first t with top[t] >= kmin_s + d*2^shift_s   (shared memory)
+//   lvl[k][j] keys[j * 8^k] - top[bucket], k < h     -- u32, groups of 8 = one 32-byte sector
+//   wide bit  bucket t spans >= 2^32-1 bytes -> binary search over keys[] instead of lvl[]
+// A lookup = dir (2 LDS) + ~1 LDS search step + top (1 LDS) + h sector gathers.
 constexpr int MAXL = 6;
-constexpr int TOPMAX = 16384;  // 128 KiB of u64 splitters in shared memory
+constexpr int TOPMAX = 16384;
+constexpr int DIRMAX = 16384;
+constexpr int MAXSEG = 32;
+constexpr int RUN_SMEM = 1024;  // extents staged in shared memory for reverse lookups
+
 struct IndexDev {
   const uint64_t *top;
   const uint32_t *wide;
+  const uint32_t *dir;
+  const uint64_t *seg_kmin;  // [nseg]
+  const uint32_t *seg_meta;  // [4*nseg]: dir_off, nb, tend, shift
   const uint32_t *lvl[MAXL];
   const uint64_t *keys;
-  const int *meta;  // meta[0] = n, meta[1] = h, meta[2] = ntop (written by the build kernels)
-};
-
-// Reverse-index payload: position j of the devbase-sorted order -> the unit and its CPU base.
-struct __align__(16) RevRec {
-  uint64_t base;
-  uint32_t unit;
-  uint32_t pad;
+  int n, h, ntop, nseg, ndir;
 };
 
 // One input segment of a slot kernel: n u64 slots at device address ptr (8-byte aligned),
@@ -59,7 +70,7 @@ struct Seg {
   uint32_t pad;
 };
 
-// per-call status, written by the kernels with warp-aggregated atomics
+// per-launch status, written by the kernels with warp-aggregated atomics
 struct Status {
   unsigned long long nulls, hits, misses, pending, notmapped, underflow, translated, pad;
 };
@@ -92,7 +103,8 @@ enum : int {
   OP_WRITE = 1,      // write the translation to the output
   OP_INC = 2,        // refcount += inc, detect 0 -> 1 activations (forward map)
   OP_INCPLAIN = 4,   // refcount += inc (rollbacks, re-map of an array-mapped outer)
-  OP_DEC = 8,        // refcount -= inc, detect underflow and 1 -> 0 (release)
+  OP_DEC = 8,        // refcount -= inc: atomics with return (underflow / 1 -> 0 lists) or, with
+                     // dec_red, fire-and-forget reductions checked by k_release_scan afterwards
   OP_GATE = 16,      // epoch gate of Alg. 2 + journal / copy list
   OP_CHECKMAPPED = 32,  // refcount must be > 0 (unmap of a CPU pointer)
   OP_HITMASK = 64,   // record which slots were translated (rollback / completion)
@@ -102,15 +114,16 @@ enum : int { DIR_FWD = 0, DIR_REV = 1 };
 enum : int { SEL_ALL = 0, SEL_HIT = 1, SEL_NOTHIT = 2 };
 
 struct SlotArgs {
-  IndexDev ix;
+  IndexDev fx;                 // forward index over unit bases
+  IndexDev rx;                 // reverse index over device extents (DIR_REV)
+  const uint64_t *runpay;      // per extent: host - device address delta (mirrored layout)
   UnitRec *rec;
-  const RevRec *rev;
   const Seg *segs;
-  const uint64_t *seg_chunk0;  // [nseg+1] prefix of 4-slot chunks per segment
+  const uint64_t *seg_chunk0;  // [nseg+1] prefix of 2-slot chunks per segment
   int nseg;
   int sel;
   uint64_t nchunks;
-  uint8_t *hitmask;            // [nchunks], bit m = slot m of the chunk was translated
+  uint32_t *hitmask;           // 2 bits per chunk: slot m of the chunk was translated
   uint64_t epoch;
   Status *st;
   unsigned long long *lc;      // shared list counters of the call: [0] act, [1] journal, [2] free, [3] copy
@@ -119,22 +132,15 @@ struct SlotArgs {
   uint32_t *copy_list;         // units that need a copy-back (stale, not read-only)
   uint32_t *free_list;
   int lenient;
-  int smem_top;                // capacity of the shared-memory splitter array
+  int dec_red;                 // OP_DEC through reductions + k_release_scan
 };
 
 // ---- host-callable launchers (kernels.cu) ----------------------------------------------------
 int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s);
-size_t slots_smem_bytes(int smem_top);
-void launch_build_index(const uint64_t *keys, const int *n_dev, int n_cap, uint64_t *top, uint32_t *wide,
-                        uint32_t *const *lvl, const size_t *lvl_cap, int *meta, cudaStream_t s);
+void launch_build_levels(const uint64_t *keys, int n, int h, const uint32_t *wide, uint32_t *const *lvl,
+                         const size_t *lvl_cap, cudaStream_t s);
 void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags,
                   const uint64_t *epoch0, const UnitRec *old_rec, UnitRec *new_rec, cudaStream_t s);
-void launch_rev_collect(const UnitRec *rec, int n, uint64_t *keys, uint32_t *vals, int *meta, cudaStream_t s);
-void launch_rev_payload(const uint32_t *units_sorted, const uint64_t *base, const int *n_dev, int n_cap,
-                        RevRec *rev, cudaStream_t s);
-size_t sort_pairs_temp_bytes(int n);
-void launch_sort_pairs(void *temp, size_t temp_bytes, const uint64_t *kin, uint64_t *kout, const uint32_t *vin,
-                       uint32_t *vout, int n, cudaStream_t s);
 size_t sort_keys_temp_bytes(int n);
 void launch_sort_keys(void *temp, size_t temp_bytes, const uint32_t *kin, uint32_t *kout, int n, cudaStream_t s);
 void launch_unit_ops(const UnitOp *ops, int n, UnitRec *rec, cudaStream_t s);
@@ -144,5 +150,7 @@ void launch_deactivate(const uint32_t *units, int n, UnitRec *rec, cudaStream_t 
 void launch_restore_epochs(const Journal *j, int n, UnitRec *rec, cudaStream_t s);
 void launch_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t *ptrs, int n, PointInfo *out,
                           cudaStream_t s);
+void launch_release_scan(const UnitRec *rec, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
+                         cudaStream_t s);
 
 }  // namespace cgcm

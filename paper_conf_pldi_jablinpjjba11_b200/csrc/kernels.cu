@@ -1,13 +1,16 @@
 // kernels.cu -- sm_100a kernels of the CGCM hot path.
 //
-//   k_slots<DIR, OPS>   the per-pointer kernel: interval lookup (a1, greatestLTE of P:L169-170 over
-//                       a sorted u64 key array, shared-memory top level + 8-ary u32 sector levels),
-//                       then any of: forward rewrite + refcount (a2, Alg. 1), reverse rewrite (a3),
-//                       epoch gate (a4, Alg. 2), release (Alg. 3).  Pointer arrays are streamed with
-//                       256-bit loads/stores (LDG/STG.E.ENL2.256) under an L2 evict-first policy so
-//                       the table stays resident in L2.
-//   k_build_*           table / index build (a0, off the per-pointer path).
-//   small kernels       activation bookkeeping, rollback, outer-pointer lookup.
+//   k_slots<DIR, OPS>   the per-pointer kernel.  a1: interval lookup (greatestLTE of P:L169-170)
+//                       over the sorted AU bases: shared-memory radix directory + top splitters,
+//                       then h 32-byte sector levels of u32 keys, then one 16-byte record gather.
+//                       Then any of a2 forward rewrite + refcount (Alg. 1), a3 reverse rewrite,
+//                       a4 epoch gate (Alg. 2), release (Alg. 3).  Reverse lookups find the device
+//                       extent (mirrored layout: one host-device delta per extent, shared memory),
+//                       then run the forward lookup on the host address and verify it.
+//                       Pointer arrays stream through 128-bit loads/stores with an L2 evict-first
+//                       policy so the table stays L2-resident; 2 slots per thread per step.
+//   k_build_level       u32 sector levels of an index (a0, off the per-pointer path).
+//   small kernels       activation bookkeeping, rollback, release scan, outer-pointer lookup.
 // DESIGN.md §7 gives the roofline of each kernel and its algorithmic bytes.
 #include <cub/cub.cuh>
 
@@ -18,7 +21,7 @@ namespace cgcm {
 namespace {
 
 constexpr int SLOT_THREADS = 1024;
-constexpr int SEG_SMEM = 512;
+constexpr int SEG_SMEM = 256;
 
 __device__ __forceinline__ uint64_t policy_evict_first() {
   uint64_t p;
@@ -30,23 +33,21 @@ __device__ __forceinline__ uint64_t policy_evict_last() {
   asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
   return p;
 }
-
-// 256-bit streaming load/store of four pointer slots (sm_100: LDG.E.ENL2.256 / STG.E.ENL2.256)
-__device__ __forceinline__ void ld_stream4(const void *p, uint64_t pol, uint64_t v[4]) {
-  asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
-               : "=l"(v[0]), "=l"(v[1]), "=l"(v[2]), "=l"(v[3])
+// two pointer slots, streamed (no L1 allocation, L2 evict-first)
+__device__ __forceinline__ void ld_stream2(const void *p, uint64_t pol, uint64_t &a, uint64_t &b) {
+  asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;"
+               : "=l"(a), "=l"(b)
                : "l"(p), "l"(pol));
 }
-__device__ __forceinline__ void st_stream4(void *p, uint64_t pol, const uint64_t v[4]) {
-  asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.u64 [%0], {%1,%2,%3,%4}, %5;" ::"l"(p),
-               "l"(v[0]), "l"(v[1]), "l"(v[2]), "l"(v[3]), "l"(pol)
+__device__ __forceinline__ void st_stream2(void *p, uint64_t pol, uint64_t a, uint64_t b) {
+  asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u64 [%0], {%1,%2}, %3;" ::"l"(p), "l"(a), "l"(b),
+               "l"(pol)
                : "memory");
 }
 __device__ __forceinline__ void st_stream1(void *p, uint64_t pol, uint64_t v) {
-  asm volatile("st.global.L1::no_allocate.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol)
-               : "memory");
+  asm volatile("st.global.L1::no_allocate.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol) : "memory");
 }
-// one 32-byte sector of the index / record arrays, kept in L2 (evict-last)
+// index / record gathers, kept in L2 (evict-last)
 __device__ __forceinline__ void ld_sector(const void *p, uint64_t pol, uint64_t v[4]) {
   asm volatile("ld.global.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
                : "=l"(v[0]), "=l"(v[1]), "=l"(v[2]), "=l"(v[3])
@@ -58,35 +59,35 @@ __device__ __forceinline__ void ld_pair(const void *p, uint64_t pol, uint64_t &a
 __device__ __forceinline__ void red_add(int32_t *p, int32_t v) {
   asm volatile("red.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
-
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
   return m;
 }
 
-// warp-aggregated append: returns this lane's slot in the list (valid only if pred)
+// warp-aggregated append (the whole warp executes it): this lane's slot in the list if pred
 __device__ __forceinline__ unsigned long long warp_append(unsigned long long *counter, bool pred) {
-  unsigned active = __activemask();
-  unsigned want = __ballot_sync(active, pred);
+  unsigned want = __ballot_sync(0xffffffffu, pred);
   unsigned long long base = 0;
   if (want) {
     int leader = __ffs(want) - 1;
-    if ((threadIdx.x & 31) == leader) base = atomicAdd(counter, (unsigned long long)__popc(want));
-    base = __shfl_sync(active, base, leader);
+    if ((int)(threadIdx.x & 31) == leader) base = atomicAdd(counter, (unsigned long long)__popc(want));
+    base = __shfl_sync(0xffffffffu, base, leader);
   }
   return base + __popc(want & lanemask_lt());
 }
-
-// per-warp reduction of a counter, one atomic per warp (all lanes are converged at kernel end)
 __device__ __forceinline__ void flush_count(unsigned long long *dst, unsigned long long v) {
-  unsigned active = __activemask();
-  if (active == 0xffffffffu) {
-    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(active, v, o);
-    if ((threadIdx.x & 31) == 0 && v) atomicAdd(dst, v);
-  } else if (v) {
-    atomicAdd(dst, v);
-  }
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  if ((threadIdx.x & 31) == 0 && v) atomicAdd(dst, v);
+}
+// interleave the low 16 bits of x with zeros (bit i -> bit 2i)
+__device__ __forceinline__ uint32_t spread16(uint32_t x) {
+  x &= 0xFFFFu;
+  x = (x | (x << 8)) & 0x00FF00FFu;
+  x = (x | (x << 4)) & 0x0F0F0F0Fu;
+  x = (x | (x << 2)) & 0x33333333u;
+  x = (x | (x << 1)) & 0x55555555u;
+  return x;
 }
 
 // number of entries <= r among 8 sorted u32 and the largest such entry
@@ -101,219 +102,361 @@ __device__ __forceinline__ void count8(const uint64_t w[4], uint32_t r, int &c, 
   }
 }
 
+// ---- an index's top level, staged in shared memory -------------------------------------------
+struct SIdx {
+  const uint64_t *top;
+  const uint32_t *dir;
+  const uint32_t *wide;
+  const uint64_t *skmin;
+  const uint32_t *smeta;
+  const uint64_t *pay;  // reverse index with h == 0: per-extent delta, staged
+  int ntop, nseg;
+  uint64_t kfirst;
+};
+
+__host__ __device__ __forceinline__ size_t al16(size_t x) { return (x + 15) & ~size_t(15); }
+__host__ __device__ __forceinline__ size_t stage_bytes(const IndexDev &ix, bool with_pay) {
+  size_t b = al16(8 * (size_t)ix.ntop) + al16(4 * (size_t)ix.ndir) + al16(4 * (size_t)((ix.ntop + 31) / 32)) +
+             al16(8 * (size_t)ix.nseg) + al16(16 * (size_t)ix.nseg);
+  if (with_pay) b += al16(8 * (size_t)ix.ntop);
+  return b;
+}
+
+__device__ __forceinline__ unsigned char *stage(const IndexDev &ix, const uint64_t *pay, unsigned char *base,
+                                                SIdx &S) {
+  uint64_t *top = reinterpret_cast<uint64_t *>(base);
+  base += al16(8 * (size_t)ix.ntop);
+  uint32_t *dir = reinterpret_cast<uint32_t *>(base);
+  base += al16(4 * (size_t)ix.ndir);
+  uint32_t *wide = reinterpret_cast<uint32_t *>(base);
+  base += al16(4 * (size_t)((ix.ntop + 31) / 32));
+  uint64_t *skmin = reinterpret_cast<uint64_t *>(base);
+  base += al16(8 * (size_t)ix.nseg);
+  uint32_t *smeta = reinterpret_cast<uint32_t *>(base);
+  base += al16(16 * (size_t)ix.nseg);
+  uint64_t *spay = nullptr;
+  if (pay) {
+    spay = reinterpret_cast<uint64_t *>(base);
+    base += al16(8 * (size_t)ix.ntop);
+  }
+  for (int t = threadIdx.x; t < ix.ntop; t += blockDim.x) top[t] = ix.top[t];
+  for (int t = threadIdx.x; t < ix.ndir; t += blockDim.x) dir[t] = ix.dir[t];
+  for (int t = threadIdx.x; t < (ix.ntop + 31) / 32; t += blockDim.x) wide[t] = ix.wide[t];
+  for (int t = threadIdx.x; t < ix.nseg; t += blockDim.x) skmin[t] = ix.seg_kmin[t];
+  for (int t = threadIdx.x; t < 4 * ix.nseg; t += blockDim.x) smeta[t] = ix.seg_meta[t];
+  if (pay)
+    for (int t = threadIdx.x; t < ix.ntop; t += blockDim.x) spay[t] = pay[t];
+  S.top = top;
+  S.dir = dir;
+  S.wide = wide;
+  S.skmin = skmin;
+  S.smeta = smeta;
+  S.pay = spay;
+  S.ntop = ix.ntop;
+  S.nseg = ix.nseg;
+  S.kfirst = ix.ntop > 0 ? ix.top[0] : ~0ull;
+  return base;
+}
+
+// greatest t with top[t] <= p (-1 if p < top[0]); tk = top[t]
+__device__ __forceinline__ int top_search(const SIdx &S, uint64_t p, uint64_t &tk) {
+  if (p < S.kfirst) return -1;
+  int sg = 0;
+  if (S.nseg > 1) {
+    int lo = 0, len = S.nseg;
+    while (len > 1) {
+      int half = len >> 1;
+      if (S.skmin[lo + half] <= p) lo += half;
+      len -= half;
+    }
+    sg = lo;
+  }
+  const uint32_t off = S.smeta[4 * sg], nb = S.smeta[4 * sg + 1], tend = S.smeta[4 * sg + 2],
+                 sh = S.smeta[4 * sg + 3];
+  uint64_t d = (p - S.skmin[sg]) >> sh;
+  if (d >= nb) d = nb - 1;
+  uint32_t first = S.dir[off + d];
+  uint32_t last = (d + 1 < nb) ? S.dir[off + d + 1] : tend;
+  uint32_t count = last - first;
+  while (count > 0) {  // upper bound of p in top[first, last)
+    uint32_t step = count >> 1, it = first + step;
+    if (S.top[it] <= p) {
+      first = it + 1;
+      count -= step + 1;
+    } else {
+      count = step;
+    }
+  }
+  int t = (int)first - 1;
+  tk = S.top[t];
+  return t;
+}
+
+// two interleaved greatestLTE lookups through the u32 sector levels.  In: j = t, key = top[t]
+// from top_search (j < 0: no candidate).  Out: j = key index (or -1), key = keys[j].
+__device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix, uint64_t pol, const uint64_t p[2],
+                                              int j[2], uint64_t key[2]) {
+  if (ix.h == 0) return;  // j = t, key = tk already
+  uint32_t rel[2], last[2] = {0, 0};
+  bool wide[2];
+  int t0[2];
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    t0[m] = j[m];
+    int tt = j[m] < 0 ? 0 : j[m];
+    wide[m] = j[m] >= 0 && ((S.wide[tt >> 5] >> (tt & 31)) & 1u);
+    uint64_t d = p[m] - key[m];
+    rel[m] = d >= 0xFFFFFFFEull ? 0xFFFFFFFEu : (uint32_t)d;
+    if (j[m] < 0) j[m] = 0;
+  }
+  for (int k = ix.h - 1; k >= 0; --k) {
+    const uint32_t *L = ix.lvl[k];
+    uint64_t w0[4], w1[4];
+    ld_sector(L + 8 * (size_t)j[0], pol, w0);
+    ld_sector(L + 8 * (size_t)j[1], pol, w1);
+    int c;
+    uint32_t lst;
+    count8(w0, rel[0], c, lst);
+    j[0] = 8 * j[0] + c - 1;
+    last[0] = lst;
+    count8(w1, rel[1], c, lst);
+    j[1] = 8 * j[1] + c - 1;
+    last[1] = lst;
+  }
+  const int sh = 3 * ix.h;
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    key[m] += last[m];
+    if (t0[m] < 0) {
+      j[m] = -1;
+    } else if (wide[m]) {  // bucket spanning >= 4 GiB: binary search over the full u64 keys
+      int lo = t0[m] << sh, len = min(ix.n, (t0[m] + 1) << sh) - lo;
+      while (len > 1) {
+        int half = len >> 1;
+        if (ix.keys[lo + half] <= p[m]) lo += half;
+        len -= half;
+      }
+      j[m] = lo;
+      key[m] = ix.keys[lo];
+    }
+  }
+}
+
 }  // namespace
 
 // -------------------------------------------------------------------------------------------------
-// The slot kernel.  One thread handles one 32-byte-aligned chunk (4 slots) per grid-stride step;
-// the 4 lookups are interleaved level by level so their sector loads are in flight together.
+// The slot kernel.  Each thread handles one 16-byte chunk (2 slots) per warp-uniform grid-stride
+// step; the two lookups are interleaved level by level.
 // -------------------------------------------------------------------------------------------------
 template <int DIR, int OPS>
 __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ uint64_t s_seg0[SEG_SMEM + 1];
-  uint64_t *s_top = reinterpret_cast<uint64_t *>(smem);
-  uint32_t *s_wide = reinterpret_cast<uint32_t *>(smem + 8 * (size_t)a.smem_top);
-
-  const int n = a.ix.meta[0], h = a.ix.meta[1], ntop = a.ix.meta[2];
-  for (int t = threadIdx.x; t < ntop; t += blockDim.x) s_top[t] = a.ix.top[t];
-  for (int t = threadIdx.x; t < (ntop + 31) / 32; t += blockDim.x) s_wide[t] = a.ix.wide[t];
+  SIdx F, R;
+  unsigned char *sp = stage(a.fx, nullptr, smem, F);
+  if (DIR == DIR_REV) stage(a.rx, a.rx.h == 0 ? a.runpay : nullptr, sp, R);
   const int nseg_s = a.nseg <= SEG_SMEM ? a.nseg : 0;
   for (int t = threadIdx.x; t <= nseg_s; t += blockDim.x) s_seg0[t] = a.seg_chunk0[t];
   __syncthreads();
 
   const uint64_t pol_s = policy_evict_first();
   const uint64_t pol_t = policy_evict_last();
-  const uint64_t top0 = ntop > 0 ? s_top[0] : ~0ull;
-  const int sh = 3 * h;
+  constexpr bool FULLREC = (DIR == DIR_REV) || (OPS & (OP_GATE | OP_CHECKMAPPED));
+  const int lane = threadIdx.x & 31;
 
   unsigned long long c_nulls = 0, c_hits = 0, c_miss = 0, c_pend = 0, c_notm = 0, c_under = 0, c_tr = 0;
 
-  for (uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; c < a.nchunks;
-       c += (uint64_t)gridDim.x * blockDim.x) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
+    const uint64_t c = cb + lane;
+    const bool live = c < a.nchunks;
     // ---- which segment / which slots ----
-    int s;
-    if (a.nseg == 1) {
-      s = 0;
-    } else {
-      const uint64_t *sp = nseg_s ? s_seg0 : a.seg_chunk0;
+    int s = 0;
+    if (a.nseg > 1 && live) {
+      const uint64_t *spp = nseg_s ? s_seg0 : a.seg_chunk0;
       int lo = 0, len = a.nseg;  // last s with seg0[s] <= c
       while (len > 1) {
         int half = len >> 1;
-        if (sp[lo + half] <= c) lo += half;
+        if (spp[lo + half] <= c) lo += half;
         len -= half;
       }
       s = lo;
     }
-    const Seg sg = a.segs[s];
-    const uint64_t c0 = nseg_s ? s_seg0[s] : a.seg_chunk0[s];
-    const uint64_t a0 = (sg.ptr & ~31ull) + 32ull * (c - c0);
-    const uint64_t lo_addr = sg.ptr, hi_addr = sg.ptr + 8ull * sg.n;
+    Seg sg;
+    uint64_t a0 = 0;
     uint32_t valid = 0;
-#pragma unroll
-    for (int m = 0; m < 4; ++m) {
-      uint64_t ad = a0 + 8ull * m;
-      if (ad >= lo_addr && ad < hi_addr) valid |= 1u << m;
+    uint64_t v[2] = {0, 0};
+    if (live) {
+      sg = a.segs[s];
+      const uint64_t c0 = nseg_s ? s_seg0[s] : a.seg_chunk0[s];
+      a0 = (sg.ptr & ~15ull) + 16ull * (c - c0);
+      const uint64_t hi_addr = sg.ptr + 8ull * sg.n;
+      if (a0 >= sg.ptr && a0 < hi_addr) valid |= 1u;
+      if (a0 + 8 >= sg.ptr && a0 + 8 < hi_addr) valid |= 2u;
+      if (a.sel != SEL_ALL) {
+        uint32_t hm = (a.hitmask[c >> 4] >> (2 * (c & 15))) & 3u;
+        valid &= (a.sel == SEL_HIT) ? hm : ~hm;
+      }
+      ld_stream2(reinterpret_cast<const void *>(a0), pol_s, v[0], v[1]);
+    } else {
+      sg.ptr = sg.n = sg.out = 0;
+      sg.inc = 0;
     }
-    if (a.sel != SEL_ALL) {
-      uint32_t hm = a.hitmask[c];
-      valid &= (a.sel == SEL_HIT) ? hm : ~hm;
-    }
-    uint64_t v[4];
-    ld_stream4(reinterpret_cast<const void *>(a0), pol_s, v);
 
-    // ---- a1: interval lookup, 4 interleaved searches ----
-    uint64_t p[4];
-    int b[4];
+    // ---- a1: lookups ----
+    uint64_t p[2], q[2], key[2], delta[2] = {0, 0};
+    int j[2];
+    bool look[2];
 #pragma unroll
-    for (int m = 0; m < 4; ++m) {
-      p[m] = ((valid >> m) & 1) ? v[m] : 0ull;
-      b[m] = 0;
+    for (int m = 0; m < 2; ++m) {
+      look[m] = ((valid >> m) & 1) && v[m] != 0;
+      p[m] = look[m] ? v[m] : 0ull;
     }
-    for (int len = ntop; len > 1;) {
-      int half = len >> 1;
+    if (DIR == DIR_REV) {
+      // the device extent holding p, and the host address it mirrors
 #pragma unroll
-      for (int m = 0; m < 4; ++m)
-        if (s_top[b[m] + half] <= p[m]) b[m] += half;
-      len -= half;
+      for (int m = 0; m < 2; ++m) {
+        uint64_t tk = 0;
+        int t = look[m] ? top_search(R, p[m], tk) : -1;
+        j[m] = t;
+        key[m] = tk;
+      }
+      if (a.rx.h > 0) level_lookup2(R, a.rx, pol_t, p, j, key);
+#pragma unroll
+      for (int m = 0; m < 2; ++m) {
+        if (j[m] >= 0) delta[m] = a.rx.h == 0 ? R.pay[j[m]] : a.runpay[j[m]];
+        else look[m] = false;
+        q[m] = look[m] ? p[m] + delta[m] : 0ull;
+      }
+    } else {
+      q[0] = p[0];
+      q[1] = p[1];
     }
-    uint64_t key[4];
-    uint32_t rel[4], last[4];
-    int j[4];
-    bool wide[4];
 #pragma unroll
-    for (int m = 0; m < 4; ++m) {
-      uint64_t tk = ntop > 0 ? s_top[b[m]] : 0ull;
+    for (int m = 0; m < 2; ++m) {
+      uint64_t tk = 0;
+      int t = look[m] ? top_search(F, q[m], tk) : -1;
+      j[m] = t;
       key[m] = tk;
-      uint64_t d = p[m] - tk;
-      rel[m] = d >= 0xFFFFFFFEull ? 0xFFFFFFFEu : (uint32_t)d;
-      j[m] = b[m];
-      last[m] = 0;
-      wide[m] = ntop > 0 && ((s_wide[b[m] >> 5] >> (b[m] & 31)) & 1u);
     }
-    for (int k = h - 1; k >= 0; --k) {
-      const uint32_t *L = a.ix.lvl[k];
-      uint64_t w[4][4];
-#pragma unroll
-      for (int m = 0; m < 4; ++m) ld_sector(L + 8 * (size_t)j[m], pol_t, w[m]);
-#pragma unroll
-      for (int m = 0; m < 4; ++m) {
-        int cc;
-        uint32_t lst;
-        count8(w[m], rel[m], cc, lst);
-        j[m] = 8 * j[m] + cc - 1;
-        last[m] = lst;
-      }
-    }
-#pragma unroll
-    for (int m = 0; m < 4; ++m) {
-      key[m] += last[m];
-      if (wide[m]) {  // bucket spanning >= 4 GiB: binary search over the full u64 keys
-        int lo = b[m] << sh, len = min(n, (b[m] + 1) << sh) - lo;
-        while (len > 1) {
-          int half = len >> 1;
-          if (a.ix.keys[lo + half] <= p[m]) lo += half;
-          len -= half;
-        }
-        j[m] = lo;
-        key[m] = a.ix.keys[lo];
-      }
-    }
+    level_lookup2(F, a.fx, pol_t, q, j, key);
 
-    // ---- record sectors ----
-    uint64_t r[4][4];
-    uint64_t cbase[4];
-    int unit[4];
-    bool hit[4], nul[4];
+    // ---- record gathers ----
+    uint64_t r[2][4];
 #pragma unroll
-    for (int m = 0; m < 4; ++m) {
-      nul[m] = ((valid >> m) & 1) && v[m] == 0;
-      bool look = ((valid >> m) & 1) && v[m] != 0 && p[m] >= top0;
-      if (DIR == DIR_FWD) {
-        unit[m] = look ? j[m] : 0;
-        cbase[m] = key[m];
-      } else {
-        uint64_t bb = 0, uu = 0;
-        if (look) ld_pair(a.rev + j[m], pol_t, bb, uu);
-        cbase[m] = bb;
-        unit[m] = (int)(uint32_t)uu;
+    for (int m = 0; m < 2; ++m) {
+      look[m] = look[m] && j[m] >= 0;
+      r[m][0] = r[m][1] = r[m][2] = r[m][3] = 0;
+      if (look[m]) {
+        if (FULLREC) ld_sector(a.rec + j[m], pol_t, r[m]);
+        else ld_pair(a.rec + j[m], pol_t, r[m][0], r[m][1]);
       }
-      if (look) ld_sector(a.rec + unit[m], pol_t, r[m]);
-      else r[m][0] = r[m][1] = r[m][2] = r[m][3] = 0;
-      hit[m] = look && (p[m] - key[m] <= r[m][0]);  // A7: p - base <= size
+    }
+    bool hit[2];
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      hit[m] = look[m] && (q[m] - key[m] <= rec_size(r[m][0]));  // A7: p - base <= size
+      if (DIR == DIR_REV && look[m]) {
+        // the unit found from the host address must own this extent's copy (active, mirrored)
+        bool own = (rec_flags(r[m][0]) & UF_ACTIVE) && r[m][1] + delta[m] == key[m];
+        if (!(hit[m] && own)) {
+          hit[m] = false;
+          if (q[m] == key[m] && j[m] > 0) {  // one past the end of the previous unit (A7)
+            uint64_t r2[4];
+            ld_sector(a.rec + (j[m] - 1), pol_t, r2);
+            uint64_t b2 = a.fx.keys[j[m] - 1];
+            if ((rec_flags(r2[0]) & UF_ACTIVE) && r2[1] + delta[m] == b2 && q[m] - b2 == rec_size(r2[0])) {
+              hit[m] = true;
+              j[m] -= 1;
+              key[m] = b2;
+              r[m][0] = r2[0];
+              r[m][1] = r2[1];
+              r[m][2] = r2[2];
+              r[m][3] = r2[3];
+            }
+          }
+        }
+      }
     }
 
     // ---- a2/a3/a4 operations ----
-    uint64_t outv[4];
+    uint64_t outv[2] = {v[0], v[1]};
     uint32_t wrote = 0;
 #pragma unroll
-    for (int m = 0; m < 4; ++m) {
+    for (int m = 0; m < 2; ++m) {
       const bool vm = (valid >> m) & 1;
       const bool hm = vm && hit[m];
-      const bool miss = vm && !nul[m] && !hit[m];
-      c_nulls += nul[m];
+      const bool nul = vm && v[m] == 0;
+      c_nulls += nul;
       c_hits += hm;
-      c_miss += miss;
-      outv[m] = v[m];
-      UnitRec *R = a.rec + unit[m];
-      const uint64_t off = p[m] - key[m];
+      c_miss += (vm && !nul && !hm);
+      const int unit = hm ? j[m] : 0;
+      UnitRec *Rp = a.rec + unit;
+      const uint64_t off = q[m] - key[m];
+      const uint32_t fl = rec_flags(r[m][0]);
       const uint64_t devbase = r[m][1], ep = r[m][2];
       const int32_t rc = (int32_t)(uint32_t)r[m][3];
-      const uint32_t fl = (uint32_t)(r[m][3] >> 32);
       if (OPS & OP_CHECKMAPPED) c_notm += (hm && rc <= 0);
       bool act = false;
       if (OPS & OP_INC) {
         if (hm) {
-          if (rc > 0) {
-            red_add(&R->refcount, sg.inc);
+          if (fl & UF_ACTIVE) {
+            red_add(&Rp->refcount, sg.inc);
           } else {
-            int old = atomicAdd(&R->refcount, sg.inc);
-            act = (old == 0);
+            int old = atomicAdd(&Rp->refcount, sg.inc);
+            act = (old == 0);  // refcount 0 -> 1: Alg. 1's activation
           }
         }
       }
       if (OPS & OP_INCPLAIN)
-        if (hm) red_add(&R->refcount, sg.inc);
+        if (hm) red_add(&Rp->refcount, sg.inc);
       if (OPS & OP_DECPLAIN)
-        if (hm) red_add(&R->refcount, -sg.inc);
+        if (hm) red_add(&Rp->refcount, -sg.inc);
       bool freed = false;
       if (OPS & OP_DEC) {
         if (hm) {
-          int old = atomicAdd(&R->refcount, -sg.inc);
-          c_under += (old < sg.inc);
-          freed = (old == sg.inc);
+          if (a.dec_red) {
+            red_add(&Rp->refcount, -sg.inc);
+          } else {
+            int old = atomicAdd(&Rp->refcount, -sg.inc);
+            c_under += (old < sg.inc);
+            freed = (old == sg.inc);  // refcount 1 -> 0: Alg. 3's cuMemFree
+          }
         }
       }
       bool gated = false;
       uint64_t old_ep = 0;
       if (OPS & OP_GATE) {
         if (hm && ep != a.epoch) {
-          old_ep = atomicExch(reinterpret_cast<unsigned long long *>(&R->epoch), (unsigned long long)a.epoch);
+          old_ep = atomicExch(reinterpret_cast<unsigned long long *>(&Rp->epoch), (unsigned long long)a.epoch);
           gated = (old_ep != a.epoch);
         }
       }
       if (OPS & OP_WRITE) {
         if (hm) {
           if (DIR == DIR_FWD) {
-            if (devbase != 0) {
+            if (fl & UF_STORAGE) {
               outv[m] = devbase + off;  // Alg. 1: info.devptr + (ptr - info.base)
               wrote |= 1u << m;
             } else {
-              c_pend += 1;  // activated in this call: completed after the allocation
+              c_pend += 1;  // activated by this call: completed after the allocation
             }
           } else {
-            outv[m] = cbase[m] + off;  // reverse: base + (g - devbase)
+            outv[m] = q[m];  // reverse: base + (g - devbase), the mirrored host address
             wrote |= 1u << m;
           }
         }
       }
-      // list appends in convergent code
+      // list appends (the whole warp takes part)
       if (OPS & OP_INC) {
         unsigned long long ix = warp_append(&a.lc[0], act);
-        if (act) a.act_list[ix] = (uint32_t)unit[m];
+        if (act) a.act_list[ix] = (uint32_t)unit;
       }
       if (OPS & OP_DEC) {
-        unsigned long long ix = warp_append(&a.lc[2], freed);
-        if (freed) a.free_list[ix] = (uint32_t)unit[m];
+        if (!a.dec_red) {
+          unsigned long long ix = warp_append(&a.lc[2], freed);
+          if (freed) a.free_list[ix] = (uint32_t)unit;
+        }
       }
       if (OPS & OP_GATE) {
         unsigned long long ix = warp_append(&a.lc[1], gated);
@@ -321,38 +464,48 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
         if (gated) {
           Journal jn;
           jn.old_epoch = old_ep;
-          jn.unit = (uint32_t)unit[m];
+          jn.unit = (uint32_t)unit;
           jn.copy = cp ? 1u : 0u;
           a.journal[ix] = jn;
         }
         unsigned long long cx = warp_append(&a.lc[3], cp);
-        if (cp) a.copy_list[cx] = (uint32_t)unit[m];
+        if (cp) a.copy_list[cx] = (uint32_t)unit;
       }
     }
     if (OPS & OP_WRITE) {
       c_tr += __popc(wrote);
-      if (wrote) {
-        if (sg.out == 0 && valid == 0xFu) {
-          st_stream4(reinterpret_cast<void *>(a0), pol_s, outv);
-        } else {
+      if (live) {
+        if (sg.out == 0) {
+          if (wrote == 3u) {
+            st_stream2(reinterpret_cast<void *>(a0), pol_s, outv[0], outv[1]);
+          } else {
 #pragma unroll
-          for (int m = 0; m < 4; ++m)
-            if ((wrote >> m) & 1) {
-              uint64_t dst = sg.out ? sg.out + (a0 + 8ull * m - sg.ptr) : a0 + 8ull * m;
+            for (int m = 0; m < 2; ++m)
+              if ((wrote >> m) & 1) st_stream1(reinterpret_cast<void *>(a0 + 8ull * m), pol_s, outv[m]);
+          }
+        } else {  // out of place: untranslated slots (NULL, lenient misses) are copied verbatim
+#pragma unroll
+          for (int m = 0; m < 2; ++m) {
+            const bool vm = (valid >> m) & 1;
+            const bool pend = DIR == DIR_FWD && hit[m] && !((wrote >> m) & 1);
+            if (vm && !pend) {
+              uint64_t dst = sg.out + (a0 + 8ull * m - sg.ptr);
               st_stream1(reinterpret_cast<void *>(dst), pol_s, outv[m]);
             }
+          }
         }
       }
-      if (sg.out != 0) {  // out-of-place: untranslated slots (NULL, lenient misses) copied verbatim
-#pragma unroll
-        for (int m = 0; m < 4; ++m)
-          if (((valid >> m) & 1) && !((wrote >> m) & 1) && !(hit[m] && DIR == DIR_FWD)) {
-            uint64_t dst = sg.out + (a0 + 8ull * m - sg.ptr);
-            st_stream1(reinterpret_cast<void *>(dst), pol_s, v[m]);
-          }
+    }
+    if (OPS & OP_HITMASK) {
+      unsigned b0 = __ballot_sync(0xffffffffu, wrote & 1u), b1 = __ballot_sync(0xffffffffu, (wrote >> 1) & 1u);
+      if (lane == 0) {
+        uint32_t w0 = spread16(b0) | (spread16(b1) << 1);
+        uint32_t w1 = spread16(b0 >> 16) | (spread16(b1 >> 16) << 1);
+        uint64_t wi = cb >> 4;
+        a.hitmask[wi] = w0;
+        if (cb + 16 < a.nchunks) a.hitmask[wi + 1] = w1;
       }
     }
-    if (OPS & OP_HITMASK) a.hitmask[c] = (uint8_t)wrote;
   }
   flush_count(&a.st->nulls, c_nulls);
   flush_count(&a.st->hits, c_hits);
@@ -374,7 +527,6 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
   X(DIR_FWD, OP_INCPLAIN)                              /* rollback of release                    */ \
   X(DIR_FWD, OP_GATE | OP_CHECKMAPPED)                 /* unmap by CPU pointer (Alg. 2, a4)      */ \
   X(DIR_FWD, OP_WRITE | OP_INCPLAIN)                   /* rollback of reverse+release            */ \
-  X(DIR_FWD, OP_WRITE | OP_HITMASK)                    /* translate only (no refcount)           */ \
   X(DIR_REV, OP_WRITE | OP_GATE | OP_HITMASK)          /* unmapArray: reverse (a3) + gate (a4)   */ \
   X(DIR_REV, OP_WRITE | OP_GATE | OP_DEC | OP_HITMASK) /* unmapArray + releaseArray fused        */ \
   X(DIR_REV, OP_GATE)                                  /* gate only (outer up to date)           */ \
@@ -384,11 +536,13 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
   X(DIR_REV, OP_DEC)                                   /* releaseArray of an array-mapped outer  */ \
   X(DIR_REV, OP_DECPLAIN)                              /* rollback of REV INCPLAIN               */
 
-size_t slots_smem_bytes(int smem_top) { return 8 * (size_t)smem_top + 4 * (size_t)((smem_top + 31) / 32) + 16; }
+static size_t slots_smem(const SlotArgs &a, int dir) {
+  return stage_bytes(a.fx, false) + (dir == DIR_REV ? stage_bytes(a.rx, a.rx.h == 0) : 0) + 64;
+}
 
 template <int DIR, int OPS>
 static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
-  size_t smem = slots_smem_bytes(a.smem_top);
+  size_t smem = slots_smem(a, DIR);
   static size_t configured = 0;
   if (smem > 48 * 1024 && smem > configured) {
     cudaError_t e = cudaFuncSetAttribute(k_slots<DIR, OPS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -411,30 +565,10 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s) {
 }
 
 // -------------------------------------------------------------------------------------------------
-// Index build (a0): top splitters, wide bits, u32 sector levels.  n may live on the device.
+// Index levels (a0): lvl[k][j] = keys[j*8^k] - keys[bucket start], u32, padded to groups of 8
 // -------------------------------------------------------------------------------------------------
-__device__ __forceinline__ void index_shape(int n, int &h, int &ntop) {
-  h = 0;
-  while (n > 0 && ((((int64_t)n + (1ll << (3 * h)) - 1) >> (3 * h)) > TOPMAX)) ++h;
-  ntop = n > 0 ? (int)(((int64_t)n + (1ll << (3 * h)) - 1) >> (3 * h)) : 0;
-}
-
-__global__ void k_build_top(const uint64_t *keys, const int *n_dev, uint64_t *top, uint32_t *wide, int *meta) {
-  int n = *n_dev, h, ntop;
-  index_shape(n, h, ntop);
-  int t = blockIdx.x * blockDim.x + threadIdx.x;
-  if (t == 0) { meta[0] = n; meta[1] = h; meta[2] = ntop; }
-  if (t >= ntop) return;
-  int first = t << (3 * h);
-  int lastu = min(n, (t + 1) << (3 * h)) - 1;
-  top[t] = keys[first];
-  if (keys[lastu] - keys[first] >= 0xFFFFFFFFull) atomicOr(&wide[t >> 5], 1u << (t & 31));
-}
-
-__global__ void k_build_level(const uint64_t *keys, const int *meta, const uint32_t *wide, int k, uint32_t *lvl,
+__global__ void k_build_level(const uint64_t *keys, int n, int h, const uint32_t *wide, int k, uint32_t *lvl,
                               size_t cap) {
-  int n = meta[0], h = meta[1];
-  if (k >= h) return;
   int64_t cnt = ((int64_t)n + (1ll << (3 * k)) - 1) >> (3 * k);
   int64_t padded = (cnt + 7) / 8 * 8;
   for (int64_t jj = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; jj < padded && jj < (int64_t)cap;
@@ -450,17 +584,13 @@ __global__ void k_build_level(const uint64_t *keys, const int *meta, const uint3
   }
 }
 
-void launch_build_index(const uint64_t *keys, const int *n_dev, int n_cap, uint64_t *top, uint32_t *wide,
-                        uint32_t *const *lvl, const size_t *lvl_cap, int *meta, cudaStream_t s) {
-  cudaMemsetAsync(wide, 0, 4 * ((TOPMAX + 31) / 32), s);
-  (void)cudaGetLastError();
-  k_build_top<<<(TOPMAX + 255) / 256, 256, 0, s>>>(keys, n_dev, top, wide, meta);
-  for (int k = 0; k < MAXL; ++k) {
-    if (!lvl[k] || lvl_cap[k] == 0) continue;
-    int64_t cnt = ((int64_t)n_cap + (1ll << (3 * k)) - 1) >> (3 * k);
+void launch_build_levels(const uint64_t *keys, int n, int h, const uint32_t *wide, uint32_t *const *lvl,
+                         const size_t *lvl_cap, cudaStream_t s) {
+  for (int k = 0; k < h; ++k) {
+    int64_t cnt = ((int64_t)n + (1ll << (3 * k)) - 1) >> (3 * k);
     int grid = (int)std::min<int64_t>((cnt + 255) / 256 + 1, 4096);
     (void)cudaGetLastError();
-    k_build_level<<<grid, 256, 0, s>>>(keys, meta, wide, k, lvl[k], lvl_cap[k]);
+    k_build_level<<<grid, 256, 0, s>>>(keys, n, h, wide, k, lvl[k], lvl_cap[k]);
   }
 }
 
@@ -474,11 +604,11 @@ __global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *size, con
   if (o >= 0) {
     r = old_rec[o];
   } else {
-    r.size = size[i];
+    r.szf = size[i] | ((uint64_t)flags[i] << FSHIFT);
     r.devbase = 0;
     r.epoch = epoch0[i];
     r.refcount = 0;
-    r.flags = flags[i];
+    r.pad = 0;
   }
   new_rec[i] = r;
 }
@@ -490,50 +620,6 @@ void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uin
   }
 }
 
-// reverse index: key = devbase of active units (refcount > 0), inactive sorted to the end
-__global__ void k_rev_collect(const UnitRec *rec, int n, uint64_t *keys, uint32_t *vals, int *count) {
-  int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  bool act = rec[i].refcount > 0;
-  keys[i] = act ? rec[i].devbase : ~0ull;
-  vals[i] = (uint32_t)i;
-  unsigned m = __ballot_sync(__activemask(), act);
-  if (act && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(count, __popc(m));
-}
-void launch_rev_collect(const UnitRec *rec, int n, uint64_t *keys, uint32_t *vals, int *count, cudaStream_t s) {
-  cudaMemsetAsync(count, 0, sizeof(int), s);
-  if (n > 0) {
-    (void)cudaGetLastError();
-    k_rev_collect<<<(n + 255) / 256, 256, 0, s>>>(rec, n, keys, vals, count);
-  }
-}
-__global__ void k_rev_payload(const uint32_t *units, const uint64_t *base, const int *n_dev, int n_cap, RevRec *rev) {
-  int j = blockIdx.x * blockDim.x + threadIdx.x;
-  if (j >= n_cap || j >= *n_dev) return;
-  RevRec r;
-  r.unit = units[j];
-  r.base = base[r.unit];
-  r.pad = 0;
-  rev[j] = r;
-}
-void launch_rev_payload(const uint32_t *units, const uint64_t *base, const int *n_dev, int n_cap, RevRec *rev,
-                        cudaStream_t s) {
-  if (n_cap > 0) {
-    (void)cudaGetLastError();
-    k_rev_payload<<<(n_cap + 255) / 256, 256, 0, s>>>(units, base, n_dev, n_cap, rev);
-  }
-}
-
-size_t sort_pairs_temp_bytes(int n) {
-  size_t bytes = 0;
-  cub::DeviceRadixSort::SortPairs(nullptr, bytes, (const uint64_t *)nullptr, (uint64_t *)nullptr,
-                                  (const uint32_t *)nullptr, (uint32_t *)nullptr, n);
-  return bytes;
-}
-void launch_sort_pairs(void *temp, size_t temp_bytes, const uint64_t *kin, uint64_t *kout, const uint32_t *vin,
-                       uint32_t *vout, int n, cudaStream_t s) {
-  cub::DeviceRadixSort::SortPairs(temp, temp_bytes, kin, kout, vin, vout, n, 0, 64, s);
-}
 size_t sort_keys_temp_bytes(int n) {
   size_t bytes = 0;
   cub::DeviceRadixSort::SortKeys(nullptr, bytes, (const uint32_t *)nullptr, (uint32_t *)nullptr, n);
@@ -546,6 +632,10 @@ void launch_sort_keys(void *temp, size_t temp_bytes, const uint32_t *kin, uint32
 // -------------------------------------------------------------------------------------------------
 // small bookkeeping kernels
 // -------------------------------------------------------------------------------------------------
+__device__ __forceinline__ unsigned *flag_word(UnitRec &r) {
+  return reinterpret_cast<unsigned *>(&r.szf) + 1;  // flags live in the top byte of the high word
+}
+
 __global__ void k_unit_ops(const UnitOp *ops, int n, UnitRec *rec) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
@@ -554,8 +644,10 @@ __global__ void k_unit_ops(const UnitOp *ops, int n, UnitRec *rec) {
   switch (o.op) {
     case UOP_ADD_RC: atomicAdd(&r.refcount, (int32_t)(int64_t)o.val); break;
     case UOP_SET_EPOCH: r.epoch = o.val; break;
-    case UOP_OR_FLAGS: atomicOr(&r.flags, (uint32_t)o.val); break;
-    case UOP_AND_FLAGS: atomicAnd(&r.flags, (uint32_t)o.val); break;
+    case UOP_OR_FLAGS: atomicOr(flag_word(r), (uint32_t)o.val << (FSHIFT - 32)); break;
+    case UOP_AND_FLAGS:
+      atomicAnd(flag_word(r), ((uint32_t)o.val << (FSHIFT - 32)) | ((1u << (FSHIFT - 32)) - 1));
+      break;
     case UOP_SET_DEVBASE: r.devbase = o.val; break;
     case UOP_SET_RC: r.refcount = (int32_t)(int64_t)o.val; break;
   }
@@ -573,7 +665,7 @@ __global__ void k_set_devbase(const uint32_t *units, const uint64_t *devbases, i
   if (i >= n) return;
   UnitRec &r = rec[units[i]];
   r.devbase = devbases[i];
-  r.flags |= UF_STORAGE;
+  r.szf |= (uint64_t)(UF_STORAGE | UF_ACTIVE) << FSHIFT;
   if (set_epoch) r.epoch = epoch;  // A5 reading R1: an AU is coherent when it becomes active
 }
 void launch_set_devbase(const uint32_t *units, const uint64_t *devbases, int n, UnitRec *rec, uint64_t epoch,
@@ -588,12 +680,12 @@ __global__ void k_deactivate(const uint32_t *units, int n, UnitRec *rec) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   UnitRec &r = rec[units[i]];
-  if (r.refcount != 0) return;  // re-activated in the meantime (cannot happen inside one call)
-  if (r.flags & UF_GLOBAL) {
-    r.flags &= ~UF_ARRAYMAPPED;  // named region persists
+  if (r.refcount != 0) return;
+  if (rec_flags(r.szf) & UF_GLOBAL) {
+    r.szf &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE) << FSHIFT);  // named region persists
   } else {
-    r.devbase = 0;               // cuMemFree (Alg. 3)
-    r.flags &= ~(UF_ARRAYMAPPED | UF_STORAGE);
+    r.devbase = 0;  // cuMemFree (Alg. 3)
+    r.szf &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE | UF_STORAGE) << FSHIFT);
   }
 }
 void launch_deactivate(const uint32_t *units, int n, UnitRec *rec, cudaStream_t s) {
@@ -615,13 +707,39 @@ void launch_restore_epochs(const Journal *j, int n, UnitRec *rec, cudaStream_t s
   }
 }
 
+// after a release pass through reductions: units whose refcount went negative (underflow) or
+// reached 0 while active (freed by this call)
+__global__ void k_release_scan(const UnitRec *rec, int n, Status *st, unsigned long long *lc, uint32_t *free_list) {
+  unsigned long long under = 0;
+  for (int base = blockIdx.x * blockDim.x; base < n; base += gridDim.x * blockDim.x) {
+    int i = base + threadIdx.x;
+    bool fr = false;
+    if (i < n) {
+      int32_t rc = rec[i].refcount;
+      under += rc < 0;
+      fr = rc == 0 && (rec_flags(rec[i].szf) & UF_ACTIVE);
+    }
+    unsigned long long ix = warp_append(&lc[2], fr);
+    if (fr) free_list[ix] = (uint32_t)i;
+  }
+  flush_count(&st->underflow, under);
+}
+void launch_release_scan(const UnitRec *rec, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
+                         cudaStream_t s) {
+  if (n > 0) {
+    int grid = std::min((n + 255) / 256, 1184);
+    (void)cudaGetLastError();
+    k_release_scan<<<grid, 256, 0, s>>>(rec, n, st, lc, free_list);
+  }
+}
+
 // outer-pointer lookup for mapArray/unmapArray/releaseArray: one thread per pointer, plain
 // binary search over the full u64 key array (few pointers: latency, not bandwidth)
 __global__ void k_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t *ptrs, int n, PointInfo *out) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   uint64_t p = ptrs[i];
-  int nk = ix.meta[0];
+  int nk = ix.n;
   PointInfo r;
   r.unit = -1;
   r.base = r.size = r.devbase = r.epoch = 0;
@@ -636,14 +754,14 @@ __global__ void k_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t 
       len -= half;
     }
     UnitRec u = rec[lo];
-    if (p - ix.keys[lo] <= u.size) {
+    if (p - ix.keys[lo] <= rec_size(u.szf)) {
       r.unit = lo;
       r.base = ix.keys[lo];
-      r.size = u.size;
+      r.size = rec_size(u.szf);
       r.devbase = u.devbase;
       r.epoch = u.epoch;
       r.refcount = u.refcount;
-      r.flags = u.flags;
+      r.flags = rec_flags(u.szf);
     }
   }
   out[i] = r;

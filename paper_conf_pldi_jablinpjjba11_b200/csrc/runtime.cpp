@@ -155,22 +155,30 @@ struct HostUnit {
 // one device extent holding the copies of one or more host-adjacent units (mirrored layout)
 struct Run {
   uint64_t addr = 0, bytes = 0;
+  uint64_t delta = 0;  // host address - device address of every unit copy in the extent (mirrored)
   int64_t live = 0;
 };
 
-// Search-index buffers (forward: all units by base; reverse: active units by devbase)
+// Search-index buffers: forward (all units by base) and reverse (live device extents by start)
 struct IndexBufs {
-  DevBuf top, wide, meta, ndev;
+  DevBuf top, wide, dir, skmin, smeta, keys, pay;
   DevBuf lvl[MAXL];
   size_t lvl_cap[MAXL] = {0};
-  int cap = -1;
-  IndexDev view(const uint64_t *keys) const {
+  int n = 0, h = 0, ntop = 0, nseg = 0, ndir = 0;
+  IndexDev view(const uint64_t *keys_dev) const {
     IndexDev ix;
     ix.top = top.as<uint64_t>();
     ix.wide = wide.as<uint32_t>();
+    ix.dir = dir.as<uint32_t>();
+    ix.seg_kmin = skmin.as<uint64_t>();
+    ix.seg_meta = smeta.as<uint32_t>();
     for (int k = 0; k < MAXL; ++k) ix.lvl[k] = lvl[k].as<uint32_t>();
-    ix.keys = keys;
-    ix.meta = meta.as<int>();
+    ix.keys = keys_dev;
+    ix.n = n;
+    ix.h = h;
+    ix.ntop = ntop;
+    ix.nseg = nseg;
+    ix.ndir = ndir;
     return ix;
   }
 };
@@ -196,8 +204,6 @@ struct Context {
   // device table
   DevBuf rec, dbase;
   IndexBufs fwd, rev;
-  DevBuf rev_kin, rev_kout, rev_vin, rev_vout, rev_payload, rev_temp;
-  size_t rev_temp_bytes = 0;
 
   // scratch
   DevBuf status, lc, hitmask, act_list, journal, free_list, copy_list, segs, seg0, staging, staging2, staging_cb, points, ptrs, temp;
@@ -209,6 +215,7 @@ struct Context {
   // runs of device extents
   std::vector<Run> runs;
   std::vector<int64_t> free_runs;
+  std::map<uint64_t, int64_t> live_runs;  // extent start -> run id (the reverse index's keys)
 
   // pinned host arena (cgcm_malloc)
   std::vector<std::pair<char *, size_t>> hchunks;
@@ -237,27 +244,35 @@ struct Context {
     b.bytes = 0;
   }
 
-  int64_t new_run(uint64_t addr, uint64_t bytes) {
+  int64_t new_run(uint64_t addr, uint64_t bytes, uint64_t delta) {
     Run r;
     r.addr = addr;
     r.bytes = bytes;
+    r.delta = delta;
     r.live = 0;
+    int64_t id;
     if (!free_runs.empty()) {
-      int64_t id = free_runs.back();
+      id = free_runs.back();
       free_runs.pop_back();
       runs[id] = r;
-      return id;
+    } else {
+      runs.push_back(r);
+      id = (int64_t)runs.size() - 1;
     }
-    runs.push_back(r);
-    return (int64_t)runs.size() - 1;
+    live_runs[addr] = id;
+    rev_dirty = true;
+    return id;
+  }
+  void drop_run(int64_t id) {
+    arena.free(runs[id].addr, runs[id].bytes);
+    live_runs.erase(runs[id].addr);
+    runs[id] = Run();
+    free_runs.push_back(id);
+    rev_dirty = true;
   }
   void run_release(int64_t id) {
     if (id < 0) return;
-    if (--runs[id].live <= 0) {
-      arena.free(runs[id].addr, runs[id].bytes);
-      runs[id] = Run();
-      free_runs.push_back(id);
-    }
+    if (--runs[id].live <= 0) drop_run(id);
   }
 
   int sync_main() {
@@ -267,36 +282,74 @@ struct Context {
 
   // ------------------------------------------------------------------------------------------
   // index build (a0)
-  int ensure_index_bufs(IndexBufs &ib, int cap) {
-    if (ib.cap >= cap && ib.top.addr) return CGCM_OK;
-    int c = std::max(cap, 1);
-    CKS(dalloc(ib.top, 8 * (size_t)std::min(c, TOPMAX) + 64));
-    CKS(dalloc(ib.wide, 4 * (size_t)((TOPMAX + 31) / 32) + 64));
-    CKS(dalloc(ib.meta, 64));
-    CKS(dalloc(ib.ndev, 64));
-    for (int k = 0; k < MAXL; ++k) {
-      int64_t cnt = ((int64_t)c + (1ll << (3 * k)) - 1) >> (3 * k);
-      size_t need = (size_t)((cnt + 7) / 8 * 8 + 8);
-      // levels k >= h are never used; only allocate levels that can exist for this capacity
-      bool used = cnt > 1 || k == 0;
-      if (!used) {
-        dfree(ib.lvl[k]);
-        ib.lvl_cap[k] = 0;
-        continue;
-      }
-      CKS(dalloc(ib.lvl[k], 4 * need));
-      ib.lvl_cap[k] = need;
+  // Build a search index over n sorted keys (hkeys on the host, dkeys the same keys on the device):
+  // top splitters, wide bits, segments and radix directory on the host; u32 levels on the device.
+  int build_index(IndexBufs &ib, const uint64_t *hkeys, int n, const uint64_t *dkeys, int topmax, int dirmax) {
+    int h = 0;
+    while (n > 0 && ((((int64_t)n + (1ll << (3 * h)) - 1) >> (3 * h)) > topmax)) ++h;
+    int ntop = n > 0 ? (int)((((int64_t)n + (1ll << (3 * h)) - 1) >> (3 * h))) : 0;
+    std::vector<uint64_t> top(std::max(ntop, 1), 0);
+    std::vector<uint32_t> wide((ntop + 31) / 32 + 1, 0);
+    for (int t = 0; t < ntop; ++t) {
+      int64_t first = (int64_t)t << (3 * h), last = std::min<int64_t>(n, (int64_t)(t + 1) << (3 * h)) - 1;
+      top[t] = hkeys[first];
+      if (hkeys[last] - hkeys[first] >= 0xFFFFFFFFull) wide[t >> 5] |= 1u << (t & 31);
     }
-    ib.cap = c;
-    return CGCM_OK;
-  }
-  int build_index(IndexBufs &ib, const uint64_t *keys, const int *n_dev, int cap) {
+    // segments at large gaps (so that one far-away region does not flatten the directory)
+    std::vector<int> segstart;
+    for (int thr = 32; thr <= 64; ++thr) {
+      segstart.assign(1, 0);
+      for (int t = 1; t < ntop; ++t)
+        if (thr < 64 && top[t] - top[t - 1] >= (1ull << thr)) segstart.push_back(t);
+      if ((int)segstart.size() <= MAXSEG) break;
+    }
+    int nseg = ntop > 0 ? (int)segstart.size() : 0;
+    std::vector<uint64_t> skmin(std::max(nseg, 1), 0);
+    std::vector<uint32_t> smeta(4 * std::max(nseg, 1), 0), dir;
+    for (int g = 0; g < nseg; ++g) {
+      int t0 = segstart[g], t1 = g + 1 < nseg ? segstart[g + 1] : ntop;
+      uint64_t kmin = top[t0], span = top[t1 - 1] - kmin;
+      int64_t nbt = std::max<int64_t>(1, (int64_t)(dirmax - nseg) * (t1 - t0) / std::max(ntop, 1));
+      uint32_t shift = 0;
+      while (shift < 63 && (int64_t)(span >> shift) + 1 > nbt) ++shift;
+      uint32_t nb = (uint32_t)((span >> shift) + 1);
+      skmin[g] = kmin;
+      smeta[4 * g] = (uint32_t)dir.size();
+      smeta[4 * g + 1] = nb;
+      smeta[4 * g + 2] = (uint32_t)t1;
+      smeta[4 * g + 3] = shift;
+      for (uint32_t d = 0; d < nb; ++d) {
+        uint64_t bstart = kmin + ((uint64_t)d << shift);
+        dir.push_back((uint32_t)(std::lower_bound(top.begin() + t0, top.begin() + t1, bstart) - top.begin()));
+      }
+    }
+    if (dir.empty()) dir.push_back(0);
+    std::vector<uint64_t> topv(top.begin(), top.begin() + std::max(ntop, 1));
+    CKS(upload(ib.top, topv));
+    CKS(upload(ib.wide, wide));
+    CKS(upload(ib.dir, dir));
+    CKS(upload(ib.skmin, skmin));
+    CKS(upload(ib.smeta, smeta));
     uint32_t *lv[MAXL];
-    for (int k = 0; k < MAXL; ++k) lv[k] = ib.lvl[k].as<uint32_t>();
-    launch_build_index(keys, n_dev, cap, ib.top.as<uint64_t>(), ib.wide.as<uint32_t>(), lv, ib.lvl_cap,
-                       ib.meta.as<int>(), main);
-    st.kernel_launches += 2 + MAXL;
-    CK(cudaGetLastError());
+    for (int k = 0; k < MAXL; ++k) {
+      if (k < h) {
+        int64_t cnt = ((int64_t)n + (1ll << (3 * k)) - 1) >> (3 * k);
+        size_t need = (size_t)((cnt + 7) / 8 * 8 + 8);
+        CKS(dalloc(ib.lvl[k], 4 * need));
+        ib.lvl_cap[k] = need;
+      }
+      lv[k] = ib.lvl[k].as<uint32_t>();
+    }
+    if (h > 0) {
+      launch_build_levels(dkeys, n, h, ib.wide.as<uint32_t>(), lv, ib.lvl_cap, main);
+      st.kernel_launches += h;
+      CK(cudaGetLastError());
+    }
+    ib.n = n;
+    ib.h = h;
+    ib.ntop = ntop;
+    ib.nseg = nseg;
+    ib.ndir = (int)dir.size();
     return CGCM_OK;
   }
 
@@ -352,9 +405,7 @@ struct Context {
     rec = nrec;
     dbase = nbase;
     U = n;
-    CKS(ensure_index_bufs(fwd, cap));
-    CK(cudaMemcpyAsync(fwd.ndev.as<void>(), &n, sizeof(int), cudaMemcpyHostToDevice, main));
-    CKS(build_index(fwd, dbase.as<uint64_t>(), fwd.ndev.as<int>(), n));
+    CKS(build_index(fwd, hb, n, dbase.as<uint64_t>(), TOPMAX, DIRMAX));
     CK(cudaStreamSynchronize(main));
     table_dirty = false;
     rev_dirty = true;
@@ -362,28 +413,25 @@ struct Context {
     return CGCM_OK;
   }
 
+  // reverse index: the live device extents by start address, payload = host - device delta
   int ensure_rev() {
     CKS(ensure_table());
     if (!rev_dirty) return CGCM_OK;
-    int cap = std::max(U, 1);
-    CKS(dalloc(rev_kin, 8 * (size_t)cap));
-    CKS(dalloc(rev_kout, 8 * (size_t)cap));
-    CKS(dalloc(rev_vin, 4 * (size_t)cap + 64));
-    CKS(dalloc(rev_vout, 4 * (size_t)cap + 64));
-    CKS(dalloc(rev_payload, 16 * (size_t)cap));
-    size_t tb = sort_pairs_temp_bytes(cap);
-    CKS(dalloc(rev_temp, tb + 256));
-    CKS(ensure_index_bufs(rev, cap));
-    launch_rev_collect(rec.as<UnitRec>(), U, rev_kin.as<uint64_t>(), rev_vin.as<uint32_t>(), rev.ndev.as<int>(),
-                       main);
-    if (U > 0)
-      launch_sort_pairs(rev_temp.as<void>(), rev_temp.bytes, rev_kin.as<uint64_t>(), rev_kout.as<uint64_t>(),
-                        rev_vin.as<uint32_t>(), rev_vout.as<uint32_t>(), U, main);
-    launch_rev_payload(rev_vout.as<uint32_t>(), dbase.as<uint64_t>(), rev.ndev.as<int>(), U,
-                       rev_payload.as<RevRec>(), main);
-    st.kernel_launches += 3;
-    CK(cudaGetLastError());
-    CKS(build_index(rev, rev_kout.as<uint64_t>(), rev.ndev.as<int>(), cap));
+    std::vector<uint64_t> keys, pay;
+    keys.reserve(live_runs.size() + 1);
+    pay.reserve(live_runs.size() + 1);
+    for (auto &kv : live_runs) {
+      keys.push_back(kv.first);
+      pay.push_back(runs[kv.second].delta);
+    }
+    std::vector<uint64_t> kup = keys, pup = pay;
+    if (kup.empty()) {
+      kup.push_back(0);
+      pup.push_back(0);
+    }
+    CKS(upload(rev.keys, kup));
+    CKS(upload(rev.pay, pup));
+    CKS(build_index(rev, keys.data(), (int)keys.size(), rev.keys.as<uint64_t>(), RUN_SMEM, RUN_SMEM));
     rev_dirty = false;
     st.rev_rebuilds += 1;
     return CGCM_OK;
@@ -393,6 +441,7 @@ struct Context {
   // slot kernels
   struct SlotCall {
     int dir = DIR_FWD, ops = 0, sel = SEL_ALL;
+    bool dec_red = false;  // OP_DEC through reductions + k_release_scan (large batches)
     std::vector<Seg> segs;
     uint64_t nchunks = 0;
     Status res{};
@@ -408,12 +457,12 @@ struct Context {
     if (k == 0) return CGCM_OK;
     std::vector<uint64_t> c0(k + 1, 0);
     for (int s = 0; s < k; ++s) {
-      uint64_t head = (c.segs[s].ptr & 31) / 8;
-      c0[s + 1] = c0[s] + (c.segs[s].n ? (head + c.segs[s].n + 3) / 4 : 0);
+      uint64_t head = (c.segs[s].ptr & 15) / 8;
+      c0[s + 1] = c0[s] + (c.segs[s].n ? (head + c.segs[s].n + 1) / 2 : 0);
     }
     c.nchunks = c0[k];
     if (c.nchunks == 0) return CGCM_OK;
-    if ((c.ops & OP_HITMASK) || c.sel != SEL_ALL) CKS(dalloc(hitmask, (size_t)c.nchunks + 64));
+    if ((c.ops & OP_HITMASK) || c.sel != SEL_ALL) CKS(dalloc(hitmask, 4 * (size_t)(c.nchunks / 16 + 4)));
     CKS(dalloc(segs, sizeof(Seg) * (size_t)k * 4 + 256));
     CKS(dalloc(seg0, 8 * (size_t)(k + 1) * 4 + 256));
     // each launch uses its own quarter of the segment buffers (up to 4 launches in flight)
@@ -425,20 +474,18 @@ struct Context {
     SlotArgs a;
     std::memset(&a, 0, sizeof(a));
     a.rec = rec.as<UnitRec>();
-    if (c.dir == DIR_FWD) {
-      a.ix = fwd.view(dbase.as<uint64_t>());
-      a.smem_top = std::min(std::max(U, 1), TOPMAX);
-    } else {
-      a.ix = rev.view(rev_kout.as<uint64_t>());
-      a.rev = rev_payload.as<RevRec>();
-      a.smem_top = std::min(std::max(U, 1), TOPMAX);
+    a.fx = fwd.view(dbase.as<uint64_t>());
+    if (c.dir == DIR_REV) {
+      a.rx = rev.view(rev.keys.as<uint64_t>());
+      a.runpay = rev.pay.as<uint64_t>();
     }
     a.segs = dsegs;
     a.seg_chunk0 = dc0;
     a.nseg = k;
     a.sel = c.sel;
     a.nchunks = c.nchunks;
-    a.hitmask = hitmask.as<uint8_t>();
+    a.hitmask = hitmask.as<uint32_t>();
+    a.dec_red = c.dec_red ? 1 : 0;
     a.epoch = epoch;
     a.st = status.as<Status>() + st_index;
     a.lc = lc.as<unsigned long long>();
@@ -456,6 +503,12 @@ struct Context {
     }
     CK(cudaGetLastError());
     st.kernel_launches += 1;
+    if ((c.ops & OP_DEC) && c.dec_red) {  // underflow / 1 -> 0 detection after reductions
+      launch_release_scan(rec.as<UnitRec>(), U, status.as<Status>() + st_index, lc.as<unsigned long long>(),
+                          free_list.as<uint32_t>(), main);
+      st.kernel_launches += 1;
+      CK(cudaGetLastError());
+    }
     if (timed) {
       CK(cudaEventRecord(ev_t1, main));
       CK(cudaEventSynchronize(ev_t1));
@@ -556,152 +609,100 @@ struct Context {
   // activation (refcount 0 -> 1 transitions collected by the map kernel): allocate device storage
   // with host-adjacent units mirrored into one extent, write devbase (+ epoch, A5 R1), and copy
   // the units host -> device as coalesced runs on the copy stream (transfer scheduler).
+  // Activation (refcount 0 -> 1, collected by the map kernel): device storage + devbase (+ epoch,
+  // A5 R1) + the host -> device copies (the transfer scheduler).  Index-consecutive units whose host
+  // gaps are small go into one extent that MIRRORS the host span [h0, h1) (devptr == base mod 256,
+  // host gaps kept as device gaps, so copies are device-adjacent iff host-adjacent, A7) and the extent
+  // has >= 1 byte of slack at its end.  One delta (host - device) per extent is what the reverse
+  // index stores.  A host-contiguous extent of >= 256 KiB is one direct DMA; any other extent is
+  // gathered on the host into pinned staging (multithreaded) and sent as one DMA.
   int activate_units(const std::vector<uint32_t> &units, std::vector<std::pair<uint64_t, uint64_t>> *h2d_out) {
     if (units.empty()) return CGCM_OK;
+    const uint64_t PACK_SPAN = 64ull << 20, GAPMAX = 64ull << 10, PACK_MIN = 256ull << 10;
+    struct Pack {
+      size_t i, j;
+      uint64_t h0, h1;
+      bool global, gaps;
+      int64_t run;
+      uint64_t dev0;
+    };
+    std::vector<Pack> packs;
+    uint64_t bytes = 0;
+    for (size_t i = 0; i < units.size(); ++i) {
+      auto it = by_idx[units[i]];
+      uint64_t b = it->first, sz = it->second.size;
+      bytes += sz;
+      bool g = (it->second.flags & UF_GLOBAL) != 0;
+      if (!g && !packs.empty() && !packs.back().global && b >= packs.back().h1 && b - packs.back().h1 <= GAPMAX &&
+          b + sz - packs.back().h0 <= PACK_SPAN) {
+        Pack &P = packs.back();
+        P.gaps = P.gaps || b != P.h1;
+        P.h1 = b + sz;
+        P.j = i + 1;
+      } else {
+        packs.push_back({i, i + 1, b, b + sz, g, false, -1, 0});
+      }
+    }
     std::vector<uint64_t> devbases(units.size());
-    // 1) host-contiguous runs of index-consecutive, host-adjacent, non-global units
-    struct HRun { size_t i, j; uint64_t b0, end; bool global; };
-    std::vector<HRun> hr;
-    for (size_t i = 0; i < units.size();) {
-      auto it0 = by_idx[units[i]];
-      uint64_t b0 = it0->first;
-      if (it0->second.flags & UF_GLOBAL) {
-        hr.push_back({i, i + 1, b0, b0 + it0->second.size, true});
-        ++i;
+    std::vector<int64_t> created;
+    for (auto &P : packs) {
+      HostUnit &u0 = by_idx[units[P.i]]->second;
+      if (P.global && u0.run >= 0) {  // named region allocated on an earlier activation (A14)
+        P.dev0 = u0.devbase;
+        P.run = u0.run;
+        devbases[P.i] = u0.devbase;
         continue;
       }
-      size_t j = i + 1;
-      uint64_t end = b0 + it0->second.size;
-      while (j < units.size() && units[j] == units[j - 1] + 1) {
-        auto it = by_idx[units[j]];
-        if ((it->second.flags & UF_GLOBAL) || it->first != end) break;
-        end += it->second.size;
-        ++j;
-      }
-      hr.push_back({i, j, b0, end, false});
-      i = j;
-    }
-    // 2) device placement.  A run keeps its host layout (devptr == base mod 256, host-adjacent units
-    //    stay adjacent) and is followed by >= 1 byte of slack so that copies of units that are not
-    //    host-adjacent are never device-adjacent (A7).  Large runs get their own extent and a direct
-    //    copy; small runs are packed into shared extents, gathered on the host into pinned staging
-    //    and sent with one DMA per pack (the transfer scheduler's coalescing for scattered AUs).
-    const uint64_t PACK_MIN = 256ull << 10, PACK_BYTES = 64ull << 20;
-    struct Ext { int64_t run; uint64_t addr, bytes; bool packed; std::vector<size_t> hruns; std::vector<uint64_t> off; };
-    std::vector<Ext> ext;
-    std::vector<char> fresh_run;  // indexed by run id: created by this call
-    auto mark_new = [&](int64_t r) {
-      if ((size_t)r >= fresh_run.size()) fresh_run.resize(r + 1, 0);
-      fresh_run[r] = 1;
-    };
-    uint64_t bytes = 0;
-    {
-      Ext cur;
-      cur.packed = true;
-      cur.run = -1;
-      cur.bytes = 0;
-      auto flush = [&]() {
-        if (!cur.hruns.empty()) ext.push_back(cur);
-        cur = Ext();
-        cur.packed = true;
-        cur.run = -1;
-        cur.bytes = 0;
-      };
-      for (size_t r = 0; r < hr.size(); ++r) {
-        HRun &h = hr[r];
-        uint64_t len = h.end - h.b0;
-        bytes += len;
-        if (h.global) {
-          HostUnit &u = by_idx[units[h.i]]->second;
-          if (u.run >= 0) {  // named region allocated on an earlier activation (A14)
-            devbases[h.i] = u.devbase;
-            Ext e;
-            e.run = u.run; e.addr = u.devbase - (h.b0 % 256); e.bytes = 0; e.packed = false;
-            e.hruns = {r}; e.off = {h.b0 % 256};
-            ext.push_back(e);
-            continue;
-          }
-        }
-        if (len >= PACK_MIN || h.global) {
-          Ext e;
-          e.run = -1; e.packed = false; e.bytes = (h.b0 % 256) + len + 1;
-          e.hruns = {r}; e.off = {h.b0 % 256};
-          ext.push_back(e);
-          continue;
-        }
-        uint64_t o = cur.bytes ? cur.bytes : 0;
-        o += ((h.b0 % 256) + 256 - (o % 256)) % 256;
-        if (o + len + 1 > PACK_BYTES && !cur.hruns.empty()) {
-          flush();
-          o = h.b0 % 256;
-        }
-        cur.hruns.push_back(r);
-        cur.off.push_back(o);
-        cur.bytes = o + len + 1;
-      }
-      flush();
-    }
-    // 3) allocate extents
-    for (auto &e : ext) {
-      if (e.run >= 0) continue;  // existing global region
-      uint64_t a = arena.alloc(e.bytes);
+      uint64_t need = (P.h0 % 256) + (P.h1 - P.h0) + 1;
+      uint64_t a = arena.alloc(need);
       if (!a) {
-        for (auto &f : ext)
-          if (f.run >= 0 && (size_t)f.run < fresh_run.size() && fresh_run[f.run]) {
-            arena.free(runs[f.run].addr, runs[f.run].bytes);
-            runs[f.run] = Run();
-            free_runs.push_back(f.run);
+        for (int64_t r : created) drop_run(r);
+        for (auto &Q : packs)
+          for (size_t q = Q.i; q < Q.j && Q.run >= 0; ++q) {
+            HostUnit &u = by_idx[units[q]]->second;
+            if (std::find(created.begin(), created.end(), u.run) != created.end()) {
+              u.run = -1;
+              u.devbase = 0;
+            }
           }
-        for (size_t q = 0; q < units.size(); ++q) {
-          HostUnit &u = by_idx[units[q]]->second;
-          if (u.run >= 0 && (size_t)u.run < fresh_run.size() && fresh_run[u.run]) {
-            u.run = -1;
-            u.devbase = 0;
-          }
-        }
         return CGCM_E_NOMEM;
       }
-      e.addr = a;
-      e.run = new_run(a, e.bytes);
-      mark_new(e.run);
-      for (size_t k = 0; k < e.hruns.size(); ++k) {
-        HRun &h = hr[e.hruns[k]];
-        uint64_t d0 = a + e.off[k];
-        for (size_t q = h.i; q < h.j; ++q) {
-          auto it = by_idx[units[q]];
-          it->second.devbase = d0 + (it->first - h.b0);
-          it->second.run = e.run;
-          runs[e.run].live += 1;
-          devbases[q] = it->second.devbase;
-        }
+      P.dev0 = a + (P.h0 % 256);
+      P.run = new_run(a, need, P.h0 - P.dev0);
+      created.push_back(P.run);
+      for (size_t q = P.i; q < P.j; ++q) {
+        auto it = by_idx[units[q]];
+        it->second.devbase = P.dev0 + (it->first - P.h0);
+        it->second.run = P.run;
+        runs[P.run].live += 1;
+        devbases[q] = it->second.devbase;
       }
     }
-    // 4) devbase (+ epoch, A5 R1) on the device, then the copies on the side stream
     CKS(upload(up_units, units));
     CKS(upload(up_vals, devbases));
     launch_set_devbase(up_units.as<uint32_t>(), up_vals.as<uint64_t>(), (int)units.size(), rec.as<UnitRec>(), epoch,
                        (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
-    CK(cudaEventRecord(ev_copy, main));  // copies may overwrite nothing the main stream still reads
+    CK(cudaEventRecord(ev_copy, main));  // the copies wait for everything the main stream did before
     CK(cudaStreamWaitEvent(copy, ev_copy, 0));
-    for (auto &e : ext) {
-      if (!e.packed) {
-        HRun &h = hr[e.hruns[0]];
-        CKS(copy_run(e.addr + e.off[0], h.b0, h.end - h.b0, true, units, h.i, h.j, copy));
-        if (h2d_out) h2d_out->push_back({e.addr + e.off[0], h.end - h.b0});
+    for (auto &P : packs) {
+      uint64_t span = P.h1 - P.h0;
+      if (P.global || (!P.gaps && span >= PACK_MIN)) {
+        CKS(copy_run(P.dev0, P.h0, span, true, units, P.i, P.j, copy));
+        if (h2d_out) h2d_out->push_back({P.dev0, span});
         continue;
       }
       int k = pack_k;
       pack_k ^= 1;
-      CK(cudaEventSynchronize(ev_pack[k]));  // the staging buffer's previous DMA is done
-      CKS(h_pack[k].ensure(e.bytes));
+      CK(cudaEventSynchronize(ev_pack[k]));  // this staging buffer's previous DMA is done
+      CKS(h_pack[k].ensure(span));
       char *stg = h_pack[k].as<char>();
-      gather(e, hr, stg);
-      CK(cudaMemcpyAsync(reinterpret_cast<void *>(e.addr), stg, e.bytes, cudaMemcpyHostToDevice, copy));
+      gather(units, P.i, P.j, P.h0, stg);
+      CK(cudaMemcpyAsync(reinterpret_cast<void *>(P.dev0), stg, span, cudaMemcpyHostToDevice, copy));
       CK(cudaEventRecord(ev_pack[k], copy));
       st.h2d_memcpy_calls += 1;
-      if (h2d_out) h2d_out->push_back({e.addr, e.bytes});
+      if (h2d_out) h2d_out->push_back({P.dev0, span});
     }
     CK(cudaEventRecord(ev_copy, copy));
     CK(cudaStreamWaitEvent(main, ev_copy, 0));
@@ -711,29 +712,24 @@ struct Context {
     rev_dirty = true;
     return CGCM_OK;
   }
-  template <class E, class H>
-  void gather(const E &e, const std::vector<H> &hr, char *stg) {
+  // host gather of units [i, j) into staging at their mirrored offsets (base - h0)
+  void gather(const std::vector<uint32_t> &units, size_t i, size_t j, uint64_t h0, char *stg) {
+    size_t n = j - i;
     uint64_t total = 0;
-    for (size_t k = 0; k < e.hruns.size(); ++k) total += hr[e.hruns[k]].end - hr[e.hruns[k]].b0;
+    for (size_t q = i; q < j; ++q) total += by_idx[units[q]]->second.size;
     unsigned T = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
-    if (total < (8ull << 20) || T == 1) {
-      for (size_t k = 0; k < e.hruns.size(); ++k) {
-        const H &h = hr[e.hruns[k]];
-        std::memcpy(stg + e.off[k], reinterpret_cast<const void *>(h.b0), h.end - h.b0);
+    auto work = [&](size_t lo, size_t hi) {
+      for (size_t q = lo; q < hi; ++q) {
+        auto it = by_idx[units[q]];
+        std::memcpy(stg + (it->first - h0), reinterpret_cast<const void *>(it->first), it->second.size);
       }
+    };
+    if (total < (8ull << 20) || T == 1 || n < 64) {
+      work(i, j);
       return;
     }
     std::vector<std::thread> th;
-    size_t n = e.hruns.size();
-    for (unsigned t = 0; t < T; ++t) {
-      size_t lo = n * t / T, hi = n * (t + 1) / T;
-      th.emplace_back([&, lo, hi] {
-        for (size_t k = lo; k < hi; ++k) {
-          const H &h = hr[e.hruns[k]];
-          std::memcpy(stg + e.off[k], reinterpret_cast<const void *>(h.b0), h.end - h.b0);
-        }
-      });
-    }
+    for (unsigned t = 0; t < T; ++t) th.emplace_back(work, i + n * t / T, i + n * (t + 1) / T);
     for (auto &x : th) x.join();
   }
 
@@ -1006,6 +1002,7 @@ struct Context {
     c.dir = DIR_REV;
     c.ops = write ? (OP_WRITE | OP_GATE | OP_HITMASK | (dec ? OP_DEC : 0)) : (OP_GATE | (dec ? OP_DEC : 0));
     c.segs = segs;
+    c.dec_red = dec && total >= (uint64_t)U / 8;
     CKS(launch(c, 0, false, false, true));
     Status sts[8];
     unsigned long long lcs[4];
@@ -1198,7 +1195,7 @@ int cgcm_setContext(void *ctx) {
 
 // ---- registration --------------------------------------------------------------------------
 static int declare_one(Context *C, uint64_t b, uint64_t s, uint32_t fl, const char *name) {
-  if (b == 0 || s == 0 || b + s < b) return CGCM_E_INVALID;
+  if (b == 0 || s == 0 || b + s < b || s > MAX_UNIT_SIZE) return CGCM_E_INVALID;
   auto succ = C->reg.lower_bound(b);
   if (succ != C->reg.end() && succ->first < b + s) return CGCM_E_OVERLAP;
   if (succ != C->reg.begin()) {
@@ -1233,7 +1230,7 @@ int cgcm_declareBatch(void *const *bases, const size_t *sizes, size_t n, unsigne
   std::sort(ord.begin(), ord.end(), [&](size_t a, size_t b) { return B(a) < B(b); });
   for (size_t q = 0; q < n; ++q) {  // validate everything first (all-or-nothing)
     uint64_t b = B(ord[q]), s = sizes[ord[q]];
-    if (b == 0 || s == 0 || b + s < b) return CGCM_E_INVALID;
+    if (b == 0 || s == 0 || b + s < b || s > MAX_UNIT_SIZE) return CGCM_E_INVALID;
     if (q + 1 < n && b + s > B(ord[q + 1])) return CGCM_E_OVERLAP;
     auto succ = C->reg.lower_bound(b);
     if (succ != C->reg.end() && succ->first < b + s) return CGCM_E_OVERLAP;
@@ -1449,6 +1446,7 @@ int cgcm_releaseBatch(const void *const *cpu, size_t n) {
   c.dir = DIR_FWD;
   c.ops = OP_DEC;
   c.segs = {Seg{d, n, 0, 1, 0}};
+  c.dec_red = n >= (size_t)C->U / 8;
   CKS(C->launch(c, 0));
   Status sts[8];
   unsigned long long lcs[4];
@@ -1759,6 +1757,7 @@ int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
   SlotCall R, F;
   R.dir = DIR_REV; R.ops = OP_DEC; R.segs = rsegs;
   F.dir = DIR_FWD; F.ops = OP_DEC; F.segs = fsegs;
+  R.dec_red = F.dec_red = total >= (uint64_t)C->U / 8;
   CKS(C->launch(R, 0));
   CKS(C->launch(F, 1));
   Status sts[8];
@@ -1835,14 +1834,15 @@ int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
   for (size_t i = 0; i < m; ++i) {
     const UnitRec &r = recs[i];
     cgcm_unit_t &u = out[i];
+    const uint32_t fl = rec_flags(r.szf);
     u.base = C->by_idx[i]->first;
-    u.size = r.size;
+    u.size = rec_size(r.szf);
     bool act = r.refcount > 0;
-    u.devptr = (act || ((r.flags & UF_GLOBAL) && (r.flags & UF_STORAGE))) ? r.devbase : 0;
+    u.devptr = (act || ((fl & UF_GLOBAL) && (fl & UF_STORAGE))) ? r.devbase : 0;
     u.refCount = r.refcount;
     u.epoch = r.epoch;
-    u.flags = ((r.flags & UF_GLOBAL) ? CGCM_UNIT_GLOBAL : 0) | ((r.flags & UF_READONLY) ? CGCM_UNIT_READONLY : 0) |
-              ((r.flags & UF_ARRAYMAPPED) ? CGCM_UNIT_ARRAYMAPPED : 0) | (act ? CGCM_UNIT_ACTIVE : 0);
+    u.flags = ((fl & UF_GLOBAL) ? CGCM_UNIT_GLOBAL : 0) | ((fl & UF_READONLY) ? CGCM_UNIT_READONLY : 0) |
+              ((fl & UF_ARRAYMAPPED) ? CGCM_UNIT_ARRAYMAPPED : 0) | (act ? CGCM_UNIT_ACTIVE : 0);
     u.pad = 0;
   }
   return (size_t)C->U <= cap ? CGCM_OK : CGCM_E_NOMEM;
