@@ -9,14 +9,15 @@ namespace cgcm {
 
 // Allocation-unit record (D3): one 32-byte sector per unit, indexed by the unit's rank
 // in base order.  The first 16 bytes are everything a forward translation needs (one 16-byte
-// gather): size, the unit's flags in the size word's top byte, and the device base.
-//   szf     = size (bits 0..55) | flags (bits 56..63)
-//   devbase = device copy (valid iff UF_STORAGE)
+// gather):
+//   endf    = base + size (bits 0..56) | flags (bits 57..63)   -- acceptance: p <= end (A7)
+//   delta   = devbase - base (mod 2^64), valid iff UF_STORAGE   -- translation: p + delta (Alg. 1)
 //   epoch   = Alg. 2's per-unit epoch
 //   refcount (Alg. 1/3)
+// The base itself lives in the sorted key array of the forward index.
 struct __align__(32) UnitRec {
-  uint64_t szf;
-  uint64_t devbase;
+  uint64_t endf;
+  uint64_t delta;
   uint64_t epoch;
   int32_t refcount;
   uint32_t pad;
@@ -28,13 +29,13 @@ enum : uint32_t {
   UF_READONLY = 2u,     // never copied back (Alg. 2)
   UF_ARRAYMAPPED = 4u,  // device copy holds translated pointers (A12)
   UF_ACTIVE = 8u,       // refcount > 0 at the start of the current call (stable during a call)
-  UF_STORAGE = 16u      // devbase valid
+  UF_STORAGE = 16u      // delta (device copy) valid
 };
-constexpr int FSHIFT = 56;
-constexpr uint64_t SIZE_MASK = (1ull << FSHIFT) - 1;
-constexpr uint64_t MAX_UNIT_SIZE = SIZE_MASK;
-__host__ __device__ __forceinline__ uint64_t rec_size(uint64_t szf) { return szf & SIZE_MASK; }
-__host__ __device__ __forceinline__ uint32_t rec_flags(uint64_t szf) { return (uint32_t)(szf >> FSHIFT); }
+constexpr int FSHIFT = 57;
+constexpr uint64_t ADDR_MASK = (1ull << FSHIFT) - 1;
+constexpr uint64_t ADDR_LIMIT = ADDR_MASK;  // base + size must stay below 2^57 (A26)
+__host__ __device__ __forceinline__ uint64_t rec_end(uint64_t endf) { return endf & ADDR_MASK; }
+__host__ __device__ __forceinline__ uint32_t rec_flags(uint64_t endf) { return (uint32_t)(endf >> FSHIFT); }
 
 // Sorted-key search index, built by the host (top level, directory) and the device (levels):
 //   keys      n sorted u64 (AU bases for the forward index, extent device starts for the reverse)
@@ -133,19 +134,20 @@ struct SlotArgs {
   uint32_t *free_list;
   int lenient;
   int dec_red;                 // OP_DEC through reductions + k_release_scan
+  int fx_nowide;               // the forward index has no wide bucket (specialised kernels)
 };
 
 // ---- host-callable launchers (kernels.cu) ----------------------------------------------------
 int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s);
 void launch_build_levels(const uint64_t *keys, int n, int h, const uint32_t *wide, uint32_t *const *lvl,
                          const size_t *lvl_cap, cudaStream_t s);
-void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags,
+void launch_remap(int n, const int32_t *old_idx, const uint64_t *base, const uint64_t *size, const uint32_t *flags,
                   const uint64_t *epoch0, const UnitRec *old_rec, UnitRec *new_rec, cudaStream_t s);
 size_t sort_keys_temp_bytes(int n);
 void launch_sort_keys(void *temp, size_t temp_bytes, const uint32_t *kin, uint32_t *kout, int n, cudaStream_t s);
 void launch_unit_ops(const UnitOp *ops, int n, UnitRec *rec, cudaStream_t s);
-void launch_set_devbase(const uint32_t *units, const uint64_t *devbases, int n, UnitRec *rec, uint64_t epoch,
-                        int set_epoch, cudaStream_t s);
+void launch_set_delta(const uint32_t *units, const uint64_t *deltas, int n, UnitRec *rec, uint64_t epoch,
+                      int set_epoch, cudaStream_t s);
 void launch_deactivate(const uint32_t *units, int n, UnitRec *rec, cudaStream_t s);
 void launch_restore_epochs(const Journal *j, int n, UnitRec *rec, cudaStream_t s);
 void launch_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t *ptrs, int n, PointInfo *out,

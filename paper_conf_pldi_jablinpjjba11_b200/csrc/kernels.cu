@@ -90,16 +90,15 @@ __device__ __forceinline__ uint32_t spread16(uint32_t x) {
   return x;
 }
 
-// number of entries <= r among 8 sorted u32 and the largest such entry
-__device__ __forceinline__ void count8(const uint64_t w[4], uint32_t r, int &c, uint32_t &last) {
-  c = 0;
-  last = 0;
+// number of entries <= r among 8 sorted u32 (one 32-byte level sector)
+__device__ __forceinline__ int count8(const uint64_t w[4], uint32_t r) {
+  int c = 0;
 #pragma unroll
   for (int q = 0; q < 4; ++q) {
-    uint32_t lo = (uint32_t)w[q], hi = (uint32_t)(w[q] >> 32);
-    if (lo <= r) { ++c; last = lo; }
-    if (hi <= r) { ++c; last = hi; }
+    c += ((uint32_t)w[q] <= r);
+    c += ((uint32_t)(w[q] >> 32) <= r);
   }
+  return c;
 }
 
 // ---- an index's top level, staged in shared memory -------------------------------------------
@@ -158,11 +157,12 @@ __device__ __forceinline__ unsigned char *stage(const IndexDev &ix, const uint64
   return base;
 }
 
-// greatest t with top[t] <= p (-1 if p < top[0]); tk = top[t]
+// greatest t with top[t] <= p (-1 if p < top[0]); tk = top[t].  ONESEG: the index has one segment.
+template <bool ONESEG = false>
 __device__ __forceinline__ int top_search(const SIdx &S, uint64_t p, uint64_t &tk) {
   if (p < S.kfirst) return -1;
   int sg = 0;
-  if (S.nseg > 1) {
+  if (!ONESEG && S.nseg > 1) {
     int lo = 0, len = S.nseg;
     while (len > 1) {
       int half = len >> 1;
@@ -192,12 +192,39 @@ __device__ __forceinline__ int top_search(const SIdx &S, uint64_t p, uint64_t &t
   return t;
 }
 
+// fixed-depth variant of level_lookup2 for indexes without wide buckets (the hot path)
+template <int H>
+__device__ __forceinline__ void level_lookup2_fixed(const IndexDev &ix, uint64_t pol, const uint64_t p[2], int j[2],
+                                                    const uint64_t key[2]) {
+  uint32_t rel[2];
+  bool ok[2];
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    ok[m] = j[m] >= 0;
+    uint64_t d = p[m] - key[m];
+    rel[m] = d >= 0xFFFFFFFEull ? 0xFFFFFFFEu : (uint32_t)d;
+    if (!ok[m]) j[m] = 0;
+  }
+#pragma unroll
+  for (int k = H - 1; k >= 0; --k) {
+    const uint32_t *L = ix.lvl[k];
+    uint64_t w0[4], w1[4];
+    ld_sector(L + 8 * (size_t)j[0], pol, w0);
+    ld_sector(L + 8 * (size_t)j[1], pol, w1);
+    j[0] = 8 * j[0] + count8(w0, rel[0]) - 1;
+    j[1] = 8 * j[1] + count8(w1, rel[1]) - 1;
+  }
+#pragma unroll
+  for (int m = 0; m < 2; ++m)
+    if (!ok[m]) j[m] = -1;
+}
+
 // two interleaved greatestLTE lookups through the u32 sector levels.  In: j = t, key = top[t]
-// from top_search (j < 0: no candidate).  Out: j = key index (or -1), key = keys[j].
+// from top_search (j < 0: no candidate).  Out: j = key index (or -1).
 __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix, uint64_t pol, const uint64_t p[2],
-                                              int j[2], uint64_t key[2]) {
-  if (ix.h == 0) return;  // j = t, key = tk already
-  uint32_t rel[2], last[2] = {0, 0};
+                                              int j[2], const uint64_t key[2]) {
+  if (ix.h == 0) return;
+  uint32_t rel[2];
   bool wide[2];
   int t0[2];
 #pragma unroll
@@ -207,26 +234,19 @@ __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix,
     wide[m] = j[m] >= 0 && ((S.wide[tt >> 5] >> (tt & 31)) & 1u);
     uint64_t d = p[m] - key[m];
     rel[m] = d >= 0xFFFFFFFEull ? 0xFFFFFFFEu : (uint32_t)d;
-    if (j[m] < 0) j[m] = 0;
+    j[m] = tt;
   }
   for (int k = ix.h - 1; k >= 0; --k) {
     const uint32_t *L = ix.lvl[k];
     uint64_t w0[4], w1[4];
     ld_sector(L + 8 * (size_t)j[0], pol, w0);
     ld_sector(L + 8 * (size_t)j[1], pol, w1);
-    int c;
-    uint32_t lst;
-    count8(w0, rel[0], c, lst);
-    j[0] = 8 * j[0] + c - 1;
-    last[0] = lst;
-    count8(w1, rel[1], c, lst);
-    j[1] = 8 * j[1] + c - 1;
-    last[1] = lst;
+    j[0] = 8 * j[0] + count8(w0, rel[0]) - 1;
+    j[1] = 8 * j[1] + count8(w1, rel[1]) - 1;
   }
   const int sh = 3 * ix.h;
 #pragma unroll
   for (int m = 0; m < 2; ++m) {
-    key[m] += last[m];
     if (t0[m] < 0) {
       j[m] = -1;
     } else if (wide[m]) {  // bucket spanning >= 4 GiB: binary search over the full u64 keys
@@ -237,7 +257,6 @@ __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix,
         len -= half;
       }
       j[m] = lo;
-      key[m] = ix.keys[lo];
     }
   }
 }
@@ -248,7 +267,9 @@ __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix,
 // The slot kernel.  Each thread handles one 16-byte chunk (2 slots) per warp-uniform grid-stride
 // step; the two lookups are interleaved level by level.
 // -------------------------------------------------------------------------------------------------
-template <int DIR, int OPS>
+// FH >= 0: the forward index has exactly FH levels, one address segment and no wide bucket (the
+// common case, specialised for the hot operation sets); FH < 0: generic.
+template <int DIR, int OPS, int FH>
 __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ uint64_t s_seg0[SEG_SMEM + 1];
@@ -263,85 +284,95 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
   const uint64_t pol_t = policy_evict_last();
   constexpr bool FULLREC = (DIR == DIR_REV) || (OPS & (OP_GATE | OP_CHECKMAPPED));
   const int lane = threadIdx.x & 31;
+  // single-segment calls (the common case) keep the segment in registers
+  Seg seg1 = a.segs[0];
+  const uint64_t a0base = seg1.ptr & ~15ull;
 
-  unsigned long long c_nulls = 0, c_hits = 0, c_miss = 0, c_pend = 0, c_notm = 0, c_under = 0, c_tr = 0;
+  unsigned c_nulls = 0, c_hits = 0, c_miss = 0, c_pend = 0, c_notm = 0, c_under = 0, c_tr = 0;
 
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  // software pipelining: the next iteration's two slots are loaded while this one is translated
+  const bool pf = a.nseg == 1;
+  uint64_t nv0 = 0, nv1 = 0;
+  {
+    const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (pf && c < a.nchunks) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c), pol_s, nv0, nv1);
+  }
   for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
     const uint64_t c = cb + lane;
     const bool live = c < a.nchunks;
-    // ---- which segment / which slots ----
-    int s = 0;
-    if (a.nseg > 1 && live) {
-      const uint64_t *spp = nseg_s ? s_seg0 : a.seg_chunk0;
-      int lo = 0, len = a.nseg;  // last s with seg0[s] <= c
-      while (len > 1) {
-        int half = len >> 1;
-        if (spp[lo + half] <= c) lo += half;
-        len -= half;
+    const uint64_t cv0 = nv0, cv1 = nv1;
+    if (pf && c + stride < a.nchunks)
+      ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + stride)), pol_s, nv0, nv1);
+    Seg sg = seg1;
+    uint64_t a0 = a0base + 16ull * c;
+    if (a.nseg > 1) {
+      int s = 0;
+      if (live) {
+        const uint64_t *spp = nseg_s ? s_seg0 : a.seg_chunk0;
+        int lo = 0, len = a.nseg;  // last s with seg0[s] <= c
+        while (len > 1) {
+          int half = len >> 1;
+          if (spp[lo + half] <= c) lo += half;
+          len -= half;
+        }
+        s = lo;
+        sg = a.segs[s];
       }
-      s = lo;
+      a0 = (sg.ptr & ~15ull) + 16ull * (c - (nseg_s ? s_seg0[s] : a.seg_chunk0[s]));
     }
-    Seg sg;
-    uint64_t a0 = 0;
     uint32_t valid = 0;
     uint64_t v[2] = {0, 0};
     if (live) {
-      sg = a.segs[s];
-      const uint64_t c0 = nseg_s ? s_seg0[s] : a.seg_chunk0[s];
-      a0 = (sg.ptr & ~15ull) + 16ull * (c - c0);
       const uint64_t hi_addr = sg.ptr + 8ull * sg.n;
-      if (a0 >= sg.ptr && a0 < hi_addr) valid |= 1u;
-      if (a0 + 8 >= sg.ptr && a0 + 8 < hi_addr) valid |= 2u;
+      valid = (a0 >= sg.ptr && a0 < hi_addr ? 1u : 0u) | (a0 + 8 >= sg.ptr && a0 + 8 < hi_addr ? 2u : 0u);
       if (a.sel != SEL_ALL) {
         uint32_t hm = (a.hitmask[c >> 4] >> (2 * (c & 15))) & 3u;
         valid &= (a.sel == SEL_HIT) ? hm : ~hm;
       }
-      ld_stream2(reinterpret_cast<const void *>(a0), pol_s, v[0], v[1]);
-    } else {
-      sg.ptr = sg.n = sg.out = 0;
-      sg.inc = 0;
+      if (pf) {
+        v[0] = cv0;
+        v[1] = cv1;
+      } else {
+        ld_stream2(reinterpret_cast<const void *>(a0), pol_s, v[0], v[1]);
+      }
     }
 
     // ---- a1: lookups ----
-    uint64_t p[2], q[2], key[2], delta[2] = {0, 0};
+    uint64_t q[2], key[2], dx[2] = {0, 0};
     int j[2];
     bool look[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
       look[m] = ((valid >> m) & 1) && v[m] != 0;
-      p[m] = look[m] ? v[m] : 0ull;
+      q[m] = look[m] ? v[m] : 0ull;
     }
     if (DIR == DIR_REV) {
-      // the device extent holding p, and the host address it mirrors
+      // the device extent holding the pointer, and the host address it mirrors
 #pragma unroll
       for (int m = 0; m < 2; ++m) {
         uint64_t tk = 0;
-        int t = look[m] ? top_search(R, p[m], tk) : -1;
-        j[m] = t;
+        j[m] = look[m] ? top_search(R, q[m], tk) : -1;
         key[m] = tk;
       }
-      if (a.rx.h > 0) level_lookup2(R, a.rx, pol_t, p, j, key);
+      if (a.rx.h > 0) level_lookup2(R, a.rx, pol_t, q, j, key);
 #pragma unroll
       for (int m = 0; m < 2; ++m) {
-        if (j[m] >= 0) delta[m] = a.rx.h == 0 ? R.pay[j[m]] : a.runpay[j[m]];
+        if (j[m] >= 0) dx[m] = a.rx.h == 0 ? R.pay[j[m]] : a.runpay[j[m]];
         else look[m] = false;
-        q[m] = look[m] ? p[m] + delta[m] : 0ull;
+        q[m] = look[m] ? q[m] + dx[m] : 0ull;  // host address
       }
-    } else {
-      q[0] = p[0];
-      q[1] = p[1];
     }
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
       uint64_t tk = 0;
-      int t = look[m] ? top_search(F, q[m], tk) : -1;
-      j[m] = t;
+      j[m] = look[m] ? top_search<(FH >= 0)>(F, q[m], tk) : -1;
       key[m] = tk;
     }
-    level_lookup2(F, a.fx, pol_t, q, j, key);
+    if constexpr (FH > 0) level_lookup2_fixed<FH>(a.fx, pol_t, q, j, key);
+    else if constexpr (FH < 0) level_lookup2(F, a.fx, pol_t, q, j, key);
 
-    // ---- record gathers ----
+    // ---- record gathers: {end|flags, delta} (+ {epoch, refcount}) ----
     uint64_t r[2][4];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
@@ -355,20 +386,17 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
     bool hit[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      hit[m] = look[m] && (q[m] - key[m] <= rec_size(r[m][0]));  // A7: p - base <= size
+      hit[m] = look[m] && q[m] <= rec_end(r[m][0]);  // A7: p - base <= size
       if (DIR == DIR_REV && look[m]) {
-        // the unit found from the host address must own this extent's copy (active, mirrored)
-        bool own = (rec_flags(r[m][0]) & UF_ACTIVE) && r[m][1] + delta[m] == key[m];
-        if (!(hit[m] && own)) {
+        // the unit must own this extent's copy: active, and its copy mirrors the extent
+        if (!(hit[m] && (rec_flags(r[m][0]) & UF_ACTIVE) && r[m][1] + dx[m] == 0)) {
           hit[m] = false;
-          if (q[m] == key[m] && j[m] > 0) {  // one past the end of the previous unit (A7)
+          if (j[m] > 0) {  // one past the end of the previous unit (A7)
             uint64_t r2[4];
             ld_sector(a.rec + (j[m] - 1), pol_t, r2);
-            uint64_t b2 = a.fx.keys[j[m] - 1];
-            if ((rec_flags(r2[0]) & UF_ACTIVE) && r2[1] + delta[m] == b2 && q[m] - b2 == rec_size(r2[0])) {
+            if ((rec_flags(r2[0]) & UF_ACTIVE) && r2[1] + dx[m] == 0 && q[m] == rec_end(r2[0])) {
               hit[m] = true;
               j[m] -= 1;
-              key[m] = b2;
               r[m][0] = r2[0];
               r[m][1] = r2[1];
               r[m][2] = r2[2];
@@ -392,11 +420,8 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
       c_miss += (vm && !nul && !hm);
       const int unit = hm ? j[m] : 0;
       UnitRec *Rp = a.rec + unit;
-      const uint64_t off = q[m] - key[m];
       const uint32_t fl = rec_flags(r[m][0]);
-      const uint64_t devbase = r[m][1], ep = r[m][2];
-      const int32_t rc = (int32_t)(uint32_t)r[m][3];
-      if (OPS & OP_CHECKMAPPED) c_notm += (hm && rc <= 0);
+      if (OPS & OP_CHECKMAPPED) c_notm += (hm && (int32_t)(uint32_t)r[m][3] <= 0);
       bool act = false;
       if (OPS & OP_INC) {
         if (hm) {
@@ -427,7 +452,7 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
       bool gated = false;
       uint64_t old_ep = 0;
       if (OPS & OP_GATE) {
-        if (hm && ep != a.epoch) {
+        if (hm && r[m][2] != a.epoch) {
           old_ep = atomicExch(reinterpret_cast<unsigned long long *>(&Rp->epoch), (unsigned long long)a.epoch);
           gated = (old_ep != a.epoch);
         }
@@ -436,7 +461,7 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
         if (hm) {
           if (DIR == DIR_FWD) {
             if (fl & UF_STORAGE) {
-              outv[m] = devbase + off;  // Alg. 1: info.devptr + (ptr - info.base)
+              outv[m] = q[m] + r[m][1];  // Alg. 1: info.devptr + (ptr - info.base)
               wrote |= 1u << m;
             } else {
               c_pend += 1;  // activated by this call: completed after the allocation
@@ -540,25 +565,46 @@ static size_t slots_smem(const SlotArgs &a, int dir) {
   return stage_bytes(a.fx, false) + (dir == DIR_REV ? stage_bytes(a.rx, a.rx.h == 0) : 0) + 64;
 }
 
-template <int DIR, int OPS>
+template <int DIR, int OPS, int FH>
 static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
   size_t smem = slots_smem(a, DIR);
   static size_t configured = 0;
   if (smem > 48 * 1024 && smem > configured) {
-    cudaError_t e = cudaFuncSetAttribute(k_slots<DIR, OPS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e =
+        cudaFuncSetAttribute(k_slots<DIR, OPS, FH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return -1;
     configured = smem;
   }
   uint64_t want = (a.nchunks + SLOT_THREADS - 1) / SLOT_THREADS;
   int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
-  k_slots<DIR, OPS><<<grid, SLOT_THREADS, smem, s>>>(a);
+  k_slots<DIR, OPS, FH><<<grid, SLOT_THREADS, smem, s>>>(a);
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
 
+// hot operation sets get depth-specialised forward lookups
+#define CGCM_HOT_OPS(X)                             \
+  X(DIR_FWD, OP_WRITE | OP_INC | OP_HITMASK)         \
+  X(DIR_REV, OP_WRITE | OP_GATE | OP_DEC | OP_HITMASK) \
+  X(DIR_REV, OP_WRITE | OP_GATE | OP_HITMASK)
+
 int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s) {
+  // the forward index qualifies for the specialised path: one segment, no wide bucket, h <= 3
+  int fh = a.fx.nseg <= 1 && a.fx_nowide && a.fx.h <= 3 ? a.fx.h : -1;
+#define X(D, O)                                        \
+  if (dir == D && ops == (O)) {                        \
+    switch (fh) {                                      \
+      case 0: return launch_one<D, (O), 0>(a, nsm, s); \
+      case 1: return launch_one<D, (O), 1>(a, nsm, s); \
+      case 2: return launch_one<D, (O), 2>(a, nsm, s); \
+      case 3: return launch_one<D, (O), 3>(a, nsm, s); \
+      default: return launch_one<D, (O), -1>(a, nsm, s); \
+    }                                                  \
+  }
+  CGCM_HOT_OPS(X)
+#undef X
 #define X(D, O) \
-  if (dir == D && ops == (O)) return launch_one<D, (O)>(a, nsm, s);
+  if (dir == D && ops == (O)) return launch_one<D, (O), -1>(a, nsm, s);
   CGCM_SLOT_OPS(X)
 #undef X
   return -2;  // unsupported combination
@@ -595,8 +641,8 @@ void launch_build_levels(const uint64_t *keys, int n, int h, const uint32_t *wid
 }
 
 // new_rec[i] = old_rec[old_idx[i]] (surviving unit) or a fresh record (declared since the last build)
-__global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags,
-                        const uint64_t *epoch0, const UnitRec *old_rec, UnitRec *new_rec) {
+__global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *base, const uint64_t *size,
+                        const uint32_t *flags, const uint64_t *epoch0, const UnitRec *old_rec, UnitRec *new_rec) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   UnitRec r;
@@ -604,19 +650,19 @@ __global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *size, con
   if (o >= 0) {
     r = old_rec[o];
   } else {
-    r.szf = size[i] | ((uint64_t)flags[i] << FSHIFT);
-    r.devbase = 0;
+    r.endf = (base[i] + size[i]) | ((uint64_t)flags[i] << FSHIFT);
+    r.delta = 0;
     r.epoch = epoch0[i];
     r.refcount = 0;
     r.pad = 0;
   }
   new_rec[i] = r;
 }
-void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags, const uint64_t *epoch0,
-                  const UnitRec *old_rec, UnitRec *new_rec, cudaStream_t s) {
+void launch_remap(int n, const int32_t *old_idx, const uint64_t *base, const uint64_t *size, const uint32_t *flags,
+                  const uint64_t *epoch0, const UnitRec *old_rec, UnitRec *new_rec, cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
-    k_remap<<<(n + 255) / 256, 256, 0, s>>>(n, old_idx, size, flags, epoch0, old_rec, new_rec);
+    k_remap<<<(n + 255) / 256, 256, 0, s>>>(n, old_idx, base, size, flags, epoch0, old_rec, new_rec);
   }
 }
 
@@ -633,7 +679,7 @@ void launch_sort_keys(void *temp, size_t temp_bytes, const uint32_t *kin, uint32
 // small bookkeeping kernels
 // -------------------------------------------------------------------------------------------------
 __device__ __forceinline__ unsigned *flag_word(UnitRec &r) {
-  return reinterpret_cast<unsigned *>(&r.szf) + 1;  // flags live in the top byte of the high word
+  return reinterpret_cast<unsigned *>(&r.endf) + 1;  // flags live in the top bits of the high word
 }
 
 __global__ void k_unit_ops(const UnitOp *ops, int n, UnitRec *rec) {
@@ -648,7 +694,7 @@ __global__ void k_unit_ops(const UnitOp *ops, int n, UnitRec *rec) {
     case UOP_AND_FLAGS:
       atomicAnd(flag_word(r), ((uint32_t)o.val << (FSHIFT - 32)) | ((1u << (FSHIFT - 32)) - 1));
       break;
-    case UOP_SET_DEVBASE: r.devbase = o.val; break;
+    case UOP_SET_DEVBASE: r.delta = o.val; break;  // (a delta: devbase - base)
     case UOP_SET_RC: r.refcount = (int32_t)(int64_t)o.val; break;
   }
 }
@@ -659,20 +705,20 @@ void launch_unit_ops(const UnitOp *ops, int n, UnitRec *rec, cudaStream_t s) {
   }
 }
 
-__global__ void k_set_devbase(const uint32_t *units, const uint64_t *devbases, int n, UnitRec *rec, uint64_t epoch,
-                              int set_epoch) {
+__global__ void k_set_delta(const uint32_t *units, const uint64_t *deltas, int n, UnitRec *rec, uint64_t epoch,
+                            int set_epoch) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   UnitRec &r = rec[units[i]];
-  r.devbase = devbases[i];
-  r.szf |= (uint64_t)(UF_STORAGE | UF_ACTIVE) << FSHIFT;
+  r.delta = deltas[i];
+  r.endf |= (uint64_t)(UF_STORAGE | UF_ACTIVE) << FSHIFT;
   if (set_epoch) r.epoch = epoch;  // A5 reading R1: an AU is coherent when it becomes active
 }
-void launch_set_devbase(const uint32_t *units, const uint64_t *devbases, int n, UnitRec *rec, uint64_t epoch,
-                        int set_epoch, cudaStream_t s) {
+void launch_set_delta(const uint32_t *units, const uint64_t *deltas, int n, UnitRec *rec, uint64_t epoch,
+                      int set_epoch, cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
-    k_set_devbase<<<(n + 255) / 256, 256, 0, s>>>(units, devbases, n, rec, epoch, set_epoch);
+    k_set_delta<<<(n + 255) / 256, 256, 0, s>>>(units, deltas, n, rec, epoch, set_epoch);
   }
 }
 
@@ -681,11 +727,11 @@ __global__ void k_deactivate(const uint32_t *units, int n, UnitRec *rec) {
   if (i >= n) return;
   UnitRec &r = rec[units[i]];
   if (r.refcount != 0) return;
-  if (rec_flags(r.szf) & UF_GLOBAL) {
-    r.szf &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE) << FSHIFT);  // named region persists
+  if (rec_flags(r.endf) & UF_GLOBAL) {
+    r.endf &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE) << FSHIFT);  // named region persists
   } else {
-    r.devbase = 0;  // cuMemFree (Alg. 3)
-    r.szf &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE | UF_STORAGE) << FSHIFT);
+    r.delta = 0;  // cuMemFree (Alg. 3)
+    r.endf &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE | UF_STORAGE) << FSHIFT);
   }
 }
 void launch_deactivate(const uint32_t *units, int n, UnitRec *rec, cudaStream_t s) {
@@ -710,14 +756,14 @@ void launch_restore_epochs(const Journal *j, int n, UnitRec *rec, cudaStream_t s
 // after a release pass through reductions: units whose refcount went negative (underflow) or
 // reached 0 while active (freed by this call)
 __global__ void k_release_scan(const UnitRec *rec, int n, Status *st, unsigned long long *lc, uint32_t *free_list) {
-  unsigned long long under = 0;
+  unsigned under = 0;
   for (int base = blockIdx.x * blockDim.x; base < n; base += gridDim.x * blockDim.x) {
     int i = base + threadIdx.x;
     bool fr = false;
     if (i < n) {
       int32_t rc = rec[i].refcount;
       under += rc < 0;
-      fr = rc == 0 && (rec_flags(rec[i].szf) & UF_ACTIVE);
+      fr = rc == 0 && (rec_flags(rec[i].endf) & UF_ACTIVE);
     }
     unsigned long long ix = warp_append(&lc[2], fr);
     if (fr) free_list[ix] = (uint32_t)i;
@@ -754,14 +800,14 @@ __global__ void k_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t 
       len -= half;
     }
     UnitRec u = rec[lo];
-    if (p - ix.keys[lo] <= rec_size(u.szf)) {
+    if (p <= rec_end(u.endf)) {
       r.unit = lo;
       r.base = ix.keys[lo];
-      r.size = rec_size(u.szf);
-      r.devbase = u.devbase;
+      r.size = rec_end(u.endf) - r.base;
+      r.flags = rec_flags(u.endf);
+      r.devbase = (r.flags & UF_STORAGE) ? r.base + u.delta : 0;
       r.epoch = u.epoch;
       r.refcount = u.refcount;
-      r.flags = rec_flags(u.szf);
     }
   }
   out[i] = r;

@@ -165,6 +165,7 @@ struct IndexBufs {
   DevBuf lvl[MAXL];
   size_t lvl_cap[MAXL] = {0};
   int n = 0, h = 0, ntop = 0, nseg = 0, ndir = 0;
+  bool any_wide = false;
   IndexDev view(const uint64_t *keys_dev) const {
     IndexDev ix;
     ix.top = top.as<uint64_t>();
@@ -350,6 +351,8 @@ struct Context {
     ib.ntop = ntop;
     ib.nseg = nseg;
     ib.ndir = (int)dir.size();
+    ib.any_wide = false;
+    for (uint32_t w : wide) ib.any_wide = ib.any_wide || w != 0;
     return CGCM_OK;
   }
 
@@ -393,7 +396,7 @@ struct Context {
       const uint64_t *depoch = dsize + (size_t)n;
       const int32_t *dold = tmp2.as<int32_t>();
       const uint32_t *dflags = reinterpret_cast<const uint32_t *>(dold + n);
-      launch_remap(n, dold, dsize, dflags, depoch, rec.as<UnitRec>(), nrec.as<UnitRec>(), main);
+      launch_remap(n, dold, nbase.as<uint64_t>(), dsize, dflags, depoch, rec.as<UnitRec>(), nrec.as<UnitRec>(), main);
       st.kernel_launches += 1;
       CK(cudaGetLastError());
       CK(cudaStreamSynchronize(main));
@@ -475,6 +478,7 @@ struct Context {
     std::memset(&a, 0, sizeof(a));
     a.rec = rec.as<UnitRec>();
     a.fx = fwd.view(dbase.as<uint64_t>());
+    a.fx_nowide = fwd.any_wide ? 0 : 1;
     if (c.dir == DIR_REV) {
       a.rx = rev.view(rev.keys.as<uint64_t>());
       a.runpay = rev.pay.as<uint64_t>();
@@ -678,10 +682,12 @@ struct Context {
         devbases[q] = it->second.devbase;
       }
     }
+    std::vector<uint64_t> deltas(units.size());
+    for (size_t q = 0; q < units.size(); ++q) deltas[q] = devbases[q] - by_idx[units[q]]->first;
     CKS(upload(up_units, units));
-    CKS(upload(up_vals, devbases));
-    launch_set_devbase(up_units.as<uint32_t>(), up_vals.as<uint64_t>(), (int)units.size(), rec.as<UnitRec>(), epoch,
-                       (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
+    CKS(upload(up_vals, deltas));
+    launch_set_delta(up_units.as<uint32_t>(), up_vals.as<uint64_t>(), (int)units.size(), rec.as<UnitRec>(), epoch,
+                     (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
     CK(cudaEventRecord(ev_copy, main));  // the copies wait for everything the main stream did before
@@ -1195,7 +1201,7 @@ int cgcm_setContext(void *ctx) {
 
 // ---- registration --------------------------------------------------------------------------
 static int declare_one(Context *C, uint64_t b, uint64_t s, uint32_t fl, const char *name) {
-  if (b == 0 || s == 0 || b + s < b || s > MAX_UNIT_SIZE) return CGCM_E_INVALID;
+  if (b == 0 || s == 0 || b + s < b || b + s >= ADDR_LIMIT) return CGCM_E_INVALID;
   auto succ = C->reg.lower_bound(b);
   if (succ != C->reg.end() && succ->first < b + s) return CGCM_E_OVERLAP;
   if (succ != C->reg.begin()) {
@@ -1230,7 +1236,7 @@ int cgcm_declareBatch(void *const *bases, const size_t *sizes, size_t n, unsigne
   std::sort(ord.begin(), ord.end(), [&](size_t a, size_t b) { return B(a) < B(b); });
   for (size_t q = 0; q < n; ++q) {  // validate everything first (all-or-nothing)
     uint64_t b = B(ord[q]), s = sizes[ord[q]];
-    if (b == 0 || s == 0 || b + s < b || s > MAX_UNIT_SIZE) return CGCM_E_INVALID;
+    if (b == 0 || s == 0 || b + s < b || b + s >= ADDR_LIMIT) return CGCM_E_INVALID;
     if (q + 1 < n && b + s > B(ord[q + 1])) return CGCM_E_OVERLAP;
     auto succ = C->reg.lower_bound(b);
     if (succ != C->reg.end() && succ->first < b + s) return CGCM_E_OVERLAP;
@@ -1834,11 +1840,11 @@ int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
   for (size_t i = 0; i < m; ++i) {
     const UnitRec &r = recs[i];
     cgcm_unit_t &u = out[i];
-    const uint32_t fl = rec_flags(r.szf);
+    const uint32_t fl = rec_flags(r.endf);
     u.base = C->by_idx[i]->first;
-    u.size = rec_size(r.szf);
+    u.size = rec_end(r.endf) - u.base;
     bool act = r.refcount > 0;
-    u.devptr = (act || ((fl & UF_GLOBAL) && (fl & UF_STORAGE))) ? r.devbase : 0;
+    u.devptr = ((fl & UF_STORAGE) && (act || (fl & UF_GLOBAL))) ? u.base + r.delta : 0;
     u.refCount = r.refcount;
     u.epoch = r.epoch;
     u.flags = ((fl & UF_GLOBAL) ? CGCM_UNIT_GLOBAL : 0) | ((fl & UF_READONLY) ? CGCM_UNIT_READONLY : 0) |
