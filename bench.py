@@ -62,7 +62,7 @@ def start_clock_sampler(uuid: str | None):
     cmd = ["nvidia-smi", "--query-gpu=uuid,clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
            "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
            "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
-           "--format=csv,noheader,nounits", "-lms", "100"]
+           "--format=csv,noheader,nounits", "-lms", "20"]
     if uuid:
         cmd[1:1] = ["-i", uuid]
     try:
