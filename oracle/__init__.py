@@ -82,6 +82,7 @@ def lib():
             "ref_devLookup": (C.c_int, [vp, u64, pu64, pu64]),
             "ref_kernel_scale": (C.c_int, [vp, u64, u64, u64, C.c_double]),
             "ref_kernel_treesum_level": (C.c_int, [vp, u64, u64, u64, u64, u64]),
+            "ref_kernel_gemm_rows": (C.c_int, [vp, u64, u64, u64, u64, u64, u64, C.c_double, C.c_double]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -243,3 +244,6 @@ class Oracle:
 
     def kernel_treesum_level(self, child_dev, root_dev, nnodes, lo, hi):
         return self.L.ref_kernel_treesum_level(self.h, child_dev, root_dev, nnodes, lo, hi)
+
+    def kernel_gemm_rows(self, A, B, Cm, n, row0, nrows, alpha, beta):
+        return self.L.ref_kernel_gemm_rows(self.h, A, B, Cm, n, row0, nrows, alpha, beta)

@@ -644,4 +644,24 @@ int ref_kernel_treesum_level(void *h, uint64_t child_dev, uint64_t root_dev, uin
   return 0;
 }
 
+// S2: PolyBench-shaped gemm on jagged fp64 matrices (config B), long-double accumulation.
+int ref_kernel_gemm_rows(void *h, uint64_t A_rows, uint64_t B_rows, uint64_t C_rows, uint64_t n, uint64_t row0,
+                         uint64_t nrows, double alpha, double beta) {
+  Oracle *o = O(h);
+  std::vector<u64> brow(n);
+  for (u64 k = 0; k < n; ++k) brow[k] = o->dev.get64(B_rows + 8 * k);
+  for (u64 i = row0; i < row0 + nrows && i < n; ++i) {
+    u64 arow = o->dev.get64(A_rows + 8 * i), crow = o->dev.get64(C_rows + 8 * i);
+    std::vector<double> a(n);
+    o->dev.read(arow, a.data(), 8 * n);
+    for (u64 j = 0; j < n; ++j) {
+      long double acc = 0.0L;
+      for (u64 k = 0; k < n; ++k) acc += (long double)a[k] * (long double)o->dev.getf(brow[k] + 8 * j);
+      double c = o->dev.getf(crow + 8 * j);
+      o->dev.putf(crow + 8 * j, (double)((long double)alpha * acc + (long double)beta * (long double)c));
+    }
+  }
+  return 0;
+}
+
 }  // extern "C"

@@ -105,6 +105,10 @@ int ref_devLookup(void *h, uint64_t g, uint64_t *base, uint64_t *devptr);
 int ref_kernel_scale(void *h, uint64_t rows_dev, uint64_t nrows, uint64_t ncols, double alpha);
 int ref_kernel_treesum_level(void *h, uint64_t child_dev, uint64_t root_dev, uint64_t nnodes,
                              uint64_t lo, uint64_t hi);
+/* S2 (config B): C[i][j] = alpha * sum_k A[i][k]*B[k][j] + beta * C[i][j] for rows [row0, row0+nrows),
+   through translated row pointers; accumulated in long double (the accurate reference, A21) */
+int ref_kernel_gemm_rows(void *h, uint64_t A_rows, uint64_t B_rows, uint64_t C_rows, uint64_t n, uint64_t row0,
+                         uint64_t nrows, double alpha, double beta);
 
 #ifdef __cplusplus
 }

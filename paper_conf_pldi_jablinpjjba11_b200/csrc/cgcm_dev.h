@@ -7,35 +7,43 @@
 
 namespace cgcm {
 
-// Allocation-unit record (D3): one 32-byte sector per unit, indexed by the unit's rank
-// in base order.  The first 16 bytes are everything a forward translation needs (one 16-byte
-// gather):
-//   endf    = base + size (bits 0..56) | flags (bits 57..63)   -- acceptance: p <= end (A7)
-//   delta   = devbase - base (mod 2^64), valid iff UF_STORAGE   -- translation: p + delta (Alg. 1)
-//   epoch   = Alg. 2's per-unit epoch
-//   refcount (Alg. 1/3)
-// The base itself lives in the sorted key array of the forward index.
-struct __align__(32) UnitRec {
-  uint64_t endf;
-  uint64_t delta;
-  uint64_t epoch;
-  int32_t refcount;
-  uint32_t pad;
+// The allocation-unit table (D3) as columns indexed by the unit's rank in base order.
+// A forward translation touches one 8-byte word per slot (hot) plus the refcount reduction:
+//   hot[u]   = size (bits 0..31; 0xFFFFFFFF = see size64) | extent id (bits 32..55) | flags (56..63)
+//   rc[u]    = refCount (i32, Alg. 1/3)
+//   epoch[u] = Alg. 2's per-unit epoch, u32 relative to the context's epoch origin (A28)
+//   base[u]  = the sorted key array of the forward index; size64[u] = full size (cold)
+//   ext_delta[e] = devbase - base for every unit copy in device extent e (mirrored layout):
+//              translation = p + ext_delta[extent(u)]  (Alg. 1: devptr + (ptr - base))
+struct TableDev {
+  uint64_t *hot;
+  int32_t *rc;
+  uint32_t *epoch;
+  const uint64_t *base;
+  const uint64_t *size64;
+  const uint64_t *ext_delta;
+  int n_ext;
 };
-static_assert(sizeof(UnitRec) == 32, "UnitRec must be one sector");
 
 enum : uint32_t {
   UF_GLOBAL = 1u,       // declareGlobal: named region persists (A14)
   UF_READONLY = 2u,     // never copied back (Alg. 2)
   UF_ARRAYMAPPED = 4u,  // device copy holds translated pointers (A12)
   UF_ACTIVE = 8u,       // refcount > 0 at the start of the current call (stable during a call)
-  UF_STORAGE = 16u      // delta (device copy) valid
+  UF_STORAGE = 16u      // the unit has a device copy (extent id valid)
 };
-constexpr int FSHIFT = 57;
-constexpr uint64_t ADDR_MASK = (1ull << FSHIFT) - 1;
-constexpr uint64_t ADDR_LIMIT = ADDR_MASK;  // base + size must stay below 2^57 (A26)
-__host__ __device__ __forceinline__ uint64_t rec_end(uint64_t endf) { return endf & ADDR_MASK; }
-__host__ __device__ __forceinline__ uint32_t rec_flags(uint64_t endf) { return (uint32_t)(endf >> FSHIFT); }
+constexpr int FSHIFT = 56;
+constexpr int ESHIFT = 32;
+constexpr uint64_t EXT_MASK = (1ull << 24) - 1;
+constexpr uint64_t NO_EXT = EXT_MASK;
+constexpr uint32_t BIG_SIZE = 0xFFFFFFFFu;
+constexpr uint64_t ADDR_LIMIT = (1ull << 57) - 1;  // base + size must stay below 2^57 (A26)
+__host__ __device__ __forceinline__ uint32_t hot_size32(uint64_t h) { return (uint32_t)h; }
+__host__ __device__ __forceinline__ uint32_t hot_ext(uint64_t h) { return (uint32_t)((h >> ESHIFT) & EXT_MASK); }
+__host__ __device__ __forceinline__ uint32_t hot_flags(uint64_t h) { return (uint32_t)(h >> FSHIFT); }
+__host__ __device__ __forceinline__ uint64_t make_hot(uint64_t size, uint64_t ext, uint32_t flags) {
+  return (size >= BIG_SIZE ? (uint64_t)BIG_SIZE : size) | ((ext & EXT_MASK) << ESHIFT) | ((uint64_t)flags << FSHIFT);
+}
 
 // Sorted-key search index, built by the host (top level, directory) and the device (levels):
 //   keys      n sorted u64 (AU bases for the forward index, extent device starts for the reverse)
@@ -48,9 +56,10 @@ __host__ __device__ __forceinline__ uint32_t rec_flags(uint64_t endf) { return (
 // A lookup = dir (2 LDS) + ~1 LDS search step + top (1 LDS) + h sector gathers.
 constexpr int MAXL = 6;
 constexpr int TOPMAX = 16384;
-constexpr int DIRMAX = 16384;
+constexpr int DIRMAX = 12288;
 constexpr int MAXSEG = 32;
 constexpr int RUN_SMEM = 1024;  // extents staged in shared memory for reverse lookups
+constexpr int EXT_SMEM = 2048;  // extent deltas staged in shared memory for forward translations
 
 struct IndexDev {
   const uint64_t *top;
@@ -79,9 +88,10 @@ struct Status {
 // gate journal entry: the unit whose epoch this call changed, its old epoch, and whether it needs
 // a copy-back (stale and not read-only)
 struct __align__(16) Journal {
-  uint64_t old_epoch;
+  uint32_t old_epoch;
   uint32_t unit;
   uint32_t copy;
+  uint32_t pad;
 };
 
 // outer-pointer lookup result (mapArray & friends)
@@ -92,8 +102,7 @@ struct PointInfo {
 };
 
 // single-unit bookkeeping ops applied by k_unit_ops (one thread per op)
-enum : uint32_t { UOP_ADD_RC = 1, UOP_SET_EPOCH = 2, UOP_OR_FLAGS = 3, UOP_AND_FLAGS = 4,
-                  UOP_SET_DEVBASE = 5, UOP_SET_RC = 6 };
+enum : uint32_t { UOP_ADD_RC = 1, UOP_SET_EPOCH = 2, UOP_OR_FLAGS = 3, UOP_AND_FLAGS = 4, UOP_SET_RC = 6 };
 struct UnitOp {
   uint32_t unit, op;
   uint64_t val;
@@ -117,15 +126,16 @@ enum : int { SEL_ALL = 0, SEL_HIT = 1, SEL_NOTHIT = 2 };
 struct SlotArgs {
   IndexDev fx;                 // forward index over unit bases
   IndexDev rx;                 // reverse index over device extents (DIR_REV)
-  const uint64_t *runpay;      // per extent: host - device address delta (mirrored layout)
-  UnitRec *rec;
+  const uint64_t *runpay;      // per sorted extent: host - device address delta (mirrored layout)
+  const uint32_t *runid;       // per sorted extent: its extent id
+  TableDev tab;
   const Seg *segs;
   const uint64_t *seg_chunk0;  // [nseg+1] prefix of 2-slot chunks per segment
   int nseg;
   int sel;
   uint64_t nchunks;
   uint32_t *hitmask;           // 2 bits per chunk: slot m of the chunk was translated
-  uint64_t epoch;
+  uint32_t epoch;               // globalEpoch - origin
   Status *st;
   unsigned long long *lc;      // shared list counters of the call: [0] act, [1] journal, [2] free, [3] copy
   uint32_t *act_list;
@@ -141,18 +151,18 @@ struct SlotArgs {
 int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s);
 void launch_build_levels(const uint64_t *keys, int n, int h, const uint32_t *wide, uint32_t *const *lvl,
                          const size_t *lvl_cap, cudaStream_t s);
-void launch_remap(int n, const int32_t *old_idx, const uint64_t *base, const uint64_t *size, const uint32_t *flags,
-                  const uint64_t *epoch0, const UnitRec *old_rec, UnitRec *new_rec, cudaStream_t s);
+void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags, const uint32_t *epoch0,
+                  TableDev old_tab, TableDev new_tab, cudaStream_t s);
 size_t sort_keys_temp_bytes(int n);
 void launch_sort_keys(void *temp, size_t temp_bytes, const uint32_t *kin, uint32_t *kout, int n, cudaStream_t s);
-void launch_unit_ops(const UnitOp *ops, int n, UnitRec *rec, cudaStream_t s);
-void launch_set_delta(const uint32_t *units, const uint64_t *deltas, int n, UnitRec *rec, uint64_t epoch,
-                      int set_epoch, cudaStream_t s);
-void launch_deactivate(const uint32_t *units, int n, UnitRec *rec, cudaStream_t s);
-void launch_restore_epochs(const Journal *j, int n, UnitRec *rec, cudaStream_t s);
-void launch_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t *ptrs, int n, PointInfo *out,
-                          cudaStream_t s);
-void launch_release_scan(const UnitRec *rec, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
+void launch_unit_ops(const UnitOp *ops, int n, TableDev tab, cudaStream_t s);
+void launch_set_ext(const uint32_t *units, const uint32_t *exts, int n, TableDev tab, uint32_t epoch, int set_epoch,
+                    cudaStream_t s);
+void launch_deactivate(const uint32_t *units, int n, TableDev tab, cudaStream_t s);
+void launch_restore_epochs(const Journal *j, int n, TableDev tab, cudaStream_t s);
+void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n, PointInfo *out, cudaStream_t s);
+void launch_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
                          cudaStream_t s);
+void launch_rebase_epochs(TableDev tab, int n, uint32_t cur, cudaStream_t s);
 
 }  // namespace cgcm

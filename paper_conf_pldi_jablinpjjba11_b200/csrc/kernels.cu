@@ -90,15 +90,23 @@ __device__ __forceinline__ uint32_t spread16(uint32_t x) {
   return x;
 }
 
-// number of entries <= r among 8 sorted u32 (one 32-byte level sector)
-__device__ __forceinline__ int count8(const uint64_t w[4], uint32_t r) {
+// number of entries <= r among 8 sorted u32 (one 32-byte level sector), and the largest of them
+__device__ __forceinline__ int count8(const uint64_t w[4], uint32_t r, uint32_t &last) {
   int c = 0;
 #pragma unroll
   for (int q = 0; q < 4; ++q) {
-    c += ((uint32_t)w[q] <= r);
-    c += ((uint32_t)(w[q] >> 32) <= r);
+    const uint32_t lo = (uint32_t)w[q], hi = (uint32_t)(w[q] >> 32);
+    if (lo <= r) last = lo;
+    if (hi <= r) last = hi;
+    c += (lo <= r);
+    c += (hi <= r);
   }
   return c;
+}
+__device__ __forceinline__ uint64_t ld_u64(const uint64_t *p, uint64_t pol) {
+  uint64_t v;
+  asm volatile("ld.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+  return v;
 }
 
 // ---- an index's top level, staged in shared memory -------------------------------------------
@@ -109,6 +117,7 @@ struct SIdx {
   const uint64_t *skmin;
   const uint32_t *smeta;
   const uint64_t *pay;  // reverse index with h == 0: per-extent delta, staged
+  const uint32_t *rid;  // ... and the extent ids
   int ntop, nseg;
   uint64_t kfirst;
 };
@@ -117,12 +126,12 @@ __host__ __device__ __forceinline__ size_t al16(size_t x) { return (x + 15) & ~s
 __host__ __device__ __forceinline__ size_t stage_bytes(const IndexDev &ix, bool with_pay) {
   size_t b = al16(8 * (size_t)ix.ntop) + al16(4 * (size_t)ix.ndir) + al16(4 * (size_t)((ix.ntop + 31) / 32)) +
              al16(8 * (size_t)ix.nseg) + al16(16 * (size_t)ix.nseg);
-  if (with_pay) b += al16(8 * (size_t)ix.ntop);
+  if (with_pay) b += al16(8 * (size_t)ix.ntop) + al16(4 * (size_t)ix.ntop);
   return b;
 }
 
-__device__ __forceinline__ unsigned char *stage(const IndexDev &ix, const uint64_t *pay, unsigned char *base,
-                                                SIdx &S) {
+__device__ __forceinline__ unsigned char *stage(const IndexDev &ix, const uint64_t *pay, const uint32_t *rid,
+                                                unsigned char *base, SIdx &S) {
   uint64_t *top = reinterpret_cast<uint64_t *>(base);
   base += al16(8 * (size_t)ix.ntop);
   uint32_t *dir = reinterpret_cast<uint32_t *>(base);
@@ -134,9 +143,12 @@ __device__ __forceinline__ unsigned char *stage(const IndexDev &ix, const uint64
   uint32_t *smeta = reinterpret_cast<uint32_t *>(base);
   base += al16(16 * (size_t)ix.nseg);
   uint64_t *spay = nullptr;
+  uint32_t *srid = nullptr;
   if (pay) {
     spay = reinterpret_cast<uint64_t *>(base);
     base += al16(8 * (size_t)ix.ntop);
+    srid = reinterpret_cast<uint32_t *>(base);
+    base += al16(4 * (size_t)ix.ntop);
   }
   for (int t = threadIdx.x; t < ix.ntop; t += blockDim.x) top[t] = ix.top[t];
   for (int t = threadIdx.x; t < ix.ndir; t += blockDim.x) dir[t] = ix.dir[t];
@@ -144,13 +156,17 @@ __device__ __forceinline__ unsigned char *stage(const IndexDev &ix, const uint64
   for (int t = threadIdx.x; t < ix.nseg; t += blockDim.x) skmin[t] = ix.seg_kmin[t];
   for (int t = threadIdx.x; t < 4 * ix.nseg; t += blockDim.x) smeta[t] = ix.seg_meta[t];
   if (pay)
-    for (int t = threadIdx.x; t < ix.ntop; t += blockDim.x) spay[t] = pay[t];
+    for (int t = threadIdx.x; t < ix.ntop; t += blockDim.x) {
+      spay[t] = pay[t];
+      srid[t] = rid[t];
+    }
   S.top = top;
   S.dir = dir;
   S.wide = wide;
   S.skmin = skmin;
   S.smeta = smeta;
   S.pay = spay;
+  S.rid = srid;
   S.ntop = ix.ntop;
   S.nseg = ix.nseg;
   S.kfirst = ix.ntop > 0 ? ix.top[0] : ~0ull;
@@ -195,8 +211,8 @@ __device__ __forceinline__ int top_search(const SIdx &S, uint64_t p, uint64_t &t
 // fixed-depth variant of level_lookup2 for indexes without wide buckets (the hot path)
 template <int H>
 __device__ __forceinline__ void level_lookup2_fixed(const IndexDev &ix, uint64_t pol, const uint64_t p[2], int j[2],
-                                                    const uint64_t key[2]) {
-  uint32_t rel[2];
+                                                    uint64_t key[2]) {
+  uint32_t rel[2], last[2] = {0, 0};
   bool ok[2];
 #pragma unroll
   for (int m = 0; m < 2; ++m) {
@@ -211,20 +227,22 @@ __device__ __forceinline__ void level_lookup2_fixed(const IndexDev &ix, uint64_t
     uint64_t w0[4], w1[4];
     ld_sector(L + 8 * (size_t)j[0], pol, w0);
     ld_sector(L + 8 * (size_t)j[1], pol, w1);
-    j[0] = 8 * j[0] + count8(w0, rel[0]) - 1;
-    j[1] = 8 * j[1] + count8(w1, rel[1]) - 1;
+    j[0] = 8 * j[0] + count8(w0, rel[0], last[0]) - 1;
+    j[1] = 8 * j[1] + count8(w1, rel[1], last[1]) - 1;
   }
 #pragma unroll
-  for (int m = 0; m < 2; ++m)
+  for (int m = 0; m < 2; ++m) {
+    key[m] += last[m];
     if (!ok[m]) j[m] = -1;
+  }
 }
 
 // two interleaved greatestLTE lookups through the u32 sector levels.  In: j = t, key = top[t]
 // from top_search (j < 0: no candidate).  Out: j = key index (or -1).
 __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix, uint64_t pol, const uint64_t p[2],
-                                              int j[2], const uint64_t key[2]) {
+                                              int j[2], uint64_t key[2]) {
   if (ix.h == 0) return;
-  uint32_t rel[2];
+  uint32_t rel[2], last[2] = {0, 0};
   bool wide[2];
   int t0[2];
 #pragma unroll
@@ -241,12 +259,13 @@ __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix,
     uint64_t w0[4], w1[4];
     ld_sector(L + 8 * (size_t)j[0], pol, w0);
     ld_sector(L + 8 * (size_t)j[1], pol, w1);
-    j[0] = 8 * j[0] + count8(w0, rel[0]) - 1;
-    j[1] = 8 * j[1] + count8(w1, rel[1]) - 1;
+    j[0] = 8 * j[0] + count8(w0, rel[0], last[0]) - 1;
+    j[1] = 8 * j[1] + count8(w1, rel[1], last[1]) - 1;
   }
   const int sh = 3 * ix.h;
 #pragma unroll
   for (int m = 0; m < 2; ++m) {
+    key[m] += last[m];
     if (t0[m] < 0) {
       j[m] = -1;
     } else if (wide[m]) {  // bucket spanning >= 4 GiB: binary search over the full u64 keys
@@ -257,6 +276,7 @@ __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix,
         len -= half;
       }
       j[m] = lo;
+      key[m] = ix.keys[lo];
     }
   }
 }
@@ -274,15 +294,19 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ uint64_t s_seg0[SEG_SMEM + 1];
   SIdx F, R;
-  unsigned char *sp = stage(a.fx, nullptr, smem, F);
-  if (DIR == DIR_REV) stage(a.rx, a.rx.h == 0 ? a.runpay : nullptr, sp, R);
+  unsigned char *sp = stage(a.fx, nullptr, nullptr, smem, F);
+  if (DIR == DIR_REV) sp = stage(a.rx, a.rx.h == 0 ? a.runpay : nullptr, a.runid, sp, R);
+  // extent deltas (devbase - base of every copy in the extent), staged when few
+  const bool ext_s = a.tab.n_ext <= EXT_SMEM;
+  uint64_t *s_ext = reinterpret_cast<uint64_t *>(sp);
+  if (ext_s)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
   const int nseg_s = a.nseg <= SEG_SMEM ? a.nseg : 0;
   for (int t = threadIdx.x; t <= nseg_s; t += blockDim.x) s_seg0[t] = a.seg_chunk0[t];
   __syncthreads();
 
   const uint64_t pol_s = policy_evict_first();
   const uint64_t pol_t = policy_evict_last();
-  constexpr bool FULLREC = (DIR == DIR_REV) || (OPS & (OP_GATE | OP_CHECKMAPPED));
   const int lane = threadIdx.x & 31;
   // single-segment calls (the common case) keep the segment in registers
   Seg seg1 = a.segs[0];
@@ -340,6 +364,7 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
 
     // ---- a1: lookups ----
     uint64_t q[2], key[2], dx[2] = {0, 0};
+    uint32_t rid[2] = {0, 0};
     int j[2];
     bool look[2];
 #pragma unroll
@@ -358,8 +383,12 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
       if (a.rx.h > 0) level_lookup2(R, a.rx, pol_t, q, j, key);
 #pragma unroll
       for (int m = 0; m < 2; ++m) {
-        if (j[m] >= 0) dx[m] = a.rx.h == 0 ? R.pay[j[m]] : a.runpay[j[m]];
-        else look[m] = false;
+        if (j[m] >= 0) {
+          dx[m] = a.rx.h == 0 ? R.pay[j[m]] : a.runpay[j[m]];
+          rid[m] = a.rx.h == 0 ? R.rid[j[m]] : a.runid[j[m]];
+        } else {
+          look[m] = false;
+        }
         q[m] = look[m] ? q[m] + dx[m] : 0ull;  // host address
       }
     }
@@ -372,39 +401,44 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
     if constexpr (FH > 0) level_lookup2_fixed<FH>(a.fx, pol_t, q, j, key);
     else if constexpr (FH < 0) level_lookup2(F, a.fx, pol_t, q, j, key);
 
-    // ---- record gathers: {end|flags, delta} (+ {epoch, refcount}) ----
-    uint64_t r[2][4];
+    // ---- the unit's hot word: size | extent | flags ----
+    uint64_t hw[2] = {0, 0};
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
       look[m] = look[m] && j[m] >= 0;
-      r[m][0] = r[m][1] = r[m][2] = r[m][3] = 0;
-      if (look[m]) {
-        if (FULLREC) ld_sector(a.rec + j[m], pol_t, r[m]);
-        else ld_pair(a.rec + j[m], pol_t, r[m][0], r[m][1]);
-      }
+      if (look[m]) hw[m] = ld_u64(a.tab.hot + j[m], pol_t);
     }
     bool hit[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      hit[m] = look[m] && q[m] <= rec_end(r[m][0]);  // A7: p - base <= size
+      uint64_t sz = hot_size32(hw[m]);
+      if (look[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
+      hit[m] = look[m] && (q[m] - key[m] <= sz);  // A7: p - base <= size
       if (DIR == DIR_REV && look[m]) {
-        // the unit must own this extent's copy: active, and its copy mirrors the extent
-        if (!(hit[m] && (rec_flags(r[m][0]) & UF_ACTIVE) && r[m][1] + dx[m] == 0)) {
+        // the unit must own this extent's copy: active, and its copy lives in that extent
+        if (!(hit[m] && (hot_flags(hw[m]) & UF_ACTIVE) && hot_ext(hw[m]) == rid[m])) {
           hit[m] = false;
-          if (j[m] > 0) {  // one past the end of the previous unit (A7)
-            uint64_t r2[4];
-            ld_sector(a.rec + (j[m] - 1), pol_t, r2);
-            if ((rec_flags(r2[0]) & UF_ACTIVE) && r2[1] + dx[m] == 0 && q[m] == rec_end(r2[0])) {
+          if (j[m] > 0 && q[m] == key[m]) {  // one past the end of the previous unit (A7)
+            const uint64_t h2 = a.tab.hot[j[m] - 1], b2 = a.tab.base[j[m] - 1];
+            uint64_t s2 = hot_size32(h2);
+            if (s2 == BIG_SIZE) s2 = a.tab.size64[j[m] - 1];
+            if ((hot_flags(h2) & UF_ACTIVE) && hot_ext(h2) == rid[m] && q[m] == b2 + s2) {
               hit[m] = true;
               j[m] -= 1;
-              r[m][0] = r2[0];
-              r[m][1] = r2[1];
-              r[m][2] = r2[2];
-              r[m][3] = r2[3];
+              key[m] = b2;
+              hw[m] = h2;
             }
           }
         }
       }
+    }
+    // epoch (gate) and refcount (unmap check) columns, only where the operation needs them
+    uint32_t ep[2] = {0, 0};
+    int32_t rcv[2] = {0, 0};
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      if ((OPS & OP_GATE) && hit[m]) ep[m] = a.tab.epoch[j[m]];
+      if ((OPS & OP_CHECKMAPPED) && hit[m]) rcv[m] = a.tab.rc[j[m]];
     }
 
     // ---- a2/a3/a4 operations ----
@@ -419,41 +453,41 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
       c_hits += hm;
       c_miss += (vm && !nul && !hm);
       const int unit = hm ? j[m] : 0;
-      UnitRec *Rp = a.rec + unit;
-      const uint32_t fl = rec_flags(r[m][0]);
-      if (OPS & OP_CHECKMAPPED) c_notm += (hm && (int32_t)(uint32_t)r[m][3] <= 0);
+      int32_t *RC = a.tab.rc + unit;
+      const uint32_t fl = hot_flags(hw[m]);
+      if (OPS & OP_CHECKMAPPED) c_notm += (hm && rcv[m] <= 0);
       bool act = false;
       if (OPS & OP_INC) {
         if (hm) {
           if (fl & UF_ACTIVE) {
-            red_add(&Rp->refcount, sg.inc);
+            red_add(RC, sg.inc);
           } else {
-            int old = atomicAdd(&Rp->refcount, sg.inc);
+            int old = atomicAdd(RC, sg.inc);
             act = (old == 0);  // refcount 0 -> 1: Alg. 1's activation
           }
         }
       }
       if (OPS & OP_INCPLAIN)
-        if (hm) red_add(&Rp->refcount, sg.inc);
+        if (hm) red_add(RC, sg.inc);
       if (OPS & OP_DECPLAIN)
-        if (hm) red_add(&Rp->refcount, -sg.inc);
+        if (hm) red_add(RC, -sg.inc);
       bool freed = false;
       if (OPS & OP_DEC) {
         if (hm) {
           if (a.dec_red) {
-            red_add(&Rp->refcount, -sg.inc);
+            red_add(RC, -sg.inc);
           } else {
-            int old = atomicAdd(&Rp->refcount, -sg.inc);
+            int old = atomicAdd(RC, -sg.inc);
             c_under += (old < sg.inc);
             freed = (old == sg.inc);  // refcount 1 -> 0: Alg. 3's cuMemFree
           }
         }
       }
       bool gated = false;
-      uint64_t old_ep = 0;
+      uint32_t old_ep = 0;
       if (OPS & OP_GATE) {
-        if (hm && r[m][2] != a.epoch) {
-          old_ep = atomicExch(reinterpret_cast<unsigned long long *>(&Rp->epoch), (unsigned long long)a.epoch);
+        if (hm && ep[m] != a.epoch) {
+          old_ep = atomicExch(a.tab.epoch + unit, a.epoch);
           gated = (old_ep != a.epoch);
         }
       }
@@ -461,7 +495,8 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
         if (hm) {
           if (DIR == DIR_FWD) {
             if (fl & UF_STORAGE) {
-              outv[m] = q[m] + r[m][1];  // Alg. 1: info.devptr + (ptr - info.base)
+              const uint32_t e = hot_ext(hw[m]);
+              outv[m] = q[m] + (ext_s ? s_ext[e] : a.tab.ext_delta[e]);  // Alg. 1: devptr + (ptr - base)
               wrote |= 1u << m;
             } else {
               c_pend += 1;  // activated by this call: completed after the allocation
@@ -491,6 +526,7 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
           jn.old_epoch = old_ep;
           jn.unit = (uint32_t)unit;
           jn.copy = cp ? 1u : 0u;
+          jn.pad = 0;
           a.journal[ix] = jn;
         }
         unsigned long long cx = warp_append(&a.lc[3], cp);
@@ -562,24 +598,32 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
   X(DIR_REV, OP_DECPLAIN)                              /* rollback of REV INCPLAIN               */
 
 static size_t slots_smem(const SlotArgs &a, int dir) {
-  return stage_bytes(a.fx, false) + (dir == DIR_REV ? stage_bytes(a.rx, a.rx.h == 0) : 0) + 64;
+  return stage_bytes(a.fx, false) + (dir == DIR_REV ? stage_bytes(a.rx, a.rx.h == 0) : 0) +
+         (a.tab.n_ext <= EXT_SMEM ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
 }
 
 template <int DIR, int OPS, int FH>
 static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
   size_t smem = slots_smem(a, DIR);
-  static size_t configured = 0;
-  if (smem > 48 * 1024 && smem > configured) {
-    cudaError_t e =
-        cudaFuncSetAttribute(k_slots<DIR, OPS, FH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return -1;
-    configured = smem;
+  // the 48 KiB default covers static + dynamic shared memory: opt in to the full carve-out once
+  static bool configured = false;
+  if (!configured) {
+    cudaFuncAttributes fa;
+    cudaError_t e = cudaFuncGetAttributes(&fa, k_slots<DIR, OPS, FH>);
+    if (e != cudaSuccess) return (int)e;
+    int dev = 0, optin = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    e = cudaFuncSetAttribute(k_slots<DIR, OPS, FH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             optin - (int)fa.sharedSizeBytes);
+    if (e != cudaSuccess) return (int)e;
+    configured = true;
   }
   uint64_t want = (a.nchunks + SLOT_THREADS - 1) / SLOT_THREADS;
   int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
   k_slots<DIR, OPS, FH><<<grid, SLOT_THREADS, smem, s>>>(a);
-  return cudaGetLastError() == cudaSuccess ? 0 : -1;
+  return (int)cudaGetLastError();  // 0 or the cudaError_t of the launch
 }
 
 // hot operation sets get depth-specialised forward lookups
@@ -640,29 +684,27 @@ void launch_build_levels(const uint64_t *keys, int n, int h, const uint32_t *wid
   }
 }
 
-// new_rec[i] = old_rec[old_idx[i]] (surviving unit) or a fresh record (declared since the last build)
-__global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *base, const uint64_t *size,
-                        const uint32_t *flags, const uint64_t *epoch0, const UnitRec *old_rec, UnitRec *new_rec) {
+// new table row i = old row old_idx[i] (surviving unit) or a fresh row (declared since the last build)
+__global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags,
+                        const uint32_t *epoch0, TableDev o, TableDev t) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  UnitRec r;
-  int o = old_idx[i];
-  if (o >= 0) {
-    r = old_rec[o];
+  int k = old_idx[i];
+  if (k >= 0) {
+    t.hot[i] = o.hot[k];
+    t.rc[i] = o.rc[k];
+    t.epoch[i] = o.epoch[k];
   } else {
-    r.endf = (base[i] + size[i]) | ((uint64_t)flags[i] << FSHIFT);
-    r.delta = 0;
-    r.epoch = epoch0[i];
-    r.refcount = 0;
-    r.pad = 0;
+    t.hot[i] = make_hot(size[i], NO_EXT, flags[i]);
+    t.rc[i] = 0;
+    t.epoch[i] = epoch0[i];
   }
-  new_rec[i] = r;
 }
-void launch_remap(int n, const int32_t *old_idx, const uint64_t *base, const uint64_t *size, const uint32_t *flags,
-                  const uint64_t *epoch0, const UnitRec *old_rec, UnitRec *new_rec, cudaStream_t s) {
+void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags, const uint32_t *epoch0,
+                  TableDev old_tab, TableDev new_tab, cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
-    k_remap<<<(n + 255) / 256, 256, 0, s>>>(n, old_idx, base, size, flags, epoch0, old_rec, new_rec);
+    k_remap<<<(n + 255) / 256, 256, 0, s>>>(n, old_idx, size, flags, epoch0, old_tab, new_tab);
   }
 }
 
@@ -678,110 +720,125 @@ void launch_sort_keys(void *temp, size_t temp_bytes, const uint32_t *kin, uint32
 // -------------------------------------------------------------------------------------------------
 // small bookkeeping kernels
 // -------------------------------------------------------------------------------------------------
-__device__ __forceinline__ unsigned *flag_word(UnitRec &r) {
-  return reinterpret_cast<unsigned *>(&r.endf) + 1;  // flags live in the top bits of the high word
+__device__ __forceinline__ unsigned *flag_word(uint64_t *hot) {
+  return reinterpret_cast<unsigned *>(hot) + 1;  // flags (and the extent id) live in the high word
 }
 
-__global__ void k_unit_ops(const UnitOp *ops, int n, UnitRec *rec) {
+__global__ void k_unit_ops(const UnitOp *ops, int n, TableDev tab) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   UnitOp o = ops[i];
-  UnitRec &r = rec[o.unit];
   switch (o.op) {
-    case UOP_ADD_RC: atomicAdd(&r.refcount, (int32_t)(int64_t)o.val); break;
-    case UOP_SET_EPOCH: r.epoch = o.val; break;
-    case UOP_OR_FLAGS: atomicOr(flag_word(r), (uint32_t)o.val << (FSHIFT - 32)); break;
+    case UOP_ADD_RC: atomicAdd(tab.rc + o.unit, (int32_t)(int64_t)o.val); break;
+    case UOP_SET_EPOCH: tab.epoch[o.unit] = (uint32_t)o.val; break;
+    case UOP_OR_FLAGS: atomicOr(flag_word(tab.hot + o.unit), (uint32_t)o.val << (FSHIFT - 32)); break;
     case UOP_AND_FLAGS:
-      atomicAnd(flag_word(r), ((uint32_t)o.val << (FSHIFT - 32)) | ((1u << (FSHIFT - 32)) - 1));
+      atomicAnd(flag_word(tab.hot + o.unit), ((uint32_t)o.val << (FSHIFT - 32)) | ((1u << (FSHIFT - 32)) - 1));
       break;
-    case UOP_SET_DEVBASE: r.delta = o.val; break;  // (a delta: devbase - base)
-    case UOP_SET_RC: r.refcount = (int32_t)(int64_t)o.val; break;
+    case UOP_SET_RC: tab.rc[o.unit] = (int32_t)(int64_t)o.val; break;
   }
 }
-void launch_unit_ops(const UnitOp *ops, int n, UnitRec *rec, cudaStream_t s) {
+void launch_unit_ops(const UnitOp *ops, int n, TableDev tab, cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
-    k_unit_ops<<<(n + 255) / 256, 256, 0, s>>>(ops, n, rec);
+    k_unit_ops<<<(n + 255) / 256, 256, 0, s>>>(ops, n, tab);
   }
 }
 
-__global__ void k_set_delta(const uint32_t *units, const uint64_t *deltas, int n, UnitRec *rec, uint64_t epoch,
-                            int set_epoch) {
+// activation: the unit's copy is in extent ext[i]; epoch = globalEpoch (A5 reading R1)
+__global__ void k_set_ext(const uint32_t *units, const uint32_t *exts, int n, TableDev tab, uint32_t epoch,
+                          int set_epoch) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  UnitRec &r = rec[units[i]];
-  r.delta = deltas[i];
-  r.endf |= (uint64_t)(UF_STORAGE | UF_ACTIVE) << FSHIFT;
-  if (set_epoch) r.epoch = epoch;  // A5 reading R1: an AU is coherent when it becomes active
+  const uint32_t u = units[i];
+  uint64_t h = tab.hot[u];
+  h = (h & ~(EXT_MASK << ESHIFT)) | ((uint64_t)(exts[i] & EXT_MASK) << ESHIFT);
+  h |= (uint64_t)(UF_STORAGE | UF_ACTIVE) << FSHIFT;
+  tab.hot[u] = h;
+  if (set_epoch) tab.epoch[u] = epoch;
 }
-void launch_set_delta(const uint32_t *units, const uint64_t *deltas, int n, UnitRec *rec, uint64_t epoch,
-                      int set_epoch, cudaStream_t s) {
+void launch_set_ext(const uint32_t *units, const uint32_t *exts, int n, TableDev tab, uint32_t epoch, int set_epoch,
+                    cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
-    k_set_delta<<<(n + 255) / 256, 256, 0, s>>>(units, deltas, n, rec, epoch, set_epoch);
+    k_set_ext<<<(n + 255) / 256, 256, 0, s>>>(units, exts, n, tab, epoch, set_epoch);
   }
 }
 
-__global__ void k_deactivate(const uint32_t *units, int n, UnitRec *rec) {
+__global__ void k_deactivate(const uint32_t *units, int n, TableDev tab) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  UnitRec &r = rec[units[i]];
-  if (r.refcount != 0) return;
-  if (rec_flags(r.endf) & UF_GLOBAL) {
-    r.endf &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE) << FSHIFT);  // named region persists
+  const uint32_t u = units[i];
+  if (tab.rc[u] != 0) return;
+  uint64_t h = tab.hot[u];
+  if (hot_flags(h) & UF_GLOBAL) {
+    h &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE) << FSHIFT);  // named region persists
   } else {
-    r.delta = 0;  // cuMemFree (Alg. 3)
-    r.endf &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE | UF_STORAGE) << FSHIFT);
+    h &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE | UF_STORAGE) << FSHIFT);  // cuMemFree (Alg. 3)
+    h |= NO_EXT << ESHIFT;
   }
+  tab.hot[u] = h;
 }
-void launch_deactivate(const uint32_t *units, int n, UnitRec *rec, cudaStream_t s) {
+void launch_deactivate(const uint32_t *units, int n, TableDev tab, cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
-    k_deactivate<<<(n + 255) / 256, 256, 0, s>>>(units, n, rec);
+    k_deactivate<<<(n + 255) / 256, 256, 0, s>>>(units, n, tab);
   }
 }
 
-__global__ void k_restore_epochs(const Journal *j, int n, UnitRec *rec) {
+__global__ void k_restore_epochs(const Journal *j, int n, TableDev tab) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  rec[j[i].unit].epoch = j[i].old_epoch;
+  tab.epoch[j[i].unit] = j[i].old_epoch;
 }
-void launch_restore_epochs(const Journal *j, int n, UnitRec *rec, cudaStream_t s) {
+void launch_restore_epochs(const Journal *j, int n, TableDev tab, cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
-    k_restore_epochs<<<(n + 255) / 256, 256, 0, s>>>(j, n, rec);
+    k_restore_epochs<<<(n + 255) / 256, 256, 0, s>>>(j, n, tab);
   }
 }
 
 // after a release pass through reductions: units whose refcount went negative (underflow) or
 // reached 0 while active (freed by this call)
-__global__ void k_release_scan(const UnitRec *rec, int n, Status *st, unsigned long long *lc, uint32_t *free_list) {
+__global__ void k_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc, uint32_t *free_list) {
   unsigned under = 0;
   for (int base = blockIdx.x * blockDim.x; base < n; base += gridDim.x * blockDim.x) {
     int i = base + threadIdx.x;
     bool fr = false;
     if (i < n) {
-      int32_t rc = rec[i].refcount;
+      int32_t rc = tab.rc[i];
       under += rc < 0;
-      fr = rc == 0 && (rec_flags(rec[i].endf) & UF_ACTIVE);
+      fr = rc == 0 && (hot_flags(tab.hot[i]) & UF_ACTIVE);
     }
     unsigned long long ix = warp_append(&lc[2], fr);
     if (fr) free_list[ix] = (uint32_t)i;
   }
   flush_count(&st->underflow, under);
 }
-void launch_release_scan(const UnitRec *rec, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
+void launch_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
                          cudaStream_t s) {
   if (n > 0) {
     int grid = std::min((n + 255) / 256, 1184);
     (void)cudaGetLastError();
-    k_release_scan<<<grid, 256, 0, s>>>(rec, n, st, lc, free_list);
+    k_release_scan<<<grid, 256, 0, s>>>(tab, n, st, lc, free_list);
+  }
+}
+
+// epoch origin moves (once per 2^32 - 16 launches): the current epoch becomes 1, every other 0
+__global__ void k_rebase_epochs(TableDev tab, int n, uint32_t cur) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+    tab.epoch[i] = tab.epoch[i] == cur ? 1u : 0u;
+}
+void launch_rebase_epochs(TableDev tab, int n, uint32_t cur, cudaStream_t s) {
+  if (n > 0) {
+    (void)cudaGetLastError();
+    k_rebase_epochs<<<std::min((n + 255) / 256, 1184), 256, 0, s>>>(tab, n, cur);
   }
 }
 
 // outer-pointer lookup for mapArray/unmapArray/releaseArray: one thread per pointer, plain
 // binary search over the full u64 key array (few pointers: latency, not bandwidth)
-__global__ void k_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t *ptrs, int n, PointInfo *out) {
+__global__ void k_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n, PointInfo *out) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   uint64_t p = ptrs[i];
@@ -799,24 +856,23 @@ __global__ void k_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t 
       if (ix.keys[lo + half] <= p) lo += half;
       len -= half;
     }
-    UnitRec u = rec[lo];
-    if (p <= rec_end(u.endf)) {
+    const uint64_t h = tab.hot[lo], b = ix.keys[lo], sz = tab.size64[lo];
+    if (p - b <= sz) {
       r.unit = lo;
-      r.base = ix.keys[lo];
-      r.size = rec_end(u.endf) - r.base;
-      r.flags = rec_flags(u.endf);
-      r.devbase = (r.flags & UF_STORAGE) ? r.base + u.delta : 0;
-      r.epoch = u.epoch;
-      r.refcount = u.refcount;
+      r.base = b;
+      r.size = sz;
+      r.flags = hot_flags(h);
+      r.devbase = (r.flags & UF_STORAGE) ? b + tab.ext_delta[hot_ext(h)] : 0;
+      r.epoch = tab.epoch[lo];
+      r.refcount = tab.rc[lo];
     }
   }
   out[i] = r;
 }
-void launch_lookup_points(IndexDev ix, const UnitRec *rec, const uint64_t *ptrs, int n, PointInfo *out,
-                          cudaStream_t s) {
+void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n, PointInfo *out, cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
-    k_lookup_points<<<(n + 127) / 128, 128, 0, s>>>(ix, rec, ptrs, n, out);
+    k_lookup_points<<<(n + 127) / 128, 128, 0, s>>>(ix, tab, ptrs, n, out);
   }
 }
 

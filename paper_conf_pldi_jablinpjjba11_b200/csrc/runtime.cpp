@@ -161,7 +161,7 @@ struct Run {
 
 // Search-index buffers: forward (all units by base) and reverse (live device extents by start)
 struct IndexBufs {
-  DevBuf top, wide, dir, skmin, smeta, keys, pay;
+  DevBuf top, wide, dir, skmin, smeta, keys, pay, rid;
   DevBuf lvl[MAXL];
   size_t lvl_cap[MAXL] = {0};
   int n = 0, h = 0, ntop = 0, nseg = 0, ndir = 0;
@@ -194,6 +194,8 @@ struct Context {
   Arena arena;
   std::recursive_mutex mu;
   uint64_t epoch = 0;
+  uint64_t origin = 0;  // device epochs are u32 relative to this origin (A28)
+  uint32_t rel_epoch(uint64_t e) const { return e >= origin ? (uint32_t)(e - origin) : 0u; }
 
   // registry (host)
   std::map<uint64_t, HostUnit> reg;
@@ -203,12 +205,13 @@ struct Context {
   int U = 0;  // units in the device table
 
   // device table
-  DevBuf rec, dbase;
+  DevBuf hot, rcb, epb, size64, dbase, extd;  // unit table columns + extent deltas (by run id)
+  size_t extd_n = 0;                          // entries uploaded to extd
   IndexBufs fwd, rev;
 
   // scratch
   DevBuf status, lc, hitmask, act_list, journal, free_list, copy_list, segs, seg0, staging, staging2, staging_cb, points, ptrs, temp;
-  DevBuf up_units, up_vals, uops;
+  DevBuf up_units, up_vals, up_exts, uops;
   HostBuf h_small, h_status, h_list, h_pack[2];
   int pack_k = 0;
   cudaEvent_t ev_copy = nullptr, ev_t0 = nullptr, ev_t1 = nullptr, ev_pack[2] = {nullptr, nullptr};
@@ -243,6 +246,25 @@ struct Context {
     if (b.addr) arena.free(b.addr, b.bytes);
     b.addr = 0;
     b.bytes = 0;
+  }
+  TableDev tab() const {
+    TableDev t;
+    t.hot = hot.as<uint64_t>();
+    t.rc = rcb.as<int32_t>();
+    t.epoch = epb.as<uint32_t>();
+    t.base = dbase.as<uint64_t>();
+    t.size64 = size64.as<uint64_t>();
+    t.ext_delta = extd.as<uint64_t>();
+    t.n_ext = (int)extd_n;
+    return t;
+  }
+  // device copy of the extent deltas (devbase - base) indexed by run id
+  int sync_ext() {
+    std::vector<uint64_t> d(std::max<size_t>(runs.size(), 1), 0);
+    for (size_t r = 0; r < runs.size(); ++r) d[r] = 0 - runs[r].delta;  // runs store host - device
+    CKS(upload(extd, d));
+    extd_n = runs.size();
+    return CGCM_OK;
   }
 
   int64_t new_run(uint64_t addr, uint64_t bytes, uint64_t delta) {
@@ -310,7 +332,8 @@ struct Context {
     for (int g = 0; g < nseg; ++g) {
       int t0 = segstart[g], t1 = g + 1 < nseg ? segstart[g + 1] : ntop;
       uint64_t kmin = top[t0], span = top[t1 - 1] - kmin;
-      int64_t nbt = std::max<int64_t>(1, (int64_t)(dirmax - nseg) * (t1 - t0) / std::max(ntop, 1));
+      const int64_t dir_total = std::min<int64_t>(dirmax - nseg, std::max<int64_t>(64, 2 * (int64_t)ntop));
+      int64_t nbt = std::max<int64_t>(1, dir_total * (t1 - t0) / std::max(ntop, 1));
       uint32_t shift = 0;
       while (shift < 63 && (int64_t)(span >> shift) + 1 > nbt) ++shift;
       uint32_t nb = (uint32_t)((span >> shift) + 1);
@@ -360,14 +383,14 @@ struct Context {
   int ensure_table() {
     if (!table_dirty) return CGCM_OK;
     int n = (int)reg.size();
-    // host staging: base[n], size[n], epoch0[n], old_idx[n], flags[n]
-    size_t need = (size_t)n * (8 + 8 + 8 + 4 + 4) + 256;
+    // host staging: base[n], size[n], epoch0[n] (u32, relative), old_idx[n], flags[n]
+    size_t need = (size_t)n * (8 + 8 + 4 + 4 + 4) + 256;
     CKS(h_list.ensure(need));
     CK(cudaStreamSynchronize(main));
     CK(cudaStreamSynchronize(copy));
     uint64_t *hb = h_list.as<uint64_t>();
     uint64_t *hs = hb + n;
-    uint64_t *he = hs + n;
+    uint32_t *he = reinterpret_cast<uint32_t *>(hs + n);
     int32_t *ho = reinterpret_cast<int32_t *>(he + n);
     uint32_t *hf = reinterpret_cast<uint32_t *>(ho + n);
     by_idx.assign(n, reg.end());
@@ -375,37 +398,46 @@ struct Context {
     for (auto it = reg.begin(); it != reg.end(); ++it, ++i) {
       hb[i] = it->first;
       hs[i] = it->second.size;
-      he[i] = it->second.epoch0;
+      he[i] = rel_epoch(it->second.epoch0);
       ho[i] = it->second.idx;
       hf[i] = it->second.flags & (UF_GLOBAL | UF_READONLY);
       it->second.idx = i;
       by_idx[i] = it;
     }
-    DevBuf nrec, nbase, tmp;
+    DevBuf nhot, nrc, nep, nsize, nbase, tmp;
     int cap = std::max(n, 1);
-    CKS(dalloc(nrec, 32 * (size_t)cap));
+    CKS(dalloc(nhot, 8 * (size_t)cap));
+    CKS(dalloc(nrc, 4 * (size_t)cap + 64));
+    CKS(dalloc(nep, 4 * (size_t)cap + 64));
+    CKS(dalloc(nsize, 8 * (size_t)cap));
     CKS(dalloc(nbase, 8 * (size_t)cap));
     CKS(dalloc(tmp, (size_t)cap * 24 + 256));
     if (n > 0) {
       CK(cudaMemcpyAsync(nbase.as<void>(), hb, 8 * (size_t)n, cudaMemcpyHostToDevice, main));
-      CK(cudaMemcpyAsync(tmp.as<void>(), hs, (size_t)n * 24, cudaMemcpyHostToDevice, main));
-      DevBuf tmp2;
-      CKS(dalloc(tmp2, (size_t)n * 8 + 256));
-      CK(cudaMemcpyAsync(tmp2.as<void>(), ho, (size_t)n * 8, cudaMemcpyHostToDevice, main));
-      const uint64_t *dsize = tmp.as<uint64_t>();
-      const uint64_t *depoch = dsize + (size_t)n;
-      const int32_t *dold = tmp2.as<int32_t>();
+      CK(cudaMemcpyAsync(nsize.as<void>(), hs, 8 * (size_t)n, cudaMemcpyHostToDevice, main));
+      CK(cudaMemcpyAsync(tmp.as<void>(), he, (size_t)n * 12, cudaMemcpyHostToDevice, main));
+      const uint32_t *depoch = tmp.as<uint32_t>();
+      const int32_t *dold = reinterpret_cast<const int32_t *>(depoch + n);
       const uint32_t *dflags = reinterpret_cast<const uint32_t *>(dold + n);
-      launch_remap(n, dold, nbase.as<uint64_t>(), dsize, dflags, depoch, rec.as<UnitRec>(), nrec.as<UnitRec>(), main);
+      TableDev nt = tab();
+      nt.hot = nhot.as<uint64_t>();
+      nt.rc = nrc.as<int32_t>();
+      nt.epoch = nep.as<uint32_t>();
+      launch_remap(n, dold, nsize.as<uint64_t>(), dflags, depoch, tab(), nt, main);
       st.kernel_launches += 1;
       CK(cudaGetLastError());
       CK(cudaStreamSynchronize(main));
-      dfree(tmp2);
     }
     dfree(tmp);
-    dfree(rec);
+    dfree(hot);
+    dfree(rcb);
+    dfree(epb);
+    dfree(size64);
     dfree(dbase);
-    rec = nrec;
+    hot = nhot;
+    rcb = nrc;
+    epb = nep;
+    size64 = nsize;
     dbase = nbase;
     U = n;
     CKS(build_index(fwd, hb, n, dbase.as<uint64_t>(), TOPMAX, DIRMAX));
@@ -421,19 +453,24 @@ struct Context {
     CKS(ensure_table());
     if (!rev_dirty) return CGCM_OK;
     std::vector<uint64_t> keys, pay;
+    std::vector<uint32_t> rid;
     keys.reserve(live_runs.size() + 1);
     pay.reserve(live_runs.size() + 1);
     for (auto &kv : live_runs) {
       keys.push_back(kv.first);
       pay.push_back(runs[kv.second].delta);
+      rid.push_back((uint32_t)kv.second);
     }
     std::vector<uint64_t> kup = keys, pup = pay;
+    std::vector<uint32_t> rup = rid;
     if (kup.empty()) {
       kup.push_back(0);
       pup.push_back(0);
+      rup.push_back(0);
     }
     CKS(upload(rev.keys, kup));
     CKS(upload(rev.pay, pup));
+    CKS(upload(rev.rid, rup));
     CKS(build_index(rev, keys.data(), (int)keys.size(), rev.keys.as<uint64_t>(), RUN_SMEM, RUN_SMEM));
     rev_dirty = false;
     st.rev_rebuilds += 1;
@@ -451,6 +488,10 @@ struct Context {
   };
 
   int list_capacity() const { return std::max(U, 1); }
+  size_t slot_smem_estimate(const SlotCall &c) const {
+    (void)c;
+    return 8 * (size_t)fwd.ntop + 4 * (size_t)fwd.ndir + 12 * (size_t)rev.ntop + 4 * (size_t)rev.ndir + 8 * extd_n;
+  }
 
   // upload segments, launch, (no sync).  slot st index = which Status block to use.
   int launch(SlotCall &c, int st_index, bool reuse_hitmask_layout = false, bool timed_fwd = false,
@@ -476,12 +517,13 @@ struct Context {
     CK(cudaStreamSynchronize(main));  // the host vectors above are pageable and go out of scope
     SlotArgs a;
     std::memset(&a, 0, sizeof(a));
-    a.rec = rec.as<UnitRec>();
+    a.tab = tab();
     a.fx = fwd.view(dbase.as<uint64_t>());
     a.fx_nowide = fwd.any_wide ? 0 : 1;
     if (c.dir == DIR_REV) {
       a.rx = rev.view(rev.keys.as<uint64_t>());
       a.runpay = rev.pay.as<uint64_t>();
+      a.runid = rev.rid.as<uint32_t>();
     }
     a.segs = dsegs;
     a.seg_chunk0 = dc0;
@@ -490,7 +532,7 @@ struct Context {
     a.nchunks = c.nchunks;
     a.hitmask = hitmask.as<uint32_t>();
     a.dec_red = c.dec_red ? 1 : 0;
-    a.epoch = epoch;
+    a.epoch = rel_epoch(epoch);
     a.st = status.as<Status>() + st_index;
     a.lc = lc.as<unsigned long long>();
     a.act_list = act_list.as<uint32_t>();
@@ -502,13 +544,16 @@ struct Context {
     if (timed) CK(cudaEventRecord(ev_t0, main));
     int r = launch_slots(c.dir, c.ops, a, nsm, main);
     if (r != 0) {
-      g_last_cuda_error = r == -2 ? "unsupported slot-kernel operation set" : "k_slots launch failed";
+      g_last_cuda_error = r == -2 ? std::string("unsupported slot-kernel operation set")
+                                  : std::string("k_slots launch (dir ") + std::to_string(c.dir) + ", ops " +
+                                        std::to_string(c.ops) + ", smem " + std::to_string(slot_smem_estimate(c)) +
+                                        "): " + cudaGetErrorString((cudaError_t)r);
       return CGCM_E_CUDA;
     }
     CK(cudaGetLastError());
     st.kernel_launches += 1;
     if ((c.ops & OP_DEC) && c.dec_red) {  // underflow / 1 -> 0 detection after reductions
-      launch_release_scan(rec.as<UnitRec>(), U, status.as<Status>() + st_index, lc.as<unsigned long long>(),
+      launch_release_scan(tab(), U, status.as<Status>() + st_index, lc.as<unsigned long long>(),
                           free_list.as<uint32_t>(), main);
       st.kernel_launches += 1;
       CK(cudaGetLastError());
@@ -582,7 +627,7 @@ struct Context {
   int unit_ops(const std::vector<UnitOp> &ops) {
     if (ops.empty()) return CGCM_OK;
     CKS(upload(uops, ops));
-    launch_unit_ops(uops.as<UnitOp>(), (int)ops.size(), rec.as<UnitRec>(), main);
+    launch_unit_ops(uops.as<UnitOp>(), (int)ops.size(), tab(), main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
     return CGCM_OK;
@@ -682,12 +727,14 @@ struct Context {
         devbases[q] = it->second.devbase;
       }
     }
-    std::vector<uint64_t> deltas(units.size());
-    for (size_t q = 0; q < units.size(); ++q) deltas[q] = devbases[q] - by_idx[units[q]]->first;
+    std::vector<uint32_t> exts(units.size());
+    for (size_t q = 0; q < units.size(); ++q) exts[q] = (uint32_t)by_idx[units[q]]->second.run;
+    if (runs.size() > EXT_MASK) return CGCM_E_NOMEM;  // 2^24 live extents
+    CKS(sync_ext());
     CKS(upload(up_units, units));
-    CKS(upload(up_vals, deltas));
-    launch_set_delta(up_units.as<uint32_t>(), up_vals.as<uint64_t>(), (int)units.size(), rec.as<UnitRec>(), epoch,
-                     (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
+    CKS(upload(up_exts, exts));
+    launch_set_ext(up_units.as<uint32_t>(), up_exts.as<uint32_t>(), (int)units.size(), tab(), rel_epoch(epoch),
+                   (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
     CK(cudaEventRecord(ev_copy, main));  // the copies wait for everything the main stream did before
@@ -773,7 +820,7 @@ struct Context {
   int free_units(const std::vector<uint32_t> &units) {
     if (units.empty()) return CGCM_OK;
     CKS(upload(up_units, units));
-    launch_deactivate(up_units.as<uint32_t>(), (int)units.size(), rec.as<UnitRec>(), main);
+    launch_deactivate(up_units.as<uint32_t>(), (int)units.size(), tab(), main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(main));
@@ -1035,7 +1082,7 @@ struct Context {
   // the slot side (re-translate in-place writes, re-add released references)
   int undo_rev(SlotCall &c, uint64_t journal_count, const std::vector<Journal> &extra, bool write, bool dec) {
     if (journal_count) {
-      launch_restore_epochs(journal.as<Journal>(), (int)journal_count, rec.as<UnitRec>(), main);
+      launch_restore_epochs(journal.as<Journal>(), (int)journal_count, tab(), main);
       st.kernel_launches += 1;
       CK(cudaGetLastError());
     }
@@ -1043,7 +1090,7 @@ struct Context {
     if (!extra.empty()) {
       DevBuf jb;
       CKS(upload(jb, extra));
-      launch_restore_epochs(jb.as<Journal>(), (int)extra.size(), rec.as<UnitRec>(), main);
+      launch_restore_epochs(jb.as<Journal>(), (int)extra.size(), tab(), main);
       st.kernel_launches += 1;
       CK(cudaStreamSynchronize(main));
       dfree(jb);
@@ -1075,7 +1122,7 @@ struct Context {
     std::vector<uint64_t> v(ptrs, ptrs + k);
     CKS(upload(this->ptrs, v));
     CKS(dalloc(points, sizeof(PointInfo) * k + 64));
-    launch_lookup_points(fwd.view(dbase.as<uint64_t>()), rec.as<UnitRec>(), this->ptrs.as<uint64_t>(), (int)k,
+    launch_lookup_points(fwd.view(dbase.as<uint64_t>()), tab(), this->ptrs.as<uint64_t>(), (int)k,
                          points.as<PointInfo>(), main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
@@ -1274,7 +1321,7 @@ int cgcm_undeclare(void *base) {
   HostUnit &u = it->second;
   if (u.idx >= 0) {  // idx refers to the current device table until the next ensure_table()
     int32_t rc = 0;
-    CK(cudaMemcpyAsync(&rc, &C->rec.as<UnitRec>()[u.idx].refcount, 4, cudaMemcpyDeviceToHost, C->main));
+    CK(cudaMemcpyAsync(&rc, C->rcb.as<int32_t>() + u.idx, 4, cudaMemcpyDeviceToHost, C->main));
     CK(cudaStreamSynchronize(C->main));
     if (rc > 0) return CGCM_E_BUSY;
   }
@@ -1644,10 +1691,11 @@ int cgcm_unmapArrays(void *const *const *arrays, size_t k) {
   std::vector<Seg> rsegs_copy, rsegs_gate, fsegs_gate;
   uint64_t stage_bytes = 0;
   for (auto &o : outs) {
-    bool copy_o = o.info.epoch != C->epoch && !(o.info.flags & UF_READONLY);
-    if (o.info.epoch != C->epoch) {
-      ops.push_back({(uint32_t)o.unit, UOP_SET_EPOCH, C->epoch});
-      outer_jn.push_back({o.info.epoch, (uint32_t)o.unit, 0});
+    const uint32_t cur = C->rel_epoch(C->epoch);
+    bool copy_o = o.info.epoch != cur && !(o.info.flags & UF_READONLY);
+    if (o.info.epoch != cur) {
+      ops.push_back({(uint32_t)o.unit, UOP_SET_EPOCH, cur});
+      outer_jn.push_back({(uint32_t)o.info.epoch, (uint32_t)o.unit, 0, 0});
     }
     uint64_t n = o.info.size / 8;
     if (copy_o) {
@@ -1809,6 +1857,12 @@ int cgcm_releaseArray(void *const *cpu) { return cgcm_releaseArrays(&cpu, 1); }
 
 int cgcm_advanceEpoch(void) {
   CTX();
+  if (C->epoch + 1 - C->origin >= 0xFFFFFFF0ull) {  // move the u32 epoch origin (A28)
+    CKS(C->ensure_table());
+    launch_rebase_epochs(C->tab(), C->U, C->rel_epoch(C->epoch), C->main);
+    CK(cudaStreamSynchronize(C->main));
+    C->origin = C->epoch - 1;
+  }
   C->epoch += 1;  // "increases every time the program launches a GPU function"
   return CGCM_OK;
 }
@@ -1834,19 +1888,26 @@ int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
   CKS(C->ensure_table());
   if (n) *n = (size_t)C->U;
   if (!out || cap == 0) return (size_t)C->U <= cap ? CGCM_OK : CGCM_E_NOMEM;
-  std::vector<UnitRec> recs;
-  CKS(C->download(recs, C->rec, (size_t)C->U));
+  std::vector<uint64_t> hots, szs;
+  std::vector<uint32_t> eps;
+  std::vector<int32_t> rcs;
+  CKS(C->download(hots, C->hot, (size_t)C->U));
+  CKS(C->download(eps, C->epb, (size_t)C->U));
+  CKS(C->download(szs, C->size64, (size_t)C->U));
+  CKS(C->download(rcs, C->rcb, (size_t)C->U));
   size_t m = std::min(cap, (size_t)C->U);
   for (size_t i = 0; i < m; ++i) {
-    const UnitRec &r = recs[i];
     cgcm_unit_t &u = out[i];
-    const uint32_t fl = rec_flags(r.endf);
+    const uint32_t fl = hot_flags(hots[i]);
     u.base = C->by_idx[i]->first;
-    u.size = rec_end(r.endf) - u.base;
-    bool act = r.refcount > 0;
-    u.devptr = ((fl & UF_STORAGE) && (act || (fl & UF_GLOBAL))) ? u.base + r.delta : 0;
-    u.refCount = r.refcount;
-    u.epoch = r.epoch;
+    u.size = szs[i];
+    bool act = rcs[i] > 0;
+    uint32_t e = hot_ext(hots[i]);
+    u.devptr = ((fl & UF_STORAGE) && (act || (fl & UF_GLOBAL)) && e < C->runs.size())
+                   ? u.base - C->runs[e].delta
+                   : 0;
+    u.refCount = rcs[i];
+    u.epoch = C->origin + eps[i];
     u.flags = ((fl & UF_GLOBAL) ? CGCM_UNIT_GLOBAL : 0) | ((fl & UF_READONLY) ? CGCM_UNIT_READONLY : 0) |
               ((fl & UF_ARRAYMAPPED) ? CGCM_UNIT_ARRAYMAPPED : 0) | (act ? CGCM_UNIT_ACTIVE : 0);
     u.pad = 0;

@@ -1,0 +1,78 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py times
+(cgcm_mapArrayDevice / cgcm_unmapArrayDevice over device-resident arrays, one call per batch):
+
+* config C: 2^20 AUs, 2^26 interior pointers (all of them checked by properties, 2^16 sampled slots
+  checked one by one against the CPU oracle in replay mode);
+* config E: the full 2^22-AU table, with 32 of the 256 arrays (2^25 pointers) per call.
+
+Properties checked on every slot: refcount[u] == number of slots pointing into u (A8), the reverse
+translation restores every slot (round trip), read-only units are never copied back.
+"""
+import numpy as np
+import pytest
+
+import workloads as W
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+
+def run_full(U, arrays, slots_per_array, seed, sample=1 << 16):
+    import torch
+    import paper_conf_pldi_jablinpjjba11_b200 as cg
+    from oracle import Oracle
+
+    offs, sizes, span = W.table_layout(U, seed)
+    R = W.reserve_readonly(span)
+    bases = offs + np.uint64(R)
+    n = arrays * slots_per_array
+    ctx = cg.Context(0, arena_bytes=int(sizes.sum()) + span // 8 + n * 24 + (4 << 30))
+    try:
+        assert ctx.declareBatch(bases, sizes, readonly=True) == 0
+        ot = torch.from_numpy(offs.view(np.int64)).cuda()
+        st = torch.from_numpy(sizes.view(np.int64)).cuda()
+        q, u = W.queries_t(ot, st, n, seed)
+        d = q + R
+        orig = d.clone()
+        assert ctx.mapArrayDevice(d.data_ptr(), n) == 0
+        # A8: refcount == number of slots pointing into the unit (every unit, every slot)
+        dump = ctx.dump()
+        rc = np.array([x["refCount"] for x in dump], dtype=np.int64)
+        cnt = torch.bincount(u, minlength=U).cpu().numpy()
+        assert (rc == cnt).all()
+        dev = np.array([x["devptr"] for x in dump], dtype=np.uint64)
+        # forward translation of every slot: devptr(u) + (p - base(u))  (vectorised on the GPU)
+        devt = torch.from_numpy(dev.view(np.int64)).cuda()
+        bt = torch.from_numpy(bases.view(np.int64)).cuda()
+        assert torch.equal(d, devt[u] + (orig - bt[u]))
+        # 2^16 sampled slots one by one through the oracle (replay mode: the GPU's device addresses)
+        rng = np.random.default_rng(seed)
+        idx = np.sort(rng.choice(n, size=min(sample, n), replace=False))
+        ps = orig.cpu().numpy().view(np.uint64)[idx]
+        gs = d.cpu().numpy().view(np.uint64)[idx]
+        o = Oracle()
+        for b, s in zip(bases.tolist(), sizes.tolist()):
+            assert o.declareAlloc(b, s, readonly=True) == 0
+        units = np.unique(u.cpu().numpy()[idx])
+        for k in units.tolist():
+            o.replay(int(bases[k]), int(dev[k]))
+        stt, out = o.mapBatch(ps)
+        assert stt == 0 and (out == gs).all()
+        o.close()
+        # a3 + a4 + release: round trip, nothing copied back (read-only), all references dropped
+        ctx.advanceEpoch()
+        assert ctx.unmapArrayDevice(d.data_ptr(), n, release=True) == 0
+        assert torch.equal(d, orig)
+        s = ctx.stats()
+        assert s["d2h_units"] == 0 and s["rev_translations"] == n and s["fwd_translations"] == n
+        assert all(x["refCount"] == 0 for x in ctx.dump())
+    finally:
+        ctx.close()
+        W.release_reservation(R, span)
+
+
+def test_config_C_full_size():
+    run_full(1 << 20, 64, 1 << 20, 3)
+
+
+def test_config_E_full_table():
+    run_full(1 << 22, 32, 1 << 20, 5)

@@ -392,3 +392,56 @@ def test_random_stress(pair):
         if step % 20 == 0:
             P.check(f"step {step}")
     P.check("end")
+
+
+@pytest.mark.parametrize("promoted", [False, True])
+def test_config_B_gemm_reduced(pair, promoted):
+    """Config B shape at n = 256, 4 row-blocks of 64: 3 jagged matrices, one S2 launch per block.
+    Counts, refcounts and A/B bytes exact; C within 1e-12 relative of the oracle's long-double S2."""
+    P = pair
+    n, blk = 256, 64
+    mats, vals = [], []
+    for m in range(3):
+        v = W.config_B_values(n, 2, m)
+        rows = [P.malloc(8 * n, v[r]) for r in range(n)]
+        mats.append(P.malloc(8 * n, np.asarray(rows, dtype=np.uint64)))
+        vals.append((rows, v))
+    A, B, Cm = mats
+
+    def block(b0, devs):
+        assert P.g.sample_gemm_rows(devs[0], devs[1], devs[2], n, b0, blk, 1.5, 1.2) == 0
+        P.g.synchronize()
+        P.o.kernel_gemm_rows(devs[0], devs[1], devs[2], n, b0, blk, 1.5, 1.2)
+        P.advance()
+
+    if promoted:
+        for pp in mats:
+            P.run("mapArray", pp)
+    for b0 in range(0, n, blk):
+        devs = [P.run("mapArray", pp)[1] for pp in mats]
+        block(b0, devs)
+        if not promoted:
+            P.run("unmapArray", Cm)
+        for pp in mats:
+            P.run("releaseArray", pp)
+    if promoted:
+        P.run("unmapArray", Cm)
+        for pp in mats:
+            P.run("releaseArray", pp)
+    gd, od = P.g.dump(), P.o.dump()
+    assert gd == od
+    gs, os_ = P.g.stats(), P.o.stats()
+    for f in ("h2d_units", "h2d_bytes", "d2h_units", "d2h_bytes", "fwd_translations", "rev_translations"):
+        assert gs[f] == os_[f], f
+    blocks = n // blk
+    if promoted:
+        assert (gs["h2d_units"], gs["d2h_units"]) == (3 * (n + 1), n + 1)
+    else:
+        assert (gs["h2d_units"], gs["d2h_units"]) == (blocks * 3 * (n + 1), blocks * (n + 1))
+    for (rows, v), pp in zip(vals[:2], mats[:2]):
+        got = np.stack([np.frombuffer(host_read(a, 8 * n), dtype=np.float64) for a in rows])
+        assert got.tobytes() == v.tobytes()
+    rows_c = vals[2][0]
+    gc = np.stack([np.frombuffer(host_read(a, 8 * n), dtype=np.float64) for a in rows_c])
+    oc = np.stack([P.o.host_read(a, 8 * n).view(np.float64) for a in rows_c])
+    assert np.max(np.abs(gc - oc) / np.abs(oc)) < 1e-12
