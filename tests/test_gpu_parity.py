@@ -445,3 +445,28 @@ def test_config_B_gemm_reduced(pair, promoted):
     gc = np.stack([np.frombuffer(host_read(a, 8 * n), dtype=np.float64) for a in rows_c])
     oc = np.stack([P.o.host_read(a, 8 * n).view(np.float64) for a in rows_c])
     assert np.max(np.abs(gc - oc) / np.abs(oc)) < 1e-12
+
+
+@pytest.mark.parametrize("release", [False, True])
+def test_unmapArrayDevice_error_rolls_back(pair, release):
+    """A large reverse pass (snapshot rollback) and a small one (journal rollback) hitting an
+    unregistered device pointer: UNREGISTERED, device slots, refcounts and epochs unchanged."""
+    import torch
+    P = pair
+    offs, sizes, R, span = config_C_setup(P, 8192)
+    for n in (60000, 100):                      # >= U/8: snapshot mode; < U/8: journal mode
+        q, u = W.queries(offs, sizes, n, 3)
+        slots = (q + np.uint64(R)).astype(np.uint64)
+        d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+        assert P.g.mapArrayDevice(d.data_ptr(), n) == 0
+        P.g.advanceEpoch()
+        bad = d.clone()
+        bad[n // 2] = 12345                      # not a device copy
+        before = P.g.dump()
+        assert P.g.unmapArrayDevice(bad.data_ptr(), n, release=release) == -2
+        assert P.g.dump() == before
+        bad[n // 2] = d[n // 2]
+        assert torch.equal(bad, d)               # the in-place reverse rewrite was undone
+        assert P.g.unmapArrayDevice(d.data_ptr(), n, release=True) == 0
+        assert (d.cpu().numpy().view(np.uint64) == slots).all()
+    W.release_reservation(R, span)
