@@ -144,6 +144,7 @@ struct SlotArgs {
   uint32_t *free_list;
   int lenient;
   int dec_red;                 // OP_DEC through reductions + k_release_scan
+  int no_journal;              // the host snapshotted rc/epoch columns: no per-unit epoch journal
   int fx_nowide;               // the forward index has no wide bucket (specialised kernels)
 };
 

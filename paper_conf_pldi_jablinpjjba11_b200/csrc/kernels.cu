@@ -437,7 +437,9 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
     int32_t rcv[2] = {0, 0};
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      if ((OPS & OP_GATE) && hit[m]) ep[m] = a.tab.epoch[j[m]];
+      // read-only units under a snapshot: the gate can only set the epoch (no copy, nothing to journal)
+      if ((OPS & OP_GATE) && hit[m] && !(a.no_journal && (hot_flags(hw[m]) & UF_READONLY)))
+        ep[m] = a.tab.epoch[j[m]];
       if ((OPS & OP_CHECKMAPPED) && hit[m]) rcv[m] = a.tab.rc[j[m]];
     }
 
@@ -486,7 +488,9 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
       bool gated = false;
       uint32_t old_ep = 0;
       if (OPS & OP_GATE) {
-        if (hm && ep[m] != a.epoch) {
+        if (hm && a.no_journal && (fl & UF_READONLY)) {
+          a.tab.epoch[unit] = a.epoch;  // Alg. 2 line 3 for a read-only unit: epoch <- globalEpoch
+        } else if (hm && ep[m] != a.epoch) {
           old_ep = atomicExch(a.tab.epoch + unit, a.epoch);
           gated = (old_ep != a.epoch);
         }
@@ -519,9 +523,10 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
         }
       }
       if (OPS & OP_GATE) {
-        unsigned long long ix = warp_append(&a.lc[1], gated);
+        const bool jg = gated && !a.no_journal;
+        unsigned long long ix = warp_append(&a.lc[1], jg);
         const bool cp = gated && !(fl & UF_READONLY);  // Alg. 2: stale and not read-only
-        if (gated) {
+        if (jg) {
           Journal jn;
           jn.old_epoch = old_ep;
           jn.unit = (uint32_t)unit;

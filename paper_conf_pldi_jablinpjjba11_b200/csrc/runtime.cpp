@@ -205,7 +205,7 @@ struct Context {
   int U = 0;  // units in the device table
 
   // device table
-  DevBuf hot, rcb, epb, size64, dbase, extd;  // unit table columns + extent deltas (by run id)
+  DevBuf hot, rcb, epb, size64, dbase, extd, snap_rc, snap_ep;  // unit table columns + extent deltas
   size_t extd_n = 0;                          // entries uploaded to extd
   IndexBufs fwd, rev;
 
@@ -482,6 +482,7 @@ struct Context {
   struct SlotCall {
     int dir = DIR_FWD, ops = 0, sel = SEL_ALL;
     bool dec_red = false;  // OP_DEC through reductions + k_release_scan (large batches)
+    bool no_journal = false;  // large gate passes snapshot the rc/epoch columns instead
     std::vector<Seg> segs;
     uint64_t nchunks = 0;
     Status res{};
@@ -532,6 +533,7 @@ struct Context {
     a.nchunks = c.nchunks;
     a.hitmask = hitmask.as<uint32_t>();
     a.dec_red = c.dec_red ? 1 : 0;
+    a.no_journal = c.no_journal ? 1 : 0;
     a.epoch = rel_epoch(epoch);
     a.st = status.as<Status>() + st_index;
     a.lc = lc.as<unsigned long long>();
@@ -1055,19 +1057,28 @@ struct Context {
     c.dir = DIR_REV;
     c.ops = write ? (OP_WRITE | OP_GATE | OP_HITMASK | (dec ? OP_DEC : 0)) : (OP_GATE | (dec ? OP_DEC : 0));
     c.segs = segs;
-    c.dec_red = dec && total >= (uint64_t)U / 8;
+    // large passes: snapshot the rc/epoch columns instead of journaling every gated unit
+    c.no_journal = total >= (uint64_t)U / 8 && U >= 4096;
+    c.dec_red = dec && c.no_journal;
+    if (c.no_journal) CKS(take_snapshot());
     CKS(launch(c, 0, false, false, true));
     Status sts[8];
     unsigned long long lcs[4];
     CKS(fetch_status(sts, lcs));
     res = sts[0];
-    journal_count = lcs[1];
+    journal_count = c.no_journal ? 0 : lcs[1];
+    snapshotted = c.no_journal;
     bool strict = !(flags & CGCM_LENIENT);
     int err = CGCM_OK;
     if (sts[0].misses && strict) err = CGCM_E_UNREGISTERED;
     else if (sts[0].underflow) err = CGCM_E_NOT_MAPPED;
     if (err) {
-      CKS(undo_rev(c, lcs[1], {}, write, dec));
+      if (c.no_journal) {
+        CKS(restore_snapshot());
+        CKS(undo_rev(c, 0, {}, write, false));  // refcounts came back with the snapshot
+      } else {
+        CKS(undo_rev(c, lcs[1], {}, write, dec));
+      }
       return err;
     }
     CKS(sorted_units(copy_list, lcs[3], copy_units));
@@ -1076,6 +1087,20 @@ struct Context {
       CKS(download(f, free_list, lcs[2]));
       freed.insert(freed.end(), f.begin(), f.end());
     }
+    return CGCM_OK;
+  }
+  bool snapshotted = false;
+  int take_snapshot() {
+    CKS(dalloc(snap_rc, 4 * (size_t)U + 64));
+    CKS(dalloc(snap_ep, 4 * (size_t)U + 64));
+    CK(cudaMemcpyAsync(snap_rc.as<void>(), rcb.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
+    CK(cudaMemcpyAsync(snap_ep.as<void>(), epb.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
+    return CGCM_OK;
+  }
+  int restore_snapshot() {
+    CK(cudaMemcpyAsync(rcb.as<void>(), snap_rc.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
+    CK(cudaMemcpyAsync(epb.as<void>(), snap_ep.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
+    CK(cudaStreamSynchronize(main));
     return CGCM_OK;
   }
   // undo of a gate/reverse pass: epochs from the device journal (+ host-side extra entries), then
@@ -1422,7 +1447,12 @@ int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
     c.dir = DIR_REV;
     c.ops = OP_WRITE | OP_GATE | OP_HITMASK | (rel ? OP_DEC : 0);
     c.segs = {s};
-    C->undo_rev(c, jcount, {}, true, rel);
+    if (C->snapshotted) {
+      C->restore_snapshot();
+      C->undo_rev(c, 0, {}, true, false);
+    } else {
+      C->undo_rev(c, jcount, {}, true, rel);
+    }
     return r;
   }
   C->st.rev_translations += res.translated;
