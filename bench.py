@@ -141,7 +141,7 @@ def run_cgcm(args, rank, world, local_rank):
     t0 = time.time()
     wl = Workload(cfg, rank, world)
     total_bytes = int(wl.sizes.sum())
-    arena = total_bytes + wl.span // 8 + wl.n * 8 * 2 + (6 << 30)
+    arena = total_bytes + wl.span // 8 + wl.n * 8 * 4 + (6 << 30)
     ctx = cg.Context(local_rank, arena_bytes=arena, flags=cg.PROFILE)
     assert ctx.declareBatch(wl.bases, wl.sizes, readonly=True) == 0
     # one reference per unit held for the whole run (map promotion of the table's maps)

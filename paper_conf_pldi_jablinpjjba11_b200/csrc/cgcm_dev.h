@@ -74,10 +74,14 @@ struct IndexDev {
 
 // One input segment of a slot kernel: n u64 slots at device address ptr (8-byte aligned),
 // translated in place (out == 0) or into out.  inc = refcount delta per non-null slot.
+// shadow (optional, 12 B per slot: u64 CPU pointer[n] then u32 unit[n]): written by the forward map,
+// read by the reverse unmap of the same slots -- GPU functions do not store pointers (R13-ii,
+// P:L140-142), so an unchanged slot reverses to its recorded CPU pointer after one check.
 struct Seg {
   uint64_t ptr, n, out;
   int32_t inc;
   uint32_t pad;
+  uint64_t shadow;
 };
 
 // per-launch status, written by the kernels with warp-aggregated atomics

@@ -372,6 +372,31 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
       look[m] = ((valid >> m) & 1) && v[m] != 0;
       q[m] = look[m] ? v[m] : 0ull;
     }
+    // reverse pass over slots the forward map recorded (unchanged since, R13-ii): one check
+    bool sh[2] = {false, false};
+    int jsh[2] = {0, 0};
+    uint64_t hsh[2] = {0, 0}, hwsh[2] = {0, 0};
+    const int64_t slot0 = ((int64_t)(a0 - sg.ptr)) >> 3;  // slot index of m = 0 (-1 for a head chunk)
+    if (DIR == DIR_REV && sg.shadow) {
+#pragma unroll
+      for (int m = 0; m < 2; ++m) {
+        if (!look[m]) continue;
+        const int64_t i = slot0 + m;
+        const uint32_t u = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n)[i];
+        if (u == 0xFFFFFFFFu) continue;
+        const uint64_t h = reinterpret_cast<const uint64_t *>(sg.shadow)[i];
+        const uint64_t w = ld_u64(a.tab.hot + u, pol_t);
+        const uint32_t e = hot_ext(w);
+        if ((hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext &&
+            q[m] == h + (ext_s ? s_ext[e] : a.tab.ext_delta[e])) {
+          sh[m] = true;
+          jsh[m] = (int)u;
+          hsh[m] = h;
+          hwsh[m] = w;
+          look[m] = false;
+        }
+      }
+    }
     if (DIR == DIR_REV) {
       // the device extent holding the pointer, and the host address it mirrors
 #pragma unroll
@@ -430,6 +455,26 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
             }
           }
         }
+      }
+    }
+    if (DIR == DIR_REV) {
+#pragma unroll
+      for (int m = 0; m < 2; ++m)
+        if (sh[m]) {
+          hit[m] = true;
+          j[m] = jsh[m];
+          q[m] = hsh[m];
+          hw[m] = hwsh[m];
+        }
+    }
+    // forward map: record the shadow of every slot (CPU pointer, unit) for the reverse pass
+    if ((OPS & OP_INC) && sg.shadow && live) {
+#pragma unroll
+      for (int m = 0; m < 2; ++m) {
+        if (!((valid >> m) & 1)) continue;
+        const int64_t i = slot0 + m;
+        reinterpret_cast<uint64_t *>(sg.shadow)[i] = v[m];
+        reinterpret_cast<uint32_t *>(sg.shadow + 8 * sg.n)[i] = hit[m] ? (uint32_t)j[m] : 0xFFFFFFFFu;
       }
     }
     // epoch (gate) and refcount (unmap check) columns, only where the operation needs them

@@ -444,6 +444,7 @@ struct Context {
     CK(cudaStreamSynchronize(main));
     table_dirty = false;
     rev_dirty = true;
+    table_gen += 1;  // unit indices changed: recorded shadows are stale
     st.table_rebuilds += 1;
     return CGCM_OK;
   }
@@ -867,6 +868,7 @@ struct Context {
         s.out = off;
         s.inc = 0;
         s.pad = 0;
+        s.shadow = 0;
         if (n) c.segs.push_back(s);
         off += 8 * n;
       }
@@ -1090,6 +1092,14 @@ struct Context {
     return CGCM_OK;
   }
   bool snapshotted = false;
+  // forward-map shadows of device-resident pointer arrays, keyed by (slots, n)
+  struct Shadow {
+    DevBuf buf;
+    uint64_t gen = 0;
+    bool valid = false;
+  };
+  std::map<std::pair<uint64_t, uint64_t>, Shadow> shadows;
+  uint64_t table_gen = 0;
   int take_snapshot() {
     CKS(dalloc(snap_rc, 4 * (size_t)U + 64));
     CKS(dalloc(snap_ep, 4 * (size_t)U + 64));
@@ -1421,13 +1431,32 @@ int cgcm_free(void *p) {
 }
 
 // ---- device-resident arrays -------------------------------------------------------------------
+static constexpr size_t SHADOW_MIN = 1u << 16;
+
 int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n) {
   CTX();
   if (n == 0) return CGCM_OK;
   if (!d_slots || (reinterpret_cast<uint64_t>(d_slots) & 7)) return CGCM_E_INVALID;
   CKS(C->ensure_table());
   Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
-  return C->map_core({s}, {}, nullptr, nullptr);
+  Context::Shadow *sh = nullptr;
+  if (n >= SHADOW_MIN) {  // record (CPU pointer, unit) per slot for the reverse pass (R13-ii)
+    auto key = std::make_pair(s.ptr, (uint64_t)n);
+    sh = &C->shadows[key];
+    sh->valid = false;
+    if (C->dalloc(sh->buf, 12 * n + 64) == CGCM_OK) {
+      s.shadow = sh->buf.addr;
+    } else {
+      C->shadows.erase(key);
+      sh = nullptr;
+    }
+  }
+  int r = C->map_core({s}, {}, nullptr, nullptr);
+  if (sh && r == CGCM_OK) {
+    sh->valid = true;
+    sh->gen = C->table_gen;
+  }
+  return r;
 }
 
 int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
@@ -1435,6 +1464,13 @@ int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
   if (n == 0) return CGCM_OK;
   if (!d_slots || (reinterpret_cast<uint64_t>(d_slots) & 7)) return CGCM_E_INVALID;
   Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
+  auto shk = std::make_pair(s.ptr, (uint64_t)n);
+  auto shi = C->shadows.find(shk);
+  if (shi != C->shadows.end()) {
+    CKS(C->ensure_table());
+    if (shi->second.valid && shi->second.gen == C->table_gen) s.shadow = shi->second.buf.addr;
+    shi->second.valid = false;  // consumed: after this call the slots hold CPU pointers again
+  }
   std::vector<uint32_t> copy_units, freed;
   uint64_t jcount = 0;
   Status res{};

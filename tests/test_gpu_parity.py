@@ -470,3 +470,41 @@ def test_unmapArrayDevice_error_rolls_back(pair, release):
         assert P.g.unmapArrayDevice(d.data_ptr(), n, release=True) == 0
         assert (d.cpu().numpy().view(np.uint64) == slots).all()
     W.release_reservation(R, span)
+
+
+def test_device_array_shadow_fallback_on_modified_slots(pair):
+    """The reverse pass reads the forward pass's shadow only for unchanged slots: a GPU function that
+    permutes / clears / re-points slots (violating R13-ii on purpose) still gets the exact reverse
+    lookup of the oracle."""
+    import torch
+    P = pair
+    offs, sizes, R, span = config_C_setup(P, 4096)
+    n = (1 << 17) + 5
+    q, u = W.queries(offs, sizes, n, 3)
+    slots = (q + np.uint64(R)).astype(np.uint64)
+    d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+    assert P.g.mapArrayDevice(d.data_ptr(), n) == 0
+    P.feed_replay()
+    ref = slots.copy()
+    assert P.o.mapSlots(ref) == 0
+    assert (d.cpu().numpy().view(np.uint64) == ref).all()
+    # the "GPU function": permute a third of the slots, NULL a few, point one at a unit's start
+    perm = torch.randperm(n // 3, generator=torch.Generator().manual_seed(1)).cuda()
+    d[: n // 3] = d[: n // 3][perm]
+    d[7] = 0
+    d[n - 1] = d[n - 2]
+    ref[: n // 3] = ref[: n // 3][perm.cpu().numpy()]
+    ref[7] = 0
+    ref[n - 1] = ref[n - 2]
+    P.advance()
+    # refcounts: the NULLed slot and the duplicated one make the release unbalanced for two units;
+    # both sides must agree on the outcome (status and state)
+    st_g = P.g.unmapArrayDevice(d.data_ptr(), n, release=True)
+    st_o = P.o.unmapSlots(ref, release=True)
+    assert st_g == st_o
+    if st_g != 0:
+        return
+    got = d.cpu().numpy().view(np.uint64)
+    assert (got == ref).all()
+    P.check("after modified-slot unmap")
+    W.release_reservation(R, span)
