@@ -45,7 +45,8 @@ enum {
   CGCM_LITERAL_EPOCH = 1u, /* A5 literal reading: map never sets the AU epoch (default: R1, set at
                               activation so map->unmap with no launch copies nothing)             */
   CGCM_LENIENT = 2u,       /* A18: uncovered non-null words in pointer arrays pass through (counted) */
-  CGCM_PROFILE = 4u        /* time every hot kernel with CUDA events on its launch stream (stats)  */
+  CGCM_PROFILE = 4u,       /* time every hot kernel with CUDA events on its launch stream (stats)  */
+  CGCM_FORCE_SHADOW = 8u   /* always record the forward-map shadow of device arrays (tests)        */
 };
 
 /* ---- AU flags (declare + dump) ------------------------------------------------------------- */

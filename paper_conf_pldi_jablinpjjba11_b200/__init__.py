@@ -22,7 +22,7 @@ SAMPLES_PATH = os.path.join(HERE, "libcgcm_samples.so")
 OK = 0
 E_INVALID, E_UNREGISTERED, E_OVERLAP, E_NOT_MAPPED, E_BUSY, E_DUPLICATE, E_NOMEM, E_CUDA, E_MIXED, E_NOCTX = (
     -1, -2, -3, -4, -5, -6, -7, -8, -9, -10)
-LITERAL_EPOCH, LENIENT, PROFILE = 1, 2, 4
+LITERAL_EPOCH, LENIENT, PROFILE, FORCE_SHADOW = 1, 2, 4, 8
 UNIT_GLOBAL, UNIT_READONLY, UNIT_ARRAYMAPPED, UNIT_ACTIVE = 1, 2, 4, 8
 RELEASE = 1
 

@@ -150,6 +150,7 @@ struct SlotArgs {
   int dec_red;                 // OP_DEC through reductions + k_release_scan
   int no_journal;              // the host snapshotted rc/epoch columns: no per-unit epoch journal
   int fx_nowide;               // the forward index has no wide bucket (specialised kernels)
+  int segs_host_shadow;        // the (single) segment carries a shadow: use the shadow variant
 };
 
 // ---- host-callable launchers (kernels.cu) ----------------------------------------------------

@@ -289,8 +289,14 @@ __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix,
 // -------------------------------------------------------------------------------------------------
 // FH >= 0: the forward index has exactly FH levels, one address segment and no wide bucket (the
 // common case, specialised for the hot operation sets); FH < 0: generic.
-template <int DIR, int OPS, int FH>
-__global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
+// threads per CTA: the shadow reverse variant keeps both paths live and gets more registers
+template <int DIR, int SH>
+struct SlotCfg {
+  static constexpr int threads = 768;  // measured: 768 > 1024 (spills) > 512 on configs C and E
+};
+
+template <int DIR, int OPS, int FH, int SH>
+__global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ uint64_t s_seg0[SEG_SMEM + 1];
   SIdx F, R;
@@ -377,7 +383,7 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
     int jsh[2] = {0, 0};
     uint64_t hsh[2] = {0, 0}, hwsh[2] = {0, 0};
     const int64_t slot0 = ((int64_t)(a0 - sg.ptr)) >> 3;  // slot index of m = 0 (-1 for a head chunk)
-    if (DIR == DIR_REV && sg.shadow) {
+    if (SH && DIR == DIR_REV && sg.shadow) {
 #pragma unroll
       for (int m = 0; m < 2; ++m) {
         if (!look[m]) continue;
@@ -457,7 +463,7 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
         }
       }
     }
-    if (DIR == DIR_REV) {
+    if (SH && DIR == DIR_REV) {
 #pragma unroll
       for (int m = 0; m < 2; ++m)
         if (sh[m]) {
@@ -468,7 +474,7 @@ __global__ void __launch_bounds__(SLOT_THREADS, 1) k_slots(SlotArgs a) {
         }
     }
     // forward map: record the shadow of every slot (CPU pointer, unit) for the reverse pass
-    if ((OPS & OP_INC) && sg.shadow && live) {
+    if (SH && (OPS & OP_INC) && sg.shadow && live) {
 #pragma unroll
       for (int m = 0; m < 2; ++m) {
         if (!((valid >> m) & 1)) continue;
@@ -652,31 +658,32 @@ static size_t slots_smem(const SlotArgs &a, int dir) {
          (a.tab.n_ext <= EXT_SMEM ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
 }
 
-template <int DIR, int OPS, int FH>
+template <int DIR, int OPS, int FH, int SH>
 static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
   size_t smem = slots_smem(a, DIR);
   // the 48 KiB default covers static + dynamic shared memory: opt in to the full carve-out once
   static bool configured = false;
   if (!configured) {
     cudaFuncAttributes fa;
-    cudaError_t e = cudaFuncGetAttributes(&fa, k_slots<DIR, OPS, FH>);
+    cudaError_t e = cudaFuncGetAttributes(&fa, k_slots<DIR, OPS, FH, SH>);
     if (e != cudaSuccess) return (int)e;
     int dev = 0, optin = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    e = cudaFuncSetAttribute(k_slots<DIR, OPS, FH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    e = cudaFuncSetAttribute(k_slots<DIR, OPS, FH, SH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              optin - (int)fa.sharedSizeBytes);
     if (e != cudaSuccess) return (int)e;
     configured = true;
   }
-  uint64_t want = (a.nchunks + SLOT_THREADS - 1) / SLOT_THREADS;
+  constexpr int T = SlotCfg<DIR, SH>::threads;
+  uint64_t want = (a.nchunks + T - 1) / T;
   int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
-  k_slots<DIR, OPS, FH><<<grid, SLOT_THREADS, smem, s>>>(a);
+  k_slots<DIR, OPS, FH, SH><<<grid, T, smem, s>>>(a);
   return (int)cudaGetLastError();  // 0 or the cudaError_t of the launch
 }
 
-// hot operation sets get depth-specialised forward lookups
+// hot operation sets get depth-specialised forward lookups (and shadow variants)
 #define CGCM_HOT_OPS(X)                             \
   X(DIR_FWD, OP_WRITE | OP_INC | OP_HITMASK)         \
   X(DIR_REV, OP_WRITE | OP_GATE | OP_DEC | OP_HITMASK) \
@@ -685,20 +692,28 @@ static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
 int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s) {
   // the forward index qualifies for the specialised path: one segment, no wide bucket, h <= 3
   int fh = a.fx.nseg <= 1 && a.fx_nowide && a.fx.h <= 3 ? a.fx.h : -1;
-#define X(D, O)                                        \
-  if (dir == D && ops == (O)) {                        \
-    switch (fh) {                                      \
-      case 0: return launch_one<D, (O), 0>(a, nsm, s); \
-      case 1: return launch_one<D, (O), 1>(a, nsm, s); \
-      case 2: return launch_one<D, (O), 2>(a, nsm, s); \
-      case 3: return launch_one<D, (O), 3>(a, nsm, s); \
-      default: return launch_one<D, (O), -1>(a, nsm, s); \
-    }                                                  \
+  const bool sh = a.nseg == 1 && a.segs_host_shadow;
+#define X(D, O)                                                        \
+  if (dir == D && ops == (O)) {                                        \
+    if (sh) {                                                          \
+      switch (fh) {                                                    \
+        case 2: return launch_one<D, (O), 2, 1>(a, nsm, s);            \
+        case 3: return launch_one<D, (O), 3, 1>(a, nsm, s);            \
+        default: return launch_one<D, (O), -1, 1>(a, nsm, s);          \
+      }                                                                \
+    }                                                                  \
+    switch (fh) {                                                      \
+      case 0: return launch_one<D, (O), 0, 0>(a, nsm, s);              \
+      case 1: return launch_one<D, (O), 1, 0>(a, nsm, s);              \
+      case 2: return launch_one<D, (O), 2, 0>(a, nsm, s);              \
+      case 3: return launch_one<D, (O), 3, 0>(a, nsm, s);              \
+      default: return launch_one<D, (O), -1, 0>(a, nsm, s);            \
+    }                                                                  \
   }
   CGCM_HOT_OPS(X)
 #undef X
 #define X(D, O) \
-  if (dir == D && ops == (O)) return launch_one<D, (O), -1>(a, nsm, s);
+  if (dir == D && ops == (O)) return launch_one<D, (O), -1, 0>(a, nsm, s);
   CGCM_SLOT_OPS(X)
 #undef X
   return -2;  // unsupported combination

@@ -528,6 +528,7 @@ struct Context {
       a.runid = rev.rid.as<uint32_t>();
     }
     a.segs = dsegs;
+    a.segs_host_shadow = (k == 1 && c.segs[0].shadow != 0) ? 1 : 0;
     a.seg_chunk0 = dc0;
     a.nseg = k;
     a.sel = c.sel;
@@ -1440,7 +1441,9 @@ int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n) {
   CKS(C->ensure_table());
   Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
   Context::Shadow *sh = nullptr;
-  if (n >= SHADOW_MIN) {  // record (CPU pointer, unit) per slot for the reverse pass (R13-ii)
+  // record (CPU pointer, unit) per slot for the reverse pass (R13-ii) when a lookup costs more than
+  // the 12-byte shadow: deep indexes (measured: a loss at h = 2, a win at h = 3)
+  if (n >= SHADOW_MIN && (C->fwd.h >= 3 || (C->flags & CGCM_FORCE_SHADOW))) {
     auto key = std::make_pair(s.ptr, (uint64_t)n);
     sh = &C->shadows[key];
     sh->valid = false;

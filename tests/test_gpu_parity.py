@@ -18,10 +18,10 @@ def cgcm_mod():
     return cg
 
 
-@pytest.fixture
-def pair(cgcm_mod):
+@pytest.fixture(params=[0, 8], ids=["auto", "shadow"])
+def pair(cgcm_mod, request):
     from oracle import Oracle
-    ctx = cgcm_mod.Context(0, arena_bytes=1 << 30)
+    ctx = cgcm_mod.Context(0, arena_bytes=1 << 30, flags=request.param)
     o = Oracle()
     p = Pair(ctx, o)
     yield p
