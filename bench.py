@@ -248,6 +248,28 @@ def run_cgcm(args, rank, world, local_rank):
     return result
 
 
+def host_link(dev, nbytes=256 << 20, reps=5):
+    """Pinned host<->device copy bandwidth of this GPU's link (best of reps, CUDA events)."""
+    import torch
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    s = torch.cuda.Stream(device=dev)
+    out = {}
+    for name, fn in (("h2d", lambda: d.copy_(h, non_blocking=True)), ("d2h", lambda: h.copy_(d, non_blocking=True))):
+        best = None
+        for _ in range(reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            with torch.cuda.stream(s):
+                e0.record(s)
+                fn()
+                e1.record(s)
+            e1.synchronize()
+            ms = e0.elapsed_time(e1)
+            best = ms if best is None else min(best, ms)
+        out[name + "_gbs"] = round(nbytes / (best / 1e3) / 1e9, 1)
+    return out
+
+
 def run_e2e(args, ctx, wl, q_ref, dev, world, rank):
     """Same metric through the host-array public API: cgcm_mapArrays / unmapArrays / releaseArrays on
     the rank's pointer arrays in pinned host memory (raw arrays H2D, translated in place, reverse
@@ -293,9 +315,14 @@ def run_e2e(args, ctx, wl, q_ref, dev, world, rank):
         t = torch.tensor([ms], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
+    link = host_link(dev)
+    h2d = (st1["h2d_bytes"] - st0["h2d_bytes"]) // steps
+    d2h = (st1["d2h_bytes"] - st0["d2h_bytes"]) // steps
+    floor_ms = 1e3 * (h2d / (link["h2d_gbs"] * 1e9) + d2h / (link["d2h_gbs"] * 1e9))
     return {"value": round(2 * wl.n * world * steps / (ms / 1e3), 1), "unit": "pointer translations/s",
-            "h2d_bytes_per_step": (st1["h2d_bytes"] - st0["h2d_bytes"]) // steps,
-            "d2h_bytes_per_step": (st1["d2h_bytes"] - st0["d2h_bytes"]) // steps,
+            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+            "host_link": link, "host_link_floor_ms_per_step": round(floor_ms, 3),
+            "frac_of_host_link": round(floor_ms / (ms / steps), 4),
             "ms_per_step": round(ms / steps, 3), "steps": steps,
             "api": "cgcm_mapArrays+advanceEpoch+cgcm_unmapArrays+cgcm_releaseArrays (pinned host arrays)",
             "host_arrays_roundtrip_ok": bool(ok)}
