@@ -76,3 +76,71 @@ def test_config_C_full_size():
 
 def test_config_E_full_table():
     run_full(1 << 22, 32, 1 << 20, 5)
+
+
+def test_config_D_full_size():
+    """Config D at full size: 2^24 node AUs of 32 B (allocated in a seeded permutation order) and a child
+    table of 2^25 slots; mapArray + map(root), 24 bottom-up S3 levels, unmapArray + unmap, releases.
+    Checked: every subtree sum bit-exact against a vectorised recomputation with the same association,
+    copy counts N+1 each way, N forward / N-1 reverse translations, the child table restored."""
+    import math
+    import torch
+    import paper_conf_pldi_jablinpjjba11_b200 as cg
+    from tests.harness import host_read
+
+    N = 1 << 24
+    vals = W.tree_values(N)
+    order = W.tree_alloc_order(N)
+    pos = np.empty(N, dtype=np.int64)
+    pos[order] = np.arange(N)
+    nodes_t = torch.zeros(N * 32, dtype=torch.uint8, pin_memory=True)
+    nodes = nodes_t.data_ptr()
+    arena = nodes_t.numpy().view(np.float64).reshape(N, 4)
+    arena[:, 1] = vals[order]
+    arena.view(np.int64)[:, 0] = order
+    addr = np.uint64(nodes) + np.uint64(32) * pos.astype(np.uint64)
+    child = W.tree_children(N)
+    table_t = torch.zeros(2 * N, dtype=torch.int64, pin_memory=True)
+    table = np.where(child >= 0, addr[np.maximum(child, 0)], 0).astype(np.uint64)
+    table_t.numpy().view(np.uint64)[:] = table
+    CB = table_t.data_ptr()
+    ctx = cg.Context(0, arena_bytes=4 << 30)
+    try:
+        bases = np.uint64(nodes) + np.uint64(32) * np.arange(N, dtype=np.uint64)
+        assert ctx.declareBatch(bases, np.full(N, 32, dtype=np.uint64)) == 0
+        assert ctx.declareAlloc(CB, 16 * N) == 0
+        st, cdev = ctx.mapArray(CB)
+        assert st == 0
+        st, rdev = ctx.map(int(addr[0]))
+        assert st == 0
+        for dlev in range(int(math.log2(N)), -1, -1):
+            lo, hi = (1 << dlev) - 1, min((1 << (dlev + 1)) - 1, N)
+            assert ctx.sample_treesum_level(cdev, rdev, N, lo, hi) == 0
+            ctx.synchronize()
+            ctx.advanceEpoch()
+        assert ctx.unmapArray(CB) == 0
+        assert ctx.unmap(int(addr[0])) == 0
+        assert ctx.releaseArray(CB) == 0
+        assert ctx.release(int(addr[0])) == 0
+        s = ctx.stats()
+        assert (s["h2d_units"], s["h2d_bytes"]) == (N + 1, 48 * N)
+        assert (s["d2h_units"], s["d2h_bytes"]) == (N + 1, 48 * N)
+        assert s["fwd_translations"] == N and s["rev_translations"] == N - 1
+        assert (table_t.numpy().view(np.uint64) == table).all()
+        # subtree sums, level by level with the kernel's association: (val + left) + right
+        exp = np.zeros(N)
+        for dlev in range(int(math.log2(N)), -1, -1):
+            lo, hi = (1 << dlev) - 1, min((1 << (dlev + 1)) - 1, N)
+            i = np.arange(lo, hi)
+            sm = vals[i].copy()
+            l, r = 2 * i + 1, 2 * i + 2
+            ml, mr = l < N, r < N
+            sm[ml] = sm[ml] + exp[l[ml]]
+            sm[mr] = sm[mr] + exp[r[mr]]
+            exp[i] = sm
+        got = arena[pos, 2]
+        assert got.tobytes() == exp.tobytes()
+        assert abs(got[0] - math.fsum(vals)) <= 1e-12 * abs(math.fsum(vals))
+        assert all(u["refCount"] == 0 for u in ctx.dump()[:1000])
+    finally:
+        ctx.close()
