@@ -112,6 +112,16 @@ int cgcm_declareGlobal(const char *name, void *base, size_t size, int isReadOnly
  * mapped -> the block is not freed).  NULL on failure.                                           */
 void *cgcm_malloc(size_t n);
 int cgcm_free(void *p);
+/* calloc/realloc wrappers (NEXT-1).  cgcm_realloc keeps the AU registered under its new
+ * base (the old registration expires); a mapped AU cannot move: NULL, nothing changes (BUSY).      */
+void *cgcm_calloc(size_t nmemb, size_t size);
+void *cgcm_realloc(void *p, size_t n);
+/* declareAlloca (Table 2): an escaping "stack" variable of n bytes, from the
+ * pinned arena, registered until the innermost scope opened with cgcm_scopeEnter exits.  Scopes nest;
+ * cgcm_scopeExit returns CGCM_E_BUSY (and keeps the scope) if one of its AUs is still mapped.        */
+void *cgcm_declareAlloca(size_t n);
+int cgcm_scopeEnter(void);
+int cgcm_scopeExit(void);
 
 /* ================================ mapping (Alg. 1-3, Table 2) ==============================
  * cgcm_map (Alg. 1): *gpu_out = devptr + (cpu - base) of the AU containing `cpu`;

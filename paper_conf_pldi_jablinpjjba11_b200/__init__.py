@@ -67,6 +67,8 @@ def lib():
             "cgcm_declareBatch": (i, [vp, vp, sz, C.c_uint]), "cgcm_undeclare": (i, [vp]),
             "cgcm_declareGlobal": (i, [C.c_char_p, vp, sz, i]),
             "cgcm_malloc": (vp, [sz]), "cgcm_free": (i, [vp]),
+            "cgcm_calloc": (vp, [sz, sz]), "cgcm_realloc": (vp, [vp, sz]),
+            "cgcm_declareAlloca": (vp, [sz]), "cgcm_scopeEnter": (i, []), "cgcm_scopeExit": (i, []),
             "cgcm_map": (i, [vp, vp]), "cgcm_unmap": (i, [vp]), "cgcm_release": (i, [vp]),
             "cgcm_mapArray": (i, [vp, vp]), "cgcm_unmapArray": (i, [vp]), "cgcm_releaseArray": (i, [vp]),
             "cgcm_advanceEpoch": (i, []), "cgcm_epoch": (u64, []),
@@ -170,6 +172,21 @@ class Context:
 
     def free(self, p: int) -> int:
         return self.L.cgcm_free(p)
+
+    def calloc(self, nmemb: int, size: int) -> int:
+        return self.L.cgcm_calloc(nmemb, size) or 0
+
+    def realloc(self, p: int, n: int) -> int:
+        return self.L.cgcm_realloc(p, n) or 0
+
+    def declareAlloca(self, n: int) -> int:
+        return self.L.cgcm_declareAlloca(n) or 0
+
+    def scopeEnter(self) -> int:
+        return self.L.cgcm_scopeEnter()
+
+    def scopeExit(self) -> int:
+        return self.L.cgcm_scopeExit()
 
     # ---- Table 2 ----
     def map(self, p: int):

@@ -508,3 +508,63 @@ def test_device_array_shadow_fallback_on_modified_slots(pair):
     assert (got == ref).all()
     P.check("after modified-slot unmap")
     W.release_reservation(R, span)
+
+
+def test_heap_churn_calloc_realloc_alloca(pair):
+    """NEXT-1: heap wrappers and declareAlloca scopes keep the allocation table current under churn
+    (P:L171-179); mapped AUs cannot move or expire; every step mirrored into the oracle."""
+    P = pair
+    g, o = P.g, P.o
+    rng = np.random.default_rng(3)
+    live = {}
+    for step in range(60):
+        r = rng.random()
+        if r < 0.3 or not live:
+            n = int(rng.integers(1, 300))
+            a = g.calloc(n, 1)
+            assert a and host_read(a, n) == bytes(n)
+            assert o.declareAlloc(a, n) == 0
+            o.host_write(a, bytes(n))
+            live[a] = n
+        elif r < 0.55:
+            a = list(live)[int(rng.integers(0, len(live)))]
+            n = int(rng.integers(1, 600))
+            old = host_read(a, live[a])
+            b = g.realloc(a, n)
+            assert b
+            assert host_read(b, min(n, live[a])) == old[:min(n, live[a])]
+            assert o.undeclare(a) == 0
+            assert o.declareAlloc(b, n) == 0
+            o.host_write(b, np.frombuffer(host_read(b, n), dtype=np.uint8))
+            del live[a]
+            live[b] = n
+        elif r < 0.75:
+            a = list(live)[int(rng.integers(0, len(live)))]
+            P.units[a] = live[a]
+            P.run("map", a)
+            b = g.realloc(a, live[a] + 64)             # mapped: cannot move
+            assert b == 0
+            P.run("release", a)
+        else:
+            a = list(live)[int(rng.integers(0, len(live)))]
+            assert g.free(a) == 0 and o.undeclare(a) == 0
+            del live[a]
+            P.units.pop(a, None)
+        P.units.update(live)
+        if step % 10 == 0:
+            P.check(f"churn {step}")
+    # declareAlloca scopes
+    assert g.scopeEnter() == 0
+    xs = [g.declareAlloca(64 + 8 * k) for k in range(5)]
+    for k, x in enumerate(xs):
+        assert x and o.declareAlloc(x, 64 + 8 * k) == 0
+        o.host_write(x, np.frombuffer(host_read(x, 64 + 8 * k), dtype=np.uint8))
+        P.units[x] = 64 + 8 * k
+    P.run("map", xs[2])
+    assert g.scopeExit() == -5                         # a mapped stack variable keeps the scope
+    P.run("release", xs[2])
+    assert g.scopeExit() == 0
+    for x in xs:
+        assert o.undeclare(x) == 0
+        P.units.pop(x)
+    P.check("after scopes")

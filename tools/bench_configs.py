@@ -1,0 +1,164 @@
+#!/usr/bin/env python
+"""Secondary measurements for the configs that are not the bench line: config A (jagged
+256x256, naive-cyclic vs map-promoted, 100 iterations: us per iteration and per call), config B (jagged gemm
+4096^2, 64 row-blocks, naive vs promoted: seconds, host-link GB/s of the copies), config D (2^24-node tree:
+map+unmap GB/s over the host link, translations/s).  Prints one JSON line per measurement."""
+import json
+import math
+import os
+import sys
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import paper_conf_pldi_jablinpjjba11_b200 as cg  # noqa: E402
+import workloads as W  # noqa: E402
+
+
+def timed(fn):
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    fn()
+    torch.cuda.synchronize()
+    return time.perf_counter() - t0
+
+
+def config_A(promoted, iters=100):
+    ctx = cg.Context(0, arena_bytes=1 << 30)
+    nrows = ncols = 256
+    vals = W.config_A_values(nrows, ncols, 1)
+    rows = []
+    for r in range(nrows):
+        a = ctx.malloc(8 * ncols)
+        np.ctypeslib.as_array((np.ctypeslib.ctypes.c_double * ncols).from_address(a))[:] = vals[r]
+        rows.append(a)
+    pp = ctx.malloc(8 * nrows)
+    np.ctypeslib.as_array((np.ctypeslib.ctypes.c_uint64 * nrows).from_address(pp))[:] = rows
+    calls = {"mapArray": 0.0, "kernel": 0.0, "unmapArray": 0.0, "releaseArray": 0.0}
+
+    def tcall(name, fn):
+        t0 = time.perf_counter()
+        r = fn()
+        calls[name] += time.perf_counter() - t0
+        return r
+
+    def run():
+        if promoted:
+            st, d0 = ctx.mapArray(pp)
+        for _ in range(iters):
+            st, d = tcall("mapArray", lambda: ctx.mapArray(pp))
+            tcall("kernel", lambda: (ctx.sample_scale(d, nrows, ncols, 0.999), ctx.synchronize()))
+            ctx.advanceEpoch()
+            if not promoted:
+                tcall("unmapArray", lambda: ctx.unmapArray(pp))
+            tcall("releaseArray", lambda: ctx.releaseArray(pp))
+        if promoted:
+            ctx.unmapArray(pp)
+            ctx.releaseArray(pp)
+
+    t = timed(run)
+    s = ctx.stats()
+    ctx.close()
+    return {"config": "A", "mode": "promoted" if promoted else "naive", "iterations": iters,
+            "us_per_iteration": round(1e6 * t / iters, 1),
+            "us_per_call": {k: round(1e6 * v / iters, 1) for k, v in calls.items()},
+            "h2d_units": s["h2d_units"], "h2d_bytes": s["h2d_bytes"], "d2h_units": s["d2h_units"],
+            "d2h_bytes": s["d2h_bytes"], "h2d_memcpy_calls": s["h2d_memcpy_calls"],
+            "d2h_memcpy_calls": s["d2h_memcpy_calls"]}
+
+
+def config_B(promoted, n=4096, blk=64):
+    ctx = cg.Context(0, arena_bytes=2 << 30)
+    mats = []
+    for m in range(3):
+        v = W.config_B_values(n, 2, m)
+        rows = []
+        for r in range(n):
+            a = ctx.malloc(8 * n)
+            np.ctypeslib.as_array((np.ctypeslib.ctypes.c_double * n).from_address(a))[:] = v[r]
+            rows.append(a)
+        pp = ctx.malloc(8 * n)
+        np.ctypeslib.as_array((np.ctypeslib.ctypes.c_uint64 * n).from_address(pp))[:] = rows
+        mats.append(pp)
+    A, B, C = mats
+
+    def run():
+        if promoted:
+            for pp in mats:
+                ctx.mapArray(pp)
+        for b0 in range(0, n, blk):
+            d = [ctx.mapArray(pp)[1] for pp in mats]
+            ctx.sample_gemm_rows(d[0], d[1], d[2], n, b0, blk, 1.5, 1.2)
+            ctx.synchronize()
+            ctx.advanceEpoch()
+            if not promoted:
+                ctx.unmapArray(C)
+            for pp in mats:
+                ctx.releaseArray(pp)
+        if promoted:
+            ctx.unmapArray(C)
+            for pp in mats:
+                ctx.releaseArray(pp)
+
+    t = timed(run)
+    s = ctx.stats()
+    ctx.close()
+    moved = s["h2d_bytes"] + s["d2h_bytes"]
+    return {"config": "B", "mode": "promoted" if promoted else "naive", "seconds": round(t, 3),
+            "h2d_units": s["h2d_units"], "h2d_bytes": s["h2d_bytes"], "d2h_units": s["d2h_units"],
+            "d2h_bytes": s["d2h_bytes"], "copy_GBs_over_wall": round(moved / t / 1e9, 2),
+            "h2d_memcpy_calls": s["h2d_memcpy_calls"], "d2h_memcpy_calls": s["d2h_memcpy_calls"],
+            "gemm_flops": 2 * n ** 3}
+
+
+def config_D(N=1 << 24):
+    vals = W.tree_values(N)
+    order = W.tree_alloc_order(N)
+    pos = np.empty(N, dtype=np.int64)
+    pos[order] = np.arange(N)
+    nodes_t = torch.zeros(N * 32, dtype=torch.uint8, pin_memory=True)
+    arena = nodes_t.numpy().view(np.float64).reshape(N, 4)
+    arena[:, 1] = vals[order]
+    addr = np.uint64(nodes_t.data_ptr()) + np.uint64(32) * pos.astype(np.uint64)
+    child = W.tree_children(N)
+    table_t = torch.zeros(2 * N, dtype=torch.int64, pin_memory=True)
+    table_t.numpy().view(np.uint64)[:] = np.where(child >= 0, addr[np.maximum(child, 0)], 0)
+    ctx = cg.Context(0, arena_bytes=4 << 30)
+    bases = np.uint64(nodes_t.data_ptr()) + np.uint64(32) * np.arange(N, dtype=np.uint64)
+    ctx.declareBatch(bases, np.full(N, 32, dtype=np.uint64))
+    ctx.declareAlloc(table_t.data_ptr(), 16 * N)
+    CB, root = table_t.data_ptr(), int(addr[0])
+    tm = timed(lambda: (ctx.mapArray(CB), ctx.map(root)))
+    cdev = ctx.mapArray(CB)[1]
+    ctx.releaseArray(CB)
+    rdev = ctx.map(root)[1]
+    ctx.release(root)
+    for dlev in range(int(math.log2(N)), -1, -1):
+        lo, hi = (1 << dlev) - 1, min((1 << (dlev + 1)) - 1, N)
+        ctx.sample_treesum_level(cdev, rdev, N, lo, hi)
+        ctx.synchronize()
+        ctx.advanceEpoch()
+    tu = timed(lambda: (ctx.unmapArray(CB), ctx.unmap(root)))
+    ctx.releaseArray(CB)
+    ctx.release(root)
+    ctx.close()
+    b = 48 * N
+    return {"config": "D", "nodes": N, "map_seconds": round(tm, 4), "unmap_seconds": round(tu, 4),
+            "map_GBs": round(b / tm / 1e9, 2), "unmap_GBs": round(b / tu / 1e9, 2),
+            "map_translations_per_s": round(N / tm, 1), "unmap_translations_per_s": round((N - 1) / tu, 1)}
+
+
+if __name__ == "__main__":
+    which = sys.argv[1:] or ["A", "B", "D"]
+    for w in which:
+        if w == "A":
+            for p in (False, True):
+                print(json.dumps(config_A(p)), flush=True)
+        elif w == "B":
+            for p in (True, False):
+                print(json.dumps(config_B(p)), flush=True)
+        elif w == "D":
+            print(json.dumps(config_D()), flush=True)
