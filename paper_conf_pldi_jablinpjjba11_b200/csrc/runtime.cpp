@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdint>
 #include <cstdio>
 #include <cstring>
 #include <map>
@@ -147,9 +148,6 @@ struct HostUnit {
   uint64_t epoch0 = 0;      // globalEpoch at declaration (A20)
   int32_t idx = -1;         // rank in the device table (valid after a table build)
   std::string name;
-  uint64_t devbase = 0;     // mirror of the device copy's address (host allocates it)
-  int64_t run = -1;         // device extent holding the copy
-  bool arrayMapped = false; // mirror of UF_ARRAYMAPPED
 };
 
 // one device extent holding the copies of one or more host-adjacent units (mirrored layout)
@@ -199,7 +197,12 @@ struct Context {
 
   // registry (host)
   std::map<uint64_t, HostUnit> reg;
-  std::vector<std::map<uint64_t, HostUnit>::iterator> by_idx;
+  // per-unit host state by table rank (structure of arrays, rebuilt by ensure_table): the
+  // activation / copy-back / release loops walk these contiguously instead of the registry's nodes
+  std::vector<uint64_t> ubase, usize, udev;  // host base, size, device copy address (0: none)
+  std::vector<uint32_t> uflags;              // UF_GLOBAL | UF_READONLY
+  std::vector<int64_t> urun;                 // device extent holding the copy (-1: none)
+  std::vector<uint8_t> uarr;                 // mirror of UF_ARRAYMAPPED
   std::unordered_set<std::string> names;
   bool table_dirty = true, rev_dirty = true;
   int U = 0;  // units in the device table
@@ -225,6 +228,8 @@ struct Context {
   std::vector<std::pair<char *, size_t>> hchunks;
   std::map<uint64_t, uint64_t> hfree;                 // addr -> len
   std::unordered_map<uint64_t, uint64_t> hallocs;     // addr -> rounded len
+  std::unordered_map<uint64_t, uint64_t> hsizes;      // addr -> requested size (realloc)
+  std::vector<std::vector<uint64_t>> scopes;           // declareAlloca registrations per open scope
 
   cgcm_stats_t st{};
 
@@ -393,17 +398,31 @@ struct Context {
     uint32_t *he = reinterpret_cast<uint32_t *>(hs + n);
     int32_t *ho = reinterpret_cast<int32_t *>(he + n);
     uint32_t *hf = reinterpret_cast<uint32_t *>(ho + n);
-    by_idx.assign(n, reg.end());
+    std::vector<uint64_t> ndev(n, 0);
+    std::vector<int64_t> nrun(n, -1);
+    std::vector<uint8_t> narr(n, 0);
+    uflags.resize(n);
     int i = 0;
     for (auto it = reg.begin(); it != reg.end(); ++it, ++i) {
+      int32_t o = it->second.idx;
       hb[i] = it->first;
       hs[i] = it->second.size;
       he[i] = rel_epoch(it->second.epoch0);
-      ho[i] = it->second.idx;
+      ho[i] = o;
       hf[i] = it->second.flags & (UF_GLOBAL | UF_READONLY);
+      uflags[i] = hf[i];
+      if (o >= 0) {
+        ndev[i] = udev[o];
+        nrun[i] = urun[o];
+        narr[i] = uarr[o];
+      }
       it->second.idx = i;
-      by_idx[i] = it;
     }
+    ubase.assign(hb, hb + n);
+    usize.assign(hs, hs + n);
+    udev.swap(ndev);
+    urun.swap(nrun);
+    uarr.swap(narr);
     DevBuf nhot, nrc, nep, nsize, nbase, tmp;
     int cap = std::max(n, 1);
     CKS(dalloc(nhot, 8 * (size_t)cap));
@@ -682,10 +701,9 @@ struct Context {
     std::vector<Pack> packs;
     uint64_t bytes = 0;
     for (size_t i = 0; i < units.size(); ++i) {
-      auto it = by_idx[units[i]];
-      uint64_t b = it->first, sz = it->second.size;
+      uint64_t b = ubase[units[i]], sz = usize[units[i]];
       bytes += sz;
-      bool g = (it->second.flags & UF_GLOBAL) != 0;
+      bool g = (uflags[units[i]] & UF_GLOBAL) != 0;
       if (!g && !packs.empty() && !packs.back().global && b >= packs.back().h1 && b - packs.back().h1 <= GAPMAX &&
           b + sz - packs.back().h0 <= PACK_SPAN) {
         Pack &P = packs.back();
@@ -699,11 +717,11 @@ struct Context {
     std::vector<uint64_t> devbases(units.size());
     std::vector<int64_t> created;
     for (auto &P : packs) {
-      HostUnit &u0 = by_idx[units[P.i]]->second;
-      if (P.global && u0.run >= 0) {  // named region allocated on an earlier activation (A14)
-        P.dev0 = u0.devbase;
-        P.run = u0.run;
-        devbases[P.i] = u0.devbase;
+      uint32_t x0 = units[P.i];
+      if (P.global && urun[x0] >= 0) {  // named region allocated on an earlier activation (A14)
+        P.dev0 = udev[x0];
+        P.run = urun[x0];
+        devbases[P.i] = udev[x0];
         continue;
       }
       uint64_t need = (P.h0 % 256) + (P.h1 - P.h0) + 1;
@@ -712,10 +730,10 @@ struct Context {
         for (int64_t r : created) drop_run(r);
         for (auto &Q : packs)
           for (size_t q = Q.i; q < Q.j && Q.run >= 0; ++q) {
-            HostUnit &u = by_idx[units[q]]->second;
-            if (std::find(created.begin(), created.end(), u.run) != created.end()) {
-              u.run = -1;
-              u.devbase = 0;
+            uint32_t x = units[q];
+            if (std::find(created.begin(), created.end(), urun[x]) != created.end()) {
+              urun[x] = -1;
+              udev[x] = 0;
             }
           }
         return CGCM_E_NOMEM;
@@ -724,15 +742,15 @@ struct Context {
       P.run = new_run(a, need, P.h0 - P.dev0);
       created.push_back(P.run);
       for (size_t q = P.i; q < P.j; ++q) {
-        auto it = by_idx[units[q]];
-        it->second.devbase = P.dev0 + (it->first - P.h0);
-        it->second.run = P.run;
-        runs[P.run].live += 1;
-        devbases[q] = it->second.devbase;
+        uint32_t x = units[q];
+        udev[x] = P.dev0 + (ubase[x] - P.h0);
+        urun[x] = P.run;
+        devbases[q] = udev[x];
       }
+      runs[P.run].live += (int64_t)(P.j - P.i);
     }
     std::vector<uint32_t> exts(units.size());
-    for (size_t q = 0; q < units.size(); ++q) exts[q] = (uint32_t)by_idx[units[q]]->second.run;
+    for (size_t q = 0; q < units.size(); ++q) exts[q] = (uint32_t)urun[units[q]];
     if (runs.size() > EXT_MASK) return CGCM_E_NOMEM;  // 2^24 live extents
     CKS(sync_ext());
     CKS(upload(up_units, units));
@@ -773,12 +791,12 @@ struct Context {
   void gather(const std::vector<uint32_t> &units, size_t i, size_t j, uint64_t h0, char *stg) {
     size_t n = j - i;
     uint64_t total = 0;
-    for (size_t q = i; q < j; ++q) total += by_idx[units[q]]->second.size;
+    for (size_t q = i; q < j; ++q) total += usize[units[q]];
     unsigned T = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
     auto work = [&](size_t lo, size_t hi) {
       for (size_t q = lo; q < hi; ++q) {
-        auto it = by_idx[units[q]];
-        std::memcpy(stg + (it->first - h0), reinterpret_cast<const void *>(it->first), it->second.size);
+        uint32_t x = units[q];
+        std::memcpy(stg + (ubase[x] - h0), reinterpret_cast<const void *>(ubase[x]), usize[x]);
       }
     };
     if (total < (8ull << 20) || T == 1 || n < 64) {
@@ -809,8 +827,7 @@ struct Context {
     }
     (void)cudaGetLastError();
     for (size_t q = i; q < j; ++q) {
-      auto it = by_idx[units[q]];
-      uint64_t hb = it->first, n = it->second.size, db = dev + (hb - host);
+      uint64_t hb = ubase[units[q]], n = usize[units[q]], db = dev + (hb - host);
       if (h2d) CK(cudaMemcpyAsync(reinterpret_cast<void *>(db), reinterpret_cast<const void *>(hb), n,
                                   cudaMemcpyHostToDevice, s));
       else CK(cudaMemcpyAsync(reinterpret_cast<void *>(hb), reinterpret_cast<const void *>(db), n,
@@ -829,12 +846,11 @@ struct Context {
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(main));
     for (uint32_t x : units) {
-      HostUnit &u = by_idx[x]->second;
-      u.arrayMapped = false;
-      if (u.flags & UF_GLOBAL) continue;
-      run_release(u.run);
-      u.run = -1;
-      u.devbase = 0;
+      uarr[x] = 0;
+      if (uflags[x] & UF_GLOBAL) continue;
+      run_release(urun[x]);
+      urun[x] = -1;
+      udev[x] = 0;
       st.frees += 1;
     }
     rev_dirty = true;
@@ -846,10 +862,10 @@ struct Context {
   int copy_back(const std::vector<uint32_t> &units) {
     if (units.empty()) return CGCM_OK;
     std::vector<uint32_t> plain, arr;
-    for (uint32_t x : units) (by_idx[x]->second.arrayMapped ? arr : plain).push_back(x);
+    for (uint32_t x : units) (uarr[x] ? arr : plain).push_back(x);
     // reverse-translate the array-mapped ones into staging_cb
     uint64_t arr_bytes = 0;
-    for (uint32_t x : arr) arr_bytes += align_up(by_idx[x]->second.size / 8 * 8, 32) + 32;
+    for (uint32_t x : arr) arr_bytes += align_up(usize[x] / 8 * 8, 32) + 32;
     if (!arr.empty()) {
       CKS(ensure_rev());
       CKS(dalloc(staging_cb, arr_bytes + 256));
@@ -859,12 +875,12 @@ struct Context {
       uint64_t off = staging_cb.addr;
       std::vector<uint64_t> dst(arr.size());
       for (size_t q = 0; q < arr.size(); ++q) {
-        HostUnit &u = by_idx[arr[q]]->second;
-        uint64_t n = u.size / 8;
-        off = align_up(off, 32) + (u.devbase & 31);  // same alignment as the source
+        uint32_t x = arr[q];
+        uint64_t n = usize[x] / 8;
+        off = align_up(off, 32) + (udev[x] & 31);  // same alignment as the source
         dst[q] = off;
         Seg s;
-        s.ptr = u.devbase;
+        s.ptr = udev[x];
         s.n = n;
         s.out = off;
         s.inc = 0;
@@ -882,33 +898,32 @@ struct Context {
       st.rev_translations += sts[7].translated;
       st.passthrough += (flags & CGCM_LENIENT) ? sts[7].misses : 0;
       for (size_t q = 0; q < arr.size(); ++q) {
-        auto it = by_idx[arr[q]];
-        HostUnit &u = it->second;
-        uint64_t n = u.size / 8;
-        if (n) CK(cudaMemcpyAsync(reinterpret_cast<void *>(it->first), reinterpret_cast<void *>(dst[q]), 8 * n,
+        uint32_t x = arr[q];
+        uint64_t hb = ubase[x], sz = usize[x], db = udev[x], n = sz / 8;
+        if (n) CK(cudaMemcpyAsync(reinterpret_cast<void *>(hb), reinterpret_cast<void *>(dst[q]), 8 * n,
                                   cudaMemcpyDeviceToHost, copy));
-        if (u.size > 8 * n)
-          CK(cudaMemcpyAsync(reinterpret_cast<void *>(it->first + 8 * n), reinterpret_cast<void *>(u.devbase + 8 * n),
-                             u.size - 8 * n, cudaMemcpyDeviceToHost, copy));
-        st.d2h_memcpy_calls += 1 + (u.size > 8 * n);
+        if (sz > 8 * n)
+          CK(cudaMemcpyAsync(reinterpret_cast<void *>(hb + 8 * n), reinterpret_cast<void *>(db + 8 * n), sz - 8 * n,
+                             cudaMemcpyDeviceToHost, copy));
+        st.d2h_memcpy_calls += 1 + (sz > 8 * n);
         st.d2h_units += 1;
-        st.d2h_bytes += u.size;
+        st.d2h_bytes += sz;
       }
     }
     // plain units: coalesce host-adjacent units whose device copies are mirrored
     size_t i = 0;
     while (i < plain.size()) {
-      auto it0 = by_idx[plain[i]];
-      uint64_t h0 = it0->first, d0 = it0->second.devbase, hend = h0 + it0->second.size;
+      uint32_t x0 = plain[i];
+      uint64_t h0 = ubase[x0], d0 = udev[x0], hend = h0 + usize[x0];
       st.d2h_units += 1;
-      st.d2h_bytes += it0->second.size;
+      st.d2h_bytes += usize[x0];
       size_t j = i + 1;
       while (j < plain.size() && plain[j] == plain[j - 1] + 1) {
-        auto it = by_idx[plain[j]];
-        if (it->first != hend || it->second.devbase != d0 + (it->first - h0)) break;
-        hend += it->second.size;
+        uint32_t x = plain[j];
+        if (ubase[x] != hend || udev[x] != d0 + (ubase[x] - h0)) break;
+        hend += usize[x];
         st.d2h_units += 1;
-        st.d2h_bytes += it->second.size;
+        st.d2h_bytes += usize[x];
         ++j;
       }
       CKS(copy_run(d0, h0, hend - h0, false, plain, i, j, copy));
@@ -1363,7 +1378,11 @@ int cgcm_undeclare(void *base) {
   }
   if (u.flags & UF_GLOBAL) {
     C->names.erase(u.name);
-    if (u.run >= 0) C->run_release(u.run);
+    if (u.idx >= 0 && C->urun[u.idx] >= 0) {
+      C->run_release(C->urun[u.idx]);
+      C->urun[u.idx] = -1;
+      C->udev[u.idx] = 0;
+    }
   }
   C->reg.erase(it);
   C->table_dirty = true;
@@ -1398,6 +1417,7 @@ void *cgcm_malloc(size_t n) {
     return nullptr;
   }
   C->hallocs[a] = len;
+  C->hsizes[a] = n;
   return reinterpret_cast<void *>(a);
 }
 int cgcm_free(void *p) {
@@ -1412,6 +1432,7 @@ int cgcm_free(void *p) {
   if (s != CGCM_OK) return s;
   uint64_t len = it->second;
   C->hallocs.erase(it);
+  C->hsizes.erase(a);
   // coalesce with neighbours
   auto nx = C->hfree.lower_bound(a);
   if (nx != C->hfree.end() && nx->first == a + len) {
@@ -1428,6 +1449,74 @@ int cgcm_free(void *p) {
     }
   }
   C->hfree.emplace(a, len);
+  return CGCM_OK;
+}
+
+void *cgcm_calloc(size_t nmemb, size_t size) {
+  if (nmemb && size > SIZE_MAX / nmemb) return nullptr;
+  void *p = cgcm_malloc(nmemb * size);
+  if (p) std::memset(p, 0, nmemb * size);
+  return p;
+}
+
+void *cgcm_realloc(void *p, size_t n) {
+  Context *C = tl_ctx;
+  if (!C) return nullptr;
+  if (!p) return cgcm_malloc(n);
+  if (n == 0) {
+    cgcm_free(p);
+    return nullptr;
+  }
+  std::lock_guard<std::recursive_mutex> lk(C->mu);
+  uint64_t a = reinterpret_cast<uint64_t>(p);
+  auto it = C->hsizes.find(a);
+  if (it == C->hsizes.end()) return nullptr;
+  auto ru = C->reg.find(a);
+  if (ru != C->reg.end() && ru->second.idx >= 0) {  // a mapped AU cannot move (BUSY)
+    int32_t rc = 0;
+    if (cudaMemcpy(&rc, C->rcb.as<int32_t>() + ru->second.idx, 4, cudaMemcpyDeviceToHost) != cudaSuccess || rc > 0)
+      return nullptr;
+  }
+  size_t old = it->second;
+  void *q = cgcm_malloc(n);
+  if (!q) return nullptr;
+  std::memcpy(q, p, std::min(old, n));
+  if (cgcm_free(p) != CGCM_OK) {
+    cgcm_free(q);
+    return nullptr;
+  }
+  return q;
+}
+
+int cgcm_scopeEnter(void) {
+  CTX();
+  C->scopes.emplace_back();
+  return CGCM_OK;
+}
+void *cgcm_declareAlloca(size_t n) {
+  Context *C = tl_ctx;
+  if (!C) return nullptr;
+  std::lock_guard<std::recursive_mutex> lk(C->mu);
+  if (C->scopes.empty()) C->scopes.emplace_back();  // an implicit outermost scope
+  void *p = cgcm_malloc(n);
+  if (p) C->scopes.back().push_back(reinterpret_cast<uint64_t>(p));
+  return p;
+}
+int cgcm_scopeExit(void) {
+  CTX();
+  if (C->scopes.empty()) return CGCM_E_INVALID;
+  auto &sc = C->scopes.back();
+  // all-or-nothing: no registration expires while one of the scope's AUs is mapped
+  CKS(C->ensure_table());
+  for (uint64_t a : sc) {
+    auto ru = C->reg.find(a);
+    if (ru == C->reg.end() || ru->second.idx < 0) continue;
+    int32_t rc = 0;
+    CK(cudaMemcpy(&rc, C->rcb.as<int32_t>() + ru->second.idx, 4, cudaMemcpyDeviceToHost));
+    if (rc > 0) return CGCM_E_BUSY;
+  }
+  for (auto it = sc.rbegin(); it != sc.rend(); ++it) CKS(cgcm_free(reinterpret_cast<void *>(*it)));
+  C->scopes.pop_back();
   return CGCM_OK;
 }
 
@@ -1648,12 +1737,12 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
   std::vector<UnitOp> ops;
   std::vector<Seg> fsegs, rsegs;
   for (auto &o : outs) {
-    HostUnit &hu = C->by_idx[o.unit]->second;
+    const uint64_t hu_dev = C->udev[o.unit];
     ops.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)o.mult});
     ops.push_back({(uint32_t)o.unit, UOP_OR_FLAGS, UF_ARRAYMAPPED});
     uint64_t n = o.info.size / 8;
     if (!n) continue;
-    Seg s{hu.devbase, n, 0, o.mult, 0};
+    Seg s{hu_dev, n, 0, o.mult, 0};
     if (o.info.refcount > 0 && (o.info.flags & UF_ARRAYMAPPED)) rsegs.push_back(s);  // A9: refcounts only
     else fsegs.push_back(s);
   }
@@ -1675,7 +1764,7 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
     uint64_t frees0 = C->st.frees;
     C->st.activations -= act.size();
     C->st.h2d_units -= act.size();
-    for (uint32_t x : act) C->st.h2d_bytes -= C->by_idx[x]->second.size;
+    for (uint32_t x : act) C->st.h2d_bytes -= C->usize[x];
     C->free_units(deact);
     C->st.frees = frees0;
   };
@@ -1703,7 +1792,7 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
       }
       for (auto &sg : rsegs) {
         for (auto &o : outs)
-          if (C->by_idx[o.unit]->second.devbase == sg.ptr) {
+          if (C->udev[o.unit] == sg.ptr) {
             CK(cudaMemcpyAsync(reinterpret_cast<void *>(sg.ptr), reinterpret_cast<const void *>(o.info.base),
                                8 * sg.n, cudaMemcpyHostToDevice, C->main));
             C->st.h2d_memcpy_calls += 1;
@@ -1730,10 +1819,10 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
     C->st.null_slots += rres.nulls;
     if (C->flags & CGCM_LENIENT) C->st.passthrough += rres.misses;
   }
-  for (auto &o : outs) C->by_idx[o.unit]->second.arrayMapped = true;
+  for (auto &o : outs) C->uarr[o.unit] = 1;
   for (size_t j = 0; j < k; ++j) {
     const Outer &o = outs[which[j]];
-    uint64_t dev = C->by_idx[o.unit]->second.devbase;
+    uint64_t dev = C->udev[o.unit];
     gpu_out[j] = reinterpret_cast<void **>(dev + (reinterpret_cast<uint64_t>(arrays[j]) - o.info.base));
   }
   return CGCM_OK;
@@ -1968,7 +2057,7 @@ int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
   for (size_t i = 0; i < m; ++i) {
     cgcm_unit_t &u = out[i];
     const uint32_t fl = hot_flags(hots[i]);
-    u.base = C->by_idx[i]->first;
+    u.base = C->ubase[i];
     u.size = szs[i];
     bool act = rcs[i] > 0;
     uint32_t e = hot_ext(hots[i]);
