@@ -16,7 +16,8 @@ import os
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libcgcm.so")
+# CGCM_LIBDIR: load a variant build of the same library (kernel A/B experiments, build.py --variant)
+LIB_PATH = os.path.join(os.environ.get("CGCM_LIBDIR") or HERE, "libcgcm.so")
 SAMPLES_PATH = os.path.join(HERE, "libcgcm_samples.so")
 
 OK = 0

@@ -39,6 +39,24 @@ def _run(cmd):
     return r.stdout + r.stderr
 
 
+def build_variant(out_dir: str, defines: list[str]) -> str:
+    """Build libcgcm.so with extra -D defines into out_dir (kernel A/B experiments; the binding loads
+    it when CGCM_LIBDIR=out_dir).  Returns the library path."""
+    os.makedirs(out_dir, exist_ok=True)
+    objs = []
+    jobs = []
+    for name, src in (("kernels", os.path.join(CSRC, "kernels.cu")), ("runtime", os.path.join(CSRC, "runtime.cpp"))):
+        obj = os.path.join(out_dir, name + ".o")
+        lang = ["-x", "cu"] if src.endswith(".cu") else ["-x", "c++"]
+        jobs.append([NVCC] + ARCH + COMMON + [f"-D{d}" for d in defines] + lang + ["-c", src, "-o", obj])
+        objs.append(obj)
+    with ThreadPoolExecutor(max_workers=2) as ex:
+        list(ex.map(_run, jobs))
+    lib = os.path.join(out_dir, "libcgcm.so")
+    _run([NVCC] + ARCH + ["-shared", "-o", lib] + objs + ["-lcudart"])
+    return lib
+
+
 def build(verbose: bool = False) -> None:
     hdrs = [os.path.join(INC, "cgcm.h"), os.path.join(CSRC, "cgcm_dev.h")]
     units = {
@@ -71,5 +89,8 @@ def build(verbose: bool = False) -> None:
 
 
 if __name__ == "__main__":
-    build(verbose="-v" in sys.argv)
-    print("built", LIB)
+    if len(sys.argv) > 2 and sys.argv[1] == "--variant":  # --variant OUT_DIR [DEFINE ...]
+        print("built", build_variant(sys.argv[2], sys.argv[3:]))
+    else:
+        build(verbose="-v" in sys.argv)
+        print("built", LIB)

@@ -7,18 +7,23 @@
 
 namespace cgcm {
 
-// The allocation-unit table (D3) as columns indexed by the unit's rank in base order.
-// A forward translation touches one 8-byte word per slot (hot) plus the refcount reduction:
-//   hot[u]   = size (bits 0..31; 0xFFFFFFFF = see size64) | extent id (bits 32..55) | flags (56..63)
-//   rc[u]    = refCount (i32, Alg. 1/3)
-//   epoch[u] = Alg. 2's per-unit epoch, u32 relative to the context's epoch origin (A28)
+// The allocation-unit table (D3), indexed by the unit's rank in base order.  The
+// per-unit words a slot touches live in ONE 16-byte record, so a lookup's record gather brings the
+// refcount and epoch into L2 with the hot word (one sector per unit; the refcount reduction and the
+// epoch gate that follow hit the line the gather just fetched):
+//   rec[u].hot   = size (bits 0..31; 0xFFFFFFFF = see size64) | extent id (bits 32..55) | flags (56..63)
+//   rec[u].rc    = refCount (i32, Alg. 1/3)
+//   rec[u].epoch = Alg. 2's per-unit epoch, u32 relative to the context's epoch origin (A28)
 //   base[u]  = the sorted key array of the forward index; size64[u] = full size (cold)
 //   ext_delta[e] = devbase - base for every unit copy in device extent e (mirrored layout):
 //              translation = p + ext_delta[extent(u)]  (Alg. 1: devptr + (ptr - base))
+struct __align__(16) UnitRec {
+  uint64_t hot;
+  int32_t rc;
+  uint32_t epoch;
+};
 struct TableDev {
-  uint64_t *hot;
-  int32_t *rc;
-  uint32_t *epoch;
+  UnitRec *rec;
   const uint64_t *base;
   const uint64_t *size64;
   const uint64_t *ext_delta;

@@ -20,7 +20,6 @@ namespace cgcm {
 
 namespace {
 
-constexpr int SLOT_THREADS = 1024;
 constexpr int SEG_SMEM = 256;
 
 __device__ __forceinline__ uint64_t policy_evict_first() {
@@ -90,6 +89,20 @@ __device__ __forceinline__ uint32_t spread16(uint32_t x) {
   return x;
 }
 
+// Position of the largest entry <= r among the 8 sorted u32 of one 32-byte level sector (entry 0 is
+// always <= r on a lookup path: every group starts at its parent's key).  Branch-free 3-step binary
+// search (3 compares + 3 selects) instead of 8 compares; last8 returns the entry itself (bottom level).
+__device__ __forceinline__ int idx8(const uint64_t w[4], uint32_t r) {
+  const bool b4 = (uint32_t)w[2] <= r;                                // entry 4
+  const bool b2 = (uint32_t)(b4 ? w[3] : w[1]) <= r;                  // entry 6 or 2
+  const uint64_t wq = b4 ? (b2 ? w[3] : w[2]) : (b2 ? w[1] : w[0]);  // entries (i, i+1), i = 4*b4 + 2*b2
+  const bool b1 = (uint32_t)(wq >> 32) <= r;
+  return (b4 ? 4 : 0) + (b2 ? 2 : 0) + (b1 ? 1 : 0);
+}
+__device__ __forceinline__ uint32_t last8(const uint64_t w[4], int i) {
+  const uint64_t wq = (i & 4) ? ((i & 2) ? w[3] : w[2]) : ((i & 2) ? w[1] : w[0]);
+  return (i & 1) ? (uint32_t)(wq >> 32) : (uint32_t)wq;
+}
 // number of entries <= r among 8 sorted u32 (one 32-byte level sector), and the largest of them
 __device__ __forceinline__ int count8(const uint64_t w[4], uint32_t r, uint32_t &last) {
   int c = 0;
@@ -103,12 +116,6 @@ __device__ __forceinline__ int count8(const uint64_t w[4], uint32_t r, uint32_t 
   }
   return c;
 }
-__device__ __forceinline__ uint64_t ld_u64(const uint64_t *p, uint64_t pol) {
-  uint64_t v;
-  asm volatile("ld.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
-  return v;
-}
-
 // ---- an index's top level, staged in shared memory -------------------------------------------
 struct SIdx {
   const uint64_t *top;
@@ -227,8 +234,18 @@ __device__ __forceinline__ void level_lookup2_fixed(const IndexDev &ix, uint64_t
     uint64_t w0[4], w1[4];
     ld_sector(L + 8 * (size_t)j[0], pol, w0);
     ld_sector(L + 8 * (size_t)j[1], pol, w1);
+#ifdef CGCM_COUNT8_LINEAR
     j[0] = 8 * j[0] + count8(w0, rel[0], last[0]) - 1;
     j[1] = 8 * j[1] + count8(w1, rel[1], last[1]) - 1;
+#else
+    const int i0 = idx8(w0, rel[0]), i1 = idx8(w1, rel[1]);
+    j[0] = 8 * j[0] + i0;
+    j[1] = 8 * j[1] + i1;
+    if (k == 0) {
+      last[0] = last8(w0, i0);
+      last[1] = last8(w1, i1);
+    }
+#endif
   }
 #pragma unroll
   for (int m = 0; m < 2; ++m) {
@@ -292,7 +309,11 @@ __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix,
 // threads per CTA: the shadow reverse variant keeps both paths live and gets more registers
 template <int DIR, int SH>
 struct SlotCfg {
+#ifdef CGCM_SLOT_THREADS
+  static constexpr int threads = CGCM_SLOT_THREADS;
+#else
   static constexpr int threads = 768;  // measured: 768 > 1024 (spills) > 512 on configs C and E
+#endif
 };
 
 template <int DIR, int OPS, int FH, int SH>
@@ -381,7 +402,9 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
     // reverse pass over slots the forward map recorded (unchanged since, R13-ii): one check
     bool sh[2] = {false, false};
     int jsh[2] = {0, 0};
-    uint64_t hsh[2] = {0, 0}, hwsh[2] = {0, 0};
+    uint64_t hsh[2] = {0, 0};
+    // the unit's record: hot word (size | extent | flags), then refcount | epoch << 32
+    uint64_t hw[2] = {0, 0}, rw[2] = {0, 0};
     const int64_t slot0 = ((int64_t)(a0 - sg.ptr)) >> 3;  // slot index of m = 0 (-1 for a head chunk)
     if (SH && DIR == DIR_REV && sg.shadow) {
 #pragma unroll
@@ -391,18 +414,25 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         const uint32_t u = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n)[i];
         if (u == 0xFFFFFFFFu) continue;
         const uint64_t h = reinterpret_cast<const uint64_t *>(sg.shadow)[i];
-        const uint64_t w = ld_u64(a.tab.hot + u, pol_t);
+        uint64_t w, r;
+        ld_pair(a.tab.rec + u, pol_t, w, r);
         const uint32_t e = hot_ext(w);
         if ((hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext &&
             q[m] == h + (ext_s ? s_ext[e] : a.tab.ext_delta[e])) {
           sh[m] = true;
           jsh[m] = (int)u;
           hsh[m] = h;
-          hwsh[m] = w;
+          hw[m] = w;
+          rw[m] = r;
           look[m] = false;
         }
       }
     }
+    // full lookups only where a lane still needs one: after the shadow check most reverse warps skip
+    // the whole search (a warp-uniform branch, not predication)
+    j[0] = j[1] = -1;
+    key[0] = key[1] = 0;
+    if (!(SH && DIR == DIR_REV) || __any_sync(0xffffffffu, look[0] || look[1])) {
     if (DIR == DIR_REV) {
       // the device extent holding the pointer, and the host address it mirrors
 #pragma unroll
@@ -432,13 +462,13 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
     if constexpr (FH > 0) level_lookup2_fixed<FH>(a.fx, pol_t, q, j, key);
     else if constexpr (FH < 0) level_lookup2(F, a.fx, pol_t, q, j, key);
 
-    // ---- the unit's hot word: size | extent | flags ----
-    uint64_t hw[2] = {0, 0};
+    // ---- the unit's record: hot word (size | extent | flags), refcount, epoch: one 16-B gather ----
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
       look[m] = look[m] && j[m] >= 0;
-      if (look[m]) hw[m] = ld_u64(a.tab.hot + j[m], pol_t);
+      if (look[m]) ld_pair(a.tab.rec + j[m], pol_t, hw[m], rw[m]);
     }
+    }  // full lookups
     bool hit[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
@@ -450,7 +480,8 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         if (!(hit[m] && (hot_flags(hw[m]) & UF_ACTIVE) && hot_ext(hw[m]) == rid[m])) {
           hit[m] = false;
           if (j[m] > 0 && q[m] == key[m]) {  // one past the end of the previous unit (A7)
-            const uint64_t h2 = a.tab.hot[j[m] - 1], b2 = a.tab.base[j[m] - 1];
+            const UnitRec r2 = a.tab.rec[j[m] - 1];
+            const uint64_t h2 = r2.hot, b2 = a.tab.base[j[m] - 1];
             uint64_t s2 = hot_size32(h2);
             if (s2 == BIG_SIZE) s2 = a.tab.size64[j[m] - 1];
             if ((hot_flags(h2) & UF_ACTIVE) && hot_ext(h2) == rid[m] && q[m] == b2 + s2) {
@@ -458,6 +489,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
               j[m] -= 1;
               key[m] = b2;
               hw[m] = h2;
+              rw[m] = reinterpret_cast<const uint64_t *>(&r2)[1];
             }
           }
         }
@@ -469,8 +501,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         if (sh[m]) {
           hit[m] = true;
           j[m] = jsh[m];
-          q[m] = hsh[m];
-          hw[m] = hwsh[m];
+          q[m] = hsh[m];  // hw, rw: gathered by the shadow check
         }
     }
     // forward map: record the shadow of every slot (CPU pointer, unit) for the reverse pass
@@ -483,15 +514,13 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         reinterpret_cast<uint32_t *>(sg.shadow + 8 * sg.n)[i] = hit[m] ? (uint32_t)j[m] : 0xFFFFFFFFu;
       }
     }
-    // epoch (gate) and refcount (unmap check) columns, only where the operation needs them
-    uint32_t ep[2] = {0, 0};
-    int32_t rcv[2] = {0, 0};
+    // epoch (gate) and refcount (unmap check): from the record gathered with the hot word
+    uint32_t ep[2];
+    int32_t rcv[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      // read-only units under a snapshot: the gate can only set the epoch (no copy, nothing to journal)
-      if ((OPS & OP_GATE) && hit[m] && !(a.no_journal && (hot_flags(hw[m]) & UF_READONLY)))
-        ep[m] = a.tab.epoch[j[m]];
-      if ((OPS & OP_CHECKMAPPED) && hit[m]) rcv[m] = a.tab.rc[j[m]];
+      rcv[m] = (int32_t)(uint32_t)rw[m];
+      ep[m] = (uint32_t)(rw[m] >> 32);
     }
 
     // ---- a2/a3/a4 operations ----
@@ -506,7 +535,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
       c_hits += hm;
       c_miss += (vm && !nul && !hm);
       const int unit = hm ? j[m] : 0;
-      int32_t *RC = a.tab.rc + unit;
+      int32_t *RC = &a.tab.rec[unit].rc;
       const uint32_t fl = hot_flags(hw[m]);
       if (OPS & OP_CHECKMAPPED) c_notm += (hm && rcv[m] <= 0);
       bool act = false;
@@ -540,9 +569,10 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
       uint32_t old_ep = 0;
       if (OPS & OP_GATE) {
         if (hm && a.no_journal && (fl & UF_READONLY)) {
-          a.tab.epoch[unit] = a.epoch;  // Alg. 2 line 3 for a read-only unit: epoch <- globalEpoch
+          // Alg. 2 line 3 for a read-only unit: epoch <- globalEpoch (skipped when already current)
+          if (ep[m] != a.epoch) a.tab.rec[unit].epoch = a.epoch;
         } else if (hm && ep[m] != a.epoch) {
-          old_ep = atomicExch(a.tab.epoch + unit, a.epoch);
+          old_ep = atomicExch(&a.tab.rec[unit].epoch, a.epoch);
           gated = (old_ep != a.epoch);
         }
       }
@@ -756,13 +786,13 @@ __global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *size, con
   if (i >= n) return;
   int k = old_idx[i];
   if (k >= 0) {
-    t.hot[i] = o.hot[k];
-    t.rc[i] = o.rc[k];
-    t.epoch[i] = o.epoch[k];
+    t.rec[i] = o.rec[k];
   } else {
-    t.hot[i] = make_hot(size[i], NO_EXT, flags[i]);
-    t.rc[i] = 0;
-    t.epoch[i] = epoch0[i];
+    UnitRec r;
+    r.hot = make_hot(size[i], NO_EXT, flags[i]);
+    r.rc = 0;
+    r.epoch = epoch0[i];
+    t.rec[i] = r;
   }
 }
 void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags, const uint32_t *epoch0,
@@ -794,13 +824,13 @@ __global__ void k_unit_ops(const UnitOp *ops, int n, TableDev tab) {
   if (i >= n) return;
   UnitOp o = ops[i];
   switch (o.op) {
-    case UOP_ADD_RC: atomicAdd(tab.rc + o.unit, (int32_t)(int64_t)o.val); break;
-    case UOP_SET_EPOCH: tab.epoch[o.unit] = (uint32_t)o.val; break;
-    case UOP_OR_FLAGS: atomicOr(flag_word(tab.hot + o.unit), (uint32_t)o.val << (FSHIFT - 32)); break;
+    case UOP_ADD_RC: atomicAdd(&tab.rec[o.unit].rc, (int32_t)(int64_t)o.val); break;
+    case UOP_SET_EPOCH: tab.rec[o.unit].epoch = (uint32_t)o.val; break;
+    case UOP_OR_FLAGS: atomicOr(flag_word(&tab.rec[o.unit].hot), (uint32_t)o.val << (FSHIFT - 32)); break;
     case UOP_AND_FLAGS:
-      atomicAnd(flag_word(tab.hot + o.unit), ((uint32_t)o.val << (FSHIFT - 32)) | ((1u << (FSHIFT - 32)) - 1));
+      atomicAnd(flag_word(&tab.rec[o.unit].hot), ((uint32_t)o.val << (FSHIFT - 32)) | ((1u << (FSHIFT - 32)) - 1));
       break;
-    case UOP_SET_RC: tab.rc[o.unit] = (int32_t)(int64_t)o.val; break;
+    case UOP_SET_RC: tab.rec[o.unit].rc = (int32_t)(int64_t)o.val; break;
   }
 }
 void launch_unit_ops(const UnitOp *ops, int n, TableDev tab, cudaStream_t s) {
@@ -816,11 +846,11 @@ __global__ void k_set_ext(const uint32_t *units, const uint32_t *exts, int n, Ta
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const uint32_t u = units[i];
-  uint64_t h = tab.hot[u];
+  uint64_t h = tab.rec[u].hot;
   h = (h & ~(EXT_MASK << ESHIFT)) | ((uint64_t)(exts[i] & EXT_MASK) << ESHIFT);
   h |= (uint64_t)(UF_STORAGE | UF_ACTIVE) << FSHIFT;
-  tab.hot[u] = h;
-  if (set_epoch) tab.epoch[u] = epoch;
+  tab.rec[u].hot = h;
+  if (set_epoch) tab.rec[u].epoch = epoch;
 }
 void launch_set_ext(const uint32_t *units, const uint32_t *exts, int n, TableDev tab, uint32_t epoch, int set_epoch,
                     cudaStream_t s) {
@@ -834,15 +864,15 @@ __global__ void k_deactivate(const uint32_t *units, int n, TableDev tab) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const uint32_t u = units[i];
-  if (tab.rc[u] != 0) return;
-  uint64_t h = tab.hot[u];
+  if (tab.rec[u].rc != 0) return;
+  uint64_t h = tab.rec[u].hot;
   if (hot_flags(h) & UF_GLOBAL) {
     h &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE) << FSHIFT);  // named region persists
   } else {
     h &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE | UF_STORAGE) << FSHIFT);  // cuMemFree (Alg. 3)
     h |= NO_EXT << ESHIFT;
   }
-  tab.hot[u] = h;
+  tab.rec[u].hot = h;
 }
 void launch_deactivate(const uint32_t *units, int n, TableDev tab, cudaStream_t s) {
   if (n > 0) {
@@ -854,7 +884,7 @@ void launch_deactivate(const uint32_t *units, int n, TableDev tab, cudaStream_t 
 __global__ void k_restore_epochs(const Journal *j, int n, TableDev tab) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  tab.epoch[j[i].unit] = j[i].old_epoch;
+  tab.rec[j[i].unit].epoch = j[i].old_epoch;
 }
 void launch_restore_epochs(const Journal *j, int n, TableDev tab, cudaStream_t s) {
   if (n > 0) {
@@ -871,9 +901,9 @@ __global__ void k_release_scan(TableDev tab, int n, Status *st, unsigned long lo
     int i = base + threadIdx.x;
     bool fr = false;
     if (i < n) {
-      int32_t rc = tab.rc[i];
+      int32_t rc = tab.rec[i].rc;
       under += rc < 0;
-      fr = rc == 0 && (hot_flags(tab.hot[i]) & UF_ACTIVE);
+      fr = rc == 0 && (hot_flags(tab.rec[i].hot) & UF_ACTIVE);
     }
     unsigned long long ix = warp_append(&lc[2], fr);
     if (fr) free_list[ix] = (uint32_t)i;
@@ -892,7 +922,7 @@ void launch_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc
 // epoch origin moves (once per 2^32 - 16 launches): the current epoch becomes 1, every other 0
 __global__ void k_rebase_epochs(TableDev tab, int n, uint32_t cur) {
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-    tab.epoch[i] = tab.epoch[i] == cur ? 1u : 0u;
+    tab.rec[i].epoch = tab.rec[i].epoch == cur ? 1u : 0u;
 }
 void launch_rebase_epochs(TableDev tab, int n, uint32_t cur, cudaStream_t s) {
   if (n > 0) {
@@ -921,15 +951,15 @@ __global__ void k_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs,
       if (ix.keys[lo + half] <= p) lo += half;
       len -= half;
     }
-    const uint64_t h = tab.hot[lo], b = ix.keys[lo], sz = tab.size64[lo];
+    const uint64_t h = tab.rec[lo].hot, b = ix.keys[lo], sz = tab.size64[lo];
     if (p - b <= sz) {
       r.unit = lo;
       r.base = b;
       r.size = sz;
       r.flags = hot_flags(h);
       r.devbase = (r.flags & UF_STORAGE) ? b + tab.ext_delta[hot_ext(h)] : 0;
-      r.epoch = tab.epoch[lo];
-      r.refcount = tab.rc[lo];
+      r.epoch = tab.rec[lo].epoch;
+      r.refcount = tab.rec[lo].rc;
     }
   }
   out[i] = r;

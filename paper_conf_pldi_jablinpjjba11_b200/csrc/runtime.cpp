@@ -208,7 +208,7 @@ struct Context {
   int U = 0;  // units in the device table
 
   // device table
-  DevBuf hot, rcb, epb, size64, dbase, extd, snap_rc, snap_ep;  // unit table columns + extent deltas
+  DevBuf recb, size64, dbase, extd, snap_rec;  // unit records (UnitRec), cold columns, extent deltas
   size_t extd_n = 0;                          // entries uploaded to extd
   IndexBufs fwd, rev;
 
@@ -254,9 +254,7 @@ struct Context {
   }
   TableDev tab() const {
     TableDev t;
-    t.hot = hot.as<uint64_t>();
-    t.rc = rcb.as<int32_t>();
-    t.epoch = epb.as<uint32_t>();
+    t.rec = recb.as<UnitRec>();
     t.base = dbase.as<uint64_t>();
     t.size64 = size64.as<uint64_t>();
     t.ext_delta = extd.as<uint64_t>();
@@ -423,11 +421,9 @@ struct Context {
     udev.swap(ndev);
     urun.swap(nrun);
     uarr.swap(narr);
-    DevBuf nhot, nrc, nep, nsize, nbase, tmp;
+    DevBuf nrec, nsize, nbase, tmp;
     int cap = std::max(n, 1);
-    CKS(dalloc(nhot, 8 * (size_t)cap));
-    CKS(dalloc(nrc, 4 * (size_t)cap + 64));
-    CKS(dalloc(nep, 4 * (size_t)cap + 64));
+    CKS(dalloc(nrec, sizeof(UnitRec) * (size_t)cap + 64));
     CKS(dalloc(nsize, 8 * (size_t)cap));
     CKS(dalloc(nbase, 8 * (size_t)cap));
     CKS(dalloc(tmp, (size_t)cap * 24 + 256));
@@ -439,23 +435,17 @@ struct Context {
       const int32_t *dold = reinterpret_cast<const int32_t *>(depoch + n);
       const uint32_t *dflags = reinterpret_cast<const uint32_t *>(dold + n);
       TableDev nt = tab();
-      nt.hot = nhot.as<uint64_t>();
-      nt.rc = nrc.as<int32_t>();
-      nt.epoch = nep.as<uint32_t>();
+      nt.rec = nrec.as<UnitRec>();
       launch_remap(n, dold, nsize.as<uint64_t>(), dflags, depoch, tab(), nt, main);
       st.kernel_launches += 1;
       CK(cudaGetLastError());
       CK(cudaStreamSynchronize(main));
     }
     dfree(tmp);
-    dfree(hot);
-    dfree(rcb);
-    dfree(epb);
+    dfree(recb);
     dfree(size64);
     dfree(dbase);
-    hot = nhot;
-    rcb = nrc;
-    epb = nep;
+    recb = nrec;
     size64 = nsize;
     dbase = nbase;
     U = n;
@@ -1117,15 +1107,15 @@ struct Context {
   std::map<std::pair<uint64_t, uint64_t>, Shadow> shadows;
   uint64_t table_gen = 0;
   int take_snapshot() {
-    CKS(dalloc(snap_rc, 4 * (size_t)U + 64));
-    CKS(dalloc(snap_ep, 4 * (size_t)U + 64));
-    CK(cudaMemcpyAsync(snap_rc.as<void>(), rcb.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
-    CK(cudaMemcpyAsync(snap_ep.as<void>(), epb.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
+    CKS(dalloc(snap_rec, sizeof(UnitRec) * (size_t)U + 64));
+    CK(cudaMemcpyAsync(snap_rec.as<void>(), recb.as<void>(), sizeof(UnitRec) * (size_t)U, cudaMemcpyDeviceToDevice,
+                       main));
     return CGCM_OK;
   }
   int restore_snapshot() {
-    CK(cudaMemcpyAsync(rcb.as<void>(), snap_rc.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
-    CK(cudaMemcpyAsync(epb.as<void>(), snap_ep.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
+    // the pass does not touch hot words: restoring whole records restores refcounts and epochs
+    CK(cudaMemcpyAsync(recb.as<void>(), snap_rec.as<void>(), sizeof(UnitRec) * (size_t)U, cudaMemcpyDeviceToDevice,
+                       main));
     CK(cudaStreamSynchronize(main));
     return CGCM_OK;
   }
@@ -1372,7 +1362,7 @@ int cgcm_undeclare(void *base) {
   HostUnit &u = it->second;
   if (u.idx >= 0) {  // idx refers to the current device table until the next ensure_table()
     int32_t rc = 0;
-    CK(cudaMemcpyAsync(&rc, C->rcb.as<int32_t>() + u.idx, 4, cudaMemcpyDeviceToHost, C->main));
+    CK(cudaMemcpyAsync(&rc, &C->recb.as<UnitRec>()[u.idx].rc, 4, cudaMemcpyDeviceToHost, C->main));
     CK(cudaStreamSynchronize(C->main));
     if (rc > 0) return CGCM_E_BUSY;
   }
@@ -1474,7 +1464,7 @@ void *cgcm_realloc(void *p, size_t n) {
   auto ru = C->reg.find(a);
   if (ru != C->reg.end() && ru->second.idx >= 0) {  // a mapped AU cannot move (BUSY)
     int32_t rc = 0;
-    if (cudaMemcpy(&rc, C->rcb.as<int32_t>() + ru->second.idx, 4, cudaMemcpyDeviceToHost) != cudaSuccess || rc > 0)
+    if (cudaMemcpy(&rc, &C->recb.as<UnitRec>()[ru->second.idx].rc, 4, cudaMemcpyDeviceToHost) != cudaSuccess || rc > 0)
       return nullptr;
   }
   size_t old = it->second;
@@ -1512,7 +1502,7 @@ int cgcm_scopeExit(void) {
     auto ru = C->reg.find(a);
     if (ru == C->reg.end() || ru->second.idx < 0) continue;
     int32_t rc = 0;
-    CK(cudaMemcpy(&rc, C->rcb.as<int32_t>() + ru->second.idx, 4, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&rc, &C->recb.as<UnitRec>()[ru->second.idx].rc, 4, cudaMemcpyDeviceToHost));
     if (rc > 0) return CGCM_E_BUSY;
   }
   for (auto it = sc.rbegin(); it != sc.rend(); ++it) CKS(cgcm_free(reinterpret_cast<void *>(*it)));
@@ -2046,26 +2036,23 @@ int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
   CKS(C->ensure_table());
   if (n) *n = (size_t)C->U;
   if (!out || cap == 0) return (size_t)C->U <= cap ? CGCM_OK : CGCM_E_NOMEM;
-  std::vector<uint64_t> hots, szs;
-  std::vector<uint32_t> eps;
-  std::vector<int32_t> rcs;
-  CKS(C->download(hots, C->hot, (size_t)C->U));
-  CKS(C->download(eps, C->epb, (size_t)C->U));
+  std::vector<UnitRec> recs;
+  std::vector<uint64_t> szs;
+  CKS(C->download(recs, C->recb, (size_t)C->U));
   CKS(C->download(szs, C->size64, (size_t)C->U));
-  CKS(C->download(rcs, C->rcb, (size_t)C->U));
   size_t m = std::min(cap, (size_t)C->U);
   for (size_t i = 0; i < m; ++i) {
     cgcm_unit_t &u = out[i];
-    const uint32_t fl = hot_flags(hots[i]);
+    const uint32_t fl = hot_flags(recs[i].hot);
     u.base = C->ubase[i];
     u.size = szs[i];
-    bool act = rcs[i] > 0;
-    uint32_t e = hot_ext(hots[i]);
+    bool act = recs[i].rc > 0;
+    uint32_t e = hot_ext(recs[i].hot);
     u.devptr = ((fl & UF_STORAGE) && (act || (fl & UF_GLOBAL)) && e < C->runs.size())
                    ? u.base - C->runs[e].delta
                    : 0;
-    u.refCount = rcs[i];
-    u.epoch = C->origin + eps[i];
+    u.refCount = recs[i].rc;
+    u.epoch = C->origin + recs[i].epoch;
     u.flags = ((fl & UF_GLOBAL) ? CGCM_UNIT_GLOBAL : 0) | ((fl & UF_READONLY) ? CGCM_UNIT_READONLY : 0) |
               ((fl & UF_ARRAYMAPPED) ? CGCM_UNIT_ARRAYMAPPED : 0) | (act ? CGCM_UNIT_ACTIVE : 0);
     u.pad = 0;

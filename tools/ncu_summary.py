@@ -105,7 +105,8 @@ def main():
             if len(r) <= vi or r[mi] != "gpu__time_duration.sum":
                 continue
             v = float(r[vi].replace(",", ""))
-            v *= {"nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0, "second": 1e3}.get(r[ui], 1.0)
+            v *= {"nsecond": 1e-6, "ns": 1e-6, "usecond": 1e-3, "us": 1e-3, "msecond": 1.0, "ms": 1.0,
+                  "second": 1e3, "s": 1e3}.get(r[ui], 1.0)
             key = r[ki].split("(")[0]
             times[key] += v
             counts[key] += 1
@@ -114,6 +115,14 @@ def main():
                   "| kernel | launches | total ms | share |", "|---|---|---|---|"]
         for k, v in times.most_common(15):
             lines.append(f"| `{k[:90]}` | {counts[k]} | {v:.3f} | {100 * v / total:.1f}% |")
+        lines.append("")
+        # this library's kernels only (the bench's input generation runs torch kernels outside the timed region)
+        own = {k: v for k, v in times.items() if "cgcm::" in k}
+        tot_own = sum(own.values()) or 1.0
+        lines += ["### this library's kernels only (cgcm::*)", "",
+                  "| kernel | launches | total ms | share of cgcm time |", "|---|---|---|---|"]
+        for k, v in sorted(own.items(), key=lambda x: -x[1]):
+            lines.append(f"| `{k[:90]}` | {counts[k]} | {v:.3f} | {100 * v / tot_own:.1f}% |")
         lines.append("")
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     out = os.path.join(ROOT, "profiles", f"{args.round}_{args.config}_summary.md")
