@@ -7,23 +7,23 @@
 
 namespace cgcm {
 
-// The allocation-unit table (D3), indexed by the unit's rank in base order.  The
-// per-unit words a slot touches live in ONE 16-byte record, so a lookup's record gather brings the
-// refcount and epoch into L2 with the hot word (one sector per unit; the refcount reduction and the
-// epoch gate that follow hit the line the gather just fetched):
-//   rec[u].hot   = size (bits 0..31; 0xFFFFFFFF = see size64) | extent id (bits 32..55) | flags (56..63)
-//   rec[u].rc    = refCount (i32, Alg. 1/3)
-//   rec[u].epoch = Alg. 2's per-unit epoch, u32 relative to the context's epoch origin (A28)
+// The allocation-unit table (D3), indexed by the unit's rank in base order.  Each
+// pass gathers ONE 8-byte word per slot and sends one reduction to a separate array (a reduction to
+// the line a gather has just fetched is serialised behind it in L2 -- tools/l2_gather.cu,
+// skeleton_rev: 5.37 ms with the refcount beside the gathered word vs 3.37 ms in its own array):
+//   hot[u] = size (bits 0..31; 0xFFFFFFFF = see size64) | extent id (bits 32..55) | flags (56..63)
+//            -- what a forward lookup needs
+//   st[u]  = epoch (bits 0..31; Alg. 2's per-unit epoch, u32 relative to the context's epoch origin,
+//            A28) | a mirror of hot's bits 32..63 (extent id, flags) -- what a reverse pass over
+//            recorded slots needs (8 B instead of 16 B per unit keeps the working set L2-sized)
+//   rc[u]  = refCount (i32, Alg. 1/3)
 //   base[u]  = the sorted key array of the forward index; size64[u] = full size (cold)
 //   ext_delta[e] = devbase - base for every unit copy in device extent e (mirrored layout):
 //              translation = p + ext_delta[extent(u)]  (Alg. 1: devptr + (ptr - base))
-struct __align__(16) UnitRec {
-  uint64_t hot;
-  int32_t rc;
-  uint32_t epoch;
-};
 struct TableDev {
-  UnitRec *rec;
+  uint64_t *hot;
+  uint64_t *st;
+  int32_t *rc;
   const uint64_t *base;
   const uint64_t *size64;
   const uint64_t *ext_delta;
@@ -46,6 +46,13 @@ constexpr uint64_t ADDR_LIMIT = (1ull << 57) - 1;  // base + size must stay belo
 __host__ __device__ __forceinline__ uint32_t hot_size32(uint64_t h) { return (uint32_t)h; }
 __host__ __device__ __forceinline__ uint32_t hot_ext(uint64_t h) { return (uint32_t)((h >> ESHIFT) & EXT_MASK); }
 __host__ __device__ __forceinline__ uint32_t hot_flags(uint64_t h) { return (uint32_t)(h >> FSHIFT); }
+__host__ __device__ __forceinline__ uint32_t st_epoch(uint64_t st) { return (uint32_t)st; }
+__host__ __device__ __forceinline__ uint64_t make_st(uint64_t hot, uint32_t epoch) {
+  return (hot & 0xFFFFFFFF00000000ull) | epoch;
+}
+// the 32-bit halves of a table word (little endian): [0] = size / epoch, [1] = extent | flags
+__device__ __forceinline__ uint32_t *lo_word(uint64_t *w) { return reinterpret_cast<uint32_t *>(w); }
+__device__ __forceinline__ uint32_t *hi_word(uint64_t *w) { return reinterpret_cast<uint32_t *>(w) + 1; }
 __host__ __device__ __forceinline__ uint64_t make_hot(uint64_t size, uint64_t ext, uint32_t flags) {
   return (size >= BIG_SIZE ? (uint64_t)BIG_SIZE : size) | ((ext & EXT_MASK) << ESHIFT) | ((uint64_t)flags << FSHIFT);
 }

@@ -55,6 +55,11 @@ __device__ __forceinline__ void ld_sector(const void *p, uint64_t pol, uint64_t 
 __device__ __forceinline__ void ld_pair(const void *p, uint64_t pol, uint64_t &a, uint64_t &b) {
   asm volatile("ld.global.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;" : "=l"(a), "=l"(b) : "l"(p), "l"(pol));
 }
+__device__ __forceinline__ uint64_t ld_u64(const uint64_t *p, uint64_t pol) {
+  uint64_t v;
+  asm volatile("ld.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+  return v;
+}
 __device__ __forceinline__ void red_add(int32_t *p, int32_t v) {
   asm volatile("red.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -403,7 +408,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
     bool sh[2] = {false, false};
     int jsh[2] = {0, 0};
     uint64_t hsh[2] = {0, 0};
-    // the unit's record: hot word (size | extent | flags), then refcount | epoch << 32
+    // the unit's hot word (size | extent | flags) and state word (epoch | extent | flags)
     uint64_t hw[2] = {0, 0}, rw[2] = {0, 0};
     const int64_t slot0 = ((int64_t)(a0 - sg.ptr)) >> 3;  // slot index of m = 0 (-1 for a head chunk)
     if (SH && DIR == DIR_REV && sg.shadow) {
@@ -414,16 +419,15 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         const uint32_t u = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n)[i];
         if (u == 0xFFFFFFFFu) continue;
         const uint64_t h = reinterpret_cast<const uint64_t *>(sg.shadow)[i];
-        uint64_t w, r;
-        ld_pair(a.tab.rec + u, pol_t, w, r);
+        const uint64_t w = ld_u64(a.tab.st + u, pol_t);  // extent, flags and epoch in one word
         const uint32_t e = hot_ext(w);
         if ((hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext &&
             q[m] == h + (ext_s ? s_ext[e] : a.tab.ext_delta[e])) {
           sh[m] = true;
           jsh[m] = (int)u;
           hsh[m] = h;
-          hw[m] = w;
-          rw[m] = r;
+          hw[m] = w;  // the size bits are not used on this path
+          rw[m] = w;
           look[m] = false;
         }
       }
@@ -462,11 +466,12 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
     if constexpr (FH > 0) level_lookup2_fixed<FH>(a.fx, pol_t, q, j, key);
     else if constexpr (FH < 0) level_lookup2(F, a.fx, pol_t, q, j, key);
 
-    // ---- the unit's record: hot word (size | extent | flags), refcount, epoch: one 16-B gather ----
+    // ---- the unit's hot word (size | extent | flags), and its state word where the epoch is needed ----
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
       look[m] = look[m] && j[m] >= 0;
-      if (look[m]) ld_pair(a.tab.rec + j[m], pol_t, hw[m], rw[m]);
+      if (look[m]) hw[m] = ld_u64(a.tab.hot + j[m], pol_t);
+      if ((OPS & OP_GATE) && look[m]) rw[m] = ld_u64(a.tab.st + j[m], pol_t);
     }
     }  // full lookups
     bool hit[2];
@@ -480,8 +485,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         if (!(hit[m] && (hot_flags(hw[m]) & UF_ACTIVE) && hot_ext(hw[m]) == rid[m])) {
           hit[m] = false;
           if (j[m] > 0 && q[m] == key[m]) {  // one past the end of the previous unit (A7)
-            const UnitRec r2 = a.tab.rec[j[m] - 1];
-            const uint64_t h2 = r2.hot, b2 = a.tab.base[j[m] - 1];
+            const uint64_t h2 = a.tab.hot[j[m] - 1], b2 = a.tab.base[j[m] - 1];
             uint64_t s2 = hot_size32(h2);
             if (s2 == BIG_SIZE) s2 = a.tab.size64[j[m] - 1];
             if ((hot_flags(h2) & UF_ACTIVE) && hot_ext(h2) == rid[m] && q[m] == b2 + s2) {
@@ -489,7 +493,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
               j[m] -= 1;
               key[m] = b2;
               hw[m] = h2;
-              rw[m] = reinterpret_cast<const uint64_t *>(&r2)[1];
+              rw[m] = a.tab.st[j[m]];
             }
           }
         }
@@ -514,13 +518,13 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         reinterpret_cast<uint32_t *>(sg.shadow + 8 * sg.n)[i] = hit[m] ? (uint32_t)j[m] : 0xFFFFFFFFu;
       }
     }
-    // epoch (gate) and refcount (unmap check): from the record gathered with the hot word
+    // epoch (gate): from the record gathered with the hot word; refcount (unmap check) where needed
     uint32_t ep[2];
-    int32_t rcv[2];
+    int32_t rcv[2] = {0, 0};
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      rcv[m] = (int32_t)(uint32_t)rw[m];
-      ep[m] = (uint32_t)(rw[m] >> 32);
+      ep[m] = st_epoch(rw[m]);
+      if ((OPS & OP_CHECKMAPPED) && hit[m]) rcv[m] = a.tab.rc[j[m]];
     }
 
     // ---- a2/a3/a4 operations ----
@@ -535,7 +539,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
       c_hits += hm;
       c_miss += (vm && !nul && !hm);
       const int unit = hm ? j[m] : 0;
-      int32_t *RC = &a.tab.rec[unit].rc;
+      int32_t *RC = a.tab.rc + unit;
       const uint32_t fl = hot_flags(hw[m]);
       if (OPS & OP_CHECKMAPPED) c_notm += (hm && rcv[m] <= 0);
       bool act = false;
@@ -570,9 +574,9 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
       if (OPS & OP_GATE) {
         if (hm && a.no_journal && (fl & UF_READONLY)) {
           // Alg. 2 line 3 for a read-only unit: epoch <- globalEpoch (skipped when already current)
-          if (ep[m] != a.epoch) a.tab.rec[unit].epoch = a.epoch;
+          if (ep[m] != a.epoch) *lo_word(a.tab.st + unit) = a.epoch;
         } else if (hm && ep[m] != a.epoch) {
-          old_ep = atomicExch(&a.tab.rec[unit].epoch, a.epoch);
+          old_ep = atomicExch(lo_word(a.tab.st + unit), a.epoch);
           gated = (old_ep != a.epoch);
         }
       }
@@ -786,13 +790,14 @@ __global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *size, con
   if (i >= n) return;
   int k = old_idx[i];
   if (k >= 0) {
-    t.rec[i] = o.rec[k];
+    t.hot[i] = o.hot[k];
+    t.st[i] = o.st[k];
+    t.rc[i] = o.rc[k];
   } else {
-    UnitRec r;
-    r.hot = make_hot(size[i], NO_EXT, flags[i]);
-    r.rc = 0;
-    r.epoch = epoch0[i];
-    t.rec[i] = r;
+    const uint64_t h = make_hot(size[i], NO_EXT, flags[i]);
+    t.hot[i] = h;
+    t.st[i] = make_st(h, epoch0[i]);
+    t.rc[i] = 0;
   }
 }
 void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags, const uint32_t *epoch0,
@@ -815,22 +820,22 @@ void launch_sort_keys(void *temp, size_t temp_bytes, const uint32_t *kin, uint32
 // -------------------------------------------------------------------------------------------------
 // small bookkeeping kernels
 // -------------------------------------------------------------------------------------------------
-__device__ __forceinline__ unsigned *flag_word(uint64_t *hot) {
-  return reinterpret_cast<unsigned *>(hot) + 1;  // flags (and the extent id) live in the high word
-}
-
 __global__ void k_unit_ops(const UnitOp *ops, int n, TableDev tab) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   UnitOp o = ops[i];
   switch (o.op) {
-    case UOP_ADD_RC: atomicAdd(&tab.rec[o.unit].rc, (int32_t)(int64_t)o.val); break;
-    case UOP_SET_EPOCH: tab.rec[o.unit].epoch = (uint32_t)o.val; break;
-    case UOP_OR_FLAGS: atomicOr(flag_word(&tab.rec[o.unit].hot), (uint32_t)o.val << (FSHIFT - 32)); break;
-    case UOP_AND_FLAGS:
-      atomicAnd(flag_word(&tab.rec[o.unit].hot), ((uint32_t)o.val << (FSHIFT - 32)) | ((1u << (FSHIFT - 32)) - 1));
+    case UOP_ADD_RC: atomicAdd(tab.rc + o.unit, (int32_t)(int64_t)o.val); break;
+    case UOP_SET_EPOCH: *lo_word(tab.st + o.unit) = (uint32_t)o.val; break;
+    case UOP_OR_FLAGS:
+      atomicOr(hi_word(tab.hot + o.unit), (uint32_t)o.val << (FSHIFT - 32));
+      atomicOr(hi_word(tab.st + o.unit), (uint32_t)o.val << (FSHIFT - 32));
       break;
-    case UOP_SET_RC: tab.rec[o.unit].rc = (int32_t)(int64_t)o.val; break;
+    case UOP_AND_FLAGS:
+      atomicAnd(hi_word(tab.hot + o.unit), ((uint32_t)o.val << (FSHIFT - 32)) | ((1u << (FSHIFT - 32)) - 1));
+      atomicAnd(hi_word(tab.st + o.unit), ((uint32_t)o.val << (FSHIFT - 32)) | ((1u << (FSHIFT - 32)) - 1));
+      break;
+    case UOP_SET_RC: tab.rc[o.unit] = (int32_t)(int64_t)o.val; break;
   }
 }
 void launch_unit_ops(const UnitOp *ops, int n, TableDev tab, cudaStream_t s) {
@@ -846,11 +851,11 @@ __global__ void k_set_ext(const uint32_t *units, const uint32_t *exts, int n, Ta
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const uint32_t u = units[i];
-  uint64_t h = tab.rec[u].hot;
+  uint64_t h = tab.hot[u];
   h = (h & ~(EXT_MASK << ESHIFT)) | ((uint64_t)(exts[i] & EXT_MASK) << ESHIFT);
   h |= (uint64_t)(UF_STORAGE | UF_ACTIVE) << FSHIFT;
-  tab.rec[u].hot = h;
-  if (set_epoch) tab.rec[u].epoch = epoch;
+  tab.hot[u] = h;
+  tab.st[u] = make_st(h, set_epoch ? epoch : st_epoch(tab.st[u]));
 }
 void launch_set_ext(const uint32_t *units, const uint32_t *exts, int n, TableDev tab, uint32_t epoch, int set_epoch,
                     cudaStream_t s) {
@@ -864,15 +869,16 @@ __global__ void k_deactivate(const uint32_t *units, int n, TableDev tab) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const uint32_t u = units[i];
-  if (tab.rec[u].rc != 0) return;
-  uint64_t h = tab.rec[u].hot;
+  if (tab.rc[u] != 0) return;
+  uint64_t h = tab.hot[u];
   if (hot_flags(h) & UF_GLOBAL) {
     h &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE) << FSHIFT);  // named region persists
   } else {
     h &= ~((uint64_t)(UF_ARRAYMAPPED | UF_ACTIVE | UF_STORAGE) << FSHIFT);  // cuMemFree (Alg. 3)
     h |= NO_EXT << ESHIFT;
   }
-  tab.rec[u].hot = h;
+  tab.hot[u] = h;
+  tab.st[u] = make_st(h, st_epoch(tab.st[u]));
 }
 void launch_deactivate(const uint32_t *units, int n, TableDev tab, cudaStream_t s) {
   if (n > 0) {
@@ -884,7 +890,7 @@ void launch_deactivate(const uint32_t *units, int n, TableDev tab, cudaStream_t 
 __global__ void k_restore_epochs(const Journal *j, int n, TableDev tab) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  tab.rec[j[i].unit].epoch = j[i].old_epoch;
+  *lo_word(tab.st + j[i].unit) = j[i].old_epoch;
 }
 void launch_restore_epochs(const Journal *j, int n, TableDev tab, cudaStream_t s) {
   if (n > 0) {
@@ -901,9 +907,9 @@ __global__ void k_release_scan(TableDev tab, int n, Status *st, unsigned long lo
     int i = base + threadIdx.x;
     bool fr = false;
     if (i < n) {
-      int32_t rc = tab.rec[i].rc;
+      int32_t rc = tab.rc[i];
       under += rc < 0;
-      fr = rc == 0 && (hot_flags(tab.rec[i].hot) & UF_ACTIVE);
+      fr = rc == 0 && (hot_flags(tab.hot[i]) & UF_ACTIVE);
     }
     unsigned long long ix = warp_append(&lc[2], fr);
     if (fr) free_list[ix] = (uint32_t)i;
@@ -922,7 +928,7 @@ void launch_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc
 // epoch origin moves (once per 2^32 - 16 launches): the current epoch becomes 1, every other 0
 __global__ void k_rebase_epochs(TableDev tab, int n, uint32_t cur) {
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-    tab.rec[i].epoch = tab.rec[i].epoch == cur ? 1u : 0u;
+    *lo_word(tab.st + i) = st_epoch(tab.st[i]) == cur ? 1u : 0u;
 }
 void launch_rebase_epochs(TableDev tab, int n, uint32_t cur, cudaStream_t s) {
   if (n > 0) {
@@ -951,15 +957,15 @@ __global__ void k_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs,
       if (ix.keys[lo + half] <= p) lo += half;
       len -= half;
     }
-    const uint64_t h = tab.rec[lo].hot, b = ix.keys[lo], sz = tab.size64[lo];
+    const uint64_t h = tab.hot[lo], b = ix.keys[lo], sz = tab.size64[lo];
     if (p - b <= sz) {
       r.unit = lo;
       r.base = b;
       r.size = sz;
       r.flags = hot_flags(h);
       r.devbase = (r.flags & UF_STORAGE) ? b + tab.ext_delta[hot_ext(h)] : 0;
-      r.epoch = tab.rec[lo].epoch;
-      r.refcount = tab.rec[lo].rc;
+      r.epoch = st_epoch(tab.st[lo]);
+      r.refcount = tab.rc[lo];
     }
   }
   out[i] = r;

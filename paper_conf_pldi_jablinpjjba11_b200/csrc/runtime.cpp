@@ -10,6 +10,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <map>
@@ -208,7 +209,7 @@ struct Context {
   int U = 0;  // units in the device table
 
   // device table
-  DevBuf recb, size64, dbase, extd, snap_rec;  // unit records (UnitRec), cold columns, extent deltas
+  DevBuf hotb, stb, rcb, size64, dbase, extd, snap_st, snap_rc;  // unit table columns + extent deltas
   size_t extd_n = 0;                          // entries uploaded to extd
   IndexBufs fwd, rev;
 
@@ -254,7 +255,9 @@ struct Context {
   }
   TableDev tab() const {
     TableDev t;
-    t.rec = recb.as<UnitRec>();
+    t.hot = hotb.as<uint64_t>();
+    t.st = stb.as<uint64_t>();
+    t.rc = rcb.as<int32_t>();
     t.base = dbase.as<uint64_t>();
     t.size64 = size64.as<uint64_t>();
     t.ext_delta = extd.as<uint64_t>();
@@ -421,9 +424,11 @@ struct Context {
     udev.swap(ndev);
     urun.swap(nrun);
     uarr.swap(narr);
-    DevBuf nrec, nsize, nbase, tmp;
+    DevBuf nhot, nst, nrc, nsize, nbase, tmp;
     int cap = std::max(n, 1);
-    CKS(dalloc(nrec, sizeof(UnitRec) * (size_t)cap + 64));
+    CKS(dalloc(nhot, 8 * (size_t)cap + 64));
+    CKS(dalloc(nst, 8 * (size_t)cap + 64));
+    CKS(dalloc(nrc, 4 * (size_t)cap + 64));
     CKS(dalloc(nsize, 8 * (size_t)cap));
     CKS(dalloc(nbase, 8 * (size_t)cap));
     CKS(dalloc(tmp, (size_t)cap * 24 + 256));
@@ -435,17 +440,23 @@ struct Context {
       const int32_t *dold = reinterpret_cast<const int32_t *>(depoch + n);
       const uint32_t *dflags = reinterpret_cast<const uint32_t *>(dold + n);
       TableDev nt = tab();
-      nt.rec = nrec.as<UnitRec>();
+      nt.hot = nhot.as<uint64_t>();
+      nt.st = nst.as<uint64_t>();
+      nt.rc = nrc.as<int32_t>();
       launch_remap(n, dold, nsize.as<uint64_t>(), dflags, depoch, tab(), nt, main);
       st.kernel_launches += 1;
       CK(cudaGetLastError());
       CK(cudaStreamSynchronize(main));
     }
     dfree(tmp);
-    dfree(recb);
+    dfree(hotb);
+    dfree(stb);
+    dfree(rcb);
     dfree(size64);
     dfree(dbase);
-    recb = nrec;
+    hotb = nhot;
+    stb = nst;
+    rcb = nrc;
     size64 = nsize;
     dbase = nbase;
     U = n;
@@ -1107,15 +1118,16 @@ struct Context {
   std::map<std::pair<uint64_t, uint64_t>, Shadow> shadows;
   uint64_t table_gen = 0;
   int take_snapshot() {
-    CKS(dalloc(snap_rec, sizeof(UnitRec) * (size_t)U + 64));
-    CK(cudaMemcpyAsync(snap_rec.as<void>(), recb.as<void>(), sizeof(UnitRec) * (size_t)U, cudaMemcpyDeviceToDevice,
-                       main));
+    CKS(dalloc(snap_st, 8 * (size_t)U + 64));
+    CKS(dalloc(snap_rc, 4 * (size_t)U + 64));
+    CK(cudaMemcpyAsync(snap_rc.as<void>(), rcb.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
+    CK(cudaMemcpyAsync(snap_st.as<void>(), stb.as<void>(), 8 * (size_t)U, cudaMemcpyDeviceToDevice, main));
     return CGCM_OK;
   }
   int restore_snapshot() {
-    // the pass does not touch hot words: restoring whole records restores refcounts and epochs
-    CK(cudaMemcpyAsync(recb.as<void>(), snap_rec.as<void>(), sizeof(UnitRec) * (size_t)U, cudaMemcpyDeviceToDevice,
-                       main));
+    // the pass does not touch hot words or flags: restoring the state words restores the epochs
+    CK(cudaMemcpyAsync(rcb.as<void>(), snap_rc.as<void>(), 4 * (size_t)U, cudaMemcpyDeviceToDevice, main));
+    CK(cudaMemcpyAsync(stb.as<void>(), snap_st.as<void>(), 8 * (size_t)U, cudaMemcpyDeviceToDevice, main));
     CK(cudaStreamSynchronize(main));
     return CGCM_OK;
   }
@@ -1362,7 +1374,7 @@ int cgcm_undeclare(void *base) {
   HostUnit &u = it->second;
   if (u.idx >= 0) {  // idx refers to the current device table until the next ensure_table()
     int32_t rc = 0;
-    CK(cudaMemcpyAsync(&rc, &C->recb.as<UnitRec>()[u.idx].rc, 4, cudaMemcpyDeviceToHost, C->main));
+    CK(cudaMemcpyAsync(&rc, C->rcb.as<int32_t>() + u.idx, 4, cudaMemcpyDeviceToHost, C->main));
     CK(cudaStreamSynchronize(C->main));
     if (rc > 0) return CGCM_E_BUSY;
   }
@@ -1464,7 +1476,7 @@ void *cgcm_realloc(void *p, size_t n) {
   auto ru = C->reg.find(a);
   if (ru != C->reg.end() && ru->second.idx >= 0) {  // a mapped AU cannot move (BUSY)
     int32_t rc = 0;
-    if (cudaMemcpy(&rc, &C->recb.as<UnitRec>()[ru->second.idx].rc, 4, cudaMemcpyDeviceToHost) != cudaSuccess || rc > 0)
+    if (cudaMemcpy(&rc, C->rcb.as<int32_t>() + ru->second.idx, 4, cudaMemcpyDeviceToHost) != cudaSuccess || rc > 0)
       return nullptr;
   }
   size_t old = it->second;
@@ -1502,7 +1514,7 @@ int cgcm_scopeExit(void) {
     auto ru = C->reg.find(a);
     if (ru == C->reg.end() || ru->second.idx < 0) continue;
     int32_t rc = 0;
-    CK(cudaMemcpy(&rc, &C->recb.as<UnitRec>()[ru->second.idx].rc, 4, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&rc, C->rcb.as<int32_t>() + ru->second.idx, 4, cudaMemcpyDeviceToHost));
     if (rc > 0) return CGCM_E_BUSY;
   }
   for (auto it = sc.rbegin(); it != sc.rend(); ++it) CKS(cgcm_free(reinterpret_cast<void *>(*it)));
@@ -1521,8 +1533,12 @@ int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n) {
   Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
   Context::Shadow *sh = nullptr;
   // record (CPU pointer, unit) per slot for the reverse pass (R13-ii) when a lookup costs more than
-  // the 12-byte shadow: deep indexes (measured: a loss at h = 2, a win at h = 3)
-  if (n >= SHADOW_MIN && (C->fwd.h >= 3 || (C->flags & CGCM_FORCE_SHADOW))) {
+  // the 12-byte shadow: indexes with >= 2 levels (measured, config C (h = 2): 48.5 vs 43.5 G/s)
+  static const int shadow_min_h = [] {  // CGCM_SHADOW_MIN_H: A/B override of the depth threshold
+    const char *e = std::getenv("CGCM_SHADOW_MIN_H");
+    return e ? std::atoi(e) : 2;
+  }();
+  if (n >= SHADOW_MIN && (C->fwd.h >= shadow_min_h || (C->flags & CGCM_FORCE_SHADOW))) {
     auto key = std::make_pair(s.ptr, (uint64_t)n);
     sh = &C->shadows[key];
     sh->valid = false;
@@ -2036,23 +2052,26 @@ int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
   CKS(C->ensure_table());
   if (n) *n = (size_t)C->U;
   if (!out || cap == 0) return (size_t)C->U <= cap ? CGCM_OK : CGCM_E_NOMEM;
-  std::vector<UnitRec> recs;
+  std::vector<uint64_t> hots, sts;
+  std::vector<int32_t> rcs;
   std::vector<uint64_t> szs;
-  CKS(C->download(recs, C->recb, (size_t)C->U));
+  CKS(C->download(hots, C->hotb, (size_t)C->U));
+  CKS(C->download(sts, C->stb, (size_t)C->U));
+  CKS(C->download(rcs, C->rcb, (size_t)C->U));
   CKS(C->download(szs, C->size64, (size_t)C->U));
   size_t m = std::min(cap, (size_t)C->U);
   for (size_t i = 0; i < m; ++i) {
     cgcm_unit_t &u = out[i];
-    const uint32_t fl = hot_flags(recs[i].hot);
+    const uint32_t fl = hot_flags(hots[i]);
     u.base = C->ubase[i];
     u.size = szs[i];
-    bool act = recs[i].rc > 0;
-    uint32_t e = hot_ext(recs[i].hot);
+    bool act = rcs[i] > 0;
+    uint32_t e = hot_ext(hots[i]);
     u.devptr = ((fl & UF_STORAGE) && (act || (fl & UF_GLOBAL)) && e < C->runs.size())
                    ? u.base - C->runs[e].delta
                    : 0;
-    u.refCount = recs[i].rc;
-    u.epoch = C->origin + recs[i].epoch;
+    u.refCount = rcs[i];
+    u.epoch = C->origin + st_epoch(sts[i]);
     u.flags = ((fl & UF_GLOBAL) ? CGCM_UNIT_GLOBAL : 0) | ((fl & UF_READONLY) ? CGCM_UNIT_READONLY : 0) |
               ((fl & UF_ARRAYMAPPED) ? CGCM_UNIT_ARRAYMAPPED : 0) | (act ? CGCM_UNIT_ACTIVE : 0);
     u.pad = 0;

@@ -16,8 +16,11 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def run(libdir, config, steps):
+def run(spec, config, steps):
+    # spec = LIBDIR[@VAR=VAL,VAR=VAL]: a variant build plus environment overrides
+    libdir, _, extra = spec.partition("@")
     env = dict(os.environ, CGCM_LIBDIR=os.path.abspath(libdir))
+    env.update(kv.split("=", 1) for kv in extra.split(",") if kv)
     cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--config", config, "--steps", str(steps), "--warmup", "3",
            "--no-e2e", "--no-cpu-baseline"]
     r = subprocess.run(cmd, capture_output=True, text=True, env=env, cwd=ROOT)
@@ -40,7 +43,7 @@ def main():
     for c in a.configs.split(","):
         for rnd in range(a.rounds):
             for ld in a.libdirs:
-                print(json.dumps({"config": c, "round": rnd, "variant": os.path.basename(ld.rstrip("/")),
+                print(json.dumps({"config": c, "round": rnd, "variant": os.path.basename(ld.split("@")[0].rstrip("/")) + ld.partition("@")[1] + ld.partition("@")[2],
                                   **run(ld, c, a.steps)}), flush=True)
 
 
