@@ -46,7 +46,8 @@ enum {
                               activation so map->unmap with no launch copies nothing)             */
   CGCM_LENIENT = 2u,       /* A18: uncovered non-null words in pointer arrays pass through (counted) */
   CGCM_PROFILE = 4u,       /* time every hot kernel with CUDA events on its launch stream (stats)  */
-  CGCM_FORCE_SHADOW = 8u   /* always record the forward-map shadow of device arrays (tests)        */
+  CGCM_FORCE_SHADOW = 8u,  /* always record the forward-map shadow of device arrays (tests)        */
+  CGCM_NO_PAGEDIR = 16u    /* hot kernels search the level index instead of the page directory     */
 };
 
 /* ---- AU flags (declare + dump) ------------------------------------------------------------- */
@@ -174,6 +175,20 @@ int cgcm_resetStats(void);
 int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n);
 /* arena usage in bytes (AU copies + runtime scratch), for balance checks */
 int cgcm_arenaUsage(size_t *used, size_t *capacity);
+/* the forward search structures of the current table (built on demand, like a map would):
+ * the level index (top splitters + `levels` u32 sector levels) always exists; the page directory
+ * is what the hot kernels search when pd_segments > 0.  Implementation detail
+ * (A22), for tests and the bench.                                                              */
+typedef struct {
+  uint64_t units;             /* AUs in the device table                                          */
+  uint32_t levels;            /* sector levels below the shared-memory top of the level index     */
+  uint32_t pd_segments;       /* page-directory address segments (0: none built)                 */
+  uint64_t pd_pages;          /* 32-byte page entries                                             */
+  uint64_t pd_overflow_pages; /* pages with more than 12 unit starts (offsets in a side array)    */
+  uint64_t pd_bytes;          /* entries + overflow offsets                                       */
+  uint32_t pd_min_shift, pd_max_shift; /* page sizes 2^shift of the segments                     */
+} cgcm_index_info_t;
+int cgcm_indexInfo(cgcm_index_info_t *out);
 
 #ifdef __cplusplus
 }

@@ -23,7 +23,7 @@ SAMPLES_PATH = os.path.join(HERE, "libcgcm_samples.so")
 OK = 0
 E_INVALID, E_UNREGISTERED, E_OVERLAP, E_NOT_MAPPED, E_BUSY, E_DUPLICATE, E_NOMEM, E_CUDA, E_MIXED, E_NOCTX = (
     -1, -2, -3, -4, -5, -6, -7, -8, -9, -10)
-LITERAL_EPOCH, LENIENT, PROFILE, FORCE_SHADOW = 1, 2, 4, 8
+LITERAL_EPOCH, LENIENT, PROFILE, FORCE_SHADOW, NO_PAGEDIR = 1, 2, 4, 8, 16
 UNIT_GLOBAL, UNIT_READONLY, UNIT_ARRAYMAPPED, UNIT_ACTIVE = 1, 2, 4, 8
 RELEASE = 1
 
@@ -42,6 +42,12 @@ class Stats(C.Structure):
     _fields_ = [(f, C.c_uint64) for f in STAT_FIELDS] + [
         ("fwd_kernel_ms", C.c_double), ("rev_kernel_ms", C.c_double), ("fwd_kernel_calls", C.c_uint64),
         ("rev_kernel_calls", C.c_uint64), ("fwd_kernel_slots", C.c_uint64), ("rev_kernel_slots", C.c_uint64)]
+
+
+class IndexInfo(C.Structure):
+    _fields_ = [("units", C.c_uint64), ("levels", C.c_uint32), ("pd_segments", C.c_uint32),
+                ("pd_pages", C.c_uint64), ("pd_overflow_pages", C.c_uint64), ("pd_bytes", C.c_uint64),
+                ("pd_min_shift", C.c_uint32), ("pd_max_shift", C.c_uint32)]
 
 
 class CgcmError(RuntimeError):
@@ -81,6 +87,7 @@ def lib():
             "cgcm_stats": (i, [C.POINTER(Stats)]), "cgcm_resetStats": (i, []),
             "cgcm_dumpTable": (i, [vp, sz, C.POINTER(C.c_size_t)]),
             "cgcm_arenaUsage": (i, [C.POINTER(C.c_size_t), C.POINTER(C.c_size_t)]),
+            "cgcm_indexInfo": (i, [C.POINTER(IndexInfo)]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -281,6 +288,13 @@ class Context:
         u, c = C.c_size_t(0), C.c_size_t(0)
         self.L.cgcm_arenaUsage(C.byref(u), C.byref(c))
         return u.value, c.value
+
+    def indexInfo(self) -> dict:
+        ii = IndexInfo()
+        s = self.L.cgcm_indexInfo(C.byref(ii))
+        if s != OK:
+            raise CgcmError(f"indexInfo: {strerror(s)}")
+        return {f: getattr(ii, f) for f, _ in IndexInfo._fields_}
 
     # ---- test-only sample GPU functions on the main stream ----
     def sample_scale(self, rows_dev, nrows, ncols, alpha):

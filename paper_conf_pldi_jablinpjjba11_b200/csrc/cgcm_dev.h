@@ -84,6 +84,31 @@ struct IndexDev {
   int n, h, ntop, nseg, ndir;
 };
 
+// Page directory: the forward index of the hot kernels.  The sorted AU bases are cut
+// into address segments at the largest start-to-start distances (<= PD_MAXSEG; starts, ends and
+// metadata staged in shared memory).  Segment s has pages of 2^P_s bytes (P_s <= 15) from start_s
+// (its first base) through its last base; an address beyond its pages but before the next segment
+// lies in the tail of the segment's last unit (hit iff <= end_s, A7).
+// One 32-byte entry (one L2 sector) per page at address A:
+//   w[0]     j0 = greatestLTE(A), the unit with the greatest base <= A (0xFFFFFFFF: none)
+//   w[1]     cnt (bits 0..14): units with base in (A, A + 2^P) | bit 15: base(j0) == A
+//            | end0 (bits 16..31): min(base(j0) + size(j0) - A + 1, 0xFFFF), 0 if j0 ends before A
+//   w[2..7]  cnt <= PD_K: the offsets base - A of those units, sorted u16, padded with 0xFFFF;
+//            cnt >  PD_K: w[2] = index of the first of cnt sorted u16 offsets in ovf[] (16-aligned,
+//            padded with 0xFFFF to a whole 32-byte sector)
+// greatestLTE(p) = j0 + #{offsets <= p - A}; p hits unit j0 iff p - A < end0 (A7: p - base <= size),
+// any other candidate by its base A + offset and its size (hot word).  One sector gather per lookup.
+constexpr int PD_MAXSEG = 64;
+constexpr int PD_K = 12;
+constexpr int PD_MAXSHIFT = 15;
+struct PdDev {
+  const uint32_t *ent;        // 8 u32 per page, segments back to back
+  const uint16_t *ovf;        // overflow offsets
+  const uint64_t *seg_start;  // [2*nseg] first unit base of each segment, then end (base + size) of its last unit
+  const uint32_t *seg_meta;   // [4*nseg]: first page, npages, P, last unit
+  int nseg;                   // 0: no page directory (the level index is used)
+};
+
 // One input segment of a slot kernel: n u64 slots at device address ptr (8-byte aligned),
 // translated in place (out == 0) or into out.  inc = refcount delta per non-null slot.
 // shadow (optional, 12 B per slot: u64 CPU pointer[n] then u32 unit[n]): written by the forward map,
@@ -141,6 +166,7 @@ enum : int { SEL_ALL = 0, SEL_HIT = 1, SEL_NOTHIT = 2 };
 
 struct SlotArgs {
   IndexDev fx;                 // forward index over unit bases
+  PdDev pd;                    // page directory over the same bases (hot kernels, when built)
   IndexDev rx;                 // reverse index over device extents (DIR_REV)
   const uint64_t *runpay;      // per sorted extent: host - device address delta (mirrored layout)
   const uint32_t *runid;       // per sorted extent: its extent id

@@ -303,6 +303,115 @@ __device__ __forceinline__ void level_lookup2(const SIdx &S, const IndexDev &ix,
   }
 }
 
+// ---- page directory (cgcm_dev.h PdDev): segment starts and metadata staged in shared memory ----
+struct SPd {
+  const uint64_t *start;  // [nseg] starts, then [nseg] ends
+  const uint32_t *meta;
+  int nseg;
+};
+__host__ __device__ __forceinline__ size_t pd_stage_bytes(const PdDev &pd) {
+  return al16(16 * (size_t)pd.nseg) + al16(16 * (size_t)pd.nseg);
+}
+__device__ __forceinline__ unsigned char *stage_pd(const PdDev &pd, unsigned char *base, SPd &S) {
+  uint64_t *st = reinterpret_cast<uint64_t *>(base);
+  base += al16(16 * (size_t)pd.nseg);
+  uint32_t *mt = reinterpret_cast<uint32_t *>(base);
+  base += al16(16 * (size_t)pd.nseg);
+  for (int t = threadIdx.x; t < 2 * pd.nseg; t += blockDim.x) st[t] = pd.seg_start[t];
+  for (int t = threadIdx.x; t < 4 * pd.nseg; t += blockDim.x) mt[t] = pd.seg_meta[t];
+  S.start = st;
+  S.meta = mt;
+  S.nseg = pd.nseg;
+  return base;
+}
+// count and maximum of the u16 offsets <= r (r replicated in both halves) in one 32-bit word
+__device__ __forceinline__ void cnt_max2(uint32_t w, uint32_t rr, uint32_t &cnt, uint32_t &mx) {
+  const uint32_t m = __vcmpleu2(w, rr);
+  cnt += __popc(m);
+  mx = __vmaxu2(mx, w & m);
+}
+
+// Two interleaved greatestLTE lookups through the page directory.  In: q (host addresses), look.
+// Out: j (unit or -1), key (its base, or for a hit on the page's j0: A if base(j0) == A, else A - 1,
+// which no query equals), k0 (the unit is the page's j0: hit decided here, h0), h0.
+__device__ __forceinline__ void pd_lookup2(const SPd &S, const PdDev &pd, uint64_t pol, const uint64_t q[2],
+                                           const bool look[2], int j[2], uint64_t key[2], bool k0[2]) {
+  uint64_t w[2][4];
+  uint64_t A[2];
+  uint32_t poff[2];
+  bool ok[2];
+  int tail[2];  // beyond the segment's pages: its last unit, or -1 (miss)
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    ok[m] = look[m];
+    int s = 0;
+    if (S.nseg > 1) {
+      int lo = 0, len = S.nseg;
+      while (len > 1) {
+        const int half = len >> 1;
+        if (S.start[lo + half] <= q[m]) lo += half;
+        len -= half;
+      }
+      s = lo;
+    }
+    const uint64_t rel = q[m] - S.start[s];
+    const uint32_t P = S.meta[4 * s + 2];
+    const uint64_t pg = rel >> P;
+    ok[m] = ok[m] && q[m] >= S.start[s];
+    tail[m] = ok[m] && pg >= S.meta[4 * s + 1] ? (q[m] <= S.start[S.nseg + s] ? (int)S.meta[4 * s + 3] : -1) : -2;
+    ok[m] = ok[m] && tail[m] == -2;
+    poff[m] = (uint32_t)rel & ((1u << P) - 1u);
+    A[m] = q[m] - poff[m];
+    if (ok[m]) {
+      ld_sector(pd.ent + 8 * ((uint64_t)S.meta[4 * s] + pg), pol, w[m]);
+    } else {
+      w[m][0] = w[m][1] = w[m][2] = w[m][3] = 0;
+    }
+  }
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    const uint32_t j0 = (uint32_t)w[m][0], w1 = (uint32_t)(w[m][0] >> 32);
+    const uint32_t cnt = w1 & 0x7FFFu, end0 = w1 >> 16;
+    const uint32_t rr = poff[m] * 0x10001u;
+    uint32_t c = 0, mx = 0;
+    if (cnt <= (uint32_t)PD_K) {
+#pragma unroll
+      for (int t = 1; t < 4; ++t) {
+        cnt_max2((uint32_t)w[m][t], rr, c, mx);
+        cnt_max2((uint32_t)(w[m][t] >> 32), rr, c, mx);
+      }
+    } else {  // crowded page: the offsets continue in ovf[], one sector per 16
+      const uint16_t *o = pd.ovf + (uint32_t)w[m][1];
+      for (uint32_t t = 0; t < cnt; t += 16) {
+        uint64_t v[4];
+        ld_sector(o + t, pol, v);
+        const uint32_t c0 = c;
+#pragma unroll
+        for (int z = 0; z < 4; ++z) {
+          cnt_max2((uint32_t)v[z], rr, c, mx);
+          cnt_max2((uint32_t)(v[z] >> 32), rr, c, mx);
+        }
+        if (c - c0 < 16u * 16u) break;  // later sectors hold larger offsets only
+      }
+    }
+    const uint32_t k = c >> 4;
+    const uint32_t off = max(mx & 0xFFFFu, mx >> 16);
+    k0[m] = k == 0;
+    if (tail[m] != -2) {  // the tail of the segment's last unit (decided by its end) or a miss
+      k0[m] = true;
+      j[m] = tail[m];
+      key[m] = q[m] - 1;
+    } else if (k == 0) {
+      const bool h0 = ok[m] && j0 != 0xFFFFFFFFu && poff[m] < end0;  // A7 on the page's j0
+      j[m] = h0 ? (int)j0 : -1;
+      key[m] = (w1 & 0x8000u) ? A[m] : A[m] - 1;
+    } else {
+      j[m] = ok[m] ? (int)(j0 + k) : -1;
+      key[m] = A[m] + off;
+    }
+  }
+}
+
 }  // namespace
 
 // -------------------------------------------------------------------------------------------------
@@ -321,12 +430,17 @@ struct SlotCfg {
 #endif
 };
 
+constexpr int FH_PD = -2;  // forward lookups through the page directory
+
 template <int DIR, int OPS, int FH, int SH>
 __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ uint64_t s_seg0[SEG_SMEM + 1];
   SIdx F, R;
-  unsigned char *sp = stage(a.fx, nullptr, nullptr, smem, F);
+  SPd PD;
+  unsigned char *sp = smem;
+  if constexpr (FH == FH_PD) sp = stage_pd(a.pd, sp, PD);
+  else sp = stage(a.fx, nullptr, nullptr, sp, F);
   if (DIR == DIR_REV) sp = stage(a.rx, a.rx.h == 0 ? a.runpay : nullptr, a.runid, sp, R);
   // extent deltas (devbase - base of every copy in the extent), staged when few
   const bool ext_s = a.tab.n_ext <= EXT_SMEM;
@@ -436,6 +550,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
     // the whole search (a warp-uniform branch, not predication)
     j[0] = j[1] = -1;
     key[0] = key[1] = 0;
+    bool k0[2] = {false, false};  // page directory: the hit on the page's j0 was decided by the lookup
     if (!(SH && DIR == DIR_REV) || __any_sync(0xffffffffu, look[0] || look[1])) {
     if (DIR == DIR_REV) {
       // the device extent holding the pointer, and the host address it mirrors
@@ -457,14 +572,18 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         q[m] = look[m] ? q[m] + dx[m] : 0ull;  // host address
       }
     }
+    if constexpr (FH == FH_PD) {
+      pd_lookup2(PD, a.pd, pol_t, q, look, j, key, k0);
+    } else {
 #pragma unroll
-    for (int m = 0; m < 2; ++m) {
-      uint64_t tk = 0;
-      j[m] = look[m] ? top_search<(FH >= 0)>(F, q[m], tk) : -1;
-      key[m] = tk;
+      for (int m = 0; m < 2; ++m) {
+        uint64_t tk = 0;
+        j[m] = look[m] ? top_search<(FH >= 0)>(F, q[m], tk) : -1;
+        key[m] = tk;
+      }
+      if constexpr (FH > 0) level_lookup2_fixed<FH>(a.fx, pol_t, q, j, key);
+      else if constexpr (FH < 0) level_lookup2(F, a.fx, pol_t, q, j, key);
     }
-    if constexpr (FH > 0) level_lookup2_fixed<FH>(a.fx, pol_t, q, j, key);
-    else if constexpr (FH < 0) level_lookup2(F, a.fx, pol_t, q, j, key);
 
     // ---- the unit's hot word (size | extent | flags), and its state word where the epoch is needed ----
 #pragma unroll
@@ -479,7 +598,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
     for (int m = 0; m < 2; ++m) {
       uint64_t sz = hot_size32(hw[m]);
       if (look[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
-      hit[m] = look[m] && (q[m] - key[m] <= sz);  // A7: p - base <= size
+      hit[m] = look[m] && (k0[m] || q[m] - key[m] <= sz);  // A7: p - base <= size
       if (DIR == DIR_REV && look[m]) {
         // the unit must own this extent's copy: active, and its copy lives in that extent
         if (!(hit[m] && (hot_flags(hw[m]) & UF_ACTIVE) && hot_ext(hw[m]) == rid[m])) {
@@ -687,14 +806,14 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
   X(DIR_REV, OP_DEC)                                   /* releaseArray of an array-mapped outer  */ \
   X(DIR_REV, OP_DECPLAIN)                              /* rollback of REV INCPLAIN               */
 
-static size_t slots_smem(const SlotArgs &a, int dir) {
-  return stage_bytes(a.fx, false) + (dir == DIR_REV ? stage_bytes(a.rx, a.rx.h == 0) : 0) +
+static size_t slots_smem(const SlotArgs &a, int dir, bool pd) {
+  return (pd ? pd_stage_bytes(a.pd) : stage_bytes(a.fx, false)) + (dir == DIR_REV ? stage_bytes(a.rx, a.rx.h == 0) : 0) +
          (a.tab.n_ext <= EXT_SMEM ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
 }
 
 template <int DIR, int OPS, int FH, int SH>
 static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
-  size_t smem = slots_smem(a, DIR);
+  size_t smem = slots_smem(a, DIR, FH == FH_PD);
   // the 48 KiB default covers static + dynamic shared memory: opt in to the full carve-out once
   static bool configured = false;
   if (!configured) {
@@ -725,18 +844,20 @@ static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
 
 int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s) {
   // the forward index qualifies for the specialised path: one segment, no wide bucket, h <= 3
-  int fh = a.fx.nseg <= 1 && a.fx_nowide && a.fx.h <= 3 ? a.fx.h : -1;
+  int fh = a.pd.nseg > 0 ? FH_PD : a.fx.nseg <= 1 && a.fx_nowide && a.fx.h <= 3 ? a.fx.h : -1;
   const bool sh = a.nseg == 1 && a.segs_host_shadow;
 #define X(D, O)                                                        \
   if (dir == D && ops == (O)) {                                        \
     if (sh) {                                                          \
       switch (fh) {                                                    \
+        case FH_PD: return launch_one<D, (O), FH_PD, 1>(a, nsm, s);    \
         case 2: return launch_one<D, (O), 2, 1>(a, nsm, s);            \
         case 3: return launch_one<D, (O), 3, 1>(a, nsm, s);            \
         default: return launch_one<D, (O), -1, 1>(a, nsm, s);          \
       }                                                                \
     }                                                                  \
     switch (fh) {                                                      \
+      case FH_PD: return launch_one<D, (O), FH_PD, 0>(a, nsm, s);      \
       case 0: return launch_one<D, (O), 0, 0>(a, nsm, s);              \
       case 1: return launch_one<D, (O), 1, 0>(a, nsm, s);              \
       case 2: return launch_one<D, (O), 2, 0>(a, nsm, s);              \

@@ -212,6 +212,11 @@ struct Context {
   DevBuf hotb, stb, rcb, size64, dbase, extd, snap_st, snap_rc;  // unit table columns + extent deltas
   size_t extd_n = 0;                          // entries uploaded to extd
   IndexBufs fwd, rev;
+  // page directory over the unit bases (cgcm_dev.h PdDev; built with the table)
+  DevBuf pd_ent, pd_ovf, pd_start, pd_meta;
+  int pd_nseg = 0;
+  uint64_t pd_pages = 0, pd_ovf_pages = 0, pd_bytes = 0;
+  uint32_t pd_minP = 0, pd_maxP = 0;
 
   // scratch
   DevBuf status, lc, hitmask, act_list, journal, free_list, copy_list, segs, seg0, staging, staging2, staging_cb, points, ptrs, temp;
@@ -385,6 +390,127 @@ struct Context {
     return CGCM_OK;
   }
 
+  // Page directory (a0): cut the sorted bases at the largest start-to-start distances (>= 1 MiB, at
+  // most PD_MAXSEG segments; pages stop at a segment's last base, whose unit's tail is decided by
+  // the segment's end), give each segment the largest page size 2^P (P <= 15) whose crowded pages (more than
+  // PD_K starts) hold at most CGCM_PD_OVF (default 1 %) of its units, within a budget of
+  // max(4n, 2^20) entries overall; then one entry per page (cgcm_dev.h).  No directory (the level
+  // index serves the hot kernels) when the budget cannot be met or CGCM_NO_PAGEDIR is set.
+  int build_pd(const uint64_t *hb, const uint64_t *hs, int n) {
+    pd_nseg = 0;
+    pd_pages = pd_ovf_pages = pd_bytes = 0;
+    pd_minP = pd_maxP = 0;
+    if (n == 0 || (flags & CGCM_NO_PAGEDIR)) return CGCM_OK;
+    static const double ovf_frac = [] {
+      const char *e = std::getenv("CGCM_PD_OVF");
+      return e ? std::atof(e) : 0.01;
+    }();
+    std::vector<std::pair<uint64_t, int>> gaps;
+    for (int i = 0; i + 1 < n; ++i) {
+      const uint64_t g = hb[i + 1] - hb[i];  // start to start: a huge unit's tail needs no pages
+      if (g >= (1ull << 20)) gaps.emplace_back(g, i + 1);
+    }
+    if ((int)gaps.size() > PD_MAXSEG - 1) {
+      std::nth_element(gaps.begin(), gaps.begin() + (PD_MAXSEG - 1), gaps.end(),
+                       [](const std::pair<uint64_t, int> &a, const std::pair<uint64_t, int> &b) { return a.first > b.first; });
+      gaps.resize(PD_MAXSEG - 1);
+    }
+    std::vector<int> cut{0};
+    for (auto &g : gaps) cut.push_back(g.second);
+    std::sort(cut.begin(), cut.end());
+    cut.push_back(n);
+    const int nseg = (int)cut.size() - 1;
+    const uint64_t budget = std::max<uint64_t>(4ull * (uint64_t)n, 1ull << 20);
+    std::vector<uint32_t> Ps(nseg);
+    std::vector<uint64_t> npg(nseg);
+    uint64_t total = 0;
+    for (int s = 0; s < nseg; ++s) {
+      const int i0 = cut[s], i1 = cut[s + 1];
+      const uint64_t S = hb[i0], span = hb[i1 - 1] - S;  // pages up to the last base; beyond: its tail
+      const uint64_t cap = budget * (uint64_t)(i1 - i0) / (uint64_t)n + 1024;
+      int sel = -1;
+      for (int P = PD_MAXSHIFT; P >= 0; --P) {
+        if ((span >> P) + 1 > cap) break;
+        sel = P;
+        uint64_t ovf = 0;  // units in pages with more than PD_K starts after the page's first byte
+        for (int i = i0; i < i1;) {
+          const uint64_t pg = (hb[i] - S) >> P;
+          int k = i, c = 0;
+          while (k < i1 && ((hb[k] - S) >> P) == pg) {
+            c += ((hb[k] - S) & ((1ull << P) - 1)) != 0;
+            ++k;
+          }
+          if (c > PD_K) ovf += (uint64_t)c;
+          i = k;
+        }
+        if ((double)ovf <= ovf_frac * (double)(i1 - i0)) break;
+      }
+      if (sel < 0) return CGCM_OK;  // too sparse for the budget: the level index serves
+      Ps[s] = (uint32_t)sel;
+      npg[s] = (span >> sel) + 1;
+      total += npg[s];
+    }
+    std::vector<uint32_t> ent(8 * total);
+    std::vector<uint16_t> ovf;
+    std::vector<uint64_t> starts(2 * nseg);  // [start_s..., last_end_s...]
+    std::vector<uint32_t> meta(4 * nseg, 0);
+    uint64_t e = 0, novf = 0;
+    for (int s = 0; s < nseg; ++s) {
+      const int i0 = cut[s], i1 = cut[s + 1];
+      const uint64_t S = hb[i0], psz = 1ull << Ps[s];
+      starts[s] = S;
+      starts[nseg + s] = hb[i1 - 1] + hs[i1 - 1];
+      meta[4 * s] = (uint32_t)e;
+      meta[4 * s + 1] = (uint32_t)npg[s];
+      meta[4 * s + 2] = Ps[s];
+      meta[4 * s + 3] = (uint32_t)(i1 - 1);
+      int i = i0;  // greatestLTE(A)
+      for (uint64_t g = 0; g < npg[s]; ++g, ++e) {
+        const uint64_t A = S + (g << Ps[s]);
+        while (i + 1 < i1 && hb[i + 1] <= A) ++i;
+        int k = i + 1;
+        while (k < i1 && hb[k] < A + psz) ++k;
+        const uint32_t cnt = (uint32_t)(k - (i + 1));
+        const uint64_t e0 = hb[i] + hs[i];
+        const uint32_t end0 = e0 < A ? 0u : (uint32_t)std::min<uint64_t>(e0 - A + 1, 0xFFFF);
+        uint32_t *w = &ent[8 * e];
+        w[0] = (uint32_t)i;
+        w[1] = cnt | (hb[i] == A ? 0x8000u : 0u) | (end0 << 16);
+        uint16_t *o16 = reinterpret_cast<uint16_t *>(w + 2);
+        if (cnt <= (uint32_t)PD_K) {
+          for (int t = 0; t < 2 * 6; ++t) o16[t] = t < (int)cnt ? (uint16_t)(hb[i + 1 + t] - A) : (uint16_t)0xFFFF;
+        } else {
+          w[2] = (uint32_t)ovf.size();
+          w[3] = w[4] = w[5] = w[6] = w[7] = 0xFFFFFFFFu;
+          for (uint32_t t = 0; t < cnt; ++t) ovf.push_back((uint16_t)(hb[i + 1 + t] - A));
+          while (ovf.size() % 16) ovf.push_back(0xFFFF);
+          ++novf;
+        }
+      }
+    }
+    if (ovf.empty()) ovf.assign(16, 0xFFFF);
+    CKS(upload(pd_ent, ent));
+    CKS(upload(pd_ovf, ovf));
+    CKS(upload(pd_start, starts));
+    CKS(upload(pd_meta, meta));
+    pd_nseg = nseg;
+    pd_pages = total;
+    pd_ovf_pages = novf;
+    pd_bytes = 32 * total + 2 * ovf.size();
+    pd_minP = *std::min_element(Ps.begin(), Ps.end());
+    pd_maxP = *std::max_element(Ps.begin(), Ps.end());
+    return CGCM_OK;
+  }
+  PdDev pd_view() const {
+    PdDev p;
+    p.ent = pd_ent.as<uint32_t>();
+    p.ovf = pd_ovf.as<uint16_t>();
+    p.seg_start = pd_start.as<uint64_t>();
+    p.seg_meta = pd_meta.as<uint32_t>();
+    p.nseg = pd_nseg;
+    return p;
+  }
+
   // merge pending declares/undeclares into the device table (A19: kernels only see a compacted table)
   int ensure_table() {
     if (!table_dirty) return CGCM_OK;
@@ -461,6 +587,7 @@ struct Context {
     dbase = nbase;
     U = n;
     CKS(build_index(fwd, hb, n, dbase.as<uint64_t>(), TOPMAX, DIRMAX));
+    CKS(build_pd(hb, hs, n));
     CK(cudaStreamSynchronize(main));
     table_dirty = false;
     rev_dirty = true;
@@ -542,6 +669,7 @@ struct Context {
     a.tab = tab();
     a.fx = fwd.view(dbase.as<uint64_t>());
     a.fx_nowide = fwd.any_wide ? 0 : 1;
+    a.pd = pd_view();
     if (c.dir == DIR_REV) {
       a.rx = rev.view(rev.keys.as<uint64_t>());
       a.runpay = rev.pay.as<uint64_t>();
@@ -2082,6 +2210,22 @@ int cgcm_arenaUsage(size_t *used, size_t *capacity) {
   CTX();
   if (used) *used = C->arena.used();
   if (capacity) *capacity = C->arena.capacity();
+  return CGCM_OK;
+}
+
+int cgcm_indexInfo(cgcm_index_info_t *out) {
+  CTX();
+  if (!out) return CGCM_E_INVALID;
+  CKS(C->ensure_table());
+  std::memset(out, 0, sizeof(*out));
+  out->units = (uint64_t)C->U;
+  out->levels = (uint32_t)C->fwd.h;
+  out->pd_segments = (uint32_t)C->pd_nseg;
+  out->pd_pages = C->pd_pages;
+  out->pd_overflow_pages = C->pd_ovf_pages;
+  out->pd_bytes = C->pd_bytes;
+  out->pd_min_shift = C->pd_minP;
+  out->pd_max_shift = C->pd_maxP;
   return CGCM_OK;
 }
 

@@ -18,7 +18,7 @@ def cgcm_mod():
     return cg
 
 
-@pytest.fixture(params=[0, 8], ids=["auto", "shadow"])
+@pytest.fixture(params=[0, 8, 16], ids=["auto", "shadow", "levels"])
 def pair(cgcm_mod, request):
     from oracle import Oracle
     ctx = cgcm_mod.Context(0, arena_bytes=1 << 30, flags=request.param)
