@@ -162,7 +162,9 @@ enum : int {
   OP_DECPLAIN = 128  // refcount -= inc (rollback of OP_INC)
 };
 enum : int { DIR_FWD = 0, DIR_REV = 1 };
-enum : int { SEL_ALL = 0, SEL_HIT = 1, SEL_NOTHIT = 2 };
+// slot selection: all, those in the hit mask, those not in it, those in the slow mask (the slots a
+// pipelined pass left to the generic kernel; the pass then ORs its hits into the hit mask)
+enum : int { SEL_ALL = 0, SEL_HIT = 1, SEL_NOTHIT = 2, SEL_SLOW = 3 };
 
 struct SlotArgs {
   IndexDev fx;                 // forward index over unit bases
@@ -177,6 +179,8 @@ struct SlotArgs {
   int sel;
   uint64_t nchunks;
   uint32_t *hitmask;           // 2 bits per chunk: slot m of the chunk was translated
+  uint32_t *slowmask;          // 2 bits per chunk: left to the generic kernel by k_unmap_sh
+  unsigned long long *slowcount;  // how many (the generic pass exits at once when 0)
   uint32_t epoch;               // globalEpoch - origin
   Status *st;
   unsigned long long *lc;      // shared list counters of the call: [0] act, [1] journal, [2] free, [3] copy
@@ -189,10 +193,11 @@ struct SlotArgs {
   int no_journal;              // the host snapshotted rc/epoch columns: no per-unit epoch journal
   int fx_nowide;               // the forward index has no wide bucket (specialised kernels)
   int segs_host_shadow;        // the (single) segment carries a shadow: use the shadow variant
+  int seg_inplace;             // the (single) segment is translated in place (out == 0)
 };
 
 // ---- host-callable launchers (kernels.cu) ----------------------------------------------------
-int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s);
+int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, int *nlaunch);
 void launch_build_levels(const uint64_t *keys, int n, int h, const uint32_t *wide, uint32_t *const *lvl,
                          const size_t *lvl_cap, cudaStream_t s);
 void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uint32_t *flags, const uint32_t *epoch0,

@@ -14,6 +14,8 @@
 // DESIGN.md §7 gives the roofline of each kernel and its algorithmic bytes.
 #include <cub/cub.cuh>
 
+#include <cstdlib>
+
 #include "cgcm_dev.h"
 
 namespace cgcm {
@@ -331,7 +333,87 @@ __device__ __forceinline__ void cnt_max2(uint32_t w, uint32_t rr, uint32_t &cnt,
   mx = __vmaxu2(mx, w & m);
 }
 
-// Two interleaved greatestLTE lookups through the page directory.  In: q (host addresses), look.
+// Front half of a page-directory lookup of host address q: the segment, the page, and the entry to
+// gather (ok), or the tail of the segment's last unit (tail >= 0: that unit, -1: a miss).
+struct PdFront {
+  uint64_t A;      // the page's first address
+  uint64_t e;      // entry index
+  uint32_t poff;   // q - A
+  int tail;        // -2: look the page up; -1: miss; >= 0: the tail of this unit (decided by the end)
+  bool ok;         // gather entry e
+};
+__device__ __forceinline__ PdFront pd_front(const SPd &S, uint64_t q, bool look) {
+  PdFront f;
+  int s = 0;
+  if (S.nseg > 1) {
+    int lo = 0, len = S.nseg;
+    while (len > 1) {
+      const int half = len >> 1;
+      if (S.start[lo + half] <= q) lo += half;
+      len -= half;
+    }
+    s = lo;
+  }
+  const uint64_t rel = q - S.start[s];
+  const uint32_t P = S.meta[4 * s + 2];
+  const uint64_t pg = rel >> P;
+  const bool in = look && q >= S.start[s];
+  f.tail = in && pg >= S.meta[4 * s + 1] ? (q <= S.start[S.nseg + s] ? (int)S.meta[4 * s + 3] : -1) : -2;
+  f.ok = in && f.tail == -2;
+  if (!in) f.tail = -1;
+  f.poff = (uint32_t)rel & ((1u << P) - 1u);
+  f.A = q - f.poff;
+  f.e = (uint64_t)S.meta[4 * s] + pg;
+  return f;
+}
+// Back half: decode the gathered entry w (ignored unless f.ok).  Out: j (unit or -1), key (its base;
+// for a hit on the page's j0: A if base(j0) == A, else A - 1, which no query equals), k0 (the hit
+// was decided here from end0 or the segment end: no size check).
+__device__ __forceinline__ void pd_back(const PdDev &pd, uint64_t pol, const PdFront &f, uint64_t q,
+                                        const uint64_t w_in[4], int &j, uint64_t &key, bool &k0) {
+  if (!f.ok) {  // tail of the segment's last unit, or a miss
+    k0 = true;
+    j = f.tail;
+    key = q - 1;
+    return;
+  }
+  const uint32_t j0 = (uint32_t)w_in[0], w1 = (uint32_t)(w_in[0] >> 32);
+  const uint32_t cnt = w1 & 0x7FFFu, end0 = w1 >> 16;
+  const uint32_t rr = f.poff * 0x10001u;
+  uint32_t c = 0, mx = 0;
+  if (cnt <= (uint32_t)PD_K) {
+#pragma unroll
+    for (int t = 1; t < 4; ++t) {
+      cnt_max2((uint32_t)w_in[t], rr, c, mx);
+      cnt_max2((uint32_t)(w_in[t] >> 32), rr, c, mx);
+    }
+  } else {  // crowded page: the offsets continue in ovf[], one sector per 16
+    const uint16_t *o = pd.ovf + (uint32_t)w_in[1];
+    for (uint32_t t = 0; t < cnt; t += 16) {
+      uint64_t v[4];
+      ld_sector(o + t, pol, v);
+      const uint32_t c0 = c;
+#pragma unroll
+      for (int z = 0; z < 4; ++z) {
+        cnt_max2((uint32_t)v[z], rr, c, mx);
+        cnt_max2((uint32_t)(v[z] >> 32), rr, c, mx);
+      }
+      if (c - c0 < 16u * 16u) break;  // later sectors hold larger offsets only
+    }
+  }
+  const uint32_t k = c >> 4;
+  k0 = k == 0;
+  if (k == 0) {
+    j = (j0 != 0xFFFFFFFFu && f.poff < end0) ? (int)j0 : -1;  // A7 on the page's j0
+    key = (w1 & 0x8000u) ? f.A : f.A - 1;
+  } else {
+    j = (int)(j0 + k);
+    key = f.A + max(mx & 0xFFFFu, mx >> 16);
+  }
+}
+
+// Two interleaved greatestLTE lookups through the page directory (k_slots; written out rather than
+// through pd_front/pd_back, which costs the reverse shadow variants ~90 bytes of spills).  In: q (host addresses), look.
 // Out: j (unit or -1), key (its base, or for a hit on the page's j0: A if base(j0) == A, else A - 1,
 // which no query equals), k0 (the unit is the page's j0: hit decided here, h0), h0.
 __device__ __forceinline__ void pd_lookup2(const SPd &S, const PdDev &pd, uint64_t pol, const uint64_t q[2],
@@ -434,6 +516,7 @@ constexpr int FH_PD = -2;  // forward lookups through the page directory
 
 template <int DIR, int OPS, int FH, int SH>
 __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs a) {
+  if (a.sel == SEL_SLOW && *a.slowcount == 0) return;  // the pipelined pass decided every slot
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ uint64_t s_seg0[SEG_SMEM + 1];
   SIdx F, R;
@@ -497,8 +580,9 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
       const uint64_t hi_addr = sg.ptr + 8ull * sg.n;
       valid = (a0 >= sg.ptr && a0 < hi_addr ? 1u : 0u) | (a0 + 8 >= sg.ptr && a0 + 8 < hi_addr ? 2u : 0u);
       if (a.sel != SEL_ALL) {
-        uint32_t hm = (a.hitmask[c >> 4] >> (2 * (c & 15))) & 3u;
-        valid &= (a.sel == SEL_HIT) ? hm : ~hm;
+        const uint32_t *mk = a.sel == SEL_SLOW ? a.slowmask : a.hitmask;
+        uint32_t hm = (mk[c >> 4] >> (2 * (c & 15))) & 3u;
+        valid &= (a.sel == SEL_NOTHIT) ? ~hm : hm;
       }
       if (pf) {
         v[0] = cv0;
@@ -772,6 +856,10 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         uint32_t w0 = spread16(b0) | (spread16(b1) << 1);
         uint32_t w1 = spread16(b0 >> 16) | (spread16(b1 >> 16) << 1);
         uint64_t wi = cb >> 4;
+        if (a.sel == SEL_SLOW) {  // the pipelined pass wrote the other hits of these words
+          w0 |= a.hitmask[wi];
+          if (cb + 16 < a.nchunks) w1 |= a.hitmask[wi + 1];
+        }
         a.hitmask[wi] = w0;
         if (cb + 16 < a.nchunks) a.hitmask[wi + 1] = w1;
       }
@@ -786,6 +874,414 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
   }
   if (OPS & OP_CHECKMAPPED) flush_count(&a.st->notmapped, c_notm);
   if (OPS & OP_DEC) flush_count(&a.st->underflow, c_under);
+}
+
+// -------------------------------------------------------------------------------------------------
+// k_map_pd: the forward map of one in-place segment (mapArrayDevice; a1 + a2 of Alg. 1) through the
+// page directory, software-pipelined: while chunk t is translated, the page-directory entries of
+// chunk t+1 are already on their way into shared memory (cp.async, one 32-byte sector per slot) and
+// the slot values of chunk t+2 into registers.  The dependent L2 round trips of one chunk (entry, then
+// the unit's hot word) thus overlap those of the next.  Same results, counters and lists as
+// k_slots<DIR_FWD, OP_WRITE | OP_INC | OP_HITMASK> (which serves every other case).
+// -------------------------------------------------------------------------------------------------
+constexpr int MAP_PD_THREADS = 768;
+
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, uint64_t pol) {
+  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void lds_sector(uint32_t addr, uint64_t v[4]) {
+  asm volatile("ld.shared.v2.u64 {%0,%1}, [%2];" : "=l"(v[0]), "=l"(v[1]) : "r"(addr));
+  asm volatile("ld.shared.v2.u64 {%0,%1}, [%2];" : "=l"(v[2]), "=l"(v[3]) : "r"(addr + 16));
+}
+
+template <int SH>
+__global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  SPd PD;
+  unsigned char *sp = stage_pd(a.pd, smem, PD);
+  const bool ext_s = a.tab.n_ext <= EXT_SMEM;
+  uint64_t *s_ext = reinterpret_cast<uint64_t *>(sp);
+  if (ext_s)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
+  sp += ext_s ? al16(8 * (size_t)a.tab.n_ext) : 0;
+  // entry ring: [stage][slot m][thread] 32 bytes each
+  const uint32_t ring = (uint32_t)__cvta_generic_to_shared(sp);
+  const uint32_t my = ring + 32u * threadIdx.x;
+  const uint32_t mstride = 32u * blockDim.x, sstride = 2u * mstride;
+  __syncthreads();
+
+  const uint64_t pol_s = policy_evict_first();
+  const uint64_t pol_t = policy_evict_last();
+  const int lane = threadIdx.x & 31;
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull, hi_addr = sg.ptr + 8ull * sg.n;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned c_nulls = 0, c_hits = 0, c_miss = 0, c_pend = 0, c_tr = 0;
+
+  auto valid_of = [&](uint64_t c) -> uint32_t {
+    const uint64_t a0 = a0base + 16ull * c;
+    return c < a.nchunks ? ((a0 >= sg.ptr && a0 < hi_addr ? 1u : 0u) | (a0 + 8 >= sg.ptr && a0 + 8 < hi_addr ? 2u : 0u))
+                         : 0u;
+  };
+  // issue the entry gathers of chunk c (values v) into ring stage st
+  auto issue = [&](uint64_t c, const uint64_t v[2], uint32_t st) {
+    const uint32_t valid = valid_of(c);
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const PdFront f = pd_front(PD, v[m], ((valid >> m) & 1) && v[m] != 0);
+      if (f.ok) {
+        const uint32_t d = my + st * sstride + m * mstride;
+        const uint32_t *src = a.pd.ent + 8 * f.e;
+        cp_async16(d, src, pol_t);
+        cp_async16(d + 16, src + 4, pol_t);
+      }
+    }
+    cp_async_commit();
+  };
+
+  const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  uint64_t cv[2] = {0, 0}, nv[2] = {0, 0}, nnv[2] = {0, 0};
+  if (c_first < a.nchunks) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c_first), pol_s, cv[0], cv[1]);
+  if (c_first + stride < a.nchunks)
+    ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, nv[0], nv[1]);
+  issue(c_first, cv, 0);
+  uint32_t stage = 0;
+  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
+    const uint64_t c = cb + lane;
+    const bool live = c < a.nchunks;
+    // pipeline: values of chunk t+2 into registers, entries of chunk t+1 into the ring
+    if (c + 2 * stride < a.nchunks)
+      ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, nnv[0], nnv[1]);
+    issue(c + stride, nv, stage ^ 1u);
+    cp_async_wait<1>();  // this chunk's entries have landed
+
+    const uint64_t a0 = a0base + 16ull * c;
+    const uint32_t valid = valid_of(c);
+    const int64_t slot0 = ((int64_t)(a0 - sg.ptr)) >> 3;
+    int j[2];
+    uint64_t key[2], hw[2] = {0, 0};
+    bool look[2], k0[2];
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      look[m] = ((valid >> m) & 1) && cv[m] != 0;
+      const PdFront f = pd_front(PD, cv[m], look[m]);
+      uint64_t w[4] = {0, 0, 0, 0};
+      if (f.ok) lds_sector(my + stage * sstride + m * mstride, w);
+      pd_back(a.pd, pol_t, f, cv[m], w, j[m], key[m], k0[m]);
+      look[m] = look[m] && j[m] >= 0;
+      if (look[m]) hw[m] = ld_u64(a.tab.hot + j[m], pol_t);
+    }
+    bool hit[2];
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      uint64_t sz = hot_size32(hw[m]);
+      if (look[m] && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
+      hit[m] = look[m] && (k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
+    }
+    if (SH && live) {  // forward-map shadow: (CPU pointer, unit) per slot for the reverse pass
+      uint64_t *shp = reinterpret_cast<uint64_t *>(sg.shadow);
+      uint32_t *shu = reinterpret_cast<uint32_t *>(sg.shadow + 8 * sg.n);
+      const uint32_t u0 = hit[0] ? (uint32_t)j[0] : 0xFFFFFFFFu, u1 = hit[1] ? (uint32_t)j[1] : 0xFFFFFFFFu;
+      if (valid == 3u && !(slot0 & 1)) {
+        st_stream2(shp + slot0, pol_s, cv[0], cv[1]);
+        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1,%2}, %3;" ::"l"(shu + slot0), "r"(u0),
+                     "r"(u1), "l"(pol_s)
+                     : "memory");
+      } else {
+#pragma unroll
+        for (int m = 0; m < 2; ++m)
+          if ((valid >> m) & 1) {
+            shp[slot0 + m] = cv[m];
+            shu[slot0 + m] = m ? u1 : u0;
+          }
+      }
+    }
+    uint64_t outv[2] = {cv[0], cv[1]};
+    uint32_t wrote = 0;
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const bool vm = (valid >> m) & 1;
+      const bool nul = vm && cv[m] == 0;
+      c_nulls += nul;
+      c_hits += hit[m];
+      c_miss += (vm && !nul && !hit[m]);
+      const uint32_t fl = hot_flags(hw[m]);
+      bool act = false;
+      if (hit[m]) {
+        int32_t *RC = a.tab.rc + j[m];
+        if (fl & UF_ACTIVE) {
+          red_add(RC, sg.inc);
+        } else {
+          act = atomicAdd(RC, sg.inc) == 0;  // refcount 0 -> 1: Alg. 1's activation
+        }
+        if (fl & UF_STORAGE) {
+          const uint32_t e = hot_ext(hw[m]);
+          outv[m] = cv[m] + (ext_s ? s_ext[e] : a.tab.ext_delta[e]);  // Alg. 1: devptr + (ptr - base)
+          wrote |= 1u << m;
+        } else {
+          c_pend += 1;  // activated by this call: completed after the allocation
+        }
+      }
+      const unsigned long long ix = warp_append(&a.lc[0], act);
+      if (act) a.act_list[ix] = (uint32_t)j[m];
+    }
+    c_tr += __popc(wrote);
+    if (live) {
+      if (wrote == 3u) {
+        st_stream2(reinterpret_cast<void *>(a0), pol_s, outv[0], outv[1]);
+      } else {
+#pragma unroll
+        for (int m = 0; m < 2; ++m)
+          if ((wrote >> m) & 1) st_stream1(reinterpret_cast<void *>(a0 + 8ull * m), pol_s, outv[m]);
+      }
+    }
+    {  // hit mask: 2 bits per chunk
+      const unsigned b0 = __ballot_sync(0xffffffffu, wrote & 1u), b1 = __ballot_sync(0xffffffffu, (wrote >> 1) & 1u);
+      if (lane == 0) {
+        const uint32_t w0 = spread16(b0) | (spread16(b1) << 1);
+        const uint32_t w1 = spread16(b0 >> 16) | (spread16(b1 >> 16) << 1);
+        const uint64_t wi = cb >> 4;
+        a.hitmask[wi] = w0;
+        if (cb + 16 < a.nchunks) a.hitmask[wi + 1] = w1;
+      }
+    }
+    cv[0] = nv[0];
+    cv[1] = nv[1];
+    nv[0] = nnv[0];
+    nv[1] = nnv[1];
+    stage ^= 1u;
+  }
+  cp_async_wait<0>();
+  flush_count(&a.st->nulls, c_nulls);
+  flush_count(&a.st->hits, c_hits);
+  flush_count(&a.st->misses, c_miss);
+  flush_count(&a.st->pending, c_pend);
+  flush_count(&a.st->translated, c_tr);
+}
+
+template <int SH>
+static int launch_map_pd(const SlotArgs &a, int nsm, cudaStream_t s) {
+  const size_t smem = pd_stage_bytes(a.pd) + (a.tab.n_ext <= EXT_SMEM ? al16(8 * (size_t)a.tab.n_ext) : 0) +
+                      2ull * 2 * 32 * MAP_PD_THREADS;
+  static bool configured = false;
+  if (!configured) {
+    int dev = 0, optin = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    cudaError_t e = cudaFuncSetAttribute(k_map_pd<SH>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    if (e != cudaSuccess) return (int)e;
+    configured = true;
+  }
+  const uint64_t want = (a.nchunks + MAP_PD_THREADS - 1) / MAP_PD_THREADS;
+  const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
+  (void)cudaGetLastError();
+  k_map_pd<SH><<<grid, MAP_PD_THREADS, smem, s>>>(a);
+  return (int)cudaGetLastError();
+}
+
+// -------------------------------------------------------------------------------------------------
+// k_unmap_sh: unmapArray (+ releaseArray) of one in-place segment whose forward map recorded a shadow
+// (a3 + a4 + Alg. 3 over the slots; R13-ii: an unchanged slot reverses to its recorded CPU pointer).
+// Software-pipelined: the slot values and shadow of chunk t+2 stream into registers and the units'
+// state words of chunk t+1 are gathered while chunk t is decided.  A slot whose shadow check fails
+// (modified since the map, or not translated by it) is marked in the slow mask and left to
+// k_slots<DIR_REV, OPS> with SEL_SLOW, launched right after (it returns at once when none is).
+// Same results, counters and lists as k_slots<DIR_REV, OPS>.
+// -------------------------------------------------------------------------------------------------
+constexpr int UNMAP_SH_THREADS = 768;
+
+template <int OPS>
+__global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const bool ext_s = a.tab.n_ext <= EXT_SMEM;
+  uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
+  if (ext_s)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
+  __syncthreads();
+
+  const uint64_t pol_s = policy_evict_first();
+  const uint64_t pol_t = policy_evict_last();
+  const int lane = threadIdx.x & 31;
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull, hi_addr = sg.ptr + 8ull * sg.n;
+  const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);
+  const uint32_t *shu = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n);
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned c_nulls = 0, c_hits = 0, c_tr = 0, c_under = 0, c_slow = 0;
+
+  auto valid_of = [&](uint64_t c) -> uint32_t {
+    const uint64_t a0 = a0base + 16ull * c;
+    return c < a.nchunks ? ((a0 >= sg.ptr && a0 < hi_addr ? 1u : 0u) | (a0 + 8 >= sg.ptr && a0 + 8 < hi_addr ? 2u : 0u))
+                         : 0u;
+  };
+  // the streams of chunk c: slot values, recorded CPU pointers and units
+  struct In {
+    uint64_t g[2], h[2];
+    uint32_t u[2];
+  };
+  auto load_in = [&](uint64_t c, In &x) {
+    const uint32_t valid = valid_of(c);
+    x.g[0] = x.g[1] = x.h[0] = x.h[1] = 0;
+    x.u[0] = x.u[1] = 0xFFFFFFFFu;
+    if (!valid) return;
+    const uint64_t a0 = a0base + 16ull * c;
+    ld_stream2(reinterpret_cast<const void *>(a0), pol_s, x.g[0], x.g[1]);
+    const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
+    if (valid == 3u && !(i0 & 1)) {
+      ld_stream2(shp + i0, pol_s, x.h[0], x.h[1]);
+      asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
+                   : "=r"(x.u[0]), "=r"(x.u[1])
+                   : "l"(shu + i0), "l"(pol_s));
+    } else {
+#pragma unroll
+      for (int m = 0; m < 2; ++m)
+        if ((valid >> m) & 1) {
+          x.h[m] = shp[i0 + m];
+          x.u[m] = shu[i0 + m];
+        }
+    }
+  };
+  // the state words (epoch | extent | flags) of the recorded units of x
+  auto gather = [&](const In &x, uint64_t w[2]) {
+#pragma unroll
+    for (int m = 0; m < 2; ++m) w[m] = (x.u[m] != 0xFFFFFFFFu && x.g[m] != 0) ? ld_u64(a.tab.st + x.u[m], pol_t) : 0ull;
+  };
+
+  const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  In cur, nxt, nn;
+  uint64_t cw[2], nw[2];
+  load_in(c_first, cur);
+  load_in(c_first + stride, nxt);
+  gather(cur, cw);
+  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
+    const uint64_t c = cb + lane;
+    const bool live = c < a.nchunks;
+    load_in(c + 2 * stride, nn);
+    gather(nxt, nw);
+
+    const uint64_t a0 = a0base + 16ull * c;
+    const uint32_t valid = valid_of(c);
+    bool hit[2], slow[2];
+    uint64_t outv[2] = {cur.g[0], cur.g[1]};
+    uint32_t wrote = 0;
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const bool vm = (valid >> m) & 1;
+      const bool look = vm && cur.g[m] != 0;
+      const uint64_t w = cw[m];
+      const uint32_t e = hot_ext(w);
+      hit[m] = look && cur.u[m] != 0xFFFFFFFFu && (hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext &&
+               cur.g[m] == cur.h[m] + (ext_s ? s_ext[e] : a.tab.ext_delta[e]);
+      slow[m] = look && !hit[m];
+      c_nulls += vm && cur.g[m] == 0;
+      c_hits += hit[m];
+      const uint32_t unit = hit[m] ? cur.u[m] : 0u;
+      const uint32_t fl = hot_flags(w);
+      int32_t *RC = a.tab.rc + unit;
+      bool freed = false;
+      if (OPS & OP_DEC) {
+        if (hit[m]) {
+          if (a.dec_red) {
+            red_add(RC, -sg.inc);
+          } else {
+            const int old = atomicAdd(RC, -sg.inc);
+            c_under += (old < sg.inc);
+            freed = (old == sg.inc);  // refcount 1 -> 0: Alg. 3's cuMemFree
+          }
+        }
+      }
+      bool gated = false;
+      uint32_t old_ep = 0;
+      const uint32_t ep = st_epoch(w);
+      if (hit[m] && a.no_journal && (fl & UF_READONLY)) {
+        if (ep != a.epoch) *lo_word(a.tab.st + unit) = a.epoch;  // Alg. 2 line 3, read-only unit
+      } else if (hit[m] && ep != a.epoch) {
+        old_ep = atomicExch(lo_word(a.tab.st + unit), a.epoch);
+        gated = (old_ep != a.epoch);
+      }
+      if (hit[m]) {
+        outv[m] = cur.h[m];  // reverse: base + (g - devbase), the recorded CPU pointer
+        wrote |= 1u << m;
+      }
+      if (OPS & OP_DEC) {
+        if (!a.dec_red) {
+          const unsigned long long ix = warp_append(&a.lc[2], freed);
+          if (freed) a.free_list[ix] = unit;
+        }
+      }
+      const bool jg = gated && !a.no_journal;
+      const unsigned long long ix = warp_append(&a.lc[1], jg);
+      const bool cp = gated && !(fl & UF_READONLY);  // Alg. 2: stale and not read-only
+      if (jg) {
+        Journal jn;
+        jn.old_epoch = old_ep;
+        jn.unit = unit;
+        jn.copy = cp ? 1u : 0u;
+        jn.pad = 0;
+        a.journal[ix] = jn;
+      }
+      const unsigned long long cx = warp_append(&a.lc[3], cp);
+      if (cp) a.copy_list[cx] = unit;
+    }
+    c_tr += __popc(wrote);
+    c_slow += slow[0] + slow[1];
+    if (live) {
+      if (wrote == 3u) {
+        st_stream2(reinterpret_cast<void *>(a0), pol_s, outv[0], outv[1]);
+      } else {
+#pragma unroll
+        for (int m = 0; m < 2; ++m)
+          if ((wrote >> m) & 1) st_stream1(reinterpret_cast<void *>(a0 + 8ull * m), pol_s, outv[m]);
+      }
+    }
+    {  // hit and slow masks: 2 bits per chunk
+      const unsigned b0 = __ballot_sync(0xffffffffu, wrote & 1u), b1 = __ballot_sync(0xffffffffu, (wrote >> 1) & 1u);
+      const unsigned s0 = __ballot_sync(0xffffffffu, slow[0]), s1 = __ballot_sync(0xffffffffu, slow[1]);
+      if (lane == 0) {
+        const uint64_t wi = cb >> 4;
+        a.hitmask[wi] = spread16(b0) | (spread16(b1) << 1);
+        a.slowmask[wi] = spread16(s0) | (spread16(s1) << 1);
+        if (cb + 16 < a.nchunks) {
+          a.hitmask[wi + 1] = spread16(b0 >> 16) | (spread16(b1 >> 16) << 1);
+          a.slowmask[wi + 1] = spread16(s0 >> 16) | (spread16(s1 >> 16) << 1);
+        }
+      }
+    }
+    cur = nxt;
+    nxt = nn;
+    cw[0] = nw[0];
+    cw[1] = nw[1];
+  }
+  flush_count(&a.st->nulls, c_nulls);
+  flush_count(&a.st->hits, c_hits);
+  flush_count(&a.st->translated, c_tr);
+  flush_count(a.slowcount, c_slow);
+  if (OPS & OP_DEC) flush_count(&a.st->underflow, c_under);
+}
+
+template <int OPS>
+static int launch_unmap_sh(const SlotArgs &a, int nsm, cudaStream_t s) {
+  const size_t smem = (a.tab.n_ext <= EXT_SMEM ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
+  static bool configured = false;
+  if (!configured) {
+    int dev = 0, optin = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    cudaError_t e = cudaFuncSetAttribute(k_unmap_sh<OPS>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    if (e != cudaSuccess) return (int)e;
+    configured = true;
+  }
+  const uint64_t want = (a.nchunks + UNMAP_SH_THREADS - 1) / UNMAP_SH_THREADS;
+  const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
+  (void)cudaGetLastError();
+  k_unmap_sh<OPS><<<grid, UNMAP_SH_THREADS, smem, s>>>(a);
+  return (int)cudaGetLastError();
 }
 
 // the operation sets the runtime uses
@@ -842,7 +1338,24 @@ static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
   X(DIR_REV, OP_WRITE | OP_GATE | OP_DEC | OP_HITMASK) \
   X(DIR_REV, OP_WRITE | OP_GATE | OP_HITMASK)
 
-int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s) {
+int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, int *nlaunch) {
+  *nlaunch = 1;
+  static const bool no_pipe = std::getenv("CGCM_NO_PIPELINE") != nullptr;  // A/B experiments
+  if (dir == DIR_FWD && ops == (OP_WRITE | OP_INC | OP_HITMASK) && a.pd.nseg > 0 && a.nseg == 1 && a.seg_inplace &&
+      a.sel == SEL_ALL && !no_pipe)
+    return a.segs_host_shadow ? launch_map_pd<1>(a, nsm, s) : launch_map_pd<0>(a, nsm, s);
+  constexpr int UNMAP = OP_WRITE | OP_GATE | OP_HITMASK, UNMAP_REL = OP_WRITE | OP_GATE | OP_DEC | OP_HITMASK;
+  if (dir == DIR_REV && (ops == UNMAP || ops == UNMAP_REL) && a.nseg == 1 && a.seg_inplace && a.segs_host_shadow &&
+      a.sel == SEL_ALL && !no_pipe) {
+    // pipelined pass over the recorded slots, then the generic kernel over the slots it left
+    if (cudaMemsetAsync(a.slowcount, 0, sizeof(unsigned long long), s) != cudaSuccess) return (int)cudaGetLastError();
+    int r = ops == UNMAP ? launch_unmap_sh<UNMAP>(a, nsm, s) : launch_unmap_sh<UNMAP_REL>(a, nsm, s);
+    if (r != 0) return r;
+    SlotArgs b = a;
+    b.sel = SEL_SLOW;
+    *nlaunch = 2;
+    return launch_slots(dir, ops, b, nsm, s, &r);
+  }
   // the forward index qualifies for the specialised path: one segment, no wide bucket, h <= 3
   int fh = a.pd.nseg > 0 ? FH_PD : a.fx.nseg <= 1 && a.fx_nowide && a.fx.h <= 3 ? a.fx.h : -1;
   const bool sh = a.nseg == 1 && a.segs_host_shadow;

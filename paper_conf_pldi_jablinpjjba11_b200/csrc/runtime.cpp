@@ -219,6 +219,7 @@ struct Context {
   uint32_t pd_minP = 0, pd_maxP = 0;
 
   // scratch
+  DevBuf slowmask, slowcnt;
   DevBuf status, lc, hitmask, act_list, journal, free_list, copy_list, segs, seg0, staging, staging2, staging_cb, points, ptrs, temp;
   DevBuf up_units, up_vals, up_exts, uops;
   HostBuf h_small, h_status, h_list, h_pack[2];
@@ -400,7 +401,8 @@ struct Context {
     pd_nseg = 0;
     pd_pages = pd_ovf_pages = pd_bytes = 0;
     pd_minP = pd_maxP = 0;
-    if (n == 0 || (flags & CGCM_NO_PAGEDIR)) return CGCM_OK;
+    static const bool env_off = std::getenv("CGCM_NO_PAGEDIR") != nullptr;  // A/B experiments
+    if (n == 0 || (flags & CGCM_NO_PAGEDIR) || env_off) return CGCM_OK;
     static const double ovf_frac = [] {
       const char *e = std::getenv("CGCM_PD_OVF");
       return e ? std::atof(e) : 0.01;
@@ -656,6 +658,8 @@ struct Context {
     c.nchunks = c0[k];
     if (c.nchunks == 0) return CGCM_OK;
     if ((c.ops & OP_HITMASK) || c.sel != SEL_ALL) CKS(dalloc(hitmask, 4 * (size_t)(c.nchunks / 16 + 4)));
+    if (c.dir == DIR_REV && k == 1 && c.segs[0].shadow) CKS(dalloc(slowmask, 4 * (size_t)(c.nchunks / 16 + 4)));
+    CKS(dalloc(slowcnt, 64));
     CKS(dalloc(segs, sizeof(Seg) * (size_t)k * 4 + 256));
     CKS(dalloc(seg0, 8 * (size_t)(k + 1) * 4 + 256));
     // each launch uses its own quarter of the segment buffers (up to 4 launches in flight)
@@ -677,11 +681,14 @@ struct Context {
     }
     a.segs = dsegs;
     a.segs_host_shadow = (k == 1 && c.segs[0].shadow != 0) ? 1 : 0;
+    a.seg_inplace = (k == 1 && c.segs[0].out == 0) ? 1 : 0;
     a.seg_chunk0 = dc0;
     a.nseg = k;
     a.sel = c.sel;
     a.nchunks = c.nchunks;
     a.hitmask = hitmask.as<uint32_t>();
+    a.slowmask = slowmask.as<uint32_t>();
+    a.slowcount = slowcnt.as<unsigned long long>();
     a.dec_red = c.dec_red ? 1 : 0;
     a.no_journal = c.no_journal ? 1 : 0;
     a.epoch = rel_epoch(epoch);
@@ -694,7 +701,8 @@ struct Context {
     a.lenient = (flags & CGCM_LENIENT) ? 1 : 0;
     bool timed = (flags & CGCM_PROFILE) && (timed_fwd || timed_rev);
     if (timed) CK(cudaEventRecord(ev_t0, main));
-    int r = launch_slots(c.dir, c.ops, a, nsm, main);
+    int nl = 0;
+    int r = launch_slots(c.dir, c.ops, a, nsm, main, &nl);
     if (r != 0) {
       g_last_cuda_error = r == -2 ? std::string("unsupported slot-kernel operation set")
                                   : std::string("k_slots launch (dir ") + std::to_string(c.dir) + ", ops " +
@@ -703,7 +711,7 @@ struct Context {
       return CGCM_E_CUDA;
     }
     CK(cudaGetLastError());
-    st.kernel_launches += 1;
+    st.kernel_launches += (uint64_t)nl;
     if ((c.ops & OP_DEC) && c.dec_red) {  // underflow / 1 -> 0 detection after reductions
       launch_release_scan(tab(), U, status.as<Status>() + st_index, lc.as<unsigned long long>(),
                           free_list.as<uint32_t>(), main);
