@@ -884,7 +884,11 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
 // the unit's hot word) thus overlap those of the next.  Same results, counters and lists as
 // k_slots<DIR_FWD, OP_WRITE | OP_INC | OP_HITMASK> (which serves every other case).
 // -------------------------------------------------------------------------------------------------
+#ifdef CGCM_MAP_PD_THREADS
+constexpr int MAP_PD_THREADS = CGCM_MAP_PD_THREADS;
+#else
 constexpr int MAP_PD_THREADS = 768;
+#endif
 
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, uint64_t pol) {
   asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "l"(pol)

@@ -1365,6 +1365,12 @@ int cgcm_init(int device, void *dev_arena, size_t arena_bytes, void *main_stream
   C->flags = flags;
   int nsm = 0;
   if (cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, device) == cudaSuccess && nsm > 0) C->nsm = nsm;
+  if (const char *e = std::getenv("CGCM_L2_FETCH")) {  // A/B experiments: L2 fetch granularity (bytes)
+    size_t want = (size_t)std::atoi(e), got = 0;
+    cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, want);
+    cudaDeviceGetLimit(&got, cudaLimitMaxL2FetchGranularity);
+    std::fprintf(stderr, "cgcm: L2 fetch granularity %zu (asked %zu)\n", got, want);
+  }
   if (!dev_arena) {
     if (cudaMalloc(&C->own_arena, arena_bytes) != cudaSuccess) {
       delete C;

@@ -90,3 +90,16 @@ def test_python_binding_requires_cuda():
         pytest.skip("GPU present")
     with pytest.raises(cg.CgcmError):
         cg.Context(0, arena_bytes=1 << 20)
+
+
+def test_sass_has_no_odd_uniform_descriptor_pairs(built):
+    """ptxas 12.9 once encoded a cp.async cache-policy descriptor as desc[UR1] (an odd uniform-register
+    pair), an illegal instruction at run time (k_map_pd3's prologue).  Guard the build against it."""
+    import shutil
+    so = os.path.join(PKG, "libcgcm.so")
+    if not shutil.which("cuobjdump") or not os.path.exists(so):
+        pytest.skip("cuobjdump or libcgcm.so missing")
+    sass = subprocess.run(["cuobjdump", "-sass", so], capture_output=True, text=True).stdout
+    bad = [ln.strip() for ln in sass.splitlines() if re.search(r"desc\[UR([0-9]+)\]", ln)
+           and int(re.search(r"desc\[UR([0-9]+)\]", ln).group(1)) % 2]
+    assert not bad, bad[:4]
