@@ -177,6 +177,7 @@ struct SlotArgs {
   const uint64_t *seg_chunk0;  // [nseg+1] prefix of 2-slot chunks per segment
   int nseg;
   int sel;
+  uint64_t cbeg;               // chunks [cbeg, nchunks) of the call (a piece: multiple of 32), k_slots only
   uint64_t nchunks;
   uint32_t *hitmask;           // 2 bits per chunk: slot m of the chunk was translated
   uint32_t *slowmask;          // 2 bits per chunk: left to the generic kernel by k_unmap_sh

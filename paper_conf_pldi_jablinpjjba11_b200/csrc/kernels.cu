@@ -548,10 +548,10 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
   const bool pf = a.nseg == 1;
   uint64_t nv0 = 0, nv1 = 0;
   {
-    const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t c = a.cbeg + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (pf && c < a.nchunks) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c), pol_s, nv0, nv1);
   }
-  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
+  for (uint64_t cb = a.cbeg + (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
     const uint64_t c = cb + lane;
     const bool live = c < a.nchunks;
     const uint64_t cv0 = nv0, cv1 = nv1;
@@ -1329,7 +1329,7 @@ static int launch_one(const SlotArgs &a, int nsm, cudaStream_t s) {
     configured = true;
   }
   constexpr int T = SlotCfg<DIR, SH>::threads;
-  uint64_t want = (a.nchunks + T - 1) / T;
+  uint64_t want = (a.nchunks - a.cbeg + T - 1) / T;
   int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
   k_slots<DIR, OPS, FH, SH><<<grid, T, smem, s>>>(a);
@@ -1346,11 +1346,11 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, i
   *nlaunch = 1;
   static const bool no_pipe = std::getenv("CGCM_NO_PIPELINE") != nullptr;  // A/B experiments
   if (dir == DIR_FWD && ops == (OP_WRITE | OP_INC | OP_HITMASK) && a.pd.nseg > 0 && a.nseg == 1 && a.seg_inplace &&
-      a.sel == SEL_ALL && !no_pipe)
+      a.sel == SEL_ALL && a.cbeg == 0 && !no_pipe)
     return a.segs_host_shadow ? launch_map_pd<1>(a, nsm, s) : launch_map_pd<0>(a, nsm, s);
   constexpr int UNMAP = OP_WRITE | OP_GATE | OP_HITMASK, UNMAP_REL = OP_WRITE | OP_GATE | OP_DEC | OP_HITMASK;
   if (dir == DIR_REV && (ops == UNMAP || ops == UNMAP_REL) && a.nseg == 1 && a.seg_inplace && a.segs_host_shadow &&
-      a.sel == SEL_ALL && !no_pipe) {
+      a.sel == SEL_ALL && a.cbeg == 0 && !no_pipe) {
     // pipelined pass over the recorded slots, then the generic kernel over the slots it left
     if (cudaMemsetAsync(a.slowcount, 0, sizeof(unsigned long long), s) != cudaSuccess) return (int)cudaGetLastError();
     int r = ops == UNMAP ? launch_unmap_sh<UNMAP>(a, nsm, s) : launch_unmap_sh<UNMAP_REL>(a, nsm, s);

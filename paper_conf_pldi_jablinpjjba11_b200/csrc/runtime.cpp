@@ -636,6 +636,10 @@ struct Context {
     std::vector<Seg> segs;
     uint64_t nchunks = 0;
     Status res{};
+    // transfer overlap (mapArrays): segs are ordered by group (nondecreasing, -1 first); the chunks of
+    // group g are translated by a launch that waits for group_ev[g] (the H2D copy of their extent)
+    std::vector<int> seg_group;
+    std::vector<cudaEvent_t> group_ev;
   };
 
   int list_capacity() const { return std::max(U, 1); }
@@ -660,9 +664,9 @@ struct Context {
     if ((c.ops & OP_HITMASK) || c.sel != SEL_ALL) CKS(dalloc(hitmask, 4 * (size_t)(c.nchunks / 16 + 4)));
     if (c.dir == DIR_REV && k == 1 && c.segs[0].shadow) CKS(dalloc(slowmask, 4 * (size_t)(c.nchunks / 16 + 4)));
     CKS(dalloc(slowcnt, 64));
-    CKS(dalloc(segs, sizeof(Seg) * (size_t)k * 4 + 256));
-    CKS(dalloc(seg0, 8 * (size_t)(k + 1) * 4 + 256));
-    // each launch uses its own quarter of the segment buffers (up to 4 launches in flight)
+    CKS(dalloc(segs, sizeof(Seg) * (size_t)k * 8 + 256));
+    CKS(dalloc(seg0, 8 * (size_t)(k + 1) * 8 + 256));
+    // each launch uses its own eighth of the segment buffers (st_index 0..7, up to 8 launches in flight)
     Seg *dsegs = segs.as<Seg>() + (size_t)st_index * k;
     uint64_t *dc0 = seg0.as<uint64_t>() + (size_t)st_index * (k + 1);
     CK(cudaMemcpyAsync(dsegs, c.segs.data(), sizeof(Seg) * k, cudaMemcpyHostToDevice, main));
@@ -699,10 +703,37 @@ struct Context {
     a.copy_list = copy_list.as<uint32_t>();
     a.free_list = free_list.as<uint32_t>();
     a.lenient = (flags & CGCM_LENIENT) ? 1 : 0;
-    bool timed = (flags & CGCM_PROFILE) && (timed_fwd || timed_rev);
+    const bool pieces = !c.seg_group.empty();
+    bool timed = (flags & CGCM_PROFILE) && (timed_fwd || timed_rev) && !pieces;
     if (timed) CK(cudaEventRecord(ev_t0, main));
     int nl = 0;
-    int r = launch_slots(c.dir, c.ops, a, nsm, main, &nl);
+    int r = 0;
+    if (!pieces) {
+      r = launch_slots(c.dir, c.ops, a, nsm, main, &nl);
+    } else {
+      // one launch per copy group, each after its group's H2D copy: translation of the extents that
+      // have arrived overlaps the copies still in flight.  Piece boundaries are multiples of 32 chunks
+      // (one warp's hit-mask words); chunks of group g below the boundary ride with group g + 1,
+      // whose copy is issued after g's on the same stream.
+      uint64_t cb = 0;
+      for (int s0 = 0; s0 < k && r == 0;) {
+        const int g = c.seg_group[s0];
+        int s1 = s0;
+        while (s1 < k && c.seg_group[s1] == g) ++s1;
+        const uint64_t ce = s1 < k ? (c0[s1] & ~31ull) : c.nchunks;
+        if (g >= 0) CK(cudaStreamWaitEvent(main, c.group_ev[g], 0));
+        if (ce > cb) {
+          SlotArgs b = a;
+          b.cbeg = cb;
+          b.nchunks = ce;
+          int n1 = 0;
+          r = launch_slots(c.dir, c.ops, b, nsm, main, &n1);
+          nl += n1;
+          cb = ce;
+        }
+        s0 = s1;
+      }
+    }
     if (r != 0) {
       g_last_cuda_error = r == -2 ? std::string("unsupported slot-kernel operation set")
                                   : std::string("k_slots launch (dir ") + std::to_string(c.dir) + ", ops " +
@@ -825,7 +856,20 @@ struct Context {
   // has >= 1 byte of slack at its end.  One delta (host - device) per extent is what the reverse
   // index stores.  A host-contiguous extent of >= 256 KiB is one direct DMA; any other extent is
   // gathered on the host into pinned staging (multithreaded) and sent as one DMA.
-  int activate_units(const std::vector<uint32_t> &units, std::vector<std::pair<uint64_t, uint64_t>> *h2d_out) {
+  std::vector<cudaEvent_t> evpool;  // per-copy-group events (transfer overlap)
+  int pool_event(size_t i, cudaEvent_t &e) {
+    while (evpool.size() <= i) {
+      cudaEvent_t x;
+      CK(cudaEventCreateWithFlags(&x, cudaEventDisableTiming));
+      evpool.push_back(x);
+    }
+    e = evpool[i];
+    return CGCM_OK;
+  }
+  // pack_ev (optional): one event per pack (h2d_out entry), recorded on the copy stream after its copy;
+  // the main stream then does NOT wait for the copies -- the caller waits per pack (transfer overlap)
+  int activate_units(const std::vector<uint32_t> &units, std::vector<std::pair<uint64_t, uint64_t>> *h2d_out,
+                     std::vector<cudaEvent_t> *pack_ev = nullptr) {
     if (units.empty()) return CGCM_OK;
     const uint64_t PACK_SPAN = 64ull << 20, GAPMAX = 64ull << 10, PACK_MIN = 256ull << 10;
     struct Pack {
@@ -898,11 +942,20 @@ struct Context {
     CK(cudaGetLastError());
     CK(cudaEventRecord(ev_copy, main));  // the copies wait for everything the main stream did before
     CK(cudaStreamWaitEvent(copy, ev_copy, 0));
+    auto mark = [&]() -> int {
+      if (!pack_ev) return CGCM_OK;
+      cudaEvent_t e;
+      CKS(pool_event(pack_ev->size(), e));
+      CK(cudaEventRecord(e, copy));
+      pack_ev->push_back(e);
+      return CGCM_OK;
+    };
     for (auto &P : packs) {
       uint64_t span = P.h1 - P.h0;
       if (P.global || (!P.gaps && span >= PACK_MIN)) {
         CKS(copy_run(P.dev0, P.h0, span, true, units, P.i, P.j, copy));
         if (h2d_out) h2d_out->push_back({P.dev0, span});
+        CKS(mark());
         continue;
       }
       int k = pack_k;
@@ -915,9 +968,10 @@ struct Context {
       CK(cudaEventRecord(ev_pack[k], copy));
       st.h2d_memcpy_calls += 1;
       if (h2d_out) h2d_out->push_back({P.dev0, span});
+      CKS(mark());
     }
     CK(cudaEventRecord(ev_copy, copy));
-    CK(cudaStreamWaitEvent(main, ev_copy, 0));
+    if (!pack_ev) CK(cudaStreamWaitEvent(main, ev_copy, 0));
     st.h2d_units += units.size();
     st.h2d_bytes += bytes;
     st.activations += units.size();
@@ -1087,7 +1141,8 @@ struct Context {
   // prelaunch: optional additional REV INCPLAIN segments (array-mapped outers re-mapped, A9).
   // On error everything this function did is undone; the caller undoes its own prologue.
   int map_core(const std::vector<Seg> &fsegs, const std::vector<Seg> &rsegs, uint64_t *translated_out,
-               uint64_t *nulls_out) {
+               uint64_t *nulls_out, const std::vector<int> *seg_group = nullptr,
+               const std::vector<cudaEvent_t> *group_ev = nullptr) {
     uint64_t total = 0;
     for (auto &s : fsegs) total += s.n;
     CKS(prepare(total + 64));
@@ -1095,12 +1150,18 @@ struct Context {
     F.dir = DIR_FWD;
     F.ops = OP_WRITE | OP_INC | OP_HITMASK;
     F.segs = fsegs;
+    if (seg_group && group_ev) {
+      F.seg_group = *seg_group;
+      F.group_ev = *group_ev;
+    }
     SlotCall R;
     R.dir = DIR_REV;
     R.ops = OP_INCPLAIN;
     R.segs = rsegs;
     if (!rsegs.empty()) CKS(ensure_rev());
-    CKS(launch(F, 0, false, true, false));
+    int lr = launch(F, 0, false, true, false);
+    if (!F.seg_group.empty()) CK(cudaStreamWaitEvent(main, ev_copy, 0));  // every copy, whatever happened
+    CKS(lr);
     // hitmask is per launch: the REV pass does not use it
     if (!rsegs.empty()) CKS(launch(R, 1));
     Status sts[8];
@@ -1881,7 +1942,8 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
     if (o.info.refcount == 0) act.push_back((uint32_t)o.unit);
   std::sort(act.begin(), act.end());
   std::vector<std::pair<uint64_t, uint64_t>> copies;
-  CKS(C->activate_units(act, &copies));
+  std::vector<cudaEvent_t> pack_ev;  // transfer overlap: the outers' H2D copies, one event per extent
+  CKS(C->activate_units(act, &copies, &pack_ev));
   std::vector<UnitOp> ops;
   std::vector<Seg> fsegs, rsegs;
   for (auto &o : outs) {
@@ -1897,6 +1959,7 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
   // unit ops must not run before the outers' set_devbase: same stream, issued after
   CKS(C->unit_ops(ops));
   auto undo_prologue = [&]() {
+    cudaStreamSynchronize(C->copy);  // the outers' copies land before their storage is released
     std::vector<UnitOp> undo;
     for (auto &o : outs) {
       undo.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)(-o.mult)});
@@ -1952,8 +2015,32 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
       return r;
     }
   }
+  // translate each outer once its extent has arrived (transfer scheduler: H2D on the copy stream
+  // overlapped with translation on the main stream, one launch per extent)
+  std::vector<int> group(fsegs.size(), -1);
+  for (size_t q = 0; q < fsegs.size(); ++q)
+    for (size_t p = 0; p < copies.size(); ++p)
+      if (fsegs[q].ptr >= copies[p].first && fsegs[q].ptr < copies[p].first + copies[p].second) {
+        group[q] = (int)p;
+        break;
+      }
+  {
+    std::vector<size_t> ord(fsegs.size());
+    for (size_t q = 0; q < ord.size(); ++q) ord[q] = q;
+    std::sort(ord.begin(), ord.end(), [&](size_t x, size_t y) {
+      return group[x] != group[y] ? group[x] < group[y] : fsegs[x].ptr < fsegs[y].ptr;
+    });
+    std::vector<Seg> fs(ord.size());
+    std::vector<int> gs(ord.size());
+    for (size_t q = 0; q < ord.size(); ++q) {
+      fs[q] = fsegs[ord[q]];
+      gs[q] = group[ord[q]];
+    }
+    fsegs.swap(fs);
+    group.swap(gs);
+  }
   uint64_t tr = 0, nl = 0;
-  int r = C->map_core(fsegs, {}, &tr, &nl);
+  int r = C->map_core(fsegs, {}, &tr, &nl, &group, &pack_ev);
   if (r != CGCM_OK) {
     if (rev_done) C->rev_decref(rsegs);
     for (auto &b : backups)
