@@ -1090,54 +1090,80 @@ static int launch_map_pd(const SlotArgs &a, int nsm, cudaStream_t s) {
 }
 
 // -------------------------------------------------------------------------------------------------
-// k_unmap_sh: unmapArray (+ releaseArray) of one in-place segment whose forward map recorded a shadow
-// (a3 + a4 + Alg. 3 over the slots; R13-ii: an unchanged slot reverses to its recorded CPU pointer).
-// Software-pipelined: the slot values and shadow of chunk t+2 stream into registers and the units'
-// state words of chunk t+1 are gathered while chunk t is decided.  A slot whose shadow check fails
-// (modified since the map, or not translated by it) is marked in the slow mask and left to
-// k_slots<DIR_REV, OPS> with SEL_SLOW, launched right after (it returns at once when none is).
-// Same results, counters and lists as k_slots<DIR_REV, OPS>.
+// k_unmap_sh: the reverse pass over slots whose forward map recorded a shadow (R13-ii: an unchanged
+// slot reverses to its recorded CPU pointer): unmapArray (a3 + a4, OPS = WRITE | GATE | HITMASK),
+// fused with releaseArray (| DEC), or releaseArray alone (OPS = DEC).  Any number of segments, in
+// place or out of place.  Software-pipelined: the slot values and shadow of chunk t+2 stream into
+// registers and the units' state words of chunk t+1 are gathered while chunk t is decided.  A slot
+// whose shadow check fails (modified since the map, not translated by it, or in a segment without a
+// shadow) is marked in the slow mask and left to k_slots<DIR_REV, OPS> with SEL_SLOW, launched right
+// after (it returns at once when there is none).  Same results, counters and lists as k_slots.
 // -------------------------------------------------------------------------------------------------
 constexpr int UNMAP_SH_THREADS = 768;
 
 template <int OPS>
 __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ uint64_t s_seg0[SEG_SMEM + 1];
+  __shared__ Seg s_segs[SEG_SMEM];
   const bool ext_s = a.tab.n_ext <= EXT_SMEM;
   uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
   if (ext_s)
     for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
+  const bool seg_s = a.nseg <= SEG_SMEM;
+  if (seg_s) {
+    for (int t = threadIdx.x; t <= a.nseg; t += blockDim.x) s_seg0[t] = a.seg_chunk0[t];
+    for (int t = threadIdx.x; t < a.nseg; t += blockDim.x) s_segs[t] = a.segs[t];
+  }
   __syncthreads();
+  const uint64_t *seg0 = seg_s ? s_seg0 : a.seg_chunk0;
+  const Seg *segs = seg_s ? s_segs : a.segs;
 
   const uint64_t pol_s = policy_evict_first();
   const uint64_t pol_t = policy_evict_last();
   const int lane = threadIdx.x & 31;
-  const Seg sg = a.segs[0];
-  const uint64_t a0base = sg.ptr & ~15ull, hi_addr = sg.ptr + 8ull * sg.n;
-  const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);
-  const uint32_t *shu = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n);
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   unsigned c_nulls = 0, c_hits = 0, c_tr = 0, c_under = 0, c_slow = 0;
 
-  auto valid_of = [&](uint64_t c) -> uint32_t {
-    const uint64_t a0 = a0base + 16ull * c;
-    return c < a.nchunks ? ((a0 >= sg.ptr && a0 < hi_addr ? 1u : 0u) | (a0 + 8 >= sg.ptr && a0 + 8 < hi_addr ? 2u : 0u))
-                         : 0u;
+  // chunk c -> its segment (last s with seg0[s] <= c)
+  auto seg_of = [&](uint64_t c) -> int {
+    if (a.nseg == 1) return 0;
+    int lo = 0, len = a.nseg;
+    while (len > 1) {
+      const int half = len >> 1;
+      if (seg0[lo + half] <= c) lo += half;
+      len -= half;
+    }
+    return lo;
   };
-  // the streams of chunk c: slot values, recorded CPU pointers and units
+  // the streams of one chunk: slot values, recorded CPU pointers and units
   struct In {
+    uint64_t a0;  // address of the chunk's first word (16-byte aligned)
     uint64_t g[2], h[2];
     uint32_t u[2];
+    uint32_t valid;
+    int s;
   };
   auto load_in = [&](uint64_t c, In &x) {
-    const uint32_t valid = valid_of(c);
     x.g[0] = x.g[1] = x.h[0] = x.h[1] = 0;
     x.u[0] = x.u[1] = 0xFFFFFFFFu;
-    if (!valid) return;
-    const uint64_t a0 = a0base + 16ull * c;
+    x.valid = 0;
+    x.s = 0;
+    x.a0 = 0;
+    if (c >= a.nchunks) return;
+    const int s = seg_of(c);
+    const Seg &sg = segs[s];
+    const uint64_t a0 = (sg.ptr & ~15ull) + 16ull * (c - seg0[s]), hi = sg.ptr + 8ull * sg.n;
+    x.s = s;
+    x.a0 = a0;
+    x.valid = (a0 >= sg.ptr && a0 < hi ? 1u : 0u) | (a0 + 8 >= sg.ptr && a0 + 8 < hi ? 2u : 0u);
+    if (!x.valid) return;
     ld_stream2(reinterpret_cast<const void *>(a0), pol_s, x.g[0], x.g[1]);
+    if (!sg.shadow) return;
+    const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);
+    const uint32_t *shu = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n);
     const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
-    if (valid == 3u && !(i0 & 1)) {
+    if (x.valid == 3u && !(i0 & 1)) {
       ld_stream2(shp + i0, pol_s, x.h[0], x.h[1]);
       asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
                    : "=r"(x.u[0]), "=r"(x.u[1])
@@ -1145,7 +1171,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
     } else {
 #pragma unroll
       for (int m = 0; m < 2; ++m)
-        if ((valid >> m) & 1) {
+        if ((x.valid >> m) & 1) {
           x.h[m] = shp[i0 + m];
           x.u[m] = shu[i0 + m];
         }
@@ -1164,13 +1190,11 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   load_in(c_first + stride, nxt);
   gather(cur, cw);
   for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
-    const uint64_t c = cb + lane;
-    const bool live = c < a.nchunks;
-    load_in(c + 2 * stride, nn);
+    load_in(cb + lane + 2 * stride, nn);
     gather(nxt, nw);
 
-    const uint64_t a0 = a0base + 16ull * c;
-    const uint32_t valid = valid_of(c);
+    const uint32_t valid = cur.valid;
+    const Seg &sg = segs[cur.s];
     bool hit[2], slow[2];
     uint64_t outv[2] = {cur.g[0], cur.g[1]};
     uint32_t wrote = 0;
@@ -1199,60 +1223,71 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
             freed = (old == sg.inc);  // refcount 1 -> 0: Alg. 3's cuMemFree
           }
         }
-      }
-      bool gated = false;
-      uint32_t old_ep = 0;
-      const uint32_t ep = st_epoch(w);
-      if (hit[m] && a.no_journal && (fl & UF_READONLY)) {
-        if (ep != a.epoch) *lo_word(a.tab.st + unit) = a.epoch;  // Alg. 2 line 3, read-only unit
-      } else if (hit[m] && ep != a.epoch) {
-        old_ep = atomicExch(lo_word(a.tab.st + unit), a.epoch);
-        gated = (old_ep != a.epoch);
-      }
-      if (hit[m]) {
-        outv[m] = cur.h[m];  // reverse: base + (g - devbase), the recorded CPU pointer
-        wrote |= 1u << m;
-      }
-      if (OPS & OP_DEC) {
         if (!a.dec_red) {
           const unsigned long long ix = warp_append(&a.lc[2], freed);
           if (freed) a.free_list[ix] = unit;
         }
       }
-      const bool jg = gated && !a.no_journal;
-      const unsigned long long ix = warp_append(&a.lc[1], jg);
-      const bool cp = gated && !(fl & UF_READONLY);  // Alg. 2: stale and not read-only
-      if (jg) {
-        Journal jn;
-        jn.old_epoch = old_ep;
-        jn.unit = unit;
-        jn.copy = cp ? 1u : 0u;
-        jn.pad = 0;
-        a.journal[ix] = jn;
+      if (OPS & OP_GATE) {
+        bool gated = false;
+        uint32_t old_ep = 0;
+        const uint32_t ep = st_epoch(w);
+        if (hit[m] && a.no_journal && (fl & UF_READONLY)) {
+          if (ep != a.epoch) *lo_word(a.tab.st + unit) = a.epoch;  // Alg. 2 line 3, read-only unit
+        } else if (hit[m] && ep != a.epoch) {
+          old_ep = atomicExch(lo_word(a.tab.st + unit), a.epoch);
+          gated = (old_ep != a.epoch);
+        }
+        const bool jg = gated && !a.no_journal;
+        const unsigned long long ix = warp_append(&a.lc[1], jg);
+        const bool cp = gated && !(fl & UF_READONLY);  // Alg. 2: stale and not read-only
+        if (jg) {
+          Journal jn;
+          jn.old_epoch = old_ep;
+          jn.unit = unit;
+          jn.copy = cp ? 1u : 0u;
+          jn.pad = 0;
+          a.journal[ix] = jn;
+        }
+        const unsigned long long cx = warp_append(&a.lc[3], cp);
+        if (cp) a.copy_list[cx] = unit;
       }
-      const unsigned long long cx = warp_append(&a.lc[3], cp);
-      if (cp) a.copy_list[cx] = unit;
+      if ((OPS & OP_WRITE) && hit[m]) {
+        outv[m] = cur.h[m];  // reverse: base + (g - devbase), the recorded CPU pointer
+        wrote |= 1u << m;
+      }
     }
     c_tr += __popc(wrote);
     c_slow += slow[0] + slow[1];
-    if (live) {
-      if (wrote == 3u) {
-        st_stream2(reinterpret_cast<void *>(a0), pol_s, outv[0], outv[1]);
-      } else {
+    if (OPS & OP_WRITE) {
+      if (sg.out == 0) {
+        if (wrote == 3u) {
+          st_stream2(reinterpret_cast<void *>(cur.a0), pol_s, outv[0], outv[1]);
+        } else {
+#pragma unroll
+          for (int m = 0; m < 2; ++m)
+            if ((wrote >> m) & 1) st_stream1(reinterpret_cast<void *>(cur.a0 + 8ull * m), pol_s, outv[m]);
+        }
+      } else {  // out of place: NULL slots are copied verbatim, slow slots are left to the generic pass
 #pragma unroll
         for (int m = 0; m < 2; ++m)
-          if ((wrote >> m) & 1) st_stream1(reinterpret_cast<void *>(a0 + 8ull * m), pol_s, outv[m]);
+          if (((valid >> m) & 1) && !slow[m])
+            st_stream1(reinterpret_cast<void *>(sg.out + (cur.a0 + 8ull * m - sg.ptr)), pol_s, outv[m]);
       }
     }
     {  // hit and slow masks: 2 bits per chunk
-      const unsigned b0 = __ballot_sync(0xffffffffu, wrote & 1u), b1 = __ballot_sync(0xffffffffu, (wrote >> 1) & 1u);
       const unsigned s0 = __ballot_sync(0xffffffffu, slow[0]), s1 = __ballot_sync(0xffffffffu, slow[1]);
+      unsigned b0 = 0, b1 = 0;
+      if (OPS & OP_HITMASK) {
+        b0 = __ballot_sync(0xffffffffu, wrote & 1u);
+        b1 = __ballot_sync(0xffffffffu, (wrote >> 1) & 1u);
+      }
       if (lane == 0) {
         const uint64_t wi = cb >> 4;
-        a.hitmask[wi] = spread16(b0) | (spread16(b1) << 1);
+        if (OPS & OP_HITMASK) a.hitmask[wi] = spread16(b0) | (spread16(b1) << 1);
         a.slowmask[wi] = spread16(s0) | (spread16(s1) << 1);
         if (cb + 16 < a.nchunks) {
-          a.hitmask[wi + 1] = spread16(b0 >> 16) | (spread16(b1 >> 16) << 1);
+          if (OPS & OP_HITMASK) a.hitmask[wi + 1] = spread16(b0 >> 16) | (spread16(b1 >> 16) << 1);
           a.slowmask[wi + 1] = spread16(s0 >> 16) | (spread16(s1 >> 16) << 1);
         }
       }
@@ -1264,7 +1299,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   }
   flush_count(&a.st->nulls, c_nulls);
   flush_count(&a.st->hits, c_hits);
-  flush_count(&a.st->translated, c_tr);
+  if (OPS & OP_WRITE) flush_count(&a.st->translated, c_tr);
   flush_count(a.slowcount, c_slow);
   if (OPS & OP_DEC) flush_count(&a.st->underflow, c_under);
 }
@@ -1277,7 +1312,11 @@ static int launch_unmap_sh(const SlotArgs &a, int nsm, cudaStream_t s) {
     int dev = 0, optin = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    cudaError_t e = cudaFuncSetAttribute(k_unmap_sh<OPS>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    cudaFuncAttributes fa;
+    cudaError_t e = cudaFuncGetAttributes(&fa, k_unmap_sh<OPS>);
+    if (e != cudaSuccess) return (int)e;
+    e = cudaFuncSetAttribute(k_unmap_sh<OPS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             optin - (int)fa.sharedSizeBytes);
     if (e != cudaSuccess) return (int)e;
     configured = true;
   }
@@ -1349,11 +1388,13 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, i
       a.sel == SEL_ALL && a.cbeg == 0 && !no_pipe)
     return a.segs_host_shadow ? launch_map_pd<1>(a, nsm, s) : launch_map_pd<0>(a, nsm, s);
   constexpr int UNMAP = OP_WRITE | OP_GATE | OP_HITMASK, UNMAP_REL = OP_WRITE | OP_GATE | OP_DEC | OP_HITMASK;
-  if (dir == DIR_REV && (ops == UNMAP || ops == UNMAP_REL) && a.nseg == 1 && a.seg_inplace && a.segs_host_shadow &&
+  if (dir == DIR_REV && (ops == UNMAP || ops == UNMAP_REL || ops == OP_DEC) && a.segs_host_shadow &&
       a.sel == SEL_ALL && a.cbeg == 0 && !no_pipe) {
     // pipelined pass over the recorded slots, then the generic kernel over the slots it left
     if (cudaMemsetAsync(a.slowcount, 0, sizeof(unsigned long long), s) != cudaSuccess) return (int)cudaGetLastError();
-    int r = ops == UNMAP ? launch_unmap_sh<UNMAP>(a, nsm, s) : launch_unmap_sh<UNMAP_REL>(a, nsm, s);
+    int r = ops == UNMAP ? launch_unmap_sh<UNMAP>(a, nsm, s)
+            : ops == UNMAP_REL ? launch_unmap_sh<UNMAP_REL>(a, nsm, s)
+                               : launch_unmap_sh<OP_DEC>(a, nsm, s);
     if (r != 0) return r;
     SlotArgs b = a;
     b.sel = SEL_SLOW;
@@ -1362,7 +1403,7 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, i
   }
   // the forward index qualifies for the specialised path: one segment, no wide bucket, h <= 3
   int fh = a.pd.nseg > 0 ? FH_PD : a.fx.nseg <= 1 && a.fx_nowide && a.fx.h <= 3 ? a.fx.h : -1;
-  const bool sh = a.nseg == 1 && a.segs_host_shadow;
+  const bool sh = a.segs_host_shadow;
 #define X(D, O)                                                        \
   if (dir == D && ops == (O)) {                                        \
     if (sh) {                                                          \

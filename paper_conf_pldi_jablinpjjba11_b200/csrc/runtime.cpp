@@ -662,7 +662,7 @@ struct Context {
     c.nchunks = c0[k];
     if (c.nchunks == 0) return CGCM_OK;
     if ((c.ops & OP_HITMASK) || c.sel != SEL_ALL) CKS(dalloc(hitmask, 4 * (size_t)(c.nchunks / 16 + 4)));
-    if (c.dir == DIR_REV && k == 1 && c.segs[0].shadow) CKS(dalloc(slowmask, 4 * (size_t)(c.nchunks / 16 + 4)));
+    if (c.dir == DIR_REV) CKS(dalloc(slowmask, 4 * (size_t)(c.nchunks / 16 + 4)));
     CKS(dalloc(slowcnt, 64));
     CKS(dalloc(segs, sizeof(Seg) * (size_t)k * 8 + 256));
     CKS(dalloc(seg0, 8 * (size_t)(k + 1) * 8 + 256));
@@ -684,7 +684,8 @@ struct Context {
       a.runid = rev.rid.as<uint32_t>();
     }
     a.segs = dsegs;
-    a.segs_host_shadow = (k == 1 && c.segs[0].shadow != 0) ? 1 : 0;
+    a.segs_host_shadow = 0;
+    for (auto &sg : c.segs) a.segs_host_shadow |= sg.shadow != 0 ? 1 : 0;
     a.seg_inplace = (k == 1 && c.segs[0].out == 0) ? 1 : 0;
     a.seg_chunk0 = dc0;
     a.nseg = k;
@@ -1038,6 +1039,7 @@ struct Context {
     CK(cudaStreamSynchronize(main));
     for (uint32_t x : units) {
       uarr[x] = 0;
+      if (udev[x]) drop_shadows(udev[x]);
       if (uflags[x] & UF_GLOBAL) continue;
       run_release(urun[x]);
       urun[x] = -1;
@@ -1314,6 +1316,48 @@ struct Context {
   };
   std::map<std::pair<uint64_t, uint64_t>, Shadow> shadows;
   uint64_t table_gen = 0;
+  // Record (CPU pointer, unit) per slot for the reverse passes (R13-ii) when a lookup costs more than
+  // the 12-byte shadow: arrays of >= 2^16 slots and indexes with >= 2 levels (measured, config C
+  // (h = 2): 48.5 vs 43.5 G/s); CGCM_FORCE_SHADOW: every array (tests).  Returns the buffer (invalid until the map
+  // succeeds: commit_shadow) or 0.
+  uint64_t begin_shadow(uint64_t ptr, uint64_t n) {
+    static const int min_h = [] {  // CGCM_SHADOW_MIN_H: A/B override of the depth threshold
+      const char *e = std::getenv("CGCM_SHADOW_MIN_H");
+      return e ? std::atoi(e) : 2;
+    }();
+    if (!(flags & CGCM_FORCE_SHADOW) && (n < (1u << 16) || fwd.h < min_h)) return 0;
+    auto key = std::make_pair(ptr, n);
+    Shadow &sh = shadows[key];
+    sh.valid = false;
+    if (dalloc(sh.buf, 12 * n + 64) != CGCM_OK) {
+      shadows.erase(key);
+      return 0;
+    }
+    return sh.buf.addr;
+  }
+  void commit_shadow(uint64_t ptr, uint64_t n, bool ok) {
+    auto it = shadows.find(std::make_pair(ptr, n));
+    if (it == shadows.end()) return;
+    if (ok) {
+      it->second.valid = true;
+      it->second.gen = table_gen;
+    } else {
+      dfree(it->second.buf);
+      shadows.erase(it);
+    }
+  }
+  // the valid shadow of (ptr, n), or 0
+  uint64_t find_shadow(uint64_t ptr, uint64_t n) const {
+    auto it = shadows.find(std::make_pair(ptr, n));
+    return it != shadows.end() && it->second.valid && it->second.gen == table_gen ? it->second.buf.addr : 0;
+  }
+  // an outer's device copy is released: its shadows go with it
+  void drop_shadows(uint64_t ptr) {
+    for (auto it = shadows.lower_bound(std::make_pair(ptr, (uint64_t)0)); it != shadows.end() && it->first.first == ptr;) {
+      dfree(it->second.buf);
+      it = shadows.erase(it);
+    }
+  }
   int take_snapshot() {
     CKS(dalloc(snap_st, 8 * (size_t)U + 64));
     CKS(dalloc(snap_rc, 4 * (size_t)U + 64));
@@ -1726,7 +1770,6 @@ int cgcm_scopeExit(void) {
 }
 
 // ---- device-resident arrays -------------------------------------------------------------------
-static constexpr size_t SHADOW_MIN = 1u << 16;
 
 int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n) {
   CTX();
@@ -1734,29 +1777,9 @@ int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n) {
   if (!d_slots || (reinterpret_cast<uint64_t>(d_slots) & 7)) return CGCM_E_INVALID;
   CKS(C->ensure_table());
   Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
-  Context::Shadow *sh = nullptr;
-  // record (CPU pointer, unit) per slot for the reverse pass (R13-ii) when a lookup costs more than
-  // the 12-byte shadow: indexes with >= 2 levels (measured, config C (h = 2): 48.5 vs 43.5 G/s)
-  static const int shadow_min_h = [] {  // CGCM_SHADOW_MIN_H: A/B override of the depth threshold
-    const char *e = std::getenv("CGCM_SHADOW_MIN_H");
-    return e ? std::atoi(e) : 2;
-  }();
-  if (n >= SHADOW_MIN && (C->fwd.h >= shadow_min_h || (C->flags & CGCM_FORCE_SHADOW))) {
-    auto key = std::make_pair(s.ptr, (uint64_t)n);
-    sh = &C->shadows[key];
-    sh->valid = false;
-    if (C->dalloc(sh->buf, 12 * n + 64) == CGCM_OK) {
-      s.shadow = sh->buf.addr;
-    } else {
-      C->shadows.erase(key);
-      sh = nullptr;
-    }
-  }
+  s.shadow = C->begin_shadow(s.ptr, n);
   int r = C->map_core({s}, {}, nullptr, nullptr);
-  if (sh && r == CGCM_OK) {
-    sh->valid = true;
-    sh->gen = C->table_gen;
-  }
+  if (s.shadow) C->commit_shadow(s.ptr, n, r == CGCM_OK);
   return r;
 }
 
@@ -2039,8 +2062,11 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
     fsegs.swap(fs);
     group.swap(gs);
   }
+  for (auto &sg : fsegs) sg.shadow = C->begin_shadow(sg.ptr, sg.n);  // for unmapArrays / releaseArrays
   uint64_t tr = 0, nl = 0;
   int r = C->map_core(fsegs, {}, &tr, &nl, &group, &pack_ev);
+  for (auto &sg : fsegs)
+    if (sg.shadow) C->commit_shadow(sg.ptr, sg.n, r == CGCM_OK);
   if (r != CGCM_OK) {
     if (rev_done) C->rev_decref(rsegs);
     for (auto &b : backups)
@@ -2112,8 +2138,9 @@ int cgcm_unmapArrays(void *const *const *arrays, size_t k) {
     if (!n) continue;
     auto oc = std::find_if(outer_copies.begin(), outer_copies.end(), [&](const OC &x) { return x.unit == o.unit; });
     if (o.info.flags & UF_ARRAYMAPPED) {
-      if (oc != outer_copies.end()) rsegs_copy.push_back(Seg{o.info.devbase, n, oc->stage, 1, 0});
-      else rsegs_gate.push_back(Seg{o.info.devbase, n, 0, 1, 0});
+      const uint64_t sh = C->find_shadow(o.info.devbase, n);  // the device copy still holds what the map wrote
+      if (oc != outer_copies.end()) rsegs_copy.push_back(Seg{o.info.devbase, n, oc->stage, 1, 0, sh});
+      else rsegs_gate.push_back(Seg{o.info.devbase, n, 0, 1, 0, sh});
     } else {
       fsegs_gate.push_back(Seg{o.info.devbase, n, 0, 1, 0});  // raw CPU pointers (scalar-mapped outer)
     }
@@ -2187,7 +2214,12 @@ int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
     uint64_t n = o.info.size / 8;
     if (!n) continue;
     Seg s{o.info.devbase, n, 0, o.mult, 0};
-    ((o.info.flags & UF_ARRAYMAPPED) ? rsegs : fsegs).push_back(s);
+    if (o.info.flags & UF_ARRAYMAPPED) {
+      s.shadow = C->find_shadow(o.info.devbase, n);
+      rsegs.push_back(s);
+    } else {
+      fsegs.push_back(s);
+    }
   }
   if (!rsegs.empty()) CKS(C->ensure_rev());
   // the outers' own references go first (plain decrement); slot decrements detect underflow / zero

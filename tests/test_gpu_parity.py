@@ -568,3 +568,39 @@ def test_heap_churn_calloc_realloc_alloca(pair):
         assert o.undeclare(x) == 0
         P.units.pop(x)
     P.check("after scopes")
+
+
+def test_host_arrays_large_overlap_and_shadows(pair):
+    """mapArrays / unmapArrays / releaseArrays on outers large enough for the transfer overlap (one
+    copy group per extent: spacers keep the outers in separate extents) and for recorded shadows
+    (>= 2^16 slots), with a GPU function that re-points some slots in between (the reverse passes
+    fall back to full lookups for them).  Every slot, unit and counter against the oracle."""
+    P = pair
+    offs, sizes, R, span = config_C_setup(P, 4096)
+    ns = [(1 << 16) + 3, 1 << 17, (1 << 16) + 100]
+    outers = []
+    for k, n in enumerate(ns):
+        q, _ = W.queries(offs, sizes, n, 30 + k)
+        vals = (q + np.uint64(R)).astype(np.uint64)
+        vals[:: 97 + k] = 0
+        outers.append(P.malloc(8 * n, vals))
+        P.malloc(200 << 10)                               # spacer: the next outer is another extent
+    st, gptrs = P.run("mapArrays", outers)
+    assert st == 0
+    P.check("mapArrays")
+    P.check_device_units()
+    # the "GPU function": swap two halves of outer 1's first 1000 slots, NULL one, duplicate one
+    d1 = int(gptrs[1])
+    dev = P.g.dev_read(d1, 8 * 2000).view(np.uint64).copy()
+    new = dev.copy()
+    new[:1000], new[1000:2000] = dev[1000:2000], dev[:1000]
+    new[5] = 0
+    new[6] = new[7]
+    P.g.dev_write(d1, new)
+    P.o.dev_write(d1, new)
+    P.advance()
+    P.run("unmapArrays", outers)
+    P.check("unmapArrays")
+    st = P.run("releaseArrays", outers)
+    P.check("releaseArrays")
+    W.release_reservation(R, span)
