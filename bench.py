@@ -218,7 +218,8 @@ def run_cgcm(args, rank, world, local_rank):
             traffic = None
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": traffic,
-                "kernel": f"k_slots<{'DIR_REV' if dom == 'rev' else 'DIR_FWD'}> ({dom})",
+                # the hot kernels cgcm_mapArrayDevice / cgcm_unmapArrayDevice launch on one segment
+                "kernel": "k_unmap_sh<WRITE|GATE|DEC|HITMASK> (rev)" if dom == "rev" else "k_map_pd<shadow> (fwd)",
                 "peak_source": peak_kind,
                 "fwd_ms_per_launch": round(fwd_ms, 4), "rev_ms_per_launch": round(rev_ms, 4),
                 "fwd_gbs": round(BYTES_PER_TRANSLATION * fwd_slots / (fwd_ms / 1e3) / 1e9, 1) if fwd_ms else None,

@@ -1101,7 +1101,7 @@ static int launch_map_pd(const SlotArgs &a, int nsm, cudaStream_t s) {
 // -------------------------------------------------------------------------------------------------
 constexpr int UNMAP_SH_THREADS = 768;
 
-template <int OPS>
+template <int OPS, bool MS>  // MS: more than one segment
 __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ uint64_t s_seg0[SEG_SMEM + 1];
@@ -1118,6 +1118,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   __syncthreads();
   const uint64_t *seg0 = seg_s ? s_seg0 : a.seg_chunk0;
   const Seg *segs = seg_s ? s_segs : a.segs;
+  const Seg seg1 = a.segs[0];  // the single segment (!MS), in registers
 
   const uint64_t pol_s = policy_evict_first();
   const uint64_t pol_t = policy_evict_last();
@@ -1127,7 +1128,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
 
   // chunk c -> its segment (last s with seg0[s] <= c)
   auto seg_of = [&](uint64_t c) -> int {
-    if (a.nseg == 1) return 0;
+    if (!MS) return 0;
     int lo = 0, len = a.nseg;
     while (len > 1) {
       const int half = len >> 1;
@@ -1152,8 +1153,8 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
     x.a0 = 0;
     if (c >= a.nchunks) return;
     const int s = seg_of(c);
-    const Seg &sg = segs[s];
-    const uint64_t a0 = (sg.ptr & ~15ull) + 16ull * (c - seg0[s]), hi = sg.ptr + 8ull * sg.n;
+    const Seg &sg = MS ? segs[s] : seg1;
+    const uint64_t a0 = (sg.ptr & ~15ull) + 16ull * (c - (MS ? seg0[s] : 0ull)), hi = sg.ptr + 8ull * sg.n;
     x.s = s;
     x.a0 = a0;
     x.valid = (a0 >= sg.ptr && a0 < hi ? 1u : 0u) | (a0 + 8 >= sg.ptr && a0 + 8 < hi ? 2u : 0u);
@@ -1194,7 +1195,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
     gather(nxt, nw);
 
     const uint32_t valid = cur.valid;
-    const Seg &sg = segs[cur.s];
+    const Seg &sg = MS ? segs[cur.s] : seg1;
     bool hit[2], slow[2];
     uint64_t outv[2] = {cur.g[0], cur.g[1]};
     uint32_t wrote = 0;
@@ -1304,8 +1305,8 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   if (OPS & OP_DEC) flush_count(&a.st->underflow, c_under);
 }
 
-template <int OPS>
-static int launch_unmap_sh(const SlotArgs &a, int nsm, cudaStream_t s) {
+template <int OPS, bool MS>
+static int launch_unmap_sh1(const SlotArgs &a, int nsm, cudaStream_t s) {
   const size_t smem = (a.tab.n_ext <= EXT_SMEM ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
   static bool configured = false;
   if (!configured) {
@@ -1313,9 +1314,9 @@ static int launch_unmap_sh(const SlotArgs &a, int nsm, cudaStream_t s) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     cudaFuncAttributes fa;
-    cudaError_t e = cudaFuncGetAttributes(&fa, k_unmap_sh<OPS>);
+    cudaError_t e = cudaFuncGetAttributes(&fa, k_unmap_sh<OPS, MS>);
     if (e != cudaSuccess) return (int)e;
-    e = cudaFuncSetAttribute(k_unmap_sh<OPS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    e = cudaFuncSetAttribute(k_unmap_sh<OPS, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              optin - (int)fa.sharedSizeBytes);
     if (e != cudaSuccess) return (int)e;
     configured = true;
@@ -1323,8 +1324,12 @@ static int launch_unmap_sh(const SlotArgs &a, int nsm, cudaStream_t s) {
   const uint64_t want = (a.nchunks + UNMAP_SH_THREADS - 1) / UNMAP_SH_THREADS;
   const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
-  k_unmap_sh<OPS><<<grid, UNMAP_SH_THREADS, smem, s>>>(a);
+  k_unmap_sh<OPS, MS><<<grid, UNMAP_SH_THREADS, smem, s>>>(a);
   return (int)cudaGetLastError();
+}
+template <int OPS>
+static int launch_unmap_sh(const SlotArgs &a, int nsm, cudaStream_t s) {
+  return a.nseg > 1 ? launch_unmap_sh1<OPS, true>(a, nsm, s) : launch_unmap_sh1<OPS, false>(a, nsm, s);
 }
 
 // the operation sets the runtime uses
