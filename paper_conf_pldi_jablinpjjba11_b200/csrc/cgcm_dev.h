@@ -86,13 +86,13 @@ struct IndexDev {
 
 // Page directory: the forward index of the hot kernels.  The sorted AU bases are cut
 // into address segments at the largest start-to-start distances (<= PD_MAXSEG; starts, ends and
-// metadata staged in shared memory).  Segment s has pages of 2^P_s bytes (P_s <= 15) from start_s
+// metadata staged in shared memory).  Segment s has pages of 2^P_s bytes (P_s <= PD_MAXSHIFT) from start_s
 // (its first base) through its last base; an address beyond its pages but before the next segment
 // lies in the tail of the segment's last unit (hit iff <= end_s, A7).
 // One 32-byte entry (one L2 sector) per page at address A:
 //   w[0]     j0 = greatestLTE(A), the unit with the greatest base <= A (0xFFFFFFFF: none)
-//   w[1]     cnt (bits 0..14): units with base in (A, A + 2^P) | bit 15: base(j0) == A
-//            | end0 (bits 16..31): min(base(j0) + size(j0) - A + 1, 0xFFFF), 0 if j0 ends before A
+//   w[1]     cnt (bits 0..13): units with base in (A, A + 2^P) | bit 14: base(j0) == A
+//            | end0 (bits 15..31): min(base(j0) + size(j0) - A + 1, 0x1FFFF), 0 if j0 ends before A
 //   w[2..7]  cnt <= PD_K: the offsets base - A of those units, sorted u16, padded with 0xFFFF;
 //            cnt >  PD_K: w[2] = index of the first of cnt sorted u16 offsets in ovf[] (16-aligned,
 //            padded with 0xFFFF to a whole 32-byte sector)
@@ -100,7 +100,16 @@ struct IndexDev {
 // any other candidate by its base A + offset and its size (hot word).  One sector gather per lookup.
 constexpr int PD_MAXSEG = 64;
 constexpr int PD_K = 12;
-constexpr int PD_MAXSHIFT = 15;
+#ifdef CGCM_PD_MAXSHIFT
+constexpr int PD_MAXSHIFT = CGCM_PD_MAXSHIFT;
+#else
+constexpr int PD_MAXSHIFT = 16;  // 64 KiB pages: u16 offsets; a page holding a start at offset 0xFFFF
+                                 // (the padding value) or more than PD_CNT_MAX starts takes a smaller P
+#endif
+constexpr uint32_t PD_CNT_MAX = 0x3FFFu;
+constexpr uint32_t PD_EXACT = 1u << 14;
+constexpr int PD_END_SHIFT = 15;
+constexpr uint32_t PD_END_MAX = 0x1FFFFu;
 struct PdDev {
   const uint32_t *ent;        // 8 u32 per page, segments back to back
   const uint16_t *ovf;        // overflow offsets

@@ -378,8 +378,10 @@ __device__ __forceinline__ void pd_back(const PdDev &pd, uint64_t pol, const PdF
     return;
   }
   const uint32_t j0 = (uint32_t)w_in[0], w1 = (uint32_t)(w_in[0] >> 32);
-  const uint32_t cnt = w1 & 0x7FFFu, end0 = w1 >> 16;
-  const uint32_t rr = f.poff * 0x10001u;
+  const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
+  // padding is 0xFFFF and no start sits at offset 0xFFFF (build_pd): counting with min(poff, 0xFFFE)
+  // never counts padding and counts the same starts
+  const uint32_t rr = min(f.poff, 0xFFFEu) * 0x10001u;
   uint32_t c = 0, mx = 0;
   if (cnt <= (uint32_t)PD_K) {
 #pragma unroll
@@ -405,7 +407,7 @@ __device__ __forceinline__ void pd_back(const PdDev &pd, uint64_t pol, const PdF
   k0 = k == 0;
   if (k == 0) {
     j = (j0 != 0xFFFFFFFFu && f.poff < end0) ? (int)j0 : -1;  // A7 on the page's j0
-    key = (w1 & 0x8000u) ? f.A : f.A - 1;
+    key = (w1 & PD_EXACT) ? f.A : f.A - 1;
   } else {
     j = (int)(j0 + k);
     key = f.A + max(mx & 0xFFFFu, mx >> 16);
@@ -453,8 +455,8 @@ __device__ __forceinline__ void pd_lookup2(const SPd &S, const PdDev &pd, uint64
 #pragma unroll
   for (int m = 0; m < 2; ++m) {
     const uint32_t j0 = (uint32_t)w[m][0], w1 = (uint32_t)(w[m][0] >> 32);
-    const uint32_t cnt = w1 & 0x7FFFu, end0 = w1 >> 16;
-    const uint32_t rr = poff[m] * 0x10001u;
+    const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
+    const uint32_t rr = min(poff[m], 0xFFFEu) * 0x10001u;  // see pd_back
     uint32_t c = 0, mx = 0;
     if (cnt <= (uint32_t)PD_K) {
 #pragma unroll
@@ -486,7 +488,7 @@ __device__ __forceinline__ void pd_lookup2(const SPd &S, const PdDev &pd, uint64
     } else if (k == 0) {
       const bool h0 = ok[m] && j0 != 0xFFFFFFFFu && poff[m] < end0;  // A7 on the page's j0
       j[m] = h0 ? (int)j0 : -1;
-      key[m] = (w1 & 0x8000u) ? A[m] : A[m] - 1;
+      key[m] = (w1 & PD_EXACT) ? A[m] : A[m] - 1;
     } else {
       j[m] = ok[m] ? (int)(j0 + k) : -1;
       key[m] = A[m] + off;

@@ -393,7 +393,7 @@ struct Context {
 
   // Page directory (a0): cut the sorted bases at the largest start-to-start distances (>= 1 MiB, at
   // most PD_MAXSEG segments; pages stop at a segment's last base, whose unit's tail is decided by
-  // the segment's end), give each segment the largest page size 2^P (P <= 15) whose crowded pages (more than
+  // the segment's end), give each segment the largest page size 2^P (P <= PD_MAXSHIFT) whose crowded pages (more than
   // PD_K starts) hold at most CGCM_PD_OVF (default 1 %) of its units, within a budget of
   // max(4n, 2^20) entries overall; then one entry per page (cgcm_dev.h).  No directory (the level
   // index serves the hot kernels) when the budget cannot be met or CGCM_NO_PAGEDIR is set.
@@ -433,18 +433,23 @@ struct Context {
       int sel = -1;
       for (int P = PD_MAXSHIFT; P >= 0; --P) {
         if ((span >> P) + 1 > cap) break;
-        sel = P;
         uint64_t ovf = 0;  // units in pages with more than PD_K starts after the page's first byte
-        for (int i = i0; i < i1;) {
+        bool fits = true;  // every page: <= PD_CNT_MAX starts, none at offset 0xFFFF (the padding value)
+        for (int i = i0; i < i1 && fits;) {
           const uint64_t pg = (hb[i] - S) >> P;
           int k = i, c = 0;
           while (k < i1 && ((hb[k] - S) >> P) == pg) {
-            c += ((hb[k] - S) & ((1ull << P) - 1)) != 0;
+            const uint64_t o = (hb[k] - S) & ((1ull << P) - 1);
+            c += o != 0;
+            fits = fits && o != 0xFFFF;
             ++k;
           }
           if (c > PD_K) ovf += (uint64_t)c;
+          fits = fits && (uint32_t)c <= PD_CNT_MAX;
           i = k;
         }
+        if (!fits) continue;
+        sel = P;
         if ((double)ovf <= ovf_frac * (double)(i1 - i0)) break;
       }
       if (sel < 0) return CGCM_OK;  // too sparse for the budget: the level index serves
@@ -474,10 +479,10 @@ struct Context {
         while (k < i1 && hb[k] < A + psz) ++k;
         const uint32_t cnt = (uint32_t)(k - (i + 1));
         const uint64_t e0 = hb[i] + hs[i];
-        const uint32_t end0 = e0 < A ? 0u : (uint32_t)std::min<uint64_t>(e0 - A + 1, 0xFFFF);
+        const uint32_t end0 = e0 < A ? 0u : (uint32_t)std::min<uint64_t>(e0 - A + 1, PD_END_MAX);
         uint32_t *w = &ent[8 * e];
         w[0] = (uint32_t)i;
-        w[1] = cnt | (hb[i] == A ? 0x8000u : 0u) | (end0 << 16);
+        w[1] = cnt | (hb[i] == A ? PD_EXACT : 0u) | (end0 << PD_END_SHIFT);
         uint16_t *o16 = reinterpret_cast<uint16_t *>(w + 2);
         if (cnt <= (uint32_t)PD_K) {
           for (int t = 0; t < 2 * 6; ++t) o16[t] = t < (int)cnt ? (uint16_t)(hb[i + 1 + t] - A) : (uint16_t)0xFFFF;

@@ -123,3 +123,78 @@ def test_pagedir_lookup_cases(table, flags):
         ctx.close()
         o.close()
         W.release_reservation(R, span)
+
+
+def layout_64k():
+    """Segments that exercise 64 KiB pages (P = 16): page offsets reach 0xFFFF (the padding value of the
+    entry's u16 offsets) and a unit's end crosses whole pages.  Segment 0 takes P = 16; segment 1 has a
+    unit starting at page offset 0xFFFF, so it must fall back to a smaller page (build_pd's rule)."""
+    offs, sizes = [], []
+    S0 = 1 << 20
+    pos = S0
+    for k in range(120):                     # ~2 starts per 64 KiB page, never crowded
+        s = 20000 + 16 * (k % 7)
+        offs.append(pos); sizes.append(s)
+        pos += 30000 + 16 * (k % 5)
+    pos = (pos + 0xFFFF) // 0x10000 * 0x10000 + S0 % 0x10000
+    big = pos                                # a unit covering whole pages, then one ending on 0xFFFF
+    offs.append(pos); sizes.append(3 * 0x10000 + 0x1234)
+    pos += 4 * 0x10000
+    offs.append(pos); sizes.append(0xFFFF)   # [A, A + 0xFFFF]: its one-past-end is the next page start
+    pos += 0x10000 + 0x10000
+    S1 = pos + (8 << 20)                     # segment 1
+    pos = S1
+    offs.append(pos); sizes.append(100)
+    offs.append(S1 + 0xFFFF); sizes.append(10)   # start at page offset 0xFFFF of a 64 KiB page
+    offs.append(S1 + 0x10000 + 0x20); sizes.append(4000)
+    pos = S1 + 0x30000
+    for k in range(60):
+        offs.append(pos); sizes.append(9000)
+        pos += 25000
+    return (np.array(offs, dtype=np.uint64), np.array(sizes, dtype=np.uint64), pos + (1 << 20), S0, S1, big)
+
+
+def test_pagedir_64k_pages():
+    import torch
+    import paper_conf_pldi_jablinpjjba11_b200 as cg
+    from oracle import Oracle
+    offs, sizes, span, S0, S1, big = layout_64k()
+    R = W.reserve_readonly(span)
+    ctx = cg.Context(0, arena_bytes=1 << 28, flags=LENIENT)
+    o = Oracle(LENIENT)
+    P = Pair(ctx, o)
+    try:
+        bases = offs + np.uint64(R)
+        assert P.g.declareBatch(bases, sizes, readonly=True) == 0
+        for b, s in zip(bases, sizes):
+            assert P.o.declareAlloc(int(b), int(s), readonly=True) == 0
+        info = P.g.indexInfo()
+        assert info["pd_segments"] == 2
+        assert info["pd_max_shift"] == 16 and info["pd_min_shift"] <= 15, info
+        q = [offs, offs + sizes - np.uint64(1), offs + sizes, offs + sizes + np.uint64(1)]
+        for S, npages in ((S0, 72), (S1, 40)):   # every page start, its last byte and neighbours
+            A = np.uint64(S) + np.arange(npages, dtype=np.uint64) * np.uint64(0x10000)
+            q += [A, A + np.uint64(0xFFFF), A + np.uint64(0xFFFE), A + np.uint64(0x8000), A + np.uint64(0x7FFF)]
+        q.append(np.array([big + 0x10000 + 0xFFFF, big + 3 * 0x10000 + 0x1234, big + 3 * 0x10000 + 0x1235],
+                          dtype=np.uint64))
+        slots = np.concatenate(q) + np.uint64(R)
+        n = len(slots)
+        d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+        assert P.g.mapArrayDevice(d.data_ptr(), n) == 0
+        P.feed_replay()
+        ref = slots.copy()
+        assert P.o.mapSlots(ref) == 0
+        got = d.cpu().numpy().view(np.uint64)
+        bad = np.nonzero(got != ref)[0]
+        assert len(bad) == 0, [(hex(int(slots[i]) - R), hex(int(got[i])), hex(int(ref[i]))) for i in bad[:8]]
+        P.check("mapped")
+        P.advance()
+        assert P.g.unmapArrayDevice(d.data_ptr(), n, release=True) == 0
+        assert P.o.unmapSlots(ref, release=True) == 0
+        got = d.cpu().numpy().view(np.uint64)
+        assert (got == ref).all() and (got == slots).all()
+        P.check("unmapped")
+    finally:
+        ctx.close()
+        o.close()
+        W.release_reservation(R, span)

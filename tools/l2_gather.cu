@@ -179,6 +179,62 @@ __global__ void __launch_bounds__(768, 1)
                  : "memory");
   }
 }
+
+// page-directory forward skeleton (k_map_pd's memory shape): a streamed 16-B load per 2 slots; per slot
+// ENT: a 32-B entry gather (dependent on the slot value), HOT: a dependent 8-B unit-word gather, RED: one
+// reduction into a separate refcount array, SH: a 12-B shadow store; the 16-B slot store.  No compute.
+template <bool ENT, bool HOT, bool RED, bool SH, bool W64 = false>
+__global__ void __launch_bounds__(768, 1)
+    k_skel_pd(uint64_t *slots, uint64_t nchunks, const uint64_t *ent, uint64_t nent, const uint64_t *hot,
+              uint64_t nunit, int32_t *rc, uint64_t *shp, uint32_t *shu) {
+  const uint64_t pl = pol_last(), pf = pol_first();
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; c < nchunks; c += stride) {
+    uint64_t x0, x1;
+    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;"
+                 : "=l"(x0), "=l"(x1)
+                 : "l"(slots + 2 * c), "l"(pf));
+    uint64_t a = mix(x0 + 2 * c), b = mix(x1 + 2 * c + 1);
+    if (ENT && !W64) {
+      uint64_t va[4], vb[4];
+      ld32(ent + 4 * (a % nent), pl, va);
+      ld32(ent + 4 * (b % nent), pl, vb);
+      a = mix(a ^ va[0]);
+      b = mix(b ^ vb[0]);
+    }
+    if (ENT && W64) {  // 64-byte entries: two 32-byte loads of one 64-byte block
+      uint64_t va[4], vb[4], wa[4], wb[4];
+      const uint64_t ea = 8 * (a % (nent / 2)), eb = 8 * (b % (nent / 2));
+      ld32(ent + ea, pl, va);
+      ld32(ent + ea + 4, pl, wa);
+      ld32(ent + eb, pl, vb);
+      ld32(ent + eb + 4, pl, wb);
+      a = mix(a ^ va[0] ^ wa[3]);
+      b = mix(b ^ vb[0] ^ wb[3]);
+    }
+    const uint64_t ia = a % nunit, ib = b % nunit;
+    uint64_t ha = 0, hb = 0;
+    if (HOT) {
+      asm volatile("ld.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(ha) : "l"(hot + ia), "l"(pl));
+      asm volatile("ld.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(hb) : "l"(hot + ib), "l"(pl));
+    }
+    if (RED) {
+      asm volatile("red.global.add.s32 [%0], %1;" ::"l"(rc + ia), "r"(1) : "memory");
+      asm volatile("red.global.add.s32 [%0], %1;" ::"l"(rc + ib), "r"(1) : "memory");
+    }
+    if (SH) {
+      asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u64 [%0], {%1,%2}, %3;" ::"l"(shp + 2 * c), "l"(x0),
+                   "l"(x1), "l"(pf)
+                   : "memory");
+      asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1,%2}, %3;" ::"l"(shu + 2 * c),
+                   "r"((uint32_t)ia), "r"((uint32_t)ib), "l"(pf)
+                   : "memory");
+    }
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u64 [%0], {%1,%2}, %3;" ::"l"(slots + 2 * c),
+                 "l"(x0 + ha), "l"(x1 + hb), "l"(pf)
+                 : "memory");
+  }
+}
 __global__ void k_fill_units(uint32_t *u, uint64_t n, uint32_t nrec) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
     u[i] = (uint32_t)(mix(i) % nrec);
@@ -306,6 +362,43 @@ int main(int argc, char **argv) {
     rev(k_skeleton_rev<true, true, true, false, true>, "shadow+gather+red(separate array)");
     rev(k_skeleton_rev<true, true, true, true, true>, "shadow+gather(no_allocate)+red(separate)");
     rev(k_skeleton_rev<true, true, true, false, true, true>, "scalar shadow+gather+red(separate)");
+    // page-directory forward skeletons: config E (39 MiB entries, 2^22 units) and C (10 MiB, 2^20)
+    for (int cfg = 0; cfg < 2; ++cfg) {
+      const uint64_t nent = cfg == 0 ? (78ull << 20) / 32 : (20ull << 20) / 32, nunit = cfg == 0 ? 1ull << 22 : 1ull << 20;
+      uint64_t *ent, *hot;
+      int32_t *rcs;
+      CK(cudaMalloc(&ent, 32 * nent));
+      CK(cudaMalloc(&hot, 8 * nunit));
+      CK(cudaMalloc(&rcs, 4 * nunit));
+      CK(cudaMemset(ent, 0x11, 32 * nent));
+      CK(cudaMemset(hot, 0, 8 * nunit));
+      CK(cudaMemset(rcs, 0, 4 * nunit));
+      auto pd = [&](auto kern, const char *what) {
+        kern<<<nsm, 768>>>(slots, nslots / 2, ent, nent, hot, nunit, rcs, shp, shu);
+        CK(cudaEventRecord(e0));
+        for (int r = 0; r < 5; ++r) kern<<<nsm, 768>>>(slots, nslots / 2, ent, nent, hot, nunit, rcs, shp, shu);
+        CK(cudaEventRecord(e1));
+        CK(cudaEventSynchronize(e1));
+        double ms = time_ms(e0, e1) / 5;
+        printf("{\"test\": \"skeleton_pd\", \"cfg\": \"%s\", \"parts\": \"%s\", \"slots\": %llu, \"ms\": %.3f, \"G_slots_per_s\": %.1f}\n",
+               cfg == 0 ? "E" : "C", what, (unsigned long long)nslots, ms, nslots / ms / 1e6);
+      };
+      pd(k_skel_pd<true, true, true, true>, "ent+hot+red+shadow");
+      pd(k_skel_pd<true, false, true, true, true>, "ent64+red+shadow");
+      pd(k_skel_pd<true, false, true, false, true>, "ent64+red");
+      pd(k_skel_pd<true, false, true, true>, "ent+red+shadow");
+      pd(k_skel_pd<true, true, true, false>, "ent+hot+red");
+      pd(k_skel_pd<true, true, false, false>, "ent+hot");
+      pd(k_skel_pd<true, false, true, false>, "ent+red");
+      pd(k_skel_pd<false, true, true, false>, "hot+red");
+      pd(k_skel_pd<true, false, false, false>, "ent");
+      pd(k_skel_pd<false, false, true, false>, "red");
+      pd(k_skel_pd<false, false, false, true>, "streams+shadow");
+      pd(k_skel_pd<false, false, false, false>, "streams");
+      CK(cudaFree(ent));
+      CK(cudaFree(hot));
+      CK(cudaFree(rcs));
+    }
     CK(cudaGetLastError());
   }
   return 0;
