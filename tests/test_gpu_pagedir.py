@@ -198,3 +198,63 @@ def test_pagedir_64k_pages():
         ctx.close()
         o.close()
         W.release_reservation(R, span)
+
+
+@pytest.mark.parametrize("flags", [0, FORCE_SHADOW], ids=["pagedir", "pagedir-shadow"])
+def test_pagedir_activation_free_cycles(flags):
+    """k_map_pd's translations must follow every activation (new extent), free and re-activation of
+    the units it lands on.  Rounds of mapArrayDevice / unmapArrayDevice(release) over different unit
+    subsets, with a pinned subset held across rounds by a second array; every translation, refcount
+    and epoch vs the oracle."""
+    import torch
+    import paper_conf_pldi_jablinpjjba11_b200 as cg
+    from oracle import Oracle
+    U = 3000
+    offs, sizes, span = W.table_layout(U, 21)
+    R = W.reserve_readonly(span)
+    ctx = cg.Context(0, arena_bytes=1 << 30, flags=flags)
+    o = Oracle()
+    P = Pair(ctx, o)
+    try:
+        bases = offs + np.uint64(R)
+        assert P.g.declareBatch(bases, sizes, readonly=True) == 0
+        for b, s in zip(bases, sizes):
+            assert P.o.declareAlloc(int(b), int(s), readonly=True) == 0
+        assert P.g.indexInfo()["pd_segments"] > 0
+        pins = (offs[::7] + np.uint64(R)).astype(np.uint64)       # held across all rounds
+        dp = torch.from_numpy(pins.view(np.int64).copy()).cuda()
+        assert P.g.mapArrayDevice(dp.data_ptr(), len(pins)) == 0
+        P.feed_replay()
+        pref = pins.copy()
+        assert P.o.mapSlots(pref) == 0
+        assert (dp.cpu().numpy().view(np.uint64) == pref).all()
+        for r in range(4):
+            q, u = W.queries(offs, sizes, 20000 + 101 * r, 30 + r)
+            keep = (u % np.uint64(4)) != np.uint64(r)              # a different subset each round
+            slots = (q[keep] + np.uint64(R)).astype(np.uint64)
+            slots[::53] = 0
+            n = len(slots)
+            d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+            assert P.g.mapArrayDevice(d.data_ptr(), n) == 0
+            P.feed_replay()
+            ref = slots.copy()
+            assert P.o.mapSlots(ref) == 0
+            got = d.cpu().numpy().view(np.uint64)
+            bad = np.nonzero(got != ref)[0]
+            assert len(bad) == 0, (r, [(hex(int(got[i])), hex(int(ref[i]))) for i in bad[:4]])
+            if r % 2:
+                P.check(f"round {r} mapped")
+            P.advance()
+            assert P.g.unmapArrayDevice(d.data_ptr(), n, release=True) == 0
+            assert P.o.unmapSlots(ref, release=True) == 0
+            assert (d.cpu().numpy().view(np.uint64) == slots).all()
+            P.check(f"round {r} released")
+        P.advance()
+        assert P.g.unmapArrayDevice(dp.data_ptr(), len(pins), release=True) == 0
+        assert P.o.unmapSlots(pref, release=True) == 0
+        P.check("pins released")
+        assert all(x["refCount"] == 0 for x in P.g.dump())
+    finally:
+        ctx.close()
+        o.close()
+        W.release_reservation(R, span)
