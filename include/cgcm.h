@@ -108,6 +108,16 @@ int cgcm_declareAllocFlags(void *base, size_t size, unsigned unit_flags);
 int cgcm_declareBatch(void *const *bases, const size_t *sizes, size_t n, unsigned unit_flags);
 int cgcm_undeclare(void *base);
 int cgcm_declareGlobal(const char *name, void *base, size_t size, int isReadOnly);
+/* cgcm_declareGlobalSymbol (NEXT-4; Alg. 1's `cuModuleGetGlobal(name)` branch, P:L214-215,
+ *   P:L219-222, and the glue-kernel globals of P:L305-310): as cgcm_declareGlobal, but the device
+ *   copy IS the __device__ variable at dev_symbol (a device address the caller obtained with
+ *   cudaGetSymbolAddress / cuModuleGetGlobal, >= size bytes, owned by its module and never freed by
+ *   the runtime).  map() returns dev_symbol + (p - base); activation copies the host bytes into the
+ *   symbol and copy-back reads them out of it, so GPU code that names the variable directly sees the
+ *   mapped data.  CGCM_E_INVALID for a NULL symbol; CGCM_E_OVERLAP if its range overlaps another
+ *   bound symbol or touches one whose host unit does not touch this one in the same order (A7:
+ *   adjacent device copies must mirror adjacent host units).                                      */
+int cgcm_declareGlobalSymbol(const char *name, void *base, size_t size, int isReadOnly, void *dev_symbol);
 /* Heap wrappers (R10): a header-free pinned host arena; every block is declared as one AU, so
  * consecutive blocks are host-adjacent and their copies coalesce.  cgcm_free undeclares (BUSY if
  * mapped -> the block is not freed).  NULL on failure.                                           */

@@ -73,6 +73,7 @@ def lib():
             "cgcm_declareAlloc": (i, [vp, sz]), "cgcm_declareAllocFlags": (i, [vp, sz, C.c_uint]),
             "cgcm_declareBatch": (i, [vp, vp, sz, C.c_uint]), "cgcm_undeclare": (i, [vp]),
             "cgcm_declareGlobal": (i, [C.c_char_p, vp, sz, i]),
+            "cgcm_declareGlobalSymbol": (i, [C.c_char_p, vp, sz, i, vp]),
             "cgcm_malloc": (vp, [sz]), "cgcm_free": (i, [vp]),
             "cgcm_calloc": (vp, [sz, sz]), "cgcm_realloc": (vp, [vp, sz]),
             "cgcm_declareAlloca": (vp, [sz]), "cgcm_scopeEnter": (i, []), "cgcm_scopeExit": (i, []),
@@ -108,6 +109,10 @@ def samples():
         S.cgcm_sample_scale.argtypes = [u64, u64, u64, C.c_double, vp]
         S.cgcm_sample_treesum_level.restype = C.c_int
         S.cgcm_sample_treesum_level.argtypes = [u64, u64, u64, u64, u64, vp]
+        S.cgcm_sample_global_addr.restype = C.c_int
+        S.cgcm_sample_global_addr.argtypes = [C.POINTER(C.c_void_p), C.POINTER(C.c_size_t)]
+        S.cgcm_sample_scale_global.restype = C.c_int
+        S.cgcm_sample_scale_global.argtypes = [C.c_double, vp]
         S.cgcm_sample_gemm_rows.restype = C.c_int
         S.cgcm_sample_gemm_rows.argtypes = [u64, u64, u64, C.c_int, C.c_int, C.c_int, C.c_double, C.c_double, vp]
         S.cgcm_test_d2h.restype = C.c_int
@@ -171,6 +176,10 @@ class Context:
 
     def declareGlobal(self, name, base, size, ro=False) -> int:
         return self.L.cgcm_declareGlobal(name.encode() if name is not None else None, base, size, int(ro))
+
+    def declareGlobalSymbol(self, name, base, size, ro, dev_symbol) -> int:
+        return self.L.cgcm_declareGlobalSymbol(name.encode() if name is not None else None, base, size, int(ro),
+                                               dev_symbol)
 
     def undeclare(self, base: int) -> int:
         return self.L.cgcm_undeclare(base)
@@ -299,6 +308,16 @@ class Context:
     # ---- test-only sample GPU functions on the main stream ----
     def sample_scale(self, rows_dev, nrows, ncols, alpha):
         return samples().cgcm_sample_scale(rows_dev, nrows, ncols, alpha, self.main.cuda_stream)
+
+    def sample_global(self):
+        """(device address, bytes) of the test-only __device__ array of libcgcm_samples.so"""
+        a, n = C.c_void_p(), C.c_size_t()
+        if samples().cgcm_sample_global_addr(C.byref(a), C.byref(n)) != 0:
+            raise CgcmError("cudaGetSymbolAddress failed")
+        return a.value, n.value
+
+    def sample_scale_global(self, alpha):
+        return samples().cgcm_sample_scale_global(alpha, self.main.cuda_stream)
 
     def sample_treesum_level(self, child_dev, root_dev, nnodes, lo, hi):
         return samples().cgcm_sample_treesum_level(child_dev, root_dev, nnodes, lo, hi, self.main.cuda_stream)

@@ -149,6 +149,7 @@ struct HostUnit {
   uint64_t epoch0 = 0;      // globalEpoch at declaration (A20)
   int32_t idx = -1;         // rank in the device table (valid after a table build)
   std::string name;
+  uint64_t sym = 0;         // declareGlobalSymbol: the bound __device__ symbol's address (NEXT-4)
 };
 
 // one device extent holding the copies of one or more host-adjacent units (mirrored layout)
@@ -156,6 +157,7 @@ struct Run {
   uint64_t addr = 0, bytes = 0;
   uint64_t delta = 0;  // host address - device address of every unit copy in the extent (mirrored)
   int64_t live = 0;
+  bool external = false;  // a bound __device__ symbol: not arena memory, never freed by the runtime
 };
 
 // Search-index buffers: forward (all units by base) and reverse (live device extents by start)
@@ -203,6 +205,7 @@ struct Context {
   std::vector<uint64_t> ubase, usize, udev;  // host base, size, device copy address (0: none)
   std::vector<uint32_t> uflags;              // UF_GLOBAL | UF_READONLY
   std::vector<int64_t> urun;                 // device extent holding the copy (-1: none)
+  std::vector<uint64_t> usym;                // bound __device__ symbol of a global (0: none)
   std::vector<uint8_t> uarr;                 // mirror of UF_ARRAYMAPPED
   std::unordered_set<std::string> names;
   bool table_dirty = true, rev_dirty = true;
@@ -299,7 +302,7 @@ struct Context {
     return id;
   }
   void drop_run(int64_t id) {
-    arena.free(runs[id].addr, runs[id].bytes);
+    if (!runs[id].external) arena.free(runs[id].addr, runs[id].bytes);
     live_runs.erase(runs[id].addr);
     runs[id] = Run();
     free_runs.push_back(id);
@@ -536,6 +539,7 @@ struct Context {
     std::vector<int64_t> nrun(n, -1);
     std::vector<uint8_t> narr(n, 0);
     uflags.resize(n);
+    usym.resize(n);
     int i = 0;
     for (auto it = reg.begin(); it != reg.end(); ++it, ++i) {
       int32_t o = it->second.idx;
@@ -545,6 +549,7 @@ struct Context {
       ho[i] = o;
       hf[i] = it->second.flags & (UF_GLOBAL | UF_READONLY);
       uflags[i] = hf[i];
+      usym[i] = it->second.sym;
       if (o >= 0) {
         ndev[i] = udev[o];
         nrun[i] = urun[o];
@@ -909,6 +914,16 @@ struct Context {
         P.dev0 = udev[x0];
         P.run = urun[x0];
         devbases[P.i] = udev[x0];
+        continue;
+      }
+      if (P.global && usym[x0]) {  // bound to a __device__ symbol: its storage is the symbol (NEXT-4)
+        P.dev0 = usym[x0];
+        P.run = new_run(P.dev0, P.h1 - P.h0, P.h0 - P.dev0);
+        runs[P.run].external = true;
+        udev[x0] = P.dev0;
+        urun[x0] = P.run;
+        devbases[P.i] = P.dev0;
+        runs[P.run].live += 1;
         continue;
       }
       uint64_t need = (P.h0 % 256) + (P.h1 - P.h0) + 1;
@@ -1552,7 +1567,7 @@ int cgcm_setContext(void *ctx) {
 }
 
 // ---- registration --------------------------------------------------------------------------
-static int declare_one(Context *C, uint64_t b, uint64_t s, uint32_t fl, const char *name) {
+static int declare_one(Context *C, uint64_t b, uint64_t s, uint32_t fl, const char *name, uint64_t sym = 0) {
   if (b == 0 || s == 0 || b + s < b || b + s >= ADDR_LIMIT) return CGCM_E_INVALID;
   auto succ = C->reg.lower_bound(b);
   if (succ != C->reg.end() && succ->first < b + s) return CGCM_E_OVERLAP;
@@ -1565,6 +1580,7 @@ static int declare_one(Context *C, uint64_t b, uint64_t s, uint32_t fl, const ch
   u.flags = fl;
   u.epoch0 = C->epoch;
   if (name) u.name = name;
+  u.sym = sym;
   C->reg.emplace_hint(succ, b, u);
   C->table_dirty = true;
   return CGCM_OK;
@@ -1615,6 +1631,26 @@ int cgcm_declareGlobal(const char *name, void *base, size_t size, int isReadOnly
   if (!name || !*name) return CGCM_E_INVALID;
   if (C->names.count(name)) return CGCM_E_DUPLICATE;
   int s = declare_one(C, reinterpret_cast<uint64_t>(base), size, UF_GLOBAL | (isReadOnly ? UF_READONLY : 0), name);
+  if (s == CGCM_OK) C->names.insert(name);
+  return s;
+}
+int cgcm_declareGlobalSymbol(const char *name, void *base, size_t size, int isReadOnly, void *dev_symbol) {
+  CTX();
+  if (!name || !*name || !dev_symbol) return CGCM_E_INVALID;
+  if (C->names.count(name)) return CGCM_E_DUPLICATE;
+  const uint64_t b = reinterpret_cast<uint64_t>(base), d = reinterpret_cast<uint64_t>(dev_symbol);
+  // A7: two device copies may touch only if their host units touch in the same order (a one-past-the-end
+  // pointer of one must reverse to the same place).  Arena extents always keep >= 1 byte of slack, so
+  // only other bound symbols can be adjacent or overlap.
+  for (auto &kv : C->reg) {
+    const HostUnit &o = kv.second;
+    if (!o.sym) continue;
+    const uint64_t ob = kv.first, os = o.size;
+    if (d < o.sym + os && o.sym < d + size) return CGCM_E_OVERLAP;
+    if (d + size == o.sym && b + size != ob) return CGCM_E_OVERLAP;
+    if (o.sym + os == d && ob + os != b) return CGCM_E_OVERLAP;
+  }
+  int s = declare_one(C, b, size, UF_GLOBAL | (isReadOnly ? UF_READONLY : 0), name, d);
   if (s == CGCM_OK) C->names.insert(name);
   return s;
 }

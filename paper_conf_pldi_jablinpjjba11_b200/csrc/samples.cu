@@ -10,7 +10,16 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+// a module-scope __device__ variable, for symbol-bound globals (cgcm_declareGlobalSymbol, NEXT-4):
+// GPU code names it directly, the way the paper's glue kernels reach globals
+__device__ double cgcm_sample_global[512];
+
 namespace {
+
+__global__ void k_scale_global(double alpha) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < 512; i += gridDim.x * blockDim.x)
+    cgcm_sample_global[i] = __dmul_rn(cgcm_sample_global[i], alpha);
+}
 
 __global__ void k_scale(const double *const *rows, uint64_t nrows, uint64_t ncols, double alpha) {
   uint64_t total = nrows * ncols;
@@ -86,3 +95,12 @@ int cgcm_test_h2d(uint64_t dst, const void *src, uint64_t n) {
 }
 
 }  // extern "C"
+
+extern "C" int cgcm_sample_global_addr(void **addr, size_t *bytes) {
+  if (cudaGetSymbolAddress(addr, cgcm_sample_global) != cudaSuccess) return -8;
+  return cudaGetSymbolSize(bytes, cgcm_sample_global) == cudaSuccess ? 0 : -8;
+}
+extern "C" int cgcm_sample_scale_global(double alpha, void *stream) {
+  k_scale_global<<<2, 256, 0, (cudaStream_t)stream>>>(alpha);
+  return cudaGetLastError() == cudaSuccess ? 0 : -8;
+}

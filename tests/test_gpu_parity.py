@@ -604,3 +604,38 @@ def test_host_arrays_large_overlap_and_shadows(pair):
     st = P.run("releaseArrays", outers)
     P.check("releaseArrays")
     W.release_reservation(R, span)
+
+
+def test_global_bound_to_device_symbol(pair):
+    """NEXT-4: a global whose device copy is a module's __device__ variable (Alg. 1's cuModuleGetGlobal
+    branch).  map returns the symbol's address, GPU code that names the
+    variable sees the host values, copy-back returns what it wrote, re-maps reuse the symbol (A14),
+    and a second symbol range overlapping it is rejected (A7)."""
+    P = pair
+    sym, nbytes = P.g.sample_global()
+    assert nbytes == 512 * 8
+    buf = HostBuf(8192)
+    vals = W.config_A_values(1, 512, 7)[0]                       # fp64 in [1, 2)
+    host_write(buf.addr, vals)
+    s1 = P.g.declareGlobalSymbol("g_sym", buf.addr, nbytes, False, sym)
+    s2 = P.o.declareGlobal("g_sym", buf.addr, nbytes)
+    assert s1 == s2 == 0
+    P.units[buf.addr] = nbytes
+    P.o.host_write(buf.addr, np.frombuffer(host_read(buf.addr, nbytes), dtype=np.uint8))
+    assert P.g.declareGlobalSymbol("g_sym2", buf.addr + 6000, 64, False, sym + 8) == -3   # overlaps g_sym
+    assert P.g.declareGlobalSymbol("g_sym", buf.addr + 6000, 64, False, sym + nbytes + 64) == -6
+    expect = vals.copy()
+    for it in range(3):
+        st, d = P.run("map", buf.addr + 8 * it)                 # interior pointer: symbol + offset
+        assert d == sym + 8 * it
+        assert P.g.sample_scale_global(ALPHA) == 0
+        P.g.synchronize()
+        expect = expect * ALPHA                                   # one correctly rounded multiply (A21)
+        P.o.dev_write(sym, expect.view(np.uint8))
+        P.advance()
+        P.run("unmap", buf.addr + 8 * it)
+        P.run("release", buf.addr + 8 * it)
+        P.check(f"symbol global, cycle {it}")
+        got = np.frombuffer(host_read(buf.addr, nbytes), dtype=np.float64)
+        assert (got == expect).all()
+    assert P.undeclare(buf.addr) == 0
