@@ -37,7 +37,8 @@ enum {
   CGCM_E_NOMEM = -7,        /* device arena / pinned host arena exhausted                           */
   CGCM_E_CUDA = -8,         /* a CUDA runtime call failed: cgcm_lastCudaError() has the detail      */
   CGCM_E_MIXED = -9,        /* reserved                                                             */
-  CGCM_E_NOCTX = -10        /* no current context on this thread                                    */
+  CGCM_E_NOCTX = -10,       /* no current context on this thread                                    */
+  CGCM_E_MODREF = -11       /* cgcm_regionEnd: the CPU accessed a promoted AU inside the region     */
 };
 
 /* ---- cgcm_init flags ----------------------------------------------------------------------- */
@@ -176,6 +177,28 @@ int cgcm_releaseArrays(void *const *const *arrays, size_t k);
 enum { CGCM_RELEASE = 1u };
 int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n);
 int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags);
+
+/* ===================== map promotion at run time (NEXT-2) ===================================
+ * The paper's map promotion (§5.1) hoists a loop's map/mapArray calls above
+ * it and its unmaps below it, so in-loop maps find their AUs active (no copies, A2) and in-loop
+ * releases never reach refCount 0; it is legal only if the CPU neither modifies nor references the
+ * promoted AUs inside the loop (¬modOrRef).  Without the compiler pass:
+ * cgcm_regionBegin: map (kind CGCM_REGION_MAP) or mapArray (CGCM_REGION_MAPARRAY) each of ptrs[0..n)
+ *   once and hold those references until cgcm_regionEnd.  All-or-nothing.  CGCM_E_BUSY if a region
+ *   is open on this context (or, with CGCM_REGION_CHECK, anywhere in the process).
+ *   CGCM_REGION_CHECK: the dynamic modOrRef checker -- the host pages of every promoted AU (for
+ *   arrays: the outer AU and every AU its slots point into) are made PROT_NONE; a CPU access to them
+ *   outside a runtime call is counted (a SIGSEGV handler reopens the page and lets the access
+ *   proceed).  Whole pages are protected, so an access to other data sharing a page also counts
+ *   (conservative).  CGCM_E_INVALID if mprotect refuses the pages (cgcm_lastCudaError has errno).
+ * cgcm_regionEnd: reopen the pages, then unmap/unmapArray + release/releaseArray every promoted
+ *   pointer (reverse order; epoch-gated copy-backs as usual).  *violations = accesses counted.
+ *   Returns CGCM_E_MODREF if any (the promoted execution may differ from the naive one: the caller's
+ *   loop must not be promoted), else the first unmap/release error, else OK.                      */
+enum { CGCM_REGION_MAP = 0u, CGCM_REGION_MAPARRAY = 1u };
+enum { CGCM_REGION_CHECK = 1u };
+int cgcm_regionBegin(void *const *ptrs, const unsigned *kinds, size_t n, unsigned flags);
+int cgcm_regionEnd(size_t *violations);
 
 /* ================================ introspection ===========================================
  * cgcm_stats: counters since init.  cgcm_dumpTable: the AU table in base order (cap entries; *n

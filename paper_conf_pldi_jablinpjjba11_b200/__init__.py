@@ -21,8 +21,8 @@ LIB_PATH = os.path.join(os.environ.get("CGCM_LIBDIR") or HERE, "libcgcm.so")
 SAMPLES_PATH = os.path.join(HERE, "libcgcm_samples.so")
 
 OK = 0
-E_INVALID, E_UNREGISTERED, E_OVERLAP, E_NOT_MAPPED, E_BUSY, E_DUPLICATE, E_NOMEM, E_CUDA, E_MIXED, E_NOCTX = (
-    -1, -2, -3, -4, -5, -6, -7, -8, -9, -10)
+E_INVALID, E_UNREGISTERED, E_OVERLAP, E_NOT_MAPPED, E_BUSY, E_DUPLICATE, E_NOMEM, E_CUDA, E_MIXED, E_NOCTX, E_MODREF = (
+    -1, -2, -3, -4, -5, -6, -7, -8, -9, -10, -11)
 LITERAL_EPOCH, LENIENT, PROFILE, FORCE_SHADOW, NO_PAGEDIR = 1, 2, 4, 8, 16
 UNIT_GLOBAL, UNIT_READONLY, UNIT_ARRAYMAPPED, UNIT_ACTIVE = 1, 2, 4, 8
 RELEASE = 1
@@ -74,6 +74,8 @@ def lib():
             "cgcm_declareBatch": (i, [vp, vp, sz, C.c_uint]), "cgcm_undeclare": (i, [vp]),
             "cgcm_declareGlobal": (i, [C.c_char_p, vp, sz, i]),
             "cgcm_declareGlobalSymbol": (i, [C.c_char_p, vp, sz, i, vp]),
+            "cgcm_regionBegin": (i, [vp, vp, sz, C.c_uint]),
+            "cgcm_regionEnd": (i, [C.POINTER(C.c_size_t)]),
             "cgcm_malloc": (vp, [sz]), "cgcm_free": (i, [vp]),
             "cgcm_calloc": (vp, [sz, sz]), "cgcm_realloc": (vp, [vp, sz]),
             "cgcm_declareAlloca": (vp, [sz]), "cgcm_scopeEnter": (i, []), "cgcm_scopeExit": (i, []),
@@ -180,6 +182,20 @@ class Context:
     def declareGlobalSymbol(self, name, base, size, ro, dev_symbol) -> int:
         return self.L.cgcm_declareGlobalSymbol(name.encode() if name is not None else None, base, size, int(ro),
                                                dev_symbol)
+
+    # ---- map-promotion regions (NEXT-2) ----
+    REGION_MAP, REGION_MAPARRAY, REGION_CHECK = 0, 1, 1
+
+    def regionBegin(self, ptrs, kinds, check=False) -> int:
+        n = len(ptrs)
+        pa = (C.c_uint64 * max(n, 1))(*ptrs)
+        ka = (C.c_uint * max(n, 1))(*kinds)
+        return self.L.cgcm_regionBegin(C.addressof(pa), C.addressof(ka), n, 1 if check else 0)
+
+    def regionEnd(self):
+        v = C.c_size_t()
+        s = self.L.cgcm_regionEnd(C.byref(v))
+        return s, v.value
 
     def undeclare(self, base: int) -> int:
         return self.L.cgcm_undeclare(base)

@@ -7,8 +7,13 @@
 // those are the kernels of kernels.cu.  Nothing in this file can fall back
 // to a CPU computation of a kernel's result.
 #include <cuda_runtime.h>
+#include <signal.h>
+#include <sys/mman.h>
+#include <unistd.h>
 
 #include <algorithm>
+#include <atomic>
+#include <cerrno>
 #include <cstdint>
 #include <cstdlib>
 #include <cstdio>
@@ -206,6 +211,9 @@ struct Context {
   std::vector<uint32_t> uflags;              // UF_GLOBAL | UF_READONLY
   std::vector<int64_t> urun;                 // device extent holding the copy (-1: none)
   std::vector<uint64_t> usym;                // bound __device__ symbol of a global (0: none)
+  // open map-promotion region (cgcm_regionBegin): the promoted pointers and their kinds
+  bool region_open = false, region_checked = false;
+  std::vector<std::pair<uint64_t, unsigned>> region;
   std::vector<uint8_t> uarr;                 // mirror of UF_ARRAYMAPPED
   std::unordered_set<std::string> names;
   bool table_dirty = true, rev_dirty = true;
@@ -1450,6 +1458,64 @@ std::mutex g_ctx_mu;
 std::unordered_set<Context *> g_contexts;
 thread_local Context *tl_ctx = nullptr;
 
+// ---- map-promotion regions and their dynamic modOrRef checker (NEXT-2) ----
+// While a checked region is open, the host pages of every promoted AU are PROT_NONE.  A CPU access
+// to one faults; the handler reopens that page and, unless a runtime call is in progress (the
+// runtime's own reads/writes of host AUs are not the program's), counts a violation: the loop did
+// modify or reference a promoted AU, which makes the promotion illegal (P:L261 ¬modOrRef).  Pages
+// the runtime touched are closed again when its call returns.  Process-wide (one signal handler).
+struct ProtRange {
+  uintptr_t lo, hi;
+};
+constexpr int PROT_MAX = 4096, TOUCH_MAX = 4096;
+static ProtRange g_prot[PROT_MAX];
+static std::atomic<int> g_nprot{0};
+static std::atomic<int> g_rt_busy{0};
+static std::atomic<unsigned long long> g_viol{0};
+static std::atomic<uintptr_t> g_viol_first{0};
+static uintptr_t g_touched[TOUCH_MAX];
+static std::atomic<int> g_ntouched{0};
+static struct sigaction g_old_segv;
+static bool g_segv_installed = false;
+static uintptr_t g_pagesz = 4096;
+
+static void on_segv(int sig, siginfo_t *si, void *uc) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(si->si_addr);
+  const int n = g_nprot.load(std::memory_order_acquire);
+  for (int i = 0; i < n; ++i)
+    if (a >= g_prot[i].lo && a < g_prot[i].hi) {
+      const uintptr_t pg = a & ~(g_pagesz - 1);
+      mprotect(reinterpret_cast<void *>(pg), g_pagesz, PROT_READ | PROT_WRITE);
+      if (g_rt_busy.load() > 0) {
+        const int k = g_ntouched.fetch_add(1);
+        if (k < TOUCH_MAX) g_touched[k] = pg;
+      } else if (g_viol.fetch_add(1) == 0) {
+        g_viol_first.store(a);
+      }
+      return;  // the access re-executes on the reopened page
+    }
+  // not a promoted page: the previous handler (or the default action on the re-executed access)
+  if ((g_old_segv.sa_flags & SA_SIGINFO) && g_old_segv.sa_sigaction) {
+    g_old_segv.sa_sigaction(sig, si, uc);
+    return;
+  }
+  if (!(g_old_segv.sa_flags & SA_SIGINFO) && g_old_segv.sa_handler != SIG_DFL && g_old_segv.sa_handler != SIG_IGN) {
+    g_old_segv.sa_handler(sig);
+    return;
+  }
+  sigaction(SIGSEGV, &g_old_segv, nullptr);
+}
+// every C-ABI call: pages the runtime itself touches in a checked region are closed again on return
+struct RtScope {
+  RtScope() { g_rt_busy.fetch_add(1); }
+  ~RtScope() {
+    if (g_rt_busy.fetch_sub(1) == 1) {
+      const int n = std::min(g_ntouched.exchange(0), TOUCH_MAX);
+      for (int i = 0; i < n && g_nprot.load() > 0; ++i) mprotect(reinterpret_cast<void *>(g_touched[i]), g_pagesz, PROT_NONE);
+    }
+  }
+};
+
 }  // namespace cgcm
 
 using namespace cgcm;
@@ -1458,6 +1524,7 @@ using SlotCall = Context::SlotCall;
 #define CTX()                                     \
   Context *C = tl_ctx;                            \
   if (!C) return CGCM_E_NOCTX;                    \
+  RtScope rts_;                                   \
   std::lock_guard<std::recursive_mutex> lk_(C->mu); \
   if (cudaSetDevice(C->device) != cudaSuccess) return CGCM_E_CUDA;
 
@@ -1477,6 +1544,7 @@ const char *cgcm_strerror(int s) {
     case CGCM_E_CUDA: return "CUDA error";
     case CGCM_E_MIXED: return "mixed";
     case CGCM_E_NOCTX: return "no current context";
+    case CGCM_E_MODREF: return "the CPU accessed a promoted allocation unit inside a map-promotion region";
   }
   return "unknown";
 }
@@ -2309,6 +2377,145 @@ int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
   // outers whose zero came from a slot decrement are already in f; outers with remaining slot refs
   // into them (self-reference) cannot be in outer_zero (their refcount exceeded mult)
   return C->free_units(f);
+}
+
+// ---- map-promotion regions (NEXT-2) ----
+int cgcm_regionBegin(void *const *ptrs, const unsigned *kinds, size_t n, unsigned flags) {
+  CTX();
+  if (C->region_open) return CGCM_E_BUSY;
+  if (n && (!ptrs || !kinds)) return CGCM_E_INVALID;
+  const bool check = (flags & CGCM_REGION_CHECK) != 0;
+  if (check && g_nprot.load() > 0) return CGCM_E_BUSY;  // one checked region per process
+  for (size_t i = 0; i < n; ++i)
+    if (kinds[i] > CGCM_REGION_MAPARRAY) return CGCM_E_INVALID;
+  // the hoisted maps (Listing 4: map/mapArray before the loop)
+  size_t done = 0;
+  int err = CGCM_OK;
+  for (; done < n && err == CGCM_OK; ++done) {
+    const void *p = ptrs[done];
+    if (kinds[done] == CGCM_REGION_MAP) {
+      void *out = nullptr;
+      err = cgcm_mapBatch(&p, 1, &out);
+    } else {
+      void **out = nullptr;
+      void *const *pp = reinterpret_cast<void *const *>(p);
+      err = cgcm_mapArrays(&pp, 1, &out);
+    }
+  }
+  auto undo = [&](size_t k) {
+    for (size_t i = k; i-- > 0;) {
+      const void *p = ptrs[i];
+      if (kinds[i] == CGCM_REGION_MAP) {
+        cgcm_releaseBatch(&p, 1);
+      } else {
+        void *const *pp = reinterpret_cast<void *const *>(p);
+        cgcm_releaseArrays(&pp, 1);
+      }
+    }
+  };
+  if (err != CGCM_OK) {
+    undo(done - 1);
+    return err;
+  }
+  if (check) {  // the host pages of every promoted AU (array outers and the AUs their slots point into)
+    std::vector<std::pair<uint64_t, uint64_t>> au;
+    auto unit_of = [&](uint64_t q) {
+      auto it = C->reg.upper_bound(q);
+      if (it == C->reg.begin()) return;
+      --it;
+      if (q - it->first <= it->second.size) au.push_back({it->first, it->first + it->second.size});
+    };
+    for (size_t i = 0; i < n; ++i) {
+      const uint64_t p = reinterpret_cast<uint64_t>(ptrs[i]);
+      unit_of(p);
+      if (kinds[i] == CGCM_REGION_MAPARRAY && !au.empty()) {
+        const uint64_t b = au.back().first, e = au.back().second;
+        for (uint64_t w = b; w + 8 <= e; w += 8) {
+          uint64_t v;
+          std::memcpy(&v, reinterpret_cast<const void *>(w), 8);
+          if (v) unit_of(v);
+        }
+      }
+    }
+    g_pagesz = (uintptr_t)sysconf(_SC_PAGESIZE);
+    std::vector<ProtRange> rr;
+    for (auto &x : au) rr.push_back({x.first & ~(g_pagesz - 1), (x.second + g_pagesz - 1) & ~(g_pagesz - 1)});
+    std::sort(rr.begin(), rr.end(), [](const ProtRange &a, const ProtRange &b) { return a.lo < b.lo; });
+    std::vector<ProtRange> m;
+    for (auto &r : rr) {
+      if (r.hi <= r.lo) continue;
+      if (!m.empty() && r.lo <= m.back().hi)
+        m.back().hi = std::max(m.back().hi, r.hi);
+      else
+        m.push_back(r);
+    }
+    if (m.size() > (size_t)PROT_MAX) {
+      undo(n);
+      return CGCM_E_NOMEM;
+    }
+    if (!g_segv_installed) {
+      struct sigaction sa;
+      std::memset(&sa, 0, sizeof(sa));
+      sa.sa_sigaction = on_segv;
+      sa.sa_flags = SA_SIGINFO;
+      sigemptyset(&sa.sa_mask);
+      if (sigaction(SIGSEGV, &sa, &g_old_segv) != 0) {
+        undo(n);
+        return CGCM_E_INVALID;
+      }
+      g_segv_installed = true;
+    }
+    for (size_t i = 0; i < m.size(); ++i) g_prot[i] = m[i];
+    g_viol.store(0);
+    g_viol_first.store(0);
+    g_nprot.store((int)m.size(), std::memory_order_release);
+    for (size_t i = 0; i < m.size(); ++i)
+      if (mprotect(reinterpret_cast<void *>(m[i].lo), m[i].hi - m[i].lo, PROT_NONE) != 0) {
+        g_last_cuda_error = std::string("mprotect: ") + std::strerror(errno);
+        for (size_t k = 0; k < i; ++k)
+          mprotect(reinterpret_cast<void *>(m[k].lo), m[k].hi - m[k].lo, PROT_READ | PROT_WRITE);
+        g_nprot.store(0);
+        undo(n);
+        return CGCM_E_INVALID;
+      }
+  }
+  C->region.clear();
+  for (size_t i = 0; i < n; ++i) C->region.push_back({reinterpret_cast<uint64_t>(ptrs[i]), kinds[i]});
+  C->region_open = true;
+  C->region_checked = check;
+  return CGCM_OK;
+}
+int cgcm_regionEnd(size_t *violations) {
+  CTX();
+  if (!C->region_open) return CGCM_E_INVALID;
+  unsigned long long v = 0;
+  if (C->region_checked) {  // reopen every page before the copy-backs write host memory
+    const int np = g_nprot.exchange(0);
+    for (int i = 0; i < np; ++i)
+      mprotect(reinterpret_cast<void *>(g_prot[i].lo), g_prot[i].hi - g_prot[i].lo, PROT_READ | PROT_WRITE);
+    v = g_viol.exchange(0);
+  }
+  // the hoisted unmaps and releases (Listing 4 after the loop, A11), in reverse order
+  int err = CGCM_OK;
+  for (size_t i = C->region.size(); i-- > 0;) {
+    const void *p = reinterpret_cast<const void *>(C->region[i].first);
+    int s1, s2;
+    if (C->region[i].second == CGCM_REGION_MAP) {
+      s1 = cgcm_unmapBatch(&p, 1);
+      s2 = cgcm_releaseBatch(&p, 1);
+    } else {
+      void *const *pp = reinterpret_cast<void *const *>(p);
+      s1 = cgcm_unmapArrays(&pp, 1);
+      s2 = cgcm_releaseArrays(&pp, 1);
+    }
+    if (err == CGCM_OK) err = s1 != CGCM_OK ? s1 : s2;
+  }
+  C->region.clear();
+  C->region_open = false;
+  C->region_checked = false;
+  if (violations) *violations = (size_t)v;
+  if (err != CGCM_OK) return err;
+  return v ? CGCM_E_MODREF : CGCM_OK;
 }
 
 int cgcm_mapArray(void *const *cpu, void ***gpu_out) {

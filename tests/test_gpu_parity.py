@@ -639,3 +639,57 @@ def test_global_bound_to_device_symbol(pair):
         got = np.frombuffer(host_read(buf.addr, nbytes), dtype=np.float64)
         assert (got == expect).all()
     assert P.undeclare(buf.addr) == 0
+
+
+@pytest.mark.parametrize("check", [False, True], ids=["region", "region+checker"])
+def test_region_promotes_config_A(pair, check):
+    """NEXT-2: cgcm_regionBegin/End perform Listing 4's hoisted mapArray / unmapArray+releaseArray
+    (A11) around a loop whose body keeps its own mapArray + releaseArray; compared
+    with the oracle running the promoted sequence explicitly.  With the modOrRef checker on, the
+    loop (which never touches host memory) records no violation."""
+    P = pair
+    nrows = ncols = 64
+    rows, pp, vals = setup_A(P, nrows, ncols)
+    assert P.g.regionBegin([pp], [P.g.REGION_MAPARRAY], check=check) == 0
+    P.feed_replay()
+    assert P.o.mapArray(pp)[0] == 0
+    for it in range(10):
+        st, d = P.run("mapArray", pp)
+        assert P.g.sample_scale(d, nrows, ncols, ALPHA) == 0
+        P.g.synchronize()
+        P.o.kernel_scale(d, nrows, ncols, ALPHA)
+        P.advance()
+        P.run("releaseArray", pp)
+    s, v = P.g.regionEnd()
+    assert (s, v) == (0, 0)
+    assert P.o.unmapArray(pp) == 0 and P.o.releaseArray(pp) == 0
+    P.check("after region")
+    st = P.g.stats()
+    assert st["h2d_units"] == nrows + 1 and st["d2h_units"] == nrows + 1   # once each way (promoted)
+    got = np.stack([np.frombuffer(host_read(a, 8 * ncols), dtype=np.float64) for a in rows])
+    exp = vals.copy()
+    for _ in range(10):
+        exp = exp * ALPHA
+    assert (got == exp).all()
+
+
+def test_region_checker_counts_cpu_accesses(pair):
+    """The dynamic modOrRef checker: a CPU read of a promoted AU inside the region is
+    counted and cgcm_regionEnd reports CGCM_E_MODREF; the access itself completes (the page is
+    reopened) and the runtime state stays equal to the oracle's."""
+    P = pair
+    buf = HostBuf(1 << 20, align=4096)
+    base = buf.addr + 8192
+    P.declare(base, 4096, np.arange(512, dtype=np.float64))
+    assert P.g.regionBegin([base], [P.g.REGION_MAP], check=True) == 0
+    P.feed_replay()
+    assert P.o.map(base)[0] == 0
+    P.advance()
+    seen = np.frombuffer(host_read(base + 64, 16), dtype=np.float64)   # the CPU references the AU
+    assert list(seen) == [8.0, 9.0]
+    s, v = P.g.regionEnd()
+    assert s == -11                                                       # CGCM_E_MODREF
+    assert v >= 1
+    assert P.o.unmap(base) == 0 and P.o.release(base) == 0
+    P.check("after checked region")
+    assert P.g.regionEnd()[0] == -1                                       # no open region

@@ -26,7 +26,10 @@ def timed(fn):
     return time.perf_counter() - t0
 
 
-def config_A(promoted, iters=100):
+def config_A(mode, iters=100):
+    """mode: naive | promoted (hand-hoisted, Listing 4) | region (cgcm_regionBegin/End, NEXT-2) |
+    region_check (+ the mprotect modOrRef checker)"""
+    promoted = mode != "naive"
     ctx = cg.Context(0, arena_bytes=1 << 30)
     nrows = ncols = 256
     vals = W.config_A_values(nrows, ncols, 1)
@@ -45,9 +48,13 @@ def config_A(promoted, iters=100):
         calls[name] += time.perf_counter() - t0
         return r
 
+    viol = [None]
+
     def run():
-        if promoted:
+        if mode == "promoted":
             st, d0 = ctx.mapArray(pp)
+        elif mode.startswith("region"):
+            assert ctx.regionBegin([pp], [ctx.REGION_MAPARRAY], check=mode == "region_check") == 0
         for _ in range(iters):
             st, d = tcall("mapArray", lambda: ctx.mapArray(pp))
             tcall("kernel", lambda: (ctx.sample_scale(d, nrows, ncols, 0.999), ctx.synchronize()))
@@ -55,14 +62,17 @@ def config_A(promoted, iters=100):
             if not promoted:
                 tcall("unmapArray", lambda: ctx.unmapArray(pp))
             tcall("releaseArray", lambda: ctx.releaseArray(pp))
-        if promoted:
+        if mode == "promoted":
             ctx.unmapArray(pp)
             ctx.releaseArray(pp)
+        elif mode.startswith("region"):
+            s_, viol[0] = ctx.regionEnd()
+            assert s_ == 0, s_
 
     t = timed(run)
     s = ctx.stats()
     ctx.close()
-    return {"config": "A", "mode": "promoted" if promoted else "naive", "iterations": iters,
+    return {"config": "A", "mode": mode, "iterations": iters, "region_violations": viol[0],
             "us_per_iteration": round(1e6 * t / iters, 1),
             "us_per_call": {k: round(1e6 * v / iters, 1) for k, v in calls.items()},
             "h2d_units": s["h2d_units"], "h2d_bytes": s["h2d_bytes"], "d2h_units": s["d2h_units"],
@@ -157,8 +167,8 @@ if __name__ == "__main__":
     which = sys.argv[1:] or ["A", "B", "D"]
     for w in which:
         if w == "A":
-            for p in (False, True):
-                print(json.dumps(config_A(p)), flush=True)
+            for m in ("naive", "promoted", "region", "region_check"):
+                print(json.dumps(config_A(m)), flush=True)
         elif w == "B":
             for p in (True, False):
                 print(json.dumps(config_B(p)), flush=True)
