@@ -234,6 +234,14 @@ struct Context {
   DevBuf status, lc, hitmask, act_list, journal, free_list, copy_list, segs, seg0, staging, staging2, staging_cb, points, ptrs, temp;
   DevBuf up_units, up_vals, up_exts, uops;
   HostBuf h_small, h_status, h_list, h_pack[2];
+  // pinned staging ring for small uploads: two halves, each fenced by an event on the main stream --
+  // an upload waits for the GPU only when it reuses a half whose copies may still be in flight
+  static constexpr size_t RING_HALF = 1 << 20;
+  HostBuf h_ring;
+  cudaEvent_t ev_ring[2] = {nullptr, nullptr};
+  bool ring_used[2] = {false, false};
+  int ring_cur = 0;
+  size_t ring_head = 0;
   int pack_k = 0;
   cudaEvent_t ev_copy = nullptr, ev_t0 = nullptr, ev_t1 = nullptr, ev_pack[2] = {nullptr, nullptr};
 
@@ -687,9 +695,16 @@ struct Context {
     // each launch uses its own eighth of the segment buffers (st_index 0..7, up to 8 launches in flight)
     Seg *dsegs = segs.as<Seg>() + (size_t)st_index * k;
     uint64_t *dc0 = seg0.as<uint64_t>() + (size_t)st_index * (k + 1);
-    CK(cudaMemcpyAsync(dsegs, c.segs.data(), sizeof(Seg) * k, cudaMemcpyHostToDevice, main));
-    CK(cudaMemcpyAsync(dc0, c0.data(), 8 * (size_t)(k + 1), cudaMemcpyHostToDevice, main));
-    CK(cudaStreamSynchronize(main));  // the host vectors above are pageable and go out of scope
+    // pinned ring (no host wait) unless the outers' H2D copies are in flight on the copy stream: a
+    // pinned upload is a DMA that would queue behind them, while a small pageable copy is not
+    if (c.seg_group.empty() && sizeof(Seg) * k + 8 * (size_t)(k + 1) <= RING_HALF / 2) {
+      CKS(ring_put(dsegs, c.segs.data(), sizeof(Seg) * k));
+      CKS(ring_put(dc0, c0.data(), 8 * (size_t)(k + 1)));
+    } else {
+      CK(cudaMemcpyAsync(dsegs, c.segs.data(), sizeof(Seg) * k, cudaMemcpyHostToDevice, main));
+      CK(cudaMemcpyAsync(dc0, c0.data(), 8 * (size_t)(k + 1), cudaMemcpyHostToDevice, main));
+      CK(cudaStreamSynchronize(main));  // the host vectors above are pageable and go out of scope
+    }
     SlotArgs a;
     std::memset(&a, 0, sizeof(a));
     a.tab = tab();
@@ -823,10 +838,30 @@ struct Context {
     std::memcpy(out.data(), h_list.p, sizeof(T) * n);
     return CGCM_OK;
   }
+  // n <= RING_HALF bytes from pageable host memory to dst, stream-ordered on main, no host wait
+  int ring_put(void *dst, const void *src, size_t n) {
+    if (!h_ring.p) {
+      CKS(h_ring.ensure(2 * RING_HALF));
+      for (auto &e : ev_ring) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
+    if (ring_head + n > RING_HALF) {
+      CK(cudaEventRecord(ev_ring[ring_cur], main));
+      ring_used[ring_cur] = true;
+      ring_cur ^= 1;
+      ring_head = 0;
+      if (ring_used[ring_cur]) CK(cudaEventSynchronize(ev_ring[ring_cur]));
+    }
+    char *p = h_ring.as<char>() + (size_t)ring_cur * RING_HALF + ring_head;
+    std::memcpy(p, src, n);
+    ring_head += (n + 255) & ~(size_t)255;
+    CK(cudaMemcpyAsync(dst, p, n, cudaMemcpyHostToDevice, main));
+    return CGCM_OK;
+  }
   template <class T>
   int upload(DevBuf &dst, const std::vector<T> &v) {
     CKS(dalloc(dst, sizeof(T) * v.size() + 64));
     if (v.empty()) return CGCM_OK;
+    if (sizeof(T) * v.size() <= RING_HALF) return ring_put(dst.as<void>(), v.data(), sizeof(T) * v.size());
     CKS(h_small.ensure(sizeof(T) * v.size()));
     CK(cudaStreamSynchronize(main));
     std::memcpy(h_small.p, v.data(), sizeof(T) * v.size());
@@ -1175,6 +1210,11 @@ struct Context {
                const std::vector<cudaEvent_t> *group_ev = nullptr) {
     uint64_t total = 0;
     for (auto &s : fsegs) total += s.n;
+    if (fsegs.empty() && rsegs.empty()) {  // nothing to translate (e.g. every outer was re-mapped, A9)
+      if (translated_out) *translated_out = 0;
+      if (nulls_out) *nulls_out = 0;
+      return CGCM_OK;
+    }
     CKS(prepare(total + 64));
     SlotCall F;
     F.dir = DIR_FWD;
@@ -1607,6 +1647,9 @@ int cgcm_finalize(void) {
   cudaStreamSynchronize(C->copy);
   for (auto &c : C->hchunks) cudaFreeHost(c.first);
   if (C->h_small.p) cudaFreeHost(C->h_small.p);
+  if (C->h_ring.p) cudaFreeHost(C->h_ring.p);
+  for (auto &e : C->ev_ring)
+    if (e) cudaEventDestroy(e);
   if (C->h_status.p) cudaFreeHost(C->h_status.p);
   if (C->h_list.p) cudaFreeHost(C->h_list.p);
   cudaEventDestroy(C->ev_copy);
