@@ -880,31 +880,18 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
 
 // -------------------------------------------------------------------------------------------------
 // k_map_pd: the forward map of one in-place segment (mapArrayDevice; a1 + a2 of Alg. 1) through the
-// page directory, software-pipelined: while chunk t is translated, the page-directory entries of
-// chunk t+1 are already on their way into shared memory (cp.async, one 32-byte sector per slot) and
-// the slot values of chunk t+2 into registers.  The dependent L2 round trips of one chunk (entry, then
-// the unit's hot word) thus overlap those of the next.  Same results, counters and lists as
+// page directory.  Per slot: one 32-byte page-entry gather (a single LDG.256: the entry as two
+// 16-byte cp.async cost 1.33 L2 requests, profiles/r01k_ab_ldg.log), one 8-byte unit-word gather,
+// one refcount reduction -- the random L2 operations that bound it (profiles/r01j_l2_model.md).
+// Both slots' entry gathers are in flight together, and the slot values of chunk t+2 are loaded
+// while chunk t is translated.  Same results, counters and lists as
 // k_slots<DIR_FWD, OP_WRITE | OP_INC | OP_HITMASK> (which serves every other case).
 // -------------------------------------------------------------------------------------------------
 #ifdef CGCM_MAP_PD_THREADS
 constexpr int MAP_PD_THREADS = CGCM_MAP_PD_THREADS;
 #else
-constexpr int MAP_PD_THREADS = 768;
+constexpr int MAP_PD_THREADS = 768;  // measured: 768 > 1024 (5.42 ms at E) > 640 > 512
 #endif
-
-__device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, uint64_t pol) {
-  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "l"(pol)
-               : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-__device__ __forceinline__ void lds_sector(uint32_t addr, uint64_t v[4]) {
-  asm volatile("ld.shared.v2.u64 {%0,%1}, [%2];" : "=l"(v[0]), "=l"(v[1]) : "r"(addr));
-  asm volatile("ld.shared.v2.u64 {%0,%1}, [%2];" : "=l"(v[2]), "=l"(v[3]) : "r"(addr + 16));
-}
 
 template <int SH>
 __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
@@ -915,11 +902,6 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
   uint64_t *s_ext = reinterpret_cast<uint64_t *>(sp);
   if (ext_s)
     for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
-  sp += ext_s ? al16(8 * (size_t)a.tab.n_ext) : 0;
-  // entry ring: [stage][slot m][thread] 32 bytes each
-  const uint32_t ring = (uint32_t)__cvta_generic_to_shared(sp);
-  const uint32_t my = ring + 32u * threadIdx.x;
-  const uint32_t mstride = 32u * blockDim.x, sstride = 2u * mstride;
   __syncthreads();
 
   const uint64_t pol_s = policy_evict_first();
@@ -935,37 +917,18 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
     return c < a.nchunks ? ((a0 >= sg.ptr && a0 < hi_addr ? 1u : 0u) | (a0 + 8 >= sg.ptr && a0 + 8 < hi_addr ? 2u : 0u))
                          : 0u;
   };
-  // issue the entry gathers of chunk c (values v) into ring stage st
-  auto issue = [&](uint64_t c, const uint64_t v[2], uint32_t st) {
-    const uint32_t valid = valid_of(c);
-#pragma unroll
-    for (int m = 0; m < 2; ++m) {
-      const PdFront f = pd_front(PD, v[m], ((valid >> m) & 1) && v[m] != 0);
-      if (f.ok) {
-        const uint32_t d = my + st * sstride + m * mstride;
-        const uint32_t *src = a.pd.ent + 8 * f.e;
-        cp_async16(d, src, pol_t);
-        cp_async16(d + 16, src + 4, pol_t);
-      }
-    }
-    cp_async_commit();
-  };
 
   const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   uint64_t cv[2] = {0, 0}, nv[2] = {0, 0}, nnv[2] = {0, 0};
   if (c_first < a.nchunks) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c_first), pol_s, cv[0], cv[1]);
   if (c_first + stride < a.nchunks)
     ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, nv[0], nv[1]);
-  issue(c_first, cv, 0);
-  uint32_t stage = 0;
   for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
     const uint64_t c = cb + lane;
     const bool live = c < a.nchunks;
-    // pipeline: values of chunk t+2 into registers, entries of chunk t+1 into the ring
+    // pipeline: values of chunk t+2 into registers
     if (c + 2 * stride < a.nchunks)
       ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, nnv[0], nnv[1]);
-    issue(c + stride, nv, stage ^ 1u);
-    cp_async_wait<1>();  // this chunk's entries have landed
 
     const uint64_t a0 = a0base + 16ull * c;
     const uint32_t valid = valid_of(c);
@@ -973,13 +936,20 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
     int j[2];
     uint64_t key[2], hw[2] = {0, 0};
     bool look[2], k0[2];
+    PdFront fr[2];
+    uint64_t ew[2][4] = {{0, 0, 0, 0}, {0, 0, 0, 0}};
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {  // a1: both page-entry gathers in flight before either is decoded
+      look[m] = ((valid >> m) & 1) && cv[m] != 0;
+      fr[m] = pd_front(PD, cv[m], look[m]);
+      if (fr[m].ok)  // one LDG.256, not allocated in L1 (random sectors: no reuse; measured 0.98 -> 0.97 ms at C)
+        asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+                     : "=l"(ew[m][0]), "=l"(ew[m][1]), "=l"(ew[m][2]), "=l"(ew[m][3])
+                     : "l"(a.pd.ent + 8 * fr[m].e), "l"(pol_t));
+    }
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      look[m] = ((valid >> m) & 1) && cv[m] != 0;
-      const PdFront f = pd_front(PD, cv[m], look[m]);
-      uint64_t w[4] = {0, 0, 0, 0};
-      if (f.ok) lds_sector(my + stage * sstride + m * mstride, w);
-      pd_back(a.pd, pol_t, f, cv[m], w, j[m], key[m], k0[m]);
+      pd_back(a.pd, pol_t, fr[m], cv[m], ew[m], j[m], key[m], k0[m]);
       look[m] = look[m] && j[m] >= 0;
       if (look[m]) hw[m] = ld_u64(a.tab.hot + j[m], pol_t);
     }
@@ -1061,9 +1031,7 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
     cv[1] = nv[1];
     nv[0] = nnv[0];
     nv[1] = nnv[1];
-    stage ^= 1u;
   }
-  cp_async_wait<0>();
   flush_count(&a.st->nulls, c_nulls);
   flush_count(&a.st->hits, c_hits);
   flush_count(&a.st->misses, c_miss);
@@ -1073,8 +1041,7 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
 
 template <int SH>
 static int launch_map_pd(const SlotArgs &a, int nsm, cudaStream_t s) {
-  const size_t smem = pd_stage_bytes(a.pd) + (a.tab.n_ext <= EXT_SMEM ? al16(8 * (size_t)a.tab.n_ext) : 0) +
-                      2ull * 2 * 32 * MAP_PD_THREADS;
+  const size_t smem = pd_stage_bytes(a.pd) + (a.tab.n_ext <= EXT_SMEM ? al16(8 * (size_t)a.tab.n_ext) : 0);
   static bool configured = false;
   if (!configured) {
     int dev = 0, optin = 0;
