@@ -62,6 +62,16 @@ __device__ __forceinline__ uint64_t ld_u64(const uint64_t *p, uint64_t pol) {
   asm volatile("ld.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
   return v;
 }
+// unit-word gathers of the hot kernels (random: no L1 reuse)
+__device__ __forceinline__ uint64_t ld_u64_hot(const uint64_t *p, uint64_t pol) {
+  uint64_t v;
+#ifdef CGCM_HOT_NOL1
+  asm volatile("ld.global.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+#else
+  asm volatile("ld.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+#endif
+  return v;
+}
 __device__ __forceinline__ void red_add(int32_t *p, int32_t v) {
   asm volatile("red.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -951,7 +961,7 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
     for (int m = 0; m < 2; ++m) {
       pd_back(a.pd, pol_t, fr[m], cv[m], ew[m], j[m], key[m], k0[m]);
       look[m] = look[m] && j[m] >= 0;
-      if (look[m]) hw[m] = ld_u64(a.tab.hot + j[m], pol_t);
+      if (look[m]) hw[m] = ld_u64_hot(a.tab.hot + j[m], pol_t);
     }
     bool hit[2];
 #pragma unroll
@@ -1150,7 +1160,8 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   // the state words (epoch | extent | flags) of the recorded units of x
   auto gather = [&](const In &x, uint64_t w[2]) {
 #pragma unroll
-    for (int m = 0; m < 2; ++m) w[m] = (x.u[m] != 0xFFFFFFFFu && x.g[m] != 0) ? ld_u64(a.tab.st + x.u[m], pol_t) : 0ull;
+    for (int m = 0; m < 2; ++m)
+      w[m] = (x.u[m] != 0xFFFFFFFFu && x.g[m] != 0) ? ld_u64_hot(a.tab.st + x.u[m], pol_t) : 0ull;
   };
 
   const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
