@@ -224,6 +224,7 @@ def run_cgcm(args, rank, world, local_rank):
                 "fwd_ms_per_launch": round(fwd_ms, 4), "rev_ms_per_launch": round(rev_ms, 4),
                 "fwd_gbs": round(BYTES_PER_TRANSLATION * fwd_slots / (fwd_ms / 1e3) / 1e9, 1) if fwd_ms else None,
                 "rev_gbs": round(BYTES_PER_TRANSLATION * rev_slots / (rev_ms / 1e3) / 1e9, 1) if rev_ms else None}
+    roofline["l2_random_ops"] = l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots)
     gpu_launches = int(st["kernel_launches"])
 
     e2e = None
@@ -247,6 +248,31 @@ def run_cgcm(args, rank, world, local_rank):
         result["cpu_baseline"] = cpu_baseline(wl, args.cpu_sample, steps=1)
     ctx.close()
     return result
+
+
+def l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots):
+    """The roof that binds: each hot kernel's time is bounded below by its random L2
+    operations per slot divided by the measured rates of those primitives on this GPU (random 32-byte
+    gathers and random red.add.s32 into L2-resident arrays, tools/l2_gather.cu, committed log).
+    k_map_pd: page entry + unit word gathers + 1 refcount RED; k_unmap_sh: state word gather + 1 RED."""
+    g, r = 238.9, 188.4  # G/s, profiles/r01j_l2_gather.log (gather32 at 48 MiB, red_s32)
+    try:
+        with open(os.path.join(ROOT, "profiles", "r01j_l2_gather.log")) as f:
+            for ln in f:
+                d = json.loads(ln)
+                if d.get("test") == "gather32" and d.get("buffer_MiB") == 48:
+                    g = d["G_per_s"]
+                if d.get("test") == "red_s32":
+                    r = d["G_per_s"]
+    except Exception:
+        pass
+    fwd_floor = fwd_slots * (2 / g + 1 / r) / 1e6  # ms
+    rev_floor = rev_slots * (1 / g + 1 / r) / 1e6
+    return {"gather_gps": g, "red_gps": r, "source": "profiles/r01j_l2_gather.log",
+            "fwd_ops_per_slot": "2 gathers + 1 RED", "rev_ops_per_slot": "1 gather + 1 RED",
+            "fwd_floor_ms": round(fwd_floor, 4), "rev_floor_ms": round(rev_floor, 4),
+            "fwd_frac": round(fwd_floor / fwd_ms, 4) if fwd_ms else None,
+            "rev_frac": round(rev_floor / rev_ms, 4) if rev_ms else None}
 
 
 def host_link(dev, nbytes=256 << 20, reps=5):
