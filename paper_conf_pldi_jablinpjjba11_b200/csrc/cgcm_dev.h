@@ -22,6 +22,7 @@ namespace cgcm {
 //              translation = p + ext_delta[extent(u)]  (Alg. 1: devptr + (ptr - base))
 struct TableDev {
   uint64_t *hot;
+  uint32_t *hotc;  // compact mirror of hot (make_hotc): the forward kernel's 4-byte unit word
   uint64_t *st;
   int32_t *rc;
   const uint64_t *base;
@@ -55,6 +56,23 @@ __device__ __forceinline__ uint32_t *lo_word(uint64_t *w) { return reinterpret_c
 __device__ __forceinline__ uint32_t *hi_word(uint64_t *w) { return reinterpret_cast<uint32_t *>(w) + 1; }
 __host__ __device__ __forceinline__ uint64_t make_hot(uint64_t size, uint64_t ext, uint32_t flags) {
   return (size >= BIG_SIZE ? (uint64_t)BIG_SIZE : size) | ((ext & EXT_MASK) << ESHIFT) | ((uint64_t)flags << FSHIFT);
+}
+
+// Compact unit word (hotc[u], 4 bytes, what k_map_pd gathers: half the bytes of hot keeps E's forward
+// working set nearer the L2): size (bits 0..17) | extent id (18..28) | ACTIVE (29) | STORAGE (30);
+// HOTC_ESC (bit 31) when the size or the extent id does not fit -- then hot[u] is read.  Every writer of
+// hot's size / extent / ACTIVE / STORAGE rewrites it (k_remap, k_set_ext, k_deactivate, k_hotc_ops).
+constexpr uint32_t HOTC_ESC = 0x80000000u;
+__host__ __device__ __forceinline__ uint32_t make_hotc(uint64_t h) {
+  const uint32_t size = hot_size32(h), ext = hot_ext(h), fl = hot_flags(h);
+  const bool stg = (fl & UF_STORAGE) != 0;
+  if (size >= (1u << 18) || (stg && ext >= (1u << 11))) return HOTC_ESC;
+  return size | ((stg ? ext : 0u) << 18) | ((fl & UF_ACTIVE) ? 1u << 29 : 0u) | (stg ? 1u << 30 : 0u);
+}
+// the hot word a compact word stands for, as far as the forward map reads it (size, extent, ACTIVE, STORAGE)
+__host__ __device__ __forceinline__ uint64_t hot_of_hotc(uint32_t c) {
+  const uint32_t fl = ((c >> 29) & 1u ? UF_ACTIVE : 0u) | ((c >> 30) & 1u ? UF_STORAGE : 0u);
+  return (uint64_t)(c & ((1u << 18) - 1)) | ((uint64_t)((c >> 18) & 0x7FFu) << ESHIFT) | ((uint64_t)fl << FSHIFT);
 }
 
 // Sorted-key search index, built by the host (top level, directory) and the device (levels):

@@ -961,8 +961,24 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
     for (int m = 0; m < 2; ++m) {
       pd_back(a.pd, pol_t, fr[m], cv[m], ew[m], j[m], key[m], k0[m]);
       look[m] = look[m] && j[m] >= 0;
+#ifdef CGCM_NO_HOTC
       if (look[m]) hw[m] = ld_u64_hot(a.tab.hot + j[m], pol_t);
+#else
+      if (look[m]) {  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
+        uint32_t c;
+        asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(c) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
+        hw[m] = c;  // decoded below, once both gathers are in flight
+      }
+#endif
     }
+#ifndef CGCM_NO_HOTC
+#pragma unroll
+    for (int m = 0; m < 2; ++m)
+      if (look[m]) {
+        const uint32_t c = (uint32_t)hw[m];
+        hw[m] = (c & HOTC_ESC) ? ld_u64_hot(a.tab.hot + j[m], pol_t) : hot_of_hotc(c);
+      }
+#endif
     bool hit[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
@@ -1455,11 +1471,13 @@ __global__ void k_remap(int n, const int32_t *old_idx, const uint64_t *size, con
   int k = old_idx[i];
   if (k >= 0) {
     t.hot[i] = o.hot[k];
+    t.hotc[i] = make_hotc(o.hot[k]);
     t.st[i] = o.st[k];
     t.rc[i] = o.rc[k];
   } else {
     const uint64_t h = make_hot(size[i], NO_EXT, flags[i]);
     t.hot[i] = h;
+    t.hotc[i] = make_hotc(h);
     t.st[i] = make_st(h, epoch0[i]);
     t.rc[i] = 0;
   }
@@ -1502,10 +1520,18 @@ __global__ void k_unit_ops(const UnitOp *ops, int n, TableDev tab) {
     case UOP_SET_RC: tab.rc[o.unit] = (int32_t)(int64_t)o.val; break;
   }
 }
+// after k_unit_ops: the compact words of every unit whose flags an op changed (from the final hot word)
+__global__ void k_hotc_ops(const UnitOp *ops, int n, TableDev tab) {
+  int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const UnitOp o = ops[i];
+  if (o.op == UOP_OR_FLAGS || o.op == UOP_AND_FLAGS) tab.hotc[o.unit] = make_hotc(tab.hot[o.unit]);
+}
 void launch_unit_ops(const UnitOp *ops, int n, TableDev tab, cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
     k_unit_ops<<<(n + 255) / 256, 256, 0, s>>>(ops, n, tab);
+    k_hotc_ops<<<(n + 255) / 256, 256, 0, s>>>(ops, n, tab);
   }
 }
 
@@ -1519,6 +1545,7 @@ __global__ void k_set_ext(const uint32_t *units, const uint32_t *exts, int n, Ta
   h = (h & ~(EXT_MASK << ESHIFT)) | ((uint64_t)(exts[i] & EXT_MASK) << ESHIFT);
   h |= (uint64_t)(UF_STORAGE | UF_ACTIVE) << FSHIFT;
   tab.hot[u] = h;
+  tab.hotc[u] = make_hotc(h);
   tab.st[u] = make_st(h, set_epoch ? epoch : st_epoch(tab.st[u]));
 }
 void launch_set_ext(const uint32_t *units, const uint32_t *exts, int n, TableDev tab, uint32_t epoch, int set_epoch,
@@ -1542,6 +1569,7 @@ __global__ void k_deactivate(const uint32_t *units, int n, TableDev tab) {
     h |= NO_EXT << ESHIFT;
   }
   tab.hot[u] = h;
+  tab.hotc[u] = make_hotc(h);
   tab.st[u] = make_st(h, st_epoch(tab.st[u]));
 }
 void launch_deactivate(const uint32_t *units, int n, TableDev tab, cudaStream_t s) {

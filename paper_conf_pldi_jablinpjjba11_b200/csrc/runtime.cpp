@@ -220,7 +220,7 @@ struct Context {
   int U = 0;  // units in the device table
 
   // device table
-  DevBuf hotb, stb, rcb, size64, dbase, extd, snap_st, snap_rc;  // unit table columns + extent deltas
+  DevBuf hotb, hotcb, stb, rcb, size64, dbase, extd, snap_st, snap_rc;  // unit table columns + extent deltas
   size_t extd_n = 0;                          // entries uploaded to extd
   IndexBufs fwd, rev;
   // page directory over the unit bases (cgcm_dev.h PdDev; built with the table)
@@ -281,6 +281,7 @@ struct Context {
   TableDev tab() const {
     TableDev t;
     t.hot = hotb.as<uint64_t>();
+    t.hotc = hotcb.as<uint32_t>();
     t.st = stb.as<uint64_t>();
     t.rc = rcb.as<int32_t>();
     t.base = dbase.as<uint64_t>();
@@ -578,9 +579,10 @@ struct Context {
     udev.swap(ndev);
     urun.swap(nrun);
     uarr.swap(narr);
-    DevBuf nhot, nst, nrc, nsize, nbase, tmp;
+    DevBuf nhot, nhotc, nst, nrc, nsize, nbase, tmp;
     int cap = std::max(n, 1);
     CKS(dalloc(nhot, 8 * (size_t)cap + 64));
+    CKS(dalloc(nhotc, 4 * (size_t)cap + 64));
     CKS(dalloc(nst, 8 * (size_t)cap + 64));
     CKS(dalloc(nrc, 4 * (size_t)cap + 64));
     CKS(dalloc(nsize, 8 * (size_t)cap));
@@ -595,6 +597,7 @@ struct Context {
       const uint32_t *dflags = reinterpret_cast<const uint32_t *>(dold + n);
       TableDev nt = tab();
       nt.hot = nhot.as<uint64_t>();
+      nt.hotc = nhotc.as<uint32_t>();
       nt.st = nst.as<uint64_t>();
       nt.rc = nrc.as<int32_t>();
       launch_remap(n, dold, nsize.as<uint64_t>(), dflags, depoch, tab(), nt, main);
@@ -604,11 +607,13 @@ struct Context {
     }
     dfree(tmp);
     dfree(hotb);
+    dfree(hotcb);
     dfree(stb);
     dfree(rcb);
     dfree(size64);
     dfree(dbase);
     hotb = nhot;
+    hotcb = nhotc;
     stb = nst;
     rcb = nrc;
     size64 = nsize;
@@ -873,7 +878,7 @@ struct Context {
     if (ops.empty()) return CGCM_OK;
     CKS(upload(uops, ops));
     launch_unit_ops(uops.as<UnitOp>(), (int)ops.size(), tab(), main);
-    st.kernel_launches += 1;
+    st.kernel_launches += 2;  // + the compact unit words (k_hotc_ops)
     CK(cudaGetLastError());
     return CGCM_OK;
   }
