@@ -235,6 +235,37 @@ __global__ void __launch_bounds__(768, 1)
                  : "memory");
   }
 }
+
+// forward with ONE returning 64-bit atomic per slot on {rc | unit word} instead of unit-word gather + RED
+__global__ void __launch_bounds__(768, 1)
+    k_skel_atom(uint64_t *slots, uint64_t nchunks, const uint64_t *ent, uint64_t nent, unsigned long long *rch,
+                uint64_t nunit, uint64_t *shp, uint32_t *shu) {
+  const uint64_t pl = pol_last(), pf = pol_first();
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; c < nchunks; c += stride) {
+    uint64_t x0, x1;
+    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;"
+                 : "=l"(x0), "=l"(x1)
+                 : "l"(slots + 2 * c), "l"(pf));
+    uint64_t a = mix(x0 + 2 * c), b = mix(x1 + 2 * c + 1);
+    uint64_t va[4], vb[4];
+    ld32(ent + 4 * (a % nent), pl, va);
+    ld32(ent + 4 * (b % nent), pl, vb);
+    a = mix(a ^ va[0]);
+    b = mix(b ^ vb[0]);
+    const uint64_t ia = a % nunit, ib = b % nunit;
+    const unsigned long long ha = atomicAdd(rch + ia, 1ull), hb = atomicAdd(rch + ib, 1ull);
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u64 [%0], {%1,%2}, %3;" ::"l"(shp + 2 * c), "l"(x0),
+                 "l"(x1), "l"(pf)
+                 : "memory");
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1,%2}, %3;" ::"l"(shu + 2 * c),
+                 "r"((uint32_t)ia), "r"((uint32_t)ib), "l"(pf)
+                 : "memory");
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u64 [%0], {%1,%2}, %3;" ::"l"(slots + 2 * c),
+                 "l"(x0 + (ha >> 32)), "l"(x1 + (hb >> 32)), "l"(pf)
+                 : "memory");
+  }
+}
 __global__ void k_fill_units(uint32_t *u, uint64_t n, uint32_t nrec) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
     u[i] = (uint32_t)(mix(i) % nrec);
@@ -364,7 +395,7 @@ int main(int argc, char **argv) {
     rev(k_skeleton_rev<true, true, true, false, true, true>, "scalar shadow+gather+red(separate)");
     // page-directory forward skeletons: config E (39 MiB entries, 2^22 units) and C (10 MiB, 2^20)
     for (int cfg = 0; cfg < 2; ++cfg) {
-      const uint64_t nent = cfg == 0 ? (78ull << 20) / 32 : (20ull << 20) / 32, nunit = cfg == 0 ? 1ull << 22 : 1ull << 20;
+      const uint64_t nent = cfg == 0 ? (39ull << 20) / 32 : (10ull << 20) / 32, nunit = cfg == 0 ? 1ull << 22 : 1ull << 20;
       uint64_t *ent, *hot;
       int32_t *rcs;
       CK(cudaMalloc(&ent, 32 * nent));
@@ -384,6 +415,20 @@ int main(int argc, char **argv) {
                cfg == 0 ? "E" : "C", what, (unsigned long long)nslots, ms, nslots / ms / 1e6);
       };
       pd(k_skel_pd<true, true, true, true>, "ent+hot+red+shadow");
+      {
+        unsigned long long *rch;
+        CK(cudaMalloc(&rch, 8 * nunit));
+        CK(cudaMemset(rch, 0, 8 * nunit));
+        k_skel_atom<<<nsm, 768>>>(slots, nslots / 2, ent, nent, rch, nunit, shp, shu);
+        CK(cudaEventRecord(e0));
+        for (int r = 0; r < 5; ++r) k_skel_atom<<<nsm, 768>>>(slots, nslots / 2, ent, nent, rch, nunit, shp, shu);
+        CK(cudaEventRecord(e1));
+        CK(cudaEventSynchronize(e1));
+        double ms = time_ms(e0, e1) / 5;
+        printf("{\"test\": \"skeleton_pd\", \"cfg\": \"%s\", \"parts\": \"ent+atom64(rc|unit)+shadow\", \"ms\": %.3f}\n",
+               cfg == 0 ? "E" : "C", ms);
+        CK(cudaFree(rch));
+      }
       pd(k_skel_pd<true, false, true, true, true>, "ent64+red+shadow");
       pd(k_skel_pd<true, false, true, false, true>, "ent64+red");
       pd(k_skel_pd<true, false, true, true>, "ent+red+shadow");
