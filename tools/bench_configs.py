@@ -167,9 +167,11 @@ if __name__ == "__main__":
     which = sys.argv[1:] or ["A", "B", "D"]
     for w in which:
         if w == "A":
+            config_A("promoted", iters=3)  # warm-up: lazy module loading, clocks (not reported)
             for m in ("naive", "promoted", "region", "region_check"):
                 print(json.dumps(config_A(m)), flush=True)
         elif w == "B":
+            config_B(True, n=256)  # warm-up: lazy module loading of the sample gemm, clocks (not reported)
             for p in (True, False):
                 print(json.dumps(config_B(p)), flush=True)
         elif w == "D":
