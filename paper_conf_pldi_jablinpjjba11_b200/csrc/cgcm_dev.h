@@ -232,7 +232,8 @@ void launch_remap(int n, const int32_t *old_idx, const uint64_t *size, const uin
                   TableDev old_tab, TableDev new_tab, cudaStream_t s);
 size_t sort_keys_temp_bytes(int n);
 void launch_sort_keys(void *temp, size_t temp_bytes, const uint32_t *kin, uint32_t *kout, int n, cudaStream_t s);
-void launch_unit_ops(const UnitOp *ops, int n, TableDev tab, cudaStream_t s);
+// hotc: also rewrite the compact unit words (an op changes ACTIVE or STORAGE)
+void launch_unit_ops(const UnitOp *ops, int n, TableDev tab, cudaStream_t s, bool hotc);
 void launch_set_ext(const uint32_t *units, const uint32_t *exts, int n, TableDev tab, uint32_t epoch, int set_epoch,
                     cudaStream_t s);
 void launch_deactivate(const uint32_t *units, int n, TableDev tab, cudaStream_t s);

@@ -1527,11 +1527,11 @@ __global__ void k_hotc_ops(const UnitOp *ops, int n, TableDev tab) {
   const UnitOp o = ops[i];
   if (o.op == UOP_OR_FLAGS || o.op == UOP_AND_FLAGS) tab.hotc[o.unit] = make_hotc(tab.hot[o.unit]);
 }
-void launch_unit_ops(const UnitOp *ops, int n, TableDev tab, cudaStream_t s) {
+void launch_unit_ops(const UnitOp *ops, int n, TableDev tab, cudaStream_t s, bool hotc) {
   if (n > 0) {
     (void)cudaGetLastError();
     k_unit_ops<<<(n + 255) / 256, 256, 0, s>>>(ops, n, tab);
-    k_hotc_ops<<<(n + 255) / 256, 256, 0, s>>>(ops, n, tab);
+    if (hotc) k_hotc_ops<<<(n + 255) / 256, 256, 0, s>>>(ops, n, tab);
   }
 }
 

@@ -877,8 +877,13 @@ struct Context {
   int unit_ops(const std::vector<UnitOp> &ops) {
     if (ops.empty()) return CGCM_OK;
     CKS(upload(uops, ops));
-    launch_unit_ops(uops.as<UnitOp>(), (int)ops.size(), tab(), main);
-    st.kernel_launches += 2;  // + the compact unit words (k_hotc_ops)
+    // the compact unit words need rewriting only if an op changes ACTIVE or STORAGE (cgcm_dev.h make_hotc)
+    bool hotc = false;
+    for (auto &o : ops)
+      hotc = hotc || (o.op == UOP_OR_FLAGS && (o.val & (UF_ACTIVE | UF_STORAGE))) ||
+             (o.op == UOP_AND_FLAGS && (~o.val & (UF_ACTIVE | UF_STORAGE)));
+    launch_unit_ops(uops.as<UnitOp>(), (int)ops.size(), tab(), main, hotc);
+    st.kernel_launches += hotc ? 2 : 1;
     CK(cudaGetLastError());
     return CGCM_OK;
   }
@@ -2046,7 +2051,7 @@ int cgcm_releaseBatch(const void *const *cpu, size_t n) {
   c.dir = DIR_FWD;
   c.ops = OP_DEC;
   c.segs = {Seg{d, n, 0, 1, 0}};
-  c.dec_red = n >= (size_t)C->U / 8;
+  c.dec_red = n >= (size_t)C->U / 8 && C->U >= 4096;  // small tables: returning atomics, no scan launch
   CKS(C->launch(c, 0));
   Status sts[8];
   unsigned long long lcs[4];
@@ -2393,7 +2398,7 @@ int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
   SlotCall R, F;
   R.dir = DIR_REV; R.ops = OP_DEC; R.segs = rsegs;
   F.dir = DIR_FWD; F.ops = OP_DEC; F.segs = fsegs;
-  R.dec_red = F.dec_red = total >= (uint64_t)C->U / 8;
+  R.dec_red = F.dec_red = total >= (uint64_t)C->U / 8 && C->U >= 4096;
   CKS(C->launch(R, 0));
   CKS(C->launch(F, 1));
   Status sts[8];
