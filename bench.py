@@ -421,7 +421,7 @@ def run_reference(args, rank, world):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=30)  # ~200 ms timed at E: several clock samples
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="cgcm", choices=["cgcm", "reference"])
     ap.add_argument("--config", default="E", choices=sorted(CONFIGS))
