@@ -227,9 +227,26 @@ def run_cgcm(args, rank, world, local_rank):
     roofline["l2_random_ops"] = l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots)
     gpu_launches = int(st["kernel_launches"])
 
+    # the e2e legs run on fresh contexts without CGCM_PROFILE (its per-launch event syncs would serialise
+    # the host threads of the duplex leg); the hot-path context is released first
+    ctx.close()
     e2e = None
     if not args.no_e2e:
-        e2e = run_e2e(args, ctx, wl, q_ref, dev, world, rank)
+        ctxa = table_context(wl, dev, local_rank, wl.n)
+        try:
+            e2e = run_e2e(args, ctxa, wl, q_ref, dev, world, rank)
+            if not args.no_duplex:
+                try:
+                    dup = run_e2e_duplex(args, ctxa, wl, q_ref, dev, world, rank, e2e["host_link"], local_rank)
+                except Exception as ex:  # e.g. not enough device memory for a second replica
+                    dup = None
+                    e2e["duplex_error"] = str(ex)[:200]
+                if dup is not None:
+                    dup["single_context"] = e2e
+                    e2e = dup
+        finally:
+            ctxa.make_current()
+            ctxa.close()
 
     result = {
         "metric": METRIC, "value": round(value, 1), "unit": "pointer translations/s",
@@ -246,7 +263,6 @@ def run_cgcm(args, rank, world, local_rank):
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         result["cpu_baseline"] = cpu_baseline(wl, args.cpu_sample, steps=1)
-    ctx.close()
     return result
 
 
@@ -275,13 +291,34 @@ def l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots):
             "rev_frac": round(rev_floor / rev_ms, 4) if rev_ms else None}
 
 
-def host_link(dev, nbytes=256 << 20, reps=5):
-    """Pinned host<->device copy bandwidth of this GPU's link (best of reps, CUDA events)."""
+def host_link(dev, nbytes=256 << 20, reps=10):
+    """Pinned host<->device copy bandwidth of this GPU's link (256 MiB, best of 10, CUDA
+    events): H2D, D2H, and both directions at once on two streams (bidir = total bytes / span)."""
     import torch
     h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
     d = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    h2 = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d2 = torch.empty(nbytes, dtype=torch.uint8, device=dev)
     s = torch.cuda.Stream(device=dev)
-    out = {}
+    s2 = torch.cuda.Stream(device=dev)
+    best = None
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e2 = torch.cuda.Event()
+        torch.cuda.synchronize(dev)
+        e0.record(s)
+        s2.wait_event(e0)
+        with torch.cuda.stream(s):
+            d.copy_(h, non_blocking=True)
+        with torch.cuda.stream(s2):
+            h2.copy_(d2, non_blocking=True)
+        e2.record(s2)
+        s.wait_event(e2)
+        e1.record(s)
+        e1.synchronize()
+        ms = e0.elapsed_time(e1)
+        best = ms if best is None else min(best, ms)
+    out = {"bidir_gbs": round(2 * nbytes / (best / 1e3) / 1e9, 1)}
     for name, fn in (("h2d", lambda: d.copy_(h, non_blocking=True)), ("d2h", lambda: h.copy_(d, non_blocking=True))):
         best = None
         for _ in range(reps):
@@ -352,6 +389,129 @@ def run_e2e(args, ctx, wl, q_ref, dev, world, rank):
             "frac_of_host_link": round(floor_ms / (ms / steps), 4),
             "ms_per_step": round(ms / steps, 3), "steps": steps,
             "api": "cgcm_mapArrays+advanceEpoch+cgcm_unmapArrays+cgcm_releaseArrays (pinned host arrays)",
+            "host_arrays_roundtrip_ok": bool(ok)}
+
+
+def table_context(wl, dev, local_rank, nslots):
+    """A context holding the workload's table, every unit kept active by one setup reference (as the
+    hot-path context), with arena room for nslots pointer slots of arrays and their scratch."""
+    import torch
+    import paper_conf_pldi_jablinpjjba11_b200 as cg
+    c = cg.Context(local_rank, arena_bytes=int(wl.sizes.sum()) + wl.span // 8 + nslots * 8 * 4 + (6 << 30))
+    assert c.declareBatch(wl.bases, wl.sizes, readonly=True) == 0
+    pins = torch.from_numpy(wl.bases.view(np.int64).copy()).to(dev)
+    s = c.mapArrayDevice(pins.data_ptr(), wl.U)
+    assert s == 0, cg.strerror(s)
+    torch.cuda.synchronize()
+    return c
+
+
+def run_e2e_duplex(args, ctx, wl, q_ref, dev, world, rank, link, local_rank):
+    """The e2e step with both directions of the (full-duplex) host link busy: the rank's arrays are
+    split into two halves, each driven through its own context (its own replica of the table, arena
+    and streams) by its own host thread, the second half one phase behind the first -- while one half
+    copies its translated arrays back (unmapArrays), the other uploads its raw arrays (mapArrays).
+    Same public calls, same bytes every step; CUDA events on the first context's main stream span
+    both threads."""
+    import ctypes
+    import threading
+    import torch
+    import paper_conf_pldi_jablinpjjba11_b200 as cg
+    A, S = wl.arrays_per_rank, wl.slots
+    if A < 2:
+        return None
+    host = np.ascontiguousarray(q_ref.cpu().numpy().view(np.uint64))
+    ctx2 = table_context(wl, dev, local_rank, (A // 2) * S)
+    try:
+        halves = [(ctx, list(range(0, A // 2))), (ctx2, list(range(A // 2, A)))]
+        outers = [[], []]
+        for k, (c, rng) in enumerate(halves):
+            c.make_current()
+            for a in rng:
+                p = c.malloc(8 * S)
+                assert p, "cgcm_malloc failed"
+                ctypes.memmove(p, host[a * S:(a + 1) * S].ctypes.data, 8 * S)
+                outers[k].append(p)
+        errs = []
+
+        trace = [] if os.environ.get("CGCM_BENCH_TRACE") else None
+
+        def step(k):
+            c, o = halves[k][0], outers[k]
+            t0 = time.perf_counter()
+            s1, _ = c.mapArrays(o)
+            if k == 0 and not lag.is_set():
+                lag.set()  # the second half starts once the first half's upload is done
+            c.advanceEpoch()
+            t1 = time.perf_counter()
+            s2 = c.unmapArrays(o)
+            t2 = time.perf_counter()
+            s3 = c.releaseArrays(o)
+            if trace is not None:
+                trace.append((k, round(1e3 * t0, 1), round(1e3 * t1, 1), round(1e3 * t2, 1), round(1e3 * time.perf_counter(), 1)))
+            if s1 or s2 or s3:
+                errs.append((k, s1, s2, s3, c.L.cgcm_lastCudaError().decode()))
+
+        def worker(k, steps):
+            halves[k][0].make_current()
+            if k == 1:
+                lag.wait()
+            for _ in range(steps):
+                step(k)
+
+        lag = threading.Event()
+        lag.set()
+        for k in (0, 1):  # warm-up, one half at a time
+            halves[k][0].make_current()
+            step(k)
+        torch.cuda.synchronize()
+        steps = max(1, min(args.steps, args.e2e_steps))
+        st0 = [c.stats() for c, _ in halves]
+        lag.clear()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev2 = torch.cuda.Event()
+        ev0.record(ctx.main)
+        ts = [threading.Thread(target=worker, args=(k, steps)) for k in (0, 1)]
+        for t in ts:
+            t.start()
+        for t in ts:
+            t.join()
+        ev2.record(ctx2.main)
+        ctx.main.wait_event(ev2)
+        ev1.record(ctx.main)
+        torch.cuda.synchronize()
+        if errs:
+            raise RuntimeError(f"e2e duplex step failed: {errs[0]}")
+        if trace:
+            z = min(x[1] for x in trace)
+            for x in sorted(trace, key=lambda r: r[1]):
+                print("duplex", x[0], [round(v - z, 1) for v in x[1:]], file=sys.stderr)
+        ms = ev0.elapsed_time(ev1)
+        st1 = [c.stats() for c, _ in halves]
+        ok = all(np.array_equal(np.ctypeslib.as_array((ctypes.c_uint64 * S).from_address(p)), host[a * S:(a + 1) * S])
+                 for k in (0, 1) for a, p in zip(halves[k][1], outers[k]))
+        for k in (0, 1):
+            halves[k][0].make_current()
+            for p in outers[k]:
+                halves[k][0].free(p)
+    finally:
+        ctx2.close()
+        ctx.make_current()
+    if world > 1:
+        import torch.distributed as dist
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    h2d = sum(b["h2d_bytes"] - a["h2d_bytes"] for a, b in zip(st0, st1)) // steps
+    d2h = sum(b["d2h_bytes"] - a["d2h_bytes"] for a, b in zip(st0, st1)) // steps
+    floor_ms = 1e3 * (h2d + d2h) / (link["bidir_gbs"] * 1e9)  # both directions busy at once
+    return {"value": round(2 * wl.n * world * steps / (ms / 1e3), 1), "unit": "pointer translations/s",
+            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+            "host_link": link, "host_link_floor_ms_per_step": round(floor_ms, 3),
+            "frac_of_host_link": round(floor_ms / (ms / steps), 4),
+            "ms_per_step": round(ms / steps, 3), "steps": steps,
+            "api": "cgcm_mapArrays+advanceEpoch+cgcm_unmapArrays+cgcm_releaseArrays (pinned host arrays), "
+                   "two halves through two contexts, one phase apart (full-duplex link)",
             "host_arrays_roundtrip_ok": bool(ok)}
 
 
@@ -426,6 +586,7 @@ def main():
     ap.add_argument("--impl", default="cgcm", choices=["cgcm", "reference"])
     ap.add_argument("--config", default="E", choices=sorted(CONFIGS))
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-duplex", action="store_true", help="e2e through one context only")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=1 << 21)

@@ -242,5 +242,8 @@ void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n
 void launch_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
                          cudaStream_t s);
 void launch_rebase_epochs(TableDev tab, int n, uint32_t cur, cudaStream_t s);
+// small host<->device transfers by a kernel through mapped pinned memory instead of a DMA: a copy
+// engine serves DMAs in order, so a few bytes queued behind another context's gigabyte would wait for it
+void launch_copy_small(void *dst, const void *src, size_t n, void *dst2, const void *src2, size_t n2, cudaStream_t s);
 
 }  // namespace cgcm

@@ -14,6 +14,7 @@
 // DESIGN.md §7 gives the roofline of each kernel and its algorithmic bytes.
 #include <cub/cub.cuh>
 
+#include <algorithm>
 #include <cstdlib>
 
 #include "cgcm_dev.h"
@@ -1667,6 +1668,34 @@ void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n
     (void)cudaGetLastError();
     k_lookup_points<<<(n + 127) / 128, 128, 0, s>>>(ix, tab, ptrs, n, out);
   }
+}
+
+// up to two byte ranges (either side may be mapped pinned host memory); 16-byte words when aligned
+__global__ void k_copy_small(unsigned char *dst, const unsigned char *src, size_t n, unsigned char *dst2,
+                             const unsigned char *src2, size_t n2) {
+  const size_t t = (size_t)blockIdx.x * blockDim.x + threadIdx.x, str = (size_t)gridDim.x * blockDim.x;
+  for (int r = 0; r < 2; ++r) {
+    unsigned char *d = r ? dst2 : dst;
+    const unsigned char *q = r ? src2 : src;
+    const size_t m = r ? n2 : n;
+    if (!m) continue;
+    if ((((uintptr_t)d | (uintptr_t)q) & 15) == 0) {
+      const size_t w = m / 16;
+      for (size_t i = t; i < w; i += str) reinterpret_cast<uint4 *>(d)[i] = reinterpret_cast<const uint4 *>(q)[i];
+      for (size_t i = 16 * w + t; i < m; i += str) d[i] = q[i];
+    } else {
+      for (size_t i = t; i < m; i += str) d[i] = q[i];
+    }
+  }
+}
+void launch_copy_small(void *dst, const void *src, size_t n, void *dst2, const void *src2, size_t n2, cudaStream_t s) {
+  const size_t words = (std::max(n, n2) + 15) / 16;
+  const int threads = 256;
+  const int blocks = (int)std::min<size_t>((words + threads - 1) / threads, 64);
+  k_copy_small<<<blocks > 0 ? blocks : 1, threads, 0, s>>>(static_cast<unsigned char *>(dst),
+                                                            static_cast<const unsigned char *>(src), n,
+                                                            static_cast<unsigned char *>(dst2),
+                                                            static_cast<const unsigned char *>(src2), n2);
 }
 
 }  // namespace cgcm

@@ -135,7 +135,7 @@ struct HostBuf {
     if (need <= bytes) return CGCM_OK;
     if (p) cudaFreeHost(p);
     size_t nb = std::max<size_t>(need, std::max<size_t>(bytes * 3 / 2, 1 << 16));
-    if (cudaHostAlloc(&p, nb, cudaHostAllocPortable) != cudaSuccess) {
+    if (cudaHostAlloc(&p, nb, cudaHostAllocPortable | cudaHostAllocMapped) != cudaSuccess) {
       p = nullptr;
       bytes = 0;
       return CGCM_E_NOMEM;
@@ -700,9 +700,9 @@ struct Context {
     // each launch uses its own eighth of the segment buffers (st_index 0..7, up to 8 launches in flight)
     Seg *dsegs = segs.as<Seg>() + (size_t)st_index * k;
     uint64_t *dc0 = seg0.as<uint64_t>() + (size_t)st_index * (k + 1);
-    // pinned ring (no host wait) unless the outers' H2D copies are in flight on the copy stream: a
-    // pinned upload is a DMA that would queue behind them, while a small pageable copy is not
-    if (c.seg_group.empty() && sizeof(Seg) * k + 8 * (size_t)(k + 1) <= RING_HALF / 2) {
+    // pinned ring: no host wait, and no DMA (read by a kernel) -- also while the outers' H2D copies
+    // are in flight on the copy stream
+    if (sizeof(Seg) * k + 8 * (size_t)(k + 1) <= RING_HALF / 2) {
       CKS(ring_put(dsegs, c.segs.data(), sizeof(Seg) * k));
       CKS(ring_put(dc0, c0.data(), 8 * (size_t)(k + 1)));
     } else {
@@ -825,8 +825,11 @@ struct Context {
   }
   // fetch the 8 Status blocks + list counters (synchronizes main)
   int fetch_status(Status out[8], unsigned long long lcs[4]) {
-    CK(cudaMemcpyAsync(h_status.p, status.as<void>(), sizeof(Status) * 8, cudaMemcpyDeviceToHost, main));
-    CK(cudaMemcpyAsync(h_status.as<char>() + sizeof(Status) * 8, lc.as<void>(), 32, cudaMemcpyDeviceToHost, main));
+    // a kernel writes them into mapped pinned memory: no DMA to queue behind other copies (cgcm_dev.h)
+    launch_copy_small(h_status.p, status.as<void>(), sizeof(Status) * 8, h_status.as<char>() + sizeof(Status) * 8,
+                      lc.as<void>(), 32, main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
     CK(cudaStreamSynchronize(main));
     std::memcpy(out, h_status.p, sizeof(Status) * 8);
     std::memcpy(lcs, h_status.as<char>() + sizeof(Status) * 8, 32);
@@ -838,7 +841,13 @@ struct Context {
     out.resize(n);
     if (!n) return CGCM_OK;
     CKS(h_list.ensure(sizeof(T) * n));
-    CK(cudaMemcpyAsync(h_list.p, src.as<void>(), sizeof(T) * n, cudaMemcpyDeviceToHost, main));
+    if (sizeof(T) * n <= (64u << 10)) {  // small: by a kernel into mapped pinned memory (no DMA queueing)
+      launch_copy_small(h_list.p, src.as<void>(), sizeof(T) * n, nullptr, nullptr, 0, main);
+      st.kernel_launches += 1;
+      CK(cudaGetLastError());
+    } else {
+      CK(cudaMemcpyAsync(h_list.p, src.as<void>(), sizeof(T) * n, cudaMemcpyDeviceToHost, main));
+    }
     CK(cudaStreamSynchronize(main));
     std::memcpy(out.data(), h_list.p, sizeof(T) * n);
     return CGCM_OK;
@@ -859,7 +868,10 @@ struct Context {
     char *p = h_ring.as<char>() + (size_t)ring_cur * RING_HALF + ring_head;
     std::memcpy(p, src, n);
     ring_head += (n + 255) & ~(size_t)255;
-    CK(cudaMemcpyAsync(dst, p, n, cudaMemcpyHostToDevice, main));
+    // read by a kernel from mapped pinned memory: no DMA to queue behind other H2D copies
+    launch_copy_small(dst, p, n, nullptr, nullptr, 0, main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
     return CGCM_OK;
   }
   template <class T>
