@@ -587,7 +587,7 @@ def main():
     ap.add_argument("--config", default="E", choices=sorted(CONFIGS))
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-duplex", action="store_true", help="e2e through one context only")
-    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=6)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=1 << 21)
     ap.add_argument("--ref-sample", type=int, default=1 << 19)
