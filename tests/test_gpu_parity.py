@@ -693,3 +693,24 @@ def test_region_checker_counts_cpu_accesses(pair):
     assert P.o.unmap(base) == 0 and P.o.release(base) == 0
     P.check("after checked region")
     assert P.g.regionEnd()[0] == -1                                       # no open region
+
+
+def test_many_small_arrays_cycle_the_upload_ring(pair):
+    """Thousands of small outers per call: every call uploads ~100s of KB of pointers, unit ops and
+    segment tables through the pinned staging ring, so its halves are retired and reused (event
+    fences) many times; every state vs the oracle after each cycle."""
+    P = pair
+    rows = [P.malloc(64, np.arange(8, dtype=np.float64) + r) for r in range(64)]
+    outers = []
+    for k in range(3000):
+        sl = np.array([rows[(k * 7 + i) % 64] + 8 * (i % 8) for i in range(4)], dtype=np.uint64)
+        outers.append(P.malloc(32, sl))
+    for cyc in range(5):
+        st, d = P.run("mapArrays", outers)
+        P.advance()
+        P.run("unmapArrays", outers)
+        P.run("releaseArrays", outers)
+        if cyc % 2 == 0:
+            P.check(f"cycle {cyc}")
+    P.check("end")
+    assert all(u["refCount"] == 0 for u in P.g.dump())
