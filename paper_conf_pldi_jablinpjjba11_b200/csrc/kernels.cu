@@ -751,9 +751,12 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
       const bool vm = (valid >> m) & 1;
       const bool hm = vm && hit[m];
       const bool nul = vm && v[m] == 0;
-      c_nulls += nul;
-      c_hits += hm;
-      c_miss += (vm && !nul && !hm);
+      // a forward pass with inc = k stands for k sequential mapArray calls of one outer (a batch
+      // naming it k times): each call maps -- and counts -- every slot (Alg. 1 per slot, A8)
+      const unsigned w = (OPS & (OP_INC | OP_INCPLAIN)) ? (unsigned)sg.inc : 1u;
+      c_nulls += nul * w;
+      c_hits += hm * w;
+      c_miss += (vm && !nul && !hm) * w;
       const int unit = hm ? j[m] : 0;
       int32_t *RC = a.tab.rc + unit;
       const uint32_t fl = hot_flags(hw[m]);
@@ -1011,9 +1014,9 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
     for (int m = 0; m < 2; ++m) {
       const bool vm = (valid >> m) & 1;
       const bool nul = vm && cv[m] == 0;
-      c_nulls += nul;
-      c_hits += hit[m];
-      c_miss += (vm && !nul && !hit[m]);
+      c_nulls += nul * (unsigned)sg.inc;  // inc = k: k sequential mapArray calls (see k_slots)
+      c_hits += hit[m] * (unsigned)sg.inc;
+      c_miss += (vm && !nul && !hit[m]) * (unsigned)sg.inc;
       const uint32_t fl = hot_flags(hw[m]);
       bool act = false;
       if (hit[m]) {

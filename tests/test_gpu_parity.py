@@ -714,3 +714,65 @@ def test_many_small_arrays_cycle_the_upload_ring(pair):
             P.check(f"cycle {cyc}")
     P.check("end")
     assert all(u["refCount"] == 0 for u in P.g.dump())
+
+
+def test_degenerate_batches(pair):
+    """Edge cases of the batch forms (SURVEY §8(b) "data-parallel batch forms (same semantics as the
+    sequential loop)"): empty batches, all-NULL batches and arrays, outer AUs with 0 / 1 slot and a
+    trailing partial word (A10: the ⌊size/8⌋ words are slots, trailing bytes verbatim), adjacent AUs
+    where one's one-past-the-end address is the next one's base (A7 greatestLTE picks the later base),
+    and one outer named twice in one mapArrays batch (sequential semantics: two references)."""
+    P = pair
+    buf = HostBuf(1 << 16)
+    for name in ("mapBatch", "unmapBatch", "releaseBatch", "mapArrays", "unmapArrays", "releaseArrays"):
+        st = P.run(name, [])
+        assert (st[0] if isinstance(st, tuple) else st) == 0, name
+    P.check("empty batches")
+    P.run("mapBatch", [0, 0, 0])
+    P.check("all-NULL batch")
+    a, b = buf.addr + 0x1000, buf.addr + 0x1040           # a ends exactly at b's base
+    P.declare(a, 64, np.arange(8, dtype=np.uint64))
+    P.declare(b, 40, np.arange(5, dtype=np.uint64) + 100)
+    st, d = P.run("mapBatch", [a + 64, a + 63, b + 40, b])
+    assert st == 0
+    P.check("adjacent boundary")
+    nul = buf.addr + 0x2000
+    P.declare(nul, 8 * 64)                                # 64 NULL slots
+    one = buf.addr + 0x3000
+    P.declare(one, 8, np.array([a + 8], dtype=np.uint64))
+    tiny = buf.addr + 0x3100
+    P.declare(tiny, 4, np.array([7, 7, 7, 7], dtype=np.uint8))  # no whole slot
+    rag = buf.addr + 0x3200
+    P.declare(rag, 20, np.concatenate([np.array([b + 16, a], dtype=np.uint64).view(np.uint8),
+                                       np.array([1, 2, 3, 4], dtype=np.uint8)]))
+    for pp in (nul, one, tiny, rag):
+        st, _ = P.run("mapArray", pp)
+        assert st == 0
+    P.check("degenerate outers mapped")
+    P.check_device_units()
+    P.advance()
+    for pp in (nul, one, tiny, rag):
+        P.run("unmapArray", pp)
+    P.check("degenerate outers unmapped")
+    for pp in (nul, one, tiny, rag):
+        P.run("releaseArray", pp)
+    P.check("degenerate outers released")
+    st, _ = P.run("mapArrays", [rag, one, rag])           # the same outer twice in one batch
+    P.check("duplicate outer mapped")
+    P.check_device_units()
+    P.advance()
+    P.run("unmapArrays", [rag, one, rag])
+    P.run("releaseArrays", [rag, one, rag])
+    P.check("duplicate outer released")
+    P.run("mapArray", rag)                                # already array-mapped: A9 re-map, twice over
+    P.run("mapArrays", [rag, rag, one])
+    P.check("duplicate re-map")
+    P.check_device_units()
+    P.advance()
+    P.run("unmapArrays", [one, rag, rag])
+    P.run("releaseArrays", [rag, rag, one])
+    P.run("releaseArray", rag)
+    P.check("duplicate re-map released")
+    P.run("releaseBatch", [a + 64, a + 63, b + 40, b])
+    P.check("end")
+    assert all(u["refCount"] == 0 for u in P.g.dump())
