@@ -776,3 +776,63 @@ def test_degenerate_batches(pair):
     P.run("releaseBatch", [a + 64, a + 63, b + 40, b])
     P.check("end")
     assert all(u["refCount"] == 0 for u in P.g.dump())
+
+
+def _nested_outers(P, order):
+    buf = HostBuf(1 << 16)
+    r0, r1, z = buf.addr + 0x1000, buf.addr + 0x1100, buf.addr + 0x1200
+    P.declare(r0, 32, np.arange(4, dtype=np.float64))
+    P.declare(r1, 48, np.arange(6, dtype=np.float64) + 0.5)
+    P.declare(z, 64, np.arange(8, dtype=np.uint64) + 9)
+    Y = buf.addr + 0x2000
+    P.declare(Y, 16, np.array([r0, r1 + 8], dtype=np.uint64))
+    X = buf.addr + 0x3000
+    P.declare(X, 24, np.array([Y, z + 8, 0], dtype=np.uint64))
+    batch = [X, Y] if order == "outer_first" else [Y, X]
+    st, _ = P.run("mapArrays", batch)
+    assert st == 0
+    P.check("nested mapped")
+    P.check_device_units()
+    P.advance()
+    P.run("unmapArrays", batch)
+    P.check("nested unmapped")
+    P.run("releaseArrays", batch)
+    P.check("nested released")
+    assert all(u["refCount"] == 0 for u in P.g.dump())
+
+
+@pytest.mark.parametrize("order", ["outer_first", "inner_first"])
+def test_nested_outers_in_one_batch(pair, order):
+    """An outer that is also an element of another outer of the same mapArrays batch (a jagged array
+    of pointer arrays): the batch has the sequential semantics of SURVEY §8(b), so whichever outer
+    comes first decides whether the inner one is activated raw (element, Alg. 1) and later
+    re-translated in place (A23), or activated as an array and then only referenced (A9)."""
+    _nested_outers(pair, order)
+
+
+def test_lenient_duplicate_outers(cgcm_mod):
+    """Lenient mode (A18): unregistered slots pass through and are counted once per mapArray call --
+    a batch naming the outer twice counts them twice, as its sequential loop would."""
+    from oracle import Oracle
+    LENIENT = 2
+    ctx = cgcm_mod.Context(0, arena_bytes=1 << 28, flags=LENIENT)
+    o = Oracle(LENIENT)
+    P = Pair(ctx, o)
+    try:
+        buf = HostBuf(1 << 16)
+        a = buf.addr + 0x1000
+        P.declare(a, 64, np.arange(8, dtype=np.uint64))
+        stray = buf.addr + 0x8000                          # never declared
+        pp = buf.addr + 0x2000
+        P.declare(pp, 32, np.array([a + 8, stray, 0, a], dtype=np.uint64))
+        st, _ = P.run("mapArrays", [pp, pp])
+        assert st == 0
+        P.check("lenient mapped")
+        P.check_device_units()
+        P.advance()
+        P.run("unmapArrays", [pp, pp])
+        P.run("releaseArrays", [pp, pp])
+        P.check("lenient released")
+    finally:
+        ctx.close()
+        o.close()
