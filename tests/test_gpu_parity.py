@@ -836,3 +836,45 @@ def test_lenient_duplicate_outers(cgcm_mod):
     finally:
         ctx.close()
         o.close()
+
+
+def _batch_errors(P):
+    buf = HostBuf(1 << 16)
+    a, b = buf.addr + 0x1000, buf.addr + 0x1100
+    P.declare(a, 64, np.arange(8, dtype=np.uint64))
+    P.declare(b, 64, np.arange(8, dtype=np.uint64) + 50)
+    pp = buf.addr + 0x2000
+    P.declare(pp, 24, np.array([a, b + 16, 0], dtype=np.uint64))
+    qq = buf.addr + 0x2100
+    P.declare(qq, 16, np.array([a + 8, buf.addr + 0x9000], dtype=np.uint64))   # second slot unregistered
+    ro = buf.addr + 0x2200
+    P.declare(ro, 16, np.array([b, a + 56], dtype=np.uint64), readonly=True)
+    undeclared = buf.addr + 0x7000
+    P.run("mapArrays", [pp, undeclared])                 # outer miss: nothing happens
+    P.check("outer miss")
+    P.run("mapArrays", [pp, qq])                         # element miss in the second outer
+    P.check("element miss")
+    st, _ = P.run("mapArrays", [pp, ro])
+    assert st == 0
+    P.check("mapped")
+    P.check_device_units()
+    P.g.dev_write(P.g.dump()[0]["devptr"], np.full(64, 0xCD, dtype=np.uint8))   # GPU writes a
+    P.o.dev_write(P.o.dump()[0]["devptr"], np.full(64, 0xCD, dtype=np.uint8))
+    P.advance()
+    P.run("unmapArrays", [pp, qq])                       # qq not mapped: no copy-back happens
+    P.check("unmap error")
+    P.run("releaseArrays", [pp, pp])                     # second release underflows the outer
+    P.check("release underflow")
+    P.run("unmapArrays", [ro, pp])                       # read-only outer: no copy of ro itself
+    P.check("unmapped")
+    P.run("releaseArrays", [ro, pp])
+    P.check("released")
+    assert all(u["refCount"] == 0 for u in P.g.dump())
+
+
+def test_batch_errors_roll_back(pair):
+    """All-or-nothing batches: an outer miss, an element miss in a later outer, an
+    unmap of an unmapped outer and a duplicate release that underflows leave refcounts, epochs, the
+    table, host and device bytes as they were; a read-only outer (Alg. 2: no copy-back) is not
+    copied back by unmapArray while its elements are."""
+    _batch_errors(pair)
