@@ -878,3 +878,38 @@ def test_batch_errors_roll_back(pair):
     table, host and device bytes as they were; a read-only outer (Alg. 2: no copy-back) is not
     copied back by unmapArray while its elements are."""
     _batch_errors(pair)
+
+
+def test_device_array_ragged_slices(pair):
+    """mapArrayDevice / unmapArrayDevice over slices that start on an odd slot (8 B off the kernels'
+    16-byte chunk grid), lengths 1, 2, 3, 31 and 1025 + 1 (ragged tails), an empty slice, and two slices
+    mapped together then unmapped in the other order (the recorded shadows are per slice)."""
+    import torch
+    P = pair
+    offs, sizes, R, span = config_C_setup(P, 2000)
+    q, u = W.queries(offs, sizes, 4096, 5)
+    slots = (q + np.uint64(R)).astype(np.uint64)
+    slots[::13] = 0
+    d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+    base = d.data_ptr()
+    assert P.g.mapArrayDevice(base + 8, 0) == 0 and P.g.unmapArrayDevice(base + 8, 0) == 0
+    P.check("empty")
+    ref = slots.copy()
+    for (s0, n) in [(1, 1), (3, 2), (5, 3), (9, 31), (101, 1026)]:
+        assert P.g.mapArrayDevice(base + 8 * s0, n) == 0
+        P.feed_replay()
+        seg = ref[s0:s0 + n].copy()
+        assert P.o.mapSlots(seg) == 0
+        ref[s0:s0 + n] = seg
+        assert (d.cpu().numpy().view(np.uint64) == ref).all(), (s0, n)
+        P.check(f"mapped {s0}+{n}")
+    P.advance()
+    for (s0, n) in [(101, 1026), (5, 3), (1, 1), (9, 31), (3, 2)]:
+        assert P.g.unmapArrayDevice(base + 8 * s0, n, release=True) == 0
+        seg = ref[s0:s0 + n].copy()
+        assert P.o.unmapSlots(seg, release=True) == 0
+        ref[s0:s0 + n] = seg
+        assert (d.cpu().numpy().view(np.uint64) == ref).all(), (s0, n)
+        P.check(f"unmapped {s0}+{n}")
+    assert (ref == slots).all()
+    W.release_reservation(R, span)
