@@ -913,3 +913,41 @@ def test_device_array_ragged_slices(pair):
         P.check(f"unmapped {s0}+{n}")
     assert (ref == slots).all()
     W.release_reservation(R, span)
+
+
+def test_global_pointer_arrays(pair):
+    """A global array of pointers (the outer is a global: never freed, keeps its device
+    copy) whose slots point at heap rows and at a read-only global, cycled naive-style twice with GPU
+    writes between map and unmap; the same devptr is reused by the second cycle."""
+    P = pair
+    buf = HostBuf(1 << 16)
+    rows = [buf.addr + 0x1000 + 0x100 * k for k in range(6)]
+    for k, r in enumerate(rows):
+        P.declare(r, 64, np.full(8, k + 0.25))
+    gro = buf.addr + 0x4000
+    P.declare_global("tbl_ro", gro, 40, ro=True)
+    host_write(gro, np.arange(5, dtype=np.uint64))
+    P.sync_host_to_oracle(gro, 40)
+    gpp = buf.addr + 0x5000
+    host_write(gpp, np.array(rows + [gro + 8, 0], dtype=np.uint64))
+    P.declare_global("row_ptrs", gpp, 8 * 8)
+    P.sync_host_to_oracle(gpp, 64)
+    devs = []
+    for cyc in range(2):
+        st, d = P.run("mapArray", gpp)
+        assert st == 0
+        devs.append(d)
+        P.check(f"cycle {cyc} mapped")
+        P.check_device_units()
+        for u in P.g.dump():
+            if u["base"] in rows[::2]:
+                P.g.dev_write(u["devptr"], np.full(64, 0x10 + cyc, dtype=np.uint8))
+                P.o.dev_write(u["devptr"], np.full(64, 0x10 + cyc, dtype=np.uint8))
+        P.advance()
+        P.run("unmapArray", gpp)
+        P.check(f"cycle {cyc} unmapped")
+        assert P.g.undeclare(rows[0]) == P.o.undeclare(rows[0])
+        P.run("releaseArray", gpp)
+        P.check(f"cycle {cyc} released")
+    assert devs[0] == devs[1]
+    assert np.frombuffer(host_read(gpp, 64), dtype=np.uint64).tolist() == rows + [gro + 8, 0]
