@@ -149,7 +149,10 @@ int cgcm_scopeExit(void);
  *   rewritten IN PLACE on the device.  *gpu_out = device address of `cpu` in that copy.
  * cgcm_unmapArray: unmap of the outer (reverse GPU->CPU rewrite when copied back, a3) and then of
  *   every element.  cgcm_releaseArray: release every element, then the outer.
- * cgcm_advanceEpoch: globalEpoch += 1; call once after every GPU function launch.  */
+ * cgcm_advanceEpoch: globalEpoch += 1; call once after every GPU function launch.
+ * cgcm_advanceEpochs: globalEpoch += n, exactly as n calls of cgcm_advanceEpoch (n launches with no
+ *   runtime call between them); n < 2^32 - 32, else CGCM_E_INVALID and nothing changes.  Used by the
+ *   tests to reach the u32 device-epoch origin move (DESIGN A28) without 4e9 calls.  */
 int cgcm_map(const void *cpu, void **gpu_out);
 int cgcm_unmap(const void *cpu);
 int cgcm_release(const void *cpu);
@@ -157,6 +160,7 @@ int cgcm_mapArray(void *const *cpu, void ***gpu_out);
 int cgcm_unmapArray(void *const *cpu);
 int cgcm_releaseArray(void *const *cpu);
 int cgcm_advanceEpoch(void);
+int cgcm_advanceEpochs(uint64_t n);
 uint64_t cgcm_epoch(void);
 
 /* ================================ data-parallel batch forms ================================

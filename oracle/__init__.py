@@ -69,7 +69,7 @@ def lib():
             "ref_release": (C.c_int, [vp, u64]),
             "ref_mapArray": (C.c_int, [vp, u64, pu64]), "ref_unmapArray": (C.c_int, [vp, u64]),
             "ref_releaseArray": (C.c_int, [vp, u64]),
-            "ref_advanceEpoch": (C.c_int, [vp]), "ref_epoch": (u64, [vp]),
+            "ref_advanceEpoch": (C.c_int, [vp]), "ref_advanceEpochs": (C.c_int, [vp, u64]), "ref_epoch": (u64, [vp]),
             "ref_mapBatch": (C.c_int, [vp, vp, st, vp]), "ref_unmapBatch": (C.c_int, [vp, vp, st]),
             "ref_releaseBatch": (C.c_int, [vp, vp, st]),
             "ref_mapArrays": (C.c_int, [vp, vp, st, vp]), "ref_unmapArrays": (C.c_int, [vp, vp, st]),
@@ -170,6 +170,9 @@ class Oracle:
 
     def advanceEpoch(self):
         return self.L.ref_advanceEpoch(self.h)
+
+    def advanceEpochs(self, n):
+        return self.L.ref_advanceEpochs(self.h, n)
 
     @property
     def epoch(self):

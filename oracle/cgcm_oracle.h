@@ -81,6 +81,7 @@ int ref_mapArray(void *h, uint64_t pp, uint64_t *gpu_out);
 int ref_unmapArray(void *h, uint64_t pp);
 int ref_releaseArray(void *h, uint64_t pp);
 int ref_advanceEpoch(void *h);
+int ref_advanceEpochs(void *h, uint64_t n);
 uint64_t ref_epoch(void *h);
 
 int ref_mapBatch(void *h, const uint64_t *ps, size_t n, uint64_t *out);

@@ -81,7 +81,7 @@ def lib():
             "cgcm_declareAlloca": (vp, [sz]), "cgcm_scopeEnter": (i, []), "cgcm_scopeExit": (i, []),
             "cgcm_map": (i, [vp, vp]), "cgcm_unmap": (i, [vp]), "cgcm_release": (i, [vp]),
             "cgcm_mapArray": (i, [vp, vp]), "cgcm_unmapArray": (i, [vp]), "cgcm_releaseArray": (i, [vp]),
-            "cgcm_advanceEpoch": (i, []), "cgcm_epoch": (u64, []),
+            "cgcm_advanceEpoch": (i, []), "cgcm_advanceEpochs": (i, [u64]), "cgcm_epoch": (u64, []),
             "cgcm_mapBatch": (i, [vp, sz, vp]), "cgcm_unmapBatch": (i, [vp, sz]),
             "cgcm_releaseBatch": (i, [vp, sz]),
             "cgcm_mapArrays": (i, [vp, sz, vp]), "cgcm_unmapArrays": (i, [vp, sz]),
@@ -246,6 +246,9 @@ class Context:
 
     def advanceEpoch(self) -> int:
         return self.L.cgcm_advanceEpoch()
+
+    def advanceEpochs(self, n: int) -> int:
+        return self.L.cgcm_advanceEpochs(n)
 
     @property
     def epoch(self) -> int:

@@ -2593,17 +2593,19 @@ int cgcm_mapArray(void *const *cpu, void ***gpu_out) {
 int cgcm_unmapArray(void *const *cpu) { return cgcm_unmapArrays(&cpu, 1); }
 int cgcm_releaseArray(void *const *cpu) { return cgcm_releaseArrays(&cpu, 1); }
 
-int cgcm_advanceEpoch(void) {
+int cgcm_advanceEpochs(uint64_t n) {
   CTX();
-  if (C->epoch + 1 - C->origin >= 0xFFFFFFF0ull) {  // move the u32 epoch origin (A28)
+  if (n >= 0xFFFFFFE0ull) return CGCM_E_INVALID;
+  if (C->epoch + n - C->origin >= 0xFFFFFFF0ull) {  // move the u32 epoch origin (A28)
     CKS(C->ensure_table());
     launch_rebase_epochs(C->tab(), C->U, C->rel_epoch(C->epoch), C->main);
     CK(cudaStreamSynchronize(C->main));
     C->origin = C->epoch - 1;
   }
-  C->epoch += 1;  // "increases every time the program launches a GPU function"
+  C->epoch += n;  // "increases every time the program launches a GPU function"
   return CGCM_OK;
 }
+int cgcm_advanceEpoch(void) { return cgcm_advanceEpochs(1); }
 uint64_t cgcm_epoch(void) {
   Context *C = tl_ctx;
   return C ? C->epoch : 0;

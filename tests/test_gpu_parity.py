@@ -951,3 +951,66 @@ def test_global_pointer_arrays(pair):
         P.check(f"cycle {cyc} released")
     assert devs[0] == devs[1]
     assert np.frombuffer(host_read(gpp, 64), dtype=np.uint64).tolist() == rows + [gro + 8, 0]
+
+
+def _check_mod_stale_epochs(P, what):
+    """Pair.check with one relaxation, DESIGN A28: after the device's u32 epoch origin moves, a unit
+    whose epoch is stale may dump a different stale value; whether it is current may not change."""
+    from tests.harness import COMPARED_STATS
+    gd, od = P.g.dump(), P.o.dump()
+    assert len(gd) == len(od), what
+    ge, oe = P.g.epoch, P.o.epoch
+    assert ge == oe, what
+    for a, b in zip(gd, od):
+        assert {k: v for k, v in a.items() if k != "epoch"} == {k: v for k, v in b.items() if k != "epoch"}, \
+            f"{what}: gpu={a} oracle={b}"
+        assert (a["epoch"] == ge) == (b["epoch"] == oe), f"{what}: currency differs gpu={a} oracle={b}"
+        if b["epoch"] == oe or b["epoch"] + 8 > oe:
+            assert a["epoch"] == b["epoch"] or a["epoch"] != ge, f"{what}: gpu={a} oracle={b}"
+    gs, os_ = P.g.stats(), P.o.stats()
+    for f in COMPARED_STATS:
+        assert gs[f] == os_[f], f"{what}: stat {f} gpu={gs[f]} oracle={os_[f]}"
+    for base, n in P.units.items():
+        assert host_read(base, n) == P.o.host_read(base, n).tobytes(), f"{what}: host bytes of {hex(base)}"
+
+
+def test_epoch_origin_move(pair):
+    """DESIGN A28: the device keeps u32 epochs relative to an origin that moves when the relative
+    epoch would reach 2^32 - 16.  Drive globalEpoch across that point with
+    cgcm_advanceEpochs (= n launches) and check every copy decision of Alg. 2 (copy iff
+    epoch != globalEpoch and not read-only, at most once per epoch) against the oracle's u64 epochs:
+    units left stale across the move, units made current just before it, read-only units."""
+    P = pair
+    buf = HostBuf(1 << 16)
+    us = [buf.addr + 0x1000 + 0x200 * k for k in range(5)]
+    for k, u in enumerate(us):
+        P.declare(u, 128, np.full(16, k + 0.5), readonly=(k == 4))
+    for u in us:
+        P.run("map", u)
+    assert P.g.advanceEpochs(0xFFFFFFE0) == P.o.advanceEpochs(0xFFFFFFE0) == -1   # bound
+    jump = 0xFFFFFFF0 - 6
+    for n in (1 << 31, jump - (1 << 31)):
+        assert P.g.advanceEpochs(n) == 0 and P.o.advanceEpochs(n) == 0
+    P.check("jumped")                                     # no origin move yet: exact
+    P.run("unmap", us[0])                                 # stale since the map: copied
+    for step in range(12):                                # the origin moves during these launches
+        for u in P.g.dump():
+            if u["base"] in (us[1], us[3]):
+                P.g.dev_write(u["devptr"], np.full(128, 0x40 + step, dtype=np.uint8))
+                P.o.dev_write(u["devptr"], np.full(128, 0x40 + step, dtype=np.uint8))
+        P.advance()
+        P.run("unmap", us[1])                             # copied every launch
+        P.run("unmap", us[1])                             # ... once
+        P.run("unmap", us[4])                             # read-only: never copied
+        if step == 4:
+            P.run("unmap", us[3])                         # current just before the move
+        _check_mod_stale_epochs(P, f"step {step}")
+    P.run("unmap", us[2])                                 # stale across the move: still copied
+    P.run("unmap", us[3])
+    _check_mod_stale_epochs(P, "after")
+    assert P.g.epoch - jump > 12 - 1
+    for u in us:
+        P.run("release", u)
+    _check_mod_stale_epochs(P, "released")
+    s = P.g.stats()
+    assert s["d2h_units"] == P.o.stats()["d2h_units"] >= 12 + 3
