@@ -1014,3 +1014,49 @@ def test_epoch_origin_move(pair):
     _check_mod_stale_epochs(P, "released")
     s = P.g.stats()
     assert s["d2h_units"] == P.o.stats()["d2h_units"] >= 12 + 3
+
+
+def test_unit_over_4GiB(cgcm_mod):
+    """A26: an AU larger than 2^32 bytes (its size lives in the cold 64-bit column; the hot word holds
+    the escape) -- interior pointers beyond 4 GiB, one-past-the-end (A7), the gap after it, through
+    mapBatch (k_slots) and mapArrayDevice (k_map_pd), against the oracle.  The AU is read-only zero
+    pages (PROT_READ reservation: no RAM), so activation copies 5 GiB H2D and nothing is copied back."""
+    import torch
+    from oracle import Oracle
+    big_size = (5 << 30) + 12345
+    span = big_size + (4 << 20)
+    R = W.reserve_readonly(span)
+    ctx = cgcm_mod.Context(0, arena_bytes=(5 << 30) + (256 << 20), flags=0)
+    o = Oracle()
+    P = Pair(ctx, o)
+    try:
+        u0, big = R, R + 0x10000
+        u2 = big + big_size + 64
+        for base, size in ((u0, 4096), (big, big_size), (u2, 1000)):
+            assert P.g.declareAlloc(base, size, True) == 0 and P.o.declareAlloc(base, size, True) == 0
+        pts = [big + (4 << 30) + 7, u0 + 8, big, big + big_size, u2 + 5, 0, big + (1 << 32), big + big_size - 1]
+        st, _ = P.run("mapBatch", pts)
+        assert st == 0
+        P.check("mapped")
+        P.run("mapBatch", [big + 8, big + big_size + 1])  # the gap after the end: UNREGISTERED
+        P.check("gap")
+        slots = np.array([big + (3 << 30) + 3, u2, big + big_size, 0, big + (1 << 32) - 8, u0 + 4095,
+                          big + 17, big + (5 << 30)], dtype=np.uint64)
+        d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+        assert P.g.mapArrayDevice(d.data_ptr(), len(slots)) == 0
+        ref = slots.copy()
+        assert P.o.mapSlots(ref) == 0
+        assert (d.cpu().numpy().view(np.uint64) == ref).all()
+        P.check("device slots mapped")
+        P.advance()
+        assert P.g.unmapArrayDevice(d.data_ptr(), len(slots), release=True) == 0
+        assert P.o.unmapSlots(ref, release=True) == 0
+        assert (d.cpu().numpy().view(np.uint64) == slots).all()
+        P.run("unmapBatch", pts)
+        P.run("releaseBatch", pts)
+        P.check("released")
+        assert all(u["refCount"] == 0 for u in P.g.dump())
+    finally:
+        ctx.close()
+        o.close()
+        W.release_reservation(R, span)
