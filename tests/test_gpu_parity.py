@@ -1060,3 +1060,44 @@ def test_unit_over_4GiB(cgcm_mod):
         ctx.close()
         o.close()
         W.release_reservation(R, span)
+
+
+def test_compact_word_escapes(pair):
+    """The forward kernel's 4-byte unit word escapes to the 8-byte hot word when a unit's size is
+    >= 2^18 B or its device extent id >= 2^11 (cgcm_dev.h make_hotc): 2600 units activated by 2600
+    separate map calls (one extent each), two units of 300 KB and 3 MiB, then 50,000 device slots
+    over all of them mapped / unmapped+released against the oracle (mapSlots / unmapSlots)."""
+    import torch
+    P = pair
+    buf = HostBuf(8 << 20)
+    K = 2600
+    bases = [buf.addr + 256 * k for k in range(K)] + [buf.addr + (1 << 20), buf.addr + (2 << 20)]
+    sizes = [64 + 8 * (k % 7) for k in range(K)] + [300000, 3 << 20]
+    for b, s in zip(bases, sizes):
+        assert P.g.declareAlloc(b, s) == 0 and P.o.declareAlloc(b, s) == 0
+    gst = [P.g.map(b)[0] for b in bases]                  # one activation (one extent) per call
+    P.feed_replay()
+    ost = [P.o.map(b)[0] for b in bases]
+    assert gst == ost == [0] * len(bases)
+    P.check("activated one by one")
+    rng = np.random.default_rng(11)
+    Q = 50000
+    u = rng.integers(0, len(bases), Q)
+    u[:2000] = rng.integers(K, K + 2, 2000)               # plenty of slots into the big units
+    off = (rng.random(Q) * (np.array(sizes, dtype=np.float64)[u] + 1)).astype(np.uint64)
+    slots = (np.array(bases, dtype=np.uint64)[u] + off).astype(np.uint64)
+    slots[::41] = 0
+    rng.shuffle(slots)
+    d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+    assert P.g.mapArrayDevice(d.data_ptr(), Q) == 0
+    ref = slots.copy()
+    assert P.o.mapSlots(ref) == 0
+    assert (d.cpu().numpy().view(np.uint64) == ref).all()
+    P.check("slots mapped")
+    P.advance()
+    assert P.g.unmapArrayDevice(d.data_ptr(), Q, release=True) == 0
+    assert P.o.unmapSlots(ref, release=True) == 0
+    assert (d.cpu().numpy().view(np.uint64) == slots).all()
+    P.check("slots unmapped")
+    P.run("releaseBatch", bases)
+    P.check("released")
