@@ -54,8 +54,8 @@ def _worker(rank, world, port, out):
     dist.destroy_process_group()
 
 
-def test_sharding_and_reduction_world2():
-    world = 2
+@pytest.mark.parametrize("world", [2, 4])
+def test_sharding_and_reduction(world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
@@ -74,7 +74,7 @@ def test_sharding_and_reduction_world2():
     for (f0, n0, st0, c0), (f1, n1, st1, c1) in zip(firsts, firsts[1:]):
         assert f0 + n0 == f1 and st0 + c0 == st1
     assert sum(s[1] for s in shards) == cfg["arrays"]
-    assert tmax == 11.0
+    assert tmax == 10.0 + world - 1
     # every slot was mapped by exactly one rank: the per-rank refcounts add up to a single-process run
     from oracle import Oracle
     wl = bench.Workload(dict(cfg), 0, 1)
