@@ -1101,3 +1101,64 @@ def test_compact_word_escapes(pair):
     P.check("slots unmapped")
     P.run("releaseBatch", bases)
     P.check("released")
+
+
+@pytest.mark.parametrize("seed,nested", [(2024, False), (7, False), (99, True)])
+def test_random_array_batches(pair, seed, nested):
+    """Seeded random differential run of the batch forms: mapArrays / unmapArrays / releaseArrays over
+    multisets of 12 outers (repeats within a batch, SURVEY §8(b) sequential semantics), GPU writes to
+    leaf units between launches, occasional unbalanced calls (NOT_MAPPED, all-or-nothing); full state
+    compared with the oracle after every call."""
+    P = pair
+    rng = np.random.default_rng(seed)
+    buf = HostBuf(1 << 20)
+    leaves = [buf.addr + 0x100 * k for k in range(64)]
+    outer_bases = [buf.addr + 0x10000 + 0x1000 * j for j in range(12)]
+    for k, a in enumerate(leaves):
+        P.declare(a, 48 + 8 * (k % 5), rng.integers(0, 255, 48 + 8 * (k % 5), dtype=np.uint8))
+    outers = []
+    for j in range(12):
+        o = buf.addr + 0x10000 + 0x1000 * j
+        n = int(rng.integers(0, 40))
+        tg = [0 if rng.random() < 0.1 else leaves[int(rng.integers(0, 64))] + 8 * int(rng.integers(0, 6))
+              for _ in range(n)]
+        if nested and j < 3 and n:                        # outers 0-2 also point at outers 9-11
+            tg[0] = outer_bases[9 + j]
+        P.declare(o, 8 * n + int(rng.integers(0, 8)) if n else 8, np.asarray(tg + [0], dtype=np.uint64)
+                  .view(np.uint8)[:8 * n + 8])
+        outers.append(o)
+    held = {o: 0 for o in outers}
+    for step in range(150):
+        r = rng.random()
+        k = int(rng.integers(1, 6))
+        if r < 0.4:
+            batch = [outers[int(i)] for i in rng.integers(0, 12, k)]
+            st, _ = P.run("mapArrays", batch)
+            if st == 0:
+                for o in batch:
+                    held[o] += 1
+        elif r < 0.6:
+            live = [o for o in outers if held[o] > 0]
+            batch = [live[int(i)] for i in rng.integers(0, len(live), k)] if live and rng.random() < 0.9 \
+                else [outers[int(i)] for i in rng.integers(0, 12, k)]
+            P.run("unmapArrays", batch)
+        elif r < 0.85:
+            live = [o for o in outers for _ in range(held[o])]
+            if live and rng.random() < 0.9:
+                idx = rng.choice(len(live), size=min(k, len(live)), replace=False)
+                batch = [live[int(i)] for i in idx]
+            else:
+                batch = [outers[int(i)] for i in rng.integers(0, 12, k)]
+            st = P.run("releaseArrays", batch)
+            if st == 0:
+                for o in batch:
+                    held[o] -= 1
+        else:
+            for u in P.g.dump():
+                if u["refCount"] > 0 and u["base"] in leaves and rng.random() < 0.3:
+                    v = rng.integers(0, 255, u["size"], dtype=np.uint8)
+                    P.g.dev_write(u["devptr"], v)
+                    P.o.dev_write(u["devptr"], v)
+            P.advance()
+        P.check(f"step {step}")
+    P.check_device_units()
