@@ -1162,3 +1162,58 @@ def test_random_array_batches(pair, seed, nested):
             P.advance()
         P.check(f"step {step}")
     P.check_device_units()
+
+
+@pytest.mark.parametrize("seed", [5, 17])
+def test_random_scalar_batches(pair, seed):
+    """Seeded random differential run of mapBatch / unmapBatch / releaseBatch over interior pointers
+    with repeats inside a batch (a batch = its sequential loop: repeated unmaps copy at most once per
+    epoch, repeated releases count down), heap AUs and two globals (never freed), GPU writes between
+    launches, unbalanced releases (NOT_MAPPED, all-or-nothing); state compared after every call."""
+    P = pair
+    rng = np.random.default_rng(seed)
+    buf = HostBuf(1 << 18)
+    units = []
+    for k in range(80):
+        b, s = buf.addr + 0x200 * k, int(rng.integers(1, 60)) * 8
+        P.declare(b, s, rng.integers(0, 255, s, dtype=np.uint8))
+        units.append((b, s))
+    for k, ro in ((0, False), (1, True)):
+        b, s = buf.addr + 0x20000 + 0x400 * k, 96
+        P.declare_global(f"g{seed}_{k}", b, s, ro=ro)
+        units.append((b, s))
+    held = {}
+    for step in range(150):
+        r = rng.random()
+        k = int(rng.integers(1, 12))
+        pick = [units[int(i)] for i in rng.integers(0, len(units), k)]
+        ps = [b + int(rng.integers(0, s + 1)) for b, s in pick]
+        if r < 0.35:
+            st, _ = P.run("mapBatch", ps)
+            if st == 0:
+                for b, _s in pick:
+                    held[b] = held.get(b, 0) + 1
+        elif r < 0.55:
+            live = [b for b, c in held.items() if c > 0]
+            if live:
+                P.run("unmapBatch", [live[int(i)] + 1 for i in rng.integers(0, len(live), k)])
+        elif r < 0.8:
+            pool = [b for b, c in held.items() for _ in range(c)]
+            if pool and rng.random() < 0.9:
+                idx = rng.choice(len(pool), size=min(k, len(pool)), replace=False)
+                batch = [pool[int(i)] for i in idx]
+            else:
+                batch = [b for b, _s in pick]
+            st = P.run("releaseBatch", batch)
+            if st == 0:
+                for b in batch:
+                    held[b] -= 1
+        else:
+            for u in P.g.dump():
+                if u["refCount"] > 0 and rng.random() < 0.3:
+                    v = rng.integers(0, 255, u["size"], dtype=np.uint8)
+                    P.g.dev_write(u["devptr"], v)
+                    P.o.dev_write(u["devptr"], v)
+            P.advance()
+        P.check(f"step {step}")
+    P.check_device_units()
