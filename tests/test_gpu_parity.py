@@ -1217,3 +1217,68 @@ def test_random_scalar_batches(pair, seed):
             P.advance()
         P.check(f"step {step}")
     P.check_device_units()
+
+
+@pytest.mark.parametrize("seed", [3, 8])
+def test_random_device_slices(pair, seed):
+    """Seeded random differential run of the device-array path (the hot kernels k_map_pd / k_unmap_sh
+    and their fallbacks): six disjoint slices of one device buffer (odd starts, ragged lengths) are
+    mapped, optionally permuted within the slice by a "GPU function" (the shadow fallback), unmapped
+    with or without the fused release (then released later through releaseBatch), interleaved with
+    scalar maps / releases of the same units and epoch advances; state compared after every call."""
+    import torch
+    P = pair
+    rng = np.random.default_rng(seed)
+    offs, sizes, R, span = config_C_setup(P, 3000, seed=seed)
+    bounds = [(1, 700), (701, 1), (703, 2050), (2760, 33), (2800, 4096 + 3), (6900, 257)]
+    total = 7200
+    q, _u = W.queries(offs, sizes, total, seed + 1)
+    slots = (q + np.uint64(R)).astype(np.uint64)
+    slots[rng.random(total) < 0.05] = 0
+    d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
+    ref = slots.copy()
+    base = d.data_ptr()
+    state = ["cpu"] * len(bounds)       # cpu: holds CPU pointers, no refs; gpu: mapped; held: CPU ptrs + refs
+    own = []
+    for step in range(80):
+        r = rng.random()
+        i = int(rng.integers(0, len(bounds)))
+        s0, n = bounds[i]
+        if r < 0.3 and state[i] == "cpu":
+            st = P.g.mapArrayDevice(base + 8 * s0, n)
+            P.feed_replay()
+            seg = ref[s0:s0 + n].copy()
+            assert st == P.o.mapSlots(seg)
+            if st == 0:
+                ref[s0:s0 + n] = seg
+                state[i] = "gpu"
+        elif r < 0.55 and state[i] == "gpu":
+            if rng.random() < 0.3 and n > 1:           # the "GPU function" permutes the slice
+                perm = rng.permutation(n)
+                ref[s0:s0 + n] = ref[s0:s0 + n][perm]
+                d[s0:s0 + n] = d[s0:s0 + n][torch.from_numpy(perm).cuda()]
+            rel = bool(rng.random() < 0.6)
+            st = P.g.unmapArrayDevice(base + 8 * s0, n, release=rel)
+            seg = ref[s0:s0 + n].copy()
+            assert st == P.o.unmapSlots(seg, release=rel)
+            if st == 0:
+                ref[s0:s0 + n] = seg
+                state[i] = "cpu" if rel else "held"
+        elif r < 0.65 and state[i] == "held":
+            nz = [int(x) for x in ref[s0:s0 + n] if x != 0]
+            st = P.run("releaseBatch", nz)
+            if st == 0:
+                state[i] = "cpu"
+        elif r < 0.8:
+            j = int(rng.integers(0, len(offs)))
+            p = R + int(offs[j]) + int(rng.integers(0, int(sizes[j]) + 1))
+            st, _ = P.run("map", p)
+            if st == 0:
+                own.append(p)
+        elif r < 0.9 and own:
+            P.run("release", own.pop(int(rng.integers(0, len(own)))))
+        else:
+            P.advance()
+        assert (d.cpu().numpy().view(np.uint64) == ref).all(), f"step {step}"
+        P.check(f"step {step}")
+    W.release_reservation(R, span)
