@@ -1282,3 +1282,45 @@ def test_random_device_slices(pair, seed):
         assert (d.cpu().numpy().view(np.uint64) == ref).all(), f"step {step}"
         P.check(f"step {step}")
     W.release_reservation(R, span)
+
+
+def test_region_mixed_kinds_and_repeats(pair):
+    """cgcm_regionBegin over an array outer named twice and two scalar AUs (one of them also an element
+    of the outer): the hoisted calls are the sequential loop in order, regionEnd unmaps + releases each
+    pointer in reverse order (Listing 4, A11); the loop body keeps its own map / release.
+    Compared with the oracle running that promoted sequence explicitly."""
+    P = pair
+    buf = HostBuf(1 << 16)
+    rows = [buf.addr + 0x200 * k for k in range(8)]
+    for k, r in enumerate(rows):
+        P.declare(r, 64, np.full(8, k + 1.0))
+    pp = buf.addr + 0x4000
+    P.declare(pp, 8 * 9, np.asarray(rows + [0], dtype=np.uint64))
+    x = buf.addr + 0x5000
+    P.declare(x, 128, np.arange(16, dtype=np.float64))
+    ptrs = [pp, x, pp, rows[3] + 8]
+    kinds = [P.g.REGION_MAPARRAY, P.g.REGION_MAP, P.g.REGION_MAPARRAY, P.g.REGION_MAP]
+    assert P.g.regionBegin(ptrs, kinds) == 0
+    P.feed_replay()
+    for p, k in zip(ptrs, kinds):
+        assert (P.o.mapArray(p) if k == P.g.REGION_MAPARRAY else P.o.map(p))[0] == 0
+    P.check("region begun")
+    for it in range(4):
+        P.run("map", x + 8)
+        for u in P.g.dump():
+            if u["base"] in (rows[it], x):
+                v = np.full(u["size"], 0x30 + it, dtype=np.uint8)
+                P.g.dev_write(u["devptr"], v)
+                P.o.dev_write(u["devptr"], v)
+        P.advance()
+        P.run("release", x + 8)
+        P.check(f"iteration {it}")
+    s, v = P.g.regionEnd()
+    assert (s, v) == (0, 0)
+    for p, k in reversed(list(zip(ptrs, kinds))):
+        if k == P.g.REGION_MAPARRAY:
+            assert P.o.unmapArray(p) == 0 and P.o.releaseArray(p) == 0
+        else:
+            assert P.o.unmap(p) == 0 and P.o.release(p) == 0
+    P.check("region ended")
+    assert all(u["refCount"] == 0 for u in P.g.dump())
