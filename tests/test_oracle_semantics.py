@@ -293,3 +293,88 @@ def test_device_copies_never_adjacent_unless_host_adjacent(oracle):
         assert o.devLookup(end) == (b, g)
         s = np.array([end], dtype=np.uint64)
         assert o.unmapSlots(s) == OK and int(s[0]) == b + 512
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_batch_forms_are_their_sequential_loops(seed):
+    """the batch forms have "the same semantics as the sequential loop".  Oracle A runs a
+    random program through mapArrays / unmapArrays / releaseArrays / mapBatch / unmapBatch / releaseBatch
+    on multisets (repeats, nested outers); oracle B runs the same program through the single calls in
+    batch order.  After every successful batch their full states agree.  A failing batch must leave A
+    unchanged (all-or-nothing) and its sequential loop must fail too (checked on a replayed copy)."""
+    rng = np.random.default_rng(seed)
+    leaves = [0x100000 + 0x100 * k for k in range(40)]
+    outers = [0x200000 + 0x1000 * j for j in range(8)]
+    regions, init = [], []
+    for k, a in enumerate(leaves):
+        n = 32 + 8 * (k % 4)
+        init.append((a, np.full(n, k, dtype=np.uint8)))
+        regions.append((a, n))
+    for j, p in enumerate(outers):
+        n = int(rng.integers(1, 12))
+        tg = [0 if rng.random() < 0.15 else leaves[int(rng.integers(0, 40))] + 8 * int(rng.integers(0, 4))
+              for _ in range(n)]
+        if j < 2:
+            tg[0] = outers[6 + j]                      # nested: outers 0, 1 point at outers 6, 7
+        init.append((p, np.asarray(tg, dtype=np.uint64)))
+        regions.append((p, 8 * n))
+    singles = {"mapArrays": "mapArray", "unmapArrays": "unmapArray", "releaseArrays": "releaseArray",
+               "mapBatch": "map", "unmapBatch": "unmap", "releaseBatch": "release"}
+
+    def fresh():
+        o = Oracle()
+        for (b, data), (_b, n) in zip(init, regions):
+            assert o.declareAlloc(b, n) == OK
+            o.host_write(b, data)
+        return o
+
+    def run_loop(o, name, batch):
+        for p in batch:
+            r = getattr(o, singles[name])(p)
+            st = r[0] if isinstance(r, tuple) else r
+            if st != OK:
+                return st
+        return OK
+
+    A, B = fresh(), fresh()
+    log = []
+    held = {"a": [], "s": []}                          # references taken: outers / scalar pointers
+    n_ok = n_err = 0
+    for step in range(150):
+        name = list(singles)[int(rng.integers(0, 6))]
+        k = int(rng.integers(1, 6))
+        kind = "a" if "Arrays" in name else "s"
+        if name.startswith("map") or not held[kind] or rng.random() < 0.1:
+            pool = outers if kind == "a" else [b + int(rng.integers(0, n + 1)) for b, n in regions[:40]]
+            batch = [pool[int(i)] for i in rng.integers(0, len(pool), k)]
+        else:
+            batch = [held[kind][int(i)] for i in rng.choice(len(held[kind]), min(k, len(held[kind])), replace=False)]
+        before = snapshot(A, regions)
+        ra = getattr(A, name)(batch)
+        sa = ra[0] if isinstance(ra, tuple) else ra
+        if sa != OK:
+            n_err += 1
+            assert snapshot(A, regions) == before, (step, name)      # all-or-nothing
+            C = fresh()
+            for nm, bt in log:
+                assert (run_loop(C, nm, bt) if nm != "advance" else C.advanceEpoch()) == OK
+            assert run_loop(C, name, batch) != OK, (step, name)       # the loop fails as well
+            C.close()
+            continue
+        n_ok += 1
+        assert run_loop(B, name, batch) == OK, (step, name)
+        log.append((name, batch))
+        if name.startswith("map"):
+            held[kind] += batch
+        elif name.startswith("release"):
+            for p in batch:
+                if p in held[kind]:                    # (a random release may hit another pointer's unit)
+                    held[kind].remove(p)
+        if rng.random() < 0.2:
+            A.advanceEpoch()
+            B.advanceEpoch()
+            log.append(("advance", None))
+        assert snapshot(A, regions) == snapshot(B, regions), (step, name)
+    assert n_ok > 100 and n_err >= 1
+    A.close()
+    B.close()
