@@ -1306,7 +1306,10 @@ struct Context {
     unsigned long long lcs[4];
     CKS(fetch_status(sts, lcs));
     res = sts[0];
-    if (sts[0].misses && !(flags & CGCM_LENIENT)) {
+    // a reverse miss means an element lost its device copy (A25) -- or, in lenient mode, a slot that
+    // passed through unregistered (A18): either way the caller re-translates from the host slots,
+    // which is what a sequential mapArray does (the oracle's semantics), lenient or not
+    if (sts[0].misses) {
       CKS(rev_decref(rsegs));
       return CGCM_E_UNREGISTERED;
     }

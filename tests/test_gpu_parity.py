@@ -1105,6 +1105,23 @@ def test_compact_word_escapes(pair):
 
 @pytest.mark.parametrize("seed,nested", [(2024, False), (7, False), (99, True)])
 def test_random_array_batches(pair, seed, nested):
+    _random_array_batches(pair, seed, nested)
+
+
+def test_random_array_batches_lenient(cgcm_mod):
+    """The same random program in lenient mode (A18) with stray (undeclared) pointers in the outers:
+    they pass through both ways and are counted per call."""
+    from oracle import Oracle
+    ctx = cgcm_mod.Context(0, arena_bytes=1 << 28, flags=2)
+    o = Oracle(2)
+    try:
+        _random_array_batches(Pair(ctx, o), 31, True, stray=True)
+    finally:
+        ctx.close()
+        o.close()
+
+
+def _random_array_batches(pair, seed, nested, stray=False):
     """Seeded random differential run of the batch forms: mapArrays / unmapArrays / releaseArrays over
     multisets of 12 outers (repeats within a batch, SURVEY §8(b) sequential semantics), GPU writes to
     leaf units between launches, occasional unbalanced calls (NOT_MAPPED, all-or-nothing); full state
@@ -1124,6 +1141,8 @@ def test_random_array_batches(pair, seed, nested):
               for _ in range(n)]
         if nested and j < 3 and n:                        # outers 0-2 also point at outers 9-11
             tg[0] = outer_bases[9 + j]
+        if stray and n > 1:
+            tg[-1] = buf.addr + 0x80000 + 8 * j          # never declared
         P.declare(o, 8 * n + int(rng.integers(0, 8)) if n else 8, np.asarray(tg + [0], dtype=np.uint64)
                   .view(np.uint8)[:8 * n + 8])
         outers.append(o)
