@@ -1240,6 +1240,22 @@ def test_random_scalar_batches(pair, seed):
 
 @pytest.mark.parametrize("seed", [3, 8])
 def test_random_device_slices(pair, seed):
+    _random_device_slices(pair, seed)
+
+
+def test_random_device_slices_lenient(cgcm_mod):
+    """The same random program in lenient mode (A18) with stray (undeclared) pointers in the slices."""
+    from oracle import Oracle
+    ctx = cgcm_mod.Context(0, arena_bytes=1 << 28, flags=2)
+    o = Oracle(2)
+    try:
+        _random_device_slices(Pair(ctx, o), 13, stray=True)
+    finally:
+        ctx.close()
+        o.close()
+
+
+def _random_device_slices(pair, seed, stray=False):
     """Seeded random differential run of the device-array path (the hot kernels k_map_pd / k_unmap_sh
     and their fallbacks): six disjoint slices of one device buffer (odd starts, ragged lengths) are
     mapped, optionally permuted within the slice by a "GPU function" (the shadow fallback), unmapped
@@ -1254,6 +1270,8 @@ def test_random_device_slices(pair, seed):
     q, _u = W.queries(offs, sizes, total, seed + 1)
     slots = (q + np.uint64(R)).astype(np.uint64)
     slots[rng.random(total) < 0.05] = 0
+    if stray:
+        slots[rng.random(total) < 0.03] = np.uint64(R + span + 64)
     d = torch.from_numpy(slots.view(np.int64).copy()).cuda()
     ref = slots.copy()
     base = d.data_ptr()
