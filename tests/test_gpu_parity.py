@@ -1185,6 +1185,10 @@ def _random_array_batches(pair, seed, nested, stray=False):
 
 @pytest.mark.parametrize("seed", [5, 17])
 def test_random_scalar_batches(pair, seed):
+    _random_scalar_batches(pair, seed)
+
+
+def _random_scalar_batches(pair, seed):
     """Seeded random differential run of mapBatch / unmapBatch / releaseBatch over interior pointers
     with repeats inside a batch (a batch = its sequential loop: repeated unmaps copy at most once per
     epoch, repeated releases count down), heap AUs and two globals (never freed), GPU writes between
@@ -1361,3 +1365,27 @@ def test_region_mixed_kinds_and_repeats(pair):
             assert P.o.unmap(p) == 0 and P.o.release(p) == 0
     P.check("region ended")
     assert all(u["refCount"] == 0 for u in P.g.dump())
+
+
+@pytest.mark.parametrize("flags,program", [(1, "arrays"), (1, "scalars"), (1, "slices"), (3, "arrays"),
+                                           (2, "scalars"), (3, "slices")],
+                         ids=["literal-arrays", "literal-scalars", "literal-slices", "literal+lenient-arrays",
+                              "lenient-scalars", "literal+lenient-slices"])
+def test_random_programs_other_modes(cgcm_mod, flags, program):
+    """The random differential programs under CGCM_LITERAL_EPOCH (A5's literal reading: map never sets
+    the AU epoch, so the first unmap after a map copies back even without a launch) and lenient mode
+    (A18), against the oracle created with the same flags."""
+    from oracle import Oracle
+    ctx = cgcm_mod.Context(0, arena_bytes=1 << 28, flags=flags)
+    o = Oracle(flags)
+    try:
+        P = Pair(ctx, o)
+        if program == "arrays":
+            _random_array_batches(P, 41, True, stray=bool(flags & 2))
+        elif program == "scalars":
+            _random_scalar_batches(P, 43)
+        else:
+            _random_device_slices(P, 47, stray=bool(flags & 2))
+    finally:
+        ctx.close()
+        o.close()
