@@ -1259,7 +1259,15 @@ def test_random_device_slices_lenient(cgcm_mod):
         o.close()
 
 
-def _random_device_slices(pair, seed, stray=False):
+@pytest.mark.parametrize("seed", [21, 22])
+def test_random_device_slices_with_table_churn(pair, seed):
+    """The device-slice program with declares / undeclares between calls (a0: the table and its index
+    are rebuilt and unit indices move while slices hold recorded shadows), new units written into slices
+    that hold CPU pointers, and slices pointing at undeclared units (UNREGISTERED, all-or-nothing)."""
+    _random_device_slices(pair, seed, churn=True)
+
+
+def _random_device_slices(pair, seed, stray=False, churn=False):
     """Seeded random differential run of the device-array path (the hot kernels k_map_pd / k_unmap_sh
     and their fallbacks): six disjoint slices of one device buffer (odd starts, ragged lengths) are
     mapped, optionally permuted within the slice by a "GPU function" (the shadow fallback), unmapped
@@ -1281,7 +1289,27 @@ def _random_device_slices(pair, seed, stray=False):
     base = d.data_ptr()
     state = ["cpu"] * len(bounds)       # cpu: holds CPU pointers, no refs; gpu: mapped; held: CPU ptrs + refs
     own = []
+    rng2 = np.random.default_rng(seed + 1000)
+    xbuf = HostBuf(1 << 16)
+    extra = []                          # heap units declared by the churn
     for step in range(80):
+        if churn and rng2.random() < 0.25:
+            if extra and rng2.random() < 0.4:
+                b = extra[int(rng2.integers(0, len(extra)))]
+                rc = {u["base"]: u["refCount"] for u in P.o.dump()}.get(b, 0)
+                assert P.undeclare(b) == (0 if rc == 0 else -5)
+                if rc == 0:
+                    extra.remove(b)
+            else:
+                b = xbuf.addr + 0x100 * int(rng2.integers(0, 256))
+                if P.declare(b, 64, rng2.integers(0, 255, 64, dtype=np.uint8)) == 0:
+                    extra.append(b)
+            j = int(rng2.integers(0, len(bounds)))
+            if state[j] == "cpu" and extra:             # point a CPU-state slot at an extra unit
+                k = bounds[j][0] + int(rng2.integers(0, bounds[j][1]))
+                v = np.uint64(extra[int(rng2.integers(0, len(extra)))] + int(rng2.integers(0, 65)))
+                ref[k] = v
+                d[k] = int(v)
         r = rng.random()
         i = int(rng.integers(0, len(bounds)))
         s0, n = bounds[i]
