@@ -201,6 +201,13 @@ struct Context {
   std::recursive_mutex mu;
   uint64_t epoch = 0;
   uint64_t origin = 0;  // device epochs are u32 relative to this origin (A28)
+  // generation of device-storage releases, and per array outer (host base) the generation at which its
+  // slots were last translated from host memory: a re-map may reverse-translate its device slots (A9)
+  // only if no storage was released since -- otherwise a slot may point at a freed copy whose address
+  // a newer unit now occupies (an element released through another path, A25), and the re-map must
+  // re-translate from the host slots as the sequential mapArray does
+  uint64_t free_gen = 0;
+  std::unordered_map<uint64_t, uint64_t> arr_gen;
   uint32_t rel_epoch(uint64_t e) const { return e >= origin ? (uint32_t)(e - origin) : 0u; }
 
   // registry (host)
@@ -327,6 +334,7 @@ struct Context {
   }
   void run_release(int64_t id) {
     if (id < 0) return;
+    free_gen += 1;  // device addresses of this unit may now be reused by another unit
     if (--runs[id].live <= 0) drop_run(id);
   }
 
@@ -2146,6 +2154,7 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
   CKS(C->activate_units(act, &copies, &pack_ev));
   std::vector<UnitOp> ops;
   std::vector<Seg> fsegs, rsegs;
+  bool rev_stale = false;
   for (auto &o : outs) {
     const uint64_t hu_dev = C->udev[o.unit];
     ops.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)o.mult});
@@ -2153,8 +2162,13 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
     uint64_t n = o.info.size / 8;
     if (!n) continue;
     Seg s{hu_dev, n, 0, o.mult, 0};
-    if (o.info.refcount > 0 && (o.info.flags & UF_ARRAYMAPPED)) rsegs.push_back(s);  // A9: refcounts only
-    else fsegs.push_back(s);
+    if (o.info.refcount > 0 && (o.info.flags & UF_ARRAYMAPPED)) {
+      rsegs.push_back(s);  // A9: refcounts only
+      auto g = C->arr_gen.find(o.info.base);
+      if (g == C->arr_gen.end() || g->second != C->free_gen) rev_stale = true;
+    } else {
+      fsegs.push_back(s);
+    }
   }
   // unit ops must not run before the outers' set_devbase: same stream, issued after
   CKS(C->unit_ops(ops));
@@ -2186,7 +2200,7 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
   struct Backup { uint64_t src, dst, n; };
   std::vector<Backup> backups;
   if (!rsegs.empty()) {
-    int r = C->rev_addref(rsegs, rres);
+    int r = rev_stale ? CGCM_E_UNREGISTERED : C->rev_addref(rsegs, rres);
     if (r == CGCM_OK) {
       rev_done = true;
     } else if (r == CGCM_E_UNREGISTERED) {
@@ -2258,6 +2272,12 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
     if (C->flags & CGCM_LENIENT) C->st.passthrough += rres.misses;
   }
   for (auto &o : outs) C->uarr[o.unit] = 1;
+  if (!rev_done)  // every outer of the call was translated from its host slots just now
+    for (auto &o : outs) C->arr_gen[o.info.base] = C->free_gen;
+  else
+    for (auto &sg : fsegs)
+      for (auto &o : outs)
+        if (C->udev[o.unit] == sg.ptr) C->arr_gen[o.info.base] = C->free_gen;
   for (size_t j = 0; j < k; ++j) {
     const Outer &o = outs[which[j]];
     uint64_t dev = C->udev[o.unit];

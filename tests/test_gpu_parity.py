@@ -1121,7 +1121,15 @@ def test_random_array_batches_lenient(cgcm_mod):
         o.close()
 
 
-def _random_array_batches(pair, seed, nested, stray=False):
+@pytest.mark.parametrize("seed", [51, 52])
+def test_random_array_batches_with_churn(pair, seed):
+    """The batch-form program with declares / undeclares of extra leaves between calls and the CPU
+    rewriting slots of outers that are not mapped (legal: A16 only forbids writes to mapped AUs), so
+    outers gain pointers to new units and to units that are later undeclared."""
+    _random_array_batches(pair, seed, True, churn=True)
+
+
+def _random_array_batches(pair, seed, nested, stray=False, churn=False):
     """Seeded random differential run of the batch forms: mapArrays / unmapArrays / releaseArrays over
     multisets of 12 outers (repeats within a batch, SURVEY §8(b) sequential semantics), GPU writes to
     leaf units between launches, occasional unbalanced calls (NOT_MAPPED, all-or-nothing); full state
@@ -1147,7 +1155,29 @@ def _random_array_batches(pair, seed, nested, stray=False):
                   .view(np.uint8)[:8 * n + 8])
         outers.append(o)
     held = {o: 0 for o in outers}
+    rng2 = np.random.default_rng(seed + 1000)
+    extra = []
     for step in range(150):
+        if churn and rng2.random() < 0.25:
+            rc = {u["base"]: u["refCount"] for u in P.o.dump()}
+            if extra and rng2.random() < 0.4:
+                b = extra[int(rng2.integers(0, len(extra)))]
+                assert P.undeclare(b) == (0 if rc.get(b, 0) == 0 else -5)
+                if rc.get(b, 0) == 0:
+                    extra.remove(b)
+            else:
+                b = buf.addr + 0x40000 + 0x100 * int(rng2.integers(0, 512))
+                if b not in extra:                     # (P.declare writes the host bytes first)
+                    assert P.declare(b, 40, rng2.integers(0, 255, 40, dtype=np.uint8)) == 0
+                    extra.append(b)
+            j = int(rng2.integers(0, 12))
+            o = outers[j]
+            size = P.units[o]
+            if rc.get(o, 0) == 0 and size >= 8 and extra:   # the CPU rewrites an unmapped outer's slot
+                slot = int(rng2.integers(0, size // 8))
+                v = extra[int(rng2.integers(0, len(extra)))] + int(rng2.integers(0, 41))
+                host_write(o + 8 * slot, np.array([v], dtype=np.uint64))
+                P.sync_host_to_oracle(o, size)
         r = rng.random()
         k = int(rng.integers(1, 6))
         if r < 0.4:
@@ -1302,7 +1332,8 @@ def _random_device_slices(pair, seed, stray=False, churn=False):
                     extra.remove(b)
             else:
                 b = xbuf.addr + 0x100 * int(rng2.integers(0, 256))
-                if P.declare(b, 64, rng2.integers(0, 255, 64, dtype=np.uint8)) == 0:
+                if b not in extra:                     # (P.declare writes the host bytes first)
+                    assert P.declare(b, 64, rng2.integers(0, 255, 64, dtype=np.uint8)) == 0
                     extra.append(b)
             j = int(rng2.integers(0, len(bounds)))
             if state[j] == "cpu" and extra:             # point a CPU-state slot at an extra unit
