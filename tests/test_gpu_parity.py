@@ -1121,7 +1121,7 @@ def test_random_array_batches_lenient(cgcm_mod):
         o.close()
 
 
-@pytest.mark.parametrize("seed", [51, 52])
+@pytest.mark.parametrize("seed", [51, 52, 53, 54, 55, 56])
 def test_random_array_batches_with_churn(pair, seed):
     """The batch-form program with declares / undeclares of extra leaves between calls and the CPU
     rewriting slots of outers that are not mapped (legal: A16 only forbids writes to mapped AUs), so
@@ -1289,7 +1289,7 @@ def test_random_device_slices_lenient(cgcm_mod):
         o.close()
 
 
-@pytest.mark.parametrize("seed", [21, 22])
+@pytest.mark.parametrize("seed", [21, 22, 23, 24])
 def test_random_device_slices_with_table_churn(pair, seed):
     """The device-slice program with declares / undeclares between calls (a0: the table and its index
     are rebuilt and unit indices move while slices hold recorded shadows), new units written into slices
