@@ -1218,7 +1218,14 @@ def test_random_scalar_batches(pair, seed):
     _random_scalar_batches(pair, seed)
 
 
-def _random_scalar_batches(pair, seed):
+@pytest.mark.parametrize("seed", [61, 62, 63])
+def test_random_scalar_batches_with_churn(pair, seed):
+    """The scalar batch program with heap AUs declared / undeclared between calls (table rebuilds while
+    units are mapped; undeclare of a mapped AU is BUSY)."""
+    _random_scalar_batches(pair, seed, churn=True)
+
+
+def _random_scalar_batches(pair, seed, churn=False):
     """Seeded random differential run of mapBatch / unmapBatch / releaseBatch over interior pointers
     with repeats inside a batch (a batch = its sequential loop: repeated unmaps copy at most once per
     epoch, repeated releases count down), heap AUs and two globals (never freed), GPU writes between
@@ -1236,7 +1243,25 @@ def _random_scalar_batches(pair, seed):
         P.declare_global(f"g{seed}_{k}", b, s, ro=ro)
         units.append((b, s))
     held = {}
+    rng2 = np.random.default_rng(seed + 1000)
+    xbuf = HostBuf(1 << 16)
+    extra = []
     for step in range(150):
+        if churn and rng2.random() < 0.3:
+            if extra and rng2.random() < 0.4:
+                b, sz = extra[int(rng2.integers(0, len(extra)))]
+                rc = {u["base"]: u["refCount"] for u in P.o.dump()}.get(b, 0)
+                assert P.undeclare(b) == (0 if rc == 0 else -5)
+                if rc == 0:
+                    extra.remove((b, sz))
+                    units.remove((b, sz))
+            else:
+                b = xbuf.addr + 0x100 * int(rng2.integers(0, 256))
+                if all(b != e[0] for e in extra):
+                    sz = 8 * int(rng2.integers(1, 32))
+                    assert P.declare(b, sz, rng2.integers(0, 255, sz, dtype=np.uint8)) == 0
+                    extra.append((b, sz))
+                    units.append((b, sz))
         r = rng.random()
         k = int(rng.integers(1, 12))
         pick = [units[int(i)] for i in rng.integers(0, len(units), k)]
