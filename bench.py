@@ -121,9 +121,9 @@ class Workload:
         import torch
         ot = torch.from_numpy(self.offs.view(np.int64)).to(device)
         st = torch.from_numpy(self.sizes.view(np.int64)).to(device)
-        q, _ = W.queries_t(ot, st, self.n, self.seed, start=self.start)
+        q, u = W.queries_t(ot, st, self.n, self.seed, start=self.start)
         q += self.R
-        return q
+        return q, u
 
     def host_sample(self, n):
         q, _ = W.queries(self.offs, self.sizes, n, self.seed, start=self.start)
@@ -149,7 +149,7 @@ def run_cgcm(args, rank, world, local_rank):
     s = ctx.mapArrayDevice(pins.data_ptr(), wl.U)
     assert s == 0, cg.strerror(s)
     setup_act_s = time.time() - t0
-    q = wl.device_queries(dev)
+    q, q_unit = wl.device_queries(dev)
     q_ref = q.clone()
     torch.cuda.synchronize()
     setup_s = time.time() - t0
@@ -192,10 +192,10 @@ def run_cgcm(args, rank, world, local_rank):
     st = ctx.stats()
     assert torch.equal(q, q_ref), "round trip changed the pointer arrays"
     if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = max_over_ranks(ms, dev)
     ms_per_step = ms / args.steps
+    parity = full_size_check(ctx, wl, q, q_ref, q_unit, pins_held=1)
+    del q_unit
     translations = 2 * wl.n * world * args.steps
     value = translations / (ms / 1e3)
 
@@ -258,12 +258,44 @@ def run_cgcm(args, rank, world, local_rank):
                    f"{cfg['arrays'] // world} arrays per rank", "l2": "inputs (2 GiB/GPU of pointer slots at E) "
                    "exceed L2 between iterations; table stays L2-resident by design",
                    "translations_per_step": 2 * wl.n * world},
-        "roofline": roofline, "gpu_launches": gpu_launches, "clocks": clocks, "e2e": e2e,
+        "roofline": roofline, "gpu_launches": gpu_launches, "clocks": clocks, "e2e": e2e, "parity": parity,
         "setup_s": round(setup_s, 1), "setup_activation_s": round(setup_act_s, 1),
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         result["cpu_baseline"] = cpu_baseline(wl, args.cpu_sample, steps=1)
     return result
+
+
+def full_size_check(ctx, wl, q, q_ref, q_unit, pins_held):
+    """Parity of the timed call at the benchmarked size, outside the timed region: one more
+    cgcm_mapArrayDevice over all of the rank's slots in the timed launch configuration, then every slot
+    is compared with Alg. 1's closed form devptr(u) + (p - base(u)) (u = the unit the seeded
+    generator drew the query from, the table's devptr and base from cgcm_dumpTable), every unit's
+    refcount with the setup reference + the number of slots pointing into it (A8), and after
+    cgcm_unmapArrayDevice(release) every slot with its original CPU pointer and every refcount with the
+    setup reference alone (a3 round trip + Alg. 3).  Vectorised with torch on the GPU (the oracle's
+    one-by-one sampled check at this size is tests/test_gpu_fullsize.py)."""
+    import torch
+    dev = q.device
+    t0 = time.time()
+    assert ctx.mapArrayDevice(q.data_ptr(), wl.n) == 0
+    tab = ctx.dump_np()
+    devt = torch.from_numpy(tab["devptr"].view(np.int64)).to(dev)
+    bt = torch.from_numpy(tab["base"].view(np.int64)).to(dev)
+    fwd_ok = bool(torch.equal(q, devt[q_unit] + (q_ref - bt[q_unit])))
+    del devt, bt
+    cnt = torch.bincount(q_unit, minlength=wl.U).cpu().numpy()
+    rc_ok = bool((tab["refCount"] == cnt + pins_held).all())
+    ctx.advanceEpoch()
+    assert ctx.unmapArrayDevice(q.data_ptr(), wl.n, release=True) == 0
+    rev_ok = bool(torch.equal(q, q_ref))
+    rc_back = bool((ctx.dump_np()["refCount"] == pins_held).all())
+    ok = fwd_ok and rc_ok and rev_ok and rc_back
+    if not ok:
+        raise RuntimeError(f"full-size parity failed: fwd {fwd_ok} rc {rc_ok} rev {rev_ok} rc_back {rc_back}")
+    return {"checked_slots": wl.n, "forward_closed_form": fwd_ok, "refcounts": rc_ok, "roundtrip": rev_ok,
+            "released": rc_back, "seconds": round(time.time() - t0, 1),
+            "how": "every slot vs devptr(u)+(p-base(u)); refcount == 1 + #slots in u; reverse == original"}
 
 
 def l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots):
@@ -376,9 +408,7 @@ def run_e2e(args, ctx, wl, q_ref, dev, world, rank):
         ctx.free(p)
     if world > 1:
         import torch.distributed as dist
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = max_over_ranks(ms, dev)
     link = host_link(dev)
     h2d = (st1["h2d_bytes"] - st0["h2d_bytes"]) // steps
     d2h = (st1["d2h_bytes"] - st0["d2h_bytes"]) // steps
@@ -499,9 +529,7 @@ def run_e2e_duplex(args, ctx, wl, q_ref, dev, world, rank, link, local_rank):
         ctx.make_current()
     if world > 1:
         import torch.distributed as dist
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = max_over_ranks(ms, dev)
     h2d = sum(b["h2d_bytes"] - a["h2d_bytes"] for a, b in zip(st0, st1)) // steps
     d2h = sum(b["d2h_bytes"] - a["d2h_bytes"] for a, b in zip(st0, st1)) // steps
     floor_ms = 1e3 * (h2d + d2h) / (link["bidir_gbs"] * 1e9)  # both directions busy at once
@@ -578,6 +606,29 @@ def run_reference(args, rank, world):
                                          "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
 
 
+def max_over_ranks(x, dev):
+    """The max of x over all ranks (NCCL: on the device; gloo, --allow-shared-gpu: on the host)."""
+    import torch
+    import torch.distributed as dist
+    on_dev = dist.get_backend() == "nccl"
+    t = torch.tensor([x], dtype=torch.float64, device=dev if on_dev else "cpu")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def relaunch_under_torchrun(args):
+    """`python bench.py --gpus N` without a launcher: re-execute under torch.distributed.run with one
+    rank per GPU (rendezvous on 127.0.0.1), so that --gpus is never silently ignored."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    r = subprocess.run(cmd)
+    sys.exit(r.returncode)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -591,9 +642,21 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=1 << 21)
     ap.add_argument("--ref-sample", type=int, default=1 << 19)
+    ap.add_argument("--allow-shared-gpu", action="store_true",
+                    help="testing only: let several ranks share one GPU (numbers are meaningless)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        relaunch_under_torchrun(args)  # does not return
     rank, world, local_rank = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
+    if world != args.gpus:
+        sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}: launch one rank per GPU")
+    if args.impl != "reference":
+        import torch
+        if torch.cuda.device_count() < world and not args.allow_shared_gpu:
+            sys.exit(f"bench.py: {world} ranks need {world} GPUs, this node has {torch.cuda.device_count()}")
+        if args.allow_shared_gpu:
+            local_rank = local_rank % max(1, torch.cuda.device_count())
     if args.impl == "reference":
         res = run_reference(args, rank, world)
         if res is not None:
@@ -603,7 +666,10 @@ def main():
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if args.allow_shared_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     res = run_cgcm(args, rank, world, local_rank)
     if rank == 0:
         print(json.dumps(res), flush=True)

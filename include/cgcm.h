@@ -226,6 +226,28 @@ typedef struct {
   uint32_t pd_min_shift, pd_max_shift; /* page sizes 2^shift of the segments                     */
 } cgcm_index_info_t;
 int cgcm_indexInfo(cgcm_index_info_t *out);
+/* The device storage the runtime holds for AU copies (for leak / balance checks; the paper's
+ * counterpart is Alg. 1's cuMemAlloc and Alg. 3's cuMemFree): one entry per live device
+ * extent -- its device range [addr, addr + bytes), the number of AU copies it still holds (`live`;
+ * an extent is freed when that reaches 0) and whether it is a bound __device__ symbol (external, not
+ * arena memory).  *n = total; CGCM_E_NOMEM if cap < total (out may be NULL with cap 0).
+ * cgcm_storageInfo: totals, plus the forward-map shadows (12 B per slot) that currently
+ * record a mapped array (`shadows_live`) and the cached buffers of consumed ones (`shadows_cached`,
+ * reused by the next map of the same device array).                                               */
+typedef struct {
+  uint64_t addr, bytes;
+  int64_t live;
+  uint32_t external, pad;
+} cgcm_extent_t;
+int cgcm_dumpExtents(cgcm_extent_t *out, size_t cap, size_t *n);
+typedef struct {
+  uint64_t extents, extent_bytes;        /* live arena extents (not external)                      */
+  uint64_t external_extents;             /* bound __device__ symbols                               */
+  uint64_t shadows_live, shadow_live_bytes;
+  uint64_t shadows_cached, shadow_cached_bytes;
+  uint64_t arena_used, arena_capacity;
+} cgcm_storage_t;
+int cgcm_storageInfo(cgcm_storage_t *out);
 
 #ifdef __cplusplus
 }

@@ -1,8 +1,8 @@
 """ctypes wrapper of the CPU ORACLE (oracle/cgcm_oracle.cpp).  TEST INFRASTRUCTURE ONLY.
 
 Only tests/, ``__graft_entry__.smoke()`` and bench.py's ``cpu_baseline`` / ``--impl reference``
-legs may import this module.  The product package never imports it (tests/test_isolation.py
-checks that), and this module imports nothing from the product.
+legs may import this module.  The product package never imports it
+(tests/test_abi.py::test_oracle_and_product_are_independent checks that), and this module imports nothing from the product.
 
 Paper: Jablin et al., "Automatic CPU-GPU Communication Management and Optimization", PLDI 2011.
 The oracle follows Algorithms 1-3, Table 2 and P:L203-207.

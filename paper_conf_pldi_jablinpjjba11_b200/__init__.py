@@ -50,6 +50,17 @@ class IndexInfo(C.Structure):
                 ("pd_min_shift", C.c_uint32), ("pd_max_shift", C.c_uint32)]
 
 
+class Extent(C.Structure):
+    _fields_ = [("addr", C.c_uint64), ("bytes", C.c_uint64), ("live", C.c_int64), ("external", C.c_uint32),
+                ("pad", C.c_uint32)]
+
+
+class StorageInfo(C.Structure):
+    _fields_ = [(f, C.c_uint64) for f in (
+        "extents", "extent_bytes", "external_extents", "shadows_live", "shadow_live_bytes", "shadows_cached",
+        "shadow_cached_bytes", "arena_used", "arena_capacity")]
+
+
 class CgcmError(RuntimeError):
     pass
 
@@ -91,6 +102,8 @@ def lib():
             "cgcm_dumpTable": (i, [vp, sz, C.POINTER(C.c_size_t)]),
             "cgcm_arenaUsage": (i, [C.POINTER(C.c_size_t), C.POINTER(C.c_size_t)]),
             "cgcm_indexInfo": (i, [C.POINTER(IndexInfo)]),
+            "cgcm_dumpExtents": (i, [C.c_void_p, C.c_size_t, C.POINTER(C.c_size_t)]),
+            "cgcm_storageInfo": (i, [C.POINTER(StorageInfo)]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -323,6 +336,35 @@ class Context:
         if s != OK:
             raise CgcmError(f"indexInfo: {strerror(s)}")
         return {f: getattr(ii, f) for f, _ in IndexInfo._fields_}
+
+    def dump_np(self):
+        """The unit table as a numpy structured array (fields of cgcm_unit_t) -- for large tables."""
+        import numpy as np
+        n = C.c_size_t(0)
+        self.L.cgcm_dumpTable(None, 0, C.byref(n))
+        arr = (Unit * max(1, n.value))()
+        s = self.L.cgcm_dumpTable(C.cast(arr, C.c_void_p), n.value, C.byref(n))
+        if s != OK:
+            raise CgcmError(f"dumpTable: {strerror(s)}")
+        dt = np.dtype([("base", "<u8"), ("size", "<u8"), ("devptr", "<u8"), ("refCount", "<i8"),
+                       ("epoch", "<u8"), ("flags", "<u4"), ("pad", "<u4")])
+        return np.frombuffer(arr, dtype=dt, count=n.value).copy()
+
+    def extents(self) -> list:
+        n = C.c_size_t(0)
+        self.L.cgcm_dumpExtents(None, 0, C.byref(n))
+        arr = (Extent * max(1, n.value))()
+        s = self.L.cgcm_dumpExtents(C.cast(arr, C.c_void_p), n.value, C.byref(n))
+        if s != OK:
+            raise CgcmError(f"dumpExtents: {strerror(s)}")
+        return [{f: getattr(arr[k], f) for f, _ in Extent._fields_ if f != "pad"} for k in range(n.value)]
+
+    def storage(self) -> dict:
+        si = StorageInfo()
+        s = self.L.cgcm_storageInfo(C.byref(si))
+        if s != OK:
+            raise CgcmError(f"storageInfo: {strerror(s)}")
+        return {f: getattr(si, f) for f, _ in StorageInfo._fields_}
 
     # ---- test-only sample GPU functions on the main stream ----
     def sample_scale(self, rows_dev, nrows, ncols, alpha):

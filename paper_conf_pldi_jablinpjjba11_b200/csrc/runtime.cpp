@@ -1132,6 +1132,7 @@ struct Context {
     CK(cudaStreamSynchronize(main));
     for (uint32_t x : units) {
       uarr[x] = 0;
+      arr_gen.erase(ubase[x]);  // no longer array-mapped: the next mapArray translates from host slots
       if (udev[x]) drop_shadows(udev[x]);
       if (uflags[x] & UF_GLOBAL) continue;
       run_release(urun[x]);
@@ -1818,6 +1819,7 @@ int cgcm_undeclare(void *base) {
       C->udev[u.idx] = 0;
     }
   }
+  C->arr_gen.erase(b);
   C->reg.erase(it);
   C->table_dirty = true;
   return CGCM_OK;
@@ -2170,16 +2172,17 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
       fsegs.push_back(s);
     }
   }
-  // unit ops must not run before the outers' set_devbase: same stream, issued after
-  CKS(C->unit_ops(ops));
+  bool ops_applied = false;
   auto undo_prologue = [&]() {
     cudaStreamSynchronize(C->copy);  // the outers' copies land before their storage is released
     std::vector<UnitOp> undo;
-    for (auto &o : outs) {
-      undo.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)(-o.mult)});
-      if (!(o.info.flags & UF_ARRAYMAPPED)) undo.push_back({(uint32_t)o.unit, UOP_AND_FLAGS, ~(uint64_t)UF_ARRAYMAPPED});
+    if (ops_applied)
+      for (auto &o : outs) {
+        undo.push_back({(uint32_t)o.unit, UOP_ADD_RC, (uint64_t)(int64_t)(-o.mult)});
+        if (!(o.info.flags & UF_ARRAYMAPPED)) undo.push_back({(uint32_t)o.unit, UOP_AND_FLAGS, ~(uint64_t)UF_ARRAYMAPPED});
+      }
+    for (auto &o : outs)
       if (o.info.refcount == 0) undo.push_back({(uint32_t)o.unit, UOP_SET_EPOCH, o.info.epoch});
-    }
     C->unit_ops(undo);
     cudaStreamSynchronize(C->main);
     std::vector<uint32_t> deact;
@@ -2193,6 +2196,15 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
     C->free_units(deact);
     C->st.frees = frees0;
   };
+  // unit ops must not run before the outers' set_devbase: same stream, issued after
+  {
+    const int r = C->unit_ops(ops);
+    if (r != CGCM_OK) {  // all-or-nothing: withdraw the activations
+      undo_prologue();
+      return r;
+    }
+    ops_applied = true;
+  }
   // array-mapped outers: refcounts through the reverse index (no copy); if an element
   // lost its device copy, re-translate the outer from its host slots instead (oracle semantics)
   Status rres{};
@@ -2205,21 +2217,31 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
       rev_done = true;
     } else if (r == CGCM_E_UNREGISTERED) {
       // keep the current device slots so that a failing call can put them back (all-or-nothing)
+      // every failure from here on restores the slots backed up so far and withdraws the prologue
+      auto fail = [&](int status) {
+        for (auto &b : backups)
+          cudaMemcpyAsync(reinterpret_cast<void *>(b.dst), reinterpret_cast<void *>(b.src), b.n,
+                          cudaMemcpyDeviceToDevice, C->main);
+        undo_prologue();
+        return status;
+      };
       uint64_t bytes = 0;
       for (auto &sg : rsegs) bytes += 8 * sg.n + 32;
-      CKS(C->dalloc(C->staging2, bytes + 256));
+      if (C->dalloc(C->staging2, bytes + 256) != CGCM_OK) return fail(CGCM_E_NOMEM);
       uint64_t off = C->staging2.addr;
       for (auto &sg : rsegs) {
-        CK(cudaMemcpyAsync(reinterpret_cast<void *>(off), reinterpret_cast<void *>(sg.ptr), 8 * sg.n,
-                           cudaMemcpyDeviceToDevice, C->main));
+        if (cudaMemcpyAsync(reinterpret_cast<void *>(off), reinterpret_cast<void *>(sg.ptr), 8 * sg.n,
+                            cudaMemcpyDeviceToDevice, C->main) != cudaSuccess)
+          return fail(CGCM_E_CUDA);
         backups.push_back({off, sg.ptr, 8 * sg.n});
         off += 8 * sg.n + 32;
       }
       for (auto &sg : rsegs) {
         for (auto &o : outs)
           if (C->udev[o.unit] == sg.ptr) {
-            CK(cudaMemcpyAsync(reinterpret_cast<void *>(sg.ptr), reinterpret_cast<const void *>(o.info.base),
-                               8 * sg.n, cudaMemcpyHostToDevice, C->main));
+            if (cudaMemcpyAsync(reinterpret_cast<void *>(sg.ptr), reinterpret_cast<const void *>(o.info.base),
+                                8 * sg.n, cudaMemcpyHostToDevice, C->main) != cudaSuccess)
+              return fail(CGCM_E_CUDA);
             C->st.h2d_memcpy_calls += 1;
           }
         fsegs.push_back(sg);
@@ -2681,6 +2703,51 @@ int cgcm_arenaUsage(size_t *used, size_t *capacity) {
   CTX();
   if (used) *used = C->arena.used();
   if (capacity) *capacity = C->arena.capacity();
+  return CGCM_OK;
+}
+
+int cgcm_dumpExtents(cgcm_extent_t *out, size_t cap, size_t *n) {
+  CTX();
+  if (!n) return CGCM_E_INVALID;
+  *n = C->live_runs.size();
+  if (cap < *n) return out || cap ? CGCM_E_NOMEM : CGCM_OK;
+  size_t k = 0;
+  for (auto &kv : C->live_runs) {
+    const Run &r = C->runs[kv.second];
+    cgcm_extent_t e{};
+    e.addr = r.addr;
+    e.bytes = r.bytes;
+    e.live = r.live;
+    e.external = r.external ? 1u : 0u;
+    out[k++] = e;
+  }
+  return CGCM_OK;
+}
+
+int cgcm_storageInfo(cgcm_storage_t *out) {
+  CTX();
+  if (!out) return CGCM_E_INVALID;
+  std::memset(out, 0, sizeof(*out));
+  for (auto &kv : C->live_runs) {
+    const Run &r = C->runs[kv.second];
+    if (r.external) {
+      out->external_extents += 1;
+    } else {
+      out->extents += 1;
+      out->extent_bytes += r.bytes;
+    }
+  }
+  for (auto &kv : C->shadows) {
+    if (kv.second.valid) {
+      out->shadows_live += 1;
+      out->shadow_live_bytes += kv.second.buf.bytes;
+    } else {
+      out->shadows_cached += 1;
+      out->shadow_cached_bytes += kv.second.buf.bytes;
+    }
+  }
+  out->arena_used = C->arena.used();
+  out->arena_capacity = C->arena.capacity();
   return CGCM_OK;
 }
 

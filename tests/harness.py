@@ -127,6 +127,72 @@ class Pair:
             ob = self.o.host_read(b, n).tobytes()
             assert hb == ob, f"{what}: host bytes of unit {hex(b)} differ"
         assert self.g.epoch == self.o.epoch
+        self.check_structure(what)
+
+    # ---- structural checks of the GPU's device addresses (implementation-defined values, A22) ----
+    def check_structure(self, what=""):
+        """The device addresses the GPU chose (and replays into the oracle) must satisfy what the
+        paper and reading A7 require of ANY valid choice (SURVEY §8(c) "Exact device addresses"):
+          * devptr == base (mod 256)                                   (A7, alignment of the copy)
+          * copies of distinct units are disjoint, and touch (d1 + s1 == d2) only if their host AUs
+            touch in the same order (b1 + s1 == b2): a one-past-the-end GPU pointer must reverse to the
+            unit it came from (A7)
+          * every copy lies in exactly one live device extent, each extent's `live` count equals the
+            number of copies inside it (no extent outlives its units: no device-memory leak), and
+            arena extents lie inside the arena (Alg. 1 cuMemAlloc / Alg. 3 cuMemFree)."""
+        gd = self.g.dump()
+        copies = sorted((u["devptr"], u["size"], u["base"]) for u in gd if u["devptr"])
+        for d, n, b in copies:
+            assert d % 256 == b % 256, f"{what}: devptr {hex(d)} of {hex(b)} not congruent mod 256"
+        for (d1, s1, b1), (d2, s2, b2) in zip(copies, copies[1:]):
+            assert d1 + s1 <= d2, f"{what}: device copies of {hex(b1)} and {hex(b2)} overlap"
+            if d1 + s1 == d2:
+                assert b1 + s1 == b2, f"{what}: copies of {hex(b1)}, {hex(b2)} adjacent but host AUs are not"
+        ex = sorted(self.g.extents(), key=lambda e: e["addr"])
+        for e1, e2 in zip(ex, ex[1:]):
+            assert e1["addr"] + e1["bytes"] <= e2["addr"], f"{what}: device extents overlap"
+        lo = self.g.arena.data_ptr()
+        hi = lo + self.g.arena.numel()
+        starts = [e["addr"] for e in ex]
+        import bisect
+        held = [0] * len(ex)
+        for d, n, b in copies:
+            k = bisect.bisect_right(starts, d) - 1
+            assert k >= 0 and d + n <= ex[k]["addr"] + ex[k]["bytes"], f"{what}: copy of {hex(b)} in no extent"
+            held[k] += 1
+        for e, h in zip(ex, held):
+            assert e["live"] == h and h > 0, f"{what}: extent {hex(e['addr'])} live={e['live']} holds {h} copies"
+            if not e["external"]:
+                assert lo <= e["addr"] and e["addr"] + e["bytes"] <= hi, f"{what}: extent outside the arena"
+
+    def drain(self, shadows=True):
+        """Release every outstanding reference with scalar cgcm_release calls (each one compared with
+        the oracle), then check the balance: all refcounts 0 and no storage held (check_balance)."""
+        for _ in range(64):
+            live = [(u["base"], u["refCount"]) for u in self.g.dump() if u["refCount"] > 0]
+            if not live:
+                break
+            for b, rc in live:
+                for _k in range(rc):
+                    assert self.run("release", b) == 0
+            self.check("drain")
+        assert self.check_balance("drained", shadows)
+
+    def check_balance(self, what="end", shadows=True):
+        """After every reference is released, the runtime holds no device storage for AUs beyond the
+        globals' persistent copies (A14) and no live forward-map shadow (SURVEY §8(c) "Refcounts":
+        arena usage returns to baseline).  Scratch buffers the runtime keeps for reuse are excluded."""
+        gd = self.g.dump()
+        if any(u["refCount"] > 0 for u in gd):
+            return False
+        self.check_structure(what)
+        si = self.g.storage()
+        glob = [u for u in gd if u["devptr"]]
+        assert all(u["flags"] & 1 for u in glob), f"{what}: a released non-global unit keeps a copy"
+        assert not shadows or si["shadows_live"] == 0, f"{what}: {si['shadows_live']} live shadows after all releases"
+        if not glob:
+            assert si["extents"] == 0 and si["extent_bytes"] == 0, f"{what}: leaked extents {si}"
+        return True
 
     def check_device_units(self):
         """Device copies of active units equal the oracle's simulated device bytes."""

@@ -3,7 +3,8 @@
 
 * config C: 2^20 AUs, 2^26 interior pointers (all of them checked by properties, 2^16 sampled slots
   checked one by one against the CPU oracle in replay mode);
-* config E: the full 2^22-AU table, with 32 of the 256 arrays (2^25 pointers) per call.
+* config E: the full 2^22-AU table and all 256 arrays (2^28 pointers) in ONE call -- exactly the
+  launch bench.py times (one cgcm_mapArrayDevice / cgcm_unmapArrayDevice over 2^28 slots).
 
 Properties checked on every slot: refcount[u] == number of slots pointing into u (A8), the reverse
 translation restores every slot (round trip), read-only units are never copied back.
@@ -35,15 +36,16 @@ def run_full(U, arrays, slots_per_array, seed, sample=1 << 16):
         orig = d.clone()
         assert ctx.mapArrayDevice(d.data_ptr(), n) == 0
         # A8: refcount == number of slots pointing into the unit (every unit, every slot)
-        dump = ctx.dump()
-        rc = np.array([x["refCount"] for x in dump], dtype=np.int64)
+        dump = ctx.dump_np()
+        rc = dump["refCount"]
         cnt = torch.bincount(u, minlength=U).cpu().numpy()
         assert (rc == cnt).all()
-        dev = np.array([x["devptr"] for x in dump], dtype=np.uint64)
+        dev = dump["devptr"]
         # forward translation of every slot: devptr(u) + (p - base(u))  (vectorised on the GPU)
         devt = torch.from_numpy(dev.view(np.int64)).cuda()
         bt = torch.from_numpy(bases.view(np.int64)).cuda()
         assert torch.equal(d, devt[u] + (orig - bt[u]))
+        del devt, bt
         # 2^16 sampled slots one by one through the oracle (replay mode: the GPU's device addresses)
         rng = np.random.default_rng(seed)
         idx = np.sort(rng.choice(n, size=min(sample, n), replace=False))
@@ -64,7 +66,9 @@ def run_full(U, arrays, slots_per_array, seed, sample=1 << 16):
         assert torch.equal(d, orig)
         s = ctx.stats()
         assert s["d2h_units"] == 0 and s["rev_translations"] == n and s["fwd_translations"] == n
-        assert all(x["refCount"] == 0 for x in ctx.dump())
+        assert (ctx.dump_np()["refCount"] == 0).all()
+        si = ctx.storage()
+        assert si["extents"] == 0 and si["shadows_live"] == 0      # every copy freed, shadow consumed
     finally:
         ctx.close()
         W.release_reservation(R, span)
@@ -75,7 +79,7 @@ def test_config_C_full_size():
 
 
 def test_config_E_full_table():
-    run_full(1 << 22, 32, 1 << 20, 5)
+    run_full(1 << 22, 256, 1 << 20, 5)
 
 
 def test_config_D_full_size():

@@ -378,3 +378,83 @@ def test_batch_forms_are_their_sequential_loops(seed):
     assert n_ok > 100 and n_err >= 1
     A.close()
     B.close()
+
+
+# ---- A18 lenient mode, pinned by hand (VERDICT r1 "What's weak" 1) -----------------------------------
+# Reading A18 (field-insensitive typing may label a struct holding data words
+# as a pointer array): in lenient mode a non-null word that no AU covers passes through unchanged, is
+# counted once per word per call (`passthrough`), and takes no reference; unmap/release of an
+# uncovered pointer are no-ops returning OK.  Every expected value below is counted by hand from that
+# reading; none is read back from the oracle.
+def _lenient_setup(o):
+    A, B, PP = 0x10000, 0x20000, 0x30000
+    STRAY = 0x50000                                   # below DEV0, in no host AU and no device copy
+    assert o.declareAlloc(A, 64) == OK
+    assert o.declareAlloc(B, 64) == OK
+    o.host_write(A, np.arange(64, dtype=np.uint8))
+    o.host_write(B, np.arange(64, 128, dtype=np.uint8))
+    words = np.array([A + 8, STRAY, 0, B, STRAY], dtype=np.uint64)   # the stray word twice, one NULL
+    assert o.declareAlloc(PP, 8 * len(words)) == OK
+    o.host_write(PP, words)
+    return A, B, PP, STRAY, words
+
+
+def test_lenient_mode_hand_counts():
+    from oracle import LENIENT
+    o = Oracle(LENIENT)
+    try:
+        A, B, PP, STRAY, words = _lenient_setup(o)
+        st, d = o.mapArray(PP)
+        assert st == OK
+        u = {x["base"]: x for x in o.dump()}
+        dev = o.dev_read(u[PP]["devptr"], 8 * len(words)).view(np.uint64)
+        # device slots: translated, stray raw (twice), NULL, translated
+        assert list(dev) == [u[A]["devptr"] + 8, STRAY, 0, u[B]["devptr"], STRAY]
+        s = o.stats()
+        assert s["passthrough"] == 2                      # per word, not per distinct value or per call
+        assert s["null_slots"] == 1
+        assert s["fwd_translations"] == 2                 # A+8 and B only
+        assert s["h2d_units"] == 3 and s["activations"] == 3
+        assert (u[PP]["refCount"], u[A]["refCount"], u[B]["refCount"]) == (1, 1, 1)   # no ref for STRAY
+        o.advanceEpoch()
+        assert o.unmapArray(PP) == OK
+        host = o.host_read(PP, 8 * len(words)).view(np.uint64)
+        assert (host == words).all()                      # the stray word comes back unchanged
+        s = o.stats()
+        assert s["passthrough"] == 4                      # + 2: the outer is reversed once, its 2 stray words each pass
+        assert s["rev_translations"] == 2
+        assert s["d2h_units"] == 3                        # outer + A + B; nothing for STRAY
+        # scalar calls on an uncovered pointer: OK and no effect
+        before = (o.dump(), o.stats())
+        assert o.unmap(STRAY) == OK and o.release(STRAY) == OK
+        assert (o.dump(), o.stats()) == before
+        st, t = o.map(STRAY)
+        assert st == OK and t == STRAY and o.stats()["passthrough"] == 5
+        assert o.releaseArray(PP) == OK
+        assert all(x["refCount"] == 0 for x in o.dump())
+        assert o.stats()["frees"] == 3
+        # device slots: the same stray passes through mapSlots / unmapSlots
+        slots = np.array([STRAY, A + 1, 0], dtype=np.uint64)
+        assert o.mapSlots(slots) == OK
+        assert int(slots[0]) == STRAY and int(slots[2]) == 0
+        assert {x["base"]: x for x in o.dump()}[A]["refCount"] == 1
+        o.advanceEpoch()
+        assert o.unmapSlots(slots, release=True) == OK
+        assert list(slots) == [STRAY, A + 1, 0]
+        assert all(x["refCount"] == 0 for x in o.dump())
+    finally:
+        o.close()
+
+
+def test_strict_mode_rejects_the_same_program():
+    o = Oracle()
+    try:
+        A, B, PP, STRAY, words = _lenient_setup(o)
+        before = (o.dump(), o.stats())
+        assert o.mapArray(PP)[0] == E_UNREGISTERED        # A18 strict: every non-null slot must hit
+        assert (o.dump(), o.stats()) == before            # all-or-nothing
+        assert o.map(STRAY)[0] == E_UNREGISTERED
+        assert o.unmap(STRAY) == E_UNREGISTERED and o.release(STRAY) == E_UNREGISTERED
+        assert o.mapSlots(np.array([STRAY], dtype=np.uint64)) == E_UNREGISTERED
+    finally:
+        o.close()
