@@ -222,7 +222,16 @@ struct SlotArgs {
   int fx_nowide;               // the forward index has no wide bucket (specialised kernels)
   int segs_host_shadow;        // the (single) segment carries a shadow: use the shadow variant
   int seg_inplace;             // the (single) segment is translated in place (out == 0)
+  // deferred references (DESIGN.md §6 "Deferred references"): k_map_pd records the reference of a slot
+  // whose unit is already ACTIVE in the slot's shadow word (SH_DEFER) instead of adding it to rc;
+  // k_unmap_sh with defer set drops such a reference on a released hit and adds it to rc otherwise
+  int defer;
 };
+// shadow unit word: unit index | SH_DEFER (the slot's reference is not in rc yet); SH_NONE: no unit
+constexpr uint32_t SH_NONE = 0xFFFFFFFFu;
+constexpr uint32_t SH_DEFER = 0x80000000u;
+__host__ __device__ __forceinline__ uint32_t sh_unit(uint32_t w) { return w == SH_NONE ? SH_NONE : (w & ~SH_DEFER); }
+__host__ __device__ __forceinline__ bool sh_deferred(uint32_t w) { return w != SH_NONE && (w & SH_DEFER); }
 
 // ---- host-callable launchers (kernels.cu) ----------------------------------------------------
 int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, int *nlaunch);
@@ -242,6 +251,8 @@ void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n
 void launch_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
                          cudaStream_t s);
 void launch_rebase_epochs(TableDev tab, int n, uint32_t cur, cudaStream_t s);
+// add every deferred reference recorded in a shadow's n unit words to rc (they become ordinary references)
+void launch_materialise(const uint32_t *shadow_units, uint64_t n, int32_t *rc, cudaStream_t s);
 // small host<->device transfers by a kernel through mapped pinned memory instead of a DMA: a copy
 // engine serves DMAs in order, so a few bytes queued behind another context's gigabyte would wait for it
 void launch_copy_small(void *dst, const void *src, size_t n, void *dst2, const void *src2, size_t n2, cudaStream_t s);

@@ -627,8 +627,9 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
       for (int m = 0; m < 2; ++m) {
         if (!look[m]) continue;
         const int64_t i = slot0 + m;
-        const uint32_t u = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n)[i];
-        if (u == 0xFFFFFFFFu) continue;
+        // (a deferred reference was materialised by k_unmap_sh or the runtime before this pass)
+        const uint32_t u = sh_unit(reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n)[i]);
+        if (u == SH_NONE) continue;
         const uint64_t h = reinterpret_cast<const uint64_t *>(sg.shadow)[i];
         const uint64_t w = ld_u64(a.tab.st + u, pol_t);  // extent, flags and epoch in one word
         const uint32_t e = hot_ext(w);
@@ -990,10 +991,17 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
       if (look[m] && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
       hit[m] = look[m] && (k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
     }
+    // deferred reference (a.defer, SH): the unit was ACTIVE when the call began, so a reference held
+    // elsewhere keeps it active until the runtime materialises this one -- the slot's
+    // shadow word records it instead of a refcount reduction
+    bool dfr[2];
+#pragma unroll
+    for (int m = 0; m < 2; ++m) dfr[m] = SH && a.defer && hit[m] && (hot_flags(hw[m]) & UF_ACTIVE);
     if (SH && live) {  // forward-map shadow: (CPU pointer, unit) per slot for the reverse pass
       uint64_t *shp = reinterpret_cast<uint64_t *>(sg.shadow);
       uint32_t *shu = reinterpret_cast<uint32_t *>(sg.shadow + 8 * sg.n);
-      const uint32_t u0 = hit[0] ? (uint32_t)j[0] : 0xFFFFFFFFu, u1 = hit[1] ? (uint32_t)j[1] : 0xFFFFFFFFu;
+      const uint32_t u0 = hit[0] ? ((uint32_t)j[0] | (dfr[0] ? SH_DEFER : 0u)) : SH_NONE;
+      const uint32_t u1 = hit[1] ? ((uint32_t)j[1] | (dfr[1] ? SH_DEFER : 0u)) : SH_NONE;
       if (valid == 3u && !(slot0 & 1)) {
         st_stream2(shp + slot0, pol_s, cv[0], cv[1]);
         asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1,%2}, %3;" ::"l"(shu + slot0), "r"(u0),
@@ -1022,7 +1030,7 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
       if (hit[m]) {
         int32_t *RC = a.tab.rc + j[m];
         if (fl & UF_ACTIVE) {
-          red_add(RC, sg.inc);
+          if (!dfr[m]) red_add(RC, sg.inc);
         } else {
           act = atomicAdd(RC, sg.inc) == 0;  // refcount 0 -> 1: Alg. 1's activation
         }
@@ -1140,7 +1148,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   struct In {
     uint64_t a0;  // address of the chunk's first word (16-byte aligned)
     uint64_t g[2], h[2];
-    uint32_t u[2];
+    uint32_t u[2];  // shadow unit words as recorded (SH_DEFER bit included)
     uint32_t valid;
     int s;
   };
@@ -1181,7 +1189,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   auto gather = [&](const In &x, uint64_t w[2]) {
 #pragma unroll
     for (int m = 0; m < 2; ++m)
-      w[m] = (x.u[m] != 0xFFFFFFFFu && x.g[m] != 0) ? ld_u64_hot(a.tab.st + x.u[m], pol_t) : 0ull;
+      w[m] = (x.u[m] != SH_NONE && x.g[m] != 0) ? ld_u64_hot(a.tab.st + sh_unit(x.u[m]), pol_t) : 0ull;
   };
 
   const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -1205,17 +1213,23 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
       const bool look = vm && cur.g[m] != 0;
       const uint64_t w = cw[m];
       const uint32_t e = hot_ext(w);
-      hit[m] = look && cur.u[m] != 0xFFFFFFFFu && (hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext &&
+      const uint32_t su = sh_unit(cur.u[m]);
+      hit[m] = look && su != SH_NONE && (hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext &&
                cur.g[m] == cur.h[m] + (ext_s ? s_ext[e] : a.tab.ext_delta[e]);
       slow[m] = look && !hit[m];
       c_nulls += vm && cur.g[m] == 0;
       c_hits += hit[m];
-      const uint32_t unit = hit[m] ? cur.u[m] : 0u;
+      const uint32_t unit = hit[m] ? su : 0u;
       const uint32_t fl = hot_flags(w);
       int32_t *RC = a.tab.rc + unit;
       bool freed = false;
+      // a deferred reference (recorded by k_map_pd) is dropped by a released hit; any other slot turns
+      // it into an ordinary reference first (the slow pass then treats the slot like any other)
+      const bool dfr = a.defer && vm && sh_deferred(cur.u[m]);  // (also if a GPU function wrote NULL there)
+      const bool drop = dfr && hit[m] && (OPS & OP_DEC);
+      if (dfr && !drop) red_add(a.tab.rc + su, 1);
       if (OPS & OP_DEC) {
-        if (hit[m]) {
+        if (hit[m] && !drop) {
           if (a.dec_red) {
             red_add(RC, -sg.inc);
           } else {
@@ -1619,6 +1633,21 @@ void launch_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc
     (void)cudaGetLastError();
     k_release_scan<<<grid, 256, 0, s>>>(tab, n, st, lc, free_list);
   }
+}
+
+// deferred references of one shadow become ordinary references (DESIGN.md §6 "Deferred references")
+__global__ void k_materialise(const uint32_t *units, uint64_t n, int32_t *rc) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t w = units[i];
+    if (sh_deferred(w)) red_add(rc + sh_unit(w), 1);
+  }
+}
+void launch_materialise(const uint32_t *shadow_units, uint64_t n, int32_t *rc, cudaStream_t s) {
+  if (n == 0) return;
+  const uint64_t want = (n + 255) / 256;
+  const int grid = (int)std::min<uint64_t>(want, 148 * 8);
+  (void)cudaGetLastError();
+  k_materialise<<<grid, 256, 0, s>>>(shadow_units, n, rc);
 }
 
 // epoch origin moves (once per 2^32 - 16 launches): the current epoch becomes 1, every other 0

@@ -237,7 +237,7 @@ struct Context {
   uint32_t pd_minP = 0, pd_maxP = 0;
 
   // scratch
-  DevBuf slowmask, slowcnt;
+  DevBuf slowmask, slowcnt, dump_rc;
   DevBuf status, lc, hitmask, act_list, journal, free_list, copy_list, segs, seg0, staging, staging2, staging_cb, points, ptrs, temp;
   DevBuf up_units, up_vals, up_exts, uops;
   HostBuf h_small, h_status, h_list, h_pack[2];
@@ -549,6 +549,7 @@ struct Context {
   // merge pending declares/undeclares into the device table (A19: kernels only see a compacted table)
   int ensure_table() {
     if (!table_dirty) return CGCM_OK;
+    CKS(materialise_all());  // deferred references name units by their index in the table being replaced
     int n = (int)reg.size();
     // host staging: base[n], size[n], epoch0[n] (u32, relative), old_idx[n], flags[n]
     size_t need = (size_t)n * (8 + 8 + 4 + 4 + 4) + 256;
@@ -672,6 +673,7 @@ struct Context {
     int dir = DIR_FWD, ops = 0, sel = SEL_ALL;
     bool dec_red = false;  // OP_DEC through reductions + k_release_scan (large batches)
     bool no_journal = false;  // large gate passes snapshot the rc/epoch columns instead
+    bool defer = false;       // deferred references (cgcm_dev.h SlotArgs::defer)
     std::vector<Seg> segs;
     uint64_t nchunks = 0;
     Status res{};
@@ -742,6 +744,7 @@ struct Context {
     a.slowcount = slowcnt.as<unsigned long long>();
     a.dec_red = c.dec_red ? 1 : 0;
     a.no_journal = c.no_journal ? 1 : 0;
+    a.defer = c.defer ? 1 : 0;
     a.epoch = rel_epoch(epoch);
     a.st = status.as<Status>() + st_index;
     a.lc = lc.as<unsigned long long>();
@@ -1238,7 +1241,7 @@ struct Context {
   // On error everything this function did is undone; the caller undoes its own prologue.
   int map_core(const std::vector<Seg> &fsegs, const std::vector<Seg> &rsegs, uint64_t *translated_out,
                uint64_t *nulls_out, const std::vector<int> *seg_group = nullptr,
-               const std::vector<cudaEvent_t> *group_ev = nullptr) {
+               const std::vector<cudaEvent_t> *group_ev = nullptr, bool defer = false) {
     uint64_t total = 0;
     for (auto &s : fsegs) total += s.n;
     if (fsegs.empty() && rsegs.empty()) {  // nothing to translate (e.g. every outer was re-mapped, A9)
@@ -1251,6 +1254,7 @@ struct Context {
     F.dir = DIR_FWD;
     F.ops = OP_WRITE | OP_INC | OP_HITMASK;
     F.segs = fsegs;
+    F.defer = defer && fsegs.size() == 1 && fsegs[0].shadow != 0;
     if (seg_group && group_ev) {
       F.seg_group = *seg_group;
       F.group_ev = *group_ev;
@@ -1269,7 +1273,18 @@ struct Context {
     unsigned long long lcs[4];
     CKS(fetch_status(sts, lcs));
     bool strict = !(flags & CGCM_LENIENT);
+    // a failing call first turns the references it deferred into ordinary ones, which undo_map drops
+    auto undo_deferred = [&]() -> int {
+      if (F.defer) {
+        launch_materialise(reinterpret_cast<const uint32_t *>(fsegs[0].shadow + 8 * fsegs[0].n), fsegs[0].n,
+                           rcb.as<int32_t>(), main);
+        st.kernel_launches += 1;
+        CK(cudaGetLastError());
+      }
+      return CGCM_OK;
+    };
     if ((sts[0].misses || sts[1].misses) && strict) {
+      CKS(undo_deferred());
       CKS(undo_map(F, R));
       return CGCM_E_UNREGISTERED;
     }
@@ -1279,6 +1294,7 @@ struct Context {
       CKS(sorted_units(act_list, lcs[0], units));
       int r = activate_units(units, nullptr);
       if (r != CGCM_OK) {
+        CKS(undo_deferred());
         CKS(undo_map(F, R));
         return r;
       }
@@ -1368,7 +1384,7 @@ struct Context {
   // reverse unmap over device slot segments (GPU pointers): a3 + a4 (+ release)
   //   ops: OP_WRITE|OP_GATE|OP_HITMASK [|OP_DEC] or OP_GATE
   int unmap_rev_core(const std::vector<Seg> &segs, bool write, bool dec, std::vector<uint32_t> &copy_units,
-                     std::vector<uint32_t> &freed, uint64_t &journal_count, Status &res) {
+                     std::vector<uint32_t> &freed, uint64_t &journal_count, Status &res, bool defer = false) {
     CKS(ensure_rev());
     uint64_t total = 0;
     for (auto &s : segs) total += s.n;
@@ -1377,8 +1393,10 @@ struct Context {
     c.dir = DIR_REV;
     c.ops = write ? (OP_WRITE | OP_GATE | OP_HITMASK | (dec ? OP_DEC : 0)) : (OP_GATE | (dec ? OP_DEC : 0));
     c.segs = segs;
-    // large passes: snapshot the rc/epoch columns instead of journaling every gated unit
-    c.no_journal = total >= (uint64_t)U / 8 && U >= 4096;
+    c.defer = defer;
+    // large passes: snapshot the rc/epoch columns instead of journaling every gated unit; a pass over
+    // deferred references always does (its rollback is: restore the snapshot, then materialise)
+    c.no_journal = (total >= (uint64_t)U / 8 && U >= 4096) || defer;
     c.dec_red = dec && c.no_journal;
     if (c.no_journal) CKS(take_snapshot());
     CKS(launch(c, 0, false, false, true));
@@ -1415,7 +1433,34 @@ struct Context {
     DevBuf buf;
     uint64_t gen = 0;
     bool valid = false;
+    bool deferred = false;  // its unit words may carry deferred references (SH_DEFER)
   };
+  // Deferred references: the last cgcm_mapArrayDevice may have recorded references in
+  // its shadow instead of rc.  Every other call that reads or changes refcounts (or replaces the table)
+  // first adds them to rc -- only the matching cgcm_unmapArrayDevice(..., CGCM_RELEASE) drops them.
+  int materialise(std::pair<const std::pair<uint64_t, uint64_t>, Shadow> &kv) {
+    if (!kv.second.deferred) return CGCM_OK;
+    const uint64_t n = kv.first.second;
+    launch_materialise(reinterpret_cast<const uint32_t *>(kv.second.buf.addr + 8 * n), n, rcb.as<int32_t>(), main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
+    kv.second.deferred = false;
+    return CGCM_OK;
+  }
+  int materialise_all(const Shadow *except = nullptr) {
+    if (!any_deferred) return CGCM_OK;
+    bool left = false;
+    for (auto &kv : shadows) {
+      if (&kv.second == except) {
+        left = left || kv.second.deferred;
+        continue;
+      }
+      CKS(materialise(kv));
+    }
+    any_deferred = left;
+    return CGCM_OK;
+  }
+  bool any_deferred = false;
   std::map<std::pair<uint64_t, uint64_t>, Shadow> shadows;
   uint64_t table_gen = 0;
   // Record (CPU pointer, unit) per slot for the reverse passes (R13-ii) when a lookup costs more than
@@ -1456,6 +1501,7 @@ struct Context {
   // an outer's device copy is released: its shadows go with it
   void drop_shadows(uint64_t ptr) {
     for (auto it = shadows.lower_bound(std::make_pair(ptr, (uint64_t)0)); it != shadows.end() && it->first.first == ptr;) {
+      materialise(*it);
       dfree(it->second.buf);
       it = shadows.erase(it);
     }
@@ -1601,6 +1647,11 @@ using SlotCall = Context::SlotCall;
   RtScope rts_;                                   \
   std::lock_guard<std::recursive_mutex> lk_(C->mu); \
   if (cudaSetDevice(C->device) != cudaSuccess) return CGCM_E_CUDA;
+
+// every call that reads or changes refcounts first materialises deferred references
+#define CTXM() \
+  CTX();       \
+  CKS(C->materialise_all());
 
 // ============================== C ABI ==========================================================
 extern "C" {
@@ -1800,7 +1851,7 @@ int cgcm_declareGlobalSymbol(const char *name, void *base, size_t size, int isRe
   return s;
 }
 int cgcm_undeclare(void *base) {
-  CTX();
+  CTXM();
   uint64_t b = reinterpret_cast<uint64_t>(base);
   auto it = C->reg.find(b);
   if (it == C->reg.end()) return CGCM_E_UNREGISTERED;
@@ -1908,6 +1959,7 @@ void *cgcm_realloc(void *p, size_t n) {
   auto it = C->hsizes.find(a);
   if (it == C->hsizes.end()) return nullptr;
   auto ru = C->reg.find(a);
+  if (C->materialise_all() != CGCM_OK) return nullptr;
   if (ru != C->reg.end() && ru->second.idx >= 0) {  // a mapped AU cannot move (BUSY)
     int32_t rc = 0;
     if (cudaMemcpy(&rc, C->rcb.as<int32_t>() + ru->second.idx, 4, cudaMemcpyDeviceToHost) != cudaSuccess || rc > 0)
@@ -1939,7 +1991,7 @@ void *cgcm_declareAlloca(size_t n) {
   return p;
 }
 int cgcm_scopeExit(void) {
-  CTX();
+  CTXM();
   if (C->scopes.empty()) return CGCM_E_INVALID;
   auto &sc = C->scopes.back();
   // all-or-nothing: no registration expires while one of the scope's AUs is mapped
@@ -1959,14 +2011,21 @@ int cgcm_scopeExit(void) {
 // ---- device-resident arrays -------------------------------------------------------------------
 
 int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n) {
-  CTX();
+  CTXM();
   if (n == 0) return CGCM_OK;
   if (!d_slots || (reinterpret_cast<uint64_t>(d_slots) & 7)) return CGCM_E_INVALID;
   CKS(C->ensure_table());
   Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
   s.shadow = C->begin_shadow(s.ptr, n);
-  int r = C->map_core({s}, {}, nullptr, nullptr);
-  if (s.shadow) C->commit_shadow(s.ptr, n, r == CGCM_OK);
+  // with a shadow, references to units already active are deferred into it
+  int r = C->map_core({s}, {}, nullptr, nullptr, nullptr, nullptr, s.shadow != 0);
+  if (s.shadow) {
+    C->commit_shadow(s.ptr, n, r == CGCM_OK);
+    if (r == CGCM_OK) {
+      C->shadows[std::make_pair(s.ptr, (uint64_t)n)].deferred = true;
+      C->any_deferred = true;
+    }
+  }
   return r;
 }
 
@@ -1977,6 +2036,12 @@ int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
   Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
   auto shk = std::make_pair(s.ptr, (uint64_t)n);
   auto shi = C->shadows.find(shk);
+  bool rel = (flags & CGCM_RELEASE) != 0;
+  // the references the matching mapArrayDevice deferred are dropped by this pass when it releases
+  // them; in every other case they become ordinary references first (as all others do here)
+  const bool defer = rel && shi != C->shadows.end() && shi->second.valid && shi->second.deferred &&
+                     shi->second.gen == C->table_gen && !C->table_dirty;
+  CKS(C->materialise_all(defer ? &shi->second : nullptr));
   if (shi != C->shadows.end()) {
     CKS(C->ensure_table());
     if (shi->second.valid && shi->second.gen == C->table_gen) s.shadow = shi->second.buf.addr;
@@ -1985,8 +2050,9 @@ int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
   std::vector<uint32_t> copy_units, freed;
   uint64_t jcount = 0;
   Status res{};
-  bool rel = (flags & CGCM_RELEASE) != 0;
-  CKS(C->unmap_rev_core({s}, true, rel, copy_units, freed, jcount, res));
+  // (on failure the snapshot restores rc and the shadow keeps its deferred references: the next call
+  // materialises them)
+  CKS(C->unmap_rev_core({s}, true, rel, copy_units, freed, jcount, res, defer));
   int r = C->copy_back(copy_units);
   if (r != CGCM_OK) {
     // reverse translation of an array-mapped element failed: undo the whole call
@@ -2001,6 +2067,10 @@ int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
       C->undo_rev(c, jcount, {}, true, rel);
     }
     return r;
+  }
+  if (defer) {  // every deferred reference was dropped or materialised by the pass
+    shi->second.deferred = false;
+    C->any_deferred = false;
   }
   C->st.rev_translations += res.translated;
   if (C->flags & CGCM_LENIENT) C->st.passthrough += res.misses;
@@ -2020,7 +2090,7 @@ static int stage_in(Context *C, const void *const *cpu, size_t n, uint64_t &dptr
 }
 
 int cgcm_mapBatch(const void *const *cpu, size_t n, void **gpu_out) {
-  CTX();
+  CTXM();
   if (n == 0) return CGCM_OK;
   if (!cpu || !gpu_out) return CGCM_E_INVALID;
   CKS(C->ensure_table());
@@ -2035,7 +2105,7 @@ int cgcm_mapBatch(const void *const *cpu, size_t n, void **gpu_out) {
 }
 
 int cgcm_unmapBatch(const void *const *cpu, size_t n) {
-  CTX();
+  CTXM();
   if (n == 0) return CGCM_OK;
   if (!cpu) return CGCM_E_INVALID;
   CKS(C->ensure_table());
@@ -2065,7 +2135,7 @@ int cgcm_unmapBatch(const void *const *cpu, size_t n) {
 }
 
 int cgcm_releaseBatch(const void *const *cpu, size_t n) {
-  CTX();
+  CTXM();
   if (n == 0) return CGCM_OK;
   if (!cpu) return CGCM_E_INVALID;
   CKS(C->ensure_table());
@@ -2137,7 +2207,7 @@ int distinct_outers(const std::vector<PointInfo> &infos, std::vector<Outer> &out
 }  // namespace
 
 int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
-  CTX();
+  CTXM();
   if (k == 0) return CGCM_OK;
   if (!arrays || !gpu_out) return CGCM_E_INVALID;
   std::vector<PointInfo> infos;
@@ -2309,7 +2379,7 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
 }
 
 int cgcm_unmapArrays(void *const *const *arrays, size_t k) {
-  CTX();
+  CTXM();
   if (k == 0) return CGCM_OK;
   if (!arrays) return CGCM_E_INVALID;
   std::vector<PointInfo> infos;
@@ -2418,7 +2488,7 @@ int cgcm_unmapArrays(void *const *const *arrays, size_t k) {
 }
 
 int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
-  CTX();
+  CTXM();
   if (k == 0) return CGCM_OK;
   if (!arrays) return CGCM_E_INVALID;
   std::vector<PointInfo> infos;
@@ -2491,7 +2561,7 @@ int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
 
 // ---- map-promotion regions (NEXT-2) ----
 int cgcm_regionBegin(void *const *ptrs, const unsigned *kinds, size_t n, unsigned flags) {
-  CTX();
+  CTXM();
   if (C->region_open) return CGCM_E_BUSY;
   if (n && (!ptrs || !kinds)) return CGCM_E_INVALID;
   const bool check = (flags & CGCM_REGION_CHECK) != 0;
@@ -2596,7 +2666,7 @@ int cgcm_regionBegin(void *const *ptrs, const unsigned *kinds, size_t n, unsigne
   return CGCM_OK;
 }
 int cgcm_regionEnd(size_t *violations) {
-  CTX();
+  CTXM();
   if (!C->region_open) return CGCM_E_INVALID;
   unsigned long long v = 0;
   if (C->region_checked) {  // reopen every page before the copy-backs write host memory
@@ -2678,7 +2748,20 @@ int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
   std::vector<uint64_t> szs;
   CKS(C->download(hots, C->hotb, (size_t)C->U));
   CKS(C->download(sts, C->stb, (size_t)C->U));
-  CKS(C->download(rcs, C->rcb, (size_t)C->U));
+  if (C->any_deferred) {
+    // refcounts as the paper defines them (deferred references included), without changing any state:
+    // the deferred references are added to a copy of rc (observing must not change the execution path)
+    CKS(C->dalloc(C->dump_rc, 4 * (size_t)C->U + 64));
+    CK(cudaMemcpyAsync(C->dump_rc.as<void>(), C->rcb.as<void>(), 4 * (size_t)C->U, cudaMemcpyDeviceToDevice, C->main));
+    for (auto &kv : C->shadows)
+      if (kv.second.deferred)
+        launch_materialise(reinterpret_cast<const uint32_t *>(kv.second.buf.addr + 8 * kv.first.second), kv.first.second,
+                           C->dump_rc.as<int32_t>(), C->main);
+    CK(cudaGetLastError());
+    CKS(C->download(rcs, C->dump_rc, (size_t)C->U));
+  } else {
+    CKS(C->download(rcs, C->rcb, (size_t)C->U));
+  }
   CKS(C->download(szs, C->size64, (size_t)C->U));
   size_t m = std::min(cap, (size_t)C->U);
   for (size_t i = 0; i < m; ++i) {
