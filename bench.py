@@ -262,7 +262,7 @@ def run_cgcm(args, rank, world, local_rank):
         "setup_s": round(setup_s, 1), "setup_activation_s": round(setup_act_s, 1),
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        result["cpu_baseline"] = cpu_baseline(wl, args.cpu_sample, steps=1)
+        result["cpu_baseline"] = cpu_baseline(wl, args.cpu_sample, steps=3)
     return result
 
 
@@ -565,19 +565,85 @@ def oracle_step(o, slots):
     return time.perf_counter() - t0, s
 
 
+def host_info():
+    """The GPU box's host CPU (record nproc and the CPU model)."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    model = ln.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "affinity": len(os.sched_getaffinity(0)), "cpu_model": model}
+
+
 def cpu_baseline(wl, sample, steps=1, o=None):
+    """The CPU oracle timed on one core (pinned with sched_setaffinity, the taskset -c of SURVEY §8(d)),
+    best of `steps` (one step when a step exceeds 10 s), on the first `sample` slots of the workload;
+    plus the timing-only all-cores std::upper_bound baseline (tools/cpu_baseline.cpp) on 1/16 of it."""
+    allowed = os.sched_getaffinity(0)
+    core = min(allowed)
     o = o or oracle_setup(wl)
     slots = wl.host_sample(sample)
     best = None
-    for _ in range(steps):
-        dt, s = oracle_step(o, slots)
-        assert (s == slots).all()
-        best = dt if best is None else min(best, dt)
+    os.sched_setaffinity(0, {core})
+    try:
+        for k in range(steps):
+            dt, s = oracle_step(o, slots)
+            assert (s == slots).all()
+            best = dt if best is None else min(best, dt)
+            if dt > 10:
+                break
+    finally:
+        os.sched_setaffinity(0, allowed)
     o.close()
-    return {"value": round(2 * sample / best, 1), "unit": "pointer translations/s", "cores": 1, "kind": "oracle",
-            "sample": f"first {sample} slots of rank 0's arrays (same table, same setup references): "
-                      f"mapSlots + advanceEpoch + unmapSlots(release), single-threaded C++ std::map oracle",
-            "seconds": round(best, 3)}
+    res = {"value": round(2 * sample / best, 1), "unit": "pointer translations/s", "cores": 1, "kind": "oracle",
+           "sample": f"first {sample} slots of rank 0's arrays (same table, same setup references): "
+                     f"mapSlots + advanceEpoch + unmapSlots(release), single-threaded C++ std::map oracle pinned "
+                     f"to core {core}, best of up to {steps}",
+           "seconds": round(best, 3), "host": host_info()}
+    try:
+        res["all_cores"] = cpu_all_cores(wl, min(wl.n, 1 << 24))
+    except Exception as ex:  # timing-only extra: never fails the bench
+        res["all_cores"] = {"error": str(ex)[:200]}
+    return res
+
+
+def cpu_all_cores(wl, n, reps=3):
+    """tools/cpu_baseline.cpp: the step as a straightforward OpenMP program over all host cores (sorted
+    table + std::upper_bound, atomic refcounts, epoch gate), timing only, best of reps."""
+    import ctypes
+    lib = build_cpu_baseline()
+    L = ctypes.CDLL(lib)
+    L.cpu_baseline_step.restype = ctypes.c_double
+    L.cpu_baseline_step.argtypes = [ctypes.c_void_p] * 3 + [ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64,
+                                                            ctypes.c_int, ctypes.c_int, ctypes.c_void_p]
+    L.cpu_baseline_threads.restype = ctypes.c_int
+    threads = len(os.sched_getaffinity(0))
+    base = np.ascontiguousarray(wl.bases, dtype=np.uint64)
+    size = np.ascontiguousarray(wl.sizes, dtype=np.uint64)
+    dev = (base - np.uint64(1 << 40)).astype(np.uint64)          # a mirrored device layout
+    slots = wl.host_sample(n)
+    ref = slots.copy()
+    tr = ctypes.c_uint64(0)
+    sec = L.cpu_baseline_step(base.ctypes.data, size.ctypes.data, dev.ctypes.data, len(base), slots.ctypes.data,
+                              n, threads, reps, ctypes.byref(tr))
+    if sec <= 0 or not (slots == ref).all():
+        raise RuntimeError("cpu baseline step failed")
+    return {"value": round(tr.value / sec, 1), "unit": "pointer translations/s", "cores": threads,
+            "kind": "all-cores std::upper_bound (tools/cpu_baseline.cpp, timing only)",
+            "sample": f"first {n} slots of rank 0's arrays (1/{max(1, wl.n // n)} of the rank's batch), best of {reps}",
+            "seconds": round(sec, 3)}
+
+
+def build_cpu_baseline():
+    src = os.path.join(ROOT, "tools", "cpu_baseline.cpp")
+    lib = os.path.join(ROOT, "tools", "libcpu_baseline.so")
+    if not os.path.exists(lib) or os.path.getmtime(lib) < os.path.getmtime(src):
+        subprocess.check_call(["g++", "-O3", "-std=c++17", "-fopenmp", "-shared", "-fPIC", "-o", lib, src])
+    return lib
 
 
 def run_reference(args, rank, world):
@@ -616,6 +682,92 @@ def max_over_ranks(x, dev):
     return float(t.item())
 
 
+def run_config_line(args):
+    """bench.py --config A|B|D: the secondary configs as one contract-shaped JSON line each,
+    with the CPU oracle timed beside them (tools/bench_configs.py holds both sides)."""
+    import importlib.util
+    import torch
+    spec = importlib.util.spec_from_file_location("bench_configs", os.path.join(ROOT, "tools", "bench_configs.py"))
+    bc = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(bc)
+    torch.cuda.set_device(0)
+    link = host_link(torch.device("cuda", 0))
+    sampler = start_clock_sampler(None)
+    common = {"n_gpus": 1, "warmup": args.warmup, "scaling": "strong", "vs_baseline": None, "dtype": "u64+f64",
+              "data": "synthetic (seeded splitmix64 values; pinned cgcm_malloc heap)"}
+    if args.config == "A":
+        for _ in range(args.warmup):
+            bc.config_A("promoted", iters=3)  # lazy module loading, clocks
+        modes = {m: bc.config_A(m) for m in ("naive", "promoted", "region", "region_check")}
+        clocks = stop_clock_sampler(sampler)
+        pro, nai = modes["promoted"], modes["naive"]
+        orc = {m: bc.oracle_A(m) for m in ("naive", "promoted")}
+        it = pro["iterations"]
+        res = {"metric": "config A (jagged 256x256 fp64, 100 iterations of mapArray/S1/unmapArray/releaseArray): "
+                         "us per iteration, map-promoted loop", "value": pro["us_per_iteration"],
+               "unit": "us/iteration", "higher_is_better": False, "steps": it,
+               "ms_per_step": round(pro["us_per_iteration"] / 1e3, 4), **common,
+               "config": {"workload": "A: 256 row AUs of 2 KiB + the row-pointer AU (BASELINE configs[0])",
+                          "mode": "promoted (Listing 4)"},
+               "modes": modes, "speedup_promoted_vs_naive": round(nai["us_per_iteration"] / pro["us_per_iteration"], 2),
+               "e2e": {"value": pro["us_per_iteration"], "unit": "us/iteration",
+                       "h2d_bytes_per_step": pro["h2d_bytes"] // it, "d2h_bytes_per_step": pro["d2h_bytes"] // it,
+                       "naive_us_per_iteration": nai["us_per_iteration"],
+                       "naive_h2d_bytes_per_step": nai["h2d_bytes"] // it, "naive_d2h_bytes_per_step": nai["d2h_bytes"] // it},
+               "roofline": {"bound": "latency", "achieved": None, "peak": None, "unit": "us/call", "frac": None,
+                            "traffic": None, "note": "512 KiB per naive iteration: call latency, not bandwidth, binds"},
+               "gpu_launches": pro["kernel_launches"], "clocks": clocks, "host_link": link,
+               "cpu_baseline": {"value": orc["promoted"]["us_per_iteration"], "unit": "us/iteration", "cores": 1,
+                                "kind": "oracle", "sample": "the whole config (100 iterations), simulated memories",
+                                "naive_us_per_iteration": orc["naive"]["us_per_iteration"], "host": host_info()}}
+    elif args.config == "B":
+        bc.config_B(True, n=256)  # warm-up
+        modes = {"promoted": bc.config_B(True), "naive": bc.config_B(False)}
+        clocks = stop_clock_sampler(sampler)
+        pro, nai = modes["promoted"], modes["naive"]
+        orc = {"promoted": bc.oracle_B(True), "naive": bc.oracle_B(False)}
+        res = {"metric": "config B (PolyBench-shaped gemm on jagged 4096^2 fp64, 64 row-blocks): seconds for the "
+                         "whole loop, map-promoted", "value": pro["seconds"], "unit": "s", "higher_is_better": False,
+               "steps": 64, "ms_per_step": round(1e3 * pro["seconds"] / 64, 3), **common,
+               "config": {"workload": "B: 3 x 4096 row AUs of 32 KiB + 3 row-pointer AUs (BASELINE configs[1])",
+                          "mode": "promoted"},
+               "modes": modes, "speedup_promoted_vs_naive": round(nai["seconds"] / pro["seconds"], 2),
+               "e2e": {"value": pro["seconds"], "unit": "s", "h2d_bytes_per_step": pro["h2d_bytes"] // 64,
+                       "d2h_bytes_per_step": pro["d2h_bytes"] // 64, "naive_seconds": nai["seconds"]},
+               "roofline": {"bound": "host_link", "achieved": round((nai["h2d_bytes"] + nai["d2h_bytes"]) / nai["seconds"] / 1e9, 2),
+                            "peak": link["h2d_gbs"], "unit": "GB/s",
+                            "frac": round((nai["h2d_bytes"] + nai["d2h_bytes"]) / nai["seconds"] / 1e9 / link["h2d_gbs"], 4),
+                            "traffic": None, "note": "naive loop: copy bytes over its wall time vs one-way link"},
+               "gpu_launches": pro["kernel_launches"], "clocks": clocks, "host_link": link,
+               "cpu_baseline": {"value": orc["promoted"]["seconds"], "unit": "s", "cores": 1, "kind": "oracle",
+                                "sample": orc["promoted"]["sample"], "naive_seconds": orc["naive"]["seconds"],
+                                "host": host_info()}}
+    elif args.config == "D":
+        bc.config_D(N=1 << 16)  # warm-up
+        d = bc.config_D()
+        clocks = stop_clock_sampler(sampler)
+        orc = bc.oracle_D(1 << 20)
+        b = 48 * d["nodes"]
+        gbs = 2 * b / (d["map_seconds"] + d["unmap_seconds"]) / 1e9
+        res = {"metric": "config D (2^24-node pointer tree): map+unmap GB/s over the host link",
+               "value": round(gbs, 2), "unit": "GB/s", "higher_is_better": True, "steps": 1,
+               "ms_per_step": round(1e3 * (d["map_seconds"] + d["unmap_seconds"]), 2), **common,
+               "config": {"workload": "D: 2^24 node AUs of 32 B + child table of 2^25 slots (BASELINE configs[3])"},
+               "detail": d,
+               "e2e": {"value": round(gbs, 2), "unit": "GB/s", "h2d_bytes_per_step": d["h2d_bytes"],
+                       "d2h_bytes_per_step": d["d2h_bytes"]},
+               "roofline": {"bound": "host_link", "achieved": round(gbs, 2), "peak": link["h2d_gbs"], "unit": "GB/s",
+                            "frac": round(gbs / link["h2d_gbs"], 4), "traffic": None},
+               "gpu_launches": d["kernel_launches"], "clocks": clocks, "host_link": link,
+               "cpu_baseline": {"value": round(2 * 48 * orc["nodes"] / (orc["map_seconds"] + orc["unmap_seconds"]) / 1e9, 4),
+                                "unit": "GB/s", "cores": 1, "kind": "oracle",
+                                "sample": f"{orc['nodes']} nodes (1/16 of 2^24), simulated memories", "detail": orc,
+                                "host": host_info()}}
+    else:
+        raise SystemExit(f"unknown config {args.config}")
+    print(json.dumps(res), flush=True)
+
+
 def relaunch_under_torchrun(args):
     """`python bench.py --gpus N` without a launcher: re-execute under torch.distributed.run with one
     rank per GPU (rendezvous on 127.0.0.1), so that --gpus is never silently ignored."""
@@ -635,7 +787,7 @@ def main():
     ap.add_argument("--steps", type=int, default=30)  # ~200 ms timed at E: several clock samples
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="cgcm", choices=["cgcm", "reference"])
-    ap.add_argument("--config", default="E", choices=sorted(CONFIGS))
+    ap.add_argument("--config", default="E", choices=sorted(CONFIGS) + ["A", "B", "D"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-duplex", action="store_true", help="e2e through one context only")
     ap.add_argument("--e2e-steps", type=int, default=6)
@@ -657,6 +809,13 @@ def main():
             sys.exit(f"bench.py: {world} ranks need {world} GPUs, this node has {torch.cuda.device_count()}")
         if args.allow_shared_gpu:
             local_rank = local_rank % max(1, torch.cuda.device_count())
+    if args.config in ("A", "B", "D"):
+        if args.impl == "reference":
+            print(json.dumps({"impl": "reference", "unavailable": "configs A/B/D: the oracle runs beside the GPU "
+                              "in the same line (cpu_baseline)"}))
+            return
+        run_config_line(args)
+        return
     if args.impl == "reference":
         res = run_reference(args, rank, world)
         if res is not None:

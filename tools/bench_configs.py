@@ -77,7 +77,7 @@ def config_A(mode, iters=100):
             "us_per_call": {k: round(1e6 * v / iters, 1) for k, v in calls.items()},
             "h2d_units": s["h2d_units"], "h2d_bytes": s["h2d_bytes"], "d2h_units": s["d2h_units"],
             "d2h_bytes": s["d2h_bytes"], "h2d_memcpy_calls": s["h2d_memcpy_calls"],
-            "d2h_memcpy_calls": s["d2h_memcpy_calls"]}
+            "d2h_memcpy_calls": s["d2h_memcpy_calls"], "kernel_launches": s["kernel_launches"]}
 
 
 def config_B(promoted, n=4096, blk=64):
@@ -121,7 +121,7 @@ def config_B(promoted, n=4096, blk=64):
             "h2d_units": s["h2d_units"], "h2d_bytes": s["h2d_bytes"], "d2h_units": s["d2h_units"],
             "d2h_bytes": s["d2h_bytes"], "copy_GBs_over_wall": round(moved / t / 1e9, 2),
             "h2d_memcpy_calls": s["h2d_memcpy_calls"], "d2h_memcpy_calls": s["d2h_memcpy_calls"],
-            "gemm_flops": 2 * n ** 3}
+            "gemm_flops": 2 * n ** 3, "kernel_launches": s["kernel_launches"]}
 
 
 def config_D(N=1 << 24):
@@ -155,12 +155,144 @@ def config_D(N=1 << 24):
     tu = timed(lambda: (ctx.unmapArray(CB), ctx.unmap(root)))
     ctx.releaseArray(CB)
     ctx.release(root)
+    s = ctx.stats()
     ctx.close()
     b = 48 * N
     return {"config": "D", "nodes": N, "declare_seconds": round(td, 4), "table_build_seconds": round(tb, 4),
             "map_seconds": round(tm, 4), "unmap_seconds": round(tu, 4),
             "map_GBs": round(b / tm / 1e9, 2), "unmap_GBs": round(b / tu / 1e9, 2),
-            "map_translations_per_s": round(N / tm, 1), "unmap_translations_per_s": round((N - 1) / tu, 1)}
+            "map_translations_per_s": round(N / tm, 1), "unmap_translations_per_s": round((N - 1) / tu, 1),
+            "h2d_bytes": s["h2d_bytes"], "d2h_bytes": s["d2h_bytes"], "kernel_launches": s["kernel_launches"],
+            "h2d_memcpy_calls": s["h2d_memcpy_calls"], "d2h_memcpy_calls": s["d2h_memcpy_calls"]}
+
+
+# ---------------------------------------------------------------------------------------------
+# The CPU oracle on the same configs (bench.py --config A|B|D cpu_baseline: "the oracle as it stands",
+# one core).  Host and device memory are the oracle's simulated memories; the addresses are synthetic.
+# ---------------------------------------------------------------------------------------------
+def _oracle():
+    sys.path.insert(0, ROOT)
+    from oracle import Oracle
+    return Oracle()
+
+
+def _oracle_jagged(o, nrows, ncols, vals, base):
+    """nrows row AUs of 8*ncols bytes, host-adjacent (as cgcm_malloc lays them out), + the row-pointer AU."""
+    rows = [base + 8 * ncols * r for r in range(nrows)]
+    for r, a in enumerate(rows):
+        assert o.declareAlloc(a, 8 * ncols) == 0
+        o.host_write(a, np.ascontiguousarray(vals[r], dtype=np.float64))
+    pp = base + 8 * ncols * nrows
+    assert o.declareAlloc(pp, 8 * nrows) == 0
+    o.host_write(pp, np.asarray(rows, dtype=np.uint64))
+    return rows, pp
+
+
+def oracle_A(mode, iters=100):
+    o = _oracle()
+    nrows = ncols = 256
+    _rows, pp = _oracle_jagged(o, nrows, ncols, W.config_A_values(nrows, ncols, 1), 0x10000000)
+    t0 = time.perf_counter()
+    if mode == "promoted":
+        assert o.mapArray(pp)[0] == 0
+    for _ in range(iters):
+        st, d = o.mapArray(pp)
+        assert st == 0
+        o.kernel_scale(d, nrows, ncols, 0.999)
+        o.advanceEpoch()
+        if mode == "naive":
+            assert o.unmapArray(pp) == 0
+        assert o.releaseArray(pp) == 0
+    if mode == "promoted":
+        assert o.unmapArray(pp) == 0 and o.releaseArray(pp) == 0
+    t = time.perf_counter() - t0
+    s = o.stats()
+    o.close()
+    return {"mode": mode, "us_per_iteration": round(1e6 * t / iters, 1), "iterations": iters,
+            "h2d_units": s["h2d_units"], "d2h_units": s["d2h_units"]}
+
+
+def oracle_B(promoted, n=4096, blk=64, gemm_rows=1):
+    """One row-block of the loop (the maps / unmaps / releases of a block, the gemm of `gemm_rows` of its
+    rows) timed on the oracle and scaled to the whole loop: blocks x (calls + blk/gemm_rows x gemm)."""
+    o = _oracle()
+    mats = []
+    for m in range(3):
+        _r, pp = _oracle_jagged(o, n, n, W.config_B_values(n, 2, m), 0x100000000 * (m + 1))
+        mats.append(pp)
+    C = mats[2]
+    t_pro = 0.0
+    if promoted:
+        t0 = time.perf_counter()
+        for pp in mats:
+            assert o.mapArray(pp)[0] == 0
+        t_pro = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    d = [o.mapArray(pp)[1] for pp in mats]
+    t_map = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    o.kernel_gemm_rows(d[0], d[1], d[2], n, 0, gemm_rows, 1.5, 1.2)
+    t_gemm = time.perf_counter() - t0
+    o.advanceEpoch()
+    t0 = time.perf_counter()
+    if not promoted:
+        assert o.unmapArray(C) == 0
+    for pp in mats:
+        assert o.releaseArray(pp) == 0
+    t_unmap = time.perf_counter() - t0
+    t_epi = 0.0
+    if promoted:
+        t0 = time.perf_counter()
+        assert o.unmapArray(C) == 0
+        for pp in mats:
+            assert o.releaseArray(pp) == 0
+        t_epi = time.perf_counter() - t0
+    o.close()
+    blocks = n // blk
+    total = t_pro + t_epi + blocks * (t_map + t_unmap + t_gemm * blk / gemm_rows)
+    return {"mode": "promoted" if promoted else "naive", "seconds": round(total, 1),
+            "sample": f"block 0 timed (its maps/unmaps/releases + the gemm of {gemm_rows} of its {blk} rows), "
+                      f"scaled x{blocks} blocks x{blk // gemm_rows} rows",
+            "per_block_calls_s": round(t_map + t_unmap, 3), "gemm_row_s": round(t_gemm / gemm_rows, 3)}
+
+
+def oracle_D(N=1 << 20):
+    """Config D's map + levels + unmap on the oracle at N nodes (a 1/16 subset of 2^24 when N = 2^20)."""
+    o = _oracle()
+    vals = W.tree_values(N)
+    order = W.tree_alloc_order(N)
+    pos = np.empty(N, dtype=np.int64)
+    pos[order] = np.arange(N)
+    nodes = 0x10000000
+    addr = np.uint64(nodes) + np.uint64(32) * pos.astype(np.uint64)
+    for k in range(N):
+        assert o.declareAlloc(nodes + 32 * k, 32) == 0
+    img = np.zeros((N, 4))
+    img[:, 1] = vals[order]
+    img.view(np.int64)[:, 0] = order
+    o.host_write(nodes, img)
+    child = W.tree_children(N)
+    CB = 0x800000000
+    assert o.declareAlloc(CB, 16 * N) == 0
+    o.host_write(CB, np.where(child >= 0, addr[np.maximum(child, 0)], 0).astype(np.uint64))
+    t0 = time.perf_counter()
+    st, cdev = o.mapArray(CB)
+    st2, rdev = o.map(int(addr[0]))
+    tm = time.perf_counter() - t0
+    assert st == 0 and st2 == 0
+    t0 = time.perf_counter()
+    for dlev in range(int(math.log2(N)), -1, -1):
+        lo, hi = (1 << dlev) - 1, min((1 << (dlev + 1)) - 1, N)
+        o.kernel_treesum_level(cdev, rdev, N, lo, hi)
+        o.advanceEpoch()
+    tk = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    assert o.unmapArray(CB) == 0 and o.unmap(int(addr[0])) == 0
+    tu = time.perf_counter() - t0
+    o.close()
+    b = 48 * N
+    return {"nodes": N, "map_seconds": round(tm, 3), "levels_seconds": round(tk, 3), "unmap_seconds": round(tu, 3),
+            "map_GBs": round(b / tm / 1e9, 4), "unmap_GBs": round(b / tu / 1e9, 4)}
 
 
 if __name__ == "__main__":
