@@ -111,19 +111,23 @@ struct IndexDev {
 //   w[0]     j0 = greatestLTE(A), the unit with the greatest base <= A (0xFFFFFFFF: none)
 //   w[1]     cnt (bits 0..13): units with base in (A, A + 2^P) | bit 14: base(j0) == A
 //            | end0 (bits 15..31): min(base(j0) + size(j0) - A + 1, 0x1FFFF), 0 if j0 ends before A
-//   w[2..7]  cnt <= PD_K: the offsets base - A of those units, sorted u16, padded with 0xFFFF;
+//   w[2..7]  cnt <= PD_K: the offsets base - A of those units, sorted u16, padded with PD_PAD;
 //            cnt >  PD_K: w[2] = index of the first of cnt sorted u16 offsets in ovf[] (16-aligned,
-//            padded with 0xFFFF to a whole 32-byte sector)
+//            padded with PD_PAD to a whole 32-byte sector)
 // greatestLTE(p) = j0 + #{offsets <= p - A}; p hits unit j0 iff p - A < end0 (A7: p - base <= size),
 // any other candidate by its base A + offset and its size (hot word).  One sector gather per lookup.
+// Pages are at most 32 KiB (P <= 15): offsets and the padding PD_PAD = 0x7FFF fit 15 bits, so four of
+// them compare against p - A in one 64-bit subtraction with a guard bit per lane (k_fwd_lean); no
+// start sits at offset PD_PAD (build_pd takes a smaller page), and lookups clamp p - A to PD_PAD - 1.
 constexpr int PD_MAXSEG = 64;
 constexpr int PD_K = 12;
 #ifdef CGCM_PD_MAXSHIFT
 constexpr int PD_MAXSHIFT = CGCM_PD_MAXSHIFT;
 #else
-constexpr int PD_MAXSHIFT = 16;  // 64 KiB pages: u16 offsets; a page holding a start at offset 0xFFFF
-                                 // (the padding value) or more than PD_CNT_MAX starts takes a smaller P
+constexpr int PD_MAXSHIFT = 15;  // 32 KiB pages (64 KiB measured no faster at E, profiles/r01j_ab_pd64.log)
 #endif
+static_assert(PD_MAXSHIFT <= 15, "page offsets must fit 15 bits");
+constexpr uint32_t PD_PAD = 0x7FFFu;
 constexpr uint32_t PD_CNT_MAX = 0x3FFFu;
 constexpr uint32_t PD_EXACT = 1u << 14;
 constexpr int PD_END_SHIFT = 15;

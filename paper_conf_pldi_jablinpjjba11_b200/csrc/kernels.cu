@@ -390,9 +390,9 @@ __device__ __forceinline__ void pd_back(const PdDev &pd, uint64_t pol, const PdF
   }
   const uint32_t j0 = (uint32_t)w_in[0], w1 = (uint32_t)(w_in[0] >> 32);
   const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
-  // padding is 0xFFFF and no start sits at offset 0xFFFF (build_pd): counting with min(poff, 0xFFFE)
+  // padding is PD_PAD and no start sits at offset PD_PAD (build_pd): counting with min(poff, PD_PAD - 1)
   // never counts padding and counts the same starts
-  const uint32_t rr = min(f.poff, 0xFFFEu) * 0x10001u;
+  const uint32_t rr = min(f.poff, PD_PAD - 1u) * 0x10001u;
   uint32_t c = 0, mx = 0;
   if (cnt <= (uint32_t)PD_K) {
 #pragma unroll
@@ -467,7 +467,7 @@ __device__ __forceinline__ void pd_lookup2(const SPd &S, const PdDev &pd, uint64
   for (int m = 0; m < 2; ++m) {
     const uint32_t j0 = (uint32_t)w[m][0], w1 = (uint32_t)(w[m][0] >> 32);
     const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
-    const uint32_t rr = min(poff[m], 0xFFFEu) * 0x10001u;  // see pd_back
+    const uint32_t rr = min(poff[m], PD_PAD - 1u) * 0x10001u;  // see pd_back
     uint32_t c = 0, mx = 0;
     if (cnt <= (uint32_t)PD_K) {
 #pragma unroll
@@ -1346,6 +1346,416 @@ static int launch_unmap_sh(const SlotArgs &a, int nsm, cudaStream_t s) {
   return a.nseg > 1 ? launch_unmap_sh1<OPS, true>(a, nsm, s) : launch_unmap_sh1<OPS, false>(a, nsm, s);
 }
 
+// -------------------------------------------------------------------------------------------------
+// k_fwd_lean: the forward map of cgcm_mapArrayDevice (a1 + a2 of Alg. 1) over ONE in-place segment with
+// a shadow, through a page directory of ONE address segment (the case of every config-C/E-shaped
+// table).  Same results, counters and lists as k_map_pd<1>; the instruction count per slot is what
+// bounds k_map_pd (profiles/r02c_E_summary.md: 327 thread instructions per slot at 63 % issue), so:
+//   * the page entry's twelve 15-bit offsets are compared with p - A four at a time, one 64-bit
+//     subtraction per four with a guard bit per lane (le4), instead of twelve emulated SIMD compares;
+//   * the segment is in registers (no shared-memory segment search), the page is one shift;
+//   * activations (units not yet active), crowded pages, escaped unit words and huge units are the
+//     rare paths; the hit mask is built with warp reductions; whole chunks are stored unconditionally
+//     (an untranslated slot is written back unchanged; ragged segment ends slot by slot).
+// -------------------------------------------------------------------------------------------------
+constexpr int FWD_LEAN_THREADS = 768;
+
+__device__ __forceinline__ uint32_t warp_or(uint32_t v) { return __reduce_or_sync(0xffffffffu, v); }
+
+// #{o <= r} among the four sorted 15-bit offsets packed in q (16-bit lanes): per lane
+// 0x8000 + r - o keeps bit 15 iff o <= r, and never borrows from the next lane (r, o < 0x8000)
+__device__ __forceinline__ uint32_t le4(uint64_t q, uint64_t r4) {
+  return __popcll(((r4 | 0x8000800080008000ull) - q) & 0x8000800080008000ull);
+}
+__device__ __forceinline__ uint32_t off_at(uint64_t q1, uint64_t q2, uint64_t q3, uint32_t i) {  // offset i < 12
+  const uint64_t q = i < 4 ? q1 : (i < 8 ? q2 : q3);
+  return (uint32_t)(q >> (16 * (i & 3))) & 0xFFFFu;
+}
+// crowded page (more than PD_K starts): count in the side array, one sector per 16 offsets
+__device__ __noinline__ void pd_crowded(const uint16_t *ovf, uint32_t first, uint32_t cnt, uint32_t r, uint32_t &k,
+                                        uint32_t &off) {
+  const uint64_t r4 = (uint64_t)r * 0x0001000100010001ull;
+  k = 0;
+  off = 0;
+  for (uint32_t t = 0; t < cnt; t += 16) {
+    uint64_t v[4];
+    asm volatile("ld.global.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(v[0]), "=l"(v[1]), "=l"(v[2]), "=l"(v[3]) : "l"(ovf + first + t));
+    uint32_t c = 0;
+#pragma unroll
+    for (int z = 0; z < 4; ++z) c += le4(v[z], r4);
+    if (c) {
+      const uint32_t i = c - 1;
+      off = (uint32_t)(v[i >> 2] >> (16 * (i & 3))) & 0xFFFFu;
+    }
+    k += c;
+    if (c < 16) break;  // later sectors hold larger offsets only
+  }
+}
+
+template <bool ES>  // ES: the extent deltas are staged in shared memory
+__global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
+  if (ES)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
+  __syncthreads();
+  const uint64_t pol_s = policy_evict_first();
+  const uint64_t pol_t = policy_evict_last();
+  const int lane = threadIdx.x & 31;
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n;
+  uint64_t *shp = reinterpret_cast<uint64_t *>(sg.shadow);
+  uint32_t *shu = reinterpret_cast<uint32_t *>(sg.shadow + 8 * sg.n);
+  // the directory's one segment: first base, end of its last unit, first entry, pages, page shift, last unit
+  const uint64_t S0 = a.pd.seg_start[0], Send = a.pd.seg_start[1];
+  const uint32_t P = a.pd.seg_meta[2], npages = a.pd.seg_meta[1], lastu = a.pd.seg_meta[3];
+  const uint32_t *ent = a.pd.ent + 8ull * a.pd.seg_meta[0];
+  const uint32_t pmask = (1u << P) - 1u;
+  const int32_t inc = sg.inc;
+  const bool defer = a.defer != 0;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned c_nulls = 0, c_hits = 0, c_miss = 0, c_pend = 0, c_tr = 0;
+
+  const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  uint64_t cv[2] = {0, 0}, nv[2] = {0, 0}, nnv[2] = {0, 0};
+  if (c_first < a.nchunks) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c_first), pol_s, cv[0], cv[1]);
+  if (c_first + stride < a.nchunks)
+    ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, nv[0], nv[1]);
+  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
+    const uint64_t c = cb + lane;
+    if (c + 2 * stride < a.nchunks)  // pipeline: the slot values of chunk t+2
+      ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, nnv[0], nnv[1]);
+    const uint64_t a0 = a0base + 16ull * c;
+    const uint32_t valid = c < a.nchunks ? ((a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u)) : 0u;
+
+    // a1: the page entry of each slot (both gathers in flight before either is decoded)
+    uint64_t ew[2][4];
+    uint32_t poff[2];
+    int j[2];
+    bool ok[2];
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const uint64_t p = cv[m];
+      const bool look = ((valid >> m) & 1) && p != 0 && p >= S0;
+      const uint64_t rel = p - S0;
+      const uint64_t pg = rel >> P;
+      ok[m] = look && pg < npages;
+      poff[m] = (uint32_t)rel & pmask;
+      // beyond the last page: the tail of the segment's last unit (decided by its end, A7), or a miss
+      j[m] = look && !ok[m] && p <= Send ? (int)lastu : -1;
+      ew[m][0] = ew[m][1] = ew[m][2] = ew[m][3] = 0;
+      if (ok[m])
+        asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+                     : "=l"(ew[m][0]), "=l"(ew[m][1]), "=l"(ew[m][2]), "=l"(ew[m][3])
+                     : "l"(ent + 8 * pg), "l"(pol_t));
+    }
+    // decode: j = j0 + #{offsets <= p - A}; the page's j0 is decided by its end, others by base + size
+    bool k0[2];
+    uint64_t key[2];
+    uint32_t cw[2];
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      k0[m] = true;
+      key[m] = 0;
+      if (ok[m]) {
+        const uint32_t j0 = (uint32_t)ew[m][0], w1 = (uint32_t)(ew[m][0] >> 32);
+        const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
+        const uint32_t r = min(poff[m], PD_PAD - 1u);
+        uint32_t k, off;
+        if (cnt <= (uint32_t)PD_K) {
+          const uint64_t r4 = (uint64_t)r * 0x0001000100010001ull;
+          k = le4(ew[m][1], r4) + le4(ew[m][2], r4) + le4(ew[m][3], r4);
+          off = k ? off_at(ew[m][1], ew[m][2], ew[m][3], k - 1) : 0u;
+        } else {
+          pd_crowded(a.pd.ovf, (uint32_t)ew[m][1], cnt, r, k, off);
+        }
+        k0[m] = k == 0;
+        j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && poff[m] < end0 ? (int)j0 : -1);
+        key[m] = cv[m] - poff[m] + off;  // the candidate's base (A + offset)
+      }
+      cw[m] = 0;
+      if (j[m] >= 0)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
+        asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
+    }
+    uint64_t outv[2] = {cv[0], cv[1]};
+    uint32_t wrote = 0, su[2];
+    bool act[2];
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const bool vm = (valid >> m) & 1;
+      const bool look = j[m] >= 0;
+      const uint64_t hw = (cw[m] & HOTC_ESC) && look ? ld_u64_hot(a.tab.hot + j[m], pol_t) : hot_of_hotc(cw[m]);
+      uint64_t sz = hot_size32(hw);
+      if (look && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
+      const bool hit = look && (k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
+      const bool nul = vm && cv[m] == 0;
+      c_nulls += nul;
+      c_hits += hit;
+      c_miss += vm && !nul && !hit;
+      const uint32_t fl = hot_flags(hw);
+      const bool active = (fl & UF_ACTIVE) != 0;
+      // deferred reference (a.defer): the unit was active when the call began -- recorded in the shadow
+      const bool dfr = defer && hit && active;
+      act[m] = false;
+      if (hit && !dfr) {
+        int32_t *RC = a.tab.rc + j[m];
+        if (active) red_add(RC, inc);
+        else act[m] = atomicAdd(RC, inc) == 0;  // refcount 0 -> 1: Alg. 1's activation
+      }
+      if (hit && (fl & UF_STORAGE)) {
+        const uint32_t e = hot_ext(hw);
+        outv[m] = cv[m] + (ES ? s_ext[e] : a.tab.ext_delta[e]);  // Alg. 1: devptr + (ptr - base)
+        wrote |= 1u << m;
+      } else {
+        c_pend += hit;  // activated by this call: completed after the allocation
+      }
+      su[m] = hit ? ((uint32_t)j[m] | (dfr ? SH_DEFER : 0u)) : SH_NONE;
+    }
+    c_tr += __popc(wrote);
+    if (__any_sync(0xffffffffu, act[0] || act[1])) {
+#pragma unroll
+      for (int m = 0; m < 2; ++m) {
+        const unsigned long long ix = warp_append(&a.lc[0], act[m]);
+        if (act[m]) a.act_list[ix] = (uint32_t)j[m];
+      }
+    }
+    // the shadow (CPU pointer, unit) and the slots
+    const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
+    if (valid == 3u) {
+      st_stream2(reinterpret_cast<void *>(a0), pol_s, outv[0], outv[1]);
+      if (!(i0 & 1)) {
+        st_stream2(shp + i0, pol_s, cv[0], cv[1]);
+        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1,%2}, %3;" ::"l"(shu + i0), "r"(su[0]),
+                     "r"(su[1]), "l"(pol_s)
+                     : "memory");
+      } else {
+#pragma unroll
+        for (int m = 0; m < 2; ++m) {
+          shp[i0 + m] = cv[m];
+          shu[i0 + m] = su[m];
+        }
+      }
+    } else if (valid) {
+#pragma unroll
+      for (int m = 0; m < 2; ++m)
+        if ((valid >> m) & 1) {
+          st_stream1(reinterpret_cast<void *>(a0 + 8ull * m), pol_s, outv[m]);
+          shp[i0 + m] = cv[m];
+          shu[i0 + m] = su[m];
+        }
+    }
+    {  // hit mask: 2 bits per chunk, 16 chunks per word (lanes 0-15: word cb/16, lanes 16-31: the next)
+      const uint32_t b = wrote << (2u * (lane & 15));
+      const uint32_t w0 = warp_or(lane < 16 ? b : 0u), w1 = warp_or(lane < 16 ? 0u : b);
+      const uint64_t wi = cb >> 4;
+      if (lane == 0) a.hitmask[wi] = w0;
+      else if (lane == 16 && cb + 16 < a.nchunks) a.hitmask[wi + 1] = w1;
+    }
+    cv[0] = nv[0];
+    cv[1] = nv[1];
+    nv[0] = nnv[0];
+    nv[1] = nnv[1];
+  }
+  flush_count(&a.st->nulls, (unsigned long long)c_nulls * (unsigned)inc);  // inc = k: k sequential calls
+  flush_count(&a.st->hits, (unsigned long long)c_hits * (unsigned)inc);
+  flush_count(&a.st->misses, (unsigned long long)c_miss * (unsigned)inc);
+  flush_count(&a.st->pending, c_pend);
+  flush_count(&a.st->translated, c_tr);
+}
+
+template <bool ES>
+static int launch_fwd_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
+  const size_t smem = (ES ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
+  static bool configured = false;
+  if (!configured) {
+    int dev = 0, optin = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    cudaError_t e = cudaFuncSetAttribute(k_fwd_lean<ES>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    if (e != cudaSuccess) return (int)e;
+    configured = true;
+  }
+  const uint64_t want = (a.nchunks + FWD_LEAN_THREADS - 1) / FWD_LEAN_THREADS;
+  const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
+  (void)cudaGetLastError();
+  k_fwd_lean<ES><<<grid, FWD_LEAN_THREADS, smem, s>>>(a);
+  return (int)cudaGetLastError();
+}
+
+// -------------------------------------------------------------------------------------------------
+// k_rev_lean: the reverse pass of cgcm_unmapArrayDevice (a3 + a4 [+ Alg. 3 release]) over ONE in-place
+// segment that carries the forward map's shadow, in snapshot mode (no per-unit journal; releases as
+// reductions checked afterwards by k_release_scan).  Same decisions, counters and lists as
+// k_unmap_sh<WRITE|GATE|HITMASK[|DEC], false> in that mode, with the bookkeeping cut to what a slot
+// needs: the rare paths (copy list, deferred materialisation) run under warp votes, the hit / slow
+// masks are built with warp reductions (redux.sync), and the slot stores are unconditional 16-byte
+// writes of whole chunks (a slot that is not translated is written back unchanged; only the ragged
+// ends of the segment are stored slot by slot).  Slots whose shadow check fails go to k_slots
+// SEL_SLOW exactly as after k_unmap_sh.
+// -------------------------------------------------------------------------------------------------
+constexpr int REV_LEAN_THREADS = 768;
+
+template <bool DEC, bool ES>  // ES: the extent deltas are staged in shared memory
+__global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
+  if (ES)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
+  __syncthreads();
+  const uint64_t pol_s = policy_evict_first();
+  const uint64_t pol_t = policy_evict_last();
+  const int lane = threadIdx.x & 31;
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n;
+  const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);
+  const uint32_t *shu = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n);
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint32_t n_ext = (uint32_t)a.tab.n_ext, cur_ep = a.epoch;
+  unsigned c_nulls = 0, c_hits = 0, c_slow = 0;
+
+  struct In {
+    uint64_t g[2], h[2];
+    uint32_t u[2];
+    uint32_t valid;
+  };
+  auto load_in = [&](uint64_t c, In &x) {
+    x.g[0] = x.g[1] = x.h[0] = x.h[1] = 0;
+    x.u[0] = x.u[1] = SH_NONE;
+    x.valid = 0;
+    if (c >= a.nchunks) return;
+    const uint64_t a0 = a0base + 16ull * c;
+    x.valid = (a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u);
+    const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
+    if (x.valid == 3u && !(i0 & 1)) {
+      ld_stream2(reinterpret_cast<const void *>(a0), pol_s, x.g[0], x.g[1]);
+      ld_stream2(shp + i0, pol_s, x.h[0], x.h[1]);
+      asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
+                   : "=r"(x.u[0]), "=r"(x.u[1])
+                   : "l"(shu + i0), "l"(pol_s));
+    } else {
+#pragma unroll
+      for (int m = 0; m < 2; ++m)
+        if ((x.valid >> m) & 1) {
+          x.g[m] = reinterpret_cast<const uint64_t *>(a0)[m];
+          x.h[m] = shp[i0 + m];
+          x.u[m] = shu[i0 + m];
+        }
+    }
+  };
+  auto gather = [&](const In &x, uint64_t w[2]) {
+#pragma unroll
+    for (int m = 0; m < 2; ++m)
+      w[m] = (x.u[m] != SH_NONE && x.g[m] != 0) ? ld_u64_hot(a.tab.st + sh_unit(x.u[m]), pol_t) : 0ull;
+  };
+
+  const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  In cur, nxt, nn;
+  uint64_t cw[2], nw[2];
+  load_in(c_first, cur);
+  load_in(c_first + stride, nxt);
+  gather(cur, cw);
+  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
+    const uint64_t c = cb + lane;
+    load_in(c + 2 * stride, nn);
+    gather(nxt, nw);
+
+    bool hit[2], slow[2], cp[2];
+    uint64_t outv[2];
+    bool rare = false;
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const bool vm = (cur.valid >> m) & 1;
+      const uint64_t g = cur.g[m], w = cw[m];
+      const uint32_t e = hot_ext(w), fl = hot_flags(w), su = sh_unit(cur.u[m]);
+      const uint64_t delta = e < n_ext ? (ES ? s_ext[e] : a.tab.ext_delta[e]) : 0ull;
+      const bool look = vm && g != 0;
+      hit[m] = look && su != SH_NONE && (fl & UF_ACTIVE) && e < n_ext && g == cur.h[m] + delta;
+      slow[m] = look && !hit[m];
+      c_nulls += vm && g == 0;
+      c_hits += hit[m];
+      outv[m] = hit[m] ? cur.h[m] : g;  // reverse: base + (g - devbase), the recorded CPU pointer
+      // Alg. 2: the epoch gate of a hit whose unit is stale (rare after the first slot of each unit)
+      const bool stale = hit[m] && st_epoch(w) != cur_ep;
+      cp[m] = false;
+      if (stale) {
+        if (fl & UF_READONLY) {
+          *lo_word(a.tab.st + su) = cur_ep;  // Alg. 2 line 3 only: never copied back
+        } else {
+          cp[m] = atomicExch(lo_word(a.tab.st + su), cur_ep) != cur_ep;  // stale and not read-only: copy
+        }
+      }
+      // references: a deferred one (a.defer) is dropped by a released hit, materialised otherwise
+      const bool dfr = a.defer && vm && sh_deferred(cur.u[m]);
+      const bool drop = DEC && dfr && hit[m];
+      if (dfr && !drop) red_add(a.tab.rc + su, 1);
+      if (DEC && hit[m] && !drop) red_add(a.tab.rc + su, -sg.inc);  // Alg. 3, checked by k_release_scan
+      rare = rare || cp[m];
+    }
+    c_slow += slow[0] + slow[1];
+    if (__any_sync(0xffffffffu, rare)) {  // copy list of this warp's stale writable units
+#pragma unroll
+      for (int m = 0; m < 2; ++m) {
+        const unsigned long long cx = warp_append(&a.lc[3], cp[m]);
+        if (cp[m]) a.copy_list[cx] = sh_unit(cur.u[m]);
+      }
+    }
+    if (cur.valid == 3u) {
+      st_stream2(reinterpret_cast<void *>(a0base + 16ull * c), pol_s, outv[0], outv[1]);
+    } else {
+#pragma unroll
+      for (int m = 0; m < 2; ++m)
+        if ((cur.valid >> m) & 1) st_stream1(reinterpret_cast<void *>(a0base + 16ull * c + 8ull * m), pol_s, outv[m]);
+    }
+    {  // 2 bits per chunk, 16 chunks per word: lanes 0-15 make word cb/16, lanes 16-31 the next
+      const uint32_t sh = 2u * (lane & 15);
+      const uint32_t hb = ((hit[0] ? 1u : 0u) | (hit[1] ? 2u : 0u)) << sh;
+      const uint32_t sb = ((slow[0] ? 1u : 0u) | (slow[1] ? 2u : 0u)) << sh;
+      const uint32_t lo = lane < 16;
+      const uint32_t h0 = warp_or(lo ? hb : 0u), h1 = warp_or(lo ? 0u : hb);
+      const uint32_t s0 = warp_or(lo ? sb : 0u), s1 = warp_or(lo ? 0u : sb);
+      const uint64_t wi = cb >> 4;
+      if (lane == 0) {
+        a.hitmask[wi] = h0;
+        a.slowmask[wi] = s0;
+      } else if (lane == 16 && cb + 16 < a.nchunks) {
+        a.hitmask[wi + 1] = h1;
+        a.slowmask[wi + 1] = s1;
+      }
+    }
+    cur = nxt;
+    nxt = nn;
+    cw[0] = nw[0];
+    cw[1] = nw[1];
+  }
+  flush_count(&a.st->nulls, c_nulls);
+  flush_count(&a.st->hits, c_hits);
+  flush_count(&a.st->translated, c_hits);
+  flush_count(a.slowcount, c_slow);
+}
+
+template <bool DEC, bool ES>
+static int launch_rev_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
+  const size_t smem = (ES ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
+  static bool configured = false;
+  if (!configured) {
+    int dev = 0, optin = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    cudaError_t e = cudaFuncSetAttribute(k_rev_lean<DEC, ES>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    if (e != cudaSuccess) return (int)e;
+    configured = true;
+  }
+  const uint64_t want = (a.nchunks + REV_LEAN_THREADS - 1) / REV_LEAN_THREADS;
+  const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
+  (void)cudaGetLastError();
+  k_rev_lean<DEC, ES><<<grid, REV_LEAN_THREADS, smem, s>>>(a);
+  return (int)cudaGetLastError();
+}
+template <bool DEC>
+static int launch_rev_lean(const SlotArgs &a, int nsm, cudaStream_t s) {
+  return a.tab.n_ext <= EXT_SMEM ? launch_rev_lean1<DEC, true>(a, nsm, s) : launch_rev_lean1<DEC, false>(a, nsm, s);
+}
+
 // the operation sets the runtime uses
 #define CGCM_SLOT_OPS(X)                                                                          \
   X(DIR_FWD, OP_WRITE | OP_INC | OP_HITMASK)           /* map: forward rewrite + refcount (a2)   */ \
@@ -1405,13 +1815,23 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, i
   static const bool no_pipe = std::getenv("CGCM_NO_PIPELINE") != nullptr;  // A/B experiments
   if (dir == DIR_FWD && ops == (OP_WRITE | OP_INC | OP_HITMASK) && a.pd.nseg > 0 && a.nseg == 1 && a.seg_inplace &&
       a.sel == SEL_ALL && a.cbeg == 0 && !no_pipe)
+  {
+    static const bool no_lean = std::getenv("CGCM_NO_LEAN") != nullptr;  // A/B experiments
+    if (a.segs_host_shadow && a.pd.nseg == 1 && !no_lean)
+      return a.tab.n_ext <= EXT_SMEM ? launch_fwd_lean1<true>(a, nsm, s) : launch_fwd_lean1<false>(a, nsm, s);
     return a.segs_host_shadow ? launch_map_pd<1>(a, nsm, s) : launch_map_pd<0>(a, nsm, s);
+  }
   constexpr int UNMAP = OP_WRITE | OP_GATE | OP_HITMASK, UNMAP_REL = OP_WRITE | OP_GATE | OP_DEC | OP_HITMASK;
   if (dir == DIR_REV && (ops == UNMAP || ops == UNMAP_REL || ops == OP_DEC) && a.segs_host_shadow &&
       a.sel == SEL_ALL && a.cbeg == 0 && !no_pipe) {
     // pipelined pass over the recorded slots, then the generic kernel over the slots it left
     if (cudaMemsetAsync(a.slowcount, 0, sizeof(unsigned long long), s) != cudaSuccess) return (int)cudaGetLastError();
-    int r = ops == UNMAP ? launch_unmap_sh<UNMAP>(a, nsm, s)
+    static const bool no_lean = std::getenv("CGCM_NO_LEAN") != nullptr;  // A/B experiments
+    // the lean pass: one in-place segment with a shadow, snapshot mode (releases as reductions)
+    const bool lean = !no_lean && ops != OP_DEC && a.nseg == 1 && a.seg_inplace && a.no_journal &&
+                      (ops == UNMAP || a.dec_red);
+    int r = lean ? (ops == UNMAP ? launch_rev_lean<false>(a, nsm, s) : launch_rev_lean<true>(a, nsm, s))
+            : ops == UNMAP ? launch_unmap_sh<UNMAP>(a, nsm, s)
             : ops == UNMAP_REL ? launch_unmap_sh<UNMAP_REL>(a, nsm, s)
                                : launch_unmap_sh<OP_DEC>(a, nsm, s);
     if (r != 0) return r;

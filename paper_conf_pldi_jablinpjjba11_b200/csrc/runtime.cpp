@@ -462,14 +462,14 @@ struct Context {
       for (int P = PD_MAXSHIFT; P >= 0; --P) {
         if ((span >> P) + 1 > cap) break;
         uint64_t ovf = 0;  // units in pages with more than PD_K starts after the page's first byte
-        bool fits = true;  // every page: <= PD_CNT_MAX starts, none at offset 0xFFFF (the padding value)
+        bool fits = true;  // every page: <= PD_CNT_MAX starts, none at offset PD_PAD (the padding value)
         for (int i = i0; i < i1 && fits;) {
           const uint64_t pg = (hb[i] - S) >> P;
           int k = i, c = 0;
           while (k < i1 && ((hb[k] - S) >> P) == pg) {
             const uint64_t o = (hb[k] - S) & ((1ull << P) - 1);
             c += o != 0;
-            fits = fits && o != 0xFFFF;
+            fits = fits && o != PD_PAD;
             ++k;
           }
           if (c > PD_K) ovf += (uint64_t)c;
@@ -513,17 +513,17 @@ struct Context {
         w[1] = cnt | (hb[i] == A ? PD_EXACT : 0u) | (end0 << PD_END_SHIFT);
         uint16_t *o16 = reinterpret_cast<uint16_t *>(w + 2);
         if (cnt <= (uint32_t)PD_K) {
-          for (int t = 0; t < 2 * 6; ++t) o16[t] = t < (int)cnt ? (uint16_t)(hb[i + 1 + t] - A) : (uint16_t)0xFFFF;
+          for (int t = 0; t < 2 * 6; ++t) o16[t] = t < (int)cnt ? (uint16_t)(hb[i + 1 + t] - A) : (uint16_t)PD_PAD;
         } else {
           w[2] = (uint32_t)ovf.size();
           w[3] = w[4] = w[5] = w[6] = w[7] = 0xFFFFFFFFu;
           for (uint32_t t = 0; t < cnt; ++t) ovf.push_back((uint16_t)(hb[i + 1 + t] - A));
-          while (ovf.size() % 16) ovf.push_back(0xFFFF);
+          while (ovf.size() % 16) ovf.push_back((uint16_t)PD_PAD);
           ++novf;
         }
       }
     }
-    if (ovf.empty()) ovf.assign(16, 0xFFFF);
+    if (ovf.empty()) ovf.assign(16, (uint16_t)PD_PAD);
     CKS(upload(pd_ent, ent));
     CKS(upload(pd_ovf, ovf));
     CKS(upload(pd_start, starts));

@@ -125,40 +125,44 @@ def test_pagedir_lookup_cases(table, flags):
         W.release_reservation(R, span)
 
 
-def layout_64k():
-    """Segments that exercise 64 KiB pages (P = 16): page offsets reach 0xFFFF (the padding value of the
-    entry's u16 offsets) and a unit's end crosses whole pages.  Segment 0 takes P = 16; segment 1 has a
-    unit starting at page offset 0xFFFF, so it must fall back to a smaller page (build_pd's rule)."""
+PG = 0x8000                                  # the largest page: 32 KiB (cgcm_dev.h PD_MAXSHIFT = 15)
+
+
+def layout_max_pages():
+    """Segments that exercise the largest pages (P = 15): page offsets reach PD_PAD = 0x7FFF (the padding
+    value of the entry's u16 offsets) and a unit's end crosses whole pages.  Segment 0 takes P = 15;
+    segment 1 has a unit starting at page offset 0x7FFF, so it must fall back to a smaller page
+    (build_pd's rule)."""
     offs, sizes = [], []
     S0 = 1 << 20
     pos = S0
-    for k in range(120):                     # ~2 starts per 64 KiB page, never crowded
-        s = 20000 + 16 * (k % 7)
+    for k in range(120):                     # ~2 starts per 32 KiB page, never crowded
+        s = 10000 + 16 * (k % 7)
         offs.append(pos); sizes.append(s)
-        pos += 30000 + 16 * (k % 5)
-    pos = (pos + 0xFFFF) // 0x10000 * 0x10000 + S0 % 0x10000
-    big = pos                                # a unit covering whole pages, then one ending on 0xFFFF
-    offs.append(pos); sizes.append(3 * 0x10000 + 0x1234)
-    pos += 4 * 0x10000
-    offs.append(pos); sizes.append(0xFFFF)   # [A, A + 0xFFFF]: its one-past-end is the next page start
-    pos += 0x10000 + 0x10000
+        pos += 15000 + 16 * (k % 5)
+    pos = (pos + PG - 1) // PG * PG + S0 % PG
+    big = pos                                # a unit covering whole pages, then one ending on PG - 1
+    offs.append(pos); sizes.append(3 * PG + 0x1234)
+    pos += 4 * PG
+    offs.append(pos); sizes.append(PG - 1)   # [A, A + PG - 1]: its one-past-end is the next page start
+    pos += 2 * PG
     S1 = pos + (8 << 20)                     # segment 1
     pos = S1
     offs.append(pos); sizes.append(100)
-    offs.append(S1 + 0xFFFF); sizes.append(10)   # start at page offset 0xFFFF of a 64 KiB page
-    offs.append(S1 + 0x10000 + 0x20); sizes.append(4000)
-    pos = S1 + 0x30000
+    offs.append(S1 + PG - 1); sizes.append(10)   # start at page offset 0x7FFF of a 32 KiB page
+    offs.append(S1 + PG + 0x20); sizes.append(4000)
+    pos = S1 + 3 * PG
     for k in range(60):
-        offs.append(pos); sizes.append(9000)
-        pos += 25000
+        offs.append(pos); sizes.append(4500)
+        pos += 12500
     return (np.array(offs, dtype=np.uint64), np.array(sizes, dtype=np.uint64), pos + (1 << 20), S0, S1, big)
 
 
-def test_pagedir_64k_pages():
+def test_pagedir_max_pages():
     import torch
     import paper_conf_pldi_jablinpjjba11_b200 as cg
     from oracle import Oracle
-    offs, sizes, span, S0, S1, big = layout_64k()
+    offs, sizes, span, S0, S1, big = layout_max_pages()
     R = W.reserve_readonly(span)
     ctx = cg.Context(0, arena_bytes=1 << 28, flags=LENIENT)
     o = Oracle(LENIENT)
@@ -170,12 +174,12 @@ def test_pagedir_64k_pages():
             assert P.o.declareAlloc(int(b), int(s), readonly=True) == 0
         info = P.g.indexInfo()
         assert info["pd_segments"] == 2
-        assert info["pd_max_shift"] == 16 and info["pd_min_shift"] <= 15, info
+        assert info["pd_max_shift"] == 15 and info["pd_min_shift"] <= 14, info
         q = [offs, offs + sizes - np.uint64(1), offs + sizes, offs + sizes + np.uint64(1)]
         for S, npages in ((S0, 72), (S1, 40)):   # every page start, its last byte and neighbours
-            A = np.uint64(S) + np.arange(npages, dtype=np.uint64) * np.uint64(0x10000)
-            q += [A, A + np.uint64(0xFFFF), A + np.uint64(0xFFFE), A + np.uint64(0x8000), A + np.uint64(0x7FFF)]
-        q.append(np.array([big + 0x10000 + 0xFFFF, big + 3 * 0x10000 + 0x1234, big + 3 * 0x10000 + 0x1235],
+            A = np.uint64(S) + np.arange(npages, dtype=np.uint64) * np.uint64(PG)
+            q += [A, A + np.uint64(PG - 1), A + np.uint64(PG - 2), A + np.uint64(PG // 2), A + np.uint64(PG // 2 - 1)]
+        q.append(np.array([big + PG + PG - 1, big + 3 * PG + 0x1234, big + 3 * PG + 0x1235],
                           dtype=np.uint64))
         slots = np.concatenate(q) + np.uint64(R)
         n = len(slots)
