@@ -204,6 +204,40 @@ enum { CGCM_REGION_CHECK = 1u };
 int cgcm_regionBegin(void *const *ptrs, const unsigned *kinds, size_t n, unsigned flags);
 int cgcm_regionEnd(size_t *violations);
 
+/* ================================ glue kernels (NEXT-4) ====================================
+ * P:L305-310 (§5.3 "Glue Kernels"): "Sometimes small CPU code regions between two GPU functions prevent
+ * map promotion.  The performance of this code is inconsequential, but transforming it into a
+ * single-threaded GPU function obviates the need to copy the allocation units between GPU and CPU
+ * memories."  The paper's compiler lowers such a region; at run time the region is given as a short
+ * program for a single GPU thread over 32 64-bit registers:
+ *   r[0..nptrs) = the GPU translations of cpu_ptrs[] (Alg. 1's devptr + (ptr - base) of AUs that must
+ *                 be mapped: refCount > 0, else CGCM_E_NOT_MAPPED; not in an AU: CGCM_E_UNREGISTERED;
+ *                 NULL stays 0), the other registers 0;
+ *   ops (dst, a, b are register numbers < 32, imm a signed 64-bit immediate):
+ *     MOVI  r[dst] = imm                      ADD/SUB/MUL  r[dst] = r[a] op r[b] (u64, wrapping)
+ *     ADDI  r[dst] = r[a] + imm               FADD/FSUB/FMUL/FDIV  binary64 op of r[a], r[b] (RN, no FMA)
+ *     LD    r[dst] = *(u64 *)(r[a] + imm)     ST  *(u64 *)(r[a] + imm) = r[b]
+ *     BNZ   if r[a] != 0: continue at instruction imm (0 <= imm < n)      HALT  stop
+ *   Every LD/ST address must lie, with its 8 bytes, inside the device copy of an ACTIVE unit (a pointer
+ *   loaded from an array-mapped AU is a GPU pointer, so pointer chasing works on device data);
+ *   otherwise CGCM_E_UNREGISTERED.  More than max_steps executed instructions, an unknown op, a
+ *   register >= 32 or a jump out of range: CGCM_E_INVALID.  A failed program may have executed some
+ *   stores (a GPU function is not transactional).
+ * The program runs on main_stream, one thread, and the call returns when it is done.  It is a GPU
+ * function launch: call cgcm_advanceEpoch() after it like after any launch.  regs_out
+ * (optional, 32 entries) receives the final registers.                                          */
+typedef struct {
+  uint32_t op, dst, a, b;
+  int64_t imm;
+} cgcm_glue_op_t;
+enum {
+  CGCM_GLUE_MOVI = 1, CGCM_GLUE_ADD = 2, CGCM_GLUE_ADDI = 3, CGCM_GLUE_SUB = 4, CGCM_GLUE_MUL = 5,
+  CGCM_GLUE_FADD = 6, CGCM_GLUE_FSUB = 7, CGCM_GLUE_FMUL = 8, CGCM_GLUE_FDIV = 9, CGCM_GLUE_LD = 10,
+  CGCM_GLUE_ST = 11, CGCM_GLUE_BNZ = 12, CGCM_GLUE_HALT = 13
+};
+int cgcm_launchGlue(const cgcm_glue_op_t *prog, size_t n, const void *const *cpu_ptrs, size_t nptrs,
+                    uint64_t max_steps, uint64_t *regs_out);
+
 /* ================================ introspection ===========================================
  * cgcm_stats: counters since init.  cgcm_dumpTable: the AU table in base order (cap entries; *n
  *   = total; CGCM_E_NOMEM if cap < total).  cgcm_resetStats zeroes the counters.                */

@@ -44,7 +44,7 @@ def build(force: bool = False) -> str:
     src = os.path.join(HERE, "cgcm_oracle.cpp")
     if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < max(
             os.path.getmtime(src), os.path.getmtime(os.path.join(HERE, "cgcm_oracle.h"))):
-        subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-Wall", "-o", LIB, src])
+        subprocess.check_call(["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-shared", "-fPIC", "-Wall", "-o", LIB, src])
     return LIB
 
 
@@ -80,6 +80,7 @@ def lib():
             "ref_replayDevptr": (C.c_int, [vp, u64, u64]),
             "ref_lookup": (C.c_int, [vp, u64, pu64, pu64]),
             "ref_devLookup": (C.c_int, [vp, u64, pu64, pu64]),
+            "ref_runGlue": (C.c_int, [vp, vp, st, vp, st, u64, vp]),
             "ref_kernel_scale": (C.c_int, [vp, u64, u64, u64, C.c_double]),
             "ref_kernel_treesum_level": (C.c_int, [vp, u64, u64, u64, u64, u64]),
             "ref_kernel_gemm_rows": (C.c_int, [vp, u64, u64, u64, u64, u64, u64, C.c_double, C.c_double]),
@@ -93,6 +94,13 @@ def lib():
 
 def _u64arr(xs) -> np.ndarray:
     return np.ascontiguousarray(np.asarray(xs, dtype=np.uint64))
+
+
+GLUE_OP = np.dtype([("op", "<u4"), ("dst", "<u4"), ("a", "<u4"), ("b", "<u4"), ("imm", "<i8")])
+
+
+def glue_program(rows) -> np.ndarray:
+    return np.array([tuple(int(v) for v in r) for r in rows], dtype=GLUE_OP)
 
 
 class Oracle:
@@ -247,6 +255,15 @@ class Oracle:
 
     def kernel_treesum_level(self, child_dev, root_dev, nnodes, lo, hi):
         return self.L.ref_kernel_treesum_level(self.h, child_dev, root_dev, nnodes, lo, hi)
+
+    def runGlue(self, prog, ptrs, max_steps=1 << 20):
+        """The glue-kernel program (rows of (op, dst, a, b, imm)) on the simulated device; (status, regs)."""
+        arr = glue_program(prog)
+        p = _u64arr(ptrs)
+        regs = np.zeros(32, dtype=np.uint64)
+        s = self.L.ref_runGlue(self.h, arr.ctypes.data, len(arr), p.ctypes.data, len(p), max_steps,
+                               regs.ctypes.data)
+        return s, regs
 
     def kernel_gemm_rows(self, A, B, Cm, n, row0, nrows, alpha, beta):
         return self.L.ref_kernel_gemm_rows(self.h, A, B, Cm, n, row0, nrows, alpha, beta)

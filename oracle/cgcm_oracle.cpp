@@ -618,6 +618,66 @@ int ref_devLookup(void *h, uint64_t g, uint64_t *base, uint64_t *devptr) {
   return 0;
 }
 
+// Glue kernel (NEXT-4; §5.3: a small CPU region "transform[ed] ... into a single-threaded GPU
+// function"): the glue program of the C ABI (cgcm_launchGlue), run by one interpreter loop on the
+// simulated device.  r[i] = Alg. 1's devptr + (p - base) of cpu_ptrs[i], whose unit must be mapped.
+// Every LD/ST of 8 bytes must lie in the device copy of an active unit (devLookup).  Plain C++ doubles
+// (round to nearest; the file is compiled with -ffp-contract=off, so no FMA).
+int ref_runGlue(void *h, const void *prog_v, size_t n, const uint64_t *ptrs, size_t nptrs, uint64_t max_steps,
+                uint64_t *regs_out) {
+  struct Op { uint32_t op, dst, a, b; int64_t imm; };
+  const Op *prog = static_cast<const Op *>(prog_v);
+  Oracle *o = O(h);
+  const size_t NR = 32;
+  if (nptrs > NR) return REF_E_INVALID;
+  u64 r[32] = {0};
+  for (size_t i = 0; i < nptrs; ++i) {
+    if (ptrs[i] == 0) continue;
+    Unit *u = o->lookup(ptrs[i]);
+    if (!u) return REF_E_UNREGISTERED;
+    if (u->refCount <= 0) return REF_E_NOT_MAPPED;
+    r[i] = u->devptr + (ptrs[i] - u->base);
+  }
+  auto dbl = [](u64 x) { double d; std::memcpy(&d, &x, 8); return d; };
+  auto bits = [](double d) { u64 x; std::memcpy(&x, &d, 8); return x; };
+  auto inside = [&](u64 g) {  // 8 bytes inside an active unit's device copy
+    Unit *v = o->devLookup(g);
+    return v && (g % 8) == 0 && g - v->devptr + 8 <= v->size;
+  };
+  int st = REF_OK;
+  u64 steps = 0;
+  size_t pc = 0;
+  while (pc < n) {
+    if (++steps > max_steps) { st = REF_E_INVALID; break; }
+    const Op &x = prog[pc];
+    if (x.dst >= NR || x.a >= NR || x.b >= NR) { st = REF_E_INVALID; break; }
+    size_t next = pc + 1;
+    const u64 a = r[x.a], b = r[x.b];
+    if (x.op == 1) r[x.dst] = (u64)x.imm;
+    else if (x.op == 2) r[x.dst] = a + b;
+    else if (x.op == 3) r[x.dst] = a + (u64)x.imm;
+    else if (x.op == 4) r[x.dst] = a - b;
+    else if (x.op == 5) r[x.dst] = a * b;
+    else if (x.op == 6) r[x.dst] = bits(dbl(a) + dbl(b));
+    else if (x.op == 7) r[x.dst] = bits(dbl(a) - dbl(b));
+    else if (x.op == 8) r[x.dst] = bits(dbl(a) * dbl(b));
+    else if (x.op == 9) r[x.dst] = bits(dbl(a) / dbl(b));
+    else if (x.op == 10 || x.op == 11) {
+      const u64 g = a + (u64)x.imm;
+      if (!inside(g)) { st = REF_E_UNREGISTERED; break; }
+      if (x.op == 10) r[x.dst] = o->dev.get64(g);
+      else o->dev.put64(g, b);
+    } else if (x.op == 12) {
+      if (x.imm < 0 || (u64)x.imm >= n) { st = REF_E_INVALID; break; }
+      if (a != 0) next = (size_t)x.imm;
+    } else if (x.op == 13) next = n;
+    else { st = REF_E_INVALID; break; }
+    pc = next;
+  }
+  if (regs_out) std::memcpy(regs_out, r, sizeof(r));
+  return st;
+}
+
 // S1: x *= alpha over a jagged 2-D array reached through its translated row pointers (config A).
 int ref_kernel_scale(void *h, uint64_t rows_dev, uint64_t nrows, uint64_t ncols, double alpha) {
   Oracle *o = O(h);

@@ -104,6 +104,8 @@ int ref_devLookup(void *h, uint64_t g, uint64_t *base, uint64_t *devptr);
 
 /* sample GPU functions executed on the simulated device (test-only) */
 int ref_kernel_scale(void *h, uint64_t rows_dev, uint64_t nrows, uint64_t ncols, double alpha);
+int ref_runGlue(void *h, const void *prog, size_t n, const uint64_t *ptrs, size_t nptrs, uint64_t max_steps,
+                uint64_t *regs_out);
 int ref_kernel_treesum_level(void *h, uint64_t child_dev, uint64_t root_dev, uint64_t nnodes,
                              uint64_t lo, uint64_t hi);
 /* S2 (config B): C[i][j] = alpha * sum_k A[i][k]*B[k][j] + beta * C[i][j] for rows [row0, row0+nrows),

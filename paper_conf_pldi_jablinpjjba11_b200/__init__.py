@@ -104,6 +104,7 @@ def lib():
             "cgcm_indexInfo": (i, [C.POINTER(IndexInfo)]),
             "cgcm_dumpExtents": (i, [C.c_void_p, C.c_size_t, C.POINTER(C.c_size_t)]),
             "cgcm_storageInfo": (i, [C.POINTER(StorageInfo)]),
+            "cgcm_launchGlue": (i, [C.c_void_p, C.c_size_t, C.c_void_p, C.c_size_t, C.c_uint64, C.c_void_p]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -336,6 +337,22 @@ class Context:
         if s != OK:
             raise CgcmError(f"indexInfo: {strerror(s)}")
         return {f: getattr(ii, f) for f, _ in IndexInfo._fields_}
+
+    # ---- glue kernels (NEXT-4) ----
+    GLUE = dict(MOVI=1, ADD=2, ADDI=3, SUB=4, MUL=5, FADD=6, FSUB=7, FMUL=8, FDIV=9, LD=10, ST=11, BNZ=12, HALT=13)
+
+    def launchGlue(self, prog, ptrs, max_steps=1 << 20):
+        """Run a glue program (rows of (op, dst, a, b, imm), ops by number or name) as one GPU thread over
+        the mapped AUs of ptrs (registers 0..len(ptrs)-1).  Returns (status, final registers)."""
+        import numpy as np
+        dt = np.dtype([("op", "<u4"), ("dst", "<u4"), ("a", "<u4"), ("b", "<u4"), ("imm", "<i8")])
+        rows = [((self.GLUE[r[0]] if isinstance(r[0], str) else int(r[0])),) + tuple(int(v) for v in r[1:]) for r in prog]
+        arr = np.array(rows, dtype=dt)
+        p = np.asarray([int(x) for x in ptrs], dtype=np.uint64)
+        regs = np.zeros(32, dtype=np.uint64)
+        s = self.L.cgcm_launchGlue(arr.ctypes.data if len(arr) else None, len(arr),
+                                   p.ctypes.data if len(p) else None, len(p), max_steps, regs.ctypes.data)
+        return s, regs
 
     def dump_np(self):
         """The unit table as a numpy structured array (fields of cgcm_unit_t) -- for large tables."""

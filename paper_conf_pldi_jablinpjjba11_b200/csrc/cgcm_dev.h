@@ -237,6 +237,30 @@ constexpr uint32_t SH_DEFER = 0x80000000u;
 __host__ __device__ __forceinline__ uint32_t sh_unit(uint32_t w) { return w == SH_NONE ? SH_NONE : (w & ~SH_DEFER); }
 __host__ __device__ __forceinline__ bool sh_deferred(uint32_t w) { return w != SH_NONE && (w & SH_DEFER); }
 
+// Glue kernels (NEXT-4; §5.3): a small straight-line CPU region run as a single-threaded GPU
+// function over mapped data.  The program is the C ABI's cgcm_glue_op_t list (same layout); every load
+// and store is checked against the active units' device copies (reverse index + unit table), so a
+// wrong address is an error, never an illegal access.
+struct GlueOp {
+  uint32_t op, dst, a, b;
+  int64_t imm;
+};
+constexpr int GLUE_REGS = 32;
+struct GlueArgs {
+  const GlueOp *prog;
+  int n;
+  uint64_t *regs;             // GLUE_REGS in/out
+  uint64_t max_steps;
+  int *status;                // 0, or a CGCM_E_* code (+ the failing pc in status[1])
+  TableDev tab;
+  const uint64_t *ext_keys;   // live extents' device starts, sorted (the reverse index keys)
+  const uint64_t *ext_pay;    // host - device delta of each
+  const uint32_t *ext_id;     // extent id of each
+  int n_ext_keys;
+  int U;
+};
+void launch_glue(const GlueArgs &g, cudaStream_t s);
+
 // ---- host-callable launchers (kernels.cu) ----------------------------------------------------
 int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, int *nlaunch);
 void launch_build_levels(const uint64_t *keys, int n, int h, const uint32_t *wide, uint32_t *const *lvl,

@@ -2122,6 +2122,91 @@ void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n
   }
 }
 
+// ---- glue kernels (NEXT-4): one GPU thread runs a short CPU region over mapped data ----
+// is [g, g + 8) inside the device copy of an active unit?  (extent by device start, then the unit by the
+// mirrored host address, then: the unit is ACTIVE and its copy lives in that extent)
+__device__ bool glue_ok(const GlueArgs &A, uint64_t g) {
+  if (A.n_ext_keys <= 0 || g < A.ext_keys[0]) return false;
+  int lo = 0, len = A.n_ext_keys;
+  while (len > 1) {
+    const int half = len >> 1;
+    if (A.ext_keys[lo + half] <= g) lo += half;
+    len -= half;
+  }
+  const uint64_t h = g + A.ext_pay[lo];
+  const uint32_t eid = A.ext_id[lo];
+  if (A.U <= 0 || h < A.tab.base[0]) return false;
+  int j = 0;
+  len = A.U;
+  while (len > 1) {
+    const int half = len >> 1;
+    if (A.tab.base[j + half] <= h) j += half;
+    len -= half;
+  }
+  const uint64_t w = A.tab.hot[j];
+  return (hot_flags(w) & UF_ACTIVE) && (hot_flags(w) & UF_STORAGE) && hot_ext(w) == eid &&
+         h - A.tab.base[j] <= A.tab.size64[j] && A.tab.size64[j] - (h - A.tab.base[j]) >= 8;
+}
+__global__ void k_glue(GlueArgs A) {
+  uint64_t r[GLUE_REGS];
+  for (int i = 0; i < GLUE_REGS; ++i) r[i] = A.regs[i];
+  int st = 0, pc = 0;
+  uint64_t steps = 0;
+  while (pc < A.n) {
+    if (++steps > A.max_steps) {
+      st = -1;  // CGCM_E_INVALID
+      break;
+    }
+    const GlueOp o = A.prog[pc];
+    if (o.dst >= GLUE_REGS || o.a >= GLUE_REGS || o.b >= GLUE_REGS) {
+      st = -1;
+      break;
+    }
+    const uint64_t x = r[o.a], y = r[o.b];
+    int next = pc + 1;
+    switch (o.op) {
+      case 1: r[o.dst] = (uint64_t)o.imm; break;
+      case 2: r[o.dst] = x + y; break;
+      case 3: r[o.dst] = x + (uint64_t)o.imm; break;
+      case 4: r[o.dst] = x - y; break;
+      case 5: r[o.dst] = x * y; break;
+      case 6: r[o.dst] = __double_as_longlong(__dadd_rn(__longlong_as_double(x), __longlong_as_double(y))); break;
+      case 7: r[o.dst] = __double_as_longlong(__dsub_rn(__longlong_as_double(x), __longlong_as_double(y))); break;
+      case 8: r[o.dst] = __double_as_longlong(__dmul_rn(__longlong_as_double(x), __longlong_as_double(y))); break;
+      case 9: r[o.dst] = __double_as_longlong(__ddiv_rn(__longlong_as_double(x), __longlong_as_double(y))); break;
+      case 10:
+      case 11: {
+        const uint64_t g = x + (uint64_t)o.imm;
+        if ((g & 7) || !glue_ok(A, g)) {
+          st = -2;  // CGCM_E_UNREGISTERED
+          break;
+        }
+        if (o.op == 10) r[o.dst] = *reinterpret_cast<volatile uint64_t *>(g);
+        else *reinterpret_cast<volatile uint64_t *>(g) = y;
+        break;
+      }
+      case 12:
+        if (o.imm < 0 || o.imm >= A.n) {
+          st = -1;
+          break;
+        }
+        if (x != 0) next = (int)o.imm;
+        break;
+      case 13: next = A.n; break;
+      default: st = -1; break;
+    }
+    if (st) break;
+    pc = next;
+  }
+  for (int i = 0; i < GLUE_REGS; ++i) A.regs[i] = r[i];
+  A.status[0] = st;
+  A.status[1] = pc;
+}
+void launch_glue(const GlueArgs &g, cudaStream_t s) {
+  (void)cudaGetLastError();
+  k_glue<<<1, 1, 0, s>>>(g);
+}
+
 // up to two byte ranges (either side may be mapped pinned host memory); 16-byte words when aligned
 __global__ void k_copy_small(unsigned char *dst, const unsigned char *src, size_t n, unsigned char *dst2,
                              const unsigned char *src2, size_t n2) {

@@ -13,6 +13,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <chrono>
 #include <cerrno>
 #include <cstdint>
 #include <cstdlib>
@@ -49,6 +50,23 @@ thread_local std::string g_last_cuda_error;
   } while (0)
 
 static inline uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+// CGCM_TRACE=1: host-side phase timings on stderr (wall clock of the host thread, for finding where a
+// call's time goes; off by default)
+struct Trace {
+  const char *what;
+  std::chrono::steady_clock::time_point t0;
+  static bool on() {
+    static const bool e = std::getenv("CGCM_TRACE") != nullptr;
+    return e;
+  }
+  explicit Trace(const char *w) : what(w), t0(std::chrono::steady_clock::now()) {}
+  ~Trace() {
+    if (on())
+      std::fprintf(stderr, "[cgcm] %-28s %9.3f ms\n", what,
+                   std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+  }
+};
 
 // ---------------------------------------------------------------------------------------------
 // Device arena: best-fit free list over [base, base+cap) with 256-byte granularity.  All device
@@ -237,7 +255,7 @@ struct Context {
   uint32_t pd_minP = 0, pd_maxP = 0;
 
   // scratch
-  DevBuf slowmask, slowcnt, dump_rc;
+  DevBuf slowmask, slowcnt, dump_rc, glue_prog, glue_regs, glue_status;
   DevBuf status, lc, hitmask, act_list, journal, free_list, copy_list, segs, seg0, staging, staging2, staging_cb, points, ptrs, temp;
   DevBuf up_units, up_vals, up_exts, uops;
   HostBuf h_small, h_status, h_list, h_pack[2];
@@ -548,6 +566,7 @@ struct Context {
 
   // merge pending declares/undeclares into the device table (A19: kernels only see a compacted table)
   int ensure_table() {
+    Trace trace_("ensure_table");
     if (!table_dirty) return CGCM_OK;
     CKS(materialise_all());  // deferred references name units by their index in the table being replaced
     int n = (int)reg.size();
@@ -836,6 +855,7 @@ struct Context {
   }
   // fetch the 8 Status blocks + list counters (synchronizes main)
   int fetch_status(Status out[8], unsigned long long lcs[4]) {
+    Trace trace_("fetch_status(sync)");
     // a kernel writes them into mapped pinned memory: no DMA to queue behind other copies (cgcm_dev.h)
     launch_copy_small(h_status.p, status.as<void>(), sizeof(Status) * 8, h_status.as<char>() + sizeof(Status) * 8,
                       lc.as<void>(), 32, main);
@@ -913,6 +933,7 @@ struct Context {
 
   // sorted unique unit list from a device list of n entries
   int sorted_units(const DevBuf &src, size_t n, std::vector<uint32_t> &out) {
+    Trace trace_("sorted_units");
     out.clear();
     if (!n) return CGCM_OK;
     if (n > 1) {
@@ -957,6 +978,7 @@ struct Context {
   // the main stream then does NOT wait for the copies -- the caller waits per pack (transfer overlap)
   int activate_units(const std::vector<uint32_t> &units, std::vector<std::pair<uint64_t, uint64_t>> *h2d_out,
                      std::vector<cudaEvent_t> *pack_ev = nullptr) {
+    Trace trace_("activate_units");
     if (units.empty()) return CGCM_OK;
     const uint64_t PACK_SPAN = 64ull << 20, GAPMAX = 64ull << 10, PACK_MIN = 256ull << 10;
     struct Pack {
@@ -1127,6 +1149,7 @@ struct Context {
 
   // units whose refcount reached 0: free device storage (globals keep theirs), clear flags
   int free_units(const std::vector<uint32_t> &units) {
+    Trace trace_("free_units");
     if (units.empty()) return CGCM_OK;
     CKS(upload(up_units, units));
     launch_deactivate(up_units.as<uint32_t>(), (int)units.size(), tab(), main);
@@ -1134,9 +1157,11 @@ struct Context {
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(main));
     for (uint32_t x : units) {
+      const bool was_arr = uarr[x] != 0;
+      if (was_arr) arr_gen.erase(ubase[x]);  // no longer array-mapped: the next mapArray translates from host slots
       uarr[x] = 0;
-      arr_gen.erase(ubase[x]);  // no longer array-mapped: the next mapArray translates from host slots
-      if (udev[x]) drop_shadows(udev[x]);
+      // an outer's shadows go with its copy (and a device array's, if one lived in this copy)
+      if (udev[x] && (was_arr || dev_shadows)) drop_shadows(udev[x]);
       if (uflags[x] & UF_GLOBAL) continue;
       run_release(urun[x]);
       urun[x] = -1;
@@ -1150,6 +1175,7 @@ struct Context {
   // copy-back of whole units device -> host (Alg. 2's cuMemcpyDtoH).  Array-mapped units are
   // reverse translated first (A12) -- validated before any byte moves.  Synchronous.
   int copy_back(const std::vector<uint32_t> &units) {
+    Trace trace_("copy_back");
     if (units.empty()) return CGCM_OK;
     std::vector<uint32_t> plain, arr;
     for (uint32_t x : units) (uarr[x] ? arr : plain).push_back(x);
@@ -1242,6 +1268,7 @@ struct Context {
   int map_core(const std::vector<Seg> &fsegs, const std::vector<Seg> &rsegs, uint64_t *translated_out,
                uint64_t *nulls_out, const std::vector<int> *seg_group = nullptr,
                const std::vector<cudaEvent_t> *group_ev = nullptr, bool defer = false) {
+    Trace trace_("map_core");
     uint64_t total = 0;
     for (auto &s : fsegs) total += s.n;
     if (fsegs.empty() && rsegs.empty()) {  // nothing to translate (e.g. every outer was re-mapped, A9)
@@ -1385,6 +1412,7 @@ struct Context {
   //   ops: OP_WRITE|OP_GATE|OP_HITMASK [|OP_DEC] or OP_GATE
   int unmap_rev_core(const std::vector<Seg> &segs, bool write, bool dec, std::vector<uint32_t> &copy_units,
                      std::vector<uint32_t> &freed, uint64_t &journal_count, Status &res, bool defer = false) {
+    Trace trace_("unmap_rev_core");
     CKS(ensure_rev());
     uint64_t total = 0;
     for (auto &s : segs) total += s.n;
@@ -1434,7 +1462,9 @@ struct Context {
     uint64_t gen = 0;
     bool valid = false;
     bool deferred = false;  // its unit words may carry deferred references (SH_DEFER)
+    bool device_array = false;  // cgcm_mapArrayDevice's (else a host-array outer's device copy)
   };
+  size_t dev_shadows = 0;  // shadows of device arrays (free_units checks every freed copy only then)
   // Deferred references: the last cgcm_mapArrayDevice may have recorded references in
   // its shadow instead of rc.  Every other call that reads or changes refcounts (or replaces the table)
   // first adds them to rc -- only the matching cgcm_unmapArrayDevice(..., CGCM_RELEASE) drops them.
@@ -1467,17 +1497,22 @@ struct Context {
   // the 12-byte shadow: arrays of >= 2^16 slots and indexes with >= 2 levels (measured, config C
   // (h = 2): 48.5 vs 43.5 G/s); CGCM_FORCE_SHADOW: every array (tests).  Returns the buffer (invalid until the map
   // succeeds: commit_shadow) or 0.
-  uint64_t begin_shadow(uint64_t ptr, uint64_t n) {
+  uint64_t begin_shadow(uint64_t ptr, uint64_t n, bool device_array = false) {
     static const int min_h = [] {  // CGCM_SHADOW_MIN_H: A/B override of the depth threshold
       const char *e = std::getenv("CGCM_SHADOW_MIN_H");
       return e ? std::atoi(e) : 2;
     }();
     if (!(flags & CGCM_FORCE_SHADOW) && (n < (1u << 16) || fwd.h < min_h)) return 0;
     auto key = std::make_pair(ptr, n);
-    Shadow &sh = shadows[key];
+    auto ins = shadows.emplace(key, Shadow());
+    Shadow &sh = ins.first->second;
+    if (ins.second && device_array) {
+      sh.device_array = true;
+      dev_shadows += 1;
+    }
     sh.valid = false;
     if (dalloc(sh.buf, 12 * n + 64) != CGCM_OK) {
-      shadows.erase(key);
+      erase_shadow(shadows.find(key));
       return 0;
     }
     return sh.buf.addr;
@@ -1489,9 +1524,14 @@ struct Context {
       it->second.valid = true;
       it->second.gen = table_gen;
     } else {
-      dfree(it->second.buf);
-      shadows.erase(it);
+      erase_shadow(it);
     }
+  }
+  std::map<std::pair<uint64_t, uint64_t>, Shadow>::iterator erase_shadow(
+      std::map<std::pair<uint64_t, uint64_t>, Shadow>::iterator it) {
+    dfree(it->second.buf);
+    if (it->second.device_array) dev_shadows -= 1;
+    return shadows.erase(it);
   }
   // the valid shadow of (ptr, n), or 0
   uint64_t find_shadow(uint64_t ptr, uint64_t n) const {
@@ -1502,8 +1542,7 @@ struct Context {
   void drop_shadows(uint64_t ptr) {
     for (auto it = shadows.lower_bound(std::make_pair(ptr, (uint64_t)0)); it != shadows.end() && it->first.first == ptr;) {
       materialise(*it);
-      dfree(it->second.buf);
-      it = shadows.erase(it);
+      it = erase_shadow(it);
     }
   }
   int take_snapshot() {
@@ -2016,7 +2055,7 @@ int cgcm_mapArrayDevice(uint64_t *d_slots, size_t n) {
   if (!d_slots || (reinterpret_cast<uint64_t>(d_slots) & 7)) return CGCM_E_INVALID;
   CKS(C->ensure_table());
   Seg s{reinterpret_cast<uint64_t>(d_slots), n, 0, 1, 0};
-  s.shadow = C->begin_shadow(s.ptr, n);
+  s.shadow = C->begin_shadow(s.ptr, n, true);
   // with a shadow, references to units already active are deferred into it
   int r = C->map_core({s}, {}, nullptr, nullptr, nullptr, nullptr, s.shadow != 0);
   if (s.shadow) {
@@ -2787,6 +2826,60 @@ int cgcm_arenaUsage(size_t *used, size_t *capacity) {
   if (used) *used = C->arena.used();
   if (capacity) *capacity = C->arena.capacity();
   return CGCM_OK;
+}
+
+// ---- glue kernels (NEXT-4) --------------------------------------------------------------
+int cgcm_launchGlue(const cgcm_glue_op_t *prog, size_t n, const void *const *cpu_ptrs, size_t nptrs,
+                    uint64_t max_steps, uint64_t *regs_out) {
+  CTXM();
+  static_assert(sizeof(cgcm_glue_op_t) == sizeof(GlueOp), "glue op layout");
+  if ((!prog && n) || n > (1u << 20) || nptrs > (size_t)GLUE_REGS || (nptrs && !cpu_ptrs)) return CGCM_E_INVALID;
+  std::vector<uint64_t> regs(GLUE_REGS, 0);
+  if (nptrs) {  // Alg. 1's translation of each pointer into its (already mapped) unit's device copy
+    std::vector<PointInfo> info;
+    std::vector<uint64_t> nz;
+    for (size_t i = 0; i < nptrs; ++i)
+      if (cpu_ptrs[i]) nz.push_back(reinterpret_cast<uint64_t>(cpu_ptrs[i]));
+    if (!nz.empty()) CKS(C->lookup_points(nz.data(), nz.size(), info));
+    size_t k = 0;
+    for (size_t i = 0; i < nptrs; ++i) {
+      if (!cpu_ptrs[i]) continue;
+      const PointInfo &pi = info[k++];
+      if (pi.unit < 0) return CGCM_E_UNREGISTERED;
+      if (pi.refcount <= 0 || !(pi.flags & UF_STORAGE)) return CGCM_E_NOT_MAPPED;
+      regs[i] = pi.devbase + (reinterpret_cast<uint64_t>(cpu_ptrs[i]) - pi.base);
+    }
+  }
+  CKS(C->ensure_rev());
+  std::vector<GlueOp> ops(n);
+  if (n) std::memcpy(ops.data(), prog, n * sizeof(GlueOp));
+  if (ops.empty()) ops.push_back(GlueOp{13, 0, 0, 0, 0});
+  CKS(C->upload(C->glue_prog, ops));
+  CKS(C->upload(C->glue_regs, regs));
+  CKS(C->dalloc(C->glue_status, 64));
+  GlueArgs g;
+  g.prog = C->glue_prog.as<GlueOp>();
+  g.n = (int)n;
+  g.regs = C->glue_regs.as<uint64_t>();
+  g.max_steps = max_steps;
+  g.status = C->glue_status.as<int>();
+  g.tab = C->tab();
+  g.ext_keys = C->rev.keys.as<uint64_t>();
+  g.ext_pay = C->rev.pay.as<uint64_t>();
+  g.ext_id = C->rev.rid.as<uint32_t>();
+  g.n_ext_keys = (int)C->live_runs.size();
+  g.U = C->U;
+  launch_glue(g, C->main);
+  C->st.kernel_launches += 1;
+  CK(cudaGetLastError());
+  std::vector<int> st;
+  CKS(C->download(st, C->glue_status, 2));
+  if (regs_out) {
+    std::vector<uint64_t> ro;
+    CKS(C->download(ro, C->glue_regs, GLUE_REGS));
+    std::memcpy(regs_out, ro.data(), 8 * GLUE_REGS);
+  }
+  return st[0];
 }
 
 int cgcm_dumpExtents(cgcm_extent_t *out, size_t cap, size_t *n) {
