@@ -1371,12 +1371,11 @@ __device__ __forceinline__ uint32_t off_at(uint64_t q1, uint64_t q2, uint64_t q3
   const uint64_t q = i < 4 ? q1 : (i < 8 ? q2 : q3);
   return (uint32_t)(q >> (16 * (i & 3))) & 0xFFFFu;
 }
-// crowded page (more than PD_K starts): count in the side array, one sector per 16 offsets
-__device__ __noinline__ void pd_crowded(const uint16_t *ovf, uint32_t first, uint32_t cnt, uint32_t r, uint32_t &k,
-                                        uint32_t &off) {
+// crowded page (more than PD_K starts): count in the side array, one sector per 16 offsets; returns
+// k | (offset of start k - 1) << 32
+__device__ __noinline__ uint64_t pd_crowded(const uint16_t *ovf, uint32_t first, uint32_t cnt, uint32_t r) {
   const uint64_t r4 = (uint64_t)r * 0x0001000100010001ull;
-  k = 0;
-  off = 0;
+  uint32_t k = 0, off = 0;
   for (uint32_t t = 0; t < cnt; t += 16) {
     uint64_t v[4];
     asm volatile("ld.global.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(v[0]), "=l"(v[1]), "=l"(v[2]), "=l"(v[3]) : "l"(ovf + first + t));
@@ -1390,6 +1389,7 @@ __device__ __noinline__ void pd_crowded(const uint16_t *ovf, uint32_t first, uin
     k += c;
     if (c < 16) break;  // later sectors hold larger offsets only
   }
+  return (uint64_t)k | ((uint64_t)off << 32);
 }
 
 template <bool ES>  // ES: the extent deltas are staged in shared memory
@@ -1416,62 +1416,79 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   unsigned c_nulls = 0, c_hits = 0, c_miss = 0, c_pend = 0, c_tr = 0;
 
+  auto valid_of = [&](uint64_t c) -> uint32_t {
+    const uint64_t a0 = a0base + 16ull * c;
+    return c < a.nchunks ? ((a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u)) : 0u;
+  };
+  // front half of a1 for the two slots of a chunk: the page of each, and its entry gather issued
+  // (ok); beyond the last page, the tail of the segment's last unit (jt, decided by its end, A7) or -1
+  struct Front {
+    uint64_t ew[2][4];
+    uint32_t poff[2];
+    int jt[2];
+    bool ok[2];
+  };
+  auto front = [&](const uint64_t p[2], uint32_t valid, Front &f) {
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const bool look = ((valid >> m) & 1) && p[m] != 0 && p[m] >= S0;
+      const uint64_t rel = p[m] - S0;
+      const uint64_t pg = rel >> P;
+      f.ok[m] = look && pg < npages;
+      f.poff[m] = (uint32_t)rel & pmask;
+      f.jt[m] = look && !f.ok[m] && p[m] <= Send ? (int)lastu : -1;
+      f.ew[m][0] = f.ew[m][1] = f.ew[m][2] = f.ew[m][3] = 0;
+      if (f.ok[m])  // one LDG.256, not allocated in L1
+        asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+                     : "=l"(f.ew[m][0]), "=l"(f.ew[m][1]), "=l"(f.ew[m][2]), "=l"(f.ew[m][3])
+                     : "l"(ent + 8 * pg), "l"(pol_t));
+    }
+  };
+
+  // software pipeline: slot values two chunks ahead, page-entry gathers one chunk ahead
   const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   uint64_t cv[2] = {0, 0}, nv[2] = {0, 0}, nnv[2] = {0, 0};
   if (c_first < a.nchunks) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c_first), pol_s, cv[0], cv[1]);
   if (c_first + stride < a.nchunks)
     ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, nv[0], nv[1]);
+  Front fc, fn;
+  front(cv, valid_of(c_first), fc);
   for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
     const uint64_t c = cb + lane;
-    if (c + 2 * stride < a.nchunks)  // pipeline: the slot values of chunk t+2
+    if (c + 2 * stride < a.nchunks)
       ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, nnv[0], nnv[1]);
+    front(nv, valid_of(c + stride), fn);  // the next chunk's entries are in flight while this one finishes
     const uint64_t a0 = a0base + 16ull * c;
-    const uint32_t valid = c < a.nchunks ? ((a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u)) : 0u;
+    const uint32_t valid = valid_of(c);
 
-    // a1: the page entry of each slot (both gathers in flight before either is decoded)
-    uint64_t ew[2][4];
-    uint32_t poff[2];
-    int j[2];
-    bool ok[2];
-#pragma unroll
-    for (int m = 0; m < 2; ++m) {
-      const uint64_t p = cv[m];
-      const bool look = ((valid >> m) & 1) && p != 0 && p >= S0;
-      const uint64_t rel = p - S0;
-      const uint64_t pg = rel >> P;
-      ok[m] = look && pg < npages;
-      poff[m] = (uint32_t)rel & pmask;
-      // beyond the last page: the tail of the segment's last unit (decided by its end, A7), or a miss
-      j[m] = look && !ok[m] && p <= Send ? (int)lastu : -1;
-      ew[m][0] = ew[m][1] = ew[m][2] = ew[m][3] = 0;
-      if (ok[m])
-        asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
-                     : "=l"(ew[m][0]), "=l"(ew[m][1]), "=l"(ew[m][2]), "=l"(ew[m][3])
-                     : "l"(ent + 8 * pg), "l"(pol_t));
-    }
     // decode: j = j0 + #{offsets <= p - A}; the page's j0 is decided by its end, others by base + size
+    int j[2];
     bool k0[2];
     uint64_t key[2];
     uint32_t cw[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
+      j[m] = fc.jt[m];
       k0[m] = true;
       key[m] = 0;
-      if (ok[m]) {
-        const uint32_t j0 = (uint32_t)ew[m][0], w1 = (uint32_t)(ew[m][0] >> 32);
+      if (fc.ok[m]) {
+        const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
         const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
-        const uint32_t r = min(poff[m], PD_PAD - 1u);
+        const uint32_t r = min(fc.poff[m], PD_PAD - 1u);
         uint32_t k, off;
         if (cnt <= (uint32_t)PD_K) {
-          const uint64_t r4 = (uint64_t)r * 0x0001000100010001ull;
-          k = le4(ew[m][1], r4) + le4(ew[m][2], r4) + le4(ew[m][3], r4);
-          off = k ? off_at(ew[m][1], ew[m][2], ew[m][3], k - 1) : 0u;
+          const uint32_t r2 = r | (r << 16);
+          const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
+          k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
+          off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
         } else {
-          pd_crowded(a.pd.ovf, (uint32_t)ew[m][1], cnt, r, k, off);
+          const uint64_t ko = pd_crowded(a.pd.ovf, (uint32_t)fc.ew[m][1], cnt, r);
+          k = (uint32_t)ko;
+          off = (uint32_t)(ko >> 32);
         }
         k0[m] = k == 0;
-        j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && poff[m] < end0 ? (int)j0 : -1);
-        key[m] = cv[m] - poff[m] + off;  // the candidate's base (A + offset)
+        j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
+        key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
       }
       cw[m] = 0;
       if (j[m] >= 0)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
@@ -1555,6 +1572,7 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
     cv[1] = nv[1];
     nv[0] = nnv[0];
     nv[1] = nnv[1];
+    fc = fn;
   }
   flush_count(&a.st->nulls, (unsigned long long)c_nulls * (unsigned)inc);  // inc = k: k sequential calls
   flush_count(&a.st->hits, (unsigned long long)c_hits * (unsigned)inc);
