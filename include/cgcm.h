@@ -76,6 +76,9 @@ typedef struct {
   double fwd_kernel_ms, rev_kernel_ms; /* CGCM_PROFILE: summed event time of the hot slot kernels */
   uint64_t fwd_kernel_calls, rev_kernel_calls;
   uint64_t fwd_kernel_slots, rev_kernel_slots; /* slots processed by those launches               */
+  /* NEXT-3 coherence groups: activations copied from a peer context's device copy (compared
+   * exactly with the oracle), and the device-to-device copies that moved them (reported) */
+  uint64_t peer_units, peer_bytes, peer_memcpy_calls;
 } cgcm_stats_t;
 
 /* ================================ lifecycle =================================================
@@ -203,6 +206,26 @@ enum { CGCM_REGION_MAP = 0u, CGCM_REGION_MAPARRAY = 1u };
 enum { CGCM_REGION_CHECK = 1u };
 int cgcm_regionBegin(void *const *ptrs, const unsigned *kinds, size_t n, unsigned flags);
 int cgcm_regionEnd(size_t *violations);
+
+/* ================================ coherence groups (NEXT-3) ================================
+ * The paper maps AUs between the CPU and ONE GPU (one GTX 480).  A coherence
+ * group extends that to several contexts (one per GPU, or several on one GPU) over one CPU address
+ * space: each context keeps its own table, refcounts and epochs (an epoch per GPU), and a writable AU
+ * may be active on several of them.  Reading A31: when a context activates an AU (Alg. 1's
+ * refCount 0 -> 1 copy), and another member -- the first in join order -- holds the same AU (same base
+ * and size) active and DIRTY, i.e. it launched a GPU function since the AU became coherent there (its
+ * unmap would copy the AU back, Alg. 2) and the AU is not read-only, the copy comes from that member's
+ * device copy (device to device: NVLink peer copy across GPUs) instead of the host.  Ordered after the
+ * work already on the source context's main stream.  Counted in peer_units / peer_bytes, not h2d_*.
+ * Two members writing one AU between their unmaps is undefined, as CPU writes to a mapped AU are (A16).
+ * cgcm_groupCreate: a new empty group.  cgcm_groupJoin: the current context joins (at most one group).
+ * cgcm_groupLeave: the current context leaves (also done by cgcm_finalize).  cgcm_groupDestroy: the
+ * group must be empty.  The members of a group must not be called concurrently from several threads
+ * (an activation reads the peers' tables under their locks).                                      */
+int cgcm_groupCreate(void **group_out);
+int cgcm_groupJoin(void *group);
+int cgcm_groupLeave(void);
+int cgcm_groupDestroy(void *group);
 
 /* ================================ glue kernels (NEXT-4) ====================================
  * P:L305-310 (§5.3 "Glue Kernels"): "Sometimes small CPU code regions between two GPU functions prevent

@@ -32,7 +32,7 @@ class RefUnit(C.Structure):
 
 
 STAT_FIELDS = ["h2d_units", "h2d_bytes", "d2h_units", "d2h_bytes", "activations", "frees",
-               "fwd_translations", "rev_translations", "null_slots", "passthrough"]
+               "fwd_translations", "rev_translations", "null_slots", "passthrough", "peer_units", "peer_bytes"]
 
 
 class RefStats(C.Structure):
@@ -58,7 +58,7 @@ def lib():
         L = C.CDLL(LIB)
         u64, vp, st, pu64 = C.c_uint64, C.c_void_p, C.c_size_t, C.POINTER(C.c_uint64)
         sig = {
-            "ref_create": (vp, [C.c_uint]), "ref_destroy": (None, [vp]),
+            "ref_create": (vp, [C.c_uint]), "ref_destroy": (None, [vp]), "ref_groupJoin": (C.c_int, [vp, vp]),
             "ref_declareAlloc": (C.c_int, [vp, u64, u64]),
             "ref_declareAllocFlags": (C.c_int, [vp, u64, u64, C.c_uint]),
             "ref_declareGlobal": (C.c_int, [vp, C.c_char_p, u64, u64, C.c_int]),
@@ -122,6 +122,10 @@ class Oracle:
             pass
 
     # registration
+    def groupJoin(self, leader):
+        """NEXT-3: join the coherence group of `leader` (shared host memory, own device/table/epochs)."""
+        return self.L.ref_groupJoin(self.h, leader.h)
+
     def declareAlloc(self, base, size, readonly=False):
         if readonly:
             return self.L.ref_declareAllocFlags(self.h, base, size, UNIT_READONLY)

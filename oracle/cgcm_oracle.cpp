@@ -18,6 +18,7 @@
 //   sample kernels S1/S3 ..................... pinned (numpy repeated multiply / recursive sum)
 #include "cgcm_oracle.h"
 
+#include <algorithm>
 #include <array>
 #include <climits>
 #include <cstring>
@@ -146,16 +147,21 @@ struct Oracle {
   std::map<u64, u64> active;   // devptr -> base of units with refCount > 0 (for devLookup, a3)
   std::unordered_set<std::string> globalNames;
   u64 globalEpoch = 0;         // P:L233-234; starts at 0 (A20)
-  SparseMem host, dev;
+  SparseMem ownHost, dev;
+  SparseMem *hostp = &ownHost;  // the host memory (a coherence group's members share the leader's)
+  SparseMem &host() { return *hostp; }
+  // NEXT-3 coherence group (reading A31): the members in join order, shared by all of them
+  std::shared_ptr<std::vector<Oracle *>> group;
   u64 cursor = DEV0;
   std::unordered_map<u64, u64> replay;  // base -> devptr to use at the next activation
   ref_stats_t st{};
   Txn txn;
 
-  Oracle() { host.txn = &txn; dev.txn = &txn; }
+  Oracle() { ownHost.txn = &txn; dev.txn = &txn; }
 
   // ---- transactions ------------------------------------------------------------------------
   void begin() {
+    hostp->txn = &txn;  // a shared host journals into the member whose call is running
     txn.on = true;
     txn.savedUnits.clear(); txn.activeOps.clear(); txn.savedPages.clear();
     txn.stats = st; txn.cursor = cursor; txn.replay = replay;
@@ -213,6 +219,20 @@ struct Oracle {
     cursor = d + u.size + 1 + 16;                           // 1 B slack (A7) + 16 B guard
     return d;
   }
+  // NEXT-3 (A31): the first other member of the group (join order) holding the same AU active and dirty
+  // -- it launched a GPU function since the AU became coherent there (epoch != its globalEpoch, the
+  // condition under which its unmap would copy back, Alg. 2) -- and writable; else none (the host is current)
+  Oracle *peerSource(const Unit &u) {
+    if (!group) return nullptr;
+    for (Oracle *c : *group) {
+      if (c == this) continue;
+      auto it = c->table.find(u.base);
+      if (it == c->table.end() || it->second.size != u.size) continue;
+      const Unit &cu = it->second;
+      if (cu.refCount > 0 && cu.epoch != c->globalEpoch && !cu.isReadOnly) return c;
+    }
+    return nullptr;
+  }
   // refCount 0 -> 1 transition of Alg. 1 (allocation/named region + optional HtoD copy)
   void activate(Unit &u, bool copyHtoD) {
     Unit &m = mut(u);
@@ -221,9 +241,16 @@ struct Oracle {
     } else {
       m.devptr = devAlloc(m);                                               // cuMemAlloc
     }
-    if (copyHtoD) {                                                         // cuMemcpyHtoD
-      copyMem(dev, m.devptr, host, m.base, m.size);
-      st.h2d_units += 1; st.h2d_bytes += m.size;
+    if (copyHtoD) {
+      Oracle *src = peerSource(m);
+      if (src) {  // NEXT-3 (A31): the newest copy is on a group peer's device -- copy it from there
+        const Unit &pu = src->table.at(m.base);
+        copyMem(dev, m.devptr, src->dev, pu.devptr, m.size);
+        st.peer_units += 1; st.peer_bytes += m.size;
+      } else {                                                              // cuMemcpyHtoD
+        copyMem(dev, m.devptr, host(), m.base, m.size);
+        st.h2d_units += 1; st.h2d_bytes += m.size;
+      }
     }
     if (!(flags & REF_LITERAL_EPOCH)) m.epoch = globalEpoch;  // A5 reading R1
     st.activations += 1;
@@ -263,11 +290,11 @@ struct Oracle {
             st.rev_translations += 1;
           }
         }
-        host.put64(u.base + 8 * i, h);
+        host().put64(u.base + 8 * i, h);
       }
-      copyMem(host, u.base + 8 * n, dev, u.devptr + 8 * n, u.size - 8 * n);
+      copyMem(host(), u.base + 8 * n, dev, u.devptr + 8 * n, u.size - 8 * n);
     } else {
-      copyMem(host, u.base, dev, u.devptr, u.size);
+      copyMem(host(), u.base, dev, u.devptr, u.size);
     }
     st.d2h_units += 1; st.d2h_bytes += u.size;
     return REF_OK;
@@ -311,7 +338,7 @@ struct Oracle {
   }
   std::vector<u64> hostSlots(const Unit &o) {
     std::vector<u64> q(o.size / 8);
-    for (u64 i = 0; i < q.size(); ++i) q[i] = host.get64(o.base + 8 * i);
+    for (u64 i = 0; i < q.size(); ++i) q[i] = host().get64(o.base + 8 * i);
     return q;
   }
 
@@ -326,7 +353,7 @@ struct Oracle {
     if (o->refCount == 0) {
       // activate without the raw copy: the "new array" of translated pointers is o's HtoD
       activate(*o, false);
-      copyMem(dev, o->devptr + 8 * n, host, o->base + 8 * n, o->size - 8 * n);  // trailing bytes
+      copyMem(dev, o->devptr + 8 * n, host(), o->base + 8 * n, o->size - 8 * n);  // trailing bytes
       st.h2d_units += 1; st.h2d_bytes += o->size;
     }
     if (o->refCount >= INT32_MAX) return REF_E_INVALID;
@@ -352,7 +379,7 @@ struct Oracle {
     std::vector<u64> h(o->size / 8);
     bool copy_o = o->epoch != globalEpoch && !o->isReadOnly;
     for (u64 i = 0; i < h.size(); ++i) {
-      if (!copy_o) { h[i] = host.get64(o->base + 8 * i); continue; }
+      if (!copy_o) { h[i] = host().get64(o->base + 8 * i); continue; }
       u64 g = dev.get64(o->devptr + 8 * i);
       if (!o->arrayMapped || g == 0) { h[i] = g; continue; }
       Unit *v = devLookup(g);
@@ -457,12 +484,31 @@ Oracle *O(void *h) { return static_cast<Oracle *>(h); }
 
 extern "C" {
 
+int ref_groupJoin(void *h, void *leader) {
+  Oracle *o = O(h), *l = O(leader);
+  if (o->group) return REF_E_INVALID;
+  if (!l->group) l->group = std::make_shared<std::vector<Oracle *>>(1, l);
+  if (o != l) {
+    l->group->push_back(o);
+    o->group = l->group;
+    o->hostp = l->hostp;
+  }
+  return REF_OK;
+}
+
 void *ref_create(unsigned flags) {
   Oracle *o = new Oracle();
   o->flags = flags;
   return o;
 }
-void ref_destroy(void *h) { delete O(h); }
+void ref_destroy(void *h) {
+  Oracle *o = O(h);
+  if (o->group) {  // leave the group (destroy the members before the leader, whose host they share)
+    auto &g = *o->group;
+    g.erase(std::remove(g.begin(), g.end(), o), g.end());
+  }
+  delete o;
+}
 
 int ref_declareAlloc(void *h, uint64_t base, uint64_t size) {
   return O(h)->declare(base, size, false, false, nullptr);
@@ -488,8 +534,8 @@ int ref_undeclare(void *h, uint64_t base) {
   return REF_OK;
 }
 
-int ref_hostWrite(void *h, uint64_t a, const void *s, uint64_t n) { O(h)->host.write(a, s, n); return 0; }
-int ref_hostRead(void *h, uint64_t a, void *d, uint64_t n) { O(h)->host.read(a, d, n); return 0; }
+int ref_hostWrite(void *h, uint64_t a, const void *s, uint64_t n) { O(h)->host().write(a, s, n); return 0; }
+int ref_hostRead(void *h, uint64_t a, void *d, uint64_t n) { O(h)->host().read(a, d, n); return 0; }
 int ref_devWrite(void *h, uint64_t a, const void *s, uint64_t n) { O(h)->dev.write(a, s, n); return 0; }
 int ref_devRead(void *h, uint64_t a, void *d, uint64_t n) { O(h)->dev.read(a, d, n); return 0; }
 

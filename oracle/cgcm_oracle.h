@@ -59,9 +59,13 @@ typedef struct {
   uint64_t h2d_units, h2d_bytes, d2h_units, d2h_bytes;
   uint64_t activations, frees;
   uint64_t fwd_translations, rev_translations, null_slots, passthrough;
+  uint64_t peer_units, peer_bytes;  /* NEXT-3: activations copied from a group peer's device copy */
 } ref_stats_t;
 
 void *ref_create(unsigned flags);
+/* NEXT-3 coherence group: h joins the group of `leader` (which may be h itself: a group of one); the
+ * members share one host memory (the leader's) and each keeps its own device, table and epochs. */
+int ref_groupJoin(void *h, void *leader);
 void ref_destroy(void *h);
 
 int ref_declareAlloc(void *h, uint64_t base, uint64_t size);

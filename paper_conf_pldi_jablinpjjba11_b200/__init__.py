@@ -41,7 +41,8 @@ STAT_FIELDS = ["h2d_units", "h2d_bytes", "d2h_units", "d2h_bytes", "activations"
 class Stats(C.Structure):
     _fields_ = [(f, C.c_uint64) for f in STAT_FIELDS] + [
         ("fwd_kernel_ms", C.c_double), ("rev_kernel_ms", C.c_double), ("fwd_kernel_calls", C.c_uint64),
-        ("rev_kernel_calls", C.c_uint64), ("fwd_kernel_slots", C.c_uint64), ("rev_kernel_slots", C.c_uint64)]
+        ("rev_kernel_calls", C.c_uint64), ("fwd_kernel_slots", C.c_uint64), ("rev_kernel_slots", C.c_uint64),
+        ("peer_units", C.c_uint64), ("peer_bytes", C.c_uint64), ("peer_memcpy_calls", C.c_uint64)]
 
 
 class IndexInfo(C.Structure):
@@ -105,6 +106,8 @@ def lib():
             "cgcm_dumpExtents": (i, [C.c_void_p, C.c_size_t, C.POINTER(C.c_size_t)]),
             "cgcm_storageInfo": (i, [C.POINTER(StorageInfo)]),
             "cgcm_launchGlue": (i, [C.c_void_p, C.c_size_t, C.c_void_p, C.c_size_t, C.c_uint64, C.c_void_p]),
+            "cgcm_groupCreate": (i, [C.POINTER(C.c_void_p)]), "cgcm_groupJoin": (i, [C.c_void_p]),
+            "cgcm_groupLeave": (i, []), "cgcm_groupDestroy": (i, [C.c_void_p]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -141,6 +144,19 @@ def samples():
 
 def _u64(xs) -> np.ndarray:
     return np.ascontiguousarray(np.asarray(xs, dtype=np.uint64))
+
+
+def group_create():
+    """A new coherence group (NEXT-3); contexts join it with Context.groupJoin."""
+    g = C.c_void_p()
+    s = lib().cgcm_groupCreate(C.byref(g))
+    if s != OK:
+        raise CgcmError(f"groupCreate: {strerror(s)}")
+    return g.value
+
+
+def group_destroy(g) -> int:
+    return lib().cgcm_groupDestroy(g)
 
 
 class Context:
@@ -309,7 +325,7 @@ class Context:
         self.L.cgcm_stats(C.byref(st))
         d = {f: getattr(st, f) for f in STAT_FIELDS}
         for f in ("fwd_kernel_ms", "rev_kernel_ms", "fwd_kernel_calls", "rev_kernel_calls", "fwd_kernel_slots",
-                  "rev_kernel_slots"):
+                  "rev_kernel_slots", "peer_units", "peer_bytes", "peer_memcpy_calls"):
             d[f] = getattr(st, f)
         return d
 
@@ -337,6 +353,15 @@ class Context:
         if s != OK:
             raise CgcmError(f"indexInfo: {strerror(s)}")
         return {f: getattr(ii, f) for f, _ in IndexInfo._fields_}
+
+    # ---- coherence groups (NEXT-3) ----
+    def groupJoin(self, group) -> int:
+        self.make_current()
+        return self.L.cgcm_groupJoin(group)
+
+    def groupLeave(self) -> int:
+        self.make_current()
+        return self.L.cgcm_groupLeave()
 
     # ---- glue kernels (NEXT-4) ----
     GLUE = dict(MOVI=1, ADD=2, ADDI=3, SUB=4, MUL=5, FADD=6, FSUB=7, FMUL=8, FDIV=9, LD=10, ST=11, BNZ=12, HALT=13)

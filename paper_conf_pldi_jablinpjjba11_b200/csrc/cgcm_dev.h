@@ -279,6 +279,8 @@ void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n
 void launch_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
                          cudaStream_t s);
 void launch_rebase_epochs(TableDev tab, int n, uint32_t cur, cudaStream_t s);
+// out[i] = st[idx[i]] (epoch | extent | flags) of n units (NEXT-3 peer-source queries)
+void launch_gather_state(TableDev tab, const uint32_t *idx, int n, uint64_t *out, cudaStream_t s);
 // add every deferred reference recorded in a shadow's n unit words to rc (they become ordinary references)
 void launch_materialise(const uint32_t *shadow_units, uint64_t n, int32_t *rc, cudaStream_t s);
 // small host<->device transfers by a kernel through mapped pinned memory instead of a DMA: a copy

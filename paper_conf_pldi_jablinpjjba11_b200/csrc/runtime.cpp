@@ -208,8 +208,16 @@ struct IndexBufs {
   }
 };
 
+struct Context;
+// NEXT-3 coherence group (include/cgcm.h): the member contexts in join order
+struct Group {
+  std::mutex mu;
+  std::vector<Context *> members;
+};
+
 struct Context {
   int device = 0;
+  Group *group = nullptr;
   cudaStream_t main = nullptr, copy = nullptr;
   bool own_streams = false;
   void *own_arena = nullptr;
@@ -974,10 +982,20 @@ struct Context {
     e = evpool[i];
     return CGCM_OK;
   }
+  // ---- NEXT-3: coherence-group peers as copy sources ------------------------------------------
+  struct PeerSrc {
+    Context *ctx = nullptr;  // null: the host
+    uint64_t src = 0;        // the peer's device copy
+  };
+  int peer_sources(const std::vector<uint32_t> &units, std::vector<PeerSrc> &out);
+  int copy_in_with_peers(const std::vector<uint32_t> &units, const std::vector<PeerSrc> &peer, uint64_t bytes);
+  cudaEvent_t ev_peer = nullptr;
+  DevBuf peer_idx, peer_state;
+
   // pack_ev (optional): one event per pack (h2d_out entry), recorded on the copy stream after its copy;
   // the main stream then does NOT wait for the copies -- the caller waits per pack (transfer overlap)
   int activate_units(const std::vector<uint32_t> &units, std::vector<std::pair<uint64_t, uint64_t>> *h2d_out,
-                     std::vector<cudaEvent_t> *pack_ev = nullptr) {
+                     std::vector<cudaEvent_t> *pack_ev = nullptr, bool allow_peer = false) {
     Trace trace_("activate_units");
     if (units.empty()) return CGCM_OK;
     const uint64_t PACK_SPAN = 64ull << 20, GAPMAX = 64ull << 10, PACK_MIN = 256ull << 10;
@@ -1061,6 +1079,10 @@ struct Context {
     CK(cudaGetLastError());
     CK(cudaEventRecord(ev_copy, main));  // the copies wait for everything the main stream did before
     CK(cudaStreamWaitEvent(copy, ev_copy, 0));
+    // NEXT-3 (A31): units a group peer holds active and dirty are copied from its device copy
+    std::vector<PeerSrc> peer;
+    if (allow_peer && group) CKS(peer_sources(units, peer));
+    if (!peer.empty()) return copy_in_with_peers(units, peer, bytes);
     auto mark = [&]() -> int {
       if (!pack_ev) return CGCM_OK;
       cudaEvent_t e;
@@ -1319,7 +1341,7 @@ struct Context {
     if (lcs[0] > 0) {
       std::vector<uint32_t> units;
       CKS(sorted_units(act_list, lcs[0], units));
-      int r = activate_units(units, nullptr);
+      int r = activate_units(units, nullptr, nullptr, true);
       if (r != CGCM_OK) {
         CKS(undo_deferred());
         CKS(undo_map(F, R));
@@ -1612,6 +1634,128 @@ struct Context {
   }
 };
 
+// The state words (epoch | extent | flags) of units idx[] of a peer context, read on its device.
+int Context::peer_sources(const std::vector<uint32_t> &units, std::vector<PeerSrc> &out) {
+  std::vector<Context *> members;
+  {
+    std::lock_guard<std::mutex> g(group->mu);
+    members = group->members;
+  }
+  out.assign(units.size(), PeerSrc());
+  bool any = false;
+  std::vector<size_t> todo(units.size());
+  for (size_t q = 0; q < units.size(); ++q) todo[q] = q;
+  for (Context *c : members) {
+    if (c == this || todo.empty()) continue;
+    std::lock_guard<std::recursive_mutex> lk(c->mu);
+    if (cudaSetDevice(c->device) != cudaSuccess) return CGCM_E_CUDA;
+    int r = c->ensure_table();
+    std::vector<uint32_t> cidx;
+    std::vector<size_t> which;
+    if (r == CGCM_OK)
+      for (size_t q : todo) {
+        const uint32_t x = units[q];
+        auto it = c->reg.find(ubase[x]);
+        if (it != c->reg.end() && it->second.size == usize[x] && it->second.idx >= 0) {
+          cidx.push_back((uint32_t)it->second.idx);
+          which.push_back(q);
+        }
+      }
+    std::vector<uint64_t> stw;
+    if (r == CGCM_OK && !cidx.empty()) {
+      r = c->upload(c->peer_idx, cidx);
+      if (r == CGCM_OK) r = c->dalloc(c->peer_state, 8 * cidx.size() + 64);
+      if (r == CGCM_OK) {
+        launch_gather_state(c->tab(), c->peer_idx.as<uint32_t>(), (int)cidx.size(), c->peer_state.as<uint64_t>(),
+                            c->main);
+        c->st.kernel_launches += 1;
+        r = c->download(stw, c->peer_state, cidx.size());
+      }
+    }
+    if (r == CGCM_OK && !stw.empty()) {
+      const uint32_t cur = c->rel_epoch(c->epoch);
+      std::vector<size_t> left;
+      size_t k = 0;
+      for (size_t q : todo) {
+        if (k < which.size() && which[k] == q) {
+          const uint64_t w = stw[k];
+          const uint32_t fl = hot_flags(w);
+          const uint32_t ci = cidx[k];
+          ++k;
+          // active, holding a copy, writable, and dirty: c launched since the unit became coherent there
+          if ((fl & UF_ACTIVE) && (fl & UF_STORAGE) && !(fl & UF_READONLY) && st_epoch(w) != cur && c->udev[ci]) {
+            out[q].ctx = c;
+            out[q].src = c->udev[ci];
+            any = true;
+            continue;
+          }
+        }
+        left.push_back(q);
+      }
+      todo.swap(left);
+    }
+    if (r == CGCM_OK && any) {  // the copies come after the GPU functions already queued on c
+      if (!c->ev_peer && cudaEventCreateWithFlags(&c->ev_peer, cudaEventDisableTiming) != cudaSuccess) r = CGCM_E_CUDA;
+      if (r == CGCM_OK && cudaEventRecord(c->ev_peer, c->main) != cudaSuccess) r = CGCM_E_CUDA;
+    }
+    if (cudaSetDevice(device) != cudaSuccess) return CGCM_E_CUDA;
+    if (r != CGCM_OK) return r;
+    if (any && out.size() && c->ev_peer) CK(cudaStreamWaitEvent(copy, c->ev_peer, 0));
+  }
+  if (!any) out.clear();
+  return CGCM_OK;
+}
+
+// The copy-in of an activation where some units come from group peers: host-sourced units by runs of
+// host-adjacent units (mirrored extents), peer-sourced units by runs contiguous on both sides.
+int Context::copy_in_with_peers(const std::vector<uint32_t> &units, const std::vector<PeerSrc> &peer,
+                                uint64_t bytes) {
+  size_t i = 0;
+  uint64_t pu = 0, pb = 0;
+  while (i < units.size()) {
+    const uint32_t x0 = units[i];
+    size_t j = i + 1;
+    uint64_t end = ubase[x0] + usize[x0];
+    if (!peer[i].ctx) {
+      while (j < units.size() && !peer[j].ctx && ubase[units[j]] == end &&
+             udev[units[j]] == udev[x0] + (ubase[units[j]] - ubase[x0])) {
+        end += usize[units[j]];
+        ++j;
+      }
+      CKS(copy_run(udev[x0], ubase[x0], end - ubase[x0], true, units, i, j, copy));
+      st.h2d_units += j - i;
+      for (size_t q = i; q < j; ++q) st.h2d_bytes += usize[units[q]];
+    } else {
+      Context *c = peer[i].ctx;
+      while (j < units.size() && peer[j].ctx == c && ubase[units[j]] == end &&
+             udev[units[j]] == udev[x0] + (ubase[units[j]] - ubase[x0]) &&
+             peer[j].src == peer[i].src + (ubase[units[j]] - ubase[x0])) {
+        end += usize[units[j]];
+        ++j;
+      }
+      const uint64_t n = end - ubase[x0];
+      if (c->device == device)
+        CK(cudaMemcpyAsync(reinterpret_cast<void *>(udev[x0]), reinterpret_cast<const void *>(peer[i].src), n,
+                           cudaMemcpyDeviceToDevice, copy));
+      else  // NVLink peer copy
+        CK(cudaMemcpyPeerAsync(reinterpret_cast<void *>(udev[x0]), device, reinterpret_cast<const void *>(peer[i].src),
+                               c->device, n, copy));
+      st.peer_memcpy_calls += 1;
+      pu += j - i;
+      for (size_t q = i; q < j; ++q) pb += usize[units[q]];
+    }
+    i = j;
+  }
+  st.peer_units += pu;
+  st.peer_bytes += pb;
+  (void)bytes;
+  CK(cudaEventRecord(ev_copy, copy));
+  CK(cudaStreamWaitEvent(main, ev_copy, 0));
+  st.activations += units.size();
+  rev_dirty = true;
+  return CGCM_OK;
+}
+
 // ---------------------------------------------------------------------------------------------
 std::mutex g_ctx_mu;
 std::unordered_set<Context *> g_contexts;
@@ -1759,9 +1903,48 @@ int cgcm_init(int device, void *dev_arena, size_t arena_bytes, void *main_stream
   return C->ensure_table();
 }
 
+int cgcm_groupCreate(void **group_out) {
+  if (!group_out) return CGCM_E_INVALID;
+  *group_out = new Group();
+  return CGCM_OK;
+}
+int cgcm_groupJoin(void *group) {
+  CTXM();
+  if (!group || C->group) return CGCM_E_INVALID;
+  Group *g = static_cast<Group *>(group);
+  std::lock_guard<std::mutex> lk(g->mu);
+  g->members.push_back(C);
+  C->group = g;
+  return CGCM_OK;
+}
+static int group_leave(Context *C) {
+  if (!C->group) return CGCM_E_INVALID;
+  Group *g = C->group;
+  std::lock_guard<std::mutex> lk(g->mu);
+  g->members.erase(std::remove(g->members.begin(), g->members.end(), C), g->members.end());
+  C->group = nullptr;
+  return CGCM_OK;
+}
+int cgcm_groupLeave(void) {
+  CTX();
+  return group_leave(C);
+}
+int cgcm_groupDestroy(void *group) {
+  if (!group) return CGCM_E_INVALID;
+  Group *g = static_cast<Group *>(group);
+  {
+    std::lock_guard<std::mutex> lk(g->mu);
+    if (!g->members.empty()) return CGCM_E_BUSY;
+  }
+  delete g;
+  return CGCM_OK;
+}
+
 int cgcm_finalize(void) {
   Context *C = tl_ctx;
   if (!C) return CGCM_E_NOCTX;
+  if (C->group) group_leave(C);
+  if (C->ev_peer) cudaEventDestroy(C->ev_peer);
   {
     std::lock_guard<std::mutex> g(g_ctx_mu);
     g_contexts.erase(C);

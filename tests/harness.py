@@ -12,7 +12,7 @@ import ctypes
 import numpy as np
 
 COMPARED_STATS = ["h2d_units", "h2d_bytes", "d2h_units", "d2h_bytes", "activations", "frees",
-                  "fwd_translations", "rev_translations", "null_slots", "passthrough"]
+                  "fwd_translations", "rev_translations", "null_slots", "passthrough", "peer_units", "peer_bytes"]
 
 
 def host_read(addr: int, n: int) -> bytes:
@@ -34,9 +34,28 @@ class HostBuf:
         self.addr = self.arr.ctypes.data
 
 
+class _Current:
+    """A context proxy that makes the context current before every use (several contexts driven from
+    one thread: coherence groups, NEXT-3)."""
+
+    def __init__(self, ctx):
+        object.__setattr__(self, "_ctx", ctx)
+
+    def __getattr__(self, name):
+        ctx = self._ctx
+        ctx.make_current()
+        v = getattr(ctx, name)
+        if callable(v):
+            def call(*a, **k):
+                ctx.make_current()
+                return v(*a, **k)
+            return call
+        return v
+
+
 class Pair:
-    def __init__(self, ctx, oracle):
-        self.g = ctx
+    def __init__(self, ctx, oracle, switch=False):
+        self.g = _Current(ctx) if switch else ctx
         self.o = oracle
         self.units = {}   # base -> size
 
