@@ -7,7 +7,7 @@
 set -u
 R=${1:-r02}
 mkdir -p gpurun_out/$R
-CASES="tests/test_gpu_parity.py::test_scalar_map_unmap_release tests/test_gpu_parity.py::test_mapArray_roundtrip_permutation tests/test_gpu_parity.py::test_random_device_slices tests/test_gpu_deferred.py tests/test_gpu_glue.py tests/test_gpu_group.py::test_handoff_through_a_dirty_peer"
+CASES="tests/test_gpu_parity.py::test_scalar_map_unmap_release tests/test_gpu_parity.py::test_mapArray_roundtrip_permutation tests/test_gpu_parity.py::test_random_device_slices[shadow-8] tests/test_gpu_deferred.py::test_deferred_released_by_matching_unmap[shadow] tests/test_gpu_deferred.py::test_deferred_slots_rewritten_by_gpu[shadow] tests/test_gpu_glue.py tests/test_gpu_group.py::test_handoff_through_a_dirty_peer"
 for tool in memcheck racecheck synccheck; do
   extra=""
   [ "$tool" = memcheck ] && extra="--leak-check full"
