@@ -1361,7 +1361,7 @@ static int launch_unmap_sh(const SlotArgs &a, int nsm, cudaStream_t s) {
 #ifdef CGCM_FWD_LEAN_THREADS
 constexpr int FWD_LEAN_THREADS = CGCM_FWD_LEAN_THREADS;
 #else
-constexpr int FWD_LEAN_THREADS = 640;  // two chunks in flight per thread need ~94 registers
+constexpr int FWD_LEAN_THREADS = 768;  // measured: 768 > 640 > 512 (profiles/r02f_ab.log)
 #endif
 
 __device__ __forceinline__ uint32_t warp_or(uint32_t v) { return __reduce_or_sync(0xffffffffu, v); }
@@ -1417,84 +1417,88 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
   const uint32_t pmask = (1u << P) - 1u;
   const int32_t inc = sg.inc;
   const bool defer = a.defer != 0;
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x, nch = a.nchunks;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   unsigned c_nulls = 0, c_hits = 0, c_miss = 0, c_pend = 0, c_tr = 0;
-  // valid slots of chunk c: both, except in the segment's first and last chunks
-  auto valid_exact = [&](uint64_t c) -> uint32_t {
-    const uint64_t a0 = a0base + 16ull * c;
-    return (a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u);
-  };
-  const uint32_t v_first = valid_exact(0), v_last = valid_exact(nch - 1);
-  auto valid_of = [&](uint64_t c) -> uint32_t {
-    return c < nch ? (c == 0 ? v_first : (c == nch - 1 ? v_last : 3u)) : 0u;
-  };
 
-  // one chunk in flight: its slot values, validity and page-entry gathers (front half of a1); beyond
-  // the last page: the tail of the segment's last unit (jt, decided by its end, A7) or -1
-  struct Fr {
-    uint64_t p[2];
+  auto valid_of = [&](uint64_t c) -> uint32_t {
+    const uint64_t a0 = a0base + 16ull * c;
+    return c < a.nchunks ? ((a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u)) : 0u;
+  };
+  // front half of a1 for the two slots of a chunk: the page of each, and its entry gather issued
+  // (ok); beyond the last page, the tail of the segment's last unit (jt, decided by its end, A7) or -1
+  struct Front {
     uint64_t ew[2][4];
     uint32_t poff[2];
     int jt[2];
-    uint32_t valid;
     bool ok[2];
   };
-  auto front = [&](const uint64_t v[2], uint64_t c, Fr &f) {
-    f.valid = valid_of(c);
+  auto front = [&](const uint64_t p[2], uint32_t valid, Front &f) {
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      const uint64_t p = v[m];
-      f.p[m] = p;
-      const bool look = ((f.valid >> m) & 1) && p != 0 && p >= S0;
-      const uint64_t rel = p - S0;
+      const bool look = ((valid >> m) & 1) && p[m] != 0 && p[m] >= S0;
+      const uint64_t rel = p[m] - S0;
       const uint64_t pg = rel >> P;
       f.ok[m] = look && pg < npages;
       f.poff[m] = (uint32_t)rel & pmask;
-      f.jt[m] = look && !f.ok[m] && p <= Send ? (int)lastu : -1;
+      f.jt[m] = look && !f.ok[m] && p[m] <= Send ? (int)lastu : -1;
+      f.ew[m][0] = f.ew[m][1] = f.ew[m][2] = f.ew[m][3] = 0;
       if (f.ok[m])  // one LDG.256, not allocated in L1
         asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
                      : "=l"(f.ew[m][0]), "=l"(f.ew[m][1]), "=l"(f.ew[m][2]), "=l"(f.ew[m][3])
-                     : "l"(ent + 8ull * (uint32_t)pg), "l"(pol_t));
+                     : "l"(ent + 8 * pg), "l"(pol_t));
     }
   };
-  // back half of a1 + a2 for the chunk whose front is f
-  auto finish = [&](uint64_t cb, const Fr &f) {
+
+  // software pipeline: slot values two chunks ahead, page-entry gathers one chunk ahead
+  const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  uint64_t cv[2] = {0, 0}, nv[2] = {0, 0}, nnv[2] = {0, 0};
+  if (c_first < a.nchunks) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c_first), pol_s, cv[0], cv[1]);
+  if (c_first + stride < a.nchunks)
+    ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, nv[0], nv[1]);
+  Front fc, fn;
+  front(cv, valid_of(c_first), fc);
+  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
     const uint64_t c = cb + lane;
-    const uint32_t valid = f.valid;
+    if (c + 2 * stride < a.nchunks)
+      ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, nnv[0], nnv[1]);
+    front(nv, valid_of(c + stride), fn);  // the next chunk's entries are in flight while this one finishes
+    const uint64_t a0 = a0base + 16ull * c;
+    const uint32_t valid = valid_of(c);
+
+    // decode: j = j0 + #{offsets <= p - A}; the page's j0 is decided by its end, others by base + size
     int j[2];
     bool k0[2];
     uint64_t key[2];
     uint32_t cw[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      j[m] = f.jt[m];
+      j[m] = fc.jt[m];
       k0[m] = true;
       key[m] = 0;
-      if (f.ok[m]) {  // j = j0 + #{offsets <= p - A}; j0 is decided by its end, the others by base + size
-        const uint32_t j0 = (uint32_t)f.ew[m][0], w1 = (uint32_t)(f.ew[m][0] >> 32);
+      if (fc.ok[m]) {
+        const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
         const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
-        const uint32_t r = min(f.poff[m], PD_PAD - 1u);
-        uint32_t k, off = 0;
+        const uint32_t r = min(fc.poff[m], PD_PAD - 1u);
+        uint32_t k, off;
         if (cnt <= (uint32_t)PD_K) {
           const uint32_t r2 = r | (r << 16);
           const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
-          k = le4(f.ew[m][1], r4) + le4(f.ew[m][2], r4) + le4(f.ew[m][3], r4);
-          if (k) off = off_at(f.ew[m][1], f.ew[m][2], f.ew[m][3], k - 1);
+          k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
+          off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
         } else {
-          const uint64_t ko = pd_crowded(a.pd.ovf, (uint32_t)f.ew[m][1], cnt, r);
+          const uint64_t ko = pd_crowded(a.pd.ovf, (uint32_t)fc.ew[m][1], cnt, r);
           k = (uint32_t)ko;
           off = (uint32_t)(ko >> 32);
         }
         k0[m] = k == 0;
-        j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && f.poff[m] < end0 ? (int)j0 : -1);
-        key[m] = f.p[m] - f.poff[m] + off;  // the candidate's base (A + offset)
+        j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
+        key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
       }
+      cw[m] = 0;
       if (j[m] >= 0)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
         asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
-      else
-        cw[m] = 0;
     }
-    uint64_t outv[2] = {f.p[0], f.p[1]};
+    uint64_t outv[2] = {cv[0], cv[1]};
     uint32_t wrote = 0, su[2];
     bool act[2];
 #pragma unroll
@@ -1504,8 +1508,8 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
       const uint64_t hw = (cw[m] & HOTC_ESC) && look ? ld_u64_hot(a.tab.hot + j[m], pol_t) : hot_of_hotc(cw[m]);
       uint64_t sz = hot_size32(hw);
       if (look && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
-      const bool hit = look && (k0[m] || f.p[m] - key[m] <= sz);  // A7: p - base <= size
-      const bool nul = vm && f.p[m] == 0;
+      const bool hit = look && (k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
+      const bool nul = vm && cv[m] == 0;
       c_nulls += nul;
       c_hits += hit;
       c_miss += vm && !nul && !hit;
@@ -1521,7 +1525,7 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
       }
       if (hit && (fl & UF_STORAGE)) {
         const uint32_t e = hot_ext(hw);
-        outv[m] = f.p[m] + (ES ? s_ext[e] : a.tab.ext_delta[e]);  // Alg. 1: devptr + (ptr - base)
+        outv[m] = cv[m] + (ES ? s_ext[e] : a.tab.ext_delta[e]);  // Alg. 1: devptr + (ptr - base)
         wrote |= 1u << m;
       } else {
         c_pend += hit;  // activated by this call: completed after the allocation
@@ -1537,19 +1541,18 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
       }
     }
     // the shadow (CPU pointer, unit) and the slots
-    const uint64_t a0 = a0base + 16ull * c;
     const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
     if (valid == 3u) {
       st_stream2(reinterpret_cast<void *>(a0), pol_s, outv[0], outv[1]);
       if (!(i0 & 1)) {
-        st_stream2(shp + i0, pol_s, f.p[0], f.p[1]);
+        st_stream2(shp + i0, pol_s, cv[0], cv[1]);
         asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1,%2}, %3;" ::"l"(shu + i0), "r"(su[0]),
                      "r"(su[1]), "l"(pol_s)
                      : "memory");
       } else {
 #pragma unroll
         for (int m = 0; m < 2; ++m) {
-          shp[i0 + m] = f.p[m];
+          shp[i0 + m] = cv[m];
           shu[i0 + m] = su[m];
         }
       }
@@ -1558,7 +1561,7 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
       for (int m = 0; m < 2; ++m)
         if ((valid >> m) & 1) {
           st_stream1(reinterpret_cast<void *>(a0 + 8ull * m), pol_s, outv[m]);
-          shp[i0 + m] = f.p[m];
+          shp[i0 + m] = cv[m];
           shu[i0 + m] = su[m];
         }
     }
@@ -1567,33 +1570,13 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
       const uint32_t w0 = warp_or(lane < 16 ? b : 0u), w1 = warp_or(lane < 16 ? 0u : b);
       const uint64_t wi = cb >> 4;
       if (lane == 0) a.hitmask[wi] = w0;
-      else if (lane == 16 && cb + 16 < nch) a.hitmask[wi + 1] = w1;
+      else if (lane == 16 && cb + 16 < a.nchunks) a.hitmask[wi + 1] = w1;
     }
-  };
-  auto load_vals = [&](uint64_t c, uint64_t v[2]) {
-    v[0] = v[1] = 0;
-    if (c < nch) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c), pol_s, v[0], v[1]);
-  };
-
-  // software pipeline, unrolled twice so that nothing is copied between stages: while chunk t is
-  // finished, the page entries of chunk t+1 are in flight and the slot values of chunk t+2 are loading
-  const uint64_t cf = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  uint64_t vA[2], vB[2];
-  Fr fA, fB;
-  load_vals(cf, vA);
-  load_vals(cf + stride, vB);
-  front(vA, cf, fA);
-  uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
-  while (cb < nch) {
-    load_vals(cb + lane + 2 * stride, vA);
-    front(vB, cb + lane + stride, fB);
-    finish(cb, fA);
-    cb += stride;
-    if (cb >= nch) break;
-    load_vals(cb + lane + 2 * stride, vB);
-    front(vA, cb + lane + stride, fA);
-    finish(cb, fB);
-    cb += stride;
+    cv[0] = nv[0];
+    cv[1] = nv[1];
+    nv[0] = nnv[0];
+    nv[1] = nnv[1];
+    fc = fn;
   }
   flush_count(&a.st->nulls, (unsigned long long)c_nulls * (unsigned)inc);  // inc = k: k sequential calls
   flush_count(&a.st->hits, (unsigned long long)c_hits * (unsigned)inc);

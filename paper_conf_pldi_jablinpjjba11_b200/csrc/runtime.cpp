@@ -20,6 +20,7 @@
 #include <cstdio>
 #include <cstring>
 #include <map>
+#include <memory>
 #include <mutex>
 #include <thread>
 #include <string>
@@ -1008,6 +1009,7 @@ struct Context {
     };
     std::vector<Pack> packs;
     uint64_t bytes = 0;
+    auto tr_packs = std::make_unique<Trace>("  act:packs");
     for (size_t i = 0; i < units.size(); ++i) {
       uint64_t b = ubase[units[i]], sz = usize[units[i]];
       bytes += sz;
@@ -1022,6 +1024,8 @@ struct Context {
         packs.push_back({i, i + 1, b, b + sz, g, false, -1, 0});
       }
     }
+    tr_packs.reset();
+    auto tr_alloc = std::make_unique<Trace>("  act:alloc+mirrors");
     std::vector<uint64_t> devbases(units.size());
     std::vector<int64_t> created;
     for (auto &P : packs) {
@@ -1067,6 +1071,8 @@ struct Context {
       }
       runs[P.run].live += (int64_t)(P.j - P.i);
     }
+    tr_alloc.reset();
+    auto tr_up = std::make_unique<Trace>("  act:exts+upload+set_ext");
     std::vector<uint32_t> exts(units.size());
     for (size_t q = 0; q < units.size(); ++q) exts[q] = (uint32_t)urun[units[q]];
     if (runs.size() > EXT_MASK) return CGCM_E_NOMEM;  // 2^24 live extents
@@ -1077,6 +1083,8 @@ struct Context {
                    (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
+    tr_up.reset();
+    Trace tr_copy("  act:copies");
     CK(cudaEventRecord(ev_copy, main));  // the copies wait for everything the main stream did before
     CK(cudaStreamWaitEvent(copy, ev_copy, 0));
     // NEXT-3 (A31): units a group peer holds active and dirty are copied from its device copy
