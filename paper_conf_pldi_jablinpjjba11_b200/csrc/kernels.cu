@@ -1960,6 +1960,174 @@ void launch_sort_keys(void *temp, size_t temp_bytes, const uint32_t *kin, uint32
 }
 
 // -------------------------------------------------------------------------------------------------
+// Transfer planning on the device (activation packs, copy-back runs): segmented scans over the sorted
+// unit list, so that the host handles one descriptor per DMA instead of one entry per unit.
+// -------------------------------------------------------------------------------------------------
+size_t plan_temp_bytes(int n) {
+  size_t a = 0;
+  cub::DeviceScan::InclusiveSum(nullptr, a, (const uint32_t *)nullptr, (uint32_t *)nullptr, n);
+  return a;
+}
+__device__ __forceinline__ uint64_t unit_size(const TableDev &t, uint32_t u) {
+  const uint32_t s = hot_size32(t.hot[u]);
+  return s == BIG_SIZE ? t.size64[u] : s;
+}
+__global__ void k_pack_flags(const uint32_t *S, int n, TableDev tab, uint64_t gapmax, int window, uint32_t *F,
+                             uint32_t *G, unsigned long long *cnt) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  uint64_t sz = 0;
+  bool glob = false;
+  if (i < n) {
+    const uint32_t u = S[i];
+    const uint64_t b = tab.base[u];
+    sz = unit_size(tab, u);
+    glob = hot_flags(tab.hot[u]) & UF_GLOBAL;
+    uint32_t f = 1, g = 0;
+    if (i > 0) {
+      const uint32_t v = S[i - 1];
+      const uint64_t e = tab.base[v] + unit_size(tab, v);
+      const bool gv = hot_flags(tab.hot[v]) & UF_GLOBAL;
+      f = (glob || gv || b < e || b - e > gapmax || (b >> window) != (tab.base[v] >> window)) ? 1u : 0u;
+      g = (!f && b != e) ? 1u : 0u;
+    }
+    F[i] = f;
+    G[i] = g;
+  }
+  // bytes and globals of the whole list: one atomic per warp
+  unsigned long long ws = sz, wg = glob ? 1 : 0;
+  for (int o = 16; o; o >>= 1) {
+    ws += __shfl_xor_sync(0xffffffffu, ws, o);
+    wg += __shfl_xor_sync(0xffffffffu, wg, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (ws) atomicAdd(&cnt[2], ws);
+    if (wg) atomicAdd(&cnt[1], wg);
+  }
+}
+__global__ void k_pack_first(const uint32_t *S, int n, TableDev tab, const uint32_t *F, const uint32_t *pid,
+                             PackDesc *packs) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n || !F[i]) return;
+  PackDesc &P = packs[pid[i] - 1];
+  P.first = (uint32_t)i;
+  P.h0 = tab.base[S[i]];
+}
+__global__ void k_pack_last(const uint32_t *S, int n, TableDev tab, const uint32_t *F, const uint32_t *pid,
+                            const uint32_t *gscan, PackDesc *packs) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  if (i + 1 < n && !F[i + 1]) return;
+  PackDesc &P = packs[pid[i] - 1];
+  P.last = (uint32_t)i;
+  P.h1 = tab.base[S[i]] + unit_size(tab, S[i]);
+  P.gaps = gscan[i] - gscan[P.first] > 0 ? 1u : 0u;
+  P.pad = 0;
+}
+int launch_plan_packs1(const uint32_t *S, int n, TableDev tab, uint64_t gapmax, int window, uint32_t *F, uint32_t *G,
+                       uint32_t *pid, uint32_t *gscan, unsigned long long *cnt, void *temp, size_t temp_bytes,
+                       cudaStream_t s) {
+  if (n <= 0) return 0;
+  (void)cudaGetLastError();
+  cudaMemsetAsync(cnt, 0, 32, s);
+  const int g = (n + 255) / 256;
+  k_pack_flags<<<g, 256, 0, s>>>(S, n, tab, gapmax, window, F, G, cnt);
+  size_t tb = temp_bytes;
+  cub::DeviceScan::InclusiveSum(temp, tb, F, pid, n, s);
+  tb = temp_bytes;
+  cub::DeviceScan::InclusiveSum(temp, tb, G, gscan, n, s);
+  cudaMemcpyAsync(cnt, pid + (n - 1), 4, cudaMemcpyDeviceToDevice, s);  // cnt[0] (low word) = #packs
+  return (int)cudaGetLastError();
+}
+int launch_plan_packs2(const uint32_t *S, int n, TableDev tab, const uint32_t *F, const uint32_t *pid,
+                       const uint32_t *gscan, PackDesc *packs, cudaStream_t s) {
+  if (n <= 0) return 0;
+  (void)cudaGetLastError();
+  const int g = (n + 255) / 256;
+  k_pack_first<<<g, 256, 0, s>>>(S, n, tab, F, pid, packs);
+  k_pack_last<<<g, 256, 0, s>>>(S, n, tab, F, pid, gscan, packs);
+  return (int)cudaGetLastError();
+}
+__global__ void k_plan_set_ext(const uint32_t *S, int n, const uint32_t *pid, const uint32_t *run, TableDev tab,
+                               uint32_t epoch, int set_epoch) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t u = S[i], p = pid[i] - 1;
+  uint64_t h = tab.hot[u];
+  h = (h & ~(EXT_MASK << ESHIFT)) | ((uint64_t)(run[p] & EXT_MASK) << ESHIFT);
+  h |= (uint64_t)(UF_STORAGE | UF_ACTIVE) << FSHIFT;
+  tab.hot[u] = h;
+  tab.hotc[u] = make_hotc(h);
+  tab.st[u] = make_st(h, set_epoch ? epoch : st_epoch(tab.st[u]));
+}
+void launch_plan_set_ext(const uint32_t *S, int n, const uint32_t *pid, const uint32_t *run, TableDev tab,
+                         uint32_t epoch, int set_epoch, cudaStream_t s) {
+  if (n <= 0) return;
+  (void)cudaGetLastError();
+  k_plan_set_ext<<<(n + 255) / 256, 256, 0, s>>>(S, n, pid, run, tab, epoch, set_epoch);
+}
+
+// copy-back runs: a new run unless the unit directly follows the previous one in index order, starts
+// where it ends on the host, lives in the same (mirrored) extent, and neither is array-mapped
+__global__ void k_cb_flags(const uint32_t *S, int n, TableDev tab, uint32_t *F) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t u = S[i];
+  const uint64_t hu = tab.hot[u];
+  uint32_t f = 1;
+  if (i > 0) {
+    const uint32_t v = S[i - 1];
+    const uint64_t hv = tab.hot[v];
+    const bool arr = (hot_flags(hu) | hot_flags(hv)) & UF_ARRAYMAPPED;
+    f = (arr || u != v + 1 || tab.base[u] != tab.base[v] + unit_size(tab, v) || hot_ext(hu) != hot_ext(hv)) ? 1u : 0u;
+  }
+  F[i] = f;
+}
+__global__ void k_cb_first(const uint32_t *S, int n, TableDev tab, const uint32_t *F, const uint32_t *rid,
+                           CopyRun *runs) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n || !F[i]) return;
+  const uint32_t u = S[i];
+  const uint64_t h = tab.hot[u];
+  CopyRun &R = runs[rid[i] - 1];
+  R.first = (uint32_t)i;
+  R.unit = u;
+  R.arr = (hot_flags(h) & UF_ARRAYMAPPED) ? 1u : 0u;
+  R.host = tab.base[u];
+  R.dev = tab.base[u] + tab.ext_delta[hot_ext(h)];  // Alg. 1's devptr of the run's first unit
+  R.pad = 0;
+}
+__global__ void k_cb_last(const uint32_t *S, int n, TableDev tab, const uint32_t *F, const uint32_t *rid,
+                          CopyRun *runs) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  if (i + 1 < n && !F[i + 1]) return;
+  CopyRun &R = runs[rid[i] - 1];
+  R.last = (uint32_t)i;
+  R.len = tab.base[S[i]] + unit_size(tab, S[i]) - R.host;
+}
+int launch_plan_copyback1(const uint32_t *S, int n, TableDev tab, uint32_t *F, uint32_t *rid, unsigned long long *cnt,
+                          void *temp, size_t temp_bytes, cudaStream_t s) {
+  if (n <= 0) return 0;
+  (void)cudaGetLastError();
+  cudaMemsetAsync(cnt, 0, 32, s);
+  const int g = (n + 255) / 256;
+  k_cb_flags<<<g, 256, 0, s>>>(S, n, tab, F);
+  size_t tb = temp_bytes;
+  cub::DeviceScan::InclusiveSum(temp, tb, F, rid, n, s);
+  cudaMemcpyAsync(cnt, rid + (n - 1), 4, cudaMemcpyDeviceToDevice, s);  // cnt[0] (low word) = #runs
+  return (int)cudaGetLastError();
+}
+int launch_plan_copyback2(const uint32_t *S, int n, TableDev tab, const uint32_t *F, const uint32_t *rid,
+                          CopyRun *runs, cudaStream_t s) {
+  if (n <= 0) return 0;
+  (void)cudaGetLastError();
+  const int g = (n + 255) / 256;
+  k_cb_first<<<g, 256, 0, s>>>(S, n, tab, F, rid, runs);
+  k_cb_last<<<g, 256, 0, s>>>(S, n, tab, F, rid, runs);
+  return (int)cudaGetLastError();
+}
+
+// -------------------------------------------------------------------------------------------------
 // small bookkeeping kernels
 // -------------------------------------------------------------------------------------------------
 __global__ void k_unit_ops(const UnitOp *ops, int n, TableDev tab) {

@@ -265,6 +265,13 @@ struct Context {
 
   // scratch
   DevBuf slowmask, slowcnt, dump_rc, glue_prog, glue_regs, glue_status;
+  // device-side transfer planning (activation packs, copy-back runs) for lists of >= PLAN_MIN units
+  static constexpr size_t PLAN_MIN = 1u << 16;
+  DevBuf plan_S, plan_F, plan_G, plan_pid, plan_gscan, plan_tmp, plan_cnt, plan_desc, plan_run;
+  size_t plan_tb = 0;
+  // the per-unit host mirrors (udev, urun, uarr) are not written by planned activations: stale until
+  // need_mirrors() rebuilds them from the device table (only host paths read them)
+  bool mirror_stale = false;
   DevBuf status, lc, hitmask, act_list, journal, free_list, copy_list, segs, seg0, staging, staging2, staging_cb, points, ptrs, temp;
   DevBuf up_units, up_vals, up_exts, uops;
   HostBuf h_small, h_status, h_list, h_pack[2];
@@ -578,6 +585,7 @@ struct Context {
     Trace trace_("ensure_table");
     if (!table_dirty) return CGCM_OK;
     CKS(materialise_all());  // deferred references name units by their index in the table being replaced
+    CKS(need_mirrors());     // the remap carries the per-unit host mirrors to the new indices
     int n = (int)reg.size();
     // host staging: base[n], size[n], epoch0[n] (u32, relative), old_idx[n], flags[n]
     size_t need = (size_t)n * (8 + 8 + 4 + 4 + 4) + 256;
@@ -998,6 +1006,7 @@ struct Context {
   int activate_units(const std::vector<uint32_t> &units, std::vector<std::pair<uint64_t, uint64_t>> *h2d_out,
                      std::vector<cudaEvent_t> *pack_ev = nullptr, bool allow_peer = false) {
     Trace trace_("activate_units");
+    CKS(need_mirrors());
     if (units.empty()) return CGCM_OK;
     const uint64_t PACK_SPAN = 64ull << 20, GAPMAX = 64ull << 10, PACK_MIN = 256ull << 10;
     struct Pack {
@@ -1127,6 +1136,191 @@ struct Context {
     rev_dirty = true;
     return CGCM_OK;
   }
+  // ---- device-side transfer planning -----------------------------------------------------------
+  int need_mirrors() {
+    if (!mirror_stale) return CGCM_OK;
+    Trace trace_("need_mirrors(sync)");
+    std::vector<uint64_t> hots;
+    CKS(download(hots, hotb, (size_t)U));
+    for (int x = 0; x < U; ++x) {
+      const uint32_t fl = hot_flags(hots[x]);
+      const uint32_t e = hot_ext(hots[x]);
+      if ((fl & UF_STORAGE) && e < runs.size()) {
+        urun[x] = (int64_t)e;
+        udev[x] = ubase[x] - runs[e].delta;
+      } else {
+        urun[x] = -1;
+        udev[x] = 0;
+      }
+      uarr[x] = (fl & UF_ARRAYMAPPED) ? 1 : 0;
+    }
+    mirror_stale = false;
+    return CGCM_OK;
+  }
+  // sort the n unit ids of a device list into plan_S (and size the planning scratch)
+  int plan_sort(const DevBuf &list, size_t n) {
+    plan_tb = std::max(sort_keys_temp_bytes((int)n), plan_temp_bytes((int)n)) + 256;
+    CKS(dalloc(plan_tmp, plan_tb));
+    for (DevBuf *b : {&plan_S, &plan_F, &plan_G, &plan_pid, &plan_gscan}) CKS(dalloc(*b, 4 * n + 64));
+    CKS(dalloc(plan_cnt, 64));
+    launch_sort_keys(plan_tmp.as<void>(), plan_tb, list.as<uint32_t>(), plan_S.as<uint32_t>(), (int)n, main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
+    return CGCM_OK;
+  }
+  // the sorted ids [first, last] of plan_S on the host (fallback paths of one pack / run)
+  int plan_slice(uint32_t first, uint32_t last, std::vector<uint32_t> &out) {
+    DevBuf v;
+    v.addr = plan_S.addr + 4ull * first;
+    v.bytes = 4ull * (last - first + 1);
+    return download(out, v, last - first + 1);
+  }
+  // Activation of n units (a device list) planned on the device: packs of host-adjacent units, one
+  // mirrored extent each, device addresses and extent ids written by a kernel; the host handles one
+  // descriptor per pack (allocation + one DMA).  Globals take the host path.
+  int activate_planned(const DevBuf &list, size_t n) {
+    Trace trace_("activate(planned)");
+    const uint64_t GAPMAX = 64ull << 10;
+    CKS(plan_sort(list, n));
+    int r = launch_plan_packs1(plan_S.as<uint32_t>(), (int)n, tab(), GAPMAX, 26, plan_F.as<uint32_t>(),
+                               plan_G.as<uint32_t>(), plan_pid.as<uint32_t>(), plan_gscan.as<uint32_t>(),
+                               plan_cnt.as<unsigned long long>(), plan_tmp.as<void>(), plan_tb, main);
+    st.kernel_launches += 4;
+    if (r) return CGCM_E_CUDA;
+    std::vector<unsigned long long> cnt;
+    CKS(download(cnt, plan_cnt, 4));
+    const size_t np = (size_t)(cnt[0] & 0xFFFFFFFFull);
+    const uint64_t bytes = cnt[2];
+    if (cnt[1]) {  // globals keep their named regions (A14): the host path
+      std::vector<uint32_t> units;
+      CKS(plan_slice(0, (uint32_t)n - 1, units));
+      return activate_units(units, nullptr, nullptr, true);
+    }
+    CKS(dalloc(plan_desc, sizeof(PackDesc) * np + 64));
+    if (launch_plan_packs2(plan_S.as<uint32_t>(), (int)n, tab(), plan_F.as<uint32_t>(), plan_pid.as<uint32_t>(),
+                           plan_gscan.as<uint32_t>(), plan_desc.as<PackDesc>(), main))
+      return CGCM_E_CUDA;
+    st.kernel_launches += 2;
+    std::vector<PackDesc> packs;
+    CKS(download(packs, plan_desc, np));
+    // device extents, all or nothing
+    std::vector<int64_t> created;
+    std::vector<uint32_t> rid(np);
+    std::vector<uint64_t> dev0(np);
+    for (size_t p = 0; p < np; ++p) {
+      const PackDesc &P = packs[p];
+      const uint64_t need = (P.h0 % 256) + (P.h1 - P.h0) + 1;  // >= 1 byte of slack (A7)
+      const uint64_t a = arena.alloc(need);
+      if (!a) {
+        for (int64_t x : created) drop_run(x);
+        return CGCM_E_NOMEM;
+      }
+      dev0[p] = a + (P.h0 % 256);  // devptr == base (mod 256)
+      const int64_t run = new_run(a, need, P.h0 - dev0[p]);
+      runs[run].live = (int64_t)(P.last - P.first + 1);
+      created.push_back(run);
+      rid[p] = (uint32_t)run;
+    }
+    if (runs.size() > EXT_MASK) {
+      for (int64_t x : created) drop_run(x);
+      return CGCM_E_NOMEM;
+    }
+    CKS(sync_ext());
+    CKS(upload(plan_run, rid));
+    launch_plan_set_ext(plan_S.as<uint32_t>(), (int)n, plan_pid.as<uint32_t>(), plan_run.as<uint32_t>(), tab(),
+                        rel_epoch(epoch), (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(ev_copy, main));
+    CK(cudaStreamWaitEvent(copy, ev_copy, 0));
+    for (size_t p = 0; p < np; ++p) {  // the transfer scheduler: one DMA per pack
+      const PackDesc &P = packs[p];
+      const uint64_t span = P.h1 - P.h0;
+      if (!P.gaps) {
+        cudaError_t e = cudaMemcpyAsync(reinterpret_cast<void *>(dev0[p]), reinterpret_cast<const void *>(P.h0), span,
+                                        cudaMemcpyHostToDevice, copy);
+        if (e == cudaSuccess) {
+          st.h2d_memcpy_calls += 1;
+          continue;
+        }
+        (void)cudaGetLastError();  // e.g. a span across two host allocations: unit by unit below
+      }
+      std::vector<uint32_t> units;
+      CKS(plan_slice(P.first, P.last, units));
+      if (!P.gaps) {
+        CKS(copy_run(dev0[p], P.h0, span, true, units, 0, units.size(), copy));
+        continue;
+      }
+      int k = pack_k;
+      pack_k ^= 1;
+      CK(cudaEventSynchronize(ev_pack[k]));
+      CKS(h_pack[k].ensure(span));
+      gather(units, 0, units.size(), P.h0, h_pack[k].as<char>());
+      CK(cudaMemcpyAsync(reinterpret_cast<void *>(dev0[p]), h_pack[k].p, span, cudaMemcpyHostToDevice, copy));
+      CK(cudaEventRecord(ev_pack[k], copy));
+      st.h2d_memcpy_calls += 1;
+    }
+    CK(cudaEventRecord(ev_copy, copy));
+    CK(cudaStreamWaitEvent(main, ev_copy, 0));
+    st.h2d_units += n;
+    st.h2d_bytes += bytes;
+    st.activations += n;
+    rev_dirty = true;
+    mirror_stale = true;
+    return CGCM_OK;
+  }
+  // Copy-back (Alg. 2's cuMemcpyDtoH) of the n units of a device list: plain units as one DMA per
+  // host-adjacent mirrored run, array-mapped units reverse translated first (A12).  Planned on the
+  // device for long lists.
+  int copy_back_list(const DevBuf &list, size_t n) {
+    if (n == 0) return CGCM_OK;
+    if (n < PLAN_MIN) {
+      std::vector<uint32_t> units;
+      CKS(sorted_units(list, n, units));
+      return copy_back(units);
+    }
+    Trace trace_("copy_back(planned)");
+    CKS(plan_sort(list, n));
+    if (launch_plan_copyback1(plan_S.as<uint32_t>(), (int)n, tab(), plan_F.as<uint32_t>(), plan_pid.as<uint32_t>(),
+                              plan_cnt.as<unsigned long long>(), plan_tmp.as<void>(), plan_tb, main))
+      return CGCM_E_CUDA;
+    st.kernel_launches += 2;
+    std::vector<unsigned long long> cnt;
+    CKS(download(cnt, plan_cnt, 4));
+    const size_t nr = (size_t)(cnt[0] & 0xFFFFFFFFull);
+    CKS(dalloc(plan_desc, sizeof(CopyRun) * nr + 64));
+    if (launch_plan_copyback2(plan_S.as<uint32_t>(), (int)n, tab(), plan_F.as<uint32_t>(), plan_pid.as<uint32_t>(),
+                              plan_desc.as<CopyRun>(), main))
+      return CGCM_E_CUDA;
+    st.kernel_launches += 2;
+    std::vector<CopyRun> rs;
+    CKS(download(rs, plan_desc, nr));
+    std::vector<std::pair<uint32_t, uint64_t>> arr;
+    for (auto &R : rs)
+      if (R.arr) arr.push_back({R.unit, R.dev});
+    CKS(copy_back_arr(arr));  // validated before any plain byte moves
+    for (auto &R : rs) {
+      if (R.arr) continue;
+      cudaError_t e = cudaMemcpyAsync(reinterpret_cast<void *>(R.host), reinterpret_cast<const void *>(R.dev), R.len,
+                                      cudaMemcpyDeviceToHost, copy);
+      if (e != cudaSuccess) {  // a run across two host allocations: unit by unit
+        (void)cudaGetLastError();
+        std::vector<uint32_t> units;
+        CKS(plan_slice(R.first, R.last, units));
+        for (uint32_t x : units)
+          CK(cudaMemcpyAsync(reinterpret_cast<void *>(ubase[x]), reinterpret_cast<const void *>(R.dev + (ubase[x] - R.host)),
+                             usize[x], cudaMemcpyDeviceToHost, copy));
+        st.d2h_memcpy_calls += units.size();
+      } else {
+        st.d2h_memcpy_calls += 1;
+      }
+      st.d2h_units += R.last - R.first + 1;
+      st.d2h_bytes += R.len;
+    }
+    CK(cudaStreamSynchronize(copy));
+    return CGCM_OK;
+  }
+
   // host gather of units [i, j) into staging at their mirrored offsets (base - h0)
   void gather(const std::vector<uint32_t> &units, size_t i, size_t j, uint64_t h0, char *stg) {
     size_t n = j - i;
@@ -1180,6 +1374,7 @@ struct Context {
   // units whose refcount reached 0: free device storage (globals keep theirs), clear flags
   int free_units(const std::vector<uint32_t> &units) {
     Trace trace_("free_units");
+    CKS(need_mirrors());
     if (units.empty()) return CGCM_OK;
     CKS(upload(up_units, units));
     launch_deactivate(up_units.as<uint32_t>(), (int)units.size(), tab(), main);
@@ -1204,58 +1399,67 @@ struct Context {
 
   // copy-back of whole units device -> host (Alg. 2's cuMemcpyDtoH).  Array-mapped units are
   // reverse translated first (A12) -- validated before any byte moves.  Synchronous.
+  // array-mapped units (unit, device copy): reverse translate their slots into staging (validated:
+  // a reverse miss fails the call before any byte moves, A12), then copy slots + trailing bytes back
+  int copy_back_arr(const std::vector<std::pair<uint32_t, uint64_t>> &arr) {
+    if (arr.empty()) return CGCM_OK;
+    uint64_t arr_bytes = 0;
+    for (auto &a : arr) arr_bytes += align_up(usize[a.first] / 8 * 8, 32) + 32;
+    CKS(ensure_rev());
+    CKS(dalloc(staging_cb, arr_bytes + 256));
+    SlotCall c;
+    c.dir = DIR_REV;
+    c.ops = OP_WRITE;
+    uint64_t off = staging_cb.addr;
+    std::vector<uint64_t> dst(arr.size());
+    for (size_t q = 0; q < arr.size(); ++q) {
+      const uint32_t x = arr[q].first;
+      const uint64_t db = arr[q].second, n = usize[x] / 8;
+      off = align_up(off, 32) + (db & 31);  // same alignment as the source
+      dst[q] = off;
+      Seg sg;
+      sg.ptr = db;
+      sg.n = n;
+      sg.out = off;
+      sg.inc = 0;
+      sg.pad = 0;
+      sg.shadow = 0;
+      if (n) c.segs.push_back(sg);
+      off += 8 * n;
+    }
+    CKS(prepare_small());
+    CKS(launch(c, 7));
+    Status sts[8];
+    unsigned long long lcs[4];
+    CKS(fetch_status(sts, lcs));
+    if (sts[7].misses && !(flags & CGCM_LENIENT)) return CGCM_E_UNREGISTERED;
+    st.rev_translations += sts[7].translated;
+    st.passthrough += (flags & CGCM_LENIENT) ? sts[7].misses : 0;
+    for (size_t q = 0; q < arr.size(); ++q) {
+      const uint32_t x = arr[q].first;
+      const uint64_t hb = ubase[x], sz = usize[x], db = arr[q].second, n = sz / 8;
+      if (n) CK(cudaMemcpyAsync(reinterpret_cast<void *>(hb), reinterpret_cast<void *>(dst[q]), 8 * n,
+                                cudaMemcpyDeviceToHost, copy));
+      if (sz > 8 * n)
+        CK(cudaMemcpyAsync(reinterpret_cast<void *>(hb + 8 * n), reinterpret_cast<void *>(db + 8 * n), sz - 8 * n,
+                           cudaMemcpyDeviceToHost, copy));
+      st.d2h_memcpy_calls += 1 + (sz > 8 * n);
+      st.d2h_units += 1;
+      st.d2h_bytes += sz;
+    }
+    return CGCM_OK;
+  }
   int copy_back(const std::vector<uint32_t> &units) {
     Trace trace_("copy_back");
     if (units.empty()) return CGCM_OK;
-    std::vector<uint32_t> plain, arr;
-    for (uint32_t x : units) (uarr[x] ? arr : plain).push_back(x);
-    // reverse-translate the array-mapped ones into staging_cb
-    uint64_t arr_bytes = 0;
-    for (uint32_t x : arr) arr_bytes += align_up(usize[x] / 8 * 8, 32) + 32;
-    if (!arr.empty()) {
-      CKS(ensure_rev());
-      CKS(dalloc(staging_cb, arr_bytes + 256));
-      SlotCall c;
-      c.dir = DIR_REV;
-      c.ops = OP_WRITE;
-      uint64_t off = staging_cb.addr;
-      std::vector<uint64_t> dst(arr.size());
-      for (size_t q = 0; q < arr.size(); ++q) {
-        uint32_t x = arr[q];
-        uint64_t n = usize[x] / 8;
-        off = align_up(off, 32) + (udev[x] & 31);  // same alignment as the source
-        dst[q] = off;
-        Seg s;
-        s.ptr = udev[x];
-        s.n = n;
-        s.out = off;
-        s.inc = 0;
-        s.pad = 0;
-        s.shadow = 0;
-        if (n) c.segs.push_back(s);
-        off += 8 * n;
-      }
-      CKS(prepare_small());
-      CKS(launch(c, 7));
-      Status sts[8];
-      unsigned long long lcs[4];
-      CKS(fetch_status(sts, lcs));
-      if (sts[7].misses && !(flags & CGCM_LENIENT)) return CGCM_E_UNREGISTERED;
-      st.rev_translations += sts[7].translated;
-      st.passthrough += (flags & CGCM_LENIENT) ? sts[7].misses : 0;
-      for (size_t q = 0; q < arr.size(); ++q) {
-        uint32_t x = arr[q];
-        uint64_t hb = ubase[x], sz = usize[x], db = udev[x], n = sz / 8;
-        if (n) CK(cudaMemcpyAsync(reinterpret_cast<void *>(hb), reinterpret_cast<void *>(dst[q]), 8 * n,
-                                  cudaMemcpyDeviceToHost, copy));
-        if (sz > 8 * n)
-          CK(cudaMemcpyAsync(reinterpret_cast<void *>(hb + 8 * n), reinterpret_cast<void *>(db + 8 * n), sz - 8 * n,
-                             cudaMemcpyDeviceToHost, copy));
-        st.d2h_memcpy_calls += 1 + (sz > 8 * n);
-        st.d2h_units += 1;
-        st.d2h_bytes += sz;
-      }
+    CKS(need_mirrors());
+    std::vector<uint32_t> plain;
+    std::vector<std::pair<uint32_t, uint64_t>> arr;
+    for (uint32_t x : units) {
+      if (uarr[x]) arr.push_back({x, udev[x]});
+      else plain.push_back(x);
     }
+    CKS(copy_back_arr(arr));
     // plain units: coalesce host-adjacent units whose device copies are mirrored
     size_t i = 0;
     while (i < plain.size()) {
@@ -1347,9 +1551,14 @@ struct Context {
     }
     // activations
     if (lcs[0] > 0) {
-      std::vector<uint32_t> units;
-      CKS(sorted_units(act_list, lcs[0], units));
-      int r = activate_units(units, nullptr, nullptr, true);
+      int r;
+      if (lcs[0] >= PLAN_MIN && !group) {  // planned on the device: one descriptor per pack
+        r = activate_planned(act_list, lcs[0]);
+      } else {
+        std::vector<uint32_t> units;
+        CKS(sorted_units(act_list, lcs[0], units));
+        r = activate_units(units, nullptr, nullptr, true);
+      }
       if (r != CGCM_OK) {
         CKS(undo_deferred());
         CKS(undo_map(F, R));
@@ -1477,7 +1686,8 @@ struct Context {
       }
       return err;
     }
-    CKS(sorted_units(copy_list, lcs[3], copy_units));
+    rev_copy_n = lcs[3];  // the caller copies back copy_list[0, rev_copy_n) (copy_back_list)
+    (void)copy_units;
     if (dec && lcs[2]) {
       std::vector<uint32_t> f;
       CKS(download(f, free_list, lcs[2]));
@@ -1486,6 +1696,7 @@ struct Context {
     return CGCM_OK;
   }
   bool snapshotted = false;
+  size_t rev_copy_n = 0;
   // forward-map shadows of device-resident pointer arrays, keyed by (slots, n)
   struct Shadow {
     DevBuf buf;
@@ -1658,6 +1869,7 @@ int Context::peer_sources(const std::vector<uint32_t> &units, std::vector<PeerSr
     std::lock_guard<std::recursive_mutex> lk(c->mu);
     if (cudaSetDevice(c->device) != cudaSuccess) return CGCM_E_CUDA;
     int r = c->ensure_table();
+    if (r == CGCM_OK) r = c->need_mirrors();
     std::vector<uint32_t> cidx;
     std::vector<size_t> which;
     if (r == CGCM_OK)
@@ -2086,6 +2298,7 @@ int cgcm_undeclare(void *base) {
   auto it = C->reg.find(b);
   if (it == C->reg.end()) return CGCM_E_UNREGISTERED;
   HostUnit &u = it->second;
+  CKS(C->need_mirrors());
   if (u.idx >= 0) {  // idx refers to the current device table until the next ensure_table()
     int32_t rc = 0;
     CK(cudaMemcpyAsync(&rc, C->rcb.as<int32_t>() + u.idx, 4, cudaMemcpyDeviceToHost, C->main));
@@ -2283,7 +2496,7 @@ int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
   // (on failure the snapshot restores rc and the shadow keeps its deferred references: the next call
   // materialises them)
   CKS(C->unmap_rev_core({s}, true, rel, copy_units, freed, jcount, res, defer));
-  int r = C->copy_back(copy_units);
+  int r = C->copy_back_list(C->copy_list, C->rev_copy_n);
   if (r != CGCM_OK) {
     // reverse translation of an array-mapped element failed: undo the whole call
     SlotCall c;
@@ -2353,9 +2566,7 @@ int cgcm_unmapBatch(const void *const *cpu, size_t n) {
   int err = CGCM_OK;
   if (sts[0].misses && !(C->flags & CGCM_LENIENT)) err = CGCM_E_UNREGISTERED;
   else if (sts[0].notmapped) err = CGCM_E_NOT_MAPPED;
-  std::vector<uint32_t> cu;
-  if (!err) err = C->sorted_units(C->copy_list, lcs[3], cu);
-  if (!err) err = C->copy_back(cu);
+  if (!err) err = C->copy_back_list(C->copy_list, lcs[3]);
   if (err) {
     SlotCall u;
     CKS(C->undo_rev(u, lcs[1], {}, false, false));
@@ -2438,6 +2649,7 @@ int distinct_outers(const std::vector<PointInfo> &infos, std::vector<Outer> &out
 
 int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
   CTXM();
+  CKS(C->need_mirrors());
   if (k == 0) return CGCM_OK;
   if (!arrays || !gpu_out) return CGCM_E_INVALID;
   std::vector<PointInfo> infos;
@@ -2682,11 +2894,9 @@ int cgcm_unmapArrays(void *const *const *arrays, size_t k) {
   int err = CGCM_OK;
   if ((sts[0].misses || sts[2].misses) && strict) err = CGCM_E_UNREGISTERED;
   else if (sts[2].notmapped || (sts[1].misses && strict)) err = CGCM_E_NOT_MAPPED;
-  std::vector<uint32_t> cu;
-  if (!err) err = C->sorted_units(C->copy_list, lcs[3], cu);
   // element copy-backs (array-mapped elements are reverse translated and validated first, into
   // their own staging buffer); the outers' staged slots are copied below
-  if (!err) err = C->copy_back(cu);
+  if (!err) err = C->copy_back_list(C->copy_list, lcs[3]);
   if (err) {
     SlotCall none;
     C->undo_rev(none, lcs[1], outer_jn, false, false);
