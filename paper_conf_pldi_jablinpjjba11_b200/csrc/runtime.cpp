@@ -1005,8 +1005,7 @@ struct Context {
   // the main stream then does NOT wait for the copies -- the caller waits per pack (transfer overlap)
   int activate_units(const std::vector<uint32_t> &units, std::vector<std::pair<uint64_t, uint64_t>> *h2d_out,
                      std::vector<cudaEvent_t> *pack_ev = nullptr, bool allow_peer = false) {
-    Trace trace_("activate_units");
-    CKS(need_mirrors());
+    Trace trace_("activate_units");  // (mirrors: globals never take the planned path; the rest are written here)
     if (units.empty()) return CGCM_OK;
     const uint64_t PACK_SPAN = 64ull << 20, GAPMAX = 64ull << 10, PACK_MIN = 256ull << 10;
     struct Pack {
@@ -1157,6 +1156,30 @@ struct Context {
     mirror_stale = false;
     return CGCM_OK;
   }
+  // refresh the mirrors of just these units (their state words: extent + flags) -- O(|xs|)
+  DevBuf mir_idx, mir_out;
+  int mirror_units(const std::vector<uint32_t> &xs) {
+    if (!mirror_stale || xs.empty()) return CGCM_OK;
+    CKS(upload(mir_idx, xs));
+    CKS(dalloc(mir_out, 8 * xs.size() + 64));
+    launch_gather_state(tab(), mir_idx.as<uint32_t>(), (int)xs.size(), mir_out.as<uint64_t>(), main);
+    st.kernel_launches += 1;
+    CK(cudaGetLastError());
+    std::vector<uint64_t> w;
+    CKS(download(w, mir_out, xs.size()));
+    for (size_t q = 0; q < xs.size(); ++q) {
+      const uint32_t x = xs[q], fl = hot_flags(w[q]), e = hot_ext(w[q]);
+      if ((fl & UF_STORAGE) && e < runs.size()) {
+        urun[x] = (int64_t)e;
+        udev[x] = ubase[x] - runs[e].delta;
+      } else {
+        urun[x] = -1;
+        udev[x] = 0;
+      }
+      uarr[x] = (fl & UF_ARRAYMAPPED) ? 1 : 0;
+    }
+    return CGCM_OK;
+  }
   // sort the n unit ids of a device list into plan_S (and size the planning scratch)
   int plan_sort(const DevBuf &list, size_t n) {
     plan_tb = std::max(sort_keys_temp_bytes((int)n), plan_temp_bytes((int)n)) + 256;
@@ -1181,6 +1204,7 @@ struct Context {
   int activate_planned(const DevBuf &list, size_t n) {
     Trace trace_("activate(planned)");
     const uint64_t GAPMAX = 64ull << 10;
+    auto tr1 = std::make_unique<Trace>("  plan:sort+scan+download");
     CKS(plan_sort(list, n));
     int r = launch_plan_packs1(plan_S.as<uint32_t>(), (int)n, tab(), GAPMAX, 26, plan_F.as<uint32_t>(),
                                plan_G.as<uint32_t>(), plan_pid.as<uint32_t>(), plan_gscan.as<uint32_t>(),
@@ -1203,6 +1227,8 @@ struct Context {
     st.kernel_launches += 2;
     std::vector<PackDesc> packs;
     CKS(download(packs, plan_desc, np));
+    tr1.reset();
+    auto tr2 = std::make_unique<Trace>("  plan:alloc+set_ext");
     // device extents, all or nothing
     std::vector<int64_t> created;
     std::vector<uint32_t> rid(np);
@@ -1231,6 +1257,8 @@ struct Context {
                         rel_epoch(epoch), (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
+    tr2.reset();
+    Trace tr3("  plan:copies(issue)");
     CK(cudaEventRecord(ev_copy, main));
     CK(cudaStreamWaitEvent(copy, ev_copy, 0));
     for (size_t p = 0; p < np; ++p) {  // the transfer scheduler: one DMA per pack
@@ -1374,7 +1402,7 @@ struct Context {
   // units whose refcount reached 0: free device storage (globals keep theirs), clear flags
   int free_units(const std::vector<uint32_t> &units) {
     Trace trace_("free_units");
-    CKS(need_mirrors());
+    CKS(mirror_units(units));
     if (units.empty()) return CGCM_OK;
     CKS(upload(up_units, units));
     launch_deactivate(up_units.as<uint32_t>(), (int)units.size(), tab(), main);
@@ -1452,7 +1480,7 @@ struct Context {
   int copy_back(const std::vector<uint32_t> &units) {
     Trace trace_("copy_back");
     if (units.empty()) return CGCM_OK;
-    CKS(need_mirrors());
+    CKS(mirror_units(units));
     std::vector<uint32_t> plain;
     std::vector<std::pair<uint32_t, uint64_t>> arr;
     for (uint32_t x : units) {
@@ -1869,7 +1897,7 @@ int Context::peer_sources(const std::vector<uint32_t> &units, std::vector<PeerSr
     std::lock_guard<std::recursive_mutex> lk(c->mu);
     if (cudaSetDevice(c->device) != cudaSuccess) return CGCM_E_CUDA;
     int r = c->ensure_table();
-    if (r == CGCM_OK) r = c->need_mirrors();
+
     std::vector<uint32_t> cidx;
     std::vector<size_t> which;
     if (r == CGCM_OK)
@@ -1903,9 +1931,11 @@ int Context::peer_sources(const std::vector<uint32_t> &units, std::vector<PeerSr
           const uint32_t ci = cidx[k];
           ++k;
           // active, holding a copy, writable, and dirty: c launched since the unit became coherent there
-          if ((fl & UF_ACTIVE) && (fl & UF_STORAGE) && !(fl & UF_READONLY) && st_epoch(w) != cur && c->udev[ci]) {
+          const uint32_t ce = hot_ext(w);
+          if ((fl & UF_ACTIVE) && (fl & UF_STORAGE) && !(fl & UF_READONLY) && st_epoch(w) != cur &&
+              ce < c->runs.size()) {
             out[q].ctx = c;
-            out[q].src = c->udev[ci];
+            out[q].src = c->ubase[ci] - c->runs[ce].delta;  // the peer's copy (from its device table)
             any = true;
             continue;
           }
@@ -2298,7 +2328,7 @@ int cgcm_undeclare(void *base) {
   auto it = C->reg.find(b);
   if (it == C->reg.end()) return CGCM_E_UNREGISTERED;
   HostUnit &u = it->second;
-  CKS(C->need_mirrors());
+  if (u.idx >= 0) CKS(C->mirror_units({(uint32_t)u.idx}));
   if (u.idx >= 0) {  // idx refers to the current device table until the next ensure_table()
     int32_t rc = 0;
     CK(cudaMemcpyAsync(&rc, C->rcb.as<int32_t>() + u.idx, 4, cudaMemcpyDeviceToHost, C->main));
@@ -2649,7 +2679,7 @@ int distinct_outers(const std::vector<PointInfo> &infos, std::vector<Outer> &out
 
 int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
   CTXM();
-  CKS(C->need_mirrors());
+
   if (k == 0) return CGCM_OK;
   if (!arrays || !gpu_out) return CGCM_E_INVALID;
   std::vector<PointInfo> infos;
@@ -2657,6 +2687,11 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
   std::vector<Outer> outs;
   std::vector<int> which;
   CKS(distinct_outers(infos, outs, which));
+  {
+    std::vector<uint32_t> ou;
+    for (auto &o : outs) ou.push_back((uint32_t)o.unit);
+    CKS(C->mirror_units(ou));
+  }
   // prologue: activate inactive outers (raw copy of the CPU pointer array, rewritten in place),
   // then refcount/flags of every outer -- the outer AU first (A9)
   std::vector<uint32_t> act;
