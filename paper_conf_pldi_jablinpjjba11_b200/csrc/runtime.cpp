@@ -1180,6 +1180,15 @@ struct Context {
     }
     return CGCM_OK;
   }
+  // host memory the driver has pinned (cudaHostAlloc / cudaHostRegister): a DMA may read it directly
+  static bool host_pinned(uint64_t h) {
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, reinterpret_cast<const void *>(h)) != cudaSuccess) {
+      (void)cudaGetLastError();
+      return false;
+    }
+    return at.type == cudaMemoryTypeHost;
+  }
   // sort the n unit ids of a device list into plan_S (and size the planning scratch)
   int plan_sort(const DevBuf &list, size_t n) {
     plan_tb = std::max(sort_keys_temp_bytes((int)n), plan_temp_bytes((int)n)) + 256;
@@ -1264,7 +1273,11 @@ struct Context {
     for (size_t p = 0; p < np; ++p) {  // the transfer scheduler: one DMA per pack
       const PackDesc &P = packs[p];
       const uint64_t span = P.h1 - P.h0;
-      if (!P.gaps) {
+      // a pack with host gaps in pinned memory: one DMA of the whole span (the gap bytes land in the
+      // extent's mirrored gaps, which belong to no unit); pageable memory is gathered unit by unit
+      // (its gap pages may not even be mapped)
+      if (!P.gaps || (host_pinned(P.h0) && host_pinned(P.h1 - 1))) {  // (a span across two pinned
+        // allocations is rejected by cudaMemcpyAsync, then gathered below)
         cudaError_t e = cudaMemcpyAsync(reinterpret_cast<void *>(dev0[p]), reinterpret_cast<const void *>(P.h0), span,
                                         cudaMemcpyHostToDevice, copy);
         if (e == cudaSuccess) {
