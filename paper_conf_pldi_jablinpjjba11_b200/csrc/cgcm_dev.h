@@ -313,6 +313,10 @@ int launch_plan_copyback1(const uint32_t *S, int n, TableDev tab, uint32_t *F, u
 int launch_plan_copyback2(const uint32_t *S, int n, TableDev tab, const uint32_t *F, const uint32_t *rid,
                           CopyRun *runs, cudaStream_t s);
 
+// frees of the sorted list S (duplicates counted once): run_dec[e] = copies extent e loses; arr_out =
+// (unit, extent) pairs of array-mapped units; cnt[0] = frees, cnt[1] = globals, cnt[2] = #arr pairs
+void launch_free_plan(const uint32_t *S, int n, TableDev tab, uint32_t *run_dec, int nruns, uint32_t *arr_out,
+                      unsigned long long *cnt, cudaStream_t s);
 // out[i] = st[idx[i]] (epoch | extent | flags) of n units (NEXT-3 peer-source queries)
 void launch_gather_state(TableDev tab, const uint32_t *idx, int n, uint64_t *out, cudaStream_t s);
 // add every deferred reference recorded in a shadow's n unit words to rc (they become ordinary references)

@@ -2127,6 +2127,45 @@ int launch_plan_copyback2(const uint32_t *S, int n, TableDev tab, const uint32_t
   return (int)cudaGetLastError();
 }
 
+// frees of a sorted unit list (Alg. 3's cuMemFree at refCount 0), planned before k_deactivate clears the
+// flags: per extent the number of copies it loses (warp-aggregated), the array-mapped units (the host
+// drops their shadows), counts of frees and of globals (which keep their named region)
+__global__ void k_free_plan(const uint32_t *S, int n, TableDev tab, uint32_t *run_dec, uint32_t *arr_out,
+                            unsigned long long *cnt) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  bool fr = false, glob = false, arr = false;
+  uint32_t x = 0, e = 0xFFFFFFFFu;
+  if (i < n) {
+    x = S[i];
+    if ((i == 0 || S[i - 1] != x) && tab.rc[x] == 0) {
+      const uint64_t h = tab.hot[x];
+      glob = hot_flags(h) & UF_GLOBAL;
+      fr = !glob && (hot_flags(h) & UF_STORAGE);
+      arr = hot_flags(h) & UF_ARRAYMAPPED;
+      if (fr) e = hot_ext(h);
+    }
+  }
+  const unsigned peers = __match_any_sync(0xffffffffu, e);
+  if (fr && (threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(run_dec + e, (uint32_t)__popc(peers));
+  const unsigned nf = __popc(__ballot_sync(0xffffffffu, fr)), ng = __popc(__ballot_sync(0xffffffffu, glob));
+  if ((threadIdx.x & 31) == 0) {
+    if (nf) atomicAdd(&cnt[0], (unsigned long long)nf);
+    if (ng) atomicAdd(&cnt[1], (unsigned long long)ng);
+  }
+  const unsigned long long ix = warp_append(&cnt[2], arr);
+  if (arr) {
+    arr_out[2 * ix] = x;
+    arr_out[2 * ix + 1] = fr ? e : 0xFFFFFFFFu;
+  }
+}
+void launch_free_plan(const uint32_t *S, int n, TableDev tab, uint32_t *run_dec, int nruns, uint32_t *arr_out,
+                      unsigned long long *cnt, cudaStream_t s) {
+  (void)cudaGetLastError();
+  cudaMemsetAsync(cnt, 0, 32, s);
+  cudaMemsetAsync(run_dec, 0, 4 * (size_t)(nruns > 0 ? nruns : 1), s);
+  if (n > 0) k_free_plan<<<(n + 255) / 256, 256, 0, s>>>(S, n, tab, run_dec, arr_out, cnt);
+}
+
 // -------------------------------------------------------------------------------------------------
 // small bookkeeping kernels
 // -------------------------------------------------------------------------------------------------

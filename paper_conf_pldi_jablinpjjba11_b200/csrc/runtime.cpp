@@ -1310,6 +1310,63 @@ struct Context {
     mirror_stale = true;
     return CGCM_OK;
   }
+  // Frees (Alg. 3) of the n units of a device list (+ extra host-listed units): for long lists planned on
+  // the device -- per extent the number of copies it loses, the array-mapped units listed -- so the host
+  // does O(#extents + #array-mapped) work.  Device-array shadows inside freed copies need the host path.
+  DevBuf free_dec, free_arr;
+  int free_units_list(const DevBuf &list, size_t n, const std::vector<uint32_t> &extra = {}) {
+    if (n + extra.size() == 0) return CGCM_OK;
+    if (n + extra.size() < PLAN_MIN || dev_shadows) {
+      std::vector<uint32_t> f;
+      CKS(download(f, list, n));
+      f.insert(f.end(), extra.begin(), extra.end());
+      std::sort(f.begin(), f.end());
+      f.erase(std::unique(f.begin(), f.end()), f.end());
+      return free_units(f);
+    }
+    Trace trace_("free_units(planned)");
+    const size_t m = n + extra.size();
+    // the list (+ extras) sorted into plan_S: duplicates adjacent
+    CKS(dalloc(plan_S, 4 * m + 64));
+    DevBuf tmpl;
+    const DevBuf *src = &list;
+    if (!extra.empty()) {  // append the extras behind a copy of the list
+      CKS(dalloc(plan_G, 4 * m + 64));
+      CK(cudaMemcpyAsync(plan_G.as<void>(), list.as<void>(), 4 * n, cudaMemcpyDeviceToDevice, main));
+      CK(cudaMemcpyAsync(plan_G.as<uint32_t>() + n, extra.data(), 4 * extra.size(), cudaMemcpyHostToDevice, main));
+      CK(cudaStreamSynchronize(main));  // (extra is pageable host memory)
+      src = &plan_G;
+    }
+    CKS(plan_sort(*src, m));
+    CKS(dalloc(free_dec, 4 * std::max<size_t>(runs.size(), 1) + 64));
+    CKS(dalloc(free_arr, 8 * m + 64));
+    launch_free_plan(plan_S.as<uint32_t>(), (int)m, tab(), free_dec.as<uint32_t>(), (int)runs.size(),
+                     free_arr.as<uint32_t>(), plan_cnt.as<unsigned long long>(), main);
+    launch_deactivate(plan_S.as<uint32_t>(), (int)m, tab(), main);
+    st.kernel_launches += 2;
+    CK(cudaGetLastError());
+    std::vector<unsigned long long> cnt;
+    CKS(download(cnt, plan_cnt, 4));
+    std::vector<uint32_t> dec, arr;
+    CKS(download(dec, free_dec, runs.size()));
+    CKS(download(arr, free_arr, 2 * cnt[2]));
+    for (size_t q = 0; q < cnt[2]; ++q) {  // array-mapped: their shadows go with their copies
+      const uint32_t x = arr[2 * q], e = arr[2 * q + 1];
+      arr_gen.erase(ubase[x]);
+      if (e < runs.size()) drop_shadows(ubase[x] - runs[e].delta);
+      else if (udev[x]) drop_shadows(udev[x]);  // a global: its named region stays
+    }
+    for (size_t r = 0; r < dec.size(); ++r) {
+      if (!dec[r]) continue;
+      free_gen += dec[r];
+      runs[r].live -= (int64_t)dec[r];
+      if (runs[r].live <= 0) drop_run((int64_t)r);
+    }
+    st.frees += cnt[0];
+    rev_dirty = true;
+    mirror_stale = true;
+    return CGCM_OK;
+  }
   // Copy-back (Alg. 2's cuMemcpyDtoH) of the n units of a device list: plain units as one DMA per
   // host-adjacent mirrored run, array-mapped units reverse translated first (A12).  Planned on the
   // device for long lists.
@@ -1728,16 +1785,13 @@ struct Context {
       return err;
     }
     rev_copy_n = lcs[3];  // the caller copies back copy_list[0, rev_copy_n) (copy_back_list)
+    rev_free_n = dec ? lcs[2] : 0;  // and frees free_list[0, rev_free_n) (free_units_list)
     (void)copy_units;
-    if (dec && lcs[2]) {
-      std::vector<uint32_t> f;
-      CKS(download(f, free_list, lcs[2]));
-      freed.insert(freed.end(), f.begin(), f.end());
-    }
+    (void)freed;
     return CGCM_OK;
   }
   bool snapshotted = false;
-  size_t rev_copy_n = 0;
+  size_t rev_copy_n = 0, rev_free_n = 0;
   // forward-map shadows of device-resident pointer arrays, keyed by (slots, n)
   struct Shadow {
     DevBuf buf;
@@ -2560,7 +2614,7 @@ int cgcm_unmapArrayDevice(uint64_t *d_slots, size_t n, unsigned flags) {
   }
   C->st.rev_translations += res.translated;
   if (C->flags & CGCM_LENIENT) C->st.passthrough += res.misses;
-  CKS(C->free_units(freed));
+  CKS(C->free_units_list(C->free_list, C->rev_free_n));
   return CGCM_OK;
 }
 
@@ -2648,9 +2702,7 @@ int cgcm_releaseBatch(const void *const *cpu, size_t n) {
     CK(cudaStreamSynchronize(C->main));
     return err;
   }
-  std::vector<uint32_t> f;
-  CKS(C->download(f, C->free_list, lcs[2]));
-  return C->free_units(f);
+  return C->free_units_list(C->free_list, lcs[2]);
 }
 
 int cgcm_map(const void *cpu, void **gpu_out) {
@@ -3036,15 +3088,10 @@ int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
     CK(cudaStreamSynchronize(C->main));
     return err;
   }
-  std::vector<uint32_t> f;
-  CKS(C->download(f, C->free_list, lcs[2]));
-  // an outer reaches 0 through its own decrement only if no slot pointed into it
-  for (uint32_t x : outer_zero) f.push_back(x);
-  std::sort(f.begin(), f.end());
-  f.erase(std::unique(f.begin(), f.end()), f.end());
-  // outers whose zero came from a slot decrement are already in f; outers with remaining slot refs
-  // into them (self-reference) cannot be in outer_zero (their refcount exceeded mult)
-  return C->free_units(f);
+  // an outer reaches 0 through its own decrement only if no slot pointed into it; outers whose zero came
+  // from a slot decrement are in the list too (duplicates are freed once); outers with remaining slot
+  // refs into them (self-reference) cannot be in outer_zero (their refcount exceeded mult)
+  return C->free_units_list(C->free_list, lcs[2], outer_zero);
 }
 
 // ---- map-promotion regions (NEXT-2) ----
