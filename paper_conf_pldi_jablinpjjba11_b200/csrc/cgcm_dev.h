@@ -111,16 +111,22 @@ struct IndexDev {
 //   w[0]     j0 = greatestLTE(A), the unit with the greatest base <= A (0xFFFFFFFF: none)
 //   w[1]     cnt (bits 0..13): units with base in (A, A + 2^P) | bit 14: base(j0) == A
 //            | end0 (bits 15..31): min(base(j0) + size(j0) - A + 1, 0x1FFFF), 0 if j0 ends before A
-//   w[2..7]  cnt <= PD_K: the offsets base - A of those units, sorted u16, padded with PD_PAD;
-//            cnt >  PD_K: w[2] = index of the first of cnt sorted u16 offsets in ovf[] (16-aligned,
-//            padded with PD_PAD to a whole 32-byte sector)
-// greatestLTE(p) = j0 + #{offsets <= p - A}; p hits unit j0 iff p - A < end0 (A7: p - base <= size),
-// any other candidate by its base A + offset and its size (hot word).  One sector gather per lookup.
-// Pages are at most 32 KiB (P <= 15): offsets and the padding PD_PAD = 0x7FFF fit 15 bits, so four of
-// them compare against p - A in one 64-bit subtraction with a guard bit per lane (k_fwd_lean); no
+//   w[2]     page state: PD_STATE_VALID | extent id (bits 0..23) when every unit a lookup in the page can
+//            return (j0 if it reaches into the page, j0+1 .. j0+cnt) is ACTIVE with its device copy in
+//            that extent; else 0.  Rewritten by k_pd_state before a kernel reads the directory, whenever a
+//            unit's state changed since (Context::pd_state_dirty).
+//   w[3..7]  cnt <= PD_K: candidate t (the unit j0+1+t) = start (bits 0..15: base - A) | end (bits 16..31:
+//            min(base + size - A, PD_PAD)); p hits it iff p - A <= end (A7); unused: start PD_PAD, end 0
+//            cnt >  PD_K: w[3] = index of the first of cnt sorted u16 starts in ovf[] (16-aligned, padded
+//            with PD_PAD to a whole 32-byte sector); w[2] = 0
+// greatestLTE(p) = j0 + #{starts <= p - A}; p hits unit j0 iff p - A < end0, a candidate iff p - A <= its
+// end -- decided from the entry alone.  With a valid page state the translation needs nothing else: one
+// sector gather per lookup (k_fwd_lean); otherwise the unit word is gathered.
+// Pages are at most 32 KiB (P <= 15): starts, ends and the padding PD_PAD = 0x7FFF fit 15 bits, so the
+// starts compare against p - A two per 64-bit subtraction with a guard bit per 16-bit lane (pd_count5); no
 // start sits at offset PD_PAD (build_pd takes a smaller page), and lookups clamp p - A to PD_PAD - 1.
 constexpr int PD_MAXSEG = 64;
-constexpr int PD_K = 12;
+constexpr int PD_K = 5;
 #ifdef CGCM_PD_MAXSHIFT
 constexpr int PD_MAXSHIFT = CGCM_PD_MAXSHIFT;
 #else
@@ -128,6 +134,7 @@ constexpr int PD_MAXSHIFT = 15;  // 32 KiB pages (64 KiB measured no faster at E
 #endif
 static_assert(PD_MAXSHIFT <= 15, "page offsets must fit 15 bits");
 constexpr uint32_t PD_PAD = 0x7FFFu;
+constexpr uint32_t PD_STATE_VALID = 0x80000000u;
 constexpr uint32_t PD_CNT_MAX = 0x3FFFu;
 constexpr uint32_t PD_EXACT = 1u << 14;
 constexpr int PD_END_SHIFT = 15;
@@ -317,6 +324,8 @@ int launch_plan_copyback2(const uint32_t *S, int n, TableDev tab, const uint32_t
 // (unit, extent) pairs of array-mapped units; cnt[0] = frees, cnt[1] = globals, cnt[2] = #arr pairs
 void launch_free_plan(const uint32_t *S, int n, TableDev tab, uint32_t *run_dec, int nruns, uint32_t *arr_out,
                       unsigned long long *cnt, cudaStream_t s);
+// recompute the page state word w[2] of every page entry from the units' hot words
+void launch_pd_state(PdDev pd, uint64_t npages, TableDev tab, cudaStream_t s);
 // out[i] = st[idx[i]] (epoch | extent | flags) of n units (NEXT-3 peer-source queries)
 void launch_gather_state(TableDev tab, const uint32_t *idx, int n, uint64_t *out, cudaStream_t s);
 // add every deferred reference recorded in a shadow's n unit words to rc (they become ordinary references)

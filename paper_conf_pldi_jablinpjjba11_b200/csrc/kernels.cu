@@ -344,6 +344,20 @@ __device__ __forceinline__ void cnt_max2(uint32_t w, uint32_t rr, uint32_t &cnt,
   mx = __vmaxu2(mx, w & m);
 }
 
+// #{starts <= r} among an entry's (at most PD_K = 5) candidates, and the candidate word (start | end << 16)
+// of the last of them (k > 0).  The 64-bit words e[1..3] hold w[2..7]: lane 2 of e[1] and lanes 0, 2 of
+// e[2], e[3] are starts; per lane 0x8000 + r - x keeps bit 15 iff x <= r and never borrows into the next
+// lane (every lane < 0x8000: starts and ends are 15-bit, the state word of e[1] is masked off).
+__device__ __forceinline__ uint32_t pd_count5(const uint64_t e[4], uint32_t r, uint32_t &word) {
+  const uint32_t r2 = r | (r << 16);
+  const uint64_t rg = ((uint64_t)r2 | ((uint64_t)r2 << 32)) | 0x8000800080008000ull;
+  const uint32_t k = __popcll((rg - (e[1] & 0xFFFFFFFF00000000ull)) & 0x0000800000000000ull) +
+                     __popcll((rg - e[2]) & 0x0000800000008000ull) + __popcll((rg - e[3]) & 0x0000800000008000ull);
+  const uint64_t q = k <= 1 ? e[1] : (k <= 3 ? e[2] : e[3]);
+  word = (k & 1) ? (uint32_t)(q >> 32) : (uint32_t)q;  // candidate k-1: w[3] (e1 hi), w[4] (e2 lo), ...
+  return k;
+}
+
 // Front half of a page-directory lookup of host address q: the segment, the page, and the entry to
 // gather (ok), or the tail of the segment's last unit (tail >= 0: that unit, -1: a miss).
 struct PdFront {
@@ -395,13 +409,12 @@ __device__ __forceinline__ void pd_back(const PdDev &pd, uint64_t pol, const PdF
   const uint32_t rr = min(f.poff, PD_PAD - 1u) * 0x10001u;
   uint32_t c = 0, mx = 0;
   if (cnt <= (uint32_t)PD_K) {
-#pragma unroll
-    for (int t = 1; t < 4; ++t) {
-      cnt_max2((uint32_t)w_in[t], rr, c, mx);
-      cnt_max2((uint32_t)(w_in[t] >> 32), rr, c, mx);
-    }
-  } else {  // crowded page: the offsets continue in ovf[], one sector per 16
-    const uint16_t *o = pd.ovf + (uint32_t)w_in[1];
+    uint32_t word;
+    const uint32_t kk = pd_count5(w_in, min(f.poff, PD_PAD - 1u), word);
+    c = kk << 4;  // (16 per counted start, as below)
+    mx = kk ? (word & 0xFFFFu) : 0u;
+  } else {  // crowded page: the starts continue in ovf[], one sector per 16
+    const uint16_t *o = pd.ovf + (uint32_t)(w_in[1] >> 32);
     for (uint32_t t = 0; t < cnt; t += 16) {
       uint64_t v[4];
       ld_sector(o + t, pol, v);
@@ -470,13 +483,12 @@ __device__ __forceinline__ void pd_lookup2(const SPd &S, const PdDev &pd, uint64
     const uint32_t rr = min(poff[m], PD_PAD - 1u) * 0x10001u;  // see pd_back
     uint32_t c = 0, mx = 0;
     if (cnt <= (uint32_t)PD_K) {
-#pragma unroll
-      for (int t = 1; t < 4; ++t) {
-        cnt_max2((uint32_t)w[m][t], rr, c, mx);
-        cnt_max2((uint32_t)(w[m][t] >> 32), rr, c, mx);
-      }
-    } else {  // crowded page: the offsets continue in ovf[], one sector per 16
-      const uint16_t *o = pd.ovf + (uint32_t)w[m][1];
+      uint32_t word;
+      const uint32_t kk = pd_count5(w[m], min(poff[m], PD_PAD - 1u), word);
+      c = kk << 4;
+      mx = kk ? (word & 0xFFFFu) : 0u;
+    } else {  // crowded page: the starts continue in ovf[], one sector per 16
+      const uint16_t *o = pd.ovf + (uint32_t)(w[m][1] >> 32);
       for (uint32_t t = 0; t < cnt; t += 16) {
         uint64_t v[4];
         ld_sector(o + t, pol, v);
@@ -1465,37 +1477,40 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
     const uint64_t a0 = a0base + 16ull * c;
     const uint32_t valid = valid_of(c);
 
-    // decode: j = j0 + #{offsets <= p - A}; the page's j0 is decided by its end, others by base + size
+    // decode: j = j0 + #{starts <= p - A}; j0 is decided by its end, a candidate by its end in the entry
+    // (A7); in a page whose state is valid the entry also gives ACTIVE and the extent: no unit word
     int j[2];
-    bool k0[2];
+    bool k0[2], dec[2];
     uint64_t key[2];
-    uint32_t cw[2];
+    uint32_t cw[2], ps[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
       j[m] = fc.jt[m];
       k0[m] = true;
+      dec[m] = false;
       key[m] = 0;
+      ps[m] = 0;
       if (fc.ok[m]) {
         const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
         const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
         const uint32_t r = min(fc.poff[m], PD_PAD - 1u);
-        uint32_t k, off;
         if (cnt <= (uint32_t)PD_K) {
-          const uint32_t r2 = r | (r << 16);
-          const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
-          k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
-          off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
-        } else {
-          const uint64_t ko = pd_crowded(a.pd.ovf, (uint32_t)fc.ew[m][1], cnt, r);
-          k = (uint32_t)ko;
-          off = (uint32_t)(ko >> 32);
+          uint32_t word;
+          const uint32_t k = pd_count5(fc.ew[m], r, word);
+          const bool h = k ? fc.poff[m] <= (word >> 16) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0);
+          j[m] = h ? (int)(j0 + k) : -1;
+          dec[m] = true;
+          ps[m] = (uint32_t)fc.ew[m][1];
+        } else {  // crowded page: starts in the side array, the candidate's size from its unit word
+          const uint64_t ko = pd_crowded(a.pd.ovf, (uint32_t)(fc.ew[m][1] >> 32), cnt, r);
+          const uint32_t k = (uint32_t)ko, off = (uint32_t)(ko >> 32);
+          k0[m] = k == 0;
+          j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
+          key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
         }
-        k0[m] = k == 0;
-        j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
-        key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
       }
       cw[m] = 0;
-      if (j[m] >= 0)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
+      if (j[m] >= 0 && !(ps[m] & PD_STATE_VALID))  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
         asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
     }
     uint64_t outv[2] = {cv[0], cv[1]};
@@ -1505,10 +1520,14 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
     for (int m = 0; m < 2; ++m) {
       const bool vm = (valid >> m) & 1;
       const bool look = j[m] >= 0;
-      const uint64_t hw = (cw[m] & HOTC_ESC) && look ? ld_u64_hot(a.tab.hot + j[m], pol_t) : hot_of_hotc(cw[m]);
+      uint64_t hw;
+      if (ps[m] & PD_STATE_VALID)  // every unit of the page is ACTIVE with its copy in this extent
+        hw = ((uint64_t)(ps[m] & EXT_MASK) << ESHIFT) | ((uint64_t)(UF_ACTIVE | UF_STORAGE) << FSHIFT);
+      else
+        hw = (cw[m] & HOTC_ESC) && look ? ld_u64_hot(a.tab.hot + j[m], pol_t) : hot_of_hotc(cw[m]);
       uint64_t sz = hot_size32(hw);
-      if (look && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
-      const bool hit = look && (k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
+      if (look && !dec[m] && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
+      const bool hit = look && (dec[m] || k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
       const bool nul = vm && cv[m] == 0;
       c_nulls += nul;
       c_hits += hit;
@@ -2125,6 +2144,37 @@ int launch_plan_copyback2(const uint32_t *S, int n, TableDev tab, const uint32_t
   k_cb_first<<<g, 256, 0, s>>>(S, n, tab, F, rid, runs);
   k_cb_last<<<g, 256, 0, s>>>(S, n, tab, F, rid, runs);
   return (int)cudaGetLastError();
+}
+
+// page state words (w[2] of every page entry): valid with the extent when every unit a lookup in the page
+// can return is ACTIVE with its copy in that one extent (cgcm_dev.h "Page directory")
+__global__ void k_pd_state(PdDev pd, uint64_t npages, TableDev tab) {
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < npages; e += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t *w = const_cast<uint32_t *>(pd.ent) + 8 * e;
+    const uint32_t j0 = w[0], w1 = w[1], cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
+    uint32_t state = 0;
+    if (cnt <= (uint32_t)PD_K) {
+      bool ok = true, any = false;
+      uint32_t ext = 0;
+      auto take = [&](uint32_t u) {
+        const uint64_t h = tab.hot[u];
+        const uint32_t fl = hot_flags(h), x = hot_ext(h);
+        ok = ok && (fl & UF_ACTIVE) && (fl & UF_STORAGE) && (!any || x == ext);
+        ext = x;
+        any = true;
+      };
+      if (j0 != 0xFFFFFFFFu && end0 > 0) take(j0);
+      for (uint32_t t = 0; t < cnt; ++t) take(j0 + 1 + t);
+      if (ok && any) state = PD_STATE_VALID | (ext & (uint32_t)EXT_MASK);
+    }
+    w[2] = state;
+  }
+}
+void launch_pd_state(PdDev pd, uint64_t npages, TableDev tab, cudaStream_t s) {
+  if (npages == 0) return;
+  (void)cudaGetLastError();
+  const uint64_t want = (npages + 255) / 256;
+  k_pd_state<<<(int)std::min<uint64_t>(want, 148 * 16), 256, 0, s>>>(pd, npages, tab);
 }
 
 // frees of a sorted unit list (Alg. 3's cuMemFree at refCount 0), planned before k_deactivate clears the

@@ -260,6 +260,9 @@ struct Context {
   // page directory over the unit bases (cgcm_dev.h PdDev; built with the table)
   DevBuf pd_ent, pd_ovf, pd_start, pd_meta;
   int pd_nseg = 0;
+  // the entries' page-state words (cgcm_dev.h) must be recomputed before a kernel reads the directory:
+  // set by every change of a unit's ACTIVE / STORAGE / extent (activations, frees, unit ops, rebuilds)
+  bool pd_state_dirty = true;
   uint64_t pd_pages = 0, pd_ovf_pages = 0, pd_bytes = 0;
   uint32_t pd_minP = 0, pd_maxP = 0;
 
@@ -545,12 +548,19 @@ struct Context {
         uint32_t *w = &ent[8 * e];
         w[0] = (uint32_t)i;
         w[1] = cnt | (hb[i] == A ? PD_EXACT : 0u) | (end0 << PD_END_SHIFT);
-        uint16_t *o16 = reinterpret_cast<uint16_t *>(w + 2);
+        w[2] = 0;  // page state: computed on the device (k_pd_state)
         if (cnt <= (uint32_t)PD_K) {
-          for (int t = 0; t < 2 * 6; ++t) o16[t] = t < (int)cnt ? (uint16_t)(hb[i + 1 + t] - A) : (uint16_t)PD_PAD;
+          for (int t = 0; t < PD_K; ++t) {
+            if (t < (int)cnt) {
+              const uint64_t st0 = hb[i + 1 + t] - A, en = std::min<uint64_t>(hb[i + 1 + t] + hs[i + 1 + t] - A, PD_PAD);
+              w[3 + t] = (uint32_t)st0 | ((uint32_t)en << 16);
+            } else {
+              w[3 + t] = PD_PAD;  // start PD_PAD (never <= a clamped p - A), end 0
+            }
+          }
         } else {
-          w[2] = (uint32_t)ovf.size();
-          w[3] = w[4] = w[5] = w[6] = w[7] = 0xFFFFFFFFu;
+          w[3] = (uint32_t)ovf.size();
+          w[4] = w[5] = w[6] = w[7] = 0xFFFFFFFFu;
           for (uint32_t t = 0; t < cnt; ++t) ovf.push_back((uint16_t)(hb[i + 1 + t] - A));
           while (ovf.size() % 16) ovf.push_back((uint16_t)PD_PAD);
           ++novf;
@@ -666,6 +676,7 @@ struct Context {
     U = n;
     CKS(build_index(fwd, hb, n, dbase.as<uint64_t>(), TOPMAX, DIRMAX));
     CKS(build_pd(hb, hs, n));
+    pd_state_dirty = true;
     CK(cudaStreamSynchronize(main));
     table_dirty = false;
     rev_dirty = true;
@@ -789,6 +800,12 @@ struct Context {
     a.copy_list = copy_list.as<uint32_t>();
     a.free_list = free_list.as<uint32_t>();
     a.lenient = (flags & CGCM_LENIENT) ? 1 : 0;
+    if (pd_nseg > 0 && pd_state_dirty) {
+      launch_pd_state(pd_view(), pd_pages, tab(), main);
+      st.kernel_launches += 1;
+      CK(cudaGetLastError());
+      pd_state_dirty = false;
+    }
     const bool pieces = !c.seg_group.empty();
     bool timed = (flags & CGCM_PROFILE) && (timed_fwd || timed_rev) && !pieces;
     if (timed) CK(cudaEventRecord(ev_t0, main));
@@ -944,6 +961,7 @@ struct Context {
              (o.op == UOP_AND_FLAGS && (~o.val & (UF_ACTIVE | UF_STORAGE)));
     launch_unit_ops(uops.as<UnitOp>(), (int)ops.size(), tab(), main, hotc);
     st.kernel_launches += hotc ? 2 : 1;
+    pd_state_dirty = pd_state_dirty || hotc;
     CK(cudaGetLastError());
     return CGCM_OK;
   }
@@ -1133,6 +1151,7 @@ struct Context {
     st.h2d_bytes += bytes;
     st.activations += units.size();
     rev_dirty = true;
+    pd_state_dirty = true;
     return CGCM_OK;
   }
   // ---- device-side transfer planning -----------------------------------------------------------
@@ -1307,6 +1326,7 @@ struct Context {
     st.h2d_bytes += bytes;
     st.activations += n;
     rev_dirty = true;
+    pd_state_dirty = true;
     mirror_stale = true;
     return CGCM_OK;
   }
@@ -1364,6 +1384,7 @@ struct Context {
     }
     st.frees += cnt[0];
     rev_dirty = true;
+    pd_state_dirty = true;
     mirror_stale = true;
     return CGCM_OK;
   }
@@ -1477,6 +1498,7 @@ struct Context {
     CKS(upload(up_units, units));
     launch_deactivate(up_units.as<uint32_t>(), (int)units.size(), tab(), main);
     st.kernel_launches += 1;
+    pd_state_dirty = true;
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(main));
     for (uint32_t x : units) {
@@ -2070,6 +2092,7 @@ int Context::copy_in_with_peers(const std::vector<uint32_t> &units, const std::v
   CK(cudaStreamWaitEvent(main, ev_copy, 0));
   st.activations += units.size();
   rev_dirty = true;
+  pd_state_dirty = true;
   return CGCM_OK;
 }
 
