@@ -721,6 +721,7 @@ struct Context {
     bool dec_red = false;  // OP_DEC through reductions + k_release_scan (large batches)
     bool no_journal = false;  // large gate passes snapshot the rc/epoch columns instead
     bool defer = false;       // deferred references (cgcm_dev.h SlotArgs::defer)
+    bool lazy = false;        // counters into lazy_status (folded when read), not the call's Status block
     std::vector<Seg> segs;
     uint64_t nchunks = 0;
     Status res{};
@@ -793,7 +794,7 @@ struct Context {
     a.no_journal = c.no_journal ? 1 : 0;
     a.defer = c.defer ? 1 : 0;
     a.epoch = rel_epoch(epoch);
-    a.st = status.as<Status>() + st_index;
+    a.st = c.lazy ? lazy_status.as<Status>() : status.as<Status>() + st_index;
     a.lc = lc.as<unsigned long long>();
     a.act_list = act_list.as<uint32_t>();
     a.journal = journal.as<Journal>();
@@ -1154,6 +1155,76 @@ struct Context {
     pd_state_dirty = true;
     return CGCM_OK;
   }
+  // ---- A9 re-map without a host wait -------------------------------------------------------------
+  // Counters of passes whose status nobody waits for accumulate on the device and are folded into the
+  // host statistics when they are read (cgcm_stats) or at the next full call.
+  DevBuf lazy_status;
+  bool lazy_pending = false;
+  int fold_lazy() {
+    if (!lazy_pending) return CGCM_OK;
+    std::vector<Status> v;
+    CKS(download(v, lazy_status, 1));
+    st.fwd_translations += v[0].hits;
+    st.null_slots += v[0].nulls;
+    if (flags & CGCM_LENIENT) st.passthrough += v[0].misses;
+    CK(cudaMemsetAsync(lazy_status.as<void>(), 0, sizeof(Status), main));
+    lazy_pending = false;
+    return CGCM_OK;
+  }
+  // mapArrays whose outers are ALL array-mapped (host mirrors, fresh) with no device storage released
+  // since each was last translated from its host slots (A30): its elements are held by its own slot
+  // references, so the re-map is refcounts only -- +mult per non-null slot through the reverse index
+  // and +mult on the outer -- and cannot fail for a legal program (R13-ii: GPU functions do not store
+  // pointers).  Both kernels are queued without a host wait.  Returns 1 when another path must run.
+  int remap_arrays_async(const uint64_t *ptrs, size_t k, void ***gpu_out) {
+    // (lenient mode: a stray word in the device slots could fall inside another unit's device copy, A18)
+    if (table_dirty || mirror_stale || k > 64 || (flags & CGCM_LENIENT)) return 1;
+    std::vector<std::pair<uint32_t, int>> outs;  // unit, mult
+    std::vector<uint32_t> which(k);
+    for (size_t j = 0; j < k; ++j) {
+      auto it = reg.upper_bound(ptrs[j]);
+      if (it == reg.begin()) return 1;
+      --it;
+      const HostUnit &u = it->second;
+      if (u.idx < 0 || ptrs[j] - it->first > u.size) return 1;
+      const uint32_t x = (uint32_t)u.idx;
+      if (!uarr[x] || !udev[x]) return 1;
+      auto g = arr_gen.find(ubase[x]);
+      if (g == arr_gen.end() || g->second != free_gen) return 1;
+      size_t q = 0;
+      while (q < outs.size() && outs[q].first != x) ++q;
+      if (q == outs.size()) outs.push_back({x, 0});
+      outs[q].second += 1;
+      which[j] = (uint32_t)q;
+    }
+    std::vector<UnitOp> ops;
+    std::vector<Seg> rsegs;
+    for (auto &o : outs) {
+      ops.push_back({o.first, UOP_ADD_RC, (uint64_t)(int64_t)o.second});
+      const uint64_t n = usize[o.first] / 8;
+      if (n) rsegs.push_back(Seg{udev[o.first], n, 0, o.second, 0});
+    }
+    CKS(ensure_rev());
+    CKS(unit_ops(ops));
+    if (!rsegs.empty()) {
+      CKS(dalloc(lazy_status, sizeof(Status) + 256));
+      if (!lazy_pending) CK(cudaMemsetAsync(lazy_status.as<void>(), 0, sizeof(Status), main));
+      CKS(prepare_small());
+      SlotCall R;
+      R.dir = DIR_REV;
+      R.ops = OP_INCPLAIN;
+      R.segs = rsegs;
+      R.lazy = true;
+      CKS(launch(R, 0));
+      lazy_pending = true;
+    }
+    for (size_t j = 0; j < k; ++j) {
+      const uint32_t x = outs[which[j]].first;
+      gpu_out[j] = reinterpret_cast<void **>(udev[x] + (ptrs[j] - ubase[x]));
+    }
+    return CGCM_OK;
+  }
+
   // ---- device-side transfer planning -----------------------------------------------------------
   int need_mirrors() {
     if (!mirror_stale) return CGCM_OK;
@@ -2770,6 +2841,10 @@ int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
 
   if (k == 0) return CGCM_OK;
   if (!arrays || !gpu_out) return CGCM_E_INVALID;
+  {  // the re-map of array-mapped outers in a promoted loop (A9): no host wait at all
+    const int r = C->remap_arrays_async(reinterpret_cast<const uint64_t *>(arrays), k, gpu_out);
+    if (r != 1) return r;  // 1: not that case, take the general path
+  }
   std::vector<PointInfo> infos;
   CKS(C->lookup_points(reinterpret_cast<const uint64_t *>(arrays), k, infos));
   std::vector<Outer> outs;
@@ -3288,11 +3363,13 @@ uint64_t cgcm_epoch(void) {
 int cgcm_stats(cgcm_stats_t *out) {
   CTX();
   if (!out) return CGCM_E_INVALID;
+  CKS(C->fold_lazy());
   *out = C->st;
   return CGCM_OK;
 }
 int cgcm_resetStats(void) {
   CTX();
+  CKS(C->fold_lazy());
   std::memset(&C->st, 0, sizeof(C->st));
   return CGCM_OK;
 }
