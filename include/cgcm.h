@@ -79,6 +79,8 @@ typedef struct {
   /* NEXT-3 coherence groups: activations copied from a peer context's device copy (compared
    * exactly with the oracle), and the device-to-device copies that moved them (reported) */
   uint64_t peer_units, peer_bytes, peer_memcpy_calls;
+  /* NEXT-1: declarations merged into the device table without a rebuild (delta appends) */
+  uint64_t table_merges;
 } cgcm_stats_t;
 
 /* ================================ lifecycle =================================================

@@ -42,7 +42,8 @@ class Stats(C.Structure):
     _fields_ = [(f, C.c_uint64) for f in STAT_FIELDS] + [
         ("fwd_kernel_ms", C.c_double), ("rev_kernel_ms", C.c_double), ("fwd_kernel_calls", C.c_uint64),
         ("rev_kernel_calls", C.c_uint64), ("fwd_kernel_slots", C.c_uint64), ("rev_kernel_slots", C.c_uint64),
-        ("peer_units", C.c_uint64), ("peer_bytes", C.c_uint64), ("peer_memcpy_calls", C.c_uint64)]
+        ("peer_units", C.c_uint64), ("peer_bytes", C.c_uint64), ("peer_memcpy_calls", C.c_uint64),
+        ("table_merges", C.c_uint64)]
 
 
 class IndexInfo(C.Structure):
@@ -325,7 +326,7 @@ class Context:
         self.L.cgcm_stats(C.byref(st))
         d = {f: getattr(st, f) for f in STAT_FIELDS}
         for f in ("fwd_kernel_ms", "rev_kernel_ms", "fwd_kernel_calls", "rev_kernel_calls", "fwd_kernel_slots",
-                  "rev_kernel_slots", "peer_units", "peer_bytes", "peer_memcpy_calls"):
+                  "rev_kernel_slots", "peer_units", "peer_bytes", "peer_memcpy_calls", "table_merges"):
             d[f] = getattr(st, f)
         return d
 

@@ -237,6 +237,11 @@ struct SlotArgs {
   // whose unit is already ACTIVE in the slot's shadow word (SH_DEFER) instead of adding it to rc;
   // k_unmap_sh with defer set drops such a reference on a released hit and adds it to rc otherwise
   int defer;
+  // NEXT-1 delta units (ids >= the main table's): their bases sorted, and their ids; searched only where the
+  // main lookup misses or hits exactly one past the end of its unit (A7)
+  const uint64_t *dkeys;
+  const uint32_t *dids;
+  int dn;
 };
 // shadow unit word: unit index | SH_DEFER (the slot's reference is not in rc yet); SH_NONE: no unit
 constexpr uint32_t SH_NONE = 0xFFFFFFFFu;
@@ -264,7 +269,10 @@ struct GlueArgs {
   const uint64_t *ext_pay;    // host - device delta of each
   const uint32_t *ext_id;     // extent id of each
   int n_ext_keys;
-  int U;
+  int U;                      // units of the sorted main table (delta units: dkeys / dids)
+  const uint64_t *dkeys;
+  const uint32_t *dids;
+  int dn;
 };
 void launch_glue(const GlueArgs &g, cudaStream_t s);
 
@@ -282,7 +290,8 @@ void launch_set_ext(const uint32_t *units, const uint32_t *exts, int n, TableDev
                     cudaStream_t s);
 void launch_deactivate(const uint32_t *units, int n, TableDev tab, cudaStream_t s);
 void launch_restore_epochs(const Journal *j, int n, TableDev tab, cudaStream_t s);
-void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n, PointInfo *out, cudaStream_t s);
+void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n, PointInfo *out,
+                          const uint64_t *dkeys, const uint32_t *dids, int dn, cudaStream_t s);
 void launch_release_scan(TableDev tab, int n, Status *st, unsigned long long *lc, uint32_t *free_list,
                          cudaStream_t s);
 void launch_rebase_epochs(TableDev tab, int n, uint32_t cur, cudaStream_t s);

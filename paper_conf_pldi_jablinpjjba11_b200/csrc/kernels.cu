@@ -344,6 +344,37 @@ __device__ __forceinline__ void cnt_max2(uint32_t w, uint32_t rr, uint32_t &cnt,
   mx = __vmaxu2(mx, w & m);
 }
 
+// ---- NEXT-1 delta units ---------------------------------------------------------------------------
+// The delta unit with the greatest base <= q that contains q (A7: q - base <= size), or -1; base out.
+__device__ __noinline__ int delta_hit(const uint64_t *dk, const uint32_t *di, int dn, const TableDev &tab, uint64_t q,
+                                      uint64_t &base) {
+  if (dn <= 0 || q < dk[0]) return -1;
+  int lo = 0, len = dn;
+  while (len > 1) {
+    const int half = len >> 1;
+    if (dk[lo + half] <= q) lo += half;
+    len -= half;
+  }
+  const uint32_t id = di[lo];
+  const uint64_t b = dk[lo];
+  uint64_t sz = hot_size32(tab.hot[id]);
+  if (sz == BIG_SIZE) sz = tab.size64[id];
+  if (q - b > sz) return -1;
+  base = b;
+  return (int)id;
+}
+// After the main table's lookup of q: hit (unit j, main_base its base when known) -- the delta unit that
+// greatestLTE picks instead, if any: any delta unit containing q when the main table missed, or one
+// starting exactly at q when q is one past the end of the main hit (A7: the larger base wins).
+__device__ __forceinline__ int delta_override(const SlotArgs &a, uint64_t q, bool hit, bool at_end, uint64_t &base) {
+  if (a.dn <= 0 || (hit && !at_end)) return -1;
+  uint64_t b = 0;
+  const int d = delta_hit(a.dkeys, a.dids, a.dn, a.tab, q, b);
+  if (d < 0 || (hit && b != q)) return -1;
+  base = b;
+  return d;
+}
+
 // #{starts <= r} among an entry's (at most PD_K = 5) candidates, and the candidate word (start | end << 16)
 // of the last of them (k > 0).  The 64-bit words e[1..3] hold w[2..7]: lane 2 of e[1] and lanes 0, 2 of
 // e[2], e[3] are starts; per lane 0x8000 + r - x keeps bit 15 iff x <= r and never borrows into the next
@@ -728,6 +759,29 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         }
       }
     }
+    if (a.dn > 0) {  // NEXT-1: delta units (q: the host address looked up; 0 if none)
+#pragma unroll
+      for (int m = 0; m < 2; ++m) {
+        if (q[m] == 0 || sh[m] || !((valid >> m) & 1)) continue;
+        bool at_end = false;
+        if (hit[m]) {
+          uint64_t sz = hot_size32(hw[m]);
+          if (sz == BIG_SIZE) sz = a.tab.size64[j[m]];
+          at_end = q[m] - a.tab.base[j[m]] == sz;
+        }
+        uint64_t db;
+        const int d = delta_override(a, q[m], hit[m], at_end, db);
+        if (d < 0) continue;
+        const uint64_t h2 = a.tab.hot[d];
+        // a reverse lookup: the unit must own the extent's copy (active, its copy in that extent)
+        if (DIR == DIR_REV && !((hot_flags(h2) & UF_ACTIVE) && hot_ext(h2) == rid[m])) continue;
+        hit[m] = true;
+        j[m] = d;
+        key[m] = db;
+        hw[m] = h2;
+        if (OPS & OP_GATE) rw[m] = a.tab.st[d];
+      }
+    }
     if (SH && DIR == DIR_REV) {
 #pragma unroll
       for (int m = 0; m < 2; ++m)
@@ -1000,8 +1054,18 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
       uint64_t sz = hot_size32(hw[m]);
-      if (look[m] && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
+      if (look[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
       hit[m] = look[m] && (k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
+      if (a.dn > 0 && ((valid >> m) & 1) && cv[m] != 0) {  // NEXT-1: delta units
+        const bool at_end = hit[m] && cv[m] - a.tab.base[j[m]] == sz;
+        uint64_t db;
+        const int d = delta_override(a, cv[m], hit[m], at_end, db);
+        if (d >= 0) {
+          j[m] = d;
+          hw[m] = a.tab.hot[d];
+          hit[m] = look[m] = true;
+        }
+      }
     }
     // deferred reference (a.defer, SH): the unit was ACTIVE when the call began, so a reference held
     // elsewhere keeps it active until the runtime materialises this one -- the slot's
@@ -1480,7 +1544,7 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
     // decode: j = j0 + #{starts <= p - A}; j0 is decided by its end, a candidate by its end in the entry
     // (A7); in a page whose state is valid the entry also gives ACTIVE and the extent: no unit word
     int j[2];
-    bool k0[2], dec[2];
+    bool k0[2], dec[2], ae[2];  // ae: the hit may sit exactly one past its unit's end (NEXT-1 delta units)
     uint64_t key[2];
     uint32_t cw[2], ps[2];
 #pragma unroll
@@ -1488,6 +1552,7 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
       j[m] = fc.jt[m];
       k0[m] = true;
       dec[m] = false;
+      ae[m] = fc.jt[m] >= 0 && cv[m] == Send;
       key[m] = 0;
       ps[m] = 0;
       if (fc.ok[m]) {
@@ -1498,6 +1563,7 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
           uint32_t word;
           const uint32_t k = pd_count5(fc.ew[m], r, word);
           const bool h = k ? fc.poff[m] <= (word >> 16) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0);
+          ae[m] = h && (k ? fc.poff[m] == (word >> 16) : fc.poff[m] + 1 == end0);
           j[m] = h ? (int)(j0 + k) : -1;
           dec[m] = true;
           ps[m] = (uint32_t)fc.ew[m][1];
@@ -1506,6 +1572,7 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
           const uint32_t k = (uint32_t)ko, off = (uint32_t)(ko >> 32);
           k0[m] = k == 0;
           j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
+          ae[m] = k == 0 && fc.poff[m] + 1 == end0;
           key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
         }
       }
@@ -1527,7 +1594,17 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
         hw = (cw[m] & HOTC_ESC) && look ? ld_u64_hot(a.tab.hot + j[m], pol_t) : hot_of_hotc(cw[m]);
       uint64_t sz = hot_size32(hw);
       if (look && !dec[m] && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
-      const bool hit = look && (dec[m] || k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
+      bool hit = look && (dec[m] || k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
+      if (a.dn > 0 && vm && cv[m] != 0) {  // NEXT-1: delta units (a warp-uniform branch)
+        const bool at_end = ae[m] || (look && !dec[m] && !k0[m] && cv[m] - key[m] == sz);
+        uint64_t db;
+        const int d = delta_override(a, cv[m], hit, at_end, db);
+        if (d >= 0) {
+          j[m] = d;
+          hw = ld_u64_hot(a.tab.hot + d, pol_t);
+          hit = true;
+        }
+      }
       const bool nul = vm && cv[m] == 0;
       c_nulls += nul;
       c_hits += hit;
@@ -2373,7 +2450,8 @@ void launch_rebase_epochs(TableDev tab, int n, uint32_t cur, cudaStream_t s) {
 
 // outer-pointer lookup for mapArray/unmapArray/releaseArray: one thread per pointer, plain
 // binary search over the full u64 key array (few pointers: latency, not bandwidth)
-__global__ void k_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n, PointInfo *out) {
+__global__ void k_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n, PointInfo *out,
+                                const uint64_t *dkeys, const uint32_t *dids, int dn) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   uint64_t p = ptrs[i];
@@ -2391,9 +2469,19 @@ __global__ void k_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs,
       if (ix.keys[lo + half] <= p) lo += half;
       len -= half;
     }
-    const uint64_t h = tab.hot[lo], b = ix.keys[lo], sz = tab.size64[lo];
-    if (p - b <= sz) {
-      r.unit = lo;
+    const uint64_t b = ix.keys[lo], sz = tab.size64[lo];
+    if (p - b <= sz) r.unit = lo;
+  }
+  {  // NEXT-1: a delta unit containing p when the main table missed, or starting at p after a main unit
+    uint64_t db = 0;
+    const int d = (dn > 0 && (r.unit < 0 || p - ix.keys[r.unit] == tab.size64[r.unit]))
+                      ? delta_hit(dkeys, dids, dn, tab, p, db) : -1;
+    if (d >= 0 && (r.unit < 0 || db == p)) r.unit = d;
+  }
+  if (r.unit >= 0) {
+    const int lo = r.unit;
+    const uint64_t h = tab.hot[lo], b = tab.base[lo], sz = tab.size64[lo];
+    {
       r.base = b;
       r.size = sz;
       r.flags = hot_flags(h);
@@ -2404,10 +2492,11 @@ __global__ void k_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs,
   }
   out[i] = r;
 }
-void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n, PointInfo *out, cudaStream_t s) {
+void launch_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs, int n, PointInfo *out,
+                          const uint64_t *dkeys, const uint32_t *dids, int dn, cudaStream_t s) {
   if (n > 0) {
     (void)cudaGetLastError();
-    k_lookup_points<<<(n + 127) / 128, 128, 0, s>>>(ix, tab, ptrs, n, out);
+    k_lookup_points<<<(n + 127) / 128, 128, 0, s>>>(ix, tab, ptrs, n, out, dkeys, dids, dn);
   }
 }
 
@@ -2424,17 +2513,24 @@ __device__ bool glue_ok(const GlueArgs &A, uint64_t g) {
   }
   const uint64_t h = g + A.ext_pay[lo];
   const uint32_t eid = A.ext_id[lo];
-  if (A.U <= 0 || h < A.tab.base[0]) return false;
-  int j = 0;
-  len = A.U;
-  while (len > 1) {
-    const int half = len >> 1;
-    if (A.tab.base[j + half] <= h) j += half;
-    len -= half;
+  auto owns = [&](int j) {
+    const uint64_t w = A.tab.hot[j];
+    return (hot_flags(w) & UF_ACTIVE) && (hot_flags(w) & UF_STORAGE) && hot_ext(w) == eid &&
+           h - A.tab.base[j] <= A.tab.size64[j] && A.tab.size64[j] - (h - A.tab.base[j]) >= 8;
+  };
+  if (A.U > 0 && h >= A.tab.base[0]) {
+    int j = 0;
+    len = A.U;
+    while (len > 1) {
+      const int half = len >> 1;
+      if (A.tab.base[j + half] <= h) j += half;
+      len -= half;
+    }
+    if (owns(j)) return true;
   }
-  const uint64_t w = A.tab.hot[j];
-  return (hot_flags(w) & UF_ACTIVE) && (hot_flags(w) & UF_STORAGE) && hot_ext(w) == eid &&
-         h - A.tab.base[j] <= A.tab.size64[j] && A.tab.size64[j] - (h - A.tab.base[j]) >= 8;
+  uint64_t db;  // NEXT-1: the delta units
+  const int d = delta_hit(A.dkeys, A.dids, A.dn, A.tab, h, db);
+  return d >= 0 && owns(d);
 }
 __global__ void k_glue(GlueArgs A) {
   uint64_t r[GLUE_REGS];

@@ -251,7 +251,21 @@ struct Context {
   std::vector<uint8_t> uarr;                 // mirror of UF_ARRAYMAPPED
   std::unordered_set<std::string> names;
   bool table_dirty = true, rev_dirty = true;
-  int U = 0;  // units in the device table
+  int U = 0;  // units in the device table (ids [0, U))
+  // NEXT-1 batched merge: up to DELTA_MAX declarations between two calls are appended to the device table
+  // as "delta" units (ids [Umain, U)) instead of a rebuild; the sorted main table (ids [0, Umain), base
+  // order) keeps its index and page directory, and the kernels search the small sorted delta index only
+  // where the main table misses or hits exactly one past the end of a unit (A7).  An undeclare of a unit
+  // in the device table, or too many delta units, makes the next merge a full rebuild.
+  static constexpr int DELTA_MAX = 4096;
+  int Umain = 0;
+  std::vector<uint64_t> pend;   // bases declared since the last merge, not in the device table yet
+  bool pend_over = false;       // more than DELTA_MAX of them
+  bool dirty_del = false;       // a unit of the device table was undeclared
+  std::vector<uint64_t> dk;     // delta index on the host: bases (sorted) ...
+  std::vector<uint32_t> di;     // ... and ids
+  DevBuf dkeys, dids;
+  size_t col_cap = 0;           // units the device table columns have room for
 
   // device table
   DevBuf hotb, hotcb, stb, rcb, size64, dbase, extd, snap_st, snap_rc;  // unit table columns + extent deltas
@@ -590,10 +604,81 @@ struct Context {
     return p;
   }
 
+  void note_declared(uint64_t b) {
+    if (pend_over) return;
+    if (pend.size() >= (size_t)DELTA_MAX) {
+      pend_over = true;
+      pend.clear();
+    } else {
+      pend.push_back(b);
+    }
+  }
+  // the batched merge of pending declarations (NEXT-1): append them to the columns as delta units and
+  // re-sort the small delta index -- O(#pending + #delta) host work, no registry walk, no rebuild
+  int append_delta() {
+    Trace trace_("ensure_table(delta)");
+    std::sort(pend.begin(), pend.end());
+    const size_t t = pend.size();
+    std::vector<uint64_t> nb(t), ns(t), nh(t), nst(t);
+    std::vector<uint32_t> nhc(t);
+    std::vector<int32_t> nrc(t, 0);
+    for (size_t q = 0; q < t; ++q) {
+      auto it = reg.find(pend[q]);
+      HostUnit &u = it->second;
+      const uint32_t id = (uint32_t)(U + q);
+      u.idx = (int32_t)id;
+      const uint32_t fl = u.flags & (UF_GLOBAL | UF_READONLY);
+      nb[q] = pend[q];
+      ns[q] = u.size;
+      nh[q] = make_hot(u.size, NO_EXT, fl);
+      nhc[q] = make_hotc(nh[q]);
+      nst[q] = make_st(nh[q], rel_epoch(u.epoch0));
+      ubase.push_back(pend[q]);
+      usize.push_back(u.size);
+      uflags.push_back(fl);
+      usym.push_back(u.sym);
+      udev.push_back(0);
+      urun.push_back(-1);
+      uarr.push_back(0);
+      dk.push_back(pend[q]);
+      di.push_back(id);
+    }
+    if (t) {
+      CKS(ring_put(dbase.as<uint64_t>() + U, nb.data(), 8 * t));
+      CKS(ring_put(size64.as<uint64_t>() + U, ns.data(), 8 * t));
+      CKS(ring_put(hotb.as<uint64_t>() + U, nh.data(), 8 * t));
+      CKS(ring_put(hotcb.as<uint32_t>() + U, nhc.data(), 4 * t));
+      CKS(ring_put(stb.as<uint64_t>() + U, nst.data(), 8 * t));
+      CKS(ring_put(rcb.as<int32_t>() + U, nrc.data(), 4 * t));
+    }
+    // the delta index, sorted by base
+    std::vector<size_t> ord(dk.size());
+    for (size_t q = 0; q < ord.size(); ++q) ord[q] = q;
+    std::sort(ord.begin(), ord.end(), [&](size_t x, size_t y) { return dk[x] < dk[y]; });
+    std::vector<uint64_t> k2(ord.size());
+    std::vector<uint32_t> i2(ord.size());
+    for (size_t q = 0; q < ord.size(); ++q) {
+      k2[q] = dk[ord[q]];
+      i2[q] = di[ord[q]];
+    }
+    dk.swap(k2);
+    di.swap(i2);
+    CKS(upload(dkeys, dk));
+    CKS(upload(dids, di));
+    U += (int)t;
+    pend.clear();
+    table_dirty = false;
+    st.table_merges += 1;
+    return CGCM_OK;
+  }
+
   // merge pending declares/undeclares into the device table (A19: kernels only see a compacted table)
   int ensure_table() {
     Trace trace_("ensure_table");
     if (!table_dirty) return CGCM_OK;
+    if (!dirty_del && !pend_over && Umain > 0 && dk.size() + pend.size() <= (size_t)DELTA_MAX &&
+        (size_t)U + pend.size() <= col_cap)
+      return append_delta();
     CKS(materialise_all());  // deferred references name units by their index in the table being replaced
     CKS(need_mirrors());     // the remap carries the per-unit host mirrors to the new indices
     int n = (int)reg.size();
@@ -635,7 +720,7 @@ struct Context {
     urun.swap(nrun);
     uarr.swap(narr);
     DevBuf nhot, nhotc, nst, nrc, nsize, nbase, tmp;
-    int cap = std::max(n, 1);
+    int cap = std::max(n, 1) + DELTA_MAX;  // room for delta units appended by later merges
     CKS(dalloc(nhot, 8 * (size_t)cap + 64));
     CKS(dalloc(nhotc, 4 * (size_t)cap + 64));
     CKS(dalloc(nst, 8 * (size_t)cap + 64));
@@ -674,6 +759,13 @@ struct Context {
     size64 = nsize;
     dbase = nbase;
     U = n;
+    Umain = n;
+    col_cap = (size_t)cap;
+    pend.clear();
+    pend_over = false;
+    dirty_del = false;
+    dk.clear();
+    di.clear();
     CKS(build_index(fwd, hb, n, dbase.as<uint64_t>(), TOPMAX, DIRMAX));
     CKS(build_pd(hb, hs, n));
     pd_state_dirty = true;
@@ -774,6 +866,9 @@ struct Context {
     a.fx = fwd.view(dbase.as<uint64_t>());
     a.fx_nowide = fwd.any_wide ? 0 : 1;
     a.pd = pd_view();
+    a.dkeys = dkeys.as<uint64_t>();
+    a.dids = dids.as<uint32_t>();
+    a.dn = (int)dk.size();
     if (c.dir == DIR_REV) {
       a.rx = rev.view(rev.keys.as<uint64_t>());
       a.runpay = rev.pay.as<uint64_t>();
@@ -2033,7 +2128,7 @@ struct Context {
     CKS(upload(this->ptrs, v));
     CKS(dalloc(points, sizeof(PointInfo) * k + 64));
     launch_lookup_points(fwd.view(dbase.as<uint64_t>()), tab(), this->ptrs.as<uint64_t>(), (int)k,
-                         points.as<PointInfo>(), main);
+                         points.as<PointInfo>(), dkeys.as<uint64_t>(), dids.as<uint32_t>(), (int)dk.size(), main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
     CKS(download(out, points, k));
@@ -2412,6 +2507,7 @@ static int declare_one(Context *C, uint64_t b, uint64_t s, uint32_t fl, const ch
   u.sym = sym;
   C->reg.emplace_hint(succ, b, u);
   C->table_dirty = true;
+  C->note_declared(b);
   return CGCM_OK;
 }
 
@@ -2451,6 +2547,7 @@ int cgcm_declareBatch(void *const *bases, const size_t *sizes, size_t n, unsigne
     u.epoch0 = C->epoch;
     hint = C->reg.lower_bound(B(ord[q]));
     hint = C->reg.emplace_hint(hint, B(ord[q]), u);
+    C->note_declared(B(ord[q]));
   }
   if (n) C->table_dirty = true;
   return CGCM_OK;
@@ -2505,6 +2602,12 @@ int cgcm_undeclare(void *base) {
     }
   }
   C->arr_gen.erase(b);
+  if (u.idx >= 0) {
+    C->dirty_del = true;  // the device table changes shape: the next merge rebuilds it
+  } else {                // declared and undeclared between two merges: never in the device table
+    auto pe = std::find(C->pend.begin(), C->pend.end(), b);
+    if (pe != C->pend.end()) C->pend.erase(pe);
+  }
   C->reg.erase(it);
   C->table_dirty = true;
   return CGCM_OK;
@@ -3398,9 +3501,14 @@ int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
     CKS(C->download(rcs, C->rcb, (size_t)C->U));
   }
   CKS(C->download(szs, C->size64, (size_t)C->U));
+  // in base order: the registry's order (delta units sit at ids >= Umain, NEXT-1)
+  std::vector<uint32_t> order;
+  order.reserve(C->U);
+  for (auto &kv : C->reg) order.push_back((uint32_t)kv.second.idx);
   size_t m = std::min(cap, (size_t)C->U);
-  for (size_t i = 0; i < m; ++i) {
-    cgcm_unit_t &u = out[i];
+  for (size_t q = 0; q < m; ++q) {
+    const size_t i = order[q];
+    cgcm_unit_t &u = out[q];
     const uint32_t fl = hot_flags(hots[i]);
     u.base = C->ubase[i];
     u.size = szs[i];
@@ -3464,7 +3572,10 @@ int cgcm_launchGlue(const cgcm_glue_op_t *prog, size_t n, const void *const *cpu
   g.ext_pay = C->rev.pay.as<uint64_t>();
   g.ext_id = C->rev.rid.as<uint32_t>();
   g.n_ext_keys = (int)C->live_runs.size();
-  g.U = C->U;
+  g.U = C->Umain;
+  g.dkeys = C->dkeys.as<uint64_t>();
+  g.dids = C->dids.as<uint32_t>();
+  g.dn = (int)C->dk.size();
   launch_glue(g, C->main);
   C->st.kernel_launches += 1;
   CK(cudaGetLastError());
