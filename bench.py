@@ -196,6 +196,7 @@ def run_cgcm(args, rank, world, local_rank):
     ms_per_step = ms / args.steps
     parity = full_size_check(ctx, wl, q, q_ref, q_unit, pins_held=1)
     del q_unit
+    merge = declares_between_batches(ctx, step, reps=min(16, args.steps))
     translations = 2 * wl.n * world * args.steps
     value = translations / (ms / 1e3)
 
@@ -259,11 +260,48 @@ def run_cgcm(args, rank, world, local_rank):
                    "exceed L2 between iterations; table stays L2-resident by design",
                    "translations_per_step": 2 * wl.n * world},
         "roofline": roofline, "gpu_launches": gpu_launches, "clocks": clocks, "e2e": e2e, "parity": parity,
+        "merge": merge,
         "setup_s": round(setup_s, 1), "setup_activation_s": round(setup_act_s, 1),
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         result["cpu_baseline"] = cpu_baseline(wl, args.cpu_sample, steps=3)
     return result
+
+
+def declares_between_batches(ctx, step, reps):
+    """NEXT-1: the cost of keeping the table current while map batches run -- one new AU declared
+    between every two steps of the timed workload (merged into the device table as a delta unit, no
+    rebuild), vs the same steps without declarations; CUDA events around each run."""
+    import torch
+    span = 1 << 20
+    R = W.reserve_readonly(span)
+    try:
+        def run(declare):
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            ev0.record(ctx.main)
+            for k in range(reps):
+                if declare:
+                    assert ctx.declareAlloc(R + 4096 * run.n, 1024, True) == 0
+                    run.n += 1
+                step()
+            ev1.record(ctx.main)
+            torch.cuda.synchronize()
+            return ev0.elapsed_time(ev1), time.perf_counter() - t0
+        run.n = 0
+        s0 = ctx.stats()
+        base_ms, base_wall = run(False)
+        with_ms, with_wall = run(True)
+        s1 = ctx.stats()
+        return {"declares": reps, "ms_per_step_without": round(base_ms / reps, 4),
+                "ms_per_step_with_one_declare": round(with_ms / reps, 4),
+                "us_per_declare_between_batches": round(1e3 * max(0.0, with_wall - base_wall) / reps, 1),
+                "declares_per_s_with_batches": round(reps / max(1e-9, with_wall), 1),
+                "table_merges": s1["table_merges"] - s0["table_merges"],
+                "table_rebuilds": s1["table_rebuilds"] - s0["table_rebuilds"]}
+    finally:
+        pass
 
 
 def full_size_check(ctx, wl, q, q_ref, q_unit, pins_held):
