@@ -28,6 +28,8 @@ struct TableDev {
   const uint64_t *base;
   const uint64_t *size64;
   const uint64_t *ext_delta;
+  const uint64_t *ext_lo;   // device start of every extent's range
+  const uint32_t *ext_len;  // its length (0: 4 GiB or more -- shadows of units in it always take the slow path)
   int n_ext;
 };
 
@@ -149,7 +151,7 @@ struct PdDev {
 
 // One input segment of a slot kernel: n u64 slots at device address ptr (8-byte aligned),
 // translated in place (out == 0) or into out.  inc = refcount delta per non-null slot.
-// shadow (optional, 12 B per slot: u64 CPU pointer[n] then u32 unit[n]): written by the forward map,
+// shadow (optional, 8 B per slot: make_shw(CPU pointer, unit word)): written by the forward map,
 // read by the reverse unmap of the same slots -- GPU functions do not store pointers (R13-ii,
 // P:L140-142), so an unchanged slot reverses to its recorded CPU pointer after one check.
 struct Seg {
@@ -243,9 +245,17 @@ struct SlotArgs {
   const uint32_t *dids;
   int dn;
 };
-// shadow unit word: unit index | SH_DEFER (the slot's reference is not in rc yet); SH_NONE: no unit
+// Forward-map shadow (8 B per slot): the low 32 bits of the slot's CPU pointer | the unit word << 32.  The
+// unit word is unit index | SH_DEFER (the slot's reference is not in rc yet); SH_NONE: no unit.  A reverse
+// pass accepts a slot g as unchanged iff g lies in the device range of the unit's extent e (shorter than
+// 4 GiB) and g - delta(e) has the recorded low 32 bits: both g - delta(e) and the recorded pointer lie in
+// e's host span, which is shorter than 2^32, so the two are equal and g - delta(e) is the CPU pointer.
 constexpr uint32_t SH_NONE = 0xFFFFFFFFu;
 constexpr uint32_t SH_DEFER = 0x80000000u;
+__host__ __device__ __forceinline__ uint64_t make_shw(uint64_t p, uint32_t uw) {
+  return (p & 0xFFFFFFFFull) | ((uint64_t)uw << 32);
+}
+__host__ __device__ __forceinline__ uint32_t shw_unit(uint64_t w) { return (uint32_t)(w >> 32); }
 __host__ __device__ __forceinline__ uint32_t sh_unit(uint32_t w) { return w == SH_NONE ? SH_NONE : (w & ~SH_DEFER); }
 __host__ __device__ __forceinline__ bool sh_deferred(uint32_t w) { return w != SH_NONE && (w & SH_DEFER); }
 
@@ -338,7 +348,7 @@ void launch_pd_state(PdDev pd, uint64_t npages, TableDev tab, cudaStream_t s);
 // out[i] = st[idx[i]] (epoch | extent | flags) of n units (NEXT-3 peer-source queries)
 void launch_gather_state(TableDev tab, const uint32_t *idx, int n, uint64_t *out, cudaStream_t s);
 // add every deferred reference recorded in a shadow's n unit words to rc (they become ordinary references)
-void launch_materialise(const uint32_t *shadow_units, uint64_t n, int32_t *rc, cudaStream_t s);
+void launch_materialise(const uint64_t *shadow, uint64_t n, int32_t *rc, cudaStream_t s);
 // small host<->device transfers by a kernel through mapped pinned memory instead of a DMA: a copy
 // engine serves DMAs in order, so a few bytes queued behind another context's gigabyte would wait for it
 void launch_copy_small(void *dst, const void *src, size_t n, void *dst2, const void *src2, size_t n2, cudaStream_t s);

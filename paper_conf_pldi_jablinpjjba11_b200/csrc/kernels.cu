@@ -344,6 +344,14 @@ __device__ __forceinline__ void cnt_max2(uint32_t w, uint32_t rr, uint32_t &cnt,
   mx = __vmaxu2(mx, w & m);
 }
 
+// ---- forward-map shadows (cgcm_dev.h make_shw) ----------------------------------------------------
+// The CPU pointer an unchanged slot g reverses to, given its recorded shadow word and the unit's extent e
+// (lo/len: the extent's device range), or 0 when g is not provably the recorded pointer's translation.
+__device__ __forceinline__ uint64_t sh_reverse(uint64_t g, uint64_t shw, uint64_t delta, uint64_t lo, uint32_t len) {
+  const uint64_t h = g - delta;  // mirrored layout: host = device - (devbase - base)
+  return (g - lo < (uint64_t)len && (uint32_t)h == (uint32_t)shw) ? h : 0ull;
+}
+
 // ---- NEXT-1 delta units ---------------------------------------------------------------------------
 // The delta unit with the greatest base <= q that contains q (A7: q - base <= size), or -1; base out.
 __device__ __noinline__ int delta_hit(const uint64_t *dk, const uint32_t *di, int dn, const TableDev &tab, uint64_t q,
@@ -671,13 +679,16 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
         if (!look[m]) continue;
         const int64_t i = slot0 + m;
         // (a deferred reference was materialised by k_unmap_sh or the runtime before this pass)
-        const uint32_t u = sh_unit(reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n)[i]);
+        const uint64_t shw = reinterpret_cast<const uint64_t *>(sg.shadow)[i];
+        const uint32_t u = sh_unit(shw_unit(shw));
         if (u == SH_NONE) continue;
-        const uint64_t h = reinterpret_cast<const uint64_t *>(sg.shadow)[i];
         const uint64_t w = ld_u64(a.tab.st + u, pol_t);  // extent, flags and epoch in one word
         const uint32_t e = hot_ext(w);
-        if ((hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext &&
-            q[m] == h + (ext_s ? s_ext[e] : a.tab.ext_delta[e])) {
+        const uint64_t h = (hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext
+                               ? sh_reverse(q[m], shw, ext_s ? s_ext[e] : a.tab.ext_delta[e], a.tab.ext_lo[e],
+                                            a.tab.ext_len[e])
+                               : 0ull;
+        if (h) {
           sh[m] = true;
           jsh[m] = (int)u;
           hsh[m] = h;
@@ -797,8 +808,7 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
       for (int m = 0; m < 2; ++m) {
         if (!((valid >> m) & 1)) continue;
         const int64_t i = slot0 + m;
-        reinterpret_cast<uint64_t *>(sg.shadow)[i] = v[m];
-        reinterpret_cast<uint32_t *>(sg.shadow + 8 * sg.n)[i] = hit[m] ? (uint32_t)j[m] : 0xFFFFFFFFu;
+        reinterpret_cast<uint64_t *>(sg.shadow)[i] = make_shw(v[m], hit[m] ? (uint32_t)j[m] : SH_NONE);
       }
     }
     // epoch (gate): from the record gathered with the hot word; refcount (unmap check) where needed
@@ -1075,21 +1085,14 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
     for (int m = 0; m < 2; ++m) dfr[m] = SH && a.defer && hit[m] && (hot_flags(hw[m]) & UF_ACTIVE);
     if (SH && live) {  // forward-map shadow: (CPU pointer, unit) per slot for the reverse pass
       uint64_t *shp = reinterpret_cast<uint64_t *>(sg.shadow);
-      uint32_t *shu = reinterpret_cast<uint32_t *>(sg.shadow + 8 * sg.n);
       const uint32_t u0 = hit[0] ? ((uint32_t)j[0] | (dfr[0] ? SH_DEFER : 0u)) : SH_NONE;
       const uint32_t u1 = hit[1] ? ((uint32_t)j[1] | (dfr[1] ? SH_DEFER : 0u)) : SH_NONE;
       if (valid == 3u && !(slot0 & 1)) {
-        st_stream2(shp + slot0, pol_s, cv[0], cv[1]);
-        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1,%2}, %3;" ::"l"(shu + slot0), "r"(u0),
-                     "r"(u1), "l"(pol_s)
-                     : "memory");
+        st_stream2(shp + slot0, pol_s, make_shw(cv[0], u0), make_shw(cv[1], u1));
       } else {
 #pragma unroll
         for (int m = 0; m < 2; ++m)
-          if ((valid >> m) & 1) {
-            shp[slot0 + m] = cv[m];
-            shu[slot0 + m] = m ? u1 : u0;
-          }
+          if ((valid >> m) & 1) shp[slot0 + m] = make_shw(cv[m], m ? u1 : u0);
       }
     }
     uint64_t outv[2] = {cv[0], cv[1]};
@@ -1244,22 +1247,18 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
     if (!x.valid) return;
     ld_stream2(reinterpret_cast<const void *>(a0), pol_s, x.g[0], x.g[1]);
     if (!sg.shadow) return;
-    const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);
-    const uint32_t *shu = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n);
+    const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);  // shadow words (make_shw)
     const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
     if (x.valid == 3u && !(i0 & 1)) {
       ld_stream2(shp + i0, pol_s, x.h[0], x.h[1]);
-      asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
-                   : "=r"(x.u[0]), "=r"(x.u[1])
-                   : "l"(shu + i0), "l"(pol_s));
     } else {
 #pragma unroll
       for (int m = 0; m < 2; ++m)
-        if ((x.valid >> m) & 1) {
-          x.h[m] = shp[i0 + m];
-          x.u[m] = shu[i0 + m];
-        }
+        if ((x.valid >> m) & 1) x.h[m] = shp[i0 + m];
     }
+#pragma unroll
+    for (int m = 0; m < 2; ++m)
+      if ((x.valid >> m) & 1) x.u[m] = shw_unit(x.h[m]);
   };
   // the state words (epoch | extent | flags) of the recorded units of x
   auto gather = [&](const In &x, uint64_t w[2]) {
@@ -1290,8 +1289,11 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
       const uint64_t w = cw[m];
       const uint32_t e = hot_ext(w);
       const uint32_t su = sh_unit(cur.u[m]);
-      hit[m] = look && su != SH_NONE && (hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext &&
-               cur.g[m] == cur.h[m] + (ext_s ? s_ext[e] : a.tab.ext_delta[e]);
+      const uint64_t hr = look && su != SH_NONE && (hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext
+                              ? sh_reverse(cur.g[m], cur.h[m], ext_s ? s_ext[e] : a.tab.ext_delta[e],
+                                           a.tab.ext_lo[e], a.tab.ext_len[e])
+                              : 0ull;
+      hit[m] = hr != 0;
       slow[m] = look && !hit[m];
       c_nulls += vm && cur.g[m] == 0;
       c_hits += hit[m];
@@ -1344,7 +1346,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
         if (cp) a.copy_list[cx] = unit;
       }
       if ((OPS & OP_WRITE) && hit[m]) {
-        outv[m] = cur.h[m];  // reverse: base + (g - devbase), the recorded CPU pointer
+        outv[m] = hr;  // reverse: base + (g - devbase), the recorded CPU pointer
         wrote |= 1u << m;
       }
     }
@@ -1484,8 +1486,7 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
   const int lane = threadIdx.x & 31;
   const Seg sg = a.segs[0];
   const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n;
-  uint64_t *shp = reinterpret_cast<uint64_t *>(sg.shadow);
-  uint32_t *shu = reinterpret_cast<uint32_t *>(sg.shadow + 8 * sg.n);
+  uint64_t *shp = reinterpret_cast<uint64_t *>(sg.shadow);  // shadow words (make_shw)
   // the directory's one segment: first base, end of its last unit, first entry, pages, page shift, last unit
   const uint64_t S0 = a.pd.seg_start[0], Send = a.pd.seg_start[1];
   const uint32_t P = a.pd.seg_meta[2], npages = a.pd.seg_meta[1], lastu = a.pd.seg_meta[3];
@@ -1641,24 +1642,17 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
     if (valid == 3u) {
       st_stream2(reinterpret_cast<void *>(a0), pol_s, outv[0], outv[1]);
       if (!(i0 & 1)) {
-        st_stream2(shp + i0, pol_s, cv[0], cv[1]);
-        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1,%2}, %3;" ::"l"(shu + i0), "r"(su[0]),
-                     "r"(su[1]), "l"(pol_s)
-                     : "memory");
+        st_stream2(shp + i0, pol_s, make_shw(cv[0], su[0]), make_shw(cv[1], su[1]));
       } else {
 #pragma unroll
-        for (int m = 0; m < 2; ++m) {
-          shp[i0 + m] = cv[m];
-          shu[i0 + m] = su[m];
-        }
+        for (int m = 0; m < 2; ++m) shp[i0 + m] = make_shw(cv[m], su[m]);
       }
     } else if (valid) {
 #pragma unroll
       for (int m = 0; m < 2; ++m)
         if ((valid >> m) & 1) {
           st_stream1(reinterpret_cast<void *>(a0 + 8ull * m), pol_s, outv[m]);
-          shp[i0 + m] = cv[m];
-          shu[i0 + m] = su[m];
+          shp[i0 + m] = make_shw(cv[m], su[m]);
         }
     }
     {  // hit mask: 2 bits per chunk, 16 chunks per word (lanes 0-15: word cb/16, lanes 16-31: the next)
@@ -1716,17 +1710,23 @@ constexpr int REV_LEAN_THREADS = 768;
 template <bool DEC, bool ES>  // ES: the extent deltas are staged in shared memory
 __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
+  // the extents' deltas and device ranges (the shadow check), staged when few
   uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
+  uint64_t *s_lo = s_ext + (ES ? a.tab.n_ext : 0);
+  uint32_t *s_len = reinterpret_cast<uint32_t *>(s_lo + (ES ? a.tab.n_ext : 0));
   if (ES)
-    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) {
+      s_ext[t] = a.tab.ext_delta[t];
+      s_lo[t] = a.tab.ext_lo[t];
+      s_len[t] = a.tab.ext_len[t];
+    }
   __syncthreads();
   const uint64_t pol_s = policy_evict_first();
   const uint64_t pol_t = policy_evict_last();
   const int lane = threadIdx.x & 31;
   const Seg sg = a.segs[0];
   const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n;
-  const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);
-  const uint32_t *shu = reinterpret_cast<const uint32_t *>(sg.shadow + 8 * sg.n);
+  const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);  // shadow words (make_shw)
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   const uint32_t n_ext = (uint32_t)a.tab.n_ext, cur_ep = a.epoch;
   unsigned c_nulls = 0, c_hits = 0, c_slow = 0;
@@ -1747,18 +1747,17 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
     if (x.valid == 3u && !(i0 & 1)) {
       ld_stream2(reinterpret_cast<const void *>(a0), pol_s, x.g[0], x.g[1]);
       ld_stream2(shp + i0, pol_s, x.h[0], x.h[1]);
-      asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
-                   : "=r"(x.u[0]), "=r"(x.u[1])
-                   : "l"(shu + i0), "l"(pol_s));
     } else {
 #pragma unroll
       for (int m = 0; m < 2; ++m)
         if ((x.valid >> m) & 1) {
           x.g[m] = reinterpret_cast<const uint64_t *>(a0)[m];
           x.h[m] = shp[i0 + m];
-          x.u[m] = shu[i0 + m];
         }
     }
+#pragma unroll
+    for (int m = 0; m < 2; ++m)
+      if ((x.valid >> m) & 1) x.u[m] = shw_unit(x.h[m]);
   };
   auto gather = [&](const In &x, uint64_t w[2]) {
 #pragma unroll
@@ -1785,13 +1784,16 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
       const bool vm = (cur.valid >> m) & 1;
       const uint64_t g = cur.g[m], w = cw[m];
       const uint32_t e = hot_ext(w), fl = hot_flags(w), su = sh_unit(cur.u[m]);
-      const uint64_t delta = e < n_ext ? (ES ? s_ext[e] : a.tab.ext_delta[e]) : 0ull;
       const bool look = vm && g != 0;
-      hit[m] = look && su != SH_NONE && (fl & UF_ACTIVE) && e < n_ext && g == cur.h[m] + delta;
+      const uint64_t hr = look && su != SH_NONE && (fl & UF_ACTIVE) && e < n_ext
+                              ? sh_reverse(g, cur.h[m], ES ? s_ext[e] : a.tab.ext_delta[e], ES ? s_lo[e] : a.tab.ext_lo[e],
+                                           ES ? s_len[e] : a.tab.ext_len[e])
+                              : 0ull;
+      hit[m] = hr != 0;
       slow[m] = look && !hit[m];
       c_nulls += vm && g == 0;
       c_hits += hit[m];
-      outv[m] = hit[m] ? cur.h[m] : g;  // reverse: base + (g - devbase), the recorded CPU pointer
+      outv[m] = hit[m] ? hr : g;  // reverse: base + (g - devbase), the recorded CPU pointer
       // Alg. 2: the epoch gate of a hit whose unit is stale (rare after the first slot of each unit)
       const bool stale = hit[m] && st_epoch(w) != cur_ep;
       cp[m] = false;
@@ -1853,7 +1855,7 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
 
 template <bool DEC, bool ES>
 static int launch_rev_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
-  const size_t smem = (ES ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
+  const size_t smem = (ES ? al16(20 * (size_t)a.tab.n_ext) : 0) + 64;
   static bool configured = false;
   if (!configured) {
     int dev = 0, optin = 0;
@@ -2422,13 +2424,13 @@ void launch_gather_state(TableDev tab, const uint32_t *idx, int n, uint64_t *out
 }
 
 // deferred references of one shadow become ordinary references (DESIGN.md §6 "Deferred references")
-__global__ void k_materialise(const uint32_t *units, uint64_t n, int32_t *rc) {
+__global__ void k_materialise(const uint64_t *shadow, uint64_t n, int32_t *rc) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t w = units[i];
+    const uint32_t w = shw_unit(shadow[i]);
     if (sh_deferred(w)) red_add(rc + sh_unit(w), 1);
   }
 }
-void launch_materialise(const uint32_t *shadow_units, uint64_t n, int32_t *rc, cudaStream_t s) {
+void launch_materialise(const uint64_t *shadow_units, uint64_t n, int32_t *rc, cudaStream_t s) {
   if (n == 0) return;
   const uint64_t want = (n + 255) / 256;
   const int grid = (int)std::min<uint64_t>(want, 148 * 8);

@@ -268,7 +268,7 @@ struct Context {
   size_t col_cap = 0;           // units the device table columns have room for
 
   // device table
-  DevBuf hotb, hotcb, stb, rcb, size64, dbase, extd, snap_st, snap_rc;  // unit table columns + extent deltas
+  DevBuf hotb, hotcb, stb, rcb, size64, dbase, extd, extlo, extlen, snap_st, snap_rc;  // unit table columns + extent deltas
   size_t extd_n = 0;                          // entries uploaded to extd
   IndexBufs fwd, rev;
   // page directory over the unit bases (cgcm_dev.h PdDev; built with the table)
@@ -345,14 +345,23 @@ struct Context {
     t.base = dbase.as<uint64_t>();
     t.size64 = size64.as<uint64_t>();
     t.ext_delta = extd.as<uint64_t>();
+    t.ext_lo = extlo.as<uint64_t>();
+    t.ext_len = extlen.as<uint32_t>();
     t.n_ext = (int)extd_n;
     return t;
   }
   // device copy of the extent deltas (devbase - base) indexed by run id
   int sync_ext() {
-    std::vector<uint64_t> d(std::max<size_t>(runs.size(), 1), 0);
-    for (size_t r = 0; r < runs.size(); ++r) d[r] = 0 - runs[r].delta;  // runs store host - device
+    std::vector<uint64_t> d(std::max<size_t>(runs.size(), 1), 0), lo(d.size(), 0);
+    std::vector<uint32_t> len(d.size(), 0);
+    for (size_t r = 0; r < runs.size(); ++r) {
+      d[r] = 0 - runs[r].delta;  // runs store host - device
+      lo[r] = runs[r].addr;
+      len[r] = runs[r].bytes < (1ull << 32) ? (uint32_t)runs[r].bytes : 0u;  // >= 4 GiB: shadows not used
+    }
     CKS(upload(extd, d));
+    CKS(upload(extlo, lo));
+    CKS(upload(extlen, len));
     extd_n = runs.size();
     return CGCM_OK;
   }
@@ -1823,7 +1832,7 @@ struct Context {
     // a failing call first turns the references it deferred into ordinary ones, which undo_map drops
     auto undo_deferred = [&]() -> int {
       if (F.defer) {
-        launch_materialise(reinterpret_cast<const uint32_t *>(fsegs[0].shadow + 8 * fsegs[0].n), fsegs[0].n,
+        launch_materialise(reinterpret_cast<const uint64_t *>(fsegs[0].shadow), fsegs[0].n,
                            rcb.as<int32_t>(), main);
         st.kernel_launches += 1;
         CK(cudaGetLastError());
@@ -1995,7 +2004,7 @@ struct Context {
   int materialise(std::pair<const std::pair<uint64_t, uint64_t>, Shadow> &kv) {
     if (!kv.second.deferred) return CGCM_OK;
     const uint64_t n = kv.first.second;
-    launch_materialise(reinterpret_cast<const uint32_t *>(kv.second.buf.addr + 8 * n), n, rcb.as<int32_t>(), main);
+    launch_materialise(reinterpret_cast<const uint64_t *>(kv.second.buf.addr), n, rcb.as<int32_t>(), main);
     st.kernel_launches += 1;
     CK(cudaGetLastError());
     kv.second.deferred = false;
@@ -2035,7 +2044,7 @@ struct Context {
       dev_shadows += 1;
     }
     sh.valid = false;
-    if (dalloc(sh.buf, 12 * n + 64) != CGCM_OK) {
+    if (dalloc(sh.buf, 8 * n + 64) != CGCM_OK) {  // one shadow word per slot (cgcm_dev.h make_shw)
       erase_shadow(shadows.find(key));
       return 0;
     }
@@ -3493,7 +3502,7 @@ int cgcm_dumpTable(cgcm_unit_t *out, size_t cap, size_t *n) {
     CK(cudaMemcpyAsync(C->dump_rc.as<void>(), C->rcb.as<void>(), 4 * (size_t)C->U, cudaMemcpyDeviceToDevice, C->main));
     for (auto &kv : C->shadows)
       if (kv.second.deferred)
-        launch_materialise(reinterpret_cast<const uint32_t *>(kv.second.buf.addr + 8 * kv.first.second), kv.first.second,
+        launch_materialise(reinterpret_cast<const uint64_t *>(kv.second.buf.addr), kv.first.second,
                            C->dump_rc.as<int32_t>(), C->main);
     CK(cudaGetLastError());
     CKS(C->download(rcs, C->dump_rc, (size_t)C->U));
