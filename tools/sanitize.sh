@@ -11,7 +11,7 @@ CASES="tests/test_gpu_parity.py::test_scalar_map_unmap_release tests/test_gpu_pa
 for tool in memcheck racecheck synccheck; do
   extra=""
   [ "$tool" = memcheck ] && extra="--leak-check full"
-  timeout 2400 compute-sanitizer --tool $tool $extra --error-exitcode 17 --target-processes all \
+  PYTORCH_NO_CUDA_MEMORY_CACHING=1 timeout 2400 compute-sanitizer --tool $tool $extra --error-exitcode 17 --target-processes all \
     python -m pytest $CASES -q -x -p no:cacheprovider > gpurun_out/$R/sanitize_$tool.log 2>&1
   echo "rc=$?" >> gpurun_out/$R/sanitize_$tool.log
   tail -5 gpurun_out/$R/sanitize_$tool.log
