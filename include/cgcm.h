@@ -48,7 +48,8 @@ enum {
   CGCM_LENIENT = 2u,       /* A18: uncovered non-null words in pointer arrays pass through (counted) */
   CGCM_PROFILE = 4u,       /* time every hot kernel with CUDA events on its launch stream (stats)  */
   CGCM_FORCE_SHADOW = 8u,  /* always record the forward-map shadow of device arrays (tests)        */
-  CGCM_NO_PAGEDIR = 16u    /* hot kernels search the level index instead of the page directory     */
+  CGCM_NO_PAGEDIR = 16u,   /* hot kernels search the level index instead of the page directory     */
+  CGCM_PD_V2 = 32u         /* page directory in the v2 entry format even when v3 would fit (tests) */
 };
 
 /* ---- AU flags (declare + dump) ------------------------------------------------------------- */
@@ -283,6 +284,7 @@ typedef struct {
   uint64_t pd_overflow_pages; /* pages with more than 12 unit starts (offsets in a side array)    */
   uint64_t pd_bytes;          /* entries + overflow offsets                                       */
   uint32_t pd_min_shift, pd_max_shift; /* page sizes 2^shift of the segments                     */
+  uint32_t pd_format, pad;    /* page-entry format: 3 (candidates with ends + page state) or 2      */
 } cgcm_index_info_t;
 int cgcm_indexInfo(cgcm_index_info_t *out);
 /* The device storage the runtime holds for AU copies (for leak / balance checks; the paper's

@@ -23,7 +23,7 @@ SAMPLES_PATH = os.path.join(HERE, "libcgcm_samples.so")
 OK = 0
 E_INVALID, E_UNREGISTERED, E_OVERLAP, E_NOT_MAPPED, E_BUSY, E_DUPLICATE, E_NOMEM, E_CUDA, E_MIXED, E_NOCTX, E_MODREF = (
     -1, -2, -3, -4, -5, -6, -7, -8, -9, -10, -11)
-LITERAL_EPOCH, LENIENT, PROFILE, FORCE_SHADOW, NO_PAGEDIR = 1, 2, 4, 8, 16
+LITERAL_EPOCH, LENIENT, PROFILE, FORCE_SHADOW, NO_PAGEDIR, PD_V2 = 1, 2, 4, 8, 16, 32
 UNIT_GLOBAL, UNIT_READONLY, UNIT_ARRAYMAPPED, UNIT_ACTIVE = 1, 2, 4, 8
 RELEASE = 1
 
@@ -49,7 +49,8 @@ class Stats(C.Structure):
 class IndexInfo(C.Structure):
     _fields_ = [("units", C.c_uint64), ("levels", C.c_uint32), ("pd_segments", C.c_uint32),
                 ("pd_pages", C.c_uint64), ("pd_overflow_pages", C.c_uint64), ("pd_bytes", C.c_uint64),
-                ("pd_min_shift", C.c_uint32), ("pd_max_shift", C.c_uint32)]
+                ("pd_min_shift", C.c_uint32), ("pd_max_shift", C.c_uint32), ("pd_format", C.c_uint32),
+                ("pad", C.c_uint32)]
 
 
 class Extent(C.Structure):

@@ -128,7 +128,14 @@ struct IndexDev {
 // starts compare against p - A two per 64-bit subtraction with a guard bit per 16-bit lane (pd_count5); no
 // start sits at offset PD_PAD (build_pd takes a smaller page), and lookups clamp p - A to PD_PAD - 1.
 constexpr int PD_MAXSEG = 64;
-constexpr int PD_K = 5;
+// Two entry formats, chosen per directory by build_pd: v3 (above: PD_K3 = 5 candidates with their ends and
+// a page state -- one gather per lookup) when the directory fits PD_V3_MAX_BYTES, which keeps it
+// L2-resident; otherwise v2 (PD_K2 = 12 starts in w[2..7], no ends, no state; w[2] = overflow index) with
+// pages twice as large, whose lookups gather the unit word for the size and the state (config E: a v3
+// directory would need 16 KiB pages, 80 MB -- past the ~56 MiB the L2 holds for gathers from every SM).
+constexpr int PD_K3 = 5;
+constexpr int PD_K2 = 12;
+constexpr uint64_t PD_V3_MAX_BYTES = 40ull << 20;
 #ifdef CGCM_PD_MAXSHIFT
 constexpr int PD_MAXSHIFT = CGCM_PD_MAXSHIFT;
 #else
@@ -147,6 +154,7 @@ struct PdDev {
   const uint64_t *seg_start;  // [2*nseg] first unit base of each segment, then end (base + size) of its last unit
   const uint32_t *seg_meta;   // [4*nseg]: first page, npages, P, last unit
   int nseg;                   // 0: no page directory (the level index is used)
+  int v3;                     // entry format: 1 = v3 (candidates with ends + page state), 0 = v2
 };
 
 // One input segment of a slot kernel: n u64 slots at device address ptr (8-byte aligned),

@@ -447,13 +447,19 @@ __device__ __forceinline__ void pd_back(const PdDev &pd, uint64_t pol, const PdF
   // never counts padding and counts the same starts
   const uint32_t rr = min(f.poff, PD_PAD - 1u) * 0x10001u;
   uint32_t c = 0, mx = 0;
-  if (cnt <= (uint32_t)PD_K) {
+  if (pd.v3 && cnt <= (uint32_t)PD_K3) {
     uint32_t word;
     const uint32_t kk = pd_count5(w_in, min(f.poff, PD_PAD - 1u), word);
     c = kk << 4;  // (16 per counted start, as below)
     mx = kk ? (word & 0xFFFFu) : 0u;
+  } else if (!pd.v3 && cnt <= (uint32_t)PD_K2) {  // v2: twelve starts in w[2..7]
+#pragma unroll
+    for (int t = 1; t < 4; ++t) {
+      cnt_max2((uint32_t)w_in[t], rr, c, mx);
+      cnt_max2((uint32_t)(w_in[t] >> 32), rr, c, mx);
+    }
   } else {  // crowded page: the starts continue in ovf[], one sector per 16
-    const uint16_t *o = pd.ovf + (uint32_t)(w_in[1] >> 32);
+    const uint16_t *o = pd.ovf + (pd.v3 ? (uint32_t)(w_in[1] >> 32) : (uint32_t)w_in[1]);
     for (uint32_t t = 0; t < cnt; t += 16) {
       uint64_t v[4];
       ld_sector(o + t, pol, v);
@@ -521,13 +527,19 @@ __device__ __forceinline__ void pd_lookup2(const SPd &S, const PdDev &pd, uint64
     const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
     const uint32_t rr = min(poff[m], PD_PAD - 1u) * 0x10001u;  // see pd_back
     uint32_t c = 0, mx = 0;
-    if (cnt <= (uint32_t)PD_K) {
+    if (pd.v3 && cnt <= (uint32_t)PD_K3) {
       uint32_t word;
       const uint32_t kk = pd_count5(w[m], min(poff[m], PD_PAD - 1u), word);
       c = kk << 4;
       mx = kk ? (word & 0xFFFFu) : 0u;
+    } else if (!pd.v3 && cnt <= (uint32_t)PD_K2) {  // v2: twelve starts in w[2..7]
+#pragma unroll
+      for (int t = 1; t < 4; ++t) {
+        cnt_max2((uint32_t)w[m][t], rr, c, mx);
+        cnt_max2((uint32_t)(w[m][t] >> 32), rr, c, mx);
+      }
     } else {  // crowded page: the starts continue in ovf[], one sector per 16
-      const uint16_t *o = pd.ovf + (uint32_t)(w[m][1] >> 32);
+      const uint16_t *o = pd.ovf + (pd.v3 ? (uint32_t)(w[m][1] >> 32) : (uint32_t)w[m][1]);
       for (uint32_t t = 0; t < cnt; t += 16) {
         uint64_t v[4];
         ld_sector(o + t, pol, v);
@@ -1474,7 +1486,9 @@ __device__ __noinline__ uint64_t pd_crowded(const uint16_t *ovf, uint32_t first,
   return (uint64_t)k | ((uint64_t)off << 32);
 }
 
-template <bool ES>  // ES: the extent deltas are staged in shared memory
+// ES: the extent deltas are staged in shared memory; V3: the directory's entry format (cgcm_dev.h);
+// DELTA: the table has NEXT-1 delta units (the cold path of one-past-the-end and missed slots)
+template <bool ES, bool V3, bool DELTA>
 __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
@@ -1553,32 +1567,41 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
       j[m] = fc.jt[m];
       k0[m] = true;
       dec[m] = false;
-      ae[m] = fc.jt[m] >= 0 && cv[m] == Send;
+      ae[m] = DELTA && fc.jt[m] >= 0 && cv[m] == Send;
       key[m] = 0;
       ps[m] = 0;
       if (fc.ok[m]) {
         const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
         const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
         const uint32_t r = min(fc.poff[m], PD_PAD - 1u);
-        if (cnt <= (uint32_t)PD_K) {
+        if (V3 && cnt <= (uint32_t)PD_K3) {
           uint32_t word;
           const uint32_t k = pd_count5(fc.ew[m], r, word);
           const bool h = k ? fc.poff[m] <= (word >> 16) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0);
-          ae[m] = h && (k ? fc.poff[m] == (word >> 16) : fc.poff[m] + 1 == end0);
+          if (DELTA) ae[m] = h && (k ? fc.poff[m] == (word >> 16) : fc.poff[m] + 1 == end0);
           j[m] = h ? (int)(j0 + k) : -1;
           dec[m] = true;
           ps[m] = (uint32_t)fc.ew[m][1];
+        } else if (!V3 && cnt <= (uint32_t)PD_K2) {  // v2: twelve starts, four per 64-bit subtraction (le4)
+          const uint32_t r2 = r | (r << 16);
+          const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
+          const uint32_t k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
+          const uint32_t off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
+          k0[m] = k == 0;
+          j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
+          if (DELTA) ae[m] = k == 0 && fc.poff[m] + 1 == end0;
+          key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
         } else {  // crowded page: starts in the side array, the candidate's size from its unit word
-          const uint64_t ko = pd_crowded(a.pd.ovf, (uint32_t)(fc.ew[m][1] >> 32), cnt, r);
+          const uint64_t ko = pd_crowded(a.pd.ovf, V3 ? (uint32_t)(fc.ew[m][1] >> 32) : (uint32_t)fc.ew[m][1], cnt, r);
           const uint32_t k = (uint32_t)ko, off = (uint32_t)(ko >> 32);
           k0[m] = k == 0;
           j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
-          ae[m] = k == 0 && fc.poff[m] + 1 == end0;
+          if (DELTA) ae[m] = k == 0 && fc.poff[m] + 1 == end0;
           key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
         }
       }
       cw[m] = 0;
-      if (j[m] >= 0 && !(ps[m] & PD_STATE_VALID))  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
+      if (j[m] >= 0 && !(V3 && (ps[m] & PD_STATE_VALID)))  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
         asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
     }
     uint64_t outv[2] = {cv[0], cv[1]};
@@ -1589,14 +1612,14 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
       const bool vm = (valid >> m) & 1;
       const bool look = j[m] >= 0;
       uint64_t hw;
-      if (ps[m] & PD_STATE_VALID)  // every unit of the page is ACTIVE with its copy in this extent
+      if (V3 && (ps[m] & PD_STATE_VALID))  // every unit of the page is ACTIVE with its copy in this extent
         hw = ((uint64_t)(ps[m] & EXT_MASK) << ESHIFT) | ((uint64_t)(UF_ACTIVE | UF_STORAGE) << FSHIFT);
       else
         hw = (cw[m] & HOTC_ESC) && look ? ld_u64_hot(a.tab.hot + j[m], pol_t) : hot_of_hotc(cw[m]);
       uint64_t sz = hot_size32(hw);
       if (look && !dec[m] && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
       bool hit = look && (dec[m] || k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
-      if (a.dn > 0 && vm && cv[m] != 0) {  // NEXT-1: delta units (a warp-uniform branch)
+      if (DELTA && vm && cv[m] != 0) {  // NEXT-1: delta units
         const bool at_end = ae[m] || (look && !dec[m] && !k0[m] && cv[m] - key[m] == sz);
         uint64_t db;
         const int d = delta_override(a, cv[m], hit, at_end, db);
@@ -1675,7 +1698,7 @@ __global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
   flush_count(&a.st->translated, c_tr);
 }
 
-template <bool ES>
+template <bool ES, bool V3, bool DELTA>
 static int launch_fwd_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
   const size_t smem = (ES ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
   static bool configured = false;
@@ -1683,14 +1706,14 @@ static int launch_fwd_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
     int dev = 0, optin = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    cudaError_t e = cudaFuncSetAttribute(k_fwd_lean<ES>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    cudaError_t e = cudaFuncSetAttribute(k_fwd_lean<ES, V3, DELTA>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
     if (e != cudaSuccess) return (int)e;
     configured = true;
   }
   const uint64_t want = (a.nchunks + FWD_LEAN_THREADS - 1) / FWD_LEAN_THREADS;
   const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
-  k_fwd_lean<ES><<<grid, FWD_LEAN_THREADS, smem, s>>>(a);
+  k_fwd_lean<ES, V3, DELTA><<<grid, FWD_LEAN_THREADS, smem, s>>>(a);
   return (int)cudaGetLastError();
 }
 
@@ -1710,14 +1733,13 @@ constexpr int REV_LEAN_THREADS = 768;
 template <bool DEC, bool ES>  // ES: the extent deltas are staged in shared memory
 __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
-  // the extents' deltas and device ranges (the shadow check), staged when few
-  uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
-  uint64_t *s_lo = s_ext + (ES ? a.tab.n_ext : 0);
-  uint32_t *s_len = reinterpret_cast<uint32_t *>(s_lo + (ES ? a.tab.n_ext : 0));
+  // the extents' deltas and device ranges (the shadow check), staged when few: {delta, lo} as one 16-byte
+  // word per extent (one LDS.128 per slot), the lengths beside them
+  ulonglong2 *s_dl = reinterpret_cast<ulonglong2 *>(smem);
+  uint32_t *s_len = reinterpret_cast<uint32_t *>(s_dl + (ES ? a.tab.n_ext : 0));
   if (ES)
     for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) {
-      s_ext[t] = a.tab.ext_delta[t];
-      s_lo[t] = a.tab.ext_lo[t];
+      s_dl[t] = make_ulonglong2(a.tab.ext_delta[t], a.tab.ext_lo[t]);
       s_len[t] = a.tab.ext_len[t];
     }
   __syncthreads();
@@ -1785,10 +1807,15 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
       const uint64_t g = cur.g[m], w = cw[m];
       const uint32_t e = hot_ext(w), fl = hot_flags(w), su = sh_unit(cur.u[m]);
       const bool look = vm && g != 0;
-      const uint64_t hr = look && su != SH_NONE && (fl & UF_ACTIVE) && e < n_ext
-                              ? sh_reverse(g, cur.h[m], ES ? s_ext[e] : a.tab.ext_delta[e], ES ? s_lo[e] : a.tab.ext_lo[e],
-                                           ES ? s_len[e] : a.tab.ext_len[e])
-                              : 0ull;
+      uint64_t hr = 0;
+      if (look && su != SH_NONE && (fl & UF_ACTIVE) && e < n_ext) {
+        const ulonglong2 dl = ES ? s_dl[e] : make_ulonglong2(a.tab.ext_delta[e], a.tab.ext_lo[e]);
+#ifdef CGCM_SH_NOCHECK  // timing experiment only: no range check (NOT exact)
+        hr = (uint32_t)(g - dl.x) == (uint32_t)cur.h[m] ? g - dl.x : 0ull;
+#else
+        hr = sh_reverse(g, cur.h[m], dl.x, dl.y, ES ? s_len[e] : a.tab.ext_len[e]);
+#endif
+      }
       hit[m] = hr != 0;
       slow[m] = look && !hit[m];
       c_nulls += vm && g == 0;
@@ -1855,7 +1882,7 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
 
 template <bool DEC, bool ES>
 static int launch_rev_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
-  const size_t smem = (ES ? al16(20 * (size_t)a.tab.n_ext) : 0) + 64;
+  const size_t smem = (ES ? al16(20 * (size_t)a.tab.n_ext) + 16 : 0) + 64;
   static bool configured = false;
   if (!configured) {
     int dev = 0, optin = 0;
@@ -1937,8 +1964,13 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, i
       a.sel == SEL_ALL && a.cbeg == 0 && !no_pipe)
   {
     static const bool no_lean = std::getenv("CGCM_NO_LEAN") != nullptr;  // A/B experiments
-    if (a.segs_host_shadow && a.pd.nseg == 1 && !no_lean)
-      return a.tab.n_ext <= EXT_SMEM ? launch_fwd_lean1<true>(a, nsm, s) : launch_fwd_lean1<false>(a, nsm, s);
+    if (a.segs_host_shadow && a.pd.nseg == 1 && !no_lean) {
+      const bool es = a.tab.n_ext <= EXT_SMEM, v3 = a.pd.v3 != 0, dl = a.dn > 0;
+#define FWD_LEAN(E, V, D) if (es == E && v3 == V && dl == D) return launch_fwd_lean1<E, V, D>(a, nsm, s);
+      FWD_LEAN(true, true, false) FWD_LEAN(true, false, false) FWD_LEAN(false, true, false) FWD_LEAN(false, false, false)
+      FWD_LEAN(true, true, true) FWD_LEAN(true, false, true) FWD_LEAN(false, true, true) FWD_LEAN(false, false, true)
+#undef FWD_LEAN
+    }
     return a.segs_host_shadow ? launch_map_pd<1>(a, nsm, s) : launch_map_pd<0>(a, nsm, s);
   }
   constexpr int UNMAP = OP_WRITE | OP_GATE | OP_HITMASK, UNMAP_REL = OP_WRITE | OP_GATE | OP_DEC | OP_HITMASK;
@@ -2232,7 +2264,7 @@ __global__ void k_pd_state(PdDev pd, uint64_t npages, TableDev tab) {
     uint32_t *w = const_cast<uint32_t *>(pd.ent) + 8 * e;
     const uint32_t j0 = w[0], w1 = w[1], cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
     uint32_t state = 0;
-    if (cnt <= (uint32_t)PD_K) {
+    if (cnt <= (uint32_t)PD_K3) {
       bool ok = true, any = false;
       uint32_t ext = 0;
       auto take = [&](uint32_t u) {

@@ -273,7 +273,7 @@ struct Context {
   IndexBufs fwd, rev;
   // page directory over the unit bases (cgcm_dev.h PdDev; built with the table)
   DevBuf pd_ent, pd_ovf, pd_start, pd_meta;
-  int pd_nseg = 0;
+  int pd_nseg = 0, pd_v3 = 0;
   // the entries' page-state words (cgcm_dev.h) must be recomputed before a kernel reads the directory:
   // set by every change of a unit's ACTIVE / STORAGE / extent (activations, frees, unit ops, rebuilds)
   bool pd_state_dirty = true;
@@ -514,6 +514,15 @@ struct Context {
     std::vector<uint32_t> Ps(nseg);
     std::vector<uint64_t> npg(nseg);
     uint64_t total = 0;
+    static const int force_fmt = [] {  // A/B: CGCM_PD_FORMAT=2 or 3
+      const char *e = std::getenv("CGCM_PD_FORMAT");
+      return e ? std::atoi(e) : 0;
+    }();
+    // v3 entries (PD_K3 candidates) when the directory they need stays L2-sized, else v2 (PD_K2 starts)
+    int v3 = (force_fmt == 2 || (flags & CGCM_PD_V2)) ? 0 : 1;
+  size_pages:
+    const int PD_K = v3 ? PD_K3 : PD_K2;
+    total = 0;
     for (int s = 0; s < nseg; ++s) {
       const int i0 = cut[s], i1 = cut[s + 1];
       const uint64_t S = hb[i0], span = hb[i1 - 1] - S;  // pages up to the last base; beyond: its tail
@@ -540,10 +549,20 @@ struct Context {
         sel = P;
         if ((double)ovf <= ovf_frac * (double)(i1 - i0)) break;
       }
-      if (sel < 0) return CGCM_OK;  // too sparse for the budget: the level index serves
+      if (sel < 0) {  // too sparse for the budget: the other format, or the level index serves
+        if (v3 && force_fmt != 3) {
+          v3 = 0;
+          goto size_pages;
+        }
+        return CGCM_OK;
+      }
       Ps[s] = (uint32_t)sel;
       npg[s] = (span >> sel) + 1;
       total += npg[s];
+    }
+    if (v3 && force_fmt != 3 && 32 * total > PD_V3_MAX_BYTES) {
+      v3 = 0;
+      goto size_pages;
     }
     std::vector<uint32_t> ent(8 * total);
     std::vector<uint16_t> ovf;
@@ -571,9 +590,22 @@ struct Context {
         uint32_t *w = &ent[8 * e];
         w[0] = (uint32_t)i;
         w[1] = cnt | (hb[i] == A ? PD_EXACT : 0u) | (end0 << PD_END_SHIFT);
+        if (!v3) {  // v2: up to PD_K2 sorted u16 starts in w[2..7]
+          uint16_t *o16 = reinterpret_cast<uint16_t *>(w + 2);
+          if (cnt <= (uint32_t)PD_K2) {
+            for (int t = 0; t < PD_K2; ++t) o16[t] = t < (int)cnt ? (uint16_t)(hb[i + 1 + t] - A) : (uint16_t)PD_PAD;
+          } else {
+            w[2] = (uint32_t)ovf.size();
+            w[3] = w[4] = w[5] = w[6] = w[7] = 0xFFFFFFFFu;
+            for (uint32_t t = 0; t < cnt; ++t) ovf.push_back((uint16_t)(hb[i + 1 + t] - A));
+            while (ovf.size() % 16) ovf.push_back((uint16_t)PD_PAD);
+            ++novf;
+          }
+          continue;
+        }
         w[2] = 0;  // page state: computed on the device (k_pd_state)
-        if (cnt <= (uint32_t)PD_K) {
-          for (int t = 0; t < PD_K; ++t) {
+        if (cnt <= (uint32_t)PD_K3) {
+          for (int t = 0; t < PD_K3; ++t) {
             if (t < (int)cnt) {
               const uint64_t st0 = hb[i + 1 + t] - A, en = std::min<uint64_t>(hb[i + 1 + t] + hs[i + 1 + t] - A, PD_PAD);
               w[3 + t] = (uint32_t)st0 | ((uint32_t)en << 16);
@@ -596,6 +628,7 @@ struct Context {
     CKS(upload(pd_start, starts));
     CKS(upload(pd_meta, meta));
     pd_nseg = nseg;
+    pd_v3 = v3;
     pd_pages = total;
     pd_ovf_pages = novf;
     pd_bytes = 32 * total + 2 * ovf.size();
@@ -610,6 +643,7 @@ struct Context {
     p.seg_start = pd_start.as<uint64_t>();
     p.seg_meta = pd_meta.as<uint32_t>();
     p.nseg = pd_nseg;
+    p.v3 = pd_v3;
     return p;
   }
 
@@ -905,7 +939,7 @@ struct Context {
     a.copy_list = copy_list.as<uint32_t>();
     a.free_list = free_list.as<uint32_t>();
     a.lenient = (flags & CGCM_LENIENT) ? 1 : 0;
-    if (pd_nseg > 0 && pd_state_dirty) {
+    if (pd_nseg > 0 && pd_v3 && pd_state_dirty) {
       launch_pd_state(pd_view(), pd_pages, tab(), main);
       st.kernel_launches += 1;
       CK(cudaGetLastError());
@@ -3656,6 +3690,7 @@ int cgcm_indexInfo(cgcm_index_info_t *out) {
   out->pd_bytes = C->pd_bytes;
   out->pd_min_shift = C->pd_minP;
   out->pd_max_shift = C->pd_maxP;
+  out->pd_format = C->pd_nseg ? (C->pd_v3 ? 3u : 2u) : 0u;
   return CGCM_OK;
 }
 

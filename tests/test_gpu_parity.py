@@ -18,7 +18,7 @@ def cgcm_mod():
     return cg
 
 
-@pytest.fixture(params=[0, 8, 16], ids=["auto", "shadow", "levels"])
+@pytest.fixture(params=[0, 8, 16, 40], ids=["auto", "shadow", "levels", "shadow-v2"])
 def pair(cgcm_mod, request):
     from oracle import Oracle
     ctx = cgcm_mod.Context(0, arena_bytes=1 << 30, flags=request.param)
