@@ -1238,14 +1238,13 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
   // the streams of one chunk: slot values, recorded CPU pointers and units
   struct In {
     uint64_t a0;  // address of the chunk's first word (16-byte aligned)
-    uint64_t g[2], h[2];
-    uint32_t u[2];  // shadow unit words as recorded (SH_DEFER bit included)
+    uint64_t g[2], h[2];  // slot values, shadow words (cgcm_dev.h make_shw)
     uint32_t valid;
     int s;
   };
   auto load_in = [&](uint64_t c, In &x) {
-    x.g[0] = x.g[1] = x.h[0] = x.h[1] = 0;
-    x.u[0] = x.u[1] = 0xFFFFFFFFu;
+    x.g[0] = x.g[1] = 0;
+    x.h[0] = x.h[1] = make_shw(0, SH_NONE);  // (the unit word is read where it is used: no stall at the load)
     x.valid = 0;
     x.s = 0;
     x.a0 = 0;
@@ -1268,15 +1267,12 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
       for (int m = 0; m < 2; ++m)
         if ((x.valid >> m) & 1) x.h[m] = shp[i0 + m];
     }
-#pragma unroll
-    for (int m = 0; m < 2; ++m)
-      if ((x.valid >> m) & 1) x.u[m] = shw_unit(x.h[m]);
   };
   // the state words (epoch | extent | flags) of the recorded units of x
   auto gather = [&](const In &x, uint64_t w[2]) {
 #pragma unroll
     for (int m = 0; m < 2; ++m)
-      w[m] = (x.u[m] != SH_NONE && x.g[m] != 0) ? ld_u64_hot(a.tab.st + sh_unit(x.u[m]), pol_t) : 0ull;
+      w[m] = (shw_unit(x.h[m]) != SH_NONE && x.g[m] != 0) ? ld_u64_hot(a.tab.st + sh_unit(shw_unit(x.h[m])), pol_t) : 0ull;
   };
 
   const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -1300,7 +1296,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
       const bool look = vm && cur.g[m] != 0;
       const uint64_t w = cw[m];
       const uint32_t e = hot_ext(w);
-      const uint32_t su = sh_unit(cur.u[m]);
+      const uint32_t su = sh_unit(shw_unit(cur.h[m]));
       const uint64_t hr = look && su != SH_NONE && (hot_flags(w) & UF_ACTIVE) && e < (uint32_t)a.tab.n_ext
                               ? sh_reverse(cur.g[m], cur.h[m], ext_s ? s_ext[e] : a.tab.ext_delta[e],
                                            a.tab.ext_lo[e], a.tab.ext_len[e])
@@ -1315,7 +1311,7 @@ __global__ void __launch_bounds__(UNMAP_SH_THREADS, 1) k_unmap_sh(SlotArgs a) {
       bool freed = false;
       // a deferred reference (recorded by k_map_pd) is dropped by a released hit; any other slot turns
       // it into an ordinary reference first (the slow pass then treats the slot like any other)
-      const bool dfr = a.defer && vm && sh_deferred(cur.u[m]);  // (also if a GPU function wrote NULL there)
+      const bool dfr = a.defer && vm && sh_deferred(shw_unit(cur.h[m]));  // (also if a GPU function wrote NULL there)
       const bool drop = dfr && hit[m] && (OPS & OP_DEC);
       if (dfr && !drop) red_add(a.tab.rc + su, 1);
       if (OPS & OP_DEC) {
@@ -1754,13 +1750,12 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
   unsigned c_nulls = 0, c_hits = 0, c_slow = 0;
 
   struct In {
-    uint64_t g[2], h[2];
-    uint32_t u[2];
+    uint64_t g[2], h[2];  // slot values, shadow words (cgcm_dev.h make_shw)
     uint32_t valid;
   };
   auto load_in = [&](uint64_t c, In &x) {
-    x.g[0] = x.g[1] = x.h[0] = x.h[1] = 0;
-    x.u[0] = x.u[1] = SH_NONE;
+    x.g[0] = x.g[1] = 0;
+    x.h[0] = x.h[1] = make_shw(0, SH_NONE);  // (the unit word is read where it is used: no stall at the load)
     x.valid = 0;
     if (c >= a.nchunks) return;
     const uint64_t a0 = a0base + 16ull * c;
@@ -1777,14 +1772,11 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
           x.h[m] = shp[i0 + m];
         }
     }
-#pragma unroll
-    for (int m = 0; m < 2; ++m)
-      if ((x.valid >> m) & 1) x.u[m] = shw_unit(x.h[m]);
   };
   auto gather = [&](const In &x, uint64_t w[2]) {
 #pragma unroll
     for (int m = 0; m < 2; ++m)
-      w[m] = (x.u[m] != SH_NONE && x.g[m] != 0) ? ld_u64_hot(a.tab.st + sh_unit(x.u[m]), pol_t) : 0ull;
+      w[m] = (shw_unit(x.h[m]) != SH_NONE && x.g[m] != 0) ? ld_u64_hot(a.tab.st + sh_unit(shw_unit(x.h[m])), pol_t) : 0ull;
   };
 
   const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -1805,7 +1797,7 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
     for (int m = 0; m < 2; ++m) {
       const bool vm = (cur.valid >> m) & 1;
       const uint64_t g = cur.g[m], w = cw[m];
-      const uint32_t e = hot_ext(w), fl = hot_flags(w), su = sh_unit(cur.u[m]);
+      const uint32_t e = hot_ext(w), fl = hot_flags(w), su = sh_unit(shw_unit(cur.h[m]));
       const bool look = vm && g != 0;
       uint64_t hr = 0;
       if (look && su != SH_NONE && (fl & UF_ACTIVE) && e < n_ext) {
@@ -1832,7 +1824,7 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
         }
       }
       // references: a deferred one (a.defer) is dropped by a released hit, materialised otherwise
-      const bool dfr = a.defer && vm && sh_deferred(cur.u[m]);
+      const bool dfr = a.defer && vm && sh_deferred(shw_unit(cur.h[m]));
       const bool drop = DEC && dfr && hit[m];
       if (dfr && !drop) red_add(a.tab.rc + su, 1);
       if (DEC && hit[m] && !drop) red_add(a.tab.rc + su, -sg.inc);  // Alg. 3, checked by k_release_scan
@@ -1843,7 +1835,7 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
 #pragma unroll
       for (int m = 0; m < 2; ++m) {
         const unsigned long long cx = warp_append(&a.lc[3], cp[m]);
-        if (cp[m]) a.copy_list[cx] = sh_unit(cur.u[m]);
+        if (cp[m]) a.copy_list[cx] = sh_unit(shw_unit(cur.h[m]));
       }
     }
     if (cur.valid == 3u) {
