@@ -1449,6 +1449,11 @@ constexpr int FWD_LEAN_THREADS = CGCM_FWD_LEAN_THREADS;
 #else
 constexpr int FWD_LEAN_THREADS = 768;  // measured: 768 > 640 > 512 (profiles/r02f_ab.log)
 #endif
+#ifdef CGCM_FWD_LEAN_THREADS_V3
+constexpr int FWD_LEAN_THREADS_V3 = CGCM_FWD_LEAN_THREADS_V3;
+#else
+constexpr int FWD_LEAN_THREADS_V3 = 640;  // the v3 decode needs ~90 registers
+#endif
 
 __device__ __forceinline__ uint32_t warp_or(uint32_t v) { return __reduce_or_sync(0xffffffffu, v); }
 
@@ -1485,7 +1490,7 @@ __device__ __noinline__ uint64_t pd_crowded(const uint16_t *ovf, uint32_t first,
 // ES: the extent deltas are staged in shared memory; V3: the directory's entry format (cgcm_dev.h);
 // DELTA: the table has NEXT-1 delta units (the cold path of one-past-the-end and missed slots)
 template <bool ES, bool V3, bool DELTA>
-__global__ void __launch_bounds__(FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
+__global__ void __launch_bounds__(V3 ? FWD_LEAN_THREADS_V3 : FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
   if (ES)
@@ -1706,10 +1711,11 @@ static int launch_fwd_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
     if (e != cudaSuccess) return (int)e;
     configured = true;
   }
-  const uint64_t want = (a.nchunks + FWD_LEAN_THREADS - 1) / FWD_LEAN_THREADS;
+  constexpr int T = V3 ? FWD_LEAN_THREADS_V3 : FWD_LEAN_THREADS;
+  const uint64_t want = (a.nchunks + T - 1) / T;
   const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
-  k_fwd_lean<ES, V3, DELTA><<<grid, FWD_LEAN_THREADS, smem, s>>>(a);
+  k_fwd_lean<ES, V3, DELTA><<<grid, T, smem, s>>>(a);
   return (int)cudaGetLastError();
 }
 
