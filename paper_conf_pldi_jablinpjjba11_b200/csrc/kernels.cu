@@ -371,16 +371,12 @@ __device__ __noinline__ int delta_hit(const uint64_t *dk, const uint32_t *di, in
   base = b;
   return (int)id;
 }
-// After the main table's lookup of q: hit (unit j, main_base its base when known) -- the delta unit that
-// greatestLTE picks instead, if any: any delta unit containing q when the main table missed, or one
-// starting exactly at q when q is one past the end of the main hit (A7: the larger base wins).
-__device__ __forceinline__ int delta_override(const SlotArgs &a, uint64_t q, bool hit, bool at_end, uint64_t &base) {
-  if (a.dn <= 0 || (hit && !at_end)) return -1;
-  uint64_t b = 0;
-  const int d = delta_hit(a.dkeys, a.dids, a.dn, a.tab, q, b);
-  if (d < 0 || (hit && b != q)) return -1;
-  base = b;
-  return d;
+// After the main table's lookup of q missed: the delta unit containing q, if any.  (A delta unit that
+// starts exactly where a main unit ends -- and so would win greatestLTE at that unit's one-past-the-end
+// address, A7 -- never exists: such a declaration rebuilds the table, Context::delta_touches_main.)
+__device__ __forceinline__ int delta_override(const SlotArgs &a, uint64_t q, bool hit, uint64_t &base) {
+  if (a.dn <= 0 || hit) return -1;
+  return delta_hit(a.dkeys, a.dids, a.dn, a.tab, q, base);
 }
 
 // #{starts <= r} among an entry's (at most PD_K = 5) candidates, and the candidate word (start | end << 16)
@@ -785,15 +781,9 @@ __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs
     if (a.dn > 0) {  // NEXT-1: delta units (q: the host address looked up; 0 if none)
 #pragma unroll
       for (int m = 0; m < 2; ++m) {
-        if (q[m] == 0 || sh[m] || !((valid >> m) & 1)) continue;
-        bool at_end = false;
-        if (hit[m]) {
-          uint64_t sz = hot_size32(hw[m]);
-          if (sz == BIG_SIZE) sz = a.tab.size64[j[m]];
-          at_end = q[m] - a.tab.base[j[m]] == sz;
-        }
+        if (q[m] == 0 || sh[m] || !((valid >> m) & 1) || hit[m]) continue;
         uint64_t db;
-        const int d = delta_override(a, q[m], hit[m], at_end, db);
+        const int d = delta_override(a, q[m], hit[m], db);
         if (d < 0) continue;
         const uint64_t h2 = a.tab.hot[d];
         // a reverse lookup: the unit must own the extent's copy (active, its copy in that extent)
@@ -1078,10 +1068,9 @@ __global__ void __launch_bounds__(MAP_PD_THREADS, 1) k_map_pd(SlotArgs a) {
       uint64_t sz = hot_size32(hw[m]);
       if (look[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
       hit[m] = look[m] && (k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
-      if (a.dn > 0 && ((valid >> m) & 1) && cv[m] != 0) {  // NEXT-1: delta units
-        const bool at_end = hit[m] && cv[m] - a.tab.base[j[m]] == sz;
+      if (a.dn > 0 && ((valid >> m) & 1) && cv[m] != 0 && !hit[m]) {  // NEXT-1: delta units
         uint64_t db;
-        const int d = delta_override(a, cv[m], hit[m], at_end, db);
+        const int d = delta_override(a, cv[m], hit[m], db);
         if (d >= 0) {
           j[m] = d;
           hw[m] = a.tab.hot[d];
@@ -1560,7 +1549,7 @@ __global__ void __launch_bounds__(V3 ? FWD_LEAN_THREADS_V3 : FWD_LEAN_THREADS, 1
     // decode: j = j0 + #{starts <= p - A}; j0 is decided by its end, a candidate by its end in the entry
     // (A7); in a page whose state is valid the entry also gives ACTIVE and the extent: no unit word
     int j[2];
-    bool k0[2], dec[2], ae[2];  // ae: the hit may sit exactly one past its unit's end (NEXT-1 delta units)
+    bool k0[2], dec[2];
     uint64_t key[2];
     uint32_t cw[2], ps[2];
 #pragma unroll
@@ -1568,7 +1557,6 @@ __global__ void __launch_bounds__(V3 ? FWD_LEAN_THREADS_V3 : FWD_LEAN_THREADS, 1
       j[m] = fc.jt[m];
       k0[m] = true;
       dec[m] = false;
-      ae[m] = DELTA && fc.jt[m] >= 0 && cv[m] == Send;
       key[m] = 0;
       ps[m] = 0;
       if (fc.ok[m]) {
@@ -1579,7 +1567,6 @@ __global__ void __launch_bounds__(V3 ? FWD_LEAN_THREADS_V3 : FWD_LEAN_THREADS, 1
           uint32_t word;
           const uint32_t k = pd_count5(fc.ew[m], r, word);
           const bool h = k ? fc.poff[m] <= (word >> 16) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0);
-          if (DELTA) ae[m] = h && (k ? fc.poff[m] == (word >> 16) : fc.poff[m] + 1 == end0);
           j[m] = h ? (int)(j0 + k) : -1;
           dec[m] = true;
           ps[m] = (uint32_t)fc.ew[m][1];
@@ -1590,14 +1577,12 @@ __global__ void __launch_bounds__(V3 ? FWD_LEAN_THREADS_V3 : FWD_LEAN_THREADS, 1
           const uint32_t off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
           k0[m] = k == 0;
           j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
-          if (DELTA) ae[m] = k == 0 && fc.poff[m] + 1 == end0;
           key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
         } else {  // crowded page: starts in the side array, the candidate's size from its unit word
           const uint64_t ko = pd_crowded(a.pd.ovf, V3 ? (uint32_t)(fc.ew[m][1] >> 32) : (uint32_t)fc.ew[m][1], cnt, r);
           const uint32_t k = (uint32_t)ko, off = (uint32_t)(ko >> 32);
           k0[m] = k == 0;
           j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
-          if (DELTA) ae[m] = k == 0 && fc.poff[m] + 1 == end0;
           key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
         }
       }
@@ -1620,10 +1605,9 @@ __global__ void __launch_bounds__(V3 ? FWD_LEAN_THREADS_V3 : FWD_LEAN_THREADS, 1
       uint64_t sz = hot_size32(hw);
       if (look && !dec[m] && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
       bool hit = look && (dec[m] || k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
-      if (DELTA && vm && cv[m] != 0) {  // NEXT-1: delta units
-        const bool at_end = ae[m] || (look && !dec[m] && !k0[m] && cv[m] - key[m] == sz);
+      if (DELTA && vm && cv[m] != 0 && !hit) {  // NEXT-1: delta units, where the main table missed
         uint64_t db;
-        const int d = delta_override(a, cv[m], hit, at_end, db);
+        const int d = delta_override(a, cv[m], hit, db);
         if (d >= 0) {
           j[m] = d;
           hw = ld_u64_hot(a.tab.hot + d, pol_t);
@@ -2504,11 +2488,10 @@ __global__ void k_lookup_points(IndexDev ix, TableDev tab, const uint64_t *ptrs,
     const uint64_t b = ix.keys[lo], sz = tab.size64[lo];
     if (p - b <= sz) r.unit = lo;
   }
-  {  // NEXT-1: a delta unit containing p when the main table missed, or starting at p after a main unit
+  {  // NEXT-1: a delta unit containing p when the main table missed
     uint64_t db = 0;
-    const int d = (dn > 0 && (r.unit < 0 || p - ix.keys[r.unit] == tab.size64[r.unit]))
-                      ? delta_hit(dkeys, dids, dn, tab, p, db) : -1;
-    if (d >= 0 && (r.unit < 0 || db == p)) r.unit = d;
+    const int d = (dn > 0 && r.unit < 0) ? delta_hit(dkeys, dids, dn, tab, p, db) : -1;
+    if (d >= 0) r.unit = d;
   }
   if (r.unit >= 0) {
     const int lo = r.unit;

@@ -656,6 +656,18 @@ struct Context {
       pend.push_back(b);
     }
   }
+  // A pending unit that starts exactly where a unit of the main table ends would win greatestLTE at that
+  // unit's one-past-the-end address (A7), which the main lookup decides as a hit: such a declaration
+  // takes the rebuild, so that the kernels consult the delta units only where the main table misses.
+  bool delta_touches_main() const {
+    for (uint64_t b : pend) {
+      auto it = reg.lower_bound(b);
+      if (it == reg.begin()) continue;
+      --it;
+      if (it->second.idx >= 0 && it->second.idx < Umain && it->first + it->second.size == b) return true;
+    }
+    return false;
+  }
   // the batched merge of pending declarations (NEXT-1): append them to the columns as delta units and
   // re-sort the small delta index -- O(#pending + #delta) host work, no registry walk, no rebuild
   int append_delta() {
@@ -720,7 +732,7 @@ struct Context {
     Trace trace_("ensure_table");
     if (!table_dirty) return CGCM_OK;
     if (!dirty_del && !pend_over && Umain > 0 && dk.size() + pend.size() <= (size_t)DELTA_MAX &&
-        (size_t)U + pend.size() <= col_cap)
+        (size_t)U + pend.size() <= col_cap && !delta_touches_main())
       return append_delta();
     CKS(materialise_all());  // deferred references name units by their index in the table being replaced
     CKS(need_mirrors());     // the remap carries the per-unit host mirrors to the new indices
