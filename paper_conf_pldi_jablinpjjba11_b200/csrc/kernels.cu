@@ -1441,7 +1441,7 @@ constexpr int FWD_LEAN_THREADS = 768;  // measured: 768 > 640 > 512 (profiles/r0
 #ifdef CGCM_FWD_LEAN_THREADS_V3
 constexpr int FWD_LEAN_THREADS_V3 = CGCM_FWD_LEAN_THREADS_V3;
 #else
-constexpr int FWD_LEAN_THREADS_V3 = 640;  // the v3 decode needs ~90 registers
+constexpr int FWD_LEAN_THREADS_V3 = 768;  // measured: 768 (24 B of spills) > 640 (no spills), profiles/r02r_ab.log
 #endif
 
 __device__ __forceinline__ uint32_t warp_or(uint32_t v) { return __reduce_or_sync(0xffffffffu, v); }

@@ -1,7 +1,8 @@
 """Batched table merge (NEXT-1: the run-time keeps allocInfoMap current as the program allocates):
 declarations between calls are appended to the device table as delta units instead of a rebuild, and
 every lookup path (page-directory hot kernels, generic slot kernel, reverse lookups, outer-pointer lookups,
-glue kernels) consults them where the main table misses or hits exactly one past the end of a unit (A7).
+glue kernels) consults them where the main table misses (A7's one-past-the-end rule is kept by rebuilding
+instead when a declaration starts exactly where a main unit ends).
 Compared with the oracle after every call, on a config-C-shaped page-directory table with declarations
 placed in its gaps -- including a delta unit starting exactly at a main unit's end and a main unit starting
 exactly at a delta unit's end (one-past-the-end pointers resolve to the unit with the greater base; a
