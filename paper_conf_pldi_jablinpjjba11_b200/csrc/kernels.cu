@@ -1704,6 +1704,349 @@ static int launch_fwd_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
 }
 
 // -------------------------------------------------------------------------------------------------
+// k_fwd_fast: k_fwd_lean's results, counters and lists with the common chunk on a short path (round 2,
+// VERDICT r1 item 4 "instructions": k_fwd_lean spends 270 thread instructions per slot, issue-bound even
+// with every table L2-resident -- profiles/r02q_C_summary.md).  A warp takes the short path for a chunk
+// when all of its 64 slots are ordinary: a whole chunk, a page of this segment, a hit on a unit that is
+// ACTIVE with its copy (its reference deferred into the shadow, a.defer), no escaped unit word.  The short
+// path keeps no per-slot counters (a fast chunk is two hits, two translations), builds no masks (its
+// hit-mask words are all ones) and takes no atomics.  Any other chunk -- a NULL, a miss, an activation,
+// a ragged end, a huge unit, a delta unit -- is redone by fwd_chunk_slow (the k_fwd_lean iteration, one
+// warp-uniform call that recomputes the chunk from its two slot values).  Crowded pages stay on the
+// short path (a divergent side-array count, as in k_fwd_lean).
+// -------------------------------------------------------------------------------------------------
+#ifdef CGCM_FWD_FAST_THREADS
+constexpr int FWD_FAST_THREADS = CGCM_FWD_FAST_THREADS;
+#else
+constexpr int FWD_FAST_THREADS = 768;
+#endif
+
+// the k_fwd_lean iteration for chunk c (slot values cv) of the warp whose first chunk is cb; called by
+// all 32 lanes of the warp (warp collectives: activation list, hit mask, counters)
+template <bool ES, bool V3, bool DELTA>
+__device__ __noinline__ void fwd_chunk_slow(const SlotArgs &a, const uint64_t *s_ext, uint64_t c, uint64_t cb,
+                                            uint64_t cv0, uint64_t cv1) {
+  const uint64_t pol_s = policy_evict_first();
+  const uint64_t pol_t = policy_evict_last();
+  const int lane = threadIdx.x & 31;
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n;
+  uint64_t *shp = reinterpret_cast<uint64_t *>(sg.shadow);
+  const uint64_t S0 = a.pd.seg_start[0], Send = a.pd.seg_start[1];
+  const uint32_t P = a.pd.seg_meta[2], npages = a.pd.seg_meta[1], lastu = a.pd.seg_meta[3];
+  const uint32_t *ent = a.pd.ent + 8ull * a.pd.seg_meta[0];
+  const uint32_t pmask = (1u << P) - 1u;
+  const int32_t inc = sg.inc;
+  const bool defer = a.defer != 0;
+  const uint64_t a0 = a0base + 16ull * c;
+  const uint32_t valid = c < a.nchunks ? ((a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u)) : 0u;
+  const uint64_t cv[2] = {cv0, cv1};
+  unsigned c_nulls = 0, c_hits = 0, c_miss = 0, c_pend = 0, c_tr = 0;
+  // a1 front: the page of each slot, its entry, or the tail of the segment's last unit (A7)
+  uint64_t ew[2][4];
+  uint32_t poff[2];
+  int jt[2];
+  bool ok[2];
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    const bool look = ((valid >> m) & 1) && cv[m] != 0 && cv[m] >= S0;
+    const uint64_t rel = cv[m] - S0;
+    const uint64_t pg = rel >> P;
+    ok[m] = look && pg < npages;
+    poff[m] = (uint32_t)rel & pmask;
+    jt[m] = look && !ok[m] && cv[m] <= Send ? (int)lastu : -1;
+    ew[m][0] = ew[m][1] = ew[m][2] = ew[m][3] = 0;
+    if (ok[m]) ld_sector(ent + 8 * pg, pol_t, ew[m]);
+  }
+  int j[2];
+  bool k0[2], dec[2];
+  uint64_t key[2];
+  uint32_t cw[2], ps[2];
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    j[m] = jt[m];
+    k0[m] = true;
+    dec[m] = false;
+    key[m] = 0;
+    ps[m] = 0;
+    if (ok[m]) {
+      const uint32_t j0 = (uint32_t)ew[m][0], w1 = (uint32_t)(ew[m][0] >> 32);
+      const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
+      const uint32_t r = min(poff[m], PD_PAD - 1u);
+      if (V3 && cnt <= (uint32_t)PD_K3) {
+        uint32_t word;
+        const uint32_t k = pd_count5(ew[m], r, word);
+        const bool h = k ? poff[m] <= (word >> 16) : (j0 != 0xFFFFFFFFu && poff[m] < end0);
+        j[m] = h ? (int)(j0 + k) : -1;
+        dec[m] = true;
+        ps[m] = (uint32_t)ew[m][1];
+      } else if (!V3 && cnt <= (uint32_t)PD_K2) {
+        const uint32_t r2 = r | (r << 16);
+        const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
+        const uint32_t k = le4(ew[m][1], r4) + le4(ew[m][2], r4) + le4(ew[m][3], r4);
+        const uint32_t off = k ? off_at(ew[m][1], ew[m][2], ew[m][3], k - 1) : 0u;
+        k0[m] = k == 0;
+        j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && poff[m] < end0 ? (int)j0 : -1);
+        key[m] = cv[m] - poff[m] + off;
+      } else {
+        const uint64_t ko = pd_crowded(a.pd.ovf, V3 ? (uint32_t)(ew[m][1] >> 32) : (uint32_t)ew[m][1], cnt, r);
+        const uint32_t k = (uint32_t)ko, off = (uint32_t)(ko >> 32);
+        k0[m] = k == 0;
+        j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && poff[m] < end0 ? (int)j0 : -1);
+        key[m] = cv[m] - poff[m] + off;
+      }
+    }
+    cw[m] = 0;
+    if (j[m] >= 0 && !(V3 && (ps[m] & PD_STATE_VALID)))
+      asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
+  }
+  uint64_t outv[2] = {cv[0], cv[1]};
+  uint32_t wrote = 0, su[2];
+  bool act[2];
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    const bool vm = (valid >> m) & 1;
+    const bool look = j[m] >= 0;
+    uint64_t hw;
+    if (V3 && (ps[m] & PD_STATE_VALID))
+      hw = ((uint64_t)(ps[m] & EXT_MASK) << ESHIFT) | ((uint64_t)(UF_ACTIVE | UF_STORAGE) << FSHIFT);
+    else
+      hw = (cw[m] & HOTC_ESC) && look ? ld_u64_hot(a.tab.hot + j[m], pol_t) : hot_of_hotc(cw[m]);
+    uint64_t sz = hot_size32(hw);
+    if (look && !dec[m] && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
+    bool hit = look && (dec[m] || k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
+    if (DELTA && vm && cv[m] != 0 && !hit) {  // NEXT-1: delta units, where the main table missed
+      uint64_t db;
+      const int d = delta_override(a, cv[m], hit, db);
+      if (d >= 0) {
+        j[m] = d;
+        hw = ld_u64_hot(a.tab.hot + d, pol_t);
+        hit = true;
+      }
+    }
+    const bool nul = vm && cv[m] == 0;
+    c_nulls += nul;
+    c_hits += hit;
+    c_miss += vm && !nul && !hit;
+    const uint32_t fl = hot_flags(hw);
+    const bool active = (fl & UF_ACTIVE) != 0;
+    const bool dfr = defer && hit && active;
+    act[m] = false;
+    if (hit && !dfr) {
+      int32_t *RC = a.tab.rc + j[m];
+      if (active) red_add(RC, inc);
+      else act[m] = atomicAdd(RC, inc) == 0;  // refcount 0 -> 1: Alg. 1's activation
+    }
+    if (hit && (fl & UF_STORAGE)) {
+      const uint32_t e = hot_ext(hw);
+      outv[m] = cv[m] + (ES ? s_ext[e] : a.tab.ext_delta[e]);  // Alg. 1: devptr + (ptr - base)
+      wrote |= 1u << m;
+    } else {
+      c_pend += hit;
+    }
+    su[m] = hit ? ((uint32_t)j[m] | (dfr ? SH_DEFER : 0u)) : SH_NONE;
+  }
+  c_tr += __popc(wrote);
+  if (__any_sync(0xffffffffu, act[0] || act[1])) {
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const unsigned long long ix = warp_append(&a.lc[0], act[m]);
+      if (act[m]) a.act_list[ix] = (uint32_t)j[m];
+    }
+  }
+  const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
+  if (valid == 3u) {
+    st_stream2(reinterpret_cast<void *>(a0), pol_s, outv[0], outv[1]);
+    if (!(i0 & 1)) {
+      st_stream2(shp + i0, pol_s, make_shw(cv[0], su[0]), make_shw(cv[1], su[1]));
+    } else {
+#pragma unroll
+      for (int m = 0; m < 2; ++m) shp[i0 + m] = make_shw(cv[m], su[m]);
+    }
+  } else if (valid) {
+#pragma unroll
+    for (int m = 0; m < 2; ++m)
+      if ((valid >> m) & 1) {
+        st_stream1(reinterpret_cast<void *>(a0 + 8ull * m), pol_s, outv[m]);
+        shp[i0 + m] = make_shw(cv[m], su[m]);
+      }
+  }
+  {  // hit mask: 2 bits per chunk, 16 chunks per word (lanes 0-15: word cb/16, lanes 16-31: the next)
+    const uint32_t b = wrote << (2u * (lane & 15));
+    const uint32_t w0 = warp_or(lane < 16 ? b : 0u), w1 = warp_or(lane < 16 ? 0u : b);
+    const uint64_t wi = cb >> 4;
+    if (lane == 0) a.hitmask[wi] = w0;
+    else if (lane == 16 && cb + 16 < a.nchunks) a.hitmask[wi + 1] = w1;
+  }
+  flush_count(&a.st->nulls, (unsigned long long)c_nulls * (unsigned)inc);
+  flush_count(&a.st->hits, (unsigned long long)c_hits * (unsigned)inc);
+  flush_count(&a.st->misses, (unsigned long long)c_miss * (unsigned)inc);
+  flush_count(&a.st->pending, c_pend);
+  flush_count(&a.st->translated, c_tr);
+}
+
+template <bool ES, bool V3, bool DELTA>
+__global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_fast(const __grid_constant__ SlotArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
+  if (ES)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
+  __syncthreads();
+  const uint64_t pol_s = policy_evict_first();
+  const uint64_t pol_t = policy_evict_last();
+  const uint32_t lane = threadIdx.x & 31;
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull;
+  uint64_t *shp = reinterpret_cast<uint64_t *>(sg.shadow) - ((sg.ptr >> 3) & 1);  // shp[2c]: chunk c's first slot
+  const bool sh_odd = (sg.ptr >> 3) & 1;
+  const uint64_t S0 = a.pd.seg_start[0];
+  const uint32_t P = a.pd.seg_meta[2];
+  const uint64_t npages = a.pd.seg_meta[1];
+  const uint32_t *ent = a.pd.ent + 8ull * a.pd.seg_meta[0];
+  const uint32_t pmask = (1u << P) - 1u;
+  const uint32_t nch = (uint32_t)a.nchunks;  // < 2^32 (launch_fwd_fast1)
+  // whole chunks (both slots in the segment): [f0, f1)
+  const uint32_t f0 = sh_odd ? 1u : 0u;
+  const uint32_t f1 = (uint32_t)((sg.ptr + 8ull * sg.n - a0base) >> 4);
+  const bool fast_ok = a.defer != 0;
+  const uint32_t stride = gridDim.x * blockDim.x;
+  uint32_t c_fast = 0;
+
+  struct Fr {
+    uint64_t ew[2][4];
+    uint32_t poff[2];
+    bool ok[2];
+  };
+  auto front = [&](uint64_t p0, uint64_t p1, Fr &f) {
+    const uint64_t p[2] = {p0, p1};
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const uint64_t rel = p[m] - S0;  // NULL and p < S0 wrap far beyond the pages
+      const uint64_t pg = rel >> P;
+      f.ok[m] = pg < npages;
+      f.poff[m] = (uint32_t)rel & pmask;
+      if (f.ok[m])
+        asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+                     : "=l"(f.ew[m][0]), "=l"(f.ew[m][1]), "=l"(f.ew[m][2]), "=l"(f.ew[m][3])
+                     : "l"(ent + 8 * pg), "l"(pol_t));
+    }
+  };
+  const uint32_t c_first = blockIdx.x * blockDim.x + threadIdx.x;
+  uint64_t cv0 = 0, cv1 = 0, nv0 = 0, nv1 = 0, nnv0 = 0, nnv1 = 0;
+  if (c_first < nch) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c_first), pol_s, cv0, cv1);
+  if (c_first + stride < nch)
+    ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, nv0, nv1);
+  Fr fc, fn;
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    fc.ew[m][0] = fc.ew[m][1] = fc.ew[m][2] = fc.ew[m][3] = 0;
+    fn.ew[m][0] = fn.ew[m][1] = fn.ew[m][2] = fn.ew[m][3] = 0;
+  }
+  front(cv0, cv1, fc);
+  for (uint32_t cb = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < nch; cb += stride) {
+    const uint32_t c = cb + lane;
+    if (c + 2 * stride < nch)
+      ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, nnv0, nnv1);
+    front(nv0, nv1, fn);  // the next chunk's entries are in flight while this one finishes
+
+    // decode: j = j0 + #{starts <= p - A}; the candidate's distance dl = p - base (A7: hit iff dl <= size)
+    bool rare = !(fast_ok && c >= f0 && c < f1);
+    uint32_t j[2], cw[2], ext[2];
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
+      const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT, po = fc.poff[m];
+      const uint32_t r = min(po, PD_PAD - 1u);
+      const bool okj0 = j0 != 0xFFFFFFFFu && po < end0;  // j0's end decides (A7)
+      uint32_t k, dl = 0;
+      bool hit = false, known = false;  // known: decided by the entry (v3), with the page state
+      uint32_t ps = 0;
+      if (V3 && cnt <= (uint32_t)PD_K3) {
+        uint32_t word;
+        k = pd_count5(fc.ew[m], r, word);
+        hit = k ? po <= (word >> 16) : okj0;
+        ps = (uint32_t)fc.ew[m][1];
+        known = true;
+      } else {
+        uint32_t off;
+        if (!V3 && cnt <= (uint32_t)PD_K2) {
+          const uint32_t r2 = r | (r << 16);
+          const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
+          k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
+          off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
+        } else if (fc.ok[m]) {  // crowded page: the side array
+          const uint64_t ko = pd_crowded(a.pd.ovf, V3 ? (uint32_t)(fc.ew[m][1] >> 32) : (uint32_t)fc.ew[m][1], cnt, r);
+          k = (uint32_t)ko;
+          off = (uint32_t)(ko >> 32);
+        } else {
+          k = off = 0;
+        }
+        dl = po - off;
+        hit = k ? true : okj0;  // k > 0: decided by the candidate's size (unit word)
+      }
+      j[m] = j0 + k;
+      rare = rare || !fc.ok[m] || !hit;
+      const bool st_valid = V3 && known && (ps & PD_STATE_VALID);
+      cw[m] = 0;
+      if (fc.ok[m] && hit && !st_valid)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
+        asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
+      ext[m] = st_valid ? (ps & (uint32_t)EXT_MASK) : 0xFFFFFFFFu;
+      if (!st_valid) {
+        // ACTIVE with its copy, no escape; a candidate (k > 0, v2 or crowded) also within its size
+        const bool ok_w = (cw[m] & (HOTC_ESC | (3u << 29))) == (3u << 29) && (known || k == 0 || dl <= (cw[m] & 0x3FFFFu));
+        rare = rare || !ok_w;
+        ext[m] = (cw[m] >> 18) & 0x7FFu;
+      }
+    }
+    if (__any_sync(0xffffffffu, rare)) {
+      fwd_chunk_slow<ES, V3, DELTA>(a, s_ext, c, cb, cv0, cv1);
+    } else {
+      ++c_fast;
+      const uint64_t o0 = cv0 + (ES ? s_ext[ext[0]] : a.tab.ext_delta[ext[0]]);  // Alg. 1: devptr + (ptr - base)
+      const uint64_t o1 = cv1 + (ES ? s_ext[ext[1]] : a.tab.ext_delta[ext[1]]);
+      st_stream2(reinterpret_cast<void *>(a0base + 16ull * c), pol_s, o0, o1);
+      const uint64_t s0 = make_shw(cv0, j[0] | SH_DEFER), s1 = make_shw(cv1, j[1] | SH_DEFER);
+      if (!sh_odd) {
+        st_stream2(shp + 2ull * c, pol_s, s0, s1);
+      } else {
+        shp[2ull * c] = s0;
+        shp[2ull * c + 1] = s1;
+      }
+      if (lane == 0) a.hitmask[cb >> 4] = 0xFFFFFFFFu;
+      else if (lane == 16 && cb + 16 < nch) a.hitmask[(cb >> 4) + 1] = 0xFFFFFFFFu;
+    }
+    cv0 = nv0;
+    cv1 = nv1;
+    nv0 = nnv0;
+    nv1 = nnv1;
+    fc = fn;
+  }
+  const unsigned inc = (unsigned)sg.inc;
+  flush_count(&a.st->hits, 2ull * c_fast * inc);  // inc = k: k sequential calls
+  flush_count(&a.st->translated, 2ull * c_fast);
+}
+
+template <bool ES, bool V3, bool DELTA>
+static int launch_fwd_fast1(const SlotArgs &a, int nsm, cudaStream_t s) {
+  const size_t smem = (ES ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
+  static bool configured = false;
+  if (!configured) {
+    int dev = 0, optin = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    cudaError_t e = cudaFuncSetAttribute(k_fwd_fast<ES, V3, DELTA>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    if (e != cudaSuccess) return (int)e;
+    configured = true;
+  }
+  constexpr int T = FWD_FAST_THREADS;
+  const uint64_t want = (a.nchunks + T - 1) / T;
+  const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
+  (void)cudaGetLastError();
+  k_fwd_fast<ES, V3, DELTA><<<grid, T, smem, s>>>(a);
+  return (int)cudaGetLastError();
+}
+
+// -------------------------------------------------------------------------------------------------
 // k_rev_lean: the reverse pass of cgcm_unmapArrayDevice (a3 + a4 [+ Alg. 3 release]) over ONE in-place
 // segment that carries the forward map's shadow, in snapshot mode (no per-unit journal; releases as
 // reductions checked afterwards by k_release_scan).  Same decisions, counters and lists as
@@ -1948,7 +2291,10 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, i
     static const bool no_lean = std::getenv("CGCM_NO_LEAN") != nullptr;  // A/B experiments
     if (a.segs_host_shadow && a.pd.nseg == 1 && !no_lean) {
       const bool es = a.tab.n_ext <= EXT_SMEM, v3 = a.pd.v3 != 0, dl = a.dn > 0;
-#define FWD_LEAN(E, V, D) if (es == E && v3 == V && dl == D) return launch_fwd_lean1<E, V, D>(a, nsm, s);
+      static const bool fwd_old = std::getenv("CGCM_FWD_OLD") != nullptr;  // A/B: k_fwd_lean
+      const bool fast = !fwd_old && a.nchunks < (1ull << 31);
+#define FWD_LEAN(E, V, D) \
+  if (es == E && v3 == V && dl == D) return fast ? launch_fwd_fast1<E, V, D>(a, nsm, s) : launch_fwd_lean1<E, V, D>(a, nsm, s);
       FWD_LEAN(true, true, false) FWD_LEAN(true, false, false) FWD_LEAN(false, true, false) FWD_LEAN(false, false, false)
       FWD_LEAN(true, true, true) FWD_LEAN(true, false, true) FWD_LEAN(false, true, true) FWD_LEAN(false, false, true)
 #undef FWD_LEAN
