@@ -38,6 +38,9 @@ CONFIGS = {
               "replicated 2^22-unit table"),
     "C": dict(U=1 << 20, arrays=64, slots=1 << 20, seed=3, name="C: 2^26 interior pointers, 2^20-unit table"),
     "T": dict(U=1 << 12, arrays=8, slots=1 << 12, seed=3, name="T: tiny debug configuration"),
+    # kernel experiments only (not bench lines): E's batch against smaller tables (table working set vs L2)
+    "E20": dict(U=1 << 20, arrays=256, slots=1 << 20, seed=5, name="experiment: E's batch, 2^20-unit table"),
+    "E21": dict(U=1 << 21, arrays=256, slots=1 << 20, seed=5, name="experiment: E's batch, 2^21-unit table"),
 }
 METRIC = "translated pointers/sec and map+unmap GB/s per B200 (and 8-GPU), % of HBM roofline"
 BYTES_PER_TRANSLATION = 16  # 8 B read + 8 B write of the pointer slot

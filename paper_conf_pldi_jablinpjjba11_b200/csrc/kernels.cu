@@ -1421,29 +1421,7 @@ static int launch_unmap_sh(const SlotArgs &a, int nsm, cudaStream_t s) {
   return a.nseg > 1 ? launch_unmap_sh1<OPS, true>(a, nsm, s) : launch_unmap_sh1<OPS, false>(a, nsm, s);
 }
 
-// -------------------------------------------------------------------------------------------------
-// k_fwd_lean: the forward map of cgcm_mapArrayDevice (a1 + a2 of Alg. 1) over ONE in-place segment with
-// a shadow, through a page directory of ONE address segment (the case of every config-C/E-shaped
-// table).  Same results, counters and lists as k_map_pd<1>; the instruction count per slot is what
-// bounds k_map_pd (profiles/r02c_E_summary.md: 327 thread instructions per slot at 63 % issue), so:
-//   * the page entry's twelve 15-bit offsets are compared with p - A four at a time, one 64-bit
-//     subtraction per four with a guard bit per lane (le4), instead of twelve emulated SIMD compares;
-//   * the segment is in registers (no shared-memory segment search), the page is one shift;
-//   * activations (units not yet active), crowded pages, escaped unit words and huge units are the
-//     rare paths; the hit mask is built with warp reductions; whole chunks are stored unconditionally
-//     (an untranslated slot is written back unchanged; ragged segment ends slot by slot).
-// -------------------------------------------------------------------------------------------------
-#ifdef CGCM_FWD_LEAN_THREADS
-constexpr int FWD_LEAN_THREADS = CGCM_FWD_LEAN_THREADS;
-#else
-constexpr int FWD_LEAN_THREADS = 768;  // measured: 768 > 640 > 512 (profiles/r02f_ab.log)
-#endif
-#ifdef CGCM_FWD_LEAN_THREADS_V3
-constexpr int FWD_LEAN_THREADS_V3 = CGCM_FWD_LEAN_THREADS_V3;
-#else
-constexpr int FWD_LEAN_THREADS_V3 = 768;  // measured: 768 (24 B of spills) > 640 (no spills), profiles/r02r_ab.log
-#endif
-
+// ---- helpers of the pipelined single-segment passes ---------------------------------------------
 __device__ __forceinline__ uint32_t warp_or(uint32_t v) { return __reduce_or_sync(0xffffffffu, v); }
 
 // #{o <= r} among the four sorted 15-bit offsets packed in q (16-bit lanes): per lane
@@ -1476,244 +1454,20 @@ __device__ __noinline__ uint64_t pd_crowded(const uint16_t *ovf, uint32_t first,
   return (uint64_t)k | ((uint64_t)off << 32);
 }
 
-// ES: the extent deltas are staged in shared memory; V3: the directory's entry format (cgcm_dev.h);
-// DELTA: the table has NEXT-1 delta units (the cold path of one-past-the-end and missed slots)
-template <bool ES, bool V3, bool DELTA>
-__global__ void __launch_bounds__(V3 ? FWD_LEAN_THREADS_V3 : FWD_LEAN_THREADS, 1) k_fwd_lean(SlotArgs a) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
-  if (ES)
-    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
-  __syncthreads();
-  const uint64_t pol_s = policy_evict_first();
-  const uint64_t pol_t = policy_evict_last();
-  const int lane = threadIdx.x & 31;
-  const Seg sg = a.segs[0];
-  const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n;
-  uint64_t *shp = reinterpret_cast<uint64_t *>(sg.shadow);  // shadow words (make_shw)
-  // the directory's one segment: first base, end of its last unit, first entry, pages, page shift, last unit
-  const uint64_t S0 = a.pd.seg_start[0], Send = a.pd.seg_start[1];
-  const uint32_t P = a.pd.seg_meta[2], npages = a.pd.seg_meta[1], lastu = a.pd.seg_meta[3];
-  const uint32_t *ent = a.pd.ent + 8ull * a.pd.seg_meta[0];
-  const uint32_t pmask = (1u << P) - 1u;
-  const int32_t inc = sg.inc;
-  const bool defer = a.defer != 0;
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  unsigned c_nulls = 0, c_hits = 0, c_miss = 0, c_pend = 0, c_tr = 0;
-
-  auto valid_of = [&](uint64_t c) -> uint32_t {
-    const uint64_t a0 = a0base + 16ull * c;
-    return c < a.nchunks ? ((a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u)) : 0u;
-  };
-  // front half of a1 for the two slots of a chunk: the page of each, and its entry gather issued
-  // (ok); beyond the last page, the tail of the segment's last unit (jt, decided by its end, A7) or -1
-  struct Front {
-    uint64_t ew[2][4];
-    uint32_t poff[2];
-    int jt[2];
-    bool ok[2];
-  };
-  auto front = [&](const uint64_t p[2], uint32_t valid, Front &f) {
-#pragma unroll
-    for (int m = 0; m < 2; ++m) {
-      const bool look = ((valid >> m) & 1) && p[m] != 0 && p[m] >= S0;
-      const uint64_t rel = p[m] - S0;
-      const uint64_t pg = rel >> P;
-      f.ok[m] = look && pg < npages;
-      f.poff[m] = (uint32_t)rel & pmask;
-      f.jt[m] = look && !f.ok[m] && p[m] <= Send ? (int)lastu : -1;
-      f.ew[m][0] = f.ew[m][1] = f.ew[m][2] = f.ew[m][3] = 0;
-      if (f.ok[m])  // one LDG.256, not allocated in L1
-        asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
-                     : "=l"(f.ew[m][0]), "=l"(f.ew[m][1]), "=l"(f.ew[m][2]), "=l"(f.ew[m][3])
-                     : "l"(ent + 8 * pg), "l"(pol_t));
-    }
-  };
-
-  // software pipeline: slot values two chunks ahead, page-entry gathers one chunk ahead
-  const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  uint64_t cv[2] = {0, 0}, nv[2] = {0, 0}, nnv[2] = {0, 0};
-  if (c_first < a.nchunks) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c_first), pol_s, cv[0], cv[1]);
-  if (c_first + stride < a.nchunks)
-    ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, nv[0], nv[1]);
-  Front fc, fn;
-  front(cv, valid_of(c_first), fc);
-  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
-    const uint64_t c = cb + lane;
-    if (c + 2 * stride < a.nchunks)
-      ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, nnv[0], nnv[1]);
-    front(nv, valid_of(c + stride), fn);  // the next chunk's entries are in flight while this one finishes
-    const uint64_t a0 = a0base + 16ull * c;
-    const uint32_t valid = valid_of(c);
-
-    // decode: j = j0 + #{starts <= p - A}; j0 is decided by its end, a candidate by its end in the entry
-    // (A7); in a page whose state is valid the entry also gives ACTIVE and the extent: no unit word
-    int j[2];
-    bool k0[2], dec[2];
-    uint64_t key[2];
-    uint32_t cw[2], ps[2];
-#pragma unroll
-    for (int m = 0; m < 2; ++m) {
-      j[m] = fc.jt[m];
-      k0[m] = true;
-      dec[m] = false;
-      key[m] = 0;
-      ps[m] = 0;
-      if (fc.ok[m]) {
-        const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
-        const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT;
-        const uint32_t r = min(fc.poff[m], PD_PAD - 1u);
-        if (V3 && cnt <= (uint32_t)PD_K3) {
-          uint32_t word;
-          const uint32_t k = pd_count5(fc.ew[m], r, word);
-          const bool h = k ? fc.poff[m] <= (word >> 16) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0);
-          j[m] = h ? (int)(j0 + k) : -1;
-          dec[m] = true;
-          ps[m] = (uint32_t)fc.ew[m][1];
-        } else if (!V3 && cnt <= (uint32_t)PD_K2) {  // v2: twelve starts, four per 64-bit subtraction (le4)
-          const uint32_t r2 = r | (r << 16);
-          const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
-          const uint32_t k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
-          const uint32_t off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
-          k0[m] = k == 0;
-          j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
-          key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
-        } else {  // crowded page: starts in the side array, the candidate's size from its unit word
-          const uint64_t ko = pd_crowded(a.pd.ovf, V3 ? (uint32_t)(fc.ew[m][1] >> 32) : (uint32_t)fc.ew[m][1], cnt, r);
-          const uint32_t k = (uint32_t)ko, off = (uint32_t)(ko >> 32);
-          k0[m] = k == 0;
-          j[m] = k ? (int)(j0 + k) : (j0 != 0xFFFFFFFFu && fc.poff[m] < end0 ? (int)j0 : -1);
-          key[m] = cv[m] - fc.poff[m] + off;  // the candidate's base (A + offset)
-        }
-      }
-      cw[m] = 0;
-      if (j[m] >= 0 && !(V3 && (ps[m] & PD_STATE_VALID)))  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
-        asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
-    }
-    uint64_t outv[2] = {cv[0], cv[1]};
-    uint32_t wrote = 0, su[2];
-    bool act[2];
-#pragma unroll
-    for (int m = 0; m < 2; ++m) {
-      const bool vm = (valid >> m) & 1;
-      const bool look = j[m] >= 0;
-      uint64_t hw;
-      if (V3 && (ps[m] & PD_STATE_VALID))  // every unit of the page is ACTIVE with its copy in this extent
-        hw = ((uint64_t)(ps[m] & EXT_MASK) << ESHIFT) | ((uint64_t)(UF_ACTIVE | UF_STORAGE) << FSHIFT);
-      else
-        hw = (cw[m] & HOTC_ESC) && look ? ld_u64_hot(a.tab.hot + j[m], pol_t) : hot_of_hotc(cw[m]);
-      uint64_t sz = hot_size32(hw);
-      if (look && !dec[m] && !k0[m] && sz == BIG_SIZE) sz = a.tab.size64[j[m]];
-      bool hit = look && (dec[m] || k0[m] || cv[m] - key[m] <= sz);  // A7: p - base <= size
-      if (DELTA && vm && cv[m] != 0 && !hit) {  // NEXT-1: delta units, where the main table missed
-        uint64_t db;
-        const int d = delta_override(a, cv[m], hit, db);
-        if (d >= 0) {
-          j[m] = d;
-          hw = ld_u64_hot(a.tab.hot + d, pol_t);
-          hit = true;
-        }
-      }
-      const bool nul = vm && cv[m] == 0;
-      c_nulls += nul;
-      c_hits += hit;
-      c_miss += vm && !nul && !hit;
-      const uint32_t fl = hot_flags(hw);
-      const bool active = (fl & UF_ACTIVE) != 0;
-      // deferred reference (a.defer): the unit was active when the call began -- recorded in the shadow
-      const bool dfr = defer && hit && active;
-      act[m] = false;
-      if (hit && !dfr) {
-        int32_t *RC = a.tab.rc + j[m];
-        if (active) red_add(RC, inc);
-        else act[m] = atomicAdd(RC, inc) == 0;  // refcount 0 -> 1: Alg. 1's activation
-      }
-      if (hit && (fl & UF_STORAGE)) {
-        const uint32_t e = hot_ext(hw);
-        outv[m] = cv[m] + (ES ? s_ext[e] : a.tab.ext_delta[e]);  // Alg. 1: devptr + (ptr - base)
-        wrote |= 1u << m;
-      } else {
-        c_pend += hit;  // activated by this call: completed after the allocation
-      }
-      su[m] = hit ? ((uint32_t)j[m] | (dfr ? SH_DEFER : 0u)) : SH_NONE;
-    }
-    c_tr += __popc(wrote);
-    if (__any_sync(0xffffffffu, act[0] || act[1])) {
-#pragma unroll
-      for (int m = 0; m < 2; ++m) {
-        const unsigned long long ix = warp_append(&a.lc[0], act[m]);
-        if (act[m]) a.act_list[ix] = (uint32_t)j[m];
-      }
-    }
-    // the shadow (CPU pointer, unit) and the slots
-    const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
-    if (valid == 3u) {
-      st_stream2(reinterpret_cast<void *>(a0), pol_s, outv[0], outv[1]);
-      if (!(i0 & 1)) {
-        st_stream2(shp + i0, pol_s, make_shw(cv[0], su[0]), make_shw(cv[1], su[1]));
-      } else {
-#pragma unroll
-        for (int m = 0; m < 2; ++m) shp[i0 + m] = make_shw(cv[m], su[m]);
-      }
-    } else if (valid) {
-#pragma unroll
-      for (int m = 0; m < 2; ++m)
-        if ((valid >> m) & 1) {
-          st_stream1(reinterpret_cast<void *>(a0 + 8ull * m), pol_s, outv[m]);
-          shp[i0 + m] = make_shw(cv[m], su[m]);
-        }
-    }
-    {  // hit mask: 2 bits per chunk, 16 chunks per word (lanes 0-15: word cb/16, lanes 16-31: the next)
-      const uint32_t b = wrote << (2u * (lane & 15));
-      const uint32_t w0 = warp_or(lane < 16 ? b : 0u), w1 = warp_or(lane < 16 ? 0u : b);
-      const uint64_t wi = cb >> 4;
-      if (lane == 0) a.hitmask[wi] = w0;
-      else if (lane == 16 && cb + 16 < a.nchunks) a.hitmask[wi + 1] = w1;
-    }
-    cv[0] = nv[0];
-    cv[1] = nv[1];
-    nv[0] = nnv[0];
-    nv[1] = nnv[1];
-    fc = fn;
-  }
-  flush_count(&a.st->nulls, (unsigned long long)c_nulls * (unsigned)inc);  // inc = k: k sequential calls
-  flush_count(&a.st->hits, (unsigned long long)c_hits * (unsigned)inc);
-  flush_count(&a.st->misses, (unsigned long long)c_miss * (unsigned)inc);
-  flush_count(&a.st->pending, c_pend);
-  flush_count(&a.st->translated, c_tr);
-}
-
-template <bool ES, bool V3, bool DELTA>
-static int launch_fwd_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
-  const size_t smem = (ES ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
-  static bool configured = false;
-  if (!configured) {
-    int dev = 0, optin = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    cudaError_t e = cudaFuncSetAttribute(k_fwd_lean<ES, V3, DELTA>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
-    if (e != cudaSuccess) return (int)e;
-    configured = true;
-  }
-  constexpr int T = V3 ? FWD_LEAN_THREADS_V3 : FWD_LEAN_THREADS;
-  const uint64_t want = (a.nchunks + T - 1) / T;
-  const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
-  (void)cudaGetLastError();
-  k_fwd_lean<ES, V3, DELTA><<<grid, T, smem, s>>>(a);
-  return (int)cudaGetLastError();
-}
-
 // -------------------------------------------------------------------------------------------------
-// k_fwd_fast: k_fwd_lean's results, counters and lists with the common chunk on a short path (round 2,
-// VERDICT r1 item 4 "instructions": k_fwd_lean spends 270 thread instructions per slot, issue-bound even
-// with every table L2-resident -- profiles/r02q_C_summary.md).  A warp takes the short path for a chunk
-// when all of its 64 slots are ordinary: a whole chunk, a page of this segment, a hit on a unit that is
-// ACTIVE with its copy (its reference deferred into the shadow, a.defer), no escaped unit word.  The short
-// path keeps no per-slot counters (a fast chunk is two hits, two translations), builds no masks (its
-// hit-mask words are all ones) and takes no atomics.  Any other chunk -- a NULL, a miss, an activation,
-// a ragged end, a huge unit, a delta unit -- is redone by fwd_chunk_slow (the k_fwd_lean iteration, one
-// warp-uniform call that recomputes the chunk from its two slot values).  Crowded pages stay on the
-// short path (a divergent side-array count, as in k_fwd_lean).
+// k_fwd_fast: the forward map of cgcm_mapArrayDevice (a1 + a2 of Alg. 1) over ONE in-place segment with
+// a shadow, through a page directory of ONE address segment (the case of every config-C/E-shaped table);
+// same results, counters and lists as k_map_pd<1>.  Software pipeline: slot values two chunks ahead, the
+// page entries (one LDG.256 each) one chunk ahead.  A warp takes the short path for a chunk when all of
+// its 64 slots are ordinary: a whole chunk, a page of this segment, a hit on a unit that is ACTIVE with
+// its copy (its reference deferred into the shadow, a.defer), no escaped unit word.  The short path
+// keeps no per-slot counters (a fast chunk is two hits, two translations), builds no masks (its hit-mask
+// words are all ones) and takes no atomics; crowded pages stay on it (a divergent side-array count).
+// Any other chunk -- a NULL, a miss, an activation, a ragged end, a huge unit, a delta unit -- is redone
+// by fwd_chunk_slow, one warp-uniform call that recomputes the chunk from its two slot values.
+// Round 2 (profiles/r02t_ab.log): the round-1 structure (every slot through the general code, 270
+// thread instructions per slot) took 0.709 ms at C, this one 0.556; at E 3.28 -> 3.22 ms (E is bound by
+// its two random L2 gathers per slot, not by instructions: profiles/r02u_ab_tablesize.log).
 // -------------------------------------------------------------------------------------------------
 #ifdef CGCM_FWD_FAST_THREADS
 constexpr int FWD_FAST_THREADS = CGCM_FWD_FAST_THREADS;
@@ -1721,7 +1475,7 @@ constexpr int FWD_FAST_THREADS = CGCM_FWD_FAST_THREADS;
 constexpr int FWD_FAST_THREADS = 768;
 #endif
 
-// the k_fwd_lean iteration for chunk c (slot values cv) of the warp whose first chunk is cb; called by
+// every case of chunk c (slot values cv) of the warp whose first chunk is cb; called by
 // all 32 lanes of the warp (warp collectives: activation list, hit mask, counters)
 template <bool ES, bool V3, bool DELTA>
 __device__ __noinline__ void fwd_chunk_slow(const SlotArgs &a, const uint64_t *s_ext, uint64_t c, uint64_t cb,
@@ -1904,7 +1658,7 @@ __global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_fast(const __grid_c
   const uint64_t npages = a.pd.seg_meta[1];
   const uint32_t *ent = a.pd.ent + 8ull * a.pd.seg_meta[0];
   const uint32_t pmask = (1u << P) - 1u;
-  const uint32_t nch = (uint32_t)a.nchunks;  // < 2^32 (launch_fwd_fast1)
+  const uint32_t nch = (uint32_t)a.nchunks;  // < 2^31 (launch_fwd_fast1; larger calls: k_fwd_big)
   // whole chunks (both slots in the segment): [f0, f1)
   const uint32_t f0 = sh_odd ? 1u : 0u;
   const uint32_t f1 = (uint32_t)((sg.ptr + 8ull * sg.n - a0base) >> 4);
@@ -2046,24 +1800,113 @@ static int launch_fwd_fast1(const SlotArgs &a, int nsm, cudaStream_t s) {
   return (int)cudaGetLastError();
 }
 
-// -------------------------------------------------------------------------------------------------
-// k_rev_lean: the reverse pass of cgcm_unmapArrayDevice (a3 + a4 [+ Alg. 3 release]) over ONE in-place
-// segment that carries the forward map's shadow, in snapshot mode (no per-unit journal; releases as
-// reductions checked afterwards by k_release_scan).  Same decisions, counters and lists as
-// k_unmap_sh<WRITE|GATE|HITMASK[|DEC], false> in that mode, with the bookkeeping cut to what a slot
-// needs: the rare paths (copy list, deferred materialisation) run under warp votes, the hit / slow
-// masks are built with warp reductions (redux.sync), and the slot stores are unconditional 16-byte
-// writes of whole chunks (a slot that is not translated is written back unchanged; only the ragged
-// ends of the segment are stored slot by slot).  Slots whose shadow check fails go to k_slots
-// SEL_SLOW exactly as after k_unmap_sh.
-// -------------------------------------------------------------------------------------------------
-constexpr int REV_LEAN_THREADS = 768;
+constexpr int REV_THREADS = 768;  // measured: 768 > 640 > 512 (round 2, profiles/r02f_ab.log)
 
-template <bool DEC, bool ES>  // ES: the extent deltas are staged in shared memory
-__global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
+// -------------------------------------------------------------------------------------------------
+// k_rev_fast: the reverse pass of cgcm_unmapArrayDevice (a3 + a4 [+ Alg. 3 release]) over ONE in-place
+// segment that carries the forward map's shadow, in snapshot mode (no per-unit journal; releases as
+// reductions checked afterwards by k_release_scan); same decisions, counters and lists as
+// k_unmap_sh<WRITE|GATE|HITMASK[|DEC], false> in that mode.  Pipeline: slot values and shadow words two
+// chunks ahead, the units' 8-byte state words one ahead.  A warp takes the short path for a chunk when
+// all of its 64 slots are ordinary: a whole chunk, a recorded unit that is ACTIVE with the slot provably
+// unchanged (shadow check), and an epoch gate that needs no copy (current, or stale and read-only: the
+// epoch store only); releases and deferred references are predicated reductions.  Any other chunk is
+// redone by rev_chunk_slow (copy list under a warp vote, hit / slow masks by warp reductions); slots
+// whose shadow check fails go to k_slots SEL_SLOW afterwards.  Round 2: E 1.71 -> 1.60 ms, C 0.468 ->
+// 0.436 (profiles/r02v_ab.log).
+// -------------------------------------------------------------------------------------------------
+struct RevIn {
+  uint64_t g[2], h[2];  // slot values, shadow words (cgcm_dev.h make_shw)
+  uint32_t valid;
+};
+
+// every case of chunk c (inputs x, state words w) of the warp whose first chunk is cb;
+// called by all 32 lanes of the warp
+template <bool DEC, bool ES>
+__device__ __noinline__ void rev_chunk_slow(const SlotArgs &a, const ulonglong2 *s_dl, const uint32_t *s_len, uint64_t c,
+                                            uint64_t cb, RevIn cur, uint64_t w0, uint64_t w1) {
+  const uint64_t pol_s = policy_evict_first();
+  const int lane = threadIdx.x & 31;
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull;
+  const uint32_t n_ext = (uint32_t)a.tab.n_ext, cur_ep = a.epoch;
+  const uint64_t cw[2] = {w0, w1};
+  unsigned c_nulls = 0, c_hits = 0, c_slow = 0;
+  bool hit[2], slow[2], cp[2];
+  uint64_t outv[2];
+  bool rare = false;
+#pragma unroll
+  for (int m = 0; m < 2; ++m) {
+    const bool vm = (cur.valid >> m) & 1;
+    const uint64_t g = cur.g[m], w = cw[m];
+    const uint32_t e = hot_ext(w), fl = hot_flags(w), su = sh_unit(shw_unit(cur.h[m]));
+    const bool look = vm && g != 0;
+    uint64_t hr = 0;
+    if (look && su != SH_NONE && (fl & UF_ACTIVE) && e < n_ext) {
+      const ulonglong2 dl = ES ? s_dl[e] : make_ulonglong2(a.tab.ext_delta[e], a.tab.ext_lo[e]);
+      hr = sh_reverse(g, cur.h[m], dl.x, dl.y, ES ? s_len[e] : a.tab.ext_len[e]);
+    }
+    hit[m] = hr != 0;
+    slow[m] = look && !hit[m];
+    c_nulls += vm && g == 0;
+    c_hits += hit[m];
+    outv[m] = hit[m] ? hr : g;  // reverse: base + (g - devbase), the recorded CPU pointer
+    const bool stale = hit[m] && st_epoch(w) != cur_ep;  // Alg. 2's epoch gate
+    cp[m] = false;
+    if (stale) {
+      if (fl & UF_READONLY) {
+        *lo_word(a.tab.st + su) = cur_ep;  // Alg. 2 line 3 only: never copied back
+      } else {
+        cp[m] = atomicExch(lo_word(a.tab.st + su), cur_ep) != cur_ep;  // stale and not read-only: copy
+      }
+    }
+    // references: a deferred one (a.defer) is dropped by a released hit, materialised otherwise
+    const bool dfr = a.defer && vm && sh_deferred(shw_unit(cur.h[m]));
+    const bool drop = DEC && dfr && hit[m];
+    if (dfr && !drop) red_add(a.tab.rc + su, 1);
+    if (DEC && hit[m] && !drop) red_add(a.tab.rc + su, -sg.inc);  // Alg. 3, checked by k_release_scan
+    rare = rare || cp[m];
+  }
+  c_slow += slow[0] + slow[1];
+  if (__any_sync(0xffffffffu, rare)) {  // copy list of this warp's stale writable units
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const unsigned long long cx = warp_append(&a.lc[3], cp[m]);
+      if (cp[m]) a.copy_list[cx] = sh_unit(shw_unit(cur.h[m]));
+    }
+  }
+  if (cur.valid == 3u) {
+    st_stream2(reinterpret_cast<void *>(a0base + 16ull * c), pol_s, outv[0], outv[1]);
+  } else {
+#pragma unroll
+    for (int m = 0; m < 2; ++m)
+      if ((cur.valid >> m) & 1) st_stream1(reinterpret_cast<void *>(a0base + 16ull * c + 8ull * m), pol_s, outv[m]);
+  }
+  {  // 2 bits per chunk, 16 chunks per word: lanes 0-15 make word cb/16, lanes 16-31 the next
+    const uint32_t sh = 2u * (lane & 15);
+    const uint32_t hb = ((hit[0] ? 1u : 0u) | (hit[1] ? 2u : 0u)) << sh;
+    const uint32_t sb = ((slow[0] ? 1u : 0u) | (slow[1] ? 2u : 0u)) << sh;
+    const uint32_t lo = lane < 16;
+    const uint32_t h0 = warp_or(lo ? hb : 0u), h1 = warp_or(lo ? 0u : hb);
+    const uint32_t s0 = warp_or(lo ? sb : 0u), s1 = warp_or(lo ? 0u : sb);
+    const uint64_t wi = cb >> 4;
+    if (lane == 0) {
+      a.hitmask[wi] = h0;
+      a.slowmask[wi] = s0;
+    } else if (lane == 16 && cb + 16 < a.nchunks) {
+      a.hitmask[wi + 1] = h1;
+      a.slowmask[wi + 1] = s1;
+    }
+  }
+  flush_count(&a.st->nulls, c_nulls);
+  flush_count(&a.st->hits, c_hits);
+  flush_count(&a.st->translated, c_hits);
+  flush_count(a.slowcount, c_slow);
+}
+
+template <bool DEC, bool ES>
+__global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fast(const __grid_constant__ SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
-  // the extents' deltas and device ranges (the shadow check), staged when few: {delta, lo} as one 16-byte
-  // word per extent (one LDS.128 per slot), the lengths beside them
   ulonglong2 *s_dl = reinterpret_cast<ulonglong2 *>(smem);
   uint32_t *s_len = reinterpret_cast<uint32_t *>(s_dl + (ES ? a.tab.n_ext : 0));
   if (ES)
@@ -2074,27 +1917,28 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
   __syncthreads();
   const uint64_t pol_s = policy_evict_first();
   const uint64_t pol_t = policy_evict_last();
-  const int lane = threadIdx.x & 31;
+  const uint32_t lane = threadIdx.x & 31;
   const Seg sg = a.segs[0];
   const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n;
-  const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);  // shadow words (make_shw)
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);
+  const bool sh_odd = (sg.ptr >> 3) & 1;
+  const uint32_t nch = (uint32_t)a.nchunks;  // < 2^31 (launch_rev_fast1; larger calls: k_rev_big)
+  const uint32_t f0 = sh_odd ? 1u : 0u, f1 = (uint32_t)((hi - a0base) >> 4);  // whole chunks [f0, f1)
+  const uint32_t stride = gridDim.x * blockDim.x;
   const uint32_t n_ext = (uint32_t)a.tab.n_ext, cur_ep = a.epoch;
-  unsigned c_nulls = 0, c_hits = 0, c_slow = 0;
+  const int32_t dec = -sg.inc;
+  const bool defer = a.defer != 0;
+  uint32_t c_fast = 0;
 
-  struct In {
-    uint64_t g[2], h[2];  // slot values, shadow words (cgcm_dev.h make_shw)
-    uint32_t valid;
-  };
-  auto load_in = [&](uint64_t c, In &x) {
+  auto load_in = [&](uint32_t c, RevIn &x) {
     x.g[0] = x.g[1] = 0;
-    x.h[0] = x.h[1] = make_shw(0, SH_NONE);  // (the unit word is read where it is used: no stall at the load)
+    x.h[0] = x.h[1] = make_shw(0, SH_NONE);
     x.valid = 0;
-    if (c >= a.nchunks) return;
+    if (c >= nch) return;
     const uint64_t a0 = a0base + 16ull * c;
     x.valid = (a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u);
     const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
-    if (x.valid == 3u && !(i0 & 1)) {
+    if (x.valid == 3u && !sh_odd) {
       ld_stream2(reinterpret_cast<const void *>(a0), pol_s, x.g[0], x.g[1]);
       ld_stream2(shp + i0, pol_s, x.h[0], x.h[1]);
     } else {
@@ -2106,92 +1950,61 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
         }
     }
   };
-  auto gather = [&](const In &x, uint64_t w[2]) {
+  auto gather = [&](const RevIn &x, uint64_t w[2]) {
 #pragma unroll
     for (int m = 0; m < 2; ++m)
       w[m] = (shw_unit(x.h[m]) != SH_NONE && x.g[m] != 0) ? ld_u64_hot(a.tab.st + sh_unit(shw_unit(x.h[m])), pol_t) : 0ull;
   };
 
-  const uint64_t c_first = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  In cur, nxt, nn;
+  const uint32_t c_first = blockIdx.x * blockDim.x + threadIdx.x;
+  RevIn cur, nxt, nn;
   uint64_t cw[2], nw[2];
   load_in(c_first, cur);
   load_in(c_first + stride, nxt);
   gather(cur, cw);
-  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
-    const uint64_t c = cb + lane;
+  for (uint32_t cb = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < nch; cb += stride) {
+    const uint32_t c = cb + lane;
     load_in(c + 2 * stride, nn);
     gather(nxt, nw);
 
-    bool hit[2], slow[2], cp[2];
-    uint64_t outv[2];
-    bool rare = false;
+    bool rare = !(c >= f0 && c < f1);
+    uint64_t hr[2];
+    uint32_t su[2];
+    bool stale[2], dfr[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      const bool vm = (cur.valid >> m) & 1;
       const uint64_t g = cur.g[m], w = cw[m];
-      const uint32_t e = hot_ext(w), fl = hot_flags(w), su = sh_unit(shw_unit(cur.h[m]));
-      const bool look = vm && g != 0;
-      uint64_t hr = 0;
-      if (look && su != SH_NONE && (fl & UF_ACTIVE) && e < n_ext) {
-        const ulonglong2 dl = ES ? s_dl[e] : make_ulonglong2(a.tab.ext_delta[e], a.tab.ext_lo[e]);
-#ifdef CGCM_SH_NOCHECK  // timing experiment only: no range check (NOT exact)
-        hr = (uint32_t)(g - dl.x) == (uint32_t)cur.h[m] ? g - dl.x : 0ull;
-#else
-        hr = sh_reverse(g, cur.h[m], dl.x, dl.y, ES ? s_len[e] : a.tab.ext_len[e]);
-#endif
+      const uint32_t uw = shw_unit(cur.h[m]), e = hot_ext(w), fl = hot_flags(w);
+      su[m] = uw & ~SH_DEFER;
+      ulonglong2 dl = make_ulonglong2(0, 0);
+      uint32_t len = 0;
+      if (e < n_ext) {
+        dl = ES ? s_dl[e] : make_ulonglong2(a.tab.ext_delta[e], a.tab.ext_lo[e]);
+        len = ES ? s_len[e] : a.tab.ext_len[e];
       }
-      hit[m] = hr != 0;
-      slow[m] = look && !hit[m];
-      c_nulls += vm && g == 0;
-      c_hits += hit[m];
-      outv[m] = hit[m] ? hr : g;  // reverse: base + (g - devbase), the recorded CPU pointer
-      // Alg. 2: the epoch gate of a hit whose unit is stale (rare after the first slot of each unit)
-      const bool stale = hit[m] && st_epoch(w) != cur_ep;
-      cp[m] = false;
-      if (stale) {
-        if (fl & UF_READONLY) {
-          *lo_word(a.tab.st + su) = cur_ep;  // Alg. 2 line 3 only: never copied back
-        } else {
-          cp[m] = atomicExch(lo_word(a.tab.st + su), cur_ep) != cur_ep;  // stale and not read-only: copy
-        }
-      }
-      // references: a deferred one (a.defer) is dropped by a released hit, materialised otherwise
-      const bool dfr = a.defer && vm && sh_deferred(shw_unit(cur.h[m]));
-      const bool drop = DEC && dfr && hit[m];
-      if (dfr && !drop) red_add(a.tab.rc + su, 1);
-      if (DEC && hit[m] && !drop) red_add(a.tab.rc + su, -sg.inc);  // Alg. 3, checked by k_release_scan
-      rare = rare || cp[m];
+      // unchanged since the forward map (cgcm_dev.h make_shw): the recorded CPU pointer
+      hr[m] = g - dl.x;
+      const bool ok = g != 0 && uw != SH_NONE && (fl & UF_ACTIVE) && e < n_ext && g - dl.y < (uint64_t)len &&
+                      (uint32_t)hr[m] == (uint32_t)cur.h[m] && hr[m] != 0;
+      stale[m] = st_epoch(w) != cur_ep;
+      dfr[m] = defer && (uw & SH_DEFER);
+      rare = rare || !ok || (stale[m] && !(fl & UF_READONLY));
     }
-    c_slow += slow[0] + slow[1];
-    if (__any_sync(0xffffffffu, rare)) {  // copy list of this warp's stale writable units
+    if (__any_sync(0xffffffffu, rare)) {
+      rev_chunk_slow<DEC, ES>(a, s_dl, s_len, c, cb, cur, cw[0], cw[1]);
+    } else {
+      ++c_fast;
 #pragma unroll
       for (int m = 0; m < 2; ++m) {
-        const unsigned long long cx = warp_append(&a.lc[3], cp[m]);
-        if (cp[m]) a.copy_list[cx] = sh_unit(shw_unit(cur.h[m]));
+        if (stale[m]) *lo_word(a.tab.st + su[m]) = cur_ep;  // Alg. 2 line 3 (read-only: never copied back)
+        if (DEC && !dfr[m]) red_add(a.tab.rc + su[m], dec);  // Alg. 3 (a deferred reference is dropped)
+        if (!DEC && dfr[m]) red_add(a.tab.rc + su[m], 1);   // materialised
       }
-    }
-    if (cur.valid == 3u) {
-      st_stream2(reinterpret_cast<void *>(a0base + 16ull * c), pol_s, outv[0], outv[1]);
-    } else {
-#pragma unroll
-      for (int m = 0; m < 2; ++m)
-        if ((cur.valid >> m) & 1) st_stream1(reinterpret_cast<void *>(a0base + 16ull * c + 8ull * m), pol_s, outv[m]);
-    }
-    {  // 2 bits per chunk, 16 chunks per word: lanes 0-15 make word cb/16, lanes 16-31 the next
-      const uint32_t sh = 2u * (lane & 15);
-      const uint32_t hb = ((hit[0] ? 1u : 0u) | (hit[1] ? 2u : 0u)) << sh;
-      const uint32_t sb = ((slow[0] ? 1u : 0u) | (slow[1] ? 2u : 0u)) << sh;
-      const uint32_t lo = lane < 16;
-      const uint32_t h0 = warp_or(lo ? hb : 0u), h1 = warp_or(lo ? 0u : hb);
-      const uint32_t s0 = warp_or(lo ? sb : 0u), s1 = warp_or(lo ? 0u : sb);
-      const uint64_t wi = cb >> 4;
-      if (lane == 0) {
-        a.hitmask[wi] = h0;
-        a.slowmask[wi] = s0;
-      } else if (lane == 16 && cb + 16 < a.nchunks) {
-        a.hitmask[wi + 1] = h1;
-        a.slowmask[wi + 1] = s1;
+      st_stream2(reinterpret_cast<void *>(a0base + 16ull * c), pol_s, hr[0], hr[1]);
+      if (lane == 0 || (lane == 16 && cb + 16 < nch)) {
+        const uint32_t wi = (cb >> 4) + (lane >> 4);
+        a.hitmask[wi] = 0xFFFFFFFFu;
+        a.slowmask[wi] = 0u;
       }
     }
     cur = nxt;
@@ -2199,33 +2012,115 @@ __global__ void __launch_bounds__(REV_LEAN_THREADS, 1) k_rev_lean(SlotArgs a) {
     cw[0] = nw[0];
     cw[1] = nw[1];
   }
-  flush_count(&a.st->nulls, c_nulls);
-  flush_count(&a.st->hits, c_hits);
-  flush_count(&a.st->translated, c_hits);
-  flush_count(a.slowcount, c_slow);
+  flush_count(&a.st->hits, 2ull * c_fast);
+  flush_count(&a.st->translated, 2ull * c_fast);
 }
 
 template <bool DEC, bool ES>
-static int launch_rev_lean1(const SlotArgs &a, int nsm, cudaStream_t s) {
+static int launch_rev_fast1(const SlotArgs &a, int nsm, cudaStream_t s) {
   const size_t smem = (ES ? al16(20 * (size_t)a.tab.n_ext) + 16 : 0) + 64;
   static bool configured = false;
   if (!configured) {
     int dev = 0, optin = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    cudaError_t e = cudaFuncSetAttribute(k_rev_lean<DEC, ES>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    cudaError_t e = cudaFuncSetAttribute(k_rev_fast<DEC, ES>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
     if (e != cudaSuccess) return (int)e;
     configured = true;
   }
-  const uint64_t want = (a.nchunks + REV_LEAN_THREADS - 1) / REV_LEAN_THREADS;
+  const uint64_t want = (a.nchunks + REV_THREADS - 1) / REV_THREADS;
   const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
-  k_rev_lean<DEC, ES><<<grid, REV_LEAN_THREADS, smem, s>>>(a);
+  k_rev_fast<DEC, ES><<<grid, REV_THREADS, smem, s>>>(a);
+  return (int)cudaGetLastError();
+}
+
+
+// Calls of 2^31 chunks or more (32 GiB of slots): every chunk through the general per-chunk code
+// (64-bit chunk indices; no pipeline).
+template <bool ES, bool V3, bool DELTA>
+__global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_big(const __grid_constant__ SlotArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
+  if (ES)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
+  __syncthreads();
+  const uint64_t a0base = a.segs[0].ptr & ~15ull, stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
+    const uint64_t c = cb + (threadIdx.x & 31);
+    uint64_t v0 = 0, v1 = 0;
+    if (c < a.nchunks) {
+      const uint64_t a0 = a0base + 16ull * c;
+      const Seg &sg = a.segs[0];
+      if (a0 >= sg.ptr) v0 = reinterpret_cast<const uint64_t *>(a0)[0];
+      if (a0 + 8 < sg.ptr + 8ull * sg.n) v1 = reinterpret_cast<const uint64_t *>(a0)[1];
+    }
+    fwd_chunk_slow<ES, V3, DELTA>(a, s_ext, c, cb, v0, v1);
+  }
+}
+template <bool DEC, bool ES>
+__global__ void __launch_bounds__(REV_THREADS, 1) k_rev_big(const __grid_constant__ SlotArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  ulonglong2 *s_dl = reinterpret_cast<ulonglong2 *>(smem);
+  uint32_t *s_len = reinterpret_cast<uint32_t *>(s_dl + (ES ? a.tab.n_ext : 0));
+  if (ES)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) {
+      s_dl[t] = make_ulonglong2(a.tab.ext_delta[t], a.tab.ext_lo[t]);
+      s_len[t] = a.tab.ext_len[t];
+    }
+  __syncthreads();
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n, stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);
+  for (uint64_t cb = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < a.nchunks; cb += stride) {
+    const uint64_t c = cb + (threadIdx.x & 31);
+    RevIn x;
+    x.g[0] = x.g[1] = 0;
+    x.h[0] = x.h[1] = make_shw(0, SH_NONE);
+    x.valid = 0;
+    uint64_t w[2] = {0, 0};
+    if (c < a.nchunks) {
+      const uint64_t a0 = a0base + 16ull * c;
+      x.valid = (a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u);
+      const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
+      for (int m = 0; m < 2; ++m)
+        if ((x.valid >> m) & 1) {
+          x.g[m] = reinterpret_cast<const uint64_t *>(a0)[m];
+          x.h[m] = shp[i0 + m];
+          if (shw_unit(x.h[m]) != SH_NONE && x.g[m] != 0) w[m] = a.tab.st[sh_unit(shw_unit(x.h[m]))];
+        }
+    }
+    rev_chunk_slow<DEC, ES>(a, s_dl, s_len, c, cb, x, w[0], w[1]);
+  }
+}
+template <bool ES, bool V3, bool DELTA>
+static int launch_fwd_big1(const SlotArgs &a, int nsm, cudaStream_t s) {
+  const size_t smem = (ES ? al16(8 * (size_t)a.tab.n_ext) : 0) + 64;
+  int dev = 0, optin = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  cudaError_t e = cudaFuncSetAttribute(k_fwd_big<ES, V3, DELTA>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+  if (e != cudaSuccess) return (int)e;
+  k_fwd_big<ES, V3, DELTA><<<nsm, FWD_FAST_THREADS, smem, s>>>(a);
+  return (int)cudaGetLastError();
+}
+template <bool DEC, bool ES>
+static int launch_rev_big1(const SlotArgs &a, int nsm, cudaStream_t s) {
+  const size_t smem = (ES ? al16(20 * (size_t)a.tab.n_ext) + 16 : 0) + 64;
+  int dev = 0, optin = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  cudaError_t e = cudaFuncSetAttribute(k_rev_big<DEC, ES>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+  if (e != cudaSuccess) return (int)e;
+  k_rev_big<DEC, ES><<<nsm, REV_THREADS, smem, s>>>(a);
   return (int)cudaGetLastError();
 }
 template <bool DEC>
 static int launch_rev_lean(const SlotArgs &a, int nsm, cudaStream_t s) {
-  return a.tab.n_ext <= EXT_SMEM ? launch_rev_lean1<DEC, true>(a, nsm, s) : launch_rev_lean1<DEC, false>(a, nsm, s);
+  const bool es = a.tab.n_ext <= EXT_SMEM;
+  static const bool force_big = std::getenv("CGCM_FORCE_BIG") != nullptr;  // tests: the general per-chunk code
+  if (a.nchunks >= (1ull << 31) || force_big) return es ? launch_rev_big1<DEC, true>(a, nsm, s) : launch_rev_big1<DEC, false>(a, nsm, s);
+  return es ? launch_rev_fast1<DEC, true>(a, nsm, s) : launch_rev_fast1<DEC, false>(a, nsm, s);
 }
 
 // the operation sets the runtime uses
@@ -2291,13 +2186,13 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, i
     static const bool no_lean = std::getenv("CGCM_NO_LEAN") != nullptr;  // A/B experiments
     if (a.segs_host_shadow && a.pd.nseg == 1 && !no_lean) {
       const bool es = a.tab.n_ext <= EXT_SMEM, v3 = a.pd.v3 != 0, dl = a.dn > 0;
-      static const bool fwd_old = std::getenv("CGCM_FWD_OLD") != nullptr;  // A/B: k_fwd_lean
-      const bool fast = !fwd_old && a.nchunks < (1ull << 31);
-#define FWD_LEAN(E, V, D) \
-  if (es == E && v3 == V && dl == D) return fast ? launch_fwd_fast1<E, V, D>(a, nsm, s) : launch_fwd_lean1<E, V, D>(a, nsm, s);
-      FWD_LEAN(true, true, false) FWD_LEAN(true, false, false) FWD_LEAN(false, true, false) FWD_LEAN(false, false, false)
-      FWD_LEAN(true, true, true) FWD_LEAN(true, false, true) FWD_LEAN(false, true, true) FWD_LEAN(false, false, true)
-#undef FWD_LEAN
+      static const bool force_big = std::getenv("CGCM_FORCE_BIG") != nullptr;  // tests: the general per-chunk code
+      const bool big = a.nchunks >= (1ull << 31) || force_big;
+#define FWD_PASS(E, V, D) \
+  if (es == E && v3 == V && dl == D) return big ? launch_fwd_big1<E, V, D>(a, nsm, s) : launch_fwd_fast1<E, V, D>(a, nsm, s);
+      FWD_PASS(true, true, false) FWD_PASS(true, false, false) FWD_PASS(false, true, false) FWD_PASS(false, false, false)
+      FWD_PASS(true, true, true) FWD_PASS(true, false, true) FWD_PASS(false, true, true) FWD_PASS(false, false, true)
+#undef FWD_PASS
     }
     return a.segs_host_shadow ? launch_map_pd<1>(a, nsm, s) : launch_map_pd<0>(a, nsm, s);
   }
