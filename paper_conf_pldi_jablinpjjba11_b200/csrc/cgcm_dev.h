@@ -252,6 +252,10 @@ struct SlotArgs {
   const uint64_t *dkeys;
   const uint32_t *dids;
   int dn;
+  // the pipelined single-segment passes (k_fwd_fast, k_rev_fast) list here the first chunk of every warp
+  // group they leave to the general per-chunk code (k_fwd_fix, k_rev_fix); wcount is zeroed per launch
+  uint32_t *wlist;
+  unsigned long long *wcount;
 };
 // Forward-map shadow (8 B per slot): the low 32 bits of the slot's CPU pointer | the unit word << 32.  The
 // unit word is unit index | SH_DEFER (the slot's reference is not in rc yet); SH_NONE: no unit.  A reverse

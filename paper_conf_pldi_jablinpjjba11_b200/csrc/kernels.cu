@@ -1435,7 +1435,7 @@ __device__ __forceinline__ uint32_t off_at(uint64_t q1, uint64_t q2, uint64_t q3
 }
 // crowded page (more than PD_K starts): count in the side array, one sector per 16 offsets; returns
 // k | (offset of start k - 1) << 32
-__device__ __noinline__ uint64_t pd_crowded(const uint16_t *ovf, uint32_t first, uint32_t cnt, uint32_t r) {
+__device__ __forceinline__ uint64_t pd_crowded_i(const uint16_t *ovf, uint32_t first, uint32_t cnt, uint32_t r) {
   const uint64_t r4 = (uint64_t)r * 0x0001000100010001ull;
   uint32_t k = 0, off = 0;
   for (uint32_t t = 0; t < cnt; t += 16) {
@@ -1452,6 +1452,9 @@ __device__ __noinline__ uint64_t pd_crowded(const uint16_t *ovf, uint32_t first,
     if (c < 16) break;  // later sectors hold larger offsets only
   }
   return (uint64_t)k | ((uint64_t)off << 32);
+}
+__device__ __noinline__ uint64_t pd_crowded(const uint16_t *ovf, uint32_t first, uint32_t cnt, uint32_t r) {
+  return pd_crowded_i(ovf, first, cnt, r);
 }
 
 // -------------------------------------------------------------------------------------------------
@@ -1666,7 +1669,8 @@ __global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_fast(const __grid_c
   const uint32_t stride = gridDim.x * blockDim.x;
   uint32_t c_fast = 0;
 
-  struct Fr {
+  struct Fr {  // one chunk in flight: its slot values and page entries
+    uint64_t v0, v1;
     uint64_t ew[2][4];
     uint32_t poff[2];
     bool ok[2];
@@ -1685,99 +1689,133 @@ __global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_fast(const __grid_c
                      : "l"(ent + 8 * pg), "l"(pol_t));
     }
   };
+  // one pipeline step for the warp's chunk cb: the values two chunks ahead go to (ld0, ld1), the entries
+  // of the next chunk (values pv0, pv1) to fn, and chunk fc is translated.  The loop runs the step twice
+  // with the roles of the two Fr buffers and the two value buffers swapped (no register copies).
+  auto step = [&](Fr &fc, Fr &fn, uint64_t &ld0, uint64_t &ld1, uint64_t pv0, uint64_t pv1, uint32_t cb) {
+      const uint32_t c = cb + lane;
+      if (c + 2 * stride < nch)
+        ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, ld0, ld1);
+      fn.v0 = pv0;
+      fn.v1 = pv1;
+      front(pv0, pv1, fn);  // the next chunk's entries are in flight while this one finishes
+
+      // decode: j = j0 + #{starts <= p - A}; the candidate's distance dl = p - base (A7: hit iff dl <= size)
+      bool rare = !(fast_ok && c >= f0 && c < f1);
+      uint32_t j[2], cw[2], ext[2];
+  #pragma unroll
+      for (int m = 0; m < 2; ++m) {
+        const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
+        const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT, po = fc.poff[m];
+        const uint32_t r = min(po, PD_PAD - 1u);
+        const bool okj0 = j0 != 0xFFFFFFFFu && po < end0;  // j0's end decides (A7)
+        uint32_t k, dl = 0;
+        bool hit = false, known = false;  // known: decided by the entry (v3), with the page state
+        uint32_t ps = 0;
+        if (V3 && cnt <= (uint32_t)PD_K3) {
+          uint32_t word;
+          k = pd_count5(fc.ew[m], r, word);
+          hit = k ? po <= (word >> 16) : okj0;
+          ps = (uint32_t)fc.ew[m][1];
+          known = true;
+        } else {
+          uint32_t off;
+          if (!V3 && cnt <= (uint32_t)PD_K2) {
+            const uint32_t r2 = r | (r << 16);
+            const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
+            k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
+            off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
+          } else if (fc.ok[m]) {  // crowded page: the side array
+            const uint64_t ko = pd_crowded_i(a.pd.ovf, V3 ? (uint32_t)(fc.ew[m][1] >> 32) : (uint32_t)fc.ew[m][1], cnt, r);
+            k = (uint32_t)ko;
+            off = (uint32_t)(ko >> 32);
+          } else {
+            k = off = 0;
+          }
+          dl = po - off;
+          hit = k ? true : okj0;  // k > 0: decided by the candidate's size (unit word)
+        }
+        j[m] = j0 + k;
+        rare = rare || !fc.ok[m] || !hit;
+        const bool st_valid = V3 && known && (ps & PD_STATE_VALID);
+        cw[m] = 0;
+        if (fc.ok[m] && hit && !st_valid)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
+          asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
+        ext[m] = st_valid ? (ps & (uint32_t)EXT_MASK) : 0xFFFFFFFFu;
+        if (!st_valid) {
+          // ACTIVE with its copy, no escape; a candidate (k > 0, v2 or crowded) also within its size
+          const bool ok_w = (cw[m] & (HOTC_ESC | (3u << 29))) == (3u << 29) && (known || k == 0 || dl <= (cw[m] & 0x3FFFFu));
+          rare = rare || !ok_w;
+          ext[m] = (cw[m] >> 18) & 0x7FFu;
+        }
+      }
+      if (__any_sync(0xffffffffu, rare)) {  // the whole group to k_fwd_fix (nothing written here)
+        if (lane == 0) a.wlist[atomicAdd(a.wcount, 1ull)] = cb;
+      } else {
+        ++c_fast;
+        const uint64_t o0 = fc.v0 + (ES ? s_ext[ext[0]] : a.tab.ext_delta[ext[0]]);  // Alg. 1: devptr + (ptr - base)
+        const uint64_t o1 = fc.v1 + (ES ? s_ext[ext[1]] : a.tab.ext_delta[ext[1]]);
+        st_stream2(reinterpret_cast<void *>(a0base + 16ull * c), pol_s, o0, o1);
+        const uint64_t s0 = make_shw(fc.v0, j[0] | SH_DEFER), s1 = make_shw(fc.v1, j[1] | SH_DEFER);
+        if (!sh_odd) {
+          st_stream2(shp + 2ull * c, pol_s, s0, s1);
+        } else {
+          shp[2ull * c] = s0;
+          shp[2ull * c + 1] = s1;
+        }
+        if (lane == 0) a.hitmask[cb >> 4] = 0xFFFFFFFFu;
+        else if (lane == 16 && cb + 16 < nch) a.hitmask[(cb >> 4) + 1] = 0xFFFFFFFFu;
+      }
+  };
   const uint32_t c_first = blockIdx.x * blockDim.x + threadIdx.x;
-  uint64_t cv0 = 0, cv1 = 0, nv0 = 0, nv1 = 0, nnv0 = 0, nnv1 = 0;
-  if (c_first < nch) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c_first), pol_s, cv0, cv1);
-  if (c_first + stride < nch)
-    ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, nv0, nv1);
-  Fr fc, fn;
+  Fr F0, F1;
 #pragma unroll
   for (int m = 0; m < 2; ++m) {
-    fc.ew[m][0] = fc.ew[m][1] = fc.ew[m][2] = fc.ew[m][3] = 0;
-    fn.ew[m][0] = fn.ew[m][1] = fn.ew[m][2] = fn.ew[m][3] = 0;
+    F0.ew[m][0] = F0.ew[m][1] = F0.ew[m][2] = F0.ew[m][3] = 0;
+    F1.ew[m][0] = F1.ew[m][1] = F1.ew[m][2] = F1.ew[m][3] = 0;
   }
-  front(cv0, cv1, fc);
-  for (uint32_t cb = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < nch; cb += stride) {
-    const uint32_t c = cb + lane;
-    if (c + 2 * stride < nch)
-      ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, nnv0, nnv1);
-    front(nv0, nv1, fn);  // the next chunk's entries are in flight while this one finishes
-
-    // decode: j = j0 + #{starts <= p - A}; the candidate's distance dl = p - base (A7: hit iff dl <= size)
-    bool rare = !(fast_ok && c >= f0 && c < f1);
-    uint32_t j[2], cw[2], ext[2];
-#pragma unroll
-    for (int m = 0; m < 2; ++m) {
-      const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
-      const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT, po = fc.poff[m];
-      const uint32_t r = min(po, PD_PAD - 1u);
-      const bool okj0 = j0 != 0xFFFFFFFFu && po < end0;  // j0's end decides (A7)
-      uint32_t k, dl = 0;
-      bool hit = false, known = false;  // known: decided by the entry (v3), with the page state
-      uint32_t ps = 0;
-      if (V3 && cnt <= (uint32_t)PD_K3) {
-        uint32_t word;
-        k = pd_count5(fc.ew[m], r, word);
-        hit = k ? po <= (word >> 16) : okj0;
-        ps = (uint32_t)fc.ew[m][1];
-        known = true;
-      } else {
-        uint32_t off;
-        if (!V3 && cnt <= (uint32_t)PD_K2) {
-          const uint32_t r2 = r | (r << 16);
-          const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
-          k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
-          off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
-        } else if (fc.ok[m]) {  // crowded page: the side array
-          const uint64_t ko = pd_crowded(a.pd.ovf, V3 ? (uint32_t)(fc.ew[m][1] >> 32) : (uint32_t)fc.ew[m][1], cnt, r);
-          k = (uint32_t)ko;
-          off = (uint32_t)(ko >> 32);
-        } else {
-          k = off = 0;
-        }
-        dl = po - off;
-        hit = k ? true : okj0;  // k > 0: decided by the candidate's size (unit word)
-      }
-      j[m] = j0 + k;
-      rare = rare || !fc.ok[m] || !hit;
-      const bool st_valid = V3 && known && (ps & PD_STATE_VALID);
-      cw[m] = 0;
-      if (fc.ok[m] && hit && !st_valid)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
-        asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
-      ext[m] = st_valid ? (ps & (uint32_t)EXT_MASK) : 0xFFFFFFFFu;
-      if (!st_valid) {
-        // ACTIVE with its copy, no escape; a candidate (k > 0, v2 or crowded) also within its size
-        const bool ok_w = (cw[m] & (HOTC_ESC | (3u << 29))) == (3u << 29) && (known || k == 0 || dl <= (cw[m] & 0x3FFFFu));
-        rare = rare || !ok_w;
-        ext[m] = (cw[m] >> 18) & 0x7FFu;
-      }
-    }
-    if (__any_sync(0xffffffffu, rare)) {
-      fwd_chunk_slow<ES, V3, DELTA>(a, s_ext, c, cb, cv0, cv1);
-    } else {
-      ++c_fast;
-      const uint64_t o0 = cv0 + (ES ? s_ext[ext[0]] : a.tab.ext_delta[ext[0]]);  // Alg. 1: devptr + (ptr - base)
-      const uint64_t o1 = cv1 + (ES ? s_ext[ext[1]] : a.tab.ext_delta[ext[1]]);
-      st_stream2(reinterpret_cast<void *>(a0base + 16ull * c), pol_s, o0, o1);
-      const uint64_t s0 = make_shw(cv0, j[0] | SH_DEFER), s1 = make_shw(cv1, j[1] | SH_DEFER);
-      if (!sh_odd) {
-        st_stream2(shp + 2ull * c, pol_s, s0, s1);
-      } else {
-        shp[2ull * c] = s0;
-        shp[2ull * c + 1] = s1;
-      }
-      if (lane == 0) a.hitmask[cb >> 4] = 0xFFFFFFFFu;
-      else if (lane == 16 && cb + 16 < nch) a.hitmask[(cb >> 4) + 1] = 0xFFFFFFFFu;
-    }
-    cv0 = nv0;
-    cv1 = nv1;
-    nv0 = nnv0;
-    nv1 = nnv1;
-    fc = fn;
+  uint64_t va0 = 0, va1 = 0, vb0 = 0, vb1 = 0;
+  F0.v0 = F0.v1 = 0;
+  if (c_first < nch) ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * c_first), pol_s, F0.v0, F0.v1);
+  if (c_first + stride < nch)
+    ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, vb0, vb1);
+  front(F0.v0, F0.v1, F0);
+  for (uint32_t cb = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < nch;) {
+    step(F0, F1, va0, va1, vb0, vb1, cb);
+    cb += stride;
+    if (cb >= nch) break;
+    step(F1, F0, vb0, vb1, va0, va1, cb);
+    cb += stride;
   }
   const unsigned inc = (unsigned)sg.inc;
   flush_count(&a.st->hits, 2ull * c_fast * inc);  // inc = k: k sequential calls
   flush_count(&a.st->translated, 2ull * c_fast);
+}
+
+// the warp groups k_fwd_fast listed: every chunk through fwd_chunk_slow (a NULL, a miss, an activation,
+// a ragged end ... anywhere in the group); usually none
+template <bool ES, bool V3, bool DELTA>
+__global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_fix(const __grid_constant__ SlotArgs a) {
+  const uint32_t n = (uint32_t)*a.wcount;
+  if (n == 0) return;
+  extern __shared__ __align__(16) unsigned char smem[];
+  uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
+  if (ES)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) s_ext[t] = a.tab.ext_delta[t];
+  __syncthreads();
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n;
+  const uint32_t nw = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t i = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n; i += nw) {
+    const uint64_t cb = a.wlist[i], c = cb + (threadIdx.x & 31);
+    uint64_t v0 = 0, v1 = 0;
+    if (c < a.nchunks) {
+      const uint64_t a0 = a0base + 16ull * c;
+      if (a0 >= sg.ptr) v0 = reinterpret_cast<const uint64_t *>(a0)[0];
+      if (a0 + 8 < hi) v1 = reinterpret_cast<const uint64_t *>(a0)[1];
+    }
+    fwd_chunk_slow<ES, V3, DELTA>(a, s_ext, c, cb, v0, v1);
+  }
 }
 
 template <bool ES, bool V3, bool DELTA>
@@ -1796,7 +1834,9 @@ static int launch_fwd_fast1(const SlotArgs &a, int nsm, cudaStream_t s) {
   const uint64_t want = (a.nchunks + T - 1) / T;
   const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
+  if (cudaMemsetAsync(a.wcount, 0, sizeof(unsigned long long), s) != cudaSuccess) return (int)cudaGetLastError();
   k_fwd_fast<ES, V3, DELTA><<<grid, T, smem, s>>>(a);
+  k_fwd_fix<ES, V3, DELTA><<<grid, T, smem, s>>>(a);
   return (int)cudaGetLastError();
 }
 
@@ -1990,8 +2030,8 @@ __global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fast(const __grid_consta
       dfr[m] = defer && (uw & SH_DEFER);
       rare = rare || !ok || (stale[m] && !(fl & UF_READONLY));
     }
-    if (__any_sync(0xffffffffu, rare)) {
-      rev_chunk_slow<DEC, ES>(a, s_dl, s_len, c, cb, cur, cw[0], cw[1]);
+    if (__any_sync(0xffffffffu, rare)) {  // the whole group to k_rev_fix (nothing written here)
+      if (lane == 0) a.wlist[atomicAdd(a.wcount, 1ull)] = cb;
     } else {
       ++c_fast;
 #pragma unroll
@@ -2016,6 +2056,46 @@ __global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fast(const __grid_consta
   flush_count(&a.st->translated, 2ull * c_fast);
 }
 
+// the warp groups k_rev_fast listed: every chunk through rev_chunk_slow; usually none
+template <bool DEC, bool ES>
+__global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fix(const __grid_constant__ SlotArgs a) {
+  const uint32_t n = (uint32_t)*a.wcount;
+  if (n == 0) return;
+  extern __shared__ __align__(16) unsigned char smem[];
+  ulonglong2 *s_dl = reinterpret_cast<ulonglong2 *>(smem);
+  uint32_t *s_len = reinterpret_cast<uint32_t *>(s_dl + (ES ? a.tab.n_ext : 0));
+  if (ES)
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) {
+      s_dl[t] = make_ulonglong2(a.tab.ext_delta[t], a.tab.ext_lo[t]);
+      s_len[t] = a.tab.ext_len[t];
+    }
+  __syncthreads();
+  const Seg sg = a.segs[0];
+  const uint64_t a0base = sg.ptr & ~15ull, hi = sg.ptr + 8ull * sg.n;
+  const uint64_t *shp = reinterpret_cast<const uint64_t *>(sg.shadow);
+  const uint32_t nw = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t i = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n; i += nw) {
+    const uint64_t cb = a.wlist[i], c = cb + (threadIdx.x & 31);
+    RevIn x;
+    x.g[0] = x.g[1] = 0;
+    x.h[0] = x.h[1] = make_shw(0, SH_NONE);
+    x.valid = 0;
+    uint64_t w[2] = {0, 0};
+    if (c < a.nchunks) {
+      const uint64_t a0 = a0base + 16ull * c;
+      x.valid = (a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u);
+      const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
+      for (int m = 0; m < 2; ++m)
+        if ((x.valid >> m) & 1) {
+          x.g[m] = reinterpret_cast<const uint64_t *>(a0)[m];
+          x.h[m] = shp[i0 + m];
+          if (shw_unit(x.h[m]) != SH_NONE && x.g[m] != 0) w[m] = a.tab.st[sh_unit(shw_unit(x.h[m]))];
+        }
+    }
+    rev_chunk_slow<DEC, ES>(a, s_dl, s_len, c, cb, x, w[0], w[1]);
+  }
+}
+
 template <bool DEC, bool ES>
 static int launch_rev_fast1(const SlotArgs &a, int nsm, cudaStream_t s) {
   const size_t smem = (ES ? al16(20 * (size_t)a.tab.n_ext) + 16 : 0) + 64;
@@ -2031,7 +2111,9 @@ static int launch_rev_fast1(const SlotArgs &a, int nsm, cudaStream_t s) {
   const uint64_t want = (a.nchunks + REV_THREADS - 1) / REV_THREADS;
   const int grid = (int)(want < (uint64_t)nsm ? (want ? want : 1) : (uint64_t)nsm);
   (void)cudaGetLastError();
+  if (cudaMemsetAsync(a.wcount, 0, sizeof(unsigned long long), s) != cudaSuccess) return (int)cudaGetLastError();
   k_rev_fast<DEC, ES><<<grid, REV_THREADS, smem, s>>>(a);
+  k_rev_fix<DEC, ES><<<grid, REV_THREADS, smem, s>>>(a);
   return (int)cudaGetLastError();
 }
 
@@ -2188,6 +2270,7 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, i
       const bool es = a.tab.n_ext <= EXT_SMEM, v3 = a.pd.v3 != 0, dl = a.dn > 0;
       static const bool force_big = std::getenv("CGCM_FORCE_BIG") != nullptr;  // tests: the general per-chunk code
       const bool big = a.nchunks >= (1ull << 31) || force_big;
+      *nlaunch = big ? 1 : 2;  // k_fwd_fast + k_fwd_fix
 #define FWD_PASS(E, V, D) \
   if (es == E && v3 == V && dl == D) return big ? launch_fwd_big1<E, V, D>(a, nsm, s) : launch_fwd_fast1<E, V, D>(a, nsm, s);
       FWD_PASS(true, true, false) FWD_PASS(true, false, false) FWD_PASS(false, true, false) FWD_PASS(false, false, false)
@@ -2212,7 +2295,8 @@ int launch_slots(int dir, int ops, const SlotArgs &a, int nsm, cudaStream_t s, i
     if (r != 0) return r;
     SlotArgs b = a;
     b.sel = SEL_SLOW;
-    *nlaunch = 2;
+    static const bool force_big = std::getenv("CGCM_FORCE_BIG") != nullptr;
+    *nlaunch = lean && a.nchunks < (1ull << 31) && !force_big ? 3 : 2;  // (k_rev_fast + k_rev_fix) + k_slots
     return launch_slots(dir, ops, b, nsm, s, &r);
   }
   // the forward index qualifies for the specialised path: one segment, no wide bucket, h <= 3

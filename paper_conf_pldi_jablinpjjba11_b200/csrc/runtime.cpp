@@ -281,7 +281,7 @@ struct Context {
   uint32_t pd_minP = 0, pd_maxP = 0;
 
   // scratch
-  DevBuf slowmask, slowcnt, dump_rc, glue_prog, glue_regs, glue_status;
+  DevBuf slowmask, slowcnt, wlist, dump_rc, glue_prog, glue_regs, glue_status;
   // device-side transfer planning (activation packs, copy-back runs) for lists of >= PLAN_MIN units
   static constexpr size_t PLAN_MIN = 1u << 16;
   DevBuf plan_S, plan_F, plan_G, plan_pid, plan_gscan, plan_tmp, plan_cnt, plan_desc, plan_run;
@@ -900,6 +900,7 @@ struct Context {
     if ((c.ops & OP_HITMASK) || c.sel != SEL_ALL) CKS(dalloc(hitmask, 4 * (size_t)(c.nchunks / 16 + 4)));
     if (c.dir == DIR_REV) CKS(dalloc(slowmask, 4 * (size_t)(c.nchunks / 16 + 4)));
     CKS(dalloc(slowcnt, 64));
+    CKS(dalloc(wlist, 4 * (size_t)(c.nchunks / 32 + 8)));
     CKS(dalloc(segs, sizeof(Seg) * (size_t)k * 8 + 256));
     CKS(dalloc(seg0, 8 * (size_t)(k + 1) * 8 + 256));
     // each launch uses its own eighth of the segment buffers (st_index 0..7, up to 8 launches in flight)
@@ -940,6 +941,8 @@ struct Context {
     a.hitmask = hitmask.as<uint32_t>();
     a.slowmask = slowmask.as<uint32_t>();
     a.slowcount = slowcnt.as<unsigned long long>();
+    a.wlist = wlist.as<uint32_t>();
+    a.wcount = slowcnt.as<unsigned long long>() + 1;
     a.dec_red = c.dec_red ? 1 : 0;
     a.no_journal = c.no_journal ? 1 : 0;
     a.defer = c.defer ? 1 : 0;
