@@ -193,6 +193,7 @@ def run_cgcm(args, rank, world, local_rank):
     clocks = stop_clock_sampler(sampler)
     ms = ev0.elapsed_time(ev1)
     st = ctx.stats()
+    index_format = int(ctx.indexInfo().get("pd_format", 0))
     assert torch.equal(q, q_ref), "round trip changed the pointer arrays"
     if world > 1:
         ms = max_over_ranks(ms, dev)
@@ -223,12 +224,12 @@ def run_cgcm(args, rank, world, local_rank):
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": traffic,
                 # the hot kernels cgcm_mapArrayDevice / cgcm_unmapArrayDevice launch on one segment
-                "kernel": "k_unmap_sh<WRITE|GATE|DEC|HITMASK> (rev)" if dom == "rev" else "k_map_pd<shadow> (fwd)",
+                "kernel": "k_rev_fast<DEC> (rev)" if dom == "rev" else "k_fwd_fast (fwd)",
                 "peak_source": peak_kind,
                 "fwd_ms_per_launch": round(fwd_ms, 4), "rev_ms_per_launch": round(rev_ms, 4),
                 "fwd_gbs": round(BYTES_PER_TRANSLATION * fwd_slots / (fwd_ms / 1e3) / 1e9, 1) if fwd_ms else None,
                 "rev_gbs": round(BYTES_PER_TRANSLATION * rev_slots / (rev_ms / 1e3) / 1e9, 1) if rev_ms else None}
-    roofline["l2_random_ops"] = l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots)
+    roofline["l2_random_ops"] = l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots, index_format)
     gpu_launches = int(st["kernel_launches"])
 
     # the e2e legs run on fresh contexts without CGCM_PROFILE (its per-launch event syncs would serialise
@@ -301,7 +302,8 @@ def declares_between_batches(ctx, step, reps):
         s1 = ctx.stats()
         return {"declares": reps, "ms_per_step_without": round(base_ms / reps, 4),
                 "ms_per_step_with_one_declare": round(with_ms / reps, 4),
-                "us_per_declare_between_batches": round(1e3 * max(0.0, with_wall - base_wall) / reps, 1),
+                "us_per_declare_between_batches": round(1e3 * (with_ms - base_ms) / reps, 1),  # device time
+                "us_per_declare_wall": round(1e6 * (with_wall - base_wall) / reps, 1),
                 "declares_per_s_with_batches": round(reps / max(1e-9, with_wall), 1),
                 "table_merges": s1["table_merges"] - s0["table_merges"],
                 "table_rebuilds": s1["table_rebuilds"] - s0["table_rebuilds"]}
@@ -341,11 +343,12 @@ def full_size_check(ctx, wl, q, q_ref, q_unit, pins_held):
             "how": "every slot vs devptr(u)+(p-base(u)); refcount == 1 + #slots in u; reverse == original"}
 
 
-def l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots):
-    """The roof that binds (DESIGN.md §7.1): each hot kernel's time is bounded below by its random L2
-    operations per slot divided by the measured rates of those primitives on this GPU (random 32-byte
-    gathers and random red.add.s32 into L2-resident arrays, tools/l2_gather.cu, committed log).
-    k_map_pd: page entry + unit word gathers + 1 refcount RED; k_unmap_sh: state word gather + 1 RED."""
+def l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots, pd_format):
+    """The roof that binds (DESIGN.md §7): each hot kernel's time is bounded below by its random L2
+    operations per slot divided by the measured rate of random 32-byte gathers into an L2-resident array on
+    this GPU (tools/l2_gather.cu, committed log).  With deferred references (the timed calls) neither pass
+    issues a refcount reduction: k_fwd_fast gathers the page entry and, with v2 entries (E), the unit's
+    compact word (v3 entries, C: the entry alone); k_rev_fast gathers the unit's state word."""
     g, r = 238.9, 188.4  # G/s, profiles/r01j_l2_gather.log (gather32 at 48 MiB, red_s32)
     try:
         with open(os.path.join(ROOT, "profiles", "r01j_l2_gather.log")) as f:
@@ -357,10 +360,12 @@ def l2_op_roof(fwd_ms, fwd_slots, rev_ms, rev_slots):
                     r = d["G_per_s"]
     except Exception:
         pass
-    fwd_floor = fwd_slots * (2 / g + 1 / r) / 1e6  # ms
-    rev_floor = rev_slots * (1 / g + 1 / r) / 1e6
-    return {"gather_gps": g, "red_gps": r, "source": "profiles/r01j_l2_gather.log",
-            "fwd_ops_per_slot": "2 gathers + 1 RED", "rev_ops_per_slot": "1 gather + 1 RED",
+    fg = 1 if pd_format == 3 else 2
+    fwd_floor = fwd_slots * fg / g / 1e6  # ms
+    rev_floor = rev_slots * 1 / g / 1e6
+    return {"gather_gps": g, "source": "profiles/r01j_l2_gather.log",
+            "fwd_ops_per_slot": "page entry" + (" + unit word" if fg == 2 else "") + f" (v{pd_format} entries)",
+            "rev_ops_per_slot": "state word",
             "fwd_floor_ms": round(fwd_floor, 4), "rev_floor_ms": round(rev_floor, 4),
             "fwd_frac": round(fwd_floor / fwd_ms, 4) if fwd_ms else None,
             "rev_frac": round(rev_floor / rev_ms, 4) if rev_ms else None}

@@ -1840,7 +1840,11 @@ static int launch_fwd_fast1(const SlotArgs &a, int nsm, cudaStream_t s) {
   return (int)cudaGetLastError();
 }
 
-constexpr int REV_THREADS = 768;  // measured: 768 > 640 > 512 (round 2, profiles/r02f_ab.log)
+#ifdef CGCM_REV_THREADS
+constexpr int REV_THREADS = CGCM_REV_THREADS;
+#else
+constexpr int REV_THREADS = 768;
+#endif
 
 // -------------------------------------------------------------------------------------------------
 // k_rev_fast: the reverse pass of cgcm_unmapArrayDevice (a3 + a4 [+ Alg. 3 release]) over ONE in-place
