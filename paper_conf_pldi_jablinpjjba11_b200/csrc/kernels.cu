@@ -1644,6 +1644,11 @@ __device__ __noinline__ void fwd_chunk_slow(const SlotArgs &a, const uint64_t *s
 
 template <bool ES, bool V3, bool DELTA>
 __global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_fast(const __grid_constant__ SlotArgs a) {
+#ifdef CGCM_FWD_S3
+  constexpr bool S3 = true;
+#else
+  constexpr bool S3 = false;
+#endif
   extern __shared__ __align__(16) unsigned char smem[];
   uint64_t *s_ext = reinterpret_cast<uint64_t *>(smem);
   if (ES)
@@ -1689,86 +1694,116 @@ __global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_fast(const __grid_c
                      : "l"(ent + 8 * pg), "l"(pol_t));
     }
   };
-  // one pipeline step for the warp's chunk cb: the values two chunks ahead go to (ld0, ld1), the entries
-  // of the next chunk (values pv0, pv1) to fn, and chunk fc is translated.  The loop runs the step twice
-  // with the roles of the two Fr buffers and the two value buffers swapped (no register copies).
-  auto step = [&](Fr &fc, Fr &fn, uint64_t &ld0, uint64_t &ld1, uint64_t pv0, uint64_t pv1, uint32_t cb) {
-      const uint32_t c = cb + lane;
-      if (c + 2 * stride < nch)
-        ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, ld0, ld1);
-      fn.v0 = pv0;
-      fn.v1 = pv1;
-      front(pv0, pv1, fn);  // the next chunk's entries are in flight while this one finishes
-
-      // decode: j = j0 + #{starts <= p - A}; the candidate's distance dl = p - base (A7: hit iff dl <= size)
-      bool rare = !(fast_ok && c >= f0 && c < f1);
-      uint32_t j[2], cw[2], ext[2];
-  #pragma unroll
-      for (int m = 0; m < 2; ++m) {
-        const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
-        const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT, po = fc.poff[m];
-        const uint32_t r = min(po, PD_PAD - 1u);
-        const bool okj0 = j0 != 0xFFFFFFFFu && po < end0;  // j0's end decides (A7)
-        uint32_t k, dl = 0;
-        bool hit = false, known = false;  // known: decided by the entry (v3), with the page state
-        uint32_t ps = 0;
-        if (V3 && cnt <= (uint32_t)PD_K3) {
-          uint32_t word;
-          k = pd_count5(fc.ew[m], r, word);
-          hit = k ? po <= (word >> 16) : okj0;
-          ps = (uint32_t)fc.ew[m][1];
-          known = true;
-        } else {
-          uint32_t off;
-          if (!V3 && cnt <= (uint32_t)PD_K2) {
-            const uint32_t r2 = r | (r << 16);
-            const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
-            k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
-            off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
-          } else if (fc.ok[m]) {  // crowded page: the side array
-            const uint64_t ko = pd_crowded_i(a.pd.ovf, V3 ? (uint32_t)(fc.ew[m][1] >> 32) : (uint32_t)fc.ew[m][1], cnt, r);
-            k = (uint32_t)ko;
-            off = (uint32_t)(ko >> 32);
-          } else {
-            k = off = 0;
-          }
-          dl = po - off;
-          hit = k ? true : okj0;  // k > 0: decided by the candidate's size (unit word)
-        }
-        j[m] = j0 + k;
-        rare = rare || !fc.ok[m] || !hit;
-        const bool st_valid = V3 && known && (ps & PD_STATE_VALID);
-        cw[m] = 0;
-        if (fc.ok[m] && hit && !st_valid)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
-          asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(cw[m]) : "l"(a.tab.hotc + j[m]), "l"(pol_t));
-        ext[m] = st_valid ? (ps & (uint32_t)EXT_MASK) : 0xFFFFFFFFu;
-        if (!st_valid) {
-          // ACTIVE with its copy, no escape; a candidate (k > 0, v2 or crowded) also within its size
-          const bool ok_w = (cw[m] & (HOTC_ESC | (3u << 29))) == (3u << 29) && (known || k == 0 || dl <= (cw[m] & 0x3FFFFu));
-          rare = rare || !ok_w;
-          ext[m] = (cw[m] >> 18) & 0x7FFu;
-        }
-      }
-      if (__any_sync(0xffffffffu, rare)) {  // the whole group to k_fwd_fix (nothing written here)
-        if (lane == 0) a.wlist[atomicAdd(a.wcount, 1ull)] = cb;
-      } else {
-        ++c_fast;
-        const uint64_t o0 = fc.v0 + (ES ? s_ext[ext[0]] : a.tab.ext_delta[ext[0]]);  // Alg. 1: devptr + (ptr - base)
-        const uint64_t o1 = fc.v1 + (ES ? s_ext[ext[1]] : a.tab.ext_delta[ext[1]]);
-        st_stream2(reinterpret_cast<void *>(a0base + 16ull * c), pol_s, o0, o1);
-        const uint64_t s0 = make_shw(fc.v0, j[0] | SH_DEFER), s1 = make_shw(fc.v1, j[1] | SH_DEFER);
-        if (!sh_odd) {
-          st_stream2(shp + 2ull * c, pol_s, s0, s1);
-        } else {
-          shp[2ull * c] = s0;
-          shp[2ull * c + 1] = s1;
-        }
-        if (lane == 0) a.hitmask[cb >> 4] = 0xFFFFFFFFu;
-        else if (lane == 16 && cb + 16 < nch) a.hitmask[(cb >> 4) + 1] = 0xFFFFFFFFu;
-      }
+  // a decoded chunk: its slot values, units, unit words (in flight), and per slot x = the distance the unit
+  // word's size must cover (A7: p - base <= size; 0 when the entry decided) or, with a valid page state,
+  // the extent | 2^31
+  struct Dc {
+    uint64_t v0, v1;
+    uint32_t j[2], cw[2], x[2];
+    bool rare;
   };
-  const uint32_t c_first = blockIdx.x * blockDim.x + threadIdx.x;
+  // decode chunk c: j = j0 + #{starts <= p - A}; issue the unit words the entry does not decide
+  auto decode = [&](const Fr &fc, uint32_t c, Dc &d) {
+    d.v0 = fc.v0;
+    d.v1 = fc.v1;
+    d.rare = !(fast_ok && c >= f0 && c < f1);
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      const uint32_t j0 = (uint32_t)fc.ew[m][0], w1 = (uint32_t)(fc.ew[m][0] >> 32);
+      const uint32_t cnt = w1 & PD_CNT_MAX, end0 = w1 >> PD_END_SHIFT, po = fc.poff[m];
+      const uint32_t r = min(po, PD_PAD - 1u);
+      const bool okj0 = j0 != 0xFFFFFFFFu && po < end0;  // j0's end decides (A7)
+      uint32_t k, dl = 0;
+      bool hit = false, known = false;  // known: decided by the entry (v3), with the page state
+      uint32_t ps = 0;
+      if (V3 && cnt <= (uint32_t)PD_K3) {
+        uint32_t word;
+        k = pd_count5(fc.ew[m], r, word);
+        hit = k ? po <= (word >> 16) : okj0;
+        ps = (uint32_t)fc.ew[m][1];
+        known = true;
+      } else {
+        uint32_t off;
+        if (!V3 && cnt <= (uint32_t)PD_K2) {
+          const uint32_t r2 = r | (r << 16);
+          const uint64_t r4 = (uint64_t)r2 | ((uint64_t)r2 << 32);
+          k = le4(fc.ew[m][1], r4) + le4(fc.ew[m][2], r4) + le4(fc.ew[m][3], r4);
+          off = k ? off_at(fc.ew[m][1], fc.ew[m][2], fc.ew[m][3], k - 1) : 0u;
+        } else if (fc.ok[m]) {  // crowded page: the side array
+          const uint64_t ko = pd_crowded_i(a.pd.ovf, V3 ? (uint32_t)(fc.ew[m][1] >> 32) : (uint32_t)fc.ew[m][1], cnt, r);
+          k = (uint32_t)ko;
+          off = (uint32_t)(ko >> 32);
+        } else {
+          k = off = 0;
+        }
+        dl = po - off;
+        hit = k ? true : okj0;  // k > 0: decided by the candidate's size (unit word)
+      }
+      d.j[m] = j0 + k;
+      d.rare = d.rare || !fc.ok[m] || !hit;
+      const bool st_valid = V3 && known && (ps & PD_STATE_VALID);
+      d.cw[m] = 0;
+      if (fc.ok[m] && hit && !st_valid)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
+        asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(d.cw[m]) : "l"(a.tab.hotc + d.j[m]), "l"(pol_t));
+      d.x[m] = st_valid ? ((ps & (uint32_t)EXT_MASK) | 0x80000000u) : (known || k == 0 ? 0u : dl);
+    }
+  };
+  // translate decoded chunk cb + lane, or list the warp's group for k_fwd_fix (nothing written here)
+  auto finish = [&](const Dc &d, uint32_t cb) {
+    const uint32_t c = cb + lane;
+    bool rare = d.rare;
+    uint32_t e[2];
+#pragma unroll
+    for (int m = 0; m < 2; ++m) {
+      if (d.x[m] & 0x80000000u) {
+        e[m] = d.x[m] & 0x7FFFFFFFu;
+      } else {  // ACTIVE with its copy, no escape, and within the unit's size
+        const uint32_t w = d.cw[m];
+        rare = rare || (w & (HOTC_ESC | (3u << 29))) != (3u << 29) || d.x[m] > (w & 0x3FFFFu);
+        e[m] = (w >> 18) & 0x7FFu;
+      }
+    }
+    if (__any_sync(0xffffffffu, rare)) {
+      if (lane == 0) a.wlist[atomicAdd(a.wcount, 1ull)] = cb;
+    } else {
+      ++c_fast;
+      const uint64_t o0 = d.v0 + (ES ? s_ext[e[0]] : a.tab.ext_delta[e[0]]);  // Alg. 1: devptr + (ptr - base)
+      const uint64_t o1 = d.v1 + (ES ? s_ext[e[1]] : a.tab.ext_delta[e[1]]);
+      st_stream2(reinterpret_cast<void *>(a0base + 16ull * c), pol_s, o0, o1);
+      const uint64_t s0 = make_shw(d.v0, d.j[0] | SH_DEFER), s1 = make_shw(d.v1, d.j[1] | SH_DEFER);
+      if (!sh_odd) {
+        st_stream2(shp + 2ull * c, pol_s, s0, s1);
+      } else {
+        shp[2ull * c] = s0;
+        shp[2ull * c + 1] = s1;
+      }
+      if (lane == 0) a.hitmask[cb >> 4] = 0xFFFFFFFFu;
+      else if (lane == 16 && cb + 16 < nch) a.hitmask[(cb >> 4) + 1] = 0xFFFFFFFFu;
+    }
+  };
+  // one pipeline step for the warp's chunk cb: the values two chunks ahead go to (ld0, ld1), the entries
+  // of the next chunk (values pv0, pv1) to fn, and chunk fc is decoded into dn; S3 (three stages): the
+  // chunk decoded by the previous step (dp) is translated, so its unit words had a step to arrive;
+  // otherwise chunk fc is translated at once.  The loop runs the step twice with the roles of the
+  // buffers swapped (no register copies).
+  const uint32_t cb0 = blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
+  auto step = [&](Fr &fc, Fr &fn, Dc &dn, Dc &dp, uint64_t &ld0, uint64_t &ld1, uint64_t pv0, uint64_t pv1, uint32_t cb) {
+    const uint32_t c = cb + lane;
+    if (c + 2 * stride < nch)
+      ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c + 2 * stride)), pol_s, ld0, ld1);
+    fn.v0 = pv0;
+    fn.v1 = pv1;
+    front(pv0, pv1, fn);  // the next chunk's entries are in flight while this one finishes
+    decode(fc, c, dn);
+    if (S3) {
+      if (cb != cb0) finish(dp, cb - stride);
+    } else {
+      finish(dn, cb);
+    }
+  };
+  const uint32_t c_first = cb0 + lane;
   Fr F0, F1;
+  Dc D0, D1;
 #pragma unroll
   for (int m = 0; m < 2; ++m) {
     F0.ew[m][0] = F0.ew[m][1] = F0.ew[m][2] = F0.ew[m][3] = 0;
@@ -1780,12 +1815,19 @@ __global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_fast(const __grid_c
   if (c_first + stride < nch)
     ld_stream2(reinterpret_cast<const void *>(a0base + 16ull * (c_first + stride)), pol_s, vb0, vb1);
   front(F0.v0, F0.v1, F0);
-  for (uint32_t cb = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < nch;) {
-    step(F0, F1, va0, va1, vb0, vb1, cb);
+  for (uint32_t cb = cb0; cb < nch;) {
+    step(F0, F1, D0, D1, va0, va1, vb0, vb1, cb);
     cb += stride;
-    if (cb >= nch) break;
-    step(F1, F0, vb0, vb1, va0, va1, cb);
+    if (cb >= nch) {
+      if (S3) finish(D0, cb - stride);
+      break;
+    }
+    step(F1, F0, D1, D0, vb0, vb1, va0, va1, cb);
     cb += stride;
+    if (cb >= nch) {
+      if (S3) finish(D1, cb - stride);
+      break;
+    }
   }
   const unsigned inc = (unsigned)sg.inc;
   flush_count(&a.st->hits, 2ull * c_fast * inc);  // inc = k: k sequential calls
@@ -1974,7 +2016,20 @@ __global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fast(const __grid_consta
   const bool defer = a.defer != 0;
   uint32_t c_fast = 0;
 
-  auto load_in = [&](uint32_t c, RevIn &x) {
+  const uint32_t f0w = sh_odd ? 0xFFFFFFFFu : f0;  // vector loads: whole chunks of a 16-byte-aligned shadow
+  // a chunk in flight: slot values, shadow words, validity, and the units' state words (gathered later)
+  struct Rx {
+    uint64_t g[2], h[2], w[2];
+    uint32_t valid;
+  };
+  auto load_in = [&](uint32_t c, Rx &x) {
+    if (c >= f0w && c < f1) {
+      const uint64_t a0 = a0base + 16ull * c;
+      ld_stream2(reinterpret_cast<const void *>(a0), pol_s, x.g[0], x.g[1]);
+      ld_stream2(shp + 2ull * c, pol_s, x.h[0], x.h[1]);
+      x.valid = 3u;
+      return;
+    }
     x.g[0] = x.g[1] = 0;
     x.h[0] = x.h[1] = make_shw(0, SH_NONE);
     x.valid = 0;
@@ -1982,43 +2037,33 @@ __global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fast(const __grid_consta
     const uint64_t a0 = a0base + 16ull * c;
     x.valid = (a0 >= sg.ptr ? 1u : 0u) | (a0 + 8 < hi ? 2u : 0u);
     const int64_t i0 = ((int64_t)(a0 - sg.ptr)) >> 3;
-    if (x.valid == 3u && !sh_odd) {
-      ld_stream2(reinterpret_cast<const void *>(a0), pol_s, x.g[0], x.g[1]);
-      ld_stream2(shp + i0, pol_s, x.h[0], x.h[1]);
-    } else {
-#pragma unroll
-      for (int m = 0; m < 2; ++m)
-        if ((x.valid >> m) & 1) {
-          x.g[m] = reinterpret_cast<const uint64_t *>(a0)[m];
-          x.h[m] = shp[i0 + m];
-        }
-    }
-  };
-  auto gather = [&](const RevIn &x, uint64_t w[2]) {
 #pragma unroll
     for (int m = 0; m < 2; ++m)
-      w[m] = (shw_unit(x.h[m]) != SH_NONE && x.g[m] != 0) ? ld_u64_hot(a.tab.st + sh_unit(shw_unit(x.h[m])), pol_t) : 0ull;
+      if ((x.valid >> m) & 1) {
+        x.g[m] = reinterpret_cast<const uint64_t *>(a0)[m];
+        x.h[m] = shp[i0 + m];
+      }
   };
-
-  const uint32_t c_first = blockIdx.x * blockDim.x + threadIdx.x;
-  RevIn cur, nxt, nn;
-  uint64_t cw[2], nw[2];
-  load_in(c_first, cur);
-  load_in(c_first + stride, nxt);
-  gather(cur, cw);
-  for (uint32_t cb = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); cb < nch; cb += stride) {
+  auto gather = [&](Rx &x) {
+#pragma unroll
+    for (int m = 0; m < 2; ++m)
+      x.w[m] = (shw_unit(x.h[m]) != SH_NONE && x.g[m] != 0) ? ld_u64_hot(a.tab.st + sh_unit(shw_unit(x.h[m])), pol_t) : 0ull;
+  };
+  // one pipeline step for the warp's chunk cb: values and shadow words two chunks ahead into xl, the next
+  // chunk's state words into xn, chunk xc reversed.  The loop runs it three times with the roles of the
+  // three buffers rotated (no register copies).
+  auto step = [&](Rx &xc, Rx &xn, Rx &xl, uint32_t cb) {
     const uint32_t c = cb + lane;
-    load_in(c + 2 * stride, nn);
-    gather(nxt, nw);
-
+    load_in(c + 2 * stride, xl);
+    gather(xn);
     bool rare = !(c >= f0 && c < f1);
     uint64_t hr[2];
     uint32_t su[2];
     bool stale[2], dfr[2];
 #pragma unroll
     for (int m = 0; m < 2; ++m) {
-      const uint64_t g = cur.g[m], w = cw[m];
-      const uint32_t uw = shw_unit(cur.h[m]), e = hot_ext(w), fl = hot_flags(w);
+      const uint64_t g = xc.g[m], w = xc.w[m];
+      const uint32_t uw = shw_unit(xc.h[m]), e = hot_ext(w), fl = hot_flags(w);
       su[m] = uw & ~SH_DEFER;
       ulonglong2 dl = make_ulonglong2(0, 0);
       uint32_t len = 0;
@@ -2029,7 +2074,7 @@ __global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fast(const __grid_consta
       // unchanged since the forward map (cgcm_dev.h make_shw): the recorded CPU pointer
       hr[m] = g - dl.x;
       const bool ok = g != 0 && uw != SH_NONE && (fl & UF_ACTIVE) && e < n_ext && g - dl.y < (uint64_t)len &&
-                      (uint32_t)hr[m] == (uint32_t)cur.h[m] && hr[m] != 0;
+                      (uint32_t)hr[m] == (uint32_t)xc.h[m] && hr[m] != 0;
       stale[m] = st_epoch(w) != cur_ep;
       dfr[m] = defer && (uw & SH_DEFER);
       rare = rare || !ok || (stale[m] && !(fl & UF_READONLY));
@@ -2051,10 +2096,20 @@ __global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fast(const __grid_consta
         a.slowmask[wi] = 0u;
       }
     }
-    cur = nxt;
-    nxt = nn;
-    cw[0] = nw[0];
-    cw[1] = nw[1];
+  };
+
+  const uint32_t cb0 = blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
+  Rx X0, X1, X2;
+  load_in(cb0 + lane, X0);
+  load_in(cb0 + lane + stride, X1);
+  gather(X0);
+  for (uint32_t cb = cb0; cb < nch;) {
+    step(X0, X1, X2, cb);
+    if ((cb += stride) >= nch) break;
+    step(X1, X2, X0, cb);
+    if ((cb += stride) >= nch) break;
+    step(X2, X0, X1, cb);
+    cb += stride;
   }
   flush_count(&a.st->hits, 2ull * c_fast);
   flush_count(&a.st->translated, 2ull * c_fast);
