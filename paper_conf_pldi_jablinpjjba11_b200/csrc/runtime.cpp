@@ -729,6 +729,7 @@ struct Context {
 
   // merge pending declares/undeclares into the device table (A19: kernels only see a compacted table)
   int ensure_table() {
+    if (table_dirty) leases.clear();  // a rebuild renumbers the units
     Trace trace_("ensure_table");
     if (!table_dirty) return CGCM_OK;
     if (!dirty_del && !pend_over && Umain > 0 && dk.size() + pend.size() <= (size_t)DELTA_MAX &&
@@ -888,6 +889,7 @@ struct Context {
   int launch(SlotCall &c, int st_index, bool reuse_hitmask_layout = false, bool timed_fwd = false,
              bool timed_rev = false) {
     (void)reuse_hitmask_layout;
+    if (c.ops & (OP_DEC | OP_DECPLAIN)) lease_break();
     int k = (int)c.segs.size();
     if (k == 0) return CGCM_OK;
     std::vector<uint64_t> c0(k + 1, 0);
@@ -1107,6 +1109,8 @@ struct Context {
   }
   int unit_ops(const std::vector<UnitOp> &ops) {
     if (ops.empty()) return CGCM_OK;
+    for (auto &o : ops)
+      if ((o.op == UOP_ADD_RC && (int64_t)o.val < 0) || o.op == UOP_SET_RC) lease_break();
     CKS(upload(uops, ops));
     // the compact unit words need rewriting only if an op changes ACTIVE or STORAGE (cgcm_dev.h make_hotc)
     bool hotc = false;
@@ -1329,6 +1333,60 @@ struct Context {
   // references, so the re-map is refcounts only -- +mult per non-null slot through the reverse index
   // and +mult on the outer -- and cannot fail for a legal program (R13-ii: GPU functions do not store
   // pointers).  Both kernels are queued without a host wait.  Returns 1 when another path must run.
+  // Leases: references the asynchronous re-maps above added to an outer and its elements (unit -> (dec_gen,
+  // count)).  While no other call has released a reference since (dec_gen unchanged; a table rebuild clears
+  // them), the units hold those references on top of the array mapping's own, so a releaseArray of the outer
+  // that consumes a lease cannot bring any of them to 0 or below (Alg. 3 frees nothing, no underflow):
+  // release_arrays_async queues its decrements without a host wait.
+  std::unordered_map<uint32_t, std::pair<uint64_t, uint64_t>> leases;
+  uint64_t dec_gen = 1;
+  bool lease_quiet = false;  // set while release_arrays_async issues its own decrements
+  void lease_break() {
+    if (!lease_quiet) ++dec_gen;
+  }
+  int release_arrays_async(const uint64_t *ptrs, size_t k) {
+    if (table_dirty || mirror_stale || k > 64 || (flags & CGCM_LENIENT) || leases.empty()) return 1;
+    std::vector<std::pair<uint32_t, uint64_t>> outs;  // unit, mult
+    for (size_t j = 0; j < k; ++j) {
+      auto it = reg.upper_bound(ptrs[j]);
+      if (it == reg.begin()) return 1;
+      --it;
+      const HostUnit &u = it->second;
+      if (u.idx < 0 || ptrs[j] - it->first > u.size) return 1;
+      const uint32_t x = (uint32_t)u.idx;
+      if (!uarr[x] || !udev[x]) return 1;
+      size_t q = 0;
+      while (q < outs.size() && outs[q].first != x) ++q;
+      if (q == outs.size()) outs.push_back({x, 0});
+      outs[q].second += 1;
+    }
+    for (auto &o : outs) {
+      auto l = leases.find(o.first);
+      if (l == leases.end() || l->second.first != dec_gen || l->second.second < o.second) return 1;
+    }
+    for (auto &o : outs) leases[o.first].second -= o.second;
+    std::vector<UnitOp> ops;
+    std::vector<Seg> rsegs;
+    for (auto &o : outs) {
+      ops.push_back({o.first, UOP_ADD_RC, (uint64_t)(-(int64_t)o.second)});
+      const uint64_t n = usize[o.first] / 8;
+      if (n) rsegs.push_back(Seg{udev[o.first], n, 0, (int32_t)o.second, 0});
+    }
+    lease_quiet = true;
+    int r = ensure_rev();
+    if (r == CGCM_OK) r = unit_ops(ops);
+    if (r == CGCM_OK && !rsegs.empty()) {
+      r = prepare_small(false);
+      SlotCall R;
+      R.dir = DIR_REV;
+      R.ops = OP_DEC;
+      R.segs = rsegs;
+      if (r == CGCM_OK) r = launch(R, 2);
+    }
+    lease_quiet = false;
+    if (r != CGCM_OK) lease_break();
+    return r;
+  }
   int remap_arrays_async(const uint64_t *ptrs, size_t k, void ***gpu_out) {
     // (lenient mode: a stray word in the device slots could fall inside another unit's device copy, A18)
     if (table_dirty || mirror_stale || k > 64 || (flags & CGCM_LENIENT)) return 1;
@@ -1362,7 +1420,7 @@ struct Context {
     if (!rsegs.empty()) {
       CKS(dalloc(lazy_status, sizeof(Status) + 256));
       if (!lazy_pending) CK(cudaMemsetAsync(lazy_status.as<void>(), 0, sizeof(Status), main));
-      CKS(prepare_small());
+      CKS(prepare_small(false));
       SlotCall R;
       R.dir = DIR_REV;
       R.ops = OP_INCPLAIN;
@@ -1374,6 +1432,11 @@ struct Context {
     for (size_t j = 0; j < k; ++j) {
       const uint32_t x = outs[which[j]].first;
       gpu_out[j] = reinterpret_cast<void **>(udev[x] + (ptrs[j] - ubase[x]));
+    }
+    for (auto &o : outs) {
+      auto &l = leases[o.first];
+      if (l.first != dec_gen) l = {dec_gen, 0};
+      l.second += (uint64_t)o.second;
     }
     return CGCM_OK;
   }
@@ -1716,6 +1779,7 @@ struct Context {
 
   // units whose refcount reached 0: free device storage (globals keep theirs), clear flags
   int free_units(const std::vector<uint32_t> &units) {
+    if (!units.empty()) lease_break();
     Trace trace_("free_units");
     CKS(mirror_units(units));
     if (units.empty()) return CGCM_OK;
@@ -1826,10 +1890,12 @@ struct Context {
     CK(cudaStreamSynchronize(copy));
     return CGCM_OK;
   }
-  int prepare_small() {
+  // zero = false: for passes nobody fetches the status of (the queued re-map / release): every call that
+  // reads a status block zeroes it first
+  int prepare_small(bool zero = true) {
     CKS(dalloc(status, sizeof(Status) * 8 + 256));
     CKS(dalloc(lc, 64));
-    CK(cudaMemsetAsync(status.as<void>(), 0, sizeof(Status) * 8, main));
+    if (zero) CK(cudaMemsetAsync(status.as<void>(), 0, sizeof(Status) * 8, main));
     CKS(h_status.ensure(sizeof(Status) * 8 + 64));
     int cap = list_capacity();
     CKS(dalloc(act_list, 4 * (size_t)cap + 64));
@@ -3290,6 +3356,10 @@ int cgcm_releaseArrays(void *const *const *arrays, size_t k) {
   CTXM();
   if (k == 0) return CGCM_OK;
   if (!arrays) return CGCM_E_INVALID;
+  {  // the release that matches a queued re-map (a lease): no host wait at all
+    const int r = C->release_arrays_async(reinterpret_cast<const uint64_t *>(arrays), k);
+    if (r != 1) return r;  // 1: not that case, take the general path
+  }
   std::vector<PointInfo> infos;
   CKS(C->lookup_points(reinterpret_cast<const uint64_t *>(arrays), k, infos));
   std::vector<Outer> outs;
