@@ -123,7 +123,7 @@ struct IndexDev {
 //            with PD_PAD to a whole 32-byte sector); w[2] = 0
 // greatestLTE(p) = j0 + #{starts <= p - A}; p hits unit j0 iff p - A < end0, a candidate iff p - A <= its
 // end -- decided from the entry alone.  With a valid page state the translation needs nothing else: one
-// sector gather per lookup (k_fwd_lean); otherwise the unit word is gathered.
+// sector gather per lookup (k_fwd_fast); otherwise the unit word is gathered.
 // Pages are at most 32 KiB (P <= 15): starts, ends and the padding PD_PAD = 0x7FFF fit 15 bits, so the
 // starts compare against p - A two per 64-bit subtraction with a guard bit per 16-bit lane (pd_count5); no
 // start sits at offset PD_PAD (build_pd takes a smaller page), and lookups clamp p - A to PD_PAD - 1.
