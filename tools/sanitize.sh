@@ -2,12 +2,12 @@
 # compute-sanitizer over reduced GPU parity cases (run on the GPU box through gpurun, from the repo root):
 #   tools/sanitize.sh <round>
 # memcheck (out-of-bounds / misaligned / leaks of device memory), racecheck and synccheck (shared
-# memory hazards, barrier misuse) on the hot kernels (k_fwd_lean, k_rev_lean, k_map_pd, k_unmap_sh,
-# k_slots with and without shadows), the glue interpreter, the peer-copy path and the smoke test.
+# memory hazards, barrier misuse) on the hot kernels (k_fwd_fast / k_fwd_fix, k_rev_fast / k_rev_fix, k_map_pd,
+# k_unmap_sh, k_slots with and without shadows), the queued re-map / release (leases), the glue interpreter, the peer-copy path and the smoke test.
 set -u
 R=${1:-r02}
 mkdir -p gpurun_out/$R
-CASES="tests/test_gpu_parity.py::test_scalar_map_unmap_release tests/test_gpu_parity.py::test_mapArray_roundtrip_permutation tests/test_gpu_parity.py::test_random_device_slices[shadow-8] tests/test_gpu_deferred.py::test_deferred_released_by_matching_unmap[shadow] tests/test_gpu_deferred.py::test_deferred_slots_rewritten_by_gpu[shadow] tests/test_gpu_glue.py tests/test_gpu_group.py::test_handoff_through_a_dirty_peer"
+CASES="tests/test_gpu_parity.py::test_scalar_map_unmap_release tests/test_gpu_parity.py::test_mapArray_roundtrip_permutation tests/test_gpu_parity.py::test_random_device_slices[shadow-8] tests/test_gpu_deferred.py::test_deferred_released_by_matching_unmap[shadow] tests/test_gpu_deferred.py::test_deferred_slots_rewritten_by_gpu[shadow] tests/test_gpu_glue.py tests/test_gpu_group.py::test_handoff_through_a_dirty_peer tests/test_gpu_leases.py::test_leased_releases_match_the_oracle[shadow]"
 for tool in memcheck racecheck synccheck; do
   extra=""
   [ "$tool" = memcheck ] && extra="--leak-check full"
