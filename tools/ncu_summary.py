@@ -61,7 +61,9 @@ def main():
     traffic = {}
     for row in rows:
         name = row[hdr.index("Kernel Name")]
-        kind = "rev" if "<1," in name or "(int)1," in name else "fwd"
+        # the reverse passes: k_rev_* (round 2), k_unmap_sh / k_slots<1, ...> (DIR_REV = 1); else the forward
+        kind = "rev" if ("k_rev" in name or "k_unmap" in name or
+                         ("k_slots" in name and ("<1," in name or "(int)1," in name))) else "fwd"
         lines.append(f"## {name}")
         lines.append("")
         lines.append("| metric | value |")
