@@ -1364,7 +1364,10 @@ struct Context {
       auto l = leases.find(o.first);
       if (l == leases.end() || l->second.first != dec_gen || l->second.second < o.second) return 1;
     }
-    for (auto &o : outs) leases[o.first].second -= o.second;
+    for (auto &o : outs) {
+      auto l = leases.find(o.first);
+      if ((l->second.second -= o.second) == 0) leases.erase(l);
+    }
     std::vector<UnitOp> ops;
     std::vector<Seg> rsegs;
     for (auto &o : outs) {
