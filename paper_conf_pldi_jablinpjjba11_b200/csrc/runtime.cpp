@@ -890,6 +890,7 @@ struct Context {
              bool timed_rev = false) {
     (void)reuse_hitmask_layout;
     if (c.ops & (OP_DEC | OP_DECPLAIN)) lease_break();
+    lists_fresh = false;  // the kernels below may append to the unit lists
     int k = (int)c.segs.size();
     if (k == 0) return CGCM_OK;
     std::vector<uint64_t> c0(k + 1, 0);
@@ -899,6 +900,7 @@ struct Context {
     }
     c.nchunks = c0[k];
     if (c.nchunks == 0) return CGCM_OK;
+    if (c.nchunks > (1u << 15)) launches_small = false;  // no list heads with the next status fetch
     if ((c.ops & OP_HITMASK) || c.sel != SEL_ALL) CKS(dalloc(hitmask, 4 * (size_t)(c.nchunks / 16 + 4)));
     if (c.dir == DIR_REV) CKS(dalloc(slowmask, 4 * (size_t)(c.nchunks / 16 + 4)));
     CKS(dalloc(slowcnt, 64));
@@ -1044,12 +1046,33 @@ struct Context {
     return CGCM_OK;
   }
   // fetch the 8 Status blocks + list counters (synchronizes main)
+  // Small calls: the status fetch also brings back the head of the unit lists (activation, free, copy-back;
+  // LIST_HEAD entries each), so sorting a short list needs neither a device sort nor a second host wait
+  // (sorted_units).  Valid until the next slot launch.
+  static constexpr size_t LIST_HEAD = 512;
+  HostBuf h_lists;
+  bool lists_fresh = false, launches_small = true;
+  uint64_t list_addr[3] = {0, 0, 0};
   int fetch_status(Status out[8], unsigned long long lcs[4]) {
     Trace trace_("fetch_status(sync)");
     // a kernel writes them into mapped pinned memory: no DMA to queue behind other copies (cgcm_dev.h)
     launch_copy_small(h_status.p, status.as<void>(), sizeof(Status) * 8, h_status.as<char>() + sizeof(Status) * 8,
                       lc.as<void>(), 32, main);
     st.kernel_launches += 1;
+    lists_fresh = false;
+    if (launches_small && act_list.addr && free_list.addr && copy_list.addr) {
+      const size_t m = std::min<size_t>(LIST_HEAD, (size_t)list_capacity());
+      CKS(h_lists.ensure(3 * 4 * LIST_HEAD + 64));
+      launch_copy_small(h_lists.p, act_list.as<void>(), 4 * m, h_lists.as<char>() + 4 * LIST_HEAD,
+                        free_list.as<void>(), 4 * m, main);
+      launch_copy_small(h_lists.as<char>() + 8 * LIST_HEAD, copy_list.as<void>(), 4 * m, nullptr, nullptr, 0, main);
+      st.kernel_launches += 2;
+      list_addr[0] = act_list.addr;
+      list_addr[1] = free_list.addr;
+      list_addr[2] = copy_list.addr;
+      lists_fresh = true;
+    }
+    launches_small = true;
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(main));
     std::memcpy(out, h_status.p, sizeof(Status) * 8);
@@ -1129,6 +1152,14 @@ struct Context {
     Trace trace_("sorted_units");
     out.clear();
     if (!n) return CGCM_OK;
+    if (lists_fresh && n <= std::min<size_t>(LIST_HEAD, (size_t)list_capacity()))
+      for (int l = 0; l < 3; ++l)
+        if (src.addr == list_addr[l]) {  // the head fetched with the status (fetch_status)
+          const uint32_t *h = reinterpret_cast<const uint32_t *>(h_lists.as<char>() + 4 * LIST_HEAD * l);
+          out.assign(h, h + n);
+          std::sort(out.begin(), out.end());
+          return CGCM_OK;
+        }
     if (n > 1) {
       size_t tb = sort_keys_temp_bytes((int)n);
       CKS(dalloc(temp, tb + 256 + 4 * n + 64));
@@ -2592,6 +2623,7 @@ int cgcm_finalize(void) {
     if (e) cudaEventDestroy(e);
   if (C->h_status.p) cudaFreeHost(C->h_status.p);
   if (C->h_list.p) cudaFreeHost(C->h_list.p);
+  if (C->h_lists.p) cudaFreeHost(C->h_lists.p);
   cudaEventDestroy(C->ev_copy);
   cudaEventDestroy(C->ev_pack[0]);
   cudaEventDestroy(C->ev_pack[1]);
