@@ -1461,16 +1461,18 @@ __device__ __noinline__ uint64_t pd_crowded(const uint16_t *ovf, uint32_t first,
 // k_fwd_fast: the forward map of cgcm_mapArrayDevice (a1 + a2 of Alg. 1) over ONE in-place segment with
 // a shadow, through a page directory of ONE address segment (the case of every config-C/E-shaped table);
 // same results, counters and lists as k_map_pd<1>.  Software pipeline: slot values two chunks ahead, the
-// page entries (one LDG.256 each) one chunk ahead.  A warp takes the short path for a chunk when all of
-// its 64 slots are ordinary: a whole chunk, a page of this segment, a hit on a unit that is ACTIVE with
-// its copy (its reference deferred into the shadow, a.defer), no escaped unit word.  The short path
-// keeps no per-slot counters (a fast chunk is two hits, two translations), builds no masks (its hit-mask
-// words are all ones) and takes no atomics; crowded pages stay on it (a divergent side-array count).
-// Any other chunk -- a NULL, a miss, an activation, a ragged end, a huge unit, a delta unit -- is redone
-// by fwd_chunk_slow, one warp-uniform call that recomputes the chunk from its two slot values.
-// Round 2 (profiles/r02t_ab.log): the round-1 structure (every slot through the general code, 270
-// thread instructions per slot) took 0.709 ms at C, this one 0.556; at E 3.28 -> 3.22 ms (E is bound by
-// its two random L2 gathers per slot, not by instructions: profiles/r02u_ab_tablesize.log).
+// page entries (one LDG.256 each) one chunk ahead, the unit words of a chunk gathered as soon as its
+// entries are decoded; the loop is unrolled twice with the buffers' roles swapped (no stage copies).  A
+// warp translates a group of 32 chunks on the short path when all of its 64 slots are ordinary: a whole
+// chunk, a page of this segment, a hit on a unit that is ACTIVE with its copy (its reference deferred
+// into the shadow, a.defer), no escaped unit word.  The short path keeps no per-slot counters (a fast
+// chunk is two hits, two translations), builds no masks (its hit-mask words are all ones) and takes no
+// atomics; crowded pages stay on it (a divergent side-array count).  Any other group -- a NULL, a miss,
+// an activation, a ragged end, a huge unit, a delta unit -- is left untouched and listed (a.wlist); the
+// fix-up kernel k_fwd_fix then redoes it with fwd_chunk_slow, which recomputes every case from the two
+// slot values.  Round 2 (profiles/r02t, r02x, r02z): 270 thread instructions per slot -> 148; E 3.28 ->
+// 2.75 ms, C 0.709 -> 0.478 ms per launch; E is bound by its two dependent random L2 gathers per slot
+// (DESIGN.md §7, §7.1).
 // -------------------------------------------------------------------------------------------------
 #ifdef CGCM_FWD_FAST_THREADS
 constexpr int FWD_FAST_THREADS = CGCM_FWD_FAST_THREADS;
