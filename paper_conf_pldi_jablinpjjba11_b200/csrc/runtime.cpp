@@ -1442,6 +1442,7 @@ struct Context {
       outs[q].second += 1;
       which[j] = (uint32_t)q;
     }
+    Trace trace_q("remap_async:queue");
     std::vector<UnitOp> ops;
     std::vector<Seg> rsegs;
     for (auto &o : outs) {
@@ -1449,9 +1450,13 @@ struct Context {
       const uint64_t n = usize[o.first] / 8;
       if (n) rsegs.push_back(Seg{udev[o.first], n, 0, o.second, 0});
     }
-    CKS(ensure_rev());
-    CKS(unit_ops(ops));
+    {
+      Trace t1("remap_async:unit_ops");
+      CKS(ensure_rev());
+      CKS(unit_ops(ops));
+    }
     if (!rsegs.empty()) {
+      Trace t2("remap_async:launch");
       CKS(dalloc(lazy_status, sizeof(Status) + 256));
       if (!lazy_pending) CK(cudaMemsetAsync(lazy_status.as<void>(), 0, sizeof(Status), main));
       CKS(prepare_small(false));
@@ -3099,6 +3104,7 @@ int distinct_outers(const std::vector<PointInfo> &infos, std::vector<Outer> &out
 }  // namespace
 
 int cgcm_mapArrays(void *const *const *arrays, size_t k, void ***gpu_out) {
+  Trace tt_("cgcm_mapArrays");
   CTXM();
 
   if (k == 0) return CGCM_OK;
