@@ -317,9 +317,28 @@ struct Context {
 
   cgcm_stats_t st{};
 
+  // Small inputs that repeat call after call (a promoted loop's segment table and unit ops) are uploaded
+  // only when the device bytes differ from the last upload to that range (put_memo: device address ->
+  // bytes).  Every write to those buffers goes through ring_put_memo or forgets the range (memo_forget),
+  // and so does every release or reallocation of a buffer.
+  std::map<uint64_t, std::string> put_memo;
+  void memo_forget(uint64_t lo, uint64_t n) {
+    for (auto it = put_memo.begin(); it != put_memo.end();)
+      it = (it->first < lo + n && lo < it->first + it->second.size()) ? put_memo.erase(it) : std::next(it);
+  }
+  int ring_put_memo(void *dst, const void *src, size_t n) {
+    const uint64_t key = reinterpret_cast<uint64_t>(dst);
+    auto it = put_memo.find(key);
+    if (it != put_memo.end() && it->second.size() == n && std::memcmp(it->second.data(), src, n) == 0) return CGCM_OK;
+    memo_forget(key, n);
+    CKS(ring_put(dst, src, n));
+    put_memo[key].assign(static_cast<const char *>(src), n);
+    return CGCM_OK;
+  }
   // ------------------------------------------------------------------------------------------
   int dalloc(DevBuf &b, size_t need) {  // ensure capacity (contents not preserved)
     if (need <= b.bytes && b.addr) return CGCM_OK;
+    if (b.addr) memo_forget(b.addr, b.bytes);
     if (b.addr) arena.free(b.addr, b.bytes);
     size_t nb = std::max<size_t>(need, 256);
     nb = std::max(nb, b.bytes * 3 / 2);
@@ -332,6 +351,7 @@ struct Context {
     return CGCM_OK;
   }
   void dfree(DevBuf &b) {
+    if (b.addr) memo_forget(b.addr, b.bytes);
     if (b.addr) arena.free(b.addr, b.bytes);
     b.addr = 0;
     b.bytes = 0;
@@ -913,9 +933,11 @@ struct Context {
     // pinned ring: no host wait, and no DMA (read by a kernel) -- also while the outers' H2D copies
     // are in flight on the copy stream
     if (sizeof(Seg) * k + 8 * (size_t)(k + 1) <= RING_HALF / 2) {
-      CKS(ring_put(dsegs, c.segs.data(), sizeof(Seg) * k));
-      CKS(ring_put(dc0, c0.data(), 8 * (size_t)(k + 1)));
+      CKS(ring_put_memo(dsegs, c.segs.data(), sizeof(Seg) * k));
+      CKS(ring_put_memo(dc0, c0.data(), 8 * (size_t)(k + 1)));
     } else {
+      memo_forget(reinterpret_cast<uint64_t>(dsegs), sizeof(Seg) * k);
+      memo_forget(reinterpret_cast<uint64_t>(dc0), 8 * (size_t)(k + 1));
       CK(cudaMemcpyAsync(dsegs, c.segs.data(), sizeof(Seg) * k, cudaMemcpyHostToDevice, main));
       CK(cudaMemcpyAsync(dc0, c0.data(), 8 * (size_t)(k + 1), cudaMemcpyHostToDevice, main));
       CK(cudaStreamSynchronize(main));  // the host vectors above are pageable and go out of scope
@@ -1134,7 +1156,13 @@ struct Context {
     if (ops.empty()) return CGCM_OK;
     for (auto &o : ops)
       if ((o.op == UOP_ADD_RC && (int64_t)o.val < 0) || o.op == UOP_SET_RC) lease_break();
-    CKS(upload(uops, ops));
+    CKS(dalloc(uops, sizeof(UnitOp) * ops.size() + 64));
+    if (sizeof(UnitOp) * ops.size() <= RING_HALF) {
+      CKS(ring_put_memo(uops.as<void>(), ops.data(), sizeof(UnitOp) * ops.size()));
+    } else {
+      memo_forget(uops.addr, uops.bytes);
+      CKS(upload(uops, ops));
+    }
     // the compact unit words need rewriting only if an op changes ACTIVE or STORAGE (cgcm_dev.h make_hotc)
     bool hotc = false;
     for (auto &o : ops)
