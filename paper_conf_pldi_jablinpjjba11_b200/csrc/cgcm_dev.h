@@ -256,6 +256,10 @@ struct SlotArgs {
   // group they leave to the general per-chunk code (k_fwd_fix, k_rev_fix); wcount is zeroed per launch
   uint32_t *wlist;
   unsigned long long *wcount;
+  // k_slots only: rc[rc_unit] += rc_delta once (block 0) -- the outer's reference of a queued re-map /
+  // release applied by the pass over its slots instead of a separate unit-op launch
+  uint32_t rc_unit;
+  int32_t rc_delta;
 };
 // Forward-map shadow (8 B per slot): the low 32 bits of the slot's CPU pointer | the unit word << 32.  The
 // unit word is unit index | SH_DEFER (the slot's reference is not in rc yet); SH_NONE: no unit.  A reverse

@@ -588,6 +588,8 @@ constexpr int FH_PD = -2;  // forward lookups through the page directory
 
 template <int DIR, int OPS, int FH, int SH>
 __global__ void __launch_bounds__(SlotCfg<DIR, SH>::threads, 1) k_slots(SlotArgs a) {
+  // the outer AU's own refcount change of a queued re-map / release, folded into its slot pass
+  if (a.rc_delta && a.cbeg == 0 && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(a.tab.rc + a.rc_unit, a.rc_delta);
   if (a.sel == SEL_SLOW && *a.slowcount == 0) return;  // the pipelined pass decided every slot
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ uint64_t s_seg0[SEG_SMEM + 1];

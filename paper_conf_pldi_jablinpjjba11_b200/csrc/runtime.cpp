@@ -890,6 +890,8 @@ struct Context {
     bool no_journal = false;  // large gate passes snapshot the rc/epoch columns instead
     bool defer = false;       // deferred references (cgcm_dev.h SlotArgs::defer)
     bool lazy = false;        // counters into lazy_status (folded when read), not the call's Status block
+    uint32_t rc_unit = 0;     // k_slots applies rc[rc_unit] += rc_delta once (the queued re-map / release)
+    int32_t rc_delta = 0;
     std::vector<Seg> segs;
     uint64_t nchunks = 0;
     Status res{};
@@ -969,6 +971,8 @@ struct Context {
     a.slowcount = slowcnt.as<unsigned long long>();
     a.wlist = wlist.as<uint32_t>();
     a.wcount = slowcnt.as<unsigned long long>() + 1;
+    a.rc_unit = c.rc_unit;
+    a.rc_delta = c.rc_delta;
     a.dec_red = c.dec_red ? 1 : 0;
     a.no_journal = c.no_journal ? 1 : 0;
     a.defer = c.defer ? 1 : 0;
@@ -1434,15 +1438,21 @@ struct Context {
       const uint64_t n = usize[o.first] / 8;
       if (n) rsegs.push_back(Seg{udev[o.first], n, 0, (int32_t)o.second, 0});
     }
+    // one outer with slots: its own decrement rides with the slot pass (SlotArgs::rc_delta)
+    const bool fold = outs.size() == 1 && rsegs.size() == 1;
     lease_quiet = true;
     int r = ensure_rev();
-    if (r == CGCM_OK) r = unit_ops(ops);
+    if (r == CGCM_OK && !fold) r = unit_ops(ops);
     if (r == CGCM_OK && !rsegs.empty()) {
       r = prepare_small(false);
       SlotCall R;
       R.dir = DIR_REV;
       R.ops = OP_DEC;
       R.segs = rsegs;
+      if (fold) {
+        R.rc_unit = outs[0].first;
+        R.rc_delta = -(int32_t)outs[0].second;
+      }
       if (r == CGCM_OK) r = launch(R, 2);
     }
     lease_quiet = false;
@@ -1478,10 +1488,12 @@ struct Context {
       const uint64_t n = usize[o.first] / 8;
       if (n) rsegs.push_back(Seg{udev[o.first], n, 0, o.second, 0});
     }
+    // one outer with slots: its own increment rides with the slot pass (SlotArgs::rc_delta)
+    const bool fold = outs.size() == 1 && rsegs.size() == 1;
     {
       Trace t1("remap_async:unit_ops");
       CKS(ensure_rev());
-      CKS(unit_ops(ops));
+      if (!fold) CKS(unit_ops(ops));
     }
     if (!rsegs.empty()) {
       Trace t2("remap_async:launch");
@@ -1493,6 +1505,10 @@ struct Context {
       R.ops = OP_INCPLAIN;
       R.segs = rsegs;
       R.lazy = true;
+      if (fold) {
+        R.rc_unit = outs[0].first;
+        R.rc_delta = (int32_t)outs[0].second;
+      }
       CKS(launch(R, 0));
       lazy_pending = true;
     }
