@@ -748,6 +748,12 @@ struct Context {
   }
 
   // merge pending declares/undeclares into the device table (A19: kernels only see a compacted table)
+  struct Stage {
+    std::vector<uint64_t> w;
+    size_t size() const { return 8 * w.size(); }
+    void resize(size_t bytes) { w.resize((bytes + 7) / 8); }
+    uint64_t *data() { return w.data(); }
+  } table_stage;
   int ensure_table() {
     if (table_dirty) leases.clear();  // a rebuild renumbers the units
     Trace trace_("ensure_table");
@@ -760,10 +766,15 @@ struct Context {
     int n = (int)reg.size();
     // host staging: base[n], size[n], epoch0[n] (u32, relative), old_idx[n], flags[n]
     size_t need = (size_t)n * (8 + 8 + 4 + 4 + 4) + 256;
-    CKS(h_list.ensure(need));
-    CK(cudaStreamSynchronize(main));
-    CK(cudaStreamSynchronize(copy));
-    uint64_t *hb = h_list.as<uint64_t>();
+    // pageable staging (the uploads below are followed by a host wait anyway): a pinned buffer sized to the
+    // table would cost a cudaHostAlloc here, 8-600 ms on this pool (profiles/r02bw_trace.log)
+    if (table_stage.size() < need) table_stage.resize(need);
+    {
+      Trace t1("ensure_table:wait");
+      CK(cudaStreamSynchronize(main));
+      CK(cudaStreamSynchronize(copy));
+    }
+    uint64_t *hb = reinterpret_cast<uint64_t *>(table_stage.data());
     uint64_t *hs = hb + n;
     uint32_t *he = reinterpret_cast<uint32_t *>(hs + n);
     int32_t *ho = reinterpret_cast<int32_t *>(he + n);
@@ -842,8 +853,14 @@ struct Context {
     dirty_del = false;
     dk.clear();
     di.clear();
-    CKS(build_index(fwd, hb, n, dbase.as<uint64_t>(), TOPMAX, DIRMAX));
-    CKS(build_pd(hb, hs, n));
+    {
+      Trace t2("ensure_table:index");
+      CKS(build_index(fwd, hb, n, dbase.as<uint64_t>(), TOPMAX, DIRMAX));
+    }
+    {
+      Trace t3("ensure_table:pagedir");
+      CKS(build_pd(hb, hs, n));
+    }
     pd_state_dirty = true;
     CK(cudaStreamSynchronize(main));
     table_dirty = false;
@@ -1123,11 +1140,14 @@ struct Context {
     return CGCM_OK;
   }
   // n <= RING_HALF bytes from pageable host memory to dst, stream-ordered on main, no host wait
+  int ring_init() {
+    if (h_ring.p) return CGCM_OK;
+    CKS(h_ring.ensure(2 * RING_HALF));
+    for (auto &e : ev_ring) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    return CGCM_OK;
+  }
   int ring_put(void *dst, const void *src, size_t n) {
-    if (!h_ring.p) {
-      CKS(h_ring.ensure(2 * RING_HALF));
-      for (auto &e : ev_ring) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-    }
+    CKS(ring_init());
     if (ring_head + n > RING_HALF) {
       CK(cudaEventRecord(ev_ring[ring_cur], main));
       ring_used[ring_cur] = true;
@@ -2607,6 +2627,14 @@ int cgcm_init(int device, void *dev_arena, size_t arena_bytes, void *main_stream
   cudaEventCreateWithFlags(&C->ev_pack[1], cudaEventDisableTiming);
   cudaEventCreate(&C->ev_t0);
   cudaEventCreate(&C->ev_t1);
+  // the small pinned, mapped host buffers every call path uses, allocated now: a cudaHostAlloc inside a
+  // call costs 8-600 ms on this pool (profiles/r02bw_trace.log)
+  // (best effort: a failure here only leaves the allocation to the first call that needs the buffer)
+  (void)C->h_list.ensure(1 << 20);
+  (void)C->h_status.ensure(sizeof(Status) * 8 + 64);
+  (void)C->h_small.ensure(1 << 16);
+  (void)C->h_lists.ensure(3 * 4 * Context::LIST_HEAD + 64);
+  (void)C->ring_init();
   {
     std::lock_guard<std::mutex> g(g_ctx_mu);
     g_contexts.insert(C);
