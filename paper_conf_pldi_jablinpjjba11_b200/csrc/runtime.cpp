@@ -379,9 +379,9 @@ struct Context {
       lo[r] = runs[r].addr;
       len[r] = runs[r].bytes < (1ull << 32) ? (uint32_t)runs[r].bytes : 0u;  // >= 4 GiB: shadows not used
     }
-    CKS(upload(extd, d));
-    CKS(upload(extlo, lo));
-    CKS(upload(extlen, len));
+    CKS(upload(extd, d, true));  // input-only buffers: repeated contents are not re-sent
+    CKS(upload(extlo, lo, true));
+    CKS(upload(extlen, len, true));
     extd_n = runs.size();
     return CGCM_OK;
   }
@@ -1164,11 +1164,16 @@ struct Context {
     CK(cudaGetLastError());
     return CGCM_OK;
   }
+  // memo: dst is an input-only buffer (no kernel writes it), so an upload of the bytes it already holds
+  // can be skipped (ring_put_memo)
   template <class T>
-  int upload(DevBuf &dst, const std::vector<T> &v) {
+  int upload(DevBuf &dst, const std::vector<T> &v, bool memo = false) {
     CKS(dalloc(dst, sizeof(T) * v.size() + 64));
     if (v.empty()) return CGCM_OK;
-    if (sizeof(T) * v.size() <= RING_HALF) return ring_put(dst.as<void>(), v.data(), sizeof(T) * v.size());
+    if (sizeof(T) * v.size() <= RING_HALF)
+      return memo ? ring_put_memo(dst.as<void>(), v.data(), sizeof(T) * v.size())
+                  : ring_put(dst.as<void>(), v.data(), sizeof(T) * v.size());
+    memo_forget(dst.addr, dst.bytes);
     CKS(h_small.ensure(sizeof(T) * v.size()));
     CK(cudaStreamSynchronize(main));
     std::memcpy(h_small.p, v.data(), sizeof(T) * v.size());
@@ -1344,8 +1349,8 @@ struct Context {
     for (size_t q = 0; q < units.size(); ++q) exts[q] = (uint32_t)urun[units[q]];
     if (runs.size() > EXT_MASK) return CGCM_E_NOMEM;  // 2^24 live extents
     CKS(sync_ext());
-    CKS(upload(up_units, units));
-    CKS(upload(up_exts, exts));
+    CKS(upload(up_units, units, true));
+    CKS(upload(up_exts, exts, true));
     launch_set_ext(up_units.as<uint32_t>(), up_exts.as<uint32_t>(), (int)units.size(), tab(), rel_epoch(epoch),
                    (flags & CGCM_LITERAL_EPOCH) ? 0 : 1, main);
     st.kernel_launches += 1;
@@ -1886,7 +1891,7 @@ struct Context {
     Trace trace_("free_units");
     CKS(mirror_units(units));
     if (units.empty()) return CGCM_OK;
-    CKS(upload(up_units, units));
+    CKS(upload(up_units, units, true));
     launch_deactivate(up_units.as<uint32_t>(), (int)units.size(), tab(), main);
     st.kernel_launches += 1;
     pd_state_dirty = true;
@@ -2352,7 +2357,7 @@ struct Context {
   int lookup_points(const uint64_t *ptrs, size_t k, std::vector<PointInfo> &out) {
     CKS(ensure_table());
     std::vector<uint64_t> v(ptrs, ptrs + k);
-    CKS(upload(this->ptrs, v));
+    CKS(upload(this->ptrs, v, true));
     CKS(dalloc(points, sizeof(PointInfo) * k + 64));
     launch_lookup_points(fwd.view(dbase.as<uint64_t>()), tab(), this->ptrs.as<uint64_t>(), (int)k,
                          points.as<PointInfo>(), dkeys.as<uint64_t>(), dids.as<uint32_t>(), (int)dk.size(), main);
