@@ -486,24 +486,25 @@ def table_context(wl, dev, local_rank, nslots):
 
 def run_e2e_duplex(args, ctx, wl, q_ref, dev, world, rank, link, local_rank):
     """The e2e step with both directions of the (full-duplex) host link busy: the rank's arrays are
-    split into two halves, each driven through its own context (its own replica of the table, arena
-    and streams) by its own host thread, the second half one phase behind the first -- while one half
-    copies its translated arrays back (unmapArrays), the other uploads its raw arrays (mapArrays).
-    Same public calls, same bytes every step; CUDA events on the first context's main stream span
-    both threads."""
+    split into k parts (--e2e-parts, default 2; 3 measured slower), each driven through its own context (its own replica of
+    the table, arena and streams) by its own host thread, part i starting once part i-1's first upload is
+    done -- while one part copies its translated arrays back (unmapArrays), another uploads its raw arrays
+    (mapArrays), and the per-call overheads of one part hide behind the others' copies.  Same public calls,
+    same bytes every step; CUDA events on the first context's main stream span all threads."""
     import ctypes
     import threading
     import torch
-    import paper_conf_pldi_jablinpjjba11_b200 as cg
     A, S = wl.arrays_per_rank, wl.slots
+    K = max(2, min(args.e2e_parts, A))
     if A < 2:
         return None
     host = np.ascontiguousarray(q_ref.cpu().numpy().view(np.uint64))
-    ctx2 = table_context(wl, dev, local_rank, (A // 2) * S)
+    bounds = [A * k // K for k in range(K + 1)]
+    ctxs = [ctx] + [table_context(wl, dev, local_rank, (bounds[k + 1] - bounds[k]) * S) for k in range(1, K)]
     try:
-        halves = [(ctx, list(range(0, A // 2))), (ctx2, list(range(A // 2, A)))]
-        outers = [[], []]
-        for k, (c, rng) in enumerate(halves):
+        parts = [(ctxs[k], list(range(bounds[k], bounds[k + 1]))) for k in range(K)]
+        outers = [[] for _ in range(K)]
+        for k, (c, rng) in enumerate(parts):
             c.make_current()
             for a in rng:
                 p = c.malloc(8 * S)
@@ -513,13 +514,14 @@ def run_e2e_duplex(args, ctx, wl, q_ref, dev, world, rank, link, local_rank):
         errs = []
 
         trace = [] if os.environ.get("CGCM_BENCH_TRACE") else None
+        started = [threading.Event() for _ in range(K)]
 
         def step(k):
-            c, o = halves[k][0], outers[k]
+            c, o = parts[k][0], outers[k]
             t0 = time.perf_counter()
             s1, _ = c.mapArrays(o)
-            if k == 0 and not lag.is_set():
-                lag.set()  # the second half starts once the first half's upload is done
+            if k + 1 < K and not started[k + 1].is_set():
+                started[k + 1].set()  # the next part starts once this part's first upload is done
             c.advanceEpoch()
             t1 = time.perf_counter()
             s2 = c.unmapArrays(o)
@@ -531,31 +533,32 @@ def run_e2e_duplex(args, ctx, wl, q_ref, dev, world, rank, link, local_rank):
                 errs.append((k, s1, s2, s3, c.L.cgcm_lastCudaError().decode()))
 
         def worker(k, steps):
-            halves[k][0].make_current()
-            if k == 1:
-                lag.wait()
+            parts[k][0].make_current()
+            started[k].wait()
             for _ in range(steps):
                 step(k)
 
-        lag = threading.Event()
-        lag.set()
-        for k in (0, 1):  # warm-up, one half at a time
-            halves[k][0].make_current()
+        for e in started:
+            e.set()
+        for k in range(K):  # warm-up, one part at a time
+            parts[k][0].make_current()
             step(k)
         torch.cuda.synchronize()
         steps = max(1, min(args.steps, args.e2e_steps))
-        st0 = [c.stats() for c, _ in halves]
-        lag.clear()
+        st0 = [c.stats() for c, _ in parts]
+        for e in started[1:]:
+            e.clear()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        ev2 = torch.cuda.Event()
         ev0.record(ctx.main)
-        ts = [threading.Thread(target=worker, args=(k, steps)) for k in (0, 1)]
+        ts = [threading.Thread(target=worker, args=(k, steps)) for k in range(K)]
         for t in ts:
             t.start()
         for t in ts:
             t.join()
-        ev2.record(ctx2.main)
-        ctx.main.wait_event(ev2)
+        for c in ctxs[1:]:
+            e = torch.cuda.Event()
+            e.record(c.main)
+            ctx.main.wait_event(e)
         ev1.record(ctx.main)
         torch.cuda.synchronize()
         if errs:
@@ -565,15 +568,16 @@ def run_e2e_duplex(args, ctx, wl, q_ref, dev, world, rank, link, local_rank):
             for x in sorted(trace, key=lambda r: r[1]):
                 print("duplex", x[0], [round(v - z, 1) for v in x[1:]], file=sys.stderr)
         ms = ev0.elapsed_time(ev1)
-        st1 = [c.stats() for c, _ in halves]
+        st1 = [c.stats() for c, _ in parts]
         ok = all(np.array_equal(np.ctypeslib.as_array((ctypes.c_uint64 * S).from_address(p)), host[a * S:(a + 1) * S])
-                 for k in (0, 1) for a, p in zip(halves[k][1], outers[k]))
-        for k in (0, 1):
-            halves[k][0].make_current()
+                 for k in range(K) for a, p in zip(parts[k][1], outers[k]))
+        for k in range(K):
+            parts[k][0].make_current()
             for p in outers[k]:
-                halves[k][0].free(p)
+                parts[k][0].free(p)
     finally:
-        ctx2.close()
+        for c in ctxs[1:]:
+            c.close()
         ctx.make_current()
     if world > 1:
         import torch.distributed as dist
@@ -587,7 +591,7 @@ def run_e2e_duplex(args, ctx, wl, q_ref, dev, world, rank, link, local_rank):
             "frac_of_host_link": round(floor_ms / (ms / steps), 4),
             "ms_per_step": round(ms / steps, 3), "steps": steps,
             "api": "cgcm_mapArrays+advanceEpoch+cgcm_unmapArrays+cgcm_releaseArrays (pinned host arrays), "
-                   "two halves through two contexts, one phase apart (full-duplex link)",
+                   f"{K} parts through {K} contexts, each one upload phase behind the previous (full-duplex link)",
             "host_arrays_roundtrip_ok": bool(ok)}
 
 
@@ -839,6 +843,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-duplex", action="store_true", help="e2e through one context only")
     ap.add_argument("--e2e-steps", type=int, default=6)
+    ap.add_argument("--e2e-parts", type=int, default=2, help="contexts (threads) of the duplex e2e leg (3: slower, profiles/r02e3_*)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=1 << 21)
     ap.add_argument("--ref-sample", type=int, default=1 << 19)
