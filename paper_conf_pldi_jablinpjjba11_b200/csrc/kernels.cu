@@ -1997,13 +1997,15 @@ __device__ __noinline__ void rev_chunk_slow(const SlotArgs &a, const ulonglong2 
 template <bool DEC, bool ES>
 __global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fast(const __grid_constant__ SlotArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
+  // per extent {delta, device start | 2^63 if the extent spans 4 GiB or more}: one LDS.128 per slot.  The
+  // shadow check needs no length: a slot g with 0 <= g - lo < 2^32 whose g - delta has the recorded low 32
+  // bits IS the recorded pointer p + delta (g - delta and p lie in one window of width 2^32 starting at the
+  // extent's host start, since the extent is shorter than 2^32), so it lies in the extent; a big extent's
+  // flag bit fails the check (its slots take k_rev_fix, as with the length check of sh_reverse)
   ulonglong2 *s_dl = reinterpret_cast<ulonglong2 *>(smem);
-  uint32_t *s_len = reinterpret_cast<uint32_t *>(s_dl + (ES ? a.tab.n_ext : 0));
   if (ES)
-    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x) {
-      s_dl[t] = make_ulonglong2(a.tab.ext_delta[t], a.tab.ext_lo[t]);
-      s_len[t] = a.tab.ext_len[t];
-    }
+    for (int t = threadIdx.x; t < a.tab.n_ext; t += blockDim.x)
+      s_dl[t] = make_ulonglong2(a.tab.ext_delta[t], a.tab.ext_lo[t] | (a.tab.ext_len[t] == 0 ? 1ull << 63 : 0ull));
   __syncthreads();
   const uint64_t pol_s = policy_evict_first();
   const uint64_t pol_t = policy_evict_last();
@@ -2069,15 +2071,13 @@ __global__ void __launch_bounds__(REV_THREADS, 1) k_rev_fast(const __grid_consta
       const uint64_t g = xc.g[m], w = xc.w[m];
       const uint32_t uw = shw_unit(xc.h[m]), e = hot_ext(w), fl = hot_flags(w);
       su[m] = uw & ~SH_DEFER;
-      ulonglong2 dl = make_ulonglong2(0, 0);
-      uint32_t len = 0;
-      if (e < n_ext) {
-        dl = ES ? s_dl[e] : make_ulonglong2(a.tab.ext_delta[e], a.tab.ext_lo[e]);
-        len = ES ? s_len[e] : a.tab.ext_len[e];
-      }
+      ulonglong2 dl = make_ulonglong2(0, ~0ull);
+      if (e < n_ext)
+        dl = ES ? s_dl[e]
+                : make_ulonglong2(a.tab.ext_delta[e], a.tab.ext_lo[e] | (a.tab.ext_len[e] == 0 ? 1ull << 63 : 0ull));
       // unchanged since the forward map (cgcm_dev.h make_shw): the recorded CPU pointer
       hr[m] = g - dl.x;
-      const bool ok = g != 0 && uw != SH_NONE && (fl & UF_ACTIVE) && e < n_ext && g - dl.y < (uint64_t)len &&
+      const bool ok = g != 0 && uw != SH_NONE && (fl & UF_ACTIVE) && e < n_ext && ((g - dl.y) >> 32) == 0 &&
                       (uint32_t)hr[m] == (uint32_t)xc.h[m] && hr[m] != 0;
       stale[m] = st_epoch(w) != cur_ep;
       dfr[m] = defer && (uw & SH_DEFER);
