@@ -1748,7 +1748,8 @@ __global__ void __launch_bounds__(FWD_FAST_THREADS, 1) k_fwd_fast(const __grid_c
       const bool st_valid = V3 && known && (ps & PD_STATE_VALID);
       d.cw[m] = 0;
       if (fc.ok[m] && hit && !st_valid)  // the 4-byte compact unit word (cgcm_dev.h make_hotc)
-        asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(d.cw[m]) : "l"(a.tab.hotc + d.j[m]), "l"(pol_t));
+        asm volatile("ld.global.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;"  // random: no L1 reuse (r02h1)
+                     : "=r"(d.cw[m]) : "l"(a.tab.hotc + d.j[m]), "l"(pol_t));
       d.x[m] = st_valid ? ((ps & (uint32_t)EXT_MASK) | 0x80000000u) : (known || k == 0 ? 0u : dl);
     }
   };
