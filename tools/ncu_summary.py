@@ -36,6 +36,12 @@ METRICS = [
 ]
 
 
+def kind_of(name):
+    """'rev' for the reverse passes -- k_rev_* (round 2), k_unmap_sh, k_slots<1, ...> (DIR_REV = 1) -- else 'fwd'."""
+    return "rev" if ("k_rev" in name or "k_unmap" in name or
+                     ("k_slots" in name and ("<1," in name or "(int)1," in name))) else "fwd"
+
+
 def raw_rows(report):
     out = subprocess.run(["ncu", "-i", report, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
@@ -61,9 +67,7 @@ def main():
     traffic = {}
     for row in rows:
         name = row[hdr.index("Kernel Name")]
-        # the reverse passes: k_rev_* (round 2), k_unmap_sh / k_slots<1, ...> (DIR_REV = 1); else the forward
-        kind = "rev" if ("k_rev" in name or "k_unmap" in name or
-                         ("k_slots" in name and ("<1," in name or "(int)1," in name))) else "fwd"
+        kind = kind_of(name)
         lines.append(f"## {name}")
         lines.append("")
         lines.append("| metric | value |")
